@@ -1,0 +1,251 @@
+"""Pins for the oracle's transforms (CPU only).
+
+* Fig 1-4 and Fig 6 printed examples (tests/golden, each line cited);
+* invariants that hold for any input: isomorphism of the renumbering, level
+  alignment, hole counts, 2-hop sum-weight added edges, budgets, disjoint
+  subgraphs, padded degrees;
+* special cases: k = 1 (no holes), theta > 1 (no replicas), budget 0 and
+  theta_d = 0 (identity);
+* the clustering coefficient against networkx.clustering.
+"""
+import itertools
+
+import networkx as nx
+import numpy as np
+import pytest
+from hypothesis import given, settings, strategies as st
+
+import graphgen
+from golden_io import load
+from oracle.graph import from_raw, canonicalize
+from oracle import transform as T
+
+
+# ---------------------------------------------------------------- Fig 1-4
+def test_fig1_4_renumber_and_replicate():
+    raw, meta, ex = load("fig1_4.txt")
+    g = from_raw(raw)
+    k = int(meta["k"])
+    # printed CSR offsets of nodes 0-3 (P@19861-20066)
+    assert list(g.row_ptr[:4]) == [0, 7, 13, 16]
+    assert [int(g.col[g.row_ptr[u]]) for u in range(4)] == [4, 0, 11, 19]
+    sources, level = T.bfs_forest_levels(g)
+    assert sources == [int(x) for x in ex["sources"]]
+    assert sorted(v for v in range(g.n) if level[v] == 1) == [int(x) for x in ex["level1"]]
+    new, n_slots, ranges, _ = T.renumber(g, k)
+    want = dict(tuple(map(int, p.split(":"))) for p in ex["new_of_old"])
+    assert {v: int(new[v]) for v in range(g.n)} == want
+    assert n_slots == 24 and ranges == [(0, 6), (8, 22)]
+    holes = sorted(set(range(n_slots)) - set(new.tolist()))
+    assert holes == [int(x) for x in ex["holes"]]
+    nb0 = sorted(int(new[v]) for v in g.row(0)[0])
+    assert nb0 == [int(x) for x in ex["node0_new_neighbours_before_replication"]]
+    tg = T.coalesce(g, k, T.ppm(float(meta["threshold"])))
+    assert tg.slot_kind[6] == T.REPLICA and tg.slot_to_orig[6] == 0
+    moved = sorted(q for q, w, a in tg.rows[6] if a == T.ADD_NONE)
+    added = sorted(q for q, w, a in tg.rows[6] if a == T.ADD_COALESCE)
+    assert moved == [int(x) for x in ex["replica_row_moved"]]
+    assert added == [int(x) for x in ex["replica_row_added"]]
+    assert all(w == 2 for q, w, a in tg.rows[6] if a == T.ADD_COALESCE)
+    assert sorted(q for q, _, _ in tg.rows[0]) == [int(x) for x in ex["owner_row_after"]]
+    assert tg.slot_kind[7] == T.HOLE and tg.rows[7] == []
+    D = tg.divisor()
+    assert D[0] == D[6] == int(ex["divisor_node0"][0])
+
+
+def test_fig1_4_literal_reading_differs():
+    """The literal Alg 2 l.17 reading (index j into neighbours) contradicts the
+    printed example (R6): implementing it gives node 0 different neighbours."""
+    raw, meta, ex = load("fig1_4.txt")
+    g = from_raw(raw)
+    _, level = T.bfs_forest_levels(g)
+    adj = [[v for v, _ in r] for r in g.adjacency_lists()]
+    new = {v: i for i, v in enumerate([0, 1, 2, 3, 9, 16])}
+    gid = 8
+    for j in range(max(len(a) for a in adj)):
+        for p in sorted([0, 1, 2, 3, 9, 16], key=new.get):
+            if len(adj[p]) > j and level[adj[p][j]] == 1 and adj[p][j] not in new:
+                new[adj[p][j]] = gid; gid += 1
+    lit = sorted(new[v] for v in adj[0])
+    assert lit != [int(x) for x in ex["node0_new_neighbours_before_replication"]]
+
+
+# ---------------------------------------------------------------- Fig 6
+def test_fig6_degree_padding():
+    raw, meta, ex = load("fig6.txt")
+    g = from_raw(raw)
+    kn = T.Knobs(degree_norm=True, degsim_threshold=float(meta["degsim_threshold"]),
+                 degree_target=float(meta["degree_target"]))
+    tg = T.transform(g, kn)
+    added = sorted((s, q, w) for s, row in enumerate(tg.rows) for q, w, a in row if a == T.ADD_DEGNORM)
+    want = sorted(tuple(map(int, p.split(":"))) for p in ex["added"])
+    assert added == want
+    assert len(tg.rows[1]) == 6
+    tg2 = T.transform(g, T.Knobs(degree_norm=True))          # default theta 0.3
+    assert sum(a == T.ADD_DEGNORM for row in tg2.rows for _, _, a in row) == 0
+
+
+# ---------------------------------------------------------------- invariants
+def rand_graph(seed, n, p, wmax=100):
+    rng = np.random.default_rng(seed)
+    edges = [(u, v, int(rng.integers(1, wmax + 1))) for u in range(n) for v in range(n)
+             if u != v and rng.random() < p]
+    rng.shuffle(edges)
+    edges.sort(key=lambda e: e[0])          # rows grouped, unsorted within
+    return from_raw(graphgen.from_edge_list(n, edges))
+
+
+def check_coalesce_invariants(g, tg, k, theta_ppm):
+    new = tg.owner_slot
+    # bijection onto owner slots
+    assert len(set(new.tolist())) == g.n
+    assert all(tg.slot_kind[new[v]] == T.OWNER for v in range(g.n))
+    # levels start at multiples of k, holes = (k - |L| mod k) mod k
+    for i, (a, b) in enumerate(tg.levels):
+        if i > 0:
+            assert a % k == 0
+        nxt = tg.levels[i + 1][0] if i + 1 < len(tg.levels) else tg.n_slots
+        assert nxt - b == (k - (b - a) % k) % k or (i == 0 and nxt - b == (k - b % k) % k)
+    assert tg.n_slots % k == 0
+    # logical edge set = original + added (the renumbering is an isomorphism)
+    L = tg.logical()
+    orig = {(int(s), int(d)): int(w) for s, d, w in zip(*g.edges())}
+    got = {}
+    for s, d, w, a in zip(L.src.tolist(), L.dst.tolist(), L.w.tolist(), L.added.tolist()):
+        assert (s, d) not in got, "logical graph must stay simple"
+        got[(s, d)] = (w, a)
+    for e, w in orig.items():
+        assert got[e] == (w, 0)
+    for (s, d), (w, a) in got.items():
+        if a:
+            assert (s, d) not in orig
+            best = min((orig[(s, v)] + orig[(v, d)] for v in range(g.n)
+                        if (s, v) in orig and (v, d) in orig), default=None)
+            assert best == w, "added edge must be a 2-hop path with min sum weight"
+    # replica rows only target their chunk; #replicas <= #holes
+    for s in range(tg.n_slots):
+        if tg.slot_kind[s] == T.REPLICA:
+            chunks = {q // k for q, _, _ in tg.rows[s]}
+            assert len(chunks) <= 1
+            # replica rows have no in-edges (R18)
+    for row in tg.rows:
+        for q, _, _ in row:
+            assert tg.slot_kind[q] == T.OWNER
+    assert tg.info["n_replicas"] <= tg.info["n_holes"]
+
+
+@settings(max_examples=60, deadline=None)
+@given(seed=st.integers(0, 10**6), n=st.integers(1, 40), p=st.floats(0.02, 0.4),
+       k=st.sampled_from([1, 2, 4, 8, 16]), theta=st.sampled_from([0.0, 0.3, 0.6, 1.0, 1.5]))
+def test_coalesce_invariants(seed, n, p, k, theta):
+    g = rand_graph(seed, n, p)
+    tg = T.coalesce(g, k, T.ppm(theta))
+    check_coalesce_invariants(g, tg, k, T.ppm(theta))
+    if k == 1:
+        assert tg.info["n_holes"] == 0 and tg.n_slots == g.n
+    if theta > 1.0:
+        assert tg.info["n_replicas"] == 0
+
+
+def test_coalesce_rmat_invariants():
+    g = from_raw(graphgen.rmat(9))
+    for th in (0.3, 0.6):
+        tg = T.coalesce(g, 16, T.ppm(th))
+        check_coalesce_invariants(g, tg, 16, T.ppm(th))
+
+
+def test_coalesce_road_replicates():
+    g = from_raw(graphgen.road(24))
+    tg = T.coalesce(g, 16, T.ppm(0.4))
+    check_coalesce_invariants(g, tg, 16, T.ppm(0.4))
+    assert len(tg.levels) > 10
+    assert tg.info["n_holes"] > 0
+
+
+def _two_path(L_edges, a, b):
+    return [c for c in range(max(max(x) for x in L_edges) + 1)
+            if (a, c) in L_edges and (c, b) in L_edges]
+
+
+@settings(max_examples=40, deadline=None)
+@given(seed=st.integers(0, 10**6), n=st.integers(3, 30), p=st.floats(0.05, 0.5),
+       th=st.sampled_from([0.1, 0.3, 0.5, 0.8]), budget=st.integers(0, 30))
+def test_smem_invariants(seed, n, p, th, budget):
+    g = rand_graph(seed, n, p)
+    kn = T.Knobs(smem=True, cc_threshold=th, added_edge_budget=budget, smem_max_nodes=12)
+    tg = T.transform(g, kn)
+    orig = {(int(s), int(d)): int(w) for s, d, w in zip(*g.edges())}
+    L = tg.logical()
+    final = {(int(s), int(d)): int(w) for s, d, w in zip(L.src, L.dst, L.w)}
+    adds = [(int(s), int(d), int(w)) for s, d, w, a in zip(L.src, L.dst, L.w, L.added) if a]
+    assert len(adds) <= budget
+    for (a, b, w) in adds:
+        assert (a, b) not in orig
+        # lies on a directed 2-path a->c->b of the final graph with sum weight
+        assert any(final.get((a, c), None) is not None and final.get((c, b), None) is not None
+                   and final[(a, c)] + final[(c, b)] == w for c in range(g.n))
+    U = nx.Graph()
+    U.add_nodes_from(range(g.n))
+    U.add_edges_from((s, d) for (s, d) in final)
+    cc = nx.clustering(U)
+    used = set()
+    for c, members, t in tg.tiles:
+        assert len(members) <= 12 and not (set(members) & used)
+        used |= set(members)
+        assert set(members) == {c} | set(U.neighbors(c))
+        assert cc[c] > th - 1e-12 and t in (2, 4)
+    if budget == 0:
+        assert not adds
+
+
+@settings(max_examples=40, deadline=None)
+@given(seed=st.integers(0, 10**6), n=st.integers(1, 80), p=st.floats(0.01, 0.3),
+       th=st.sampled_from([0.0, 0.2, 0.5, 0.9]), coal=st.booleans())
+def test_degnorm_invariants(seed, n, p, th, coal):
+    g = rand_graph(seed, n, p)
+    base = T.transform(g, T.Knobs(coalesce=coal, chunk_k=4))
+    tg = T.transform(g, T.Knobs(coalesce=coal, chunk_k=4, degree_norm=True, degsim_threshold=th))
+    deg0 = [len(r) for r in base.rows]
+    order = tg.sched.tolist()
+    if not coal:
+        b = [T.bucket(deg0[s]) for s in order]
+        assert b == sorted(b, reverse=True)
+    for i in range(0, len(order), 32):
+        lanes = order[i:i + 32]
+        M = max(deg0[s] for s in lanes)
+        tgt = (T.ppm(0.85) * M + 999_999) // 1_000_000
+        for s in lanes:
+            d1 = len(tg.rows[s])
+            if d1 != deg0[s]:
+                assert deg0[s] < d1 <= tgt <= M
+                assert (M - deg0[s]) * 10**6 < T.ppm(th) * M
+    if th == 0.0:
+        assert tg.info["edges_added_degnorm"] == 0
+
+
+def test_clustering_coefficient_vs_networkx():
+    g = from_raw(graphgen.rmat(8))
+    tg = T.identity(g)
+    L = T._Logical(tg)
+    U = nx.Graph()
+    U.add_nodes_from(range(g.n))
+    s, d, _ = g.edges()
+    U.add_edges_from(zip(s.tolist(), d.tolist()))
+    cc = nx.clustering(U)
+    for v in range(g.n):
+        P = L.P(v)
+        mine = L.T[v] / P if P else 0.0
+        assert abs(mine - cc[v]) < 1e-12
+    # closed forms: complete graph -> 1, star -> 0
+    K = T._Logical(T.identity(from_raw(graphgen.from_edge_list(
+        5, [(a, b, 1) for a in range(5) for b in range(5) if a != b]))))
+    assert all(K.T[v] == K.P(v) for v in range(5))
+    S = T._Logical(T.identity(from_raw(graphgen.from_edge_list(6, [(0, b, 1) for b in range(1, 6)]))))
+    assert S.T[0] == 0 and S.P(0) == 10
+
+
+def test_canonicalize_rules():
+    # self loop dropped; duplicate (0,2) merged at first position with min weight
+    g = canonicalize(3, [0, 4, 5, 5], [2, 0, 1, 2, 0], [9, 5, 3, 4, 7])
+    assert g.row_ptr.tolist() == [0, 2, 3, 3]
+    assert g.col.tolist() == [2, 1, 0] and g.w.tolist() == [4, 3, 7]
