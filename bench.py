@@ -1,0 +1,297 @@
+#!/usr/bin/env python
+"""bench.py -- Graffix B200 hot path throughput (driver contract).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--workload t24|c1|c2]
+
+A step = one pass of the whole hot path over the resident graph: an SSSP run
+(source = max out-degree vertex, reading R36) plus a PageRank run (tol 1e-9)
+to their fixed points on BASELINE.json's target configuration (RMAT-24,
+exact mode; workload "t24").  value = edges scanned per second (GTEPS) over
+all ranks; roofline = the dominant sweep kernel's algorithmic bytes per launch
+/ its CUDA-event duration, against MEASURED_PEAKS.json hbm_gbs.
+
+--impl reference times the ORACLE (the reference arm of this tier) on the
+box's host cores on a bounded sample of the workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "GTEPS (edges scanned per second) of SSSP + PageRank to their fixed points"
+UNIT = "GTEPS"
+WORKLOADS = {
+    "t24": dict(scale=24, desc="T24: RMAT-24 (GTgraph a,b,c=.45,.15,.15, EF 16), exact mode, "
+                              "SSSP (R36 source, int weights 1..100) + PageRank (d=0.85, tol 1e-9)"),
+    "c2": dict(scale=22, desc="C2: RMAT-22, exact mode, SSSP + PageRank"),
+    "c1": dict(scale=14, desc="C1: RMAT-14, exact mode, SSSP + PageRank"),
+}
+CPU_SAMPLE_SCALE = 17   # bounded oracle sample: same generator at 1/128 of T24
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class Clocks:
+    """nvidia-smi sampler running during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(device), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "50"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self) -> dict:
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except Exception:
+            self.p.kill()
+        self.f.flush()
+        rows = []
+        for line in open(self.f.name):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) >= 7:
+                rows.append(parts)
+        os.unlink(self.f.name)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"], "samples": 0}
+        sm = [float(r[0]) for r in rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[3 + i].lower() == "active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(rows)}
+
+
+def oracle_sample(scale=CPU_SAMPLE_SCALE):
+    """The oracle, as it stands, on the bounded sample (rank 0 only)."""
+    import graphgen
+    from oracle import algos as A
+    from oracle.graph import from_raw, graph_to_edgelist, sssp_source
+    g = from_raw(graphgen.rmat(scale))
+    el = graph_to_edgelist(g)
+    s = sssp_source(g)
+    t0 = time.perf_counter()
+    A.sssp_dijkstra(el, s)
+    t1 = time.perf_counter()
+    _, iters = A.pagerank(el, tol=1e-9)
+    t2 = time.perf_counter()
+    edges = g.m + iters * g.m     # Dijkstra relaxes each edge once; PR gathers m per iteration
+    return {"edges": edges, "sec": t2 - t0, "sssp_s": t1 - t0, "pr_s": t2 - t1, "pr_iters": iters,
+            "n": g.n, "m": g.m}
+
+
+def cpu_cores_used() -> int:
+    return 1   # the oracle is single-threaded Python/numpy (numpy bincount is serial)
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return 0
+    for _ in range(args.warmup):
+        oracle_sample()
+    res = [oracle_sample() for _ in range(args.steps)]
+    edges = sum(r["edges"] for r in res)
+    sec = sum(r["sec"] for r in res)
+    v = edges / sec / 1e9
+    sample = (f"oracle (oracle/algos.py Dijkstra + fp64 power-iteration PR to tol 1e-9) on RMAT-{CPU_SAMPLE_SCALE} "
+              f"(same generator, n={res[0]['n']}, m={res[0]['m']}), 1/{1 << (24 - CPU_SAMPLE_SCALE)} of T24")
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sec / len(res),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32/f64",
+            "data": "synthetic", "config": {"workload": WORKLOADS[args.workload]["desc"], "graph": f"rmat{WORKLOADS[args.workload]['scale']}",
+                                            "sample": f"rmat{CPU_SAMPLE_SCALE}"},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": cpu_cores_used(), "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line))
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="t24", choices=list(WORKLOADS))
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+
+    import torch
+    import torch.distributed as dist
+    import graphgen
+    import paper_conf_icpp_0001n20_b200 as gx
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    wl = WORKLOADS[args.workload]
+    raw = graphgen.rmat(wl["scale"])
+    ctx = gx.Context(local)
+    stream = torch.cuda.ExternalStream(ctx.stream_ptr)
+    G = gx.Graph.upload(ctx, raw.row_ptr, raw.col, raw.w)
+    n, m = G.n, G.m
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+
+    def step(profile):
+        a = G.run("sssp", source=-1, mapping="lb", profile=profile)
+        b = G.run("pagerank", tol=1e-9, mapping="lb", profile=profile)
+        return a, b
+
+    for _ in range(args.warmup):
+        step(False)
+    # ---------------- timed region (inputs resident in HBM) ----------------
+    clk = Clocks(local) if rank == 0 else None
+    runs = []
+    t_ms = []
+    for _ in range(args.steps):
+        with torch.cuda.stream(stream):
+            flush.fill_(1)                      # L2 flush between steps (not timed)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        a, b = step(True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        runs.append((a, b))
+        t_ms.append(e0.elapsed_time(e1))
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks = clk.stop() if clk else None
+    tot_ms = float(sum(t_ms))
+    if world > 1:
+        tt = torch.tensor([tot_ms], device="cuda")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        tot_ms = float(tt.item())
+    edges = sum(a["edges_scanned"] + b["edges_scanned"] for a, b in runs)
+    value = edges * world / (tot_ms * 1e-3) / 1e9
+    launches = sum(a["kernel_launches"] + b["kernel_launches"] for a, b in runs)
+
+    # dominant kernel roofline (live CUDA events around each sweep launch)
+    peak, peak_src = peaks()
+    kern = {}
+    for name, idx in (("k_sssp_lb", 0), ("k_pr_pull", 1)):
+        ms = sum(r[idx]["sweep_ms"] for r in runs)
+        nl = sum(r[idx]["sweep_launches"] for r in runs)
+        by = sum(r[idx]["sweep_bytes"] for r in runs)
+        kern[name] = {"ms_total": ms, "launches": nl, "bytes": by,
+                      "gbs": by / (ms * 1e-3) / 1e9 if ms > 0 else None,
+                      "share_of_step": ms / tot_ms if tot_ms else None}
+    dom = max(kern, key=lambda k: kern[k]["ms_total"])
+    dk = kern[dom]
+    achieved = dk["gbs"]
+    roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak if achieved else None, "traffic": None, "peak_source": peak_src,
+                "bytes_per_launch": dk["bytes"] / max(dk["launches"], 1),
+                "us_per_launch": 1e3 * dk["ms_total"] / max(dk["launches"], 1)}
+
+    a0, b0 = runs[-1]
+    per_algo = {
+        "sssp": {"gteps": a0["edges_scanned"] / (a0["loop_ms"] * 1e-3) / 1e9, "gteps_solution": m / (a0["loop_ms"] * 1e-3) / 1e9,
+                 "iterations": a0["iterations"], "loop_ms": a0["loop_ms"], "edges_scanned": a0["edges_scanned"],
+                 "roofline_frac": (a0["bytes_model"] / (a0["loop_ms"] * 1e-3) / 1e9) / peak},
+        "pagerank": {"gteps": b0["edges_scanned"] / (b0["loop_ms"] * 1e-3) / 1e9, "iterations": b0["iterations"],
+                     "loop_ms": b0["loop_ms"], "last_delta": b0["last_delta"],
+                     "roofline_frac": (b0["bytes_model"] / (b0["loop_ms"] * 1e-3) / 1e9) / peak},
+    }
+
+    # ---------------- e2e through the public API with host buffers ----------------
+    e2e = None
+    if not args.no_e2e:
+        ex = G.export()      # canonical graph (exact mode), rows sorted: caller-side canonical input
+        hrp = torch.from_numpy(ex["row_ptr"]).pin_memory()
+        hcol = torch.from_numpy(ex["col"]).pin_memory()
+        hw = torch.from_numpy(ex["w"].view(np.int32)).pin_memory()
+        hdist = torch.empty(n, dtype=torch.int32).pin_memory()
+        hrank = torch.empty(n, dtype=torch.float64).pin_memory()
+        h2d = hrp.numel() * 8 + hcol.numel() * 4 + hw.numel() * 4
+        d2h = n * 4 + n * 8
+        e2e_ms, e2e_edges = [], 0
+        for i in range(args.e2e_steps + 1):
+            torch.cuda.synchronize()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            G2 = gx.Graph.upload(ctx, hrp.numpy(), hcol.numpy(), hw.numpy().view(np.uint32), canonical=True)
+            a = G2.run("sssp", source=-1, mapping="lb")
+            b = G2.run("pagerank", tol=1e-9, mapping="lb")
+            G2.download("dist", out=hdist.numpy().view(np.uint32))
+            G2.download("rank", out=hrank.numpy())
+            e1.record(stream)
+            torch.cuda.synchronize()
+            G2.close()
+            if i > 0:                           # first pass warms the allocator
+                e2e_ms.append(e0.elapsed_time(e1))
+                e2e_edges += a["edges_scanned"] + b["edges_scanned"]
+        t = sum(e2e_ms)
+        if world > 1:
+            tt = torch.tensor([t], device="cuda")
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            t = float(tt.item())
+        e2e = {"value": e2e_edges * world / (t * 1e-3) / 1e9, "unit": UNIT, "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h, "ms_per_step": t / len(e2e_ms),
+               "note": "upload of canonical pinned CSR (GX_CANONICAL) + device CSC build + SSSP + PR + download dist, rank"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        r = oracle_sample()
+        cpu = {"value": r["edges"] / r["sec"] / 1e9, "unit": UNIT, "cores": cpu_cores_used(), "kind": "oracle",
+               "sample": f"oracle Dijkstra + fp64 PR (tol 1e-9, {r['pr_iters']} iters) on RMAT-{CPU_SAMPLE_SCALE} "
+                         f"(n={r['n']}, m={r['m']}; same generator, 1/{1 << (24 - CPU_SAMPLE_SCALE)} of T24), "
+                         f"{r['sec']:.1f} s", "host_cores": os.cpu_count()}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "u32/f64", "data": "synthetic",
+                "config": {"workload": wl["desc"], "graph": f"rmat{wl['scale']}", "n": n, "m": m,
+                           "knobs": "exact", "mapping": "lb", "l2": "flushed between steps (256 MiB write)",
+                           "parallelism": "replicas" if world > 1 else "single"},
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
+                "clocks": clocks, "per_algo": per_algo, "kernels": kern}
+        print(json.dumps(line))
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,227 @@
+/*
+ * graffix.h -- C ABI of libgraffix.so, the B200-native hot path of Graffix
+ * (Singh & Nasre, "Graffix: Efficient Graph Processing with a Tinge of
+ * GPU-Specific Approximations", ICPP 2020).  Citations "P@N" refer to
+ * /root/reference/PAPER.md (one physical line), character offset N.
+ *
+ * The path: upload a CSR graph (P@15127, §2.1 Fig 1),
+ * transform it with the three Graffix techniques (Alg 2 P@16373 coalescing;
+ * §3 P@29857 shared memory; §4 P@33145 divergence), then run the iterative
+ * vertex-centric sweeps ("main fixed-point loop repeatedly calling the
+ * primary kernel", P@40883) for SSSP / PageRank / SCC / MST / BC
+ * (P@36969), merging replica copies after every iteration (§2.4 P@28309),
+ * and download per-vertex results in ORIGINAL vertex ids.
+ *
+ * Conventions
+ *  - Plain C: no C++ or torch types cross this boundary.  Every function
+ *    returns gx_status (or a plain value) and never throws; on failure
+ *    gx_last_error() returns a thread-local message valid until the next
+ *    gx_* call on the same thread, and the object is left in its previous
+ *    valid state.
+ *  - Ownership: the library copies every input; callers keep their arrays.
+ *    All device memory is owned by the library (allocated through the hook
+ *    of gx_set_allocator, else cudaMallocAsync on the context's stream) and
+ *    released by the matching destroy call.
+ *  - Threads: one gx_graph is used by one host thread at a time.
+ *  - Multi-GPU: one gx_ctx per rank (gx_ctx_create_dist); every rank calls
+ *    every gx_* function collectively, in the same order, with the same
+ *    arguments.
+ *  - No CPU fallback: without a CUDA device the compute calls return
+ *    GX_E_CUDA.
+ */
+#ifndef GRAFFIX_H
+#define GRAFFIX_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define GX_ABI_VERSION 1
+
+typedef enum {
+  GX_OK = 0,
+  GX_E_INVALID = 1,     /* bad argument (range, monotonicity, knob bounds)     */
+  GX_E_STATE = 2,       /* call out of order (run before upload, ...)          */
+  GX_E_OOM = 3,         /* device or host allocation failed                    */
+  GX_E_CUDA = 4,        /* CUDA runtime error or no device                     */
+  GX_E_NCCL = 5,        /* NCCL error or library not loadable                  */
+  GX_E_UNSUPPORTED = 6  /* e.g. (n-1)*max(w) >= 2^32-1, m' >= 2^32            */
+} gx_status;
+
+typedef enum { GX_SSSP = 1, GX_PAGERANK = 2, GX_SCC = 3, GX_MST = 4, GX_BC = 5 } gx_algo;
+
+/* Confluence operator (§2.4, P@28421-28736): the paper's algorithm-agnostic
+ * arithmetic mean, or the algorithm-aware min (SSSP only). */
+typedef enum { GX_MERGE_MEAN = 0, GX_MERGE_MIN = 1 } gx_merge;
+
+/* Sweep mapping.  LB: edge-balanced warp-cooperative kernels (the best exact
+ * kernels).  TPV: the paper's vertex-centric mapping, one thread per slot
+ * (P@15381), lanes of a warp = 32 consecutive entries of the §4 schedule,
+ * edges in SELL-32 slabs.  AUTO = LB in exact mode, TPV when §2 or §4 is on. */
+typedef enum { GX_MAP_AUTO = 0, GX_MAP_LB = 1, GX_MAP_TPV = 2 } gx_mapping;
+
+/* upload / download flags */
+#define GX_PTRS_HOST 0u       /* pointers are host memory (pageable or pinned)   */
+#define GX_PTRS_DEVICE 1u     /* pointers are device memory of the ctx device    */
+#define GX_VALIDATE 2u        /* check monotone row_ptr, col range, weights >= 1 */
+#define GX_CANONICAL 4u       /* caller asserts: no self-loops, no duplicates    */
+
+/* download kinds */
+#define GX_OUT_DIST_U32 1        /* SSSP distance, 0xFFFFFFFF = unreachable [n]  */
+#define GX_OUT_RANK_F64 2        /* PageRank [n]                                  */
+#define GX_OUT_LABEL_I32 3       /* SCC label = min original id in the SCC [n]    */
+#define GX_OUT_BC_F64 4          /* betweenness (sampled sources) [n]             */
+#define GX_OUT_MST_WEIGHT_U64 5  /* minimum spanning forest weight [1]            */
+
+typedef struct gx_ctx gx_ctx;
+typedef struct gx_graph gx_graph;
+
+/* Knobs.  Every threshold is converted once to integer parts-per-million
+ * (floor(x*1e6 + 0.5)) so that the host transforms compare exactly. */
+typedef struct {
+  uint32_t struct_size;          /* = sizeof(gx_knobs)                                */
+  int32_t coalesce;              /* §2 on/off (Alg 2, P@16373)                        */
+  int32_t chunk_k;               /* k in 1..32, default 16 (P@25752)                  */
+  double replicate_threshold;    /* connectedness >= theta (P@24839); default 0.6;
+                                    > 1 => renumber only                              */
+  int32_t merge_op;              /* gx_merge, default GX_MERGE_MEAN                   */
+  int32_t smem;                  /* §3 on/off (P@29857)                               */
+  double cc_threshold;           /* CC > theta_cc (strict), default 0.5               */
+  int64_t added_edge_budget;     /* §3 global limit, directed edges; < 0 => m/100     */
+  int32_t smem_iters;            /* t; 0 => 2 * diameter of the subgraph (P@32282)    */
+  int32_t smem_max_nodes;        /* S_max, default 64 (<= 255)                        */
+  int32_t degree_norm;           /* §4 on/off (P@33145)                               */
+  double degsim_threshold;       /* degreeSim < theta_d (strict), default 0.3         */
+  double degree_target;          /* "degree-normalisation factor", default 0.85       */
+} gx_knobs;
+
+typedef struct {
+  int64_t n_slots, n_holes, n_replicas, holes_filled;
+  int64_t edges_added_coalesce, edges_added_smem, edges_added_degnorm;
+  int64_t n_subgraphs, subgraph_vertices, m_slots;
+  double transform_ms, extra_space_pct;
+} gx_transform_info;
+
+typedef struct {
+  int32_t iterations, converged;
+  double loop_ms;          /* device time of init + fixed-point loop (CUDA events) */
+  double last_delta;       /* PR: final L1 delta                                   */
+  int64_t edges_scanned;   /* edges relaxed / gathered over all iterations         */
+  int64_t bytes_model;     /* algorithmic bytes          */
+  int64_t vertices_active; /* sum over iterations of active slots                  */
+  int32_t kernel_launches; /* library kernels launched by this run                 */
+  int32_t sweep_launches;  /* profile: launches of the main sweep kernel            */
+  double sweep_ms;         /* profile: summed CUDA-event time of the main sweep kernel */
+  int64_t sweep_bytes;     /* algorithmic bytes moved by the main sweep kernel       */
+} gx_run_info;
+
+typedef struct {
+  uint32_t struct_size;    /* = sizeof(gx_run_opts)                                */
+  int32_t algo;            /* gx_algo                                              */
+  int64_t source;          /* SSSP source (original id); < 0 => max out-degree (R36) */
+  int32_t max_iters;       /* cap on fixed-point iterations (0 => 1000000)         */
+  int32_t mapping;         /* gx_mapping                                           */
+  double tol;              /* PR: stop when L1 delta < tol (default 1e-9)          */
+  double damping;          /* PR: d (default 0.85)                                 */
+  int32_t check_every;     /* host reads the convergence flag every c iterations   */
+  int32_t use_graphs;      /* capture the c-iteration batch in a CUDA graph         */
+  const int64_t* bc_sources; /* BC: host array of original ids                     */
+  int64_t n_bc_sources;
+  int32_t profile;         /* 1 => eager launches with a CUDA event pair around every
+                              main sweep kernel (sweep_ms / sweep_launches below)   */
+  int32_t pad_;
+} gx_run_opts;
+
+/* Transformed-graph export (debug / parity path).  Two-call protocol: call
+ * gx_export_sizes, allocate host arrays of those sizes, call
+ * gx_export_transformed; any pointer may be NULL to skip that array.  The
+ * slot CSR rows are sorted by destination slot (reading R11). */
+typedef struct {
+  int64_t n_slots, m_slots, n_tiles, tile_members_len, sched_len;
+} gx_export_sizes_t;
+
+typedef struct {
+  int64_t* row_ptr;        /* [n_slots+1]                                         */
+  int32_t* col;            /* [m_slots] destination slot                          */
+  uint32_t* w;             /* [m_slots]                                           */
+  uint8_t* edge_added;     /* [m_slots] 0 original, 1 §2 2-hop, 2 §3, 3 §4        */
+  int32_t* slot_to_orig;   /* [n_slots] -1 for holes                              */
+  uint8_t* slot_kind;      /* [n_slots] 0 owner, 1 replica, 2 hole                */
+  int32_t* sched;          /* [sched_len] lane -> slot (§4), identity otherwise   */
+  int64_t* tile_ptr;       /* [n_tiles+1] into tile_members                       */
+  int32_t* tile_members;   /* [tile_members_len] original ids, ascending per tile */
+  int32_t* tile_centre;    /* [n_tiles]                                           */
+  int32_t* tile_iters;     /* [n_tiles] t                                         */
+} gx_export_t;
+
+int gx_abi_version(void);
+const char* gx_last_error(void);
+
+/* Context on CUDA device `device`; cuda_stream NULL => the library creates
+ * its own non-blocking stream; otherwise all work is ordered on it. */
+gx_status gx_ctx_create(gx_ctx** out, int device, void* cuda_stream);
+
+/* Multi-GPU: rank 0 calls gx_get_nccl_unique_id and broadcasts the 128 bytes
+ * (the binding uses torch.distributed); every rank then calls
+ * gx_ctx_create_dist.  NCCL is dlopen'ed (torch's bundled libnccl.so.2). */
+gx_status gx_get_nccl_unique_id(uint8_t out[128]);
+gx_status gx_ctx_create_dist(gx_ctx** out, int device, void* cuda_stream, int rank,
+                             int world, const uint8_t id[128]);
+
+/* Device allocator hook (e.g. torch's caching allocator).  alloc returns a
+ * device pointer or NULL; release frees it.  Must be set before uploads. */
+typedef void* (*gx_alloc_fn)(size_t bytes, void* stream, void* user);
+typedef void (*gx_release_fn)(void* ptr, size_t bytes, void* stream, void* user);
+gx_status gx_set_allocator(gx_ctx* ctx, gx_alloc_fn alloc, gx_release_fn release, void* user);
+void gx_ctx_destroy(gx_ctx* ctx);
+gx_status gx_ctx_stream(gx_ctx* ctx, void** stream_out);
+
+/* Upload a directed CSR graph (P@15127): row u = col[row_ptr[u]..row_ptr[u+1]),
+ * weights w (NULL => all 1; must be >= 1).  Canonicalised (reading R2): self-
+ * loops dropped, a duplicate (u,v) merged into its first occurrence keeping
+ * the minimum weight, row order otherwise kept -- unless GX_CANONICAL.
+ * Errors: GX_E_INVALID (n < 0, m < 0, with GX_VALIDATE: non-monotone row_ptr,
+ * col out of [0,n), w = 0), GX_E_UNSUPPORTED (m >= 2^32 or n >= 2^31). */
+gx_status gx_graph_upload_csr(gx_ctx* ctx, gx_graph** out, int64_t n, int64_t m,
+                              const int64_t* row_ptr, const int32_t* col, const uint32_t* w,
+                              uint32_t flags);
+void gx_graph_destroy(gx_graph* g);
+gx_status gx_graph_info(gx_graph* g, int64_t* n, int64_t* m);
+
+/* Paper defaults, all techniques OFF (= exact mode). */
+gx_status gx_knobs_default(gx_knobs* k);
+
+/* Host-side transforms §2 -> §3 -> §4 (composition reading R34) and the
+ * device layouts they need.  NULL knobs => exact mode (identity).
+ * Errors: GX_E_INVALID (k not in 1..32, thresholds not in [0,1] except
+ * replicate_threshold >= 0, degree_target not in (0,1], smem_max_nodes not
+ * in 2..255). */
+gx_status gx_transform(gx_graph* g, const gx_knobs* knobs, gx_transform_info* info);
+
+gx_status gx_export_sizes(gx_graph* g, gx_export_sizes_t* sizes);
+gx_status gx_export_transformed(gx_graph* g, gx_export_t* out);
+
+/* Run one algorithm to its fixed point on the transformed graph.  Not
+ * converging within max_iters is not an error (converged = 0).
+ * Errors: GX_E_STATE (no graph), GX_E_INVALID (source out of range),
+ * GX_E_UNSUPPORTED ((n-1)*max(w) >= 2^32-1 for SSSP). */
+gx_status gx_run(gx_graph* g, gx_algo algo, int64_t source, int32_t max_iters, double tol,
+                 gx_run_info* info);
+gx_status gx_run_ex(gx_graph* g, const gx_run_opts* opts, gx_run_info* info);
+gx_status gx_run_opts_default(gx_run_opts* o);
+
+/* Copy a result (indexed by ORIGINAL vertex id; owner slots after the final
+ * merge) into `out` (host or device per flags).  count = n, or 1 for MST.
+ * Errors: GX_E_STATE (that algorithm has not run), GX_E_INVALID (count). */
+gx_status gx_download(gx_graph* g, int32_t kind, void* out, int64_t count, uint32_t flags);
+
+/* Synchronise the context stream (host wait). */
+gx_status gx_sync(gx_ctx* ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GRAFFIX_H */

@@ -1,0 +1,446 @@
+// capi.cpp -- the extern "C" boundary of libgraffix.so (include/graffix.h).
+// Argument checking, error capture, contexts, allocation, upload/download.
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <mutex>
+
+#include "gx_internal.h"
+
+namespace gx {
+
+static thread_local std::string g_last_error;
+
+void* Ctx::dmalloc(size_t b) {
+  if (b == 0) b = 16;
+  void* p = nullptr;
+  if (alloc) {
+    p = alloc(b, (void*)stream, user);
+    if (!p) GX_THROW(GX_E_OOM, "allocator hook returned NULL for " + std::to_string(b) + " bytes");
+  } else {
+    cudaError_t e = cudaMallocAsync(&p, b, stream);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      GX_THROW(GX_E_OOM, "cudaMallocAsync(" + std::to_string(b) + "): " + cudaGetErrorString(e));
+    }
+  }
+  return p;
+}
+
+void Ctx::dfree(void* p, size_t b) {
+  if (!p) return;
+  if (release) release(p, b, (void*)stream, user);
+  else cudaFreeAsync(p, stream);
+}
+
+DBuf& DBuf::operator=(DBuf&& o) noexcept {
+  if (this != &o) {
+    reset();
+    ctx = o.ctx; p = o.p; bytes = o.bytes;
+    o.p = nullptr; o.bytes = 0;
+  }
+  return *this;
+}
+
+void DBuf::reset() {
+  if (p && ctx) ctx->dfree(p, bytes);
+  p = nullptr;
+  bytes = 0;
+}
+
+void DBuf::alloc(Ctx* c, size_t b) {
+  if (p && ctx == c && bytes >= b && b > 0) return;
+  reset();
+  ctx = c;
+  p = c->dmalloc(b);
+  bytes = b ? b : 16;
+}
+
+// upload helpers implemented in devgraph.cu
+void device_upload_input(gx_graph* g, const int64_t* rp, const int32_t* col, const uint32_t* w,
+                         bool device_ptrs, bool validate);
+
+}  // namespace gx
+
+using namespace gx;
+
+#define GX_API_BEGIN try {
+#define GX_API_END                                         \
+  }                                                        \
+  catch (const gx::Error& e) {                             \
+    gx::g_last_error = e.what();                           \
+    return e.st;                                           \
+  }                                                        \
+  catch (const std::bad_alloc& e) {                        \
+    gx::g_last_error = std::string("host OOM: ") + e.what(); \
+    return GX_E_OOM;                                       \
+  }                                                        \
+  catch (const std::exception& e) {                        \
+    gx::g_last_error = e.what();                           \
+    return GX_E_INVALID;                                   \
+  }                                                        \
+  gx::g_last_error.clear();                                \
+  return GX_OK;
+
+extern "C" {
+
+int gx_abi_version(void) { return GX_ABI_VERSION; }
+
+const char* gx_last_error(void) { return gx::g_last_error.c_str(); }
+
+static void init_ctx(gx_ctx* c, int device, void* stream) {
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    GX_THROW(GX_E_CUDA, std::string("no CUDA device: ") + cudaGetErrorString(e));
+  }
+  GX_CHECK_ARG(device >= 0 && device < ndev, "device out of range");
+  c->device = device;
+  CUDA_OK(cudaSetDevice(device));
+  cudaDeviceProp prop;
+  CUDA_OK(cudaGetDeviceProperties(&prop, device));
+  if (prop.major < 10)
+    GX_THROW(GX_E_CUDA, std::string("libgraffix is built for sm_100a; device is ") + prop.name);
+  c->num_sms = prop.multiProcessorCount;
+  c->smem_optin = prop.sharedMemPerBlockOptin;
+  if (stream) {
+    c->stream = (cudaStream_t)stream;
+    c->own_stream = false;
+  } else {
+    CUDA_OK(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
+    c->own_stream = true;
+  }
+}
+
+gx_status gx_ctx_create(gx_ctx** out, int device, void* cuda_stream) {
+  GX_API_BEGIN
+  GX_CHECK_ARG(out != nullptr, "out is NULL");
+  *out = nullptr;
+  gx_ctx* c = new gx_ctx();
+  try {
+    init_ctx(c, device, cuda_stream);
+  } catch (...) {
+    delete c;
+    throw;
+  }
+  *out = c;
+  GX_API_END
+}
+
+gx_status gx_set_allocator(gx_ctx* ctx, gx_alloc_fn alloc, gx_release_fn release, void* user) {
+  GX_API_BEGIN
+  GX_CHECK_ARG(ctx != nullptr, "ctx is NULL");
+  GX_CHECK_ARG((alloc == nullptr) == (release == nullptr), "alloc and release must both be set");
+  ctx->alloc = alloc;
+  ctx->release = release;
+  ctx->user = user;
+  GX_API_END
+}
+
+gx_status gx_ctx_stream(gx_ctx* ctx, void** s) {
+  GX_API_BEGIN
+  GX_CHECK_ARG(ctx && s, "NULL argument");
+  *s = (void*)ctx->stream;
+  GX_API_END
+}
+
+void gx_comm_destroy(void* comm);  // comm.cpp
+
+void gx_ctx_destroy(gx_ctx* ctx) {
+  if (!ctx) return;
+  cudaSetDevice(ctx->device);
+  if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+  if (ctx->nccl) gx_comm_destroy(ctx->nccl);
+  if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
+  delete ctx;
+}
+
+gx_status gx_sync(gx_ctx* ctx) {
+  GX_API_BEGIN
+  GX_CHECK_ARG(ctx, "ctx is NULL");
+  CUDA_OK(cudaStreamSynchronize(ctx->stream));
+  GX_API_END
+}
+
+gx_status gx_graph_upload_csr(gx_ctx* ctx, gx_graph** out, int64_t n, int64_t m,
+                              const int64_t* row_ptr, const int32_t* col, const uint32_t* w,
+                              uint32_t flags) {
+  GX_API_BEGIN
+  GX_CHECK_ARG(ctx && out, "NULL ctx/out");
+  *out = nullptr;
+  GX_CHECK_ARG(n >= 0 && m >= 0, "n and m must be >= 0");
+  GX_CHECK_ARG(row_ptr != nullptr, "row_ptr is NULL");
+  GX_CHECK_ARG(m == 0 || col != nullptr, "col is NULL");
+  if (n >= (int64_t(1) << 31) - 1) GX_THROW(GX_E_UNSUPPORTED, "n must be < 2^31 - 1");
+  if (m >= (int64_t(1) << 32) - 1) GX_THROW(GX_E_UNSUPPORTED, "m must be < 2^32 - 1");
+  CUDA_OK(cudaSetDevice(ctx->device));
+  bool dev = flags & GX_PTRS_DEVICE;
+  bool validate = flags & GX_VALIDATE;
+  gx_graph* g = new gx_graph();
+  g->ctx = ctx;
+  gx_knobs_default(&g->knobs);
+  try {
+    if (flags & GX_CANONICAL) {
+      g->n = n;
+      g->m = m;
+      device_upload_input(g, row_ptr, col, w, dev, validate);
+    } else {
+      // canonicalise on the host (reading R2); device inputs come back first
+      std::vector<int64_t> hrp;
+      std::vector<int32_t> hcol;
+      std::vector<uint32_t> hw;
+      const int64_t* rp = row_ptr;
+      const int32_t* c = col;
+      const uint32_t* ww = w;
+      if (dev) {
+        hrp.resize(n + 1);
+        CUDA_OK(cudaMemcpy(hrp.data(), row_ptr, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost));
+        hcol.resize(m);
+        if (m) CUDA_OK(cudaMemcpy(hcol.data(), col, sizeof(int32_t) * m, cudaMemcpyDeviceToHost));
+        if (w) {
+          hw.resize(m);
+          if (m) CUDA_OK(cudaMemcpy(hw.data(), w, sizeof(uint32_t) * m, cudaMemcpyDeviceToHost));
+        }
+        rp = hrp.data(); c = hcol.data(); ww = w ? hw.data() : nullptr;
+      }
+      if (validate || true) {
+        GX_CHECK_ARG(rp[0] == 0 && rp[n] == m, "row_ptr[0] must be 0 and row_ptr[n] == m");
+        for (int64_t u = 0; u < n; u++)
+          if (rp[u + 1] < rp[u]) GX_THROW(GX_E_INVALID, "row_ptr not monotone at " + std::to_string(u));
+        if (validate) {
+          for (int64_t e = 0; e < m; e++) {
+            if (c[e] < 0 || c[e] >= n) GX_THROW(GX_E_INVALID, "col out of range at " + std::to_string(e));
+            if (ww && ww[e] == 0) GX_THROW(GX_E_INVALID, "weight 0 at " + std::to_string(e));
+          }
+        }
+      }
+      canonicalize_host(n, rp, c, ww, g->host);
+      g->host_valid = true;
+      g->n = n;
+      g->m = g->host.m;
+      device_upload_input(g, g->host.rp.data(), g->host.col.data(), g->host.w.data(), false, false);
+    }
+    build_device_exact(g);
+  } catch (...) {
+    gx_graph_destroy(g);
+    throw;
+  }
+  *out = g;
+  GX_API_END
+}
+
+void gx_graph_destroy(gx_graph* g) {
+  if (!g) return;
+  cudaSetDevice(g->ctx->device);
+  delete g;  // DBuf destructors release device memory on the ctx stream
+}
+
+gx_status gx_graph_info(gx_graph* g, int64_t* n, int64_t* m) {
+  GX_API_BEGIN
+  GX_CHECK_ARG(g, "graph is NULL");
+  if (n) *n = g->n;
+  if (m) *m = g->m;
+  GX_API_END
+}
+
+gx_status gx_knobs_default(gx_knobs* k) {
+  if (!k) return GX_E_INVALID;
+  std::memset(k, 0, sizeof(*k));
+  k->struct_size = sizeof(gx_knobs);
+  k->coalesce = 0;
+  k->chunk_k = 16;
+  k->replicate_threshold = 0.6;
+  k->merge_op = GX_MERGE_MEAN;
+  k->smem = 0;
+  k->cc_threshold = 0.5;
+  k->added_edge_budget = -1;
+  k->smem_iters = 0;
+  k->smem_max_nodes = 64;
+  k->degree_norm = 0;
+  k->degsim_threshold = 0.3;
+  k->degree_target = 0.85;
+  return GX_OK;
+}
+
+gx_status gx_run_opts_default(gx_run_opts* o) {
+  if (!o) return GX_E_INVALID;
+  std::memset(o, 0, sizeof(*o));
+  o->struct_size = sizeof(gx_run_opts);
+  o->algo = GX_SSSP;
+  o->source = -1;
+  o->max_iters = 0;
+  o->mapping = GX_MAP_AUTO;
+  o->tol = 1e-9;
+  o->damping = 0.85;
+  o->check_every = 8;
+  o->use_graphs = 1;
+  return GX_OK;
+}
+
+static void check_knobs(const gx_knobs& k) {
+  GX_CHECK_ARG(k.struct_size == sizeof(gx_knobs), "gx_knobs.struct_size mismatch");
+  GX_CHECK_ARG(k.chunk_k >= 1 && k.chunk_k <= 32, "chunk_k must be in 1..32");
+  GX_CHECK_ARG(k.replicate_threshold >= 0 && std::isfinite(k.replicate_threshold),
+               "replicate_threshold must be >= 0");
+  GX_CHECK_ARG(k.cc_threshold >= 0 && k.cc_threshold <= 1, "cc_threshold must be in [0,1]");
+  GX_CHECK_ARG(k.degsim_threshold >= 0 && k.degsim_threshold <= 1, "degsim_threshold must be in [0,1]");
+  GX_CHECK_ARG(k.degree_target > 0 && k.degree_target <= 1, "degree_target must be in (0,1]");
+  GX_CHECK_ARG(k.smem_max_nodes >= 2 && k.smem_max_nodes <= 255, "smem_max_nodes must be in 2..255");
+  GX_CHECK_ARG(k.merge_op == GX_MERGE_MEAN || k.merge_op == GX_MERGE_MIN, "merge_op invalid");
+  GX_CHECK_ARG(k.smem_iters >= 0, "smem_iters must be >= 0");
+}
+
+gx_status gx_transform(gx_graph* g, const gx_knobs* knobs, gx_transform_info* info) {
+  GX_API_BEGIN
+  GX_CHECK_ARG(g, "graph is NULL");
+  gx_knobs k;
+  gx_knobs_default(&k);
+  if (knobs) k = *knobs;
+  check_knobs(k);
+  CUDA_OK(cudaSetDevice(g->ctx->device));
+  auto t0 = std::chrono::steady_clock::now();
+  bool exact = !k.coalesce && !k.smem && !k.degree_norm;
+  if (exact) {
+    g->sg = SlotGraph();
+    g->transformed = false;
+    g->knobs = k;
+    build_device_exact(g);
+    g->sg.info.n_slots = g->n;
+    g->sg.info.m_slots = g->m;
+  } else {
+    ensure_host(g);
+    SlotGraph sg;
+    transform_host(g->host, k, sg);
+    g->sg = std::move(sg);
+    g->transformed = true;
+    g->knobs = k;
+    build_device_slots(g);
+  }
+  g->rs = RunState();
+  auto t1 = std::chrono::steady_clock::now();
+  g->sg.info.transform_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
+  if (info) *info = g->sg.info;
+  GX_API_END
+}
+
+gx_status gx_export_sizes(gx_graph* g, gx_export_sizes_t* s) {
+  GX_API_BEGIN
+  GX_CHECK_ARG(g && s, "NULL argument");
+  if (!g->transformed) {
+    ensure_host(g);
+    s->n_slots = g->n;
+    s->m_slots = g->m;
+    s->n_tiles = 0;
+    s->tile_members_len = 0;
+    s->sched_len = g->n;
+  } else {
+    const SlotGraph& sg = g->sg;
+    s->n_slots = sg.n_slots;
+    s->m_slots = sg.m_slots;
+    s->n_tiles = (int64_t)sg.tile_centre.size();
+    s->tile_members_len = (int64_t)sg.tile_members.size();
+    s->sched_len = sg.sched.empty() ? sg.n_slots : (int64_t)sg.sched.size();
+  }
+  GX_API_END
+}
+
+gx_status gx_export_transformed(gx_graph* g, gx_export_t* o) {
+  GX_API_BEGIN
+  GX_CHECK_ARG(g && o, "NULL argument");
+  if (!g->transformed) {
+    // exact mode: identity slots; rows sorted by destination (R11)
+    ensure_host(g);
+    const HostCSR& h = g->host;
+    std::vector<int64_t> rp(h.rp);
+    if (o->row_ptr) std::memcpy(o->row_ptr, rp.data(), sizeof(int64_t) * (h.n + 1));
+#pragma omp parallel for schedule(dynamic, 4096)
+    for (int64_t u = 0; u < h.n; u++) {
+      std::vector<std::pair<int32_t, uint32_t>> row;
+      for (int64_t e = h.rp[u]; e < h.rp[u + 1]; e++) row.push_back({h.col[e], h.w[e]});
+      std::sort(row.begin(), row.end());
+      for (size_t i = 0; i < row.size(); i++) {
+        int64_t e = h.rp[u] + (int64_t)i;
+        if (o->col) o->col[e] = row[i].first;
+        if (o->w) o->w[e] = row[i].second;
+        if (o->edge_added) o->edge_added[e] = 0;
+      }
+    }
+    for (int64_t v = 0; v < h.n; v++) {
+      if (o->slot_to_orig) o->slot_to_orig[v] = (int32_t)v;
+      if (o->slot_kind) o->slot_kind[v] = 0;
+      if (o->sched) o->sched[v] = (int32_t)v;
+    }
+    if (o->tile_ptr) o->tile_ptr[0] = 0;
+  } else {
+    const SlotGraph& sg = g->sg;
+    if (o->row_ptr) std::memcpy(o->row_ptr, sg.rp.data(), sizeof(int64_t) * (sg.n_slots + 1));
+    if (o->col) std::memcpy(o->col, sg.col.data(), sizeof(int32_t) * sg.m_slots);
+    if (o->w) std::memcpy(o->w, sg.w.data(), sizeof(uint32_t) * sg.m_slots);
+    if (o->edge_added) std::memcpy(o->edge_added, sg.added.data(), sg.m_slots);
+    if (o->slot_to_orig) std::memcpy(o->slot_to_orig, sg.slot_to_orig.data(), sizeof(int32_t) * sg.n_slots);
+    if (o->slot_kind) std::memcpy(o->slot_kind, sg.kind.data(), sg.n_slots);
+    if (o->sched) {
+      if (sg.sched.empty())
+        for (int64_t s = 0; s < sg.n_slots; s++) o->sched[s] = (int32_t)s;
+      else
+        std::memcpy(o->sched, sg.sched.data(), sizeof(int32_t) * sg.sched.size());
+    }
+    size_t nt = sg.tile_centre.size();
+    if (o->tile_ptr) std::memcpy(o->tile_ptr, sg.tile_ptr.data(), sizeof(int64_t) * (nt + 1));
+    if (o->tile_members && !sg.tile_members.empty())
+      std::memcpy(o->tile_members, sg.tile_members.data(), sizeof(int32_t) * sg.tile_members.size());
+    if (o->tile_centre && nt) std::memcpy(o->tile_centre, sg.tile_centre.data(), sizeof(int32_t) * nt);
+    if (o->tile_iters && nt) std::memcpy(o->tile_iters, sg.tile_iters.data(), sizeof(int32_t) * nt);
+  }
+  GX_API_END
+}
+
+gx_status gx_run_ex(gx_graph* g, const gx_run_opts* opts, gx_run_info* info) {
+  GX_API_BEGIN
+  GX_CHECK_ARG(g && opts, "NULL argument");
+  GX_CHECK_ARG(opts->struct_size == sizeof(gx_run_opts), "gx_run_opts.struct_size mismatch");
+  CUDA_OK(cudaSetDevice(g->ctx->device));
+  gx_run_opts o = *opts;
+  if (o.max_iters <= 0) o.max_iters = 1000000;
+  if (o.check_every <= 0) o.check_every = 8;
+  GX_CHECK_ARG(o.mapping >= GX_MAP_AUTO && o.mapping <= GX_MAP_TPV, "mapping invalid");
+  gx_run_info ri;
+  std::memset(&ri, 0, sizeof(ri));
+  switch (o.algo) {
+    case GX_SSSP: run_sssp(g, o, ri); break;
+    case GX_PAGERANK:
+      GX_CHECK_ARG(o.tol > 0 && o.damping > 0 && o.damping < 1, "tol must be > 0 and damping in (0,1)");
+      run_pagerank(g, o, ri);
+      break;
+    case GX_SCC: run_scc(g, o, ri); break;
+    case GX_MST: run_mst(g, o, ri); break;
+    case GX_BC: run_bc(g, o, ri); break;
+    default: GX_THROW(GX_E_INVALID, "unknown algorithm");
+  }
+  if (info) *info = ri;
+  GX_API_END
+}
+
+gx_status gx_run(gx_graph* g, gx_algo algo, int64_t source, int32_t max_iters, double tol,
+                 gx_run_info* info) {
+  gx_run_opts o;
+  gx_run_opts_default(&o);
+  o.algo = algo;
+  o.source = source;
+  o.max_iters = max_iters;
+  if (tol > 0) o.tol = tol;
+  return gx_run_ex(g, &o, info);
+}
+
+gx_status gx_download(gx_graph* g, int32_t kind, void* out, int64_t count, uint32_t flags) {
+  GX_API_BEGIN
+  GX_CHECK_ARG(g && out, "NULL argument");
+  CUDA_OK(cudaSetDevice(g->ctx->device));
+  gx::download(g, kind, out, count, flags);
+  GX_API_END
+}
+
+}  // extern "C"

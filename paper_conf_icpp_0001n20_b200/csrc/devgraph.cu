@@ -1,0 +1,362 @@
+// devgraph.cu -- device layouts of the (transformed) slot graph.
+//
+//  * out-CSR  rp u32[n'+1], adj uint2{col, w}[m']: one 8-byte coalesced load
+//    per relaxed edge (SSSP push, BC, SCC forward);
+//  * in-CSC   crp u32[n'+1], csrc i32[m'] rows sorted by source slot (built on
+//    the device with a radix sort of (dst, src) keys): PR pull, SCC backward;
+//  * PR merge-path tiles over (rows + in-edges) and the rows spanning tiles;
+//  * D u32[n'] = logical out-degree of the slot's vertex (PR divisor; for a
+//    replicated vertex the SUM over its copies);
+//  * confluence groups (owner first) with the owner's in-edges for the
+//    SSSP re-pull after a merge.
+#include <cub/cub.cuh>
+
+#include <algorithm>
+#include <numeric>
+
+#include "gx_internal.h"
+#include "kernels_common.cuh"
+
+namespace gx {
+
+// ------------------------------------------------------------------ kernels
+__global__ void k_rp64_to_u32(const int64_t* __restrict__ in, uint32_t* __restrict__ out, int64_t n1) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n1; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = (uint32_t)in[i];
+}
+
+__global__ void k_interleave(const int32_t* __restrict__ col, const uint32_t* __restrict__ w,
+                             uint2* __restrict__ adj, int64_t m) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x)
+    adj[e] = make_uint2((uint32_t)col[e], w ? w[e] : 1u);
+}
+
+__global__ void k_outdeg(const uint32_t* __restrict__ rp, uint32_t* __restrict__ D, int64_t n) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+    D[v] = rp[v + 1] - rp[v];
+}
+
+__global__ void k_validate(const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
+                           const uint32_t* __restrict__ w, int64_t n, int64_t m,
+                           unsigned int* __restrict__ err) {
+  int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x, st = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t u = tid; u < n; u += st)
+    if (rp[u + 1] < rp[u]) atomicOr(err, 1u);
+  for (int64_t e = tid; e < m; e += st) {
+    if (col[e] < 0 || col[e] >= n) atomicOr(err, 2u);
+    if (w && w[e] == 0) atomicOr(err, 4u);
+  }
+  if (tid == 0 && (rp[0] != 0 || rp[n] != m)) atomicOr(err, 8u);
+}
+
+__global__ void k_max_u32(const uint32_t* __restrict__ w, int64_t m, unsigned int* __restrict__ out) {
+  unsigned int mx = 0;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x)
+    mx = max(mx, w[e]);
+  mx = warp_max_u32(mx);
+  if ((threadIdx.x & 31) == 0 && mx) atomicMax(out, mx);
+}
+
+// key = (dst << 32) | src for every out-edge; src found by each row owner
+__global__ void k_csc_keys(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj, int64_t n,
+                           uint64_t* __restrict__ keys) {
+  // one warp per row: rows of any length stay coalesced
+  int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  int lane = threadIdx.x & 31;
+  int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t u = warp; u < n; u += nw) {
+    uint32_t a = rp[u], b = rp[u + 1];
+    for (uint32_t e = a + lane; e < b; e += 32) keys[e] = ((uint64_t)adj[e].x << 32) | (uint64_t)u;
+  }
+}
+
+__global__ void k_csc_split(const uint64_t* __restrict__ keys, int64_t m, int32_t* __restrict__ csrc,
+                            uint32_t* __restrict__ cnt) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x) {
+    uint64_t k = keys[e];
+    csrc[e] = (int32_t)(k & 0xffffffffu);
+    atomicAdd(&cnt[k >> 32], 1u);
+  }
+}
+
+// merge-path coordinate of diagonal d over (row ends A[i] = crp[i+1], edges)
+__device__ __forceinline__ void merge_path_search(int64_t d, const uint32_t* __restrict__ crp, int64_t n,
+                                                  int64_t m, int64_t& row, int64_t& edge) {
+  int64_t lo = max((int64_t)0, d - m), hi = min(d, n);
+  while (lo < hi) {
+    int64_t p = (lo + hi) >> 1;
+    if ((int64_t)crp[p + 1] <= d - p - 1) lo = p + 1;
+    else hi = p;
+  }
+  row = lo;
+  edge = d - lo;
+}
+
+__global__ void k_pr_tiles(const uint32_t* __restrict__ crp, int64_t n, int64_t m, int64_t tiles,
+                           int64_t ti, int64_t* __restrict__ trow, int64_t* __restrict__ tedge) {
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t <= tiles; t += (int64_t)gridDim.x * blockDim.x) {
+    int64_t d = min(t * ti, n + m), r, e;
+    merge_path_search(d, crp, n, m, r, e);
+    trow[t] = r;
+    tedge[t] = e;
+  }
+}
+
+// a tile's first row is split iff it started in an earlier tile
+__global__ void k_pr_split_flags(const uint32_t* __restrict__ crp, const int64_t* __restrict__ trow,
+                                 const int64_t* __restrict__ tedge, int64_t tiles, int64_t n,
+                                 uint8_t* __restrict__ flag) {
+  for (int64_t t = 1 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < tiles; t += (int64_t)gridDim.x * blockDim.x) {
+    int64_t r = trow[t];
+    if (r < n && (int64_t)crp[r] < tedge[t]) flag[r] = 1;
+  }
+}
+
+
+// ------------------------------------------------------------------ host side
+
+void device_upload_input(gx_graph* g, const int64_t* rp, const int32_t* col, const uint32_t* w,
+                         bool device_ptrs, bool validate) {
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  int64_t n = g->n, m = g->m;
+  g->in_rp.alloc(c, sizeof(int64_t) * (n + 1));
+  g->in_col.alloc(c, sizeof(int32_t) * std::max<int64_t>(m, 1));
+  g->in_w.alloc(c, sizeof(uint32_t) * std::max<int64_t>(m, 1));
+  cudaMemcpyKind kind = device_ptrs ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
+  CUDA_OK(cudaMemcpyAsync(g->in_rp.p, rp, sizeof(int64_t) * (n + 1), kind, s));
+  if (m) {
+    CUDA_OK(cudaMemcpyAsync(g->in_col.p, col, sizeof(int32_t) * m, kind, s));
+    if (w) {
+      CUDA_OK(cudaMemcpyAsync(g->in_w.p, w, sizeof(uint32_t) * m, kind, s));
+    } else {
+      launch_fill_u32(c, g->in_w.as<uint32_t>(), 1u, m);  // all-ones weights
+    }
+  }
+  DBuf scratch;
+  scratch.alloc(c, 16);
+  CUDA_OK(cudaMemsetAsync(scratch.p, 0, 16, s));
+  unsigned int* err = scratch.as<unsigned int>();
+  if (validate) {
+    k_validate<<<grid_for(c, std::max(n, m)), 256, 0, s>>>(g->in_rp.as<int64_t>(), g->in_col.as<int32_t>(),
+                                                           w ? g->in_w.as<uint32_t>() : nullptr, n, m, err);
+  }
+  if (m) k_max_u32<<<grid_for(c, m), 256, 0, s>>>(g->in_w.as<uint32_t>(), m, err + 1);
+  CUDA_OK(cudaGetLastError());
+  unsigned int h[2];
+  CUDA_OK(cudaMemcpyAsync(h, err, 8, cudaMemcpyDeviceToHost, s));
+  CUDA_OK(cudaStreamSynchronize(s));
+  if (h[0] & 8u) GX_THROW(GX_E_INVALID, "row_ptr[0] must be 0 and row_ptr[n] == m");
+  if (h[0] & 1u) GX_THROW(GX_E_INVALID, "row_ptr not monotone");
+  if (h[0] & 2u) GX_THROW(GX_E_INVALID, "col out of range");
+  if (h[0] & 4u) GX_THROW(GX_E_INVALID, "weight 0 (weights must be >= 1)");
+  g->max_w = m ? std::max(1u, h[1]) : 1u;
+}
+
+static void build_csc_and_tiles(gx_graph* g) {
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  DevGraph& d = g->dg;
+  int64_t n = d.n_slots, m = d.m_slots;
+  d.crp.alloc(c, sizeof(uint32_t) * (n + 1));
+  d.csrc.alloc(c, sizeof(int32_t) * std::max<int64_t>(m, 1));
+  if (m > 0) {
+    DBuf keys, keys2, tmp;
+    keys.alloc(c, sizeof(uint64_t) * m);
+    keys2.alloc(c, sizeof(uint64_t) * m);
+    k_csc_keys<<<grid_for(c, n * 32), 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), n,
+                                                   keys.as<uint64_t>());
+    CUDA_OK(cudaGetLastError());
+    int bits = 1;
+    while ((int64_t(1) << bits) < n) bits++;
+    size_t tb = 0;
+    cub::DoubleBuffer<uint64_t> db(keys.as<uint64_t>(), keys2.as<uint64_t>());
+    CUDA_OK(cub::DeviceRadixSort::SortKeys(nullptr, tb, db, (int64_t)m, 0, 32 + bits, s));
+    tmp.alloc(c, tb);
+    CUDA_OK(cub::DeviceRadixSort::SortKeys(tmp.p, tb, db, (int64_t)m, 0, 32 + bits, s));
+    DBuf cnt;
+    cnt.alloc(c, sizeof(uint32_t) * (n + 1));
+    CUDA_OK(cudaMemsetAsync(cnt.p, 0, sizeof(uint32_t) * (n + 1), s));
+    k_csc_split<<<grid_for(c, m), 256, 0, s>>>(db.Current(), m, d.csrc.as<int32_t>(), cnt.as<uint32_t>());
+    CUDA_OK(cudaGetLastError());
+    size_t sb = 0;
+    CUDA_OK(cub::DeviceScan::ExclusiveSum(nullptr, sb, cnt.as<uint32_t>(), d.crp.as<uint32_t>(), n + 1, s));
+    DBuf t2;
+    t2.alloc(c, sb);
+    CUDA_OK(cub::DeviceScan::ExclusiveSum(t2.p, sb, cnt.as<uint32_t>(), d.crp.as<uint32_t>(), n + 1, s));
+  } else {
+    CUDA_OK(cudaMemsetAsync(d.crp.p, 0, sizeof(uint32_t) * (n + 1), s));
+  }
+  // merge-path tiles for the PR pull
+  int64_t ti = (int64_t)d.pr_ipt * d.pr_threads;
+  d.pr_tiles = (n + m + ti - 1) / ti;
+  d.pr_tile_row.alloc(c, sizeof(int64_t) * (d.pr_tiles + 1));
+  d.pr_tile_edge.alloc(c, sizeof(int64_t) * (d.pr_tiles + 1));
+  k_pr_tiles<<<grid_for(c, d.pr_tiles + 1), 256, 0, s>>>(d.crp.as<uint32_t>(), n, m, d.pr_tiles, ti,
+                                                        d.pr_tile_row.as<int64_t>(), d.pr_tile_edge.as<int64_t>());
+  CUDA_OK(cudaGetLastError());
+  DBuf flag, idx, nsel, tmp;
+  flag.alloc(c, std::max<int64_t>(n, 1));
+  CUDA_OK(cudaMemsetAsync(flag.p, 0, std::max<int64_t>(n, 1), s));
+  if (d.pr_tiles > 1)
+    k_pr_split_flags<<<grid_for(c, d.pr_tiles), 256, 0, s>>>(d.crp.as<uint32_t>(), d.pr_tile_row.as<int64_t>(),
+                                                             d.pr_tile_edge.as<int64_t>(), d.pr_tiles, n,
+                                                             flag.as<uint8_t>());
+  idx.alloc(c, sizeof(int32_t) * std::max<int64_t>(n, 1));
+  launch_iota_i32(c, idx.as<int32_t>(), n);
+  d.pr_split.alloc(c, sizeof(int32_t) * std::max<int64_t>(d.pr_tiles, 1));
+  nsel.alloc(c, sizeof(int64_t));
+  size_t tb = 0;
+  CUDA_OK(cub::DeviceSelect::Flagged(nullptr, tb, idx.as<int32_t>(), flag.as<uint8_t>(), d.pr_split.as<int32_t>(),
+                                     nsel.as<int64_t>(), n, s));
+  tmp.alloc(c, tb);
+  CUDA_OK(cub::DeviceSelect::Flagged(tmp.p, tb, idx.as<int32_t>(), flag.as<uint8_t>(), d.pr_split.as<int32_t>(),
+                                     nsel.as<int64_t>(), n, s));
+  int64_t ns = 0;
+  CUDA_OK(cudaMemcpyAsync(&ns, nsel.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  CUDA_OK(cudaStreamSynchronize(s));
+  d.pr_n_split = ns;
+}
+
+void ensure_csc(gx_graph* g) {
+  if (g->dg.crp.p) return;
+  build_csc_and_tiles(g);
+}
+
+void build_device_exact(gx_graph* g) {
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  DevGraph& d = g->dg;
+  d = DevGraph();
+  d.n = g->n;
+  d.n_slots = g->n;
+  d.m_slots = g->m;
+  d.identity = true;
+  d.max_w = g->max_w;
+  int64_t n = d.n_slots, m = d.m_slots;
+  d.rp.alloc(c, sizeof(uint32_t) * (n + 1));
+  k_rp64_to_u32<<<grid_for(c, n + 1), 256, 0, s>>>(g->in_rp.as<int64_t>(), d.rp.as<uint32_t>(), n + 1);
+  d.adj.alloc(c, sizeof(uint2) * std::max<int64_t>(m, 1));
+  if (m) k_interleave<<<grid_for(c, m), 256, 0, s>>>(g->in_col.as<int32_t>(), g->in_w.as<uint32_t>(),
+                                                     d.adj.as<uint2>(), m);
+  d.D.alloc(c, sizeof(uint32_t) * std::max<int64_t>(n, 1));
+  k_outdeg<<<grid_for(c, n), 256, 0, s>>>(d.rp.as<uint32_t>(), d.D.as<uint32_t>(), n);
+  CUDA_OK(cudaGetLastError());
+}
+
+// Upload the host slot graph produced by transform_host.
+void build_device_slots(gx_graph* g) {
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  const SlotGraph& sg = g->sg;
+  DevGraph& d = g->dg;
+  d = DevGraph();
+  d.n = sg.n;
+  d.n_slots = sg.n_slots;
+  d.m_slots = sg.m_slots;
+  d.identity = false;
+  int64_t n = sg.n_slots, m = sg.m_slots;
+  if (m >= (int64_t(1) << 32) - 1) GX_THROW(GX_E_UNSUPPORTED, "m' must be < 2^32 - 1");
+  std::vector<uint32_t> rp32(n + 1);
+  for (int64_t i = 0; i <= n; i++) rp32[i] = (uint32_t)sg.rp[i];
+  std::vector<uint2> adj(std::max<int64_t>(m, 1));
+  uint32_t mw = 1;
+  for (int64_t e = 0; e < m; e++) {
+    adj[e] = make_uint2((uint32_t)sg.col[e], sg.w[e]);
+    mw = std::max(mw, sg.w[e]);
+  }
+  d.max_w = mw;
+  // logical out-degree per vertex, summed over its copies
+  std::vector<uint32_t> ldeg(sg.n, 0), D(std::max<int64_t>(n, 1), 0);
+  for (int64_t sl = 0; sl < n; sl++)
+    if (sg.kind[sl] != HOLE) ldeg[sg.slot_to_orig[sl]] += (uint32_t)(sg.rp[sl + 1] - sg.rp[sl]);
+  for (int64_t sl = 0; sl < n; sl++)
+    if (sg.kind[sl] != HOLE) D[sl] = ldeg[sg.slot_to_orig[sl]];
+  // groups: owner first, then replica slots ascending
+  std::vector<std::vector<int32_t>> rep(sg.n);
+  for (int64_t sl = 0; sl < n; sl++)
+    if (sg.kind[sl] == REPLICA) rep[sg.slot_to_orig[sl]].push_back((int32_t)sl);
+  std::vector<int32_t> gptr{0}, gslots, gid(std::max<int64_t>(n, 1), -1);
+  std::vector<int32_t> gown;
+  for (int64_t v = 0; v < sg.n; v++) {
+    if (rep[v].empty()) continue;
+    int32_t gi = (int32_t)gown.size();
+    gown.push_back(sg.owner_slot[v]);
+    gslots.push_back(sg.owner_slot[v]);
+    gid[sg.owner_slot[v]] = gi;
+    for (int32_t r : rep[v]) {
+      gslots.push_back(r);
+      gid[r] = gi;
+    }
+    gptr.push_back((int32_t)gslots.size());
+  }
+  d.n_groups = (int64_t)gown.size();
+  // in-edges of each group's owner slot: (src slot, w)
+  std::vector<int32_t> gin_ptr(d.n_groups + 1, 0);
+  std::vector<uint2> gin;
+  if (d.n_groups) {
+    std::vector<std::vector<uint2>> tmp(d.n_groups);
+    for (int64_t sl = 0; sl < n; sl++)
+      for (int64_t e = sg.rp[sl]; e < sg.rp[sl + 1]; e++) {
+        int32_t q = sg.col[e];
+        if (gid[q] >= 0 && gown[gid[q]] == q) tmp[gid[q]].push_back(make_uint2((uint32_t)sl, sg.w[e]));
+      }
+    for (int64_t gi = 0; gi < d.n_groups; gi++) {
+      gin_ptr[gi + 1] = gin_ptr[gi] + (int32_t)tmp[gi].size();
+      gin.insert(gin.end(), tmp[gi].begin(), tmp[gi].end());
+    }
+  }
+  auto up = [&](DBuf& b, const void* src, size_t bytes) {
+    b.alloc(c, std::max<size_t>(bytes, 16));
+    if (bytes) CUDA_OK(cudaMemcpyAsync(b.p, src, bytes, cudaMemcpyHostToDevice, s));
+  };
+  up(d.rp, rp32.data(), sizeof(uint32_t) * (n + 1));
+  up(d.adj, adj.data(), sizeof(uint2) * m);
+  up(d.D, D.data(), sizeof(uint32_t) * n);
+  up(d.owner, sg.owner_slot.data(), sizeof(int32_t) * sg.n);
+  up(d.kind, sg.kind.data(), n);
+  if (d.n_groups) {
+    up(d.gid, gid.data(), sizeof(int32_t) * n);
+    up(d.gptr, gptr.data(), sizeof(int32_t) * gptr.size());
+    up(d.gslots, gslots.data(), sizeof(int32_t) * gslots.size());
+    up(d.g_in_ptr, gin_ptr.data(), sizeof(int32_t) * gin_ptr.size());
+    up(d.g_in, gin.data(), sizeof(uint2) * gin.size());
+  }
+  // §3 tiles: members as owner slots + local CSR (u8 member indices)
+  int64_t nt = (int64_t)sg.tile_centre.size();
+  d.n_tiles = nt;
+  if (nt) {
+    std::vector<int32_t> tp(nt + 1, 0), tmem, teptr(nt + 1, 0), titers(nt);
+    std::vector<uint2> tedges;  // {src_local | dst_local << 8, w}
+    for (int64_t t = 0; t < nt; t++) {
+      std::vector<int32_t> mem;
+      for (int64_t i = sg.tile_ptr[t]; i < sg.tile_ptr[t + 1]; i++) mem.push_back(sg.owner_slot[sg.tile_members[i]]);
+      std::sort(mem.begin(), mem.end());
+      for (size_t a = 0; a < mem.size(); a++) {
+        int32_t sl = mem[a];
+        for (int64_t e = sg.rp[sl]; e < sg.rp[sl + 1]; e++) {
+          auto it = std::lower_bound(mem.begin(), mem.end(), sg.col[e]);
+          if (it != mem.end() && *it == sg.col[e]) {
+            uint32_t b = (uint32_t)(it - mem.begin());
+            tedges.push_back(make_uint2((uint32_t)a | (b << 8), sg.w[e]));
+          }
+        }
+      }
+      tmem.insert(tmem.end(), mem.begin(), mem.end());
+      tp[t + 1] = (int32_t)tmem.size();
+      teptr[t + 1] = (int32_t)tedges.size();
+      titers[t] = sg.tile_iters[t];
+      d.t_max_members = std::max<int64_t>(d.t_max_members, (int64_t)mem.size());
+      d.t_max_edges = std::max<int64_t>(d.t_max_edges, teptr[t + 1] - teptr[t]);
+    }
+    up(d.t_ptr, tp.data(), sizeof(int32_t) * tp.size());
+    up(d.t_members, tmem.data(), sizeof(int32_t) * tmem.size());
+    up(d.t_eptr, teptr.data(), sizeof(int32_t) * teptr.size());
+    up(d.t_edges, tedges.data(), sizeof(uint2) * tedges.size());
+    up(d.t_iters, titers.data(), sizeof(int32_t) * titers.size());
+  }
+  if (!sg.sched.empty()) up(d.sched, sg.sched.data(), sizeof(int32_t) * sg.sched.size());
+  CUDA_OK(cudaStreamSynchronize(s));  // host vectors go out of scope
+}
+
+}  // namespace gx

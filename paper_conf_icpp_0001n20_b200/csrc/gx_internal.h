@@ -1,0 +1,176 @@
+// gx_internal.h -- internal types of libgraffix (not part of the C ABI).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstring>
+#include <stdexcept>
+#include <string>
+#include <vector>
+
+#include "../../include/graffix.h"
+
+namespace gx {
+
+struct Error : std::runtime_error {
+  gx_status st;
+  Error(gx_status s, const std::string& m) : std::runtime_error(m), st(s) {}
+};
+
+#define GX_THROW(st, msg) throw ::gx::Error((st), (msg))
+#define GX_CHECK_ARG(cond, msg) \
+  do { if (!(cond)) GX_THROW(GX_E_INVALID, msg); } while (0)
+#define CUDA_OK(expr)                                                                  \
+  do {                                                                                 \
+    cudaError_t e_ = (expr);                                                           \
+    if (e_ != cudaSuccess) {                                                           \
+      if (e_ == cudaErrorMemoryAllocation)                                             \
+        GX_THROW(GX_E_OOM, std::string(#expr ": ") + cudaGetErrorString(e_));          \
+      GX_THROW(GX_E_CUDA, std::string(#expr ": ") + cudaGetErrorString(e_));           \
+    }                                                                                  \
+  } while (0)
+
+constexpr uint32_t INF = 0xFFFFFFFFu;
+enum SlotKind : uint8_t { OWNER = 0, REPLICA = 1, HOLE = 2 };
+enum AddKind : uint8_t { ADD_NONE = 0, ADD_COALESCE = 1, ADD_SMEM = 2, ADD_DEGNORM = 3 };
+
+struct Ctx;
+
+// Device buffer owned by the library (allocator hook or cudaMallocAsync).
+struct DBuf {
+  Ctx* ctx = nullptr;
+  void* p = nullptr;
+  size_t bytes = 0;
+  DBuf() = default;
+  DBuf(const DBuf&) = delete;
+  DBuf& operator=(const DBuf&) = delete;
+  DBuf(DBuf&& o) noexcept { *this = std::move(o); }
+  DBuf& operator=(DBuf&& o) noexcept;
+  ~DBuf() { reset(); }
+  void reset();
+  void alloc(Ctx* c, size_t b);
+  template <class T> T* as() const { return reinterpret_cast<T*>(p); }
+};
+
+struct Ctx {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  gx_alloc_fn alloc = nullptr;
+  gx_release_fn release = nullptr;
+  void* user = nullptr;
+  int rank = 0, world = 1;
+  void* nccl = nullptr;  // ncclComm_t
+  int num_sms = 148;
+  size_t smem_optin = 0;
+  void* dmalloc(size_t b);
+  void dfree(void* p, size_t b);
+};
+
+// Host canonical graph (original ids).
+struct HostCSR {
+  int64_t n = 0, m = 0;
+  std::vector<int64_t> rp;
+  std::vector<int32_t> col;
+  std::vector<uint32_t> w;
+};
+
+// Host transformed ("slot") graph; rows sorted by destination slot.
+struct SlotGraph {
+  int64_t n = 0, n_slots = 0, m_slots = 0;
+  std::vector<int64_t> rp;
+  std::vector<int32_t> col;
+  std::vector<uint32_t> w;
+  std::vector<uint8_t> added;
+  std::vector<int32_t> slot_to_orig;
+  std::vector<uint8_t> kind;
+  std::vector<int32_t> owner_slot;
+  std::vector<int32_t> sched;         // lane -> slot; empty => identity
+  std::vector<int64_t> tile_ptr;      // §3 subgraphs
+  std::vector<int32_t> tile_members, tile_centre, tile_iters;
+  gx_transform_info info{};
+};
+
+// Device layouts of the current slot graph.
+struct DevGraph {
+  int64_t n = 0, n_slots = 0, m_slots = 0;
+  bool identity = true;        // exact mode: slot == original id, no holes
+  uint32_t max_w = 1;
+  DBuf rp, adj;                // out-CSR: u32 [n_slots+1], uint2 {col, w} [m_slots]
+  DBuf crp, csrc;              // in-CSC:  u32 [n_slots+1], i32 [m_slots]
+  DBuf D;                      // u32 [n_slots]: logical out-degree (PR divisor)
+  DBuf owner;                  // i32 [n]: original id -> owner slot
+  DBuf kind;                   // u8 [n_slots] (null in exact mode)
+  DBuf gid;                    // i32 [n_slots]: group id or -1 (null if no groups)
+  DBuf gptr, gslots;           // groups: ptr [ng+1], slots (owner first)
+  int64_t n_groups = 0;
+  DBuf g_in_ptr, g_in;         // per-group owner in-edges (src slot, w) for SSSP pull
+  // PR merge-path tiles
+  int pr_ipt = 7, pr_threads = 256;
+  int64_t pr_tiles = 0;
+  DBuf pr_tile_row, pr_tile_edge;   // i64 [tiles+1]
+  DBuf pr_split;                    // i32 [n_split] rows spanning tiles
+  int64_t pr_n_split = 0;
+  // LB SSSP
+  int64_t n_heavy = 0;
+  // TPV / SELL-32 (filled on demand)
+  bool tpv_ready = false;
+  int64_t n_warps_tpv = 0;
+  DBuf sched;                  // i32 [lanes]
+  DBuf sell_off;               // u64 [warps+1] slab offsets (in edges)
+  DBuf sell_adj;               // uint2 slabs, col = -1 padding
+  DBuf csell_off, csell_src;   // PR pull slabs (in-edges), src = -1 padding
+  int64_t sell_lanes = 0;
+  // §3 tiles
+  int64_t n_tiles = 0;
+  DBuf t_ptr, t_members, t_eptr, t_edges, t_iters;  // local CSR per tile
+  int64_t t_max_members = 0, t_max_edges = 0;
+};
+
+struct RunState {
+  // SSSP / BC / SCC scratch (allocated lazily)
+  DBuf dist, mark, q[2], hq[2], hbase[2], st, changed;
+  // PR
+  DBuf x, contrib[2], ysplit, gnew, pst;
+  // BC
+  DBuf sigma, delta, bc, level;
+  // SCC / MST
+  DBuf label, label2, mst_best, comp;
+  uint64_t mst_weight = 0;
+  bool have[6] = {false, false, false, false, false, false};
+};
+
+}  // namespace gx
+
+struct gx_ctx : gx::Ctx {};
+
+struct gx_graph {
+  gx::Ctx* ctx = nullptr;
+  gx::HostCSR host;            // canonical input (host copy, lazily filled)
+  bool host_valid = false;
+  gx::DBuf in_rp, in_col, in_w;   // canonical input on device (original ids)
+  int64_t n = 0, m = 0;
+  uint32_t max_w = 1;
+  gx::SlotGraph sg;            // current transform (empty in exact mode)
+  bool transformed = false;
+  gx_knobs knobs{};
+  gx::DevGraph dg;
+  gx::RunState rs;
+};
+
+// ---- internal entry points across translation units ----
+namespace gx {
+void canonicalize_host(int64_t n, const int64_t* rp, const int32_t* col, const uint32_t* w,
+                       HostCSR& out);
+void ensure_host(gx_graph* g);
+void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out);
+void build_device_exact(gx_graph* g);
+void build_device_slots(gx_graph* g);
+void build_tpv(gx_graph* g);
+void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info);
+void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info);
+void run_scc(gx_graph* g, const gx_run_opts& o, gx_run_info& info);
+void run_mst(gx_graph* g, const gx_run_opts& o, gx_run_info& info);
+void run_bc(gx_graph* g, const gx_run_opts& o, gx_run_info& info);
+void download(gx_graph* g, int kind, void* out, int64_t count, uint32_t flags);
+}  // namespace gx

@@ -1,0 +1,130 @@
+"""GPU parity of the exact-mode sweeps with the oracle (SURVEY.md §8(a) A10,
+A11): SSSP bit-exact against Dijkstra, PageRank within L1 1e-6 (north_star).
+
+Sizes span many tiles / frontier batches with ragged tails; edge cases cover
+empty rows, unreachable vertices, self-loops and duplicates, isolated
+vertices, heavy (hub) rows, single vertices, and every launch mode."""
+import numpy as np
+import pytest
+
+import graphgen
+from gpu_util import ctx, upload
+from oracle import algos as A
+from oracle.graph import INF32, from_raw, graph_to_edgelist, sssp_source
+
+pytestmark = pytest.mark.gpu
+
+GRAPHS = {
+    "rmat12": lambda: graphgen.rmat(12),
+    "rmat14_C1": lambda: graphgen.rmat(14),
+    "uniform": lambda: graphgen.uniform(5000, 70001),
+    "road64": lambda: graphgen.road(64),
+    "star_hub": lambda: graphgen.from_edge_list(
+        5003, [(0, v, 1 + v % 7) for v in range(1, 5003)] + [(v, (v * 7) % 5003, 3) for v in range(1, 5003, 3)]),
+    "dups_loops": lambda: graphgen.from_edge_list(
+        6, [(0, 1, 5), (0, 1, 2), (0, 0, 1), (1, 2, 1), (1, 2, 9), (2, 0, 4), (3, 4, 1), (4, 3, 1), (2, 2, 3)]),
+    "isolated": lambda: graphgen.from_edge_list(5, []),
+    "single": lambda: graphgen.from_edge_list(1, []),
+}
+
+
+@pytest.mark.parametrize("name", list(GRAPHS))
+@pytest.mark.parametrize("mode", ["graphs", "eager1"])
+def test_sssp_exact_bit_exact(name, mode):
+    raw = GRAPHS[name]()
+    g = from_raw(raw)
+    s = sssp_source(g)
+    want = A.sssp_dijkstra(graph_to_edgelist(g), s)
+    G = upload(raw)
+    kw = dict(use_graphs=True, check_every=8) if mode == "graphs" else dict(use_graphs=False, check_every=1)
+    info = G.run("sssp", source=-1, mapping="lb", **kw)
+    got = G.download("dist")
+    assert info["converged"] == 1
+    assert np.array_equal(got, want), f"{np.sum(got != want)} mismatches"
+    # every other source too, for the small ones
+    if g.n <= 6:
+        for s2 in range(g.n):
+            G.run("sssp", source=s2, mapping="lb")
+            assert np.array_equal(G.download("dist"), A.sssp_dijkstra(graph_to_edgelist(g), s2))
+
+
+@pytest.mark.parametrize("name", list(GRAPHS))
+def test_pagerank_exact_l1(name):
+    raw = GRAPHS[name]()
+    g = from_raw(raw)
+    want, _ = A.pagerank(graph_to_edgelist(g), tol=1e-14)
+    G = upload(raw)
+    info = G.run("pagerank", tol=1e-12, mapping="lb")
+    got = G.download("rank")
+    assert info["converged"] == 1
+    l1 = np.abs(got - want).sum()
+    assert l1 <= 1e-6, l1
+    assert abs(got.sum() - 1.0) < 1e-6
+
+
+def test_sssp_max_iters_not_an_error():
+    raw = graphgen.road(40)
+    G = upload(raw)
+    info = G.run("sssp", max_iters=3, check_every=1)
+    assert info["converged"] == 0 and info["iterations"] == 3
+
+
+def test_errors():
+    from paper_conf_icpp_0001n20_b200 import GraffixError
+    raw = graphgen.rmat(8)
+    G = upload(raw)
+    with pytest.raises(GraffixError) as e:
+        G.download("dist")
+    assert e.value.status == 2  # GX_E_STATE
+    with pytest.raises(GraffixError) as e:
+        G.run("sssp", source=10**6)
+    assert e.value.status == 1
+    bad = raw.col.copy()
+    bad[0] = raw.n + 5
+    from paper_conf_icpp_0001n20_b200 import Graph
+    with pytest.raises(GraffixError):
+        Graph.upload(ctx(), raw.row_ptr, bad, raw.w, validate=True)
+    # overflow guard: (n-1) * max(w) >= 2^32 - 1
+    big = graphgen.from_edge_list(3, [(0, 1, 2**31), (1, 2, 2**31)])
+    Gb = upload(big)
+    with pytest.raises(GraffixError) as e:
+        Gb.run("sssp", source=0)
+    assert e.value.status == 6
+
+
+def test_device_pointer_upload_and_download():
+    import torch
+    raw = graphgen.rmat(10)
+    g = from_raw(raw)
+    from paper_conf_icpp_0001n20_b200 import Graph
+    G = Graph.upload(ctx(), torch.from_numpy(raw.row_ptr).cuda(), torch.from_numpy(raw.col).cuda(),
+                     torch.from_numpy(raw.w.view(np.int32)).cuda())
+    G.run("sssp")
+    out = torch.empty(g.n, dtype=torch.int32, device="cuda")
+    G.download("dist", out=out)
+    want = A.sssp_dijkstra(graph_to_edgelist(g), sssp_source(g))
+    assert np.array_equal(out.cpu().numpy().view(np.uint32), want)
+
+
+@pytest.mark.parametrize("scale", [24])
+def test_full_size_certificates(scale):
+    """BASELINE.json's target config (RMAT-24, exact mode) in bench.py's launch
+    configuration: SSSP checked by the O(m) certificate, PR by the residual
+    bound r/(1-d) (oracle.metrics), both on the canonical graph."""
+    from oracle.graph import canonicalize_sorted
+    from oracle.metrics import pagerank_residual, sssp_certificate
+    raw = graphgen.rmat(scale)
+    G = upload(raw)
+    g = canonicalize_sorted(raw.n, raw.row_ptr, raw.col, raw.w)
+    del raw
+    s = sssp_source(g)
+    G.run("sssp", source=-1, mapping="lb")
+    dist = G.download("dist")
+    cert = sssp_certificate(g, s, dist)
+    assert cert["ok"], cert
+    info = G.run("pagerank", tol=1e-9, mapping="lb")
+    x = G.download("rank")
+    src = np.repeat(np.arange(g.n, dtype=np.int32), np.diff(g.row_ptr))
+    r = pagerank_residual(src, g.col, g.n, x)
+    assert r["bound"] <= 1e-6, r
+    assert abs(r["mass"] - 1) < 1e-6

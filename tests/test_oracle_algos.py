@@ -270,3 +270,12 @@ def test_inaccuracy_definition():
     r = M.inaccuracy(d2, d)
     assert r["inf_mismatch"] == 1 and abs(r["inacc_pct"] - 20.0) < 1e-12
     assert M.inaccuracy(11, 10, "scalar")["inacc_pct"] == pytest.approx(10.0)
+
+
+def test_canonicalize_sorted_matches_canonicalize():
+    from oracle.graph import canonicalize_sorted
+    for G in [graphgen.rmat(11), graphgen.uniform(2000, 40000), graphgen.road(40)]:
+        a = from_raw(G)
+        b = canonicalize_sorted(G.n, G.row_ptr, G.col, G.w)
+        assert np.array_equal(a.row_ptr, b.row_ptr) and np.array_equal(a.col, b.col)
+        assert np.array_equal(a.w, b.w)
