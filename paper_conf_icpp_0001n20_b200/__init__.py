@@ -90,15 +90,20 @@ class Context:
         if not torch.cuda.is_available():
             return
         dev = self.device
+        alloc_fn = torch.cuda.caching_allocator_alloc
+        free_fn = torch.cuda.caching_allocator_delete
 
         def _alloc(nbytes, stream, user):
             try:
-                return torch.cuda.caching_allocator_alloc(int(nbytes), dev, stream or 0)
+                return alloc_fn(int(nbytes), dev, stream or 0)
             except Exception:
                 return None
 
         def _release(ptr, nbytes, stream, user):
-            torch.cuda.caching_allocator_delete(ptr)
+            try:
+                free_fn(ptr)
+            except Exception:   # interpreter shutdown: the process is exiting anyway
+                pass
 
         self._cbs = (ALLOC_FN(_alloc), RELEASE_FN(_release))
         _check(lib().gx_set_allocator(self._h, self._cbs[0], self._cbs[1], None))

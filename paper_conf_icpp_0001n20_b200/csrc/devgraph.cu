@@ -16,6 +16,7 @@
 
 #include "gx_internal.h"
 #include "kernels_common.cuh"
+#include "sell.cuh"
 
 namespace gx {
 
@@ -78,40 +79,6 @@ __global__ void k_csc_split(const uint64_t* __restrict__ keys, int64_t m, int32_
     atomicAdd(&cnt[k >> 32], 1u);
   }
 }
-
-// merge-path coordinate of diagonal d over (row ends A[i] = crp[i+1], edges)
-__device__ __forceinline__ void merge_path_search(int64_t d, const uint32_t* __restrict__ crp, int64_t n,
-                                                  int64_t m, int64_t& row, int64_t& edge) {
-  int64_t lo = max((int64_t)0, d - m), hi = min(d, n);
-  while (lo < hi) {
-    int64_t p = (lo + hi) >> 1;
-    if ((int64_t)crp[p + 1] <= d - p - 1) lo = p + 1;
-    else hi = p;
-  }
-  row = lo;
-  edge = d - lo;
-}
-
-__global__ void k_pr_tiles(const uint32_t* __restrict__ crp, int64_t n, int64_t m, int64_t tiles,
-                           int64_t ti, int64_t* __restrict__ trow, int64_t* __restrict__ tedge) {
-  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t <= tiles; t += (int64_t)gridDim.x * blockDim.x) {
-    int64_t d = min(t * ti, n + m), r, e;
-    merge_path_search(d, crp, n, m, r, e);
-    trow[t] = r;
-    tedge[t] = e;
-  }
-}
-
-// a tile's first row is split iff it started in an earlier tile
-__global__ void k_pr_split_flags(const uint32_t* __restrict__ crp, const int64_t* __restrict__ trow,
-                                 const int64_t* __restrict__ tedge, int64_t tiles, int64_t n,
-                                 uint8_t* __restrict__ flag) {
-  for (int64_t t = 1 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < tiles; t += (int64_t)gridDim.x * blockDim.x) {
-    int64_t r = trow[t];
-    if (r < n && (int64_t)crp[r] < tedge[t]) flag[r] = 1;
-  }
-}
-
 
 // ------------------------------------------------------------------ host side
 
@@ -187,35 +154,7 @@ static void build_csc_and_tiles(gx_graph* g) {
   } else {
     CUDA_OK(cudaMemsetAsync(d.crp.p, 0, sizeof(uint32_t) * (n + 1), s));
   }
-  // merge-path tiles for the PR pull
-  int64_t ti = (int64_t)d.pr_ipt * d.pr_threads;
-  d.pr_tiles = (n + m + ti - 1) / ti;
-  d.pr_tile_row.alloc(c, sizeof(int64_t) * (d.pr_tiles + 1));
-  d.pr_tile_edge.alloc(c, sizeof(int64_t) * (d.pr_tiles + 1));
-  k_pr_tiles<<<grid_for(c, d.pr_tiles + 1), 256, 0, s>>>(d.crp.as<uint32_t>(), n, m, d.pr_tiles, ti,
-                                                        d.pr_tile_row.as<int64_t>(), d.pr_tile_edge.as<int64_t>());
-  CUDA_OK(cudaGetLastError());
-  DBuf flag, idx, nsel, tmp;
-  flag.alloc(c, std::max<int64_t>(n, 1));
-  CUDA_OK(cudaMemsetAsync(flag.p, 0, std::max<int64_t>(n, 1), s));
-  if (d.pr_tiles > 1)
-    k_pr_split_flags<<<grid_for(c, d.pr_tiles), 256, 0, s>>>(d.crp.as<uint32_t>(), d.pr_tile_row.as<int64_t>(),
-                                                             d.pr_tile_edge.as<int64_t>(), d.pr_tiles, n,
-                                                             flag.as<uint8_t>());
-  idx.alloc(c, sizeof(int32_t) * std::max<int64_t>(n, 1));
-  launch_iota_i32(c, idx.as<int32_t>(), n);
-  d.pr_split.alloc(c, sizeof(int32_t) * std::max<int64_t>(d.pr_tiles, 1));
-  nsel.alloc(c, sizeof(int64_t));
-  size_t tb = 0;
-  CUDA_OK(cub::DeviceSelect::Flagged(nullptr, tb, idx.as<int32_t>(), flag.as<uint8_t>(), d.pr_split.as<int32_t>(),
-                                     nsel.as<int64_t>(), n, s));
-  tmp.alloc(c, tb);
-  CUDA_OK(cub::DeviceSelect::Flagged(tmp.p, tb, idx.as<int32_t>(), flag.as<uint8_t>(), d.pr_split.as<int32_t>(),
-                                     nsel.as<int64_t>(), n, s));
-  int64_t ns = 0;
-  CUDA_OK(cudaMemcpyAsync(&ns, nsel.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-  CUDA_OK(cudaStreamSynchronize(s));
-  d.pr_n_split = ns;
+  build_pr_sell(g);
 }
 
 void ensure_csc(gx_graph* g) {

@@ -105,12 +105,13 @@ struct DevGraph {
   DBuf gptr, gslots;           // groups: ptr [ng+1], slots (owner first)
   int64_t n_groups = 0;
   DBuf g_in_ptr, g_in;         // per-group owner in-edges (src slot, w) for SSSP pull
-  // PR merge-path tiles
-  int pr_ipt = 7, pr_threads = 256;
-  int64_t pr_tiles = 0;
-  DBuf pr_tile_row, pr_tile_edge;   // i64 [tiles+1]
-  DBuf pr_split;                    // i32 [n_split] rows spanning tiles
-  int64_t pr_n_split = 0;
+  // PR windowed SELL-32 pull layout (sell.cu): per window of PRW rows the
+  // light rows sorted by in-degree into 32-lane slices, heavy rows listed
+  int64_t pr_nwin = 0, pr_nslices = 0, pr_nheavy = 0, pr_slab_len = 0;
+  DBuf pr_lane_row, pr_heavy_row;   // i32
+  DBuf pr_win_slice, pr_win_heavy;  // i64 [nwin+1]
+  DBuf pr_slice_len, pr_slice_off;  // u32 [nslices+1], u64 [nslices+1]
+  DBuf pr_slab;                     // u32 source slots, PR_SENT padding
   // LB SSSP
   int64_t n_heavy = 0;
   // TPV / SELL-32 (filled on demand)

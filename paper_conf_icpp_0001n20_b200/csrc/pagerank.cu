@@ -4,20 +4,24 @@
 // (reading R35; D = total logical out-degree, so replica copies each divide by
 // the vertex's full out-degree and mass is not double counted, Theorem E3).
 //
-// LB pull = merge-path over (row ends + in-edges) of the CSC: every CTA gets
-// a tile of exactly IPT*256 merge items (static, precomputed once), stages
-// contrib[csrc[e]] (fp32, coalesced csrc stream + L2 gathers) and the tile's
-// row ends in shared memory, then each thread walks IPT items accumulating in
-// fp64.  Rows completing inside the tile are finalised in place (x, delta,
-// next contrib, dangling mass); rows spanning tiles accumulate into ysplit and
-// are finalised by a small fixup kernel.  Replicas are mirrors (R19): they are
-// not recomputed; the §2.4 merge (P@28309, mean, P@28609) sets every copy.
+// LB pull = windowed SELL-32 (sell.cu): one CTA per window of PRW rows.  The
+// window's light rows were sorted by in-degree into 32-lane slices, so a warp
+// reads the j-th in-edge of 32 rows with one coalesced 128-byte load (L2
+// evict_first) and every lane accumulates its own row in fp64 from fp32
+// contrib gathers (L2 evict_last) with 8 gathers in flight; rows with more
+// than PR_HEAVY in-edges are reduced warp-per-row.  Row sums stay in shared
+// memory and the PR update of the window (x, delta, next contrib, dangling
+// mass) runs in the same CTA with coalesced accesses.  Replicas are mirrors
+// (R19): not recomputed; the §2.4 merge (P@28309, mean P@28609) sets every
+// copy.
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 
 #include "gx_internal.h"
 #include "kernels_common.cuh"
 #include "ktimer.h"
+#include "sell.cuh"
 
 namespace gx {
 
@@ -30,27 +34,31 @@ struct PrState {
 };
 
 struct PrArgs {
+  // windowed SELL layout
+  const uint32_t* slab;
+  const uint32_t* slice_len;
+  const uint64_t* slice_off;
+  const int32_t* lane_row;
+  const int32_t* heavy_row;
+  const int64_t* win_slice;
+  const int64_t* win_heavy;
   const uint32_t* crp;
   const int32_t* csrc;
-  const int64_t* trow;
-  const int64_t* tedge;
-  int64_t tiles;
+  int64_t nwin;
+  int64_t n_slots;
   double* x;
   float* contrib[2];
   const uint32_t* D;
   const uint8_t* kind;   // null in exact mode
   const int32_t* gid;    // null without groups
   double* gnew;
-  double* ysplit;
-  const int32_t* split;
-  int64_t n_split;
   double base, damp, invN;
   PrState* st;
 };
 
 template <bool SLOTS>
-__device__ __forceinline__ void pr_finalize(const PrArgs& a, int64_t v, double y, double addc, float* cout,
-                                            double& my_delta, double& my_dang) {
+__device__ __forceinline__ void pr_finalize(const PrArgs& a, int64_t v, double y, double xo, uint32_t Dv, double addc,
+                                            float* cout, double& my_delta, double& my_dang) {
   if (SLOTS) {
     if (a.kind[v] != OWNER) return;  // holes stay 0; replicas are set by the merge
   }
@@ -62,20 +70,18 @@ __device__ __forceinline__ void pr_finalize(const PrArgs& a, int64_t v, double y
       return;
     }
   }
-  double xo = a.x[v];
-  a.x[v] = xn;
+  __stcs(a.x + v, xn);
   my_delta += fabs(xn - xo);
-  uint32_t Dv = a.D[v];
-  cout[v] = Dv ? (float)(xn / (double)Dv) : 0.0f;
+  __stcs(cout + v, Dv ? (float)(xn / (double)Dv) : 0.0f);
   if (!Dv) my_dang += xn;
 }
 
-template <int IPT, bool SLOTS>
-__global__ void __launch_bounds__(256) k_pr_pull(PrArgs a) {
-  constexpr int TI = IPT * 256;
-  __shared__ float s_val[TI];
-  __shared__ uint32_t s_end[TI + 1];
-  __shared__ double s_sum[TI + 1];
+constexpr int PR_CTA = 256;
+constexpr int PR_U = 8;   // gathers in flight per lane
+
+template <bool SLOTS>
+__global__ void __launch_bounds__(PR_CTA) k_pr_sell(PrArgs a) {
+  __shared__ double s_y[PRW];
   __shared__ double s_red[32];
   PrState* st = a.st;
   if (st->stop) return;
@@ -84,86 +90,75 @@ __global__ void __launch_bounds__(256) k_pr_pull(PrArgs a) {
   float* cout = a.contrib[(t + 1) & 1];
   const double addc = a.base + a.damp * st->dang[t % 3] * a.invN;
   double my_delta = 0, my_dang = 0;
-  const int tid = threadIdx.x;
-  for (int64_t tile = blockIdx.x; tile < a.tiles; tile += gridDim.x) {
-    const int64_t r0 = a.trow[tile], e0 = a.tedge[tile];
-    const int nR = (int)(a.trow[tile + 1] - r0), nE = (int)(a.tedge[tile + 1] - e0);
-    for (int k = tid; k < nE; k += 256) s_val[k] = __ldg(cin + __ldg(a.csrc + e0 + k));
-    for (int k = tid; k < nR; k += 256) s_end[k] = (uint32_t)(a.crp[r0 + k + 1] - e0);
-    for (int k = tid; k <= nR; k += 256) s_sum[k] = 0.0;
-    if (tid == 0) s_end[nR] = 0x7fffffffu;
+  const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
+  const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
+  constexpr unsigned NWARP = PR_CTA / 32;
+  for (int64_t w = blockIdx.x; w < a.nwin; w += gridDim.x) {
+    const int64_t base = w * PRW;
+    const int nrows = (int)min((int64_t)PRW, a.n_slots - base);
+    for (int i = threadIdx.x; i < PRW; i += PR_CTA) s_y[i] = 0.0;
     __syncthreads();
-    const int total = nR + nE;
-    const int d = tid * IPT;
-    if (d < total) {
-      int lo = max(d - nE, 0), hi = min(d, nR);
-      while (lo < hi) {
-        int p = (lo + hi) >> 1;
-        if ((int)s_end[p] <= d - p - 1) lo = p + 1;
-        else hi = p;
-      }
-      int i = lo, j = d - lo;
+    // light rows: lane-per-row over the SELL-32 slices of this window
+    const int64_t s1 = a.win_slice[w + 1];
+    for (int64_t sl = a.win_slice[w] + warp; sl < s1; sl += NWARP) {
+      const uint32_t L = a.slice_len[sl];
+      const uint32_t* p = a.slab + a.slice_off[sl] + lane;
+      const int32_t row = a.lane_row[sl * 32 + lane];
       double acc = 0.0;
-      bool first = true;
+      uint32_t j = 0;
+      for (; j + PR_U <= L; j += PR_U) {
+        uint32_t e[PR_U];
 #pragma unroll
-      for (int k = 0; k < IPT; k++) {
-        if (d + k < total) {
-          if (j < (int)s_end[i]) {
-            acc += (double)s_val[j];
-            j++;
-          } else {
-            if (first) {
-              atomicAdd(&s_sum[i], acc);  // may hold carries from earlier threads
-              first = false;
-            } else {
-              s_sum[i] = acc;             // row lies entirely in this thread
-            }
-            acc = 0.0;
-            i++;
-          }
+        for (int u = 0; u < PR_U; u++) e[u] = ld_stream_u32(p + 32 * (j + u), pf);
+        float v[PR_U];
+#pragma unroll
+        for (int u = 0; u < PR_U; u++) v[u] = e[u] != PR_SENT ? ld_keep_f32(cin + e[u], pl) : 0.0f;
+#pragma unroll
+        for (int u = 0; u < PR_U; u++) acc += (double)v[u];
+      }
+      for (; j < L; j++) {
+        uint32_t e = ld_stream_u32(p + 32 * j, pf);
+        if (e != PR_SENT) acc += (double)ld_keep_f32(cin + e, pl);
+      }
+      if (row >= 0) s_y[row - base] = acc;
+    }
+    // heavy rows: warp-per-row over the CSC
+    const int64_t h1 = a.win_heavy[w + 1];
+    for (int64_t h = a.win_heavy[w] + warp; h < h1; h += NWARP) {
+      const int32_t r = a.heavy_row[h];
+      const uint32_t e0 = a.crp[r], e1 = a.crp[r + 1];
+      double acc = 0.0;
+      for (uint32_t e = e0 + lane; e < e1; e += 32 * 4) {
+        float v[4];
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+          uint32_t ee = e + 32 * u;
+          v[u] = ee < e1 ? ld_keep_f32(cin + ld_stream_i32(a.csrc + ee, pf), pl) : 0.0f;
         }
+#pragma unroll
+        for (int u = 0; u < 4; u++) acc += (double)v[u];
       }
-      if (acc != 0.0) atomicAdd(&s_sum[i], acc);
+      acc = warp_sum_f64(acc);
+      if (lane == 0) s_y[r - base] = acc;
     }
     __syncthreads();
-    const bool split0 = nR > 0 && (int64_t)a.crp[r0] < e0;
-    for (int k = tid; k < nR; k += 256) {
-      double y = s_sum[k];
-      if (k == 0 && split0) {
-        atomicAdd(&a.ysplit[r0], y);
-      } else {
-        pr_finalize<SLOTS>(a, r0 + k, y, addc, cout, my_delta, my_dang);
+    // fused update of the window's rows (coalesced x / D / contrib)
+    for (int i0 = threadIdx.x; i0 < nrows; i0 += PR_CTA * 4) {
+      double xo[4];
+      uint32_t Dv[4];
+#pragma unroll
+      for (int u = 0; u < 4; u++) {
+        int i = i0 + u * PR_CTA;
+        xo[u] = i < nrows ? __ldcs(a.x + base + i) : 0.0;
+        Dv[u] = i < nrows ? __ldcs(a.D + base + i) : 0u;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; u++) {
+        int i = i0 + u * PR_CTA;
+        if (i < nrows) pr_finalize<SLOTS>(a, base + i, s_y[i], xo[u], Dv[u], addc, cout, my_delta, my_dang);
       }
     }
-    if (tid == 0) {
-      int covered = nR ? (int)s_end[nR - 1] : 0;
-      if (nE > covered) atomicAdd(&a.ysplit[r0 + nR], s_sum[nR]);
-    }
     __syncthreads();
-  }
-  double dsum = block_sum_f64(my_delta, s_red);
-  __syncthreads();
-  double gsum = block_sum_f64(my_dang, s_red);
-  if (tid == 0) {
-    if (dsum != 0.0) atomicAdd(&st->delta[(t + 1) % 3], dsum);
-    if (gsum != 0.0) atomicAdd(&st->dang[(t + 1) % 3], gsum);
-  }
-}
-
-template <bool SLOTS>
-__global__ void __launch_bounds__(256) k_pr_fixup(PrArgs a) {
-  __shared__ double s_red[32];
-  PrState* st = a.st;
-  if (st->stop) return;
-  const unsigned t = st->iter;
-  float* cout = a.contrib[(t + 1) & 1];
-  const double addc = a.base + a.damp * st->dang[t % 3] * a.invN;
-  double my_delta = 0, my_dang = 0;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < a.n_split; i += (int64_t)gridDim.x * blockDim.x) {
-    int64_t v = a.split[i];
-    double y = a.ysplit[v];
-    a.ysplit[v] = 0.0;
-    pr_finalize<SLOTS>(a, v, y, addc, cout, my_delta, my_dang);
   }
   double dsum = block_sum_f64(my_delta, s_red);
   __syncthreads();
@@ -251,15 +246,20 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   r.x.alloc(c, sizeof(double) * ns);
   r.contrib[0].alloc(c, sizeof(float) * ns);
   r.contrib[1].alloc(c, sizeof(float) * ns);
-  r.ysplit.alloc(c, sizeof(double) * (ns + 1));
   r.gnew.alloc(c, sizeof(double) * std::max<int64_t>(d.n_groups, 1));
   r.pst.alloc(c, sizeof(PrState));
   PrArgs a;
+  a.slab = d.pr_slab.as<uint32_t>();
+  a.slice_len = d.pr_slice_len.as<uint32_t>();
+  a.slice_off = d.pr_slice_off.as<uint64_t>();
+  a.lane_row = d.pr_lane_row.as<int32_t>();
+  a.heavy_row = d.pr_heavy_row.as<int32_t>();
+  a.win_slice = d.pr_win_slice.as<int64_t>();
+  a.win_heavy = d.pr_win_heavy.as<int64_t>();
   a.crp = d.crp.as<uint32_t>();
   a.csrc = d.csrc.as<int32_t>();
-  a.trow = d.pr_tile_row.as<int64_t>();
-  a.tedge = d.pr_tile_edge.as<int64_t>();
-  a.tiles = d.pr_tiles;
+  a.nwin = d.pr_nwin;
+  a.n_slots = ns;
   a.x = r.x.as<double>();
   a.contrib[0] = r.contrib[0].as<float>();
   a.contrib[1] = r.contrib[1].as<float>();
@@ -267,9 +267,6 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   a.kind = d.identity ? nullptr : d.kind.as<uint8_t>();
   a.gid = d.n_groups ? d.gid.as<int32_t>() : nullptr;
   a.gnew = r.gnew.as<double>();
-  a.ysplit = r.ysplit.as<double>();
-  a.split = d.pr_split.as<int32_t>();
-  a.n_split = d.pr_n_split;
   a.damp = o.damping;
   a.base = (1.0 - o.damping) / (double)g->n;
   a.invN = 1.0 / (double)g->n;
@@ -281,7 +278,6 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   CUDA_OK(cudaEventCreate(&e1));
   CUDA_OK(cudaEventRecord(e0, s));
   CUDA_OK(cudaMemsetAsync(r.pst.p, 0, sizeof(PrState), s));
-  CUDA_OK(cudaMemsetAsync(r.ysplit.p, 0, sizeof(double) * (ns + 1), s));
   int gi = grid_for(c, ns);
   if (slots) k_pr_init<true><<<gi, 256, 0, s>>>(a, ns, 1.0 / (double)g->n);
   else k_pr_init<false><<<gi, 256, 0, s>>>(a, ns, 1.0 / (double)g->n);
@@ -289,23 +285,17 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   int launches = 1;
 
   int occ = 0;
-  if (slots) CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_pull<7, true>, 256, 0));
-  else CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_pull<7, false>, 256, 0));
-  int grid = (int)std::max<int64_t>(1, std::min<int64_t>(d.pr_tiles, (int64_t)std::max(1, occ) * c->num_sms));
-  int grid_fix = (int)std::max<int64_t>(1, std::min<int64_t>((d.pr_n_split + 255) / 256, c->num_sms * 4));
+  if (slots) CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<true>, PR_CTA, 0));
+  else CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<false>, PR_CTA, 0));
+  int grid = (int)std::max<int64_t>(1, std::min<int64_t>(d.pr_nwin, (int64_t)std::max(1, occ) * c->num_sms));
   int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 255) / 256, c->num_sms * 4));
 
   KTimer kt(o.profile != 0, s);
   auto one_iter = [&](int& nl) {
     kt.begin();
-    if (slots) k_pr_pull<7, true><<<grid, 256, 0, s>>>(a);
-    else k_pr_pull<7, false><<<grid, 256, 0, s>>>(a);
+    if (slots) k_pr_sell<true><<<grid, PR_CTA, 0, s>>>(a);
+    else k_pr_sell<false><<<grid, PR_CTA, 0, s>>>(a);
     kt.end();
-    if (slots) {
-      if (d.pr_n_split) k_pr_fixup<true><<<grid_fix, 256, 0, s>>>(a), nl++;
-    } else {
-      if (d.pr_n_split) k_pr_fixup<false><<<grid_fix, 256, 0, s>>>(a), nl++;
-    }
     nl++;
     if (d.n_groups) {
       k_pr_merge<<<grid_merge, 256, 0, s>>>(a, d.gptr.as<int32_t>(), d.gslots.as<int32_t>(), d.n_groups);
@@ -351,9 +341,9 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   info.last_delta = h.last_delta;
   info.edges_scanned = (int64_t)h.iter * d.m_slots;
   info.vertices_active = (int64_t)h.iter * ns;
-  // bytes model: 8 B per in-edge (csrc 4 + contrib gather 4) and
-  // 28 B per slot (crp 4 + x read 8 + x write 8 + contrib write 4 + D 4)
-  info.bytes_model = (int64_t)h.iter * (8 * d.m_slots + 28 * ns);
+  // bytes model: 8 B per in-edge (source id 4 + contrib gather 4) and
+  // 24 B per slot (x read 8 + x write 8 + contrib write 4 + D 4)
+  info.bytes_model = (int64_t)h.iter * (8 * d.m_slots + 24 * ns);
   info.kernel_launches = launches;
   info.sweep_launches = kt.launches();
   info.sweep_ms = kt.total_ms();

@@ -13,7 +13,7 @@
 //   time per warp and their edges are distributed over the lanes by a warp
 //   prefix scan (every lane relaxes one edge per round: coalesced 8-byte
 //   {col, w} loads, no divergence from degree skew).  Newly improved slots
-//   are deduplicated with an iteration stamp (atomicMax) and appended with
+//   are deduplicated with a 1-bit-per-slot bitmap (atomicOr) and appended with
 //   warp-aggregated atomics.
 // TPV mapping (the paper's thread-per-vertex, §2/§4 layouts): tpv.cu.
 #include <algorithm>
@@ -28,25 +28,33 @@
 namespace gx {
 
 // ---------------------------------------------------------------- helpers
+// L2 residency: dist is the only vector gathered at
+// random, so its loads / atomics carry evict_last; the edge stream, queues
+// and row offsets carry evict_first.  Frontier dedupe uses 1-bit-per-slot
+// bitmaps (2 MB at 16M slots, always L2 resident), double-buffered by
+// iteration parity: iteration t sets bits of bm[(t+1)&1] and clears bm[t&1].
+struct SsspAux {
+  uint32_t* bm[2];             // "already in the next frontier" bitmaps
+  const uint32_t* heavy;       // bitmap: out-degree > HEAVY_DEG
+  int64_t nwords;
+};
+
 __device__ __forceinline__ void push_next(bool push, uint32_t v, const uint32_t* __restrict__ rp,
-                                          SsspCtr* nxt, int32_t* __restrict__ lq_out,
-                                          int32_t* __restrict__ hq_out, uint32_t* __restrict__ hb_out) {
+                                          const uint32_t* __restrict__ heavybm, SsspCtr* nxt,
+                                          int32_t* __restrict__ lq_out, int32_t* __restrict__ hq_out,
+                                          uint32_t* __restrict__ hb_out) {
   unsigned bal = __ballot_sync(FULL, push);
   if (!bal) return;
-  bool heavy = false;
-  uint32_t vdeg = 0;
-  if (push) {
-    vdeg = rp[v + 1] - rp[v];
-    heavy = vdeg > HEAVY_DEG;
-  }
+  const bool heavy = push && ((__ldg(heavybm + (v >> 5)) >> (v & 31)) & 1u);
   unsigned lb = __ballot_sync(FULL, push && !heavy);
   if (lb) {
     unsigned leader = __ffs(lb) - 1, base = 0;
     if (lane_id() == leader) base = atomicAdd(&nxt->lcount, (unsigned)__popc(lb));
     base = __shfl_sync(FULL, base, leader);
-    if (push && !heavy) lq_out[base + __popc(lb & lanemask_lt())] = (int32_t)v;
+    if (push && !heavy) st_stream_i32(lq_out + base + __popc(lb & lanemask_lt()), (int32_t)v, l2_evict_first());
   }
-  if (push && heavy) {
+  if (heavy) {
+    uint32_t vdeg = rp[v + 1] - rp[v];
     unsigned long long add = (1ull << 32) | (unsigned long long)((vdeg + HCHUNK - 1) / HCHUNK);
     unsigned long long old = atomicAdd(&nxt->hpack, add);
     hq_out[old >> 32] = (int32_t)v;
@@ -54,39 +62,52 @@ __device__ __forceinline__ void push_next(bool push, uint32_t v, const uint32_t*
   }
 }
 
-// relax one edge; returns true iff v must be appended to the next frontier
-__device__ __forceinline__ bool relax(uint2 ed, uint32_t du, uint32_t* __restrict__ dist,
-                                      uint32_t* __restrict__ mark, unsigned stamp) {
-  uint32_t v = ed.x;
+// relax one edge given the (possibly stale, never smaller) current distance
+// `cur` of its head; returns true iff the head must join the next frontier
+__device__ __forceinline__ bool relax2(uint2 ed, uint32_t du, uint32_t cur, uint32_t* __restrict__ dist,
+                                       uint32_t* __restrict__ bm_next, uint64_t pl) {
   uint32_t nd = du + ed.y;
   if (nd < du) nd = INF - 1;  // saturate (never the fixed point)
-  if (nd < __ldcg(dist + v)) {
-    uint32_t old = atomicMin(dist + v, nd);
-    if (nd < old && atomicMax(mark + v, stamp) < stamp) return true;
+  if (nd < cur) {
+    uint32_t old = atom_min_l2(dist + ed.x, nd, pl);
+    if (nd < old) {
+      uint32_t bit = 1u << (ed.x & 31);
+      if (!(atom_or_l2(bm_next + (ed.x >> 5), bit, pl) & bit)) return true;
+    }
   }
   return false;
 }
 
+__device__ __forceinline__ void clear_bitmap(uint32_t* bm, int64_t nwords) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nwords; i += (int64_t)gridDim.x * blockDim.x)
+    bm[i] = 0u;
+}
+
 // ---------------------------------------------------------------- LB sweep
+constexpr int SU = 4;  // edges in flight per lane per round
+
 __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj,
-                                                 uint32_t* __restrict__ dist, uint32_t* __restrict__ mark,
+                                                 uint32_t* __restrict__ dist, SsspAux ax,
                                                  SsspQueues qs, SsspState* __restrict__ st) {
   __shared__ unsigned long long sh[32];
   const unsigned t = st->iter;
   if (st->stop) return;
+  const bool odd = t & 1;
   SsspCtr* cur = &st->ctr[t % 3];
   SsspCtr* nxt = &st->ctr[(t + 1) % 3];
-  const int32_t* lq_in = qs.lq[t & 1];
-  int32_t* lq_out = qs.lq[(t + 1) & 1];
-  const int32_t* hq_in = qs.hq[t & 1];
-  const uint32_t* hb_in = qs.hb[t & 1];
-  int32_t* hq_out = qs.hq[(t + 1) & 1];
-  uint32_t* hb_out = qs.hb[(t + 1) & 1];
+  const int32_t* lq_in = odd ? qs.lq[1] : qs.lq[0];
+  int32_t* lq_out = odd ? qs.lq[0] : qs.lq[1];
+  const int32_t* hq_in = odd ? qs.hq[1] : qs.hq[0];
+  const uint32_t* hb_in = odd ? qs.hb[1] : qs.hb[0];
+  int32_t* hq_out = odd ? qs.hq[0] : qs.hq[1];
+  uint32_t* hb_out = odd ? qs.hb[0] : qs.hb[1];
   const unsigned lcount = cur->lcount;
   const unsigned long long hp = cur->hpack;
   const unsigned hcount = (unsigned)(hp >> 32), hchunks = (unsigned)(hp & 0xffffffffull);
-  const unsigned stamp = t + 1;
   const unsigned lane = lane_id();
+  const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
+  uint32_t* bm_next = odd ? ax.bm[0] : ax.bm[1];
+  clear_bitmap(odd ? ax.bm[1] : ax.bm[0], ax.nwords);
   unsigned long long my_edges = 0;
 
   // heavy slots: HCHUNK-edge work items
@@ -102,19 +123,25 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
       else hi = mid - 1;
     }
     int32_t u = hq_in[lo];
-    uint32_t du = __ldcg(dist + u);
+    uint32_t du = ld_l2_u32(dist + u, pl);
     uint32_t a = rp[u] + (c - hb_in[lo]) * HCHUNK;
     uint32_t b = min(a + (uint32_t)HCHUNK, rp[u + 1]);
-    for (uint32_t e0 = a; e0 < b; e0 += 32) {
-      uint32_t e = e0 + lane;
-      bool push = false;
-      uint32_t v = 0;
-      if (e < b) {
-        uint2 ed = adj[e];
-        v = ed.x;
-        push = relax(ed, du, dist, mark, stamp);
+    for (uint32_t e0 = a; e0 < b; e0 += 32 * SU) {
+      uint2 ed[SU];
+      bool act[SU], push[SU];
+#pragma unroll
+      for (int q = 0; q < SU; q++) {
+        uint32_t e = e0 + q * 32 + lane;
+        act[q] = e < b;
+        ed[q] = act[q] ? ld_stream_u2(adj + e, pf) : make_uint2(0, 0);
       }
-      push_next(push, v, rp, nxt, lq_out, hq_out, hb_out);
+      uint32_t cv[SU];
+#pragma unroll
+      for (int q = 0; q < SU; q++) cv[q] = act[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
+#pragma unroll
+      for (int q = 0; q < SU; q++) push[q] = act[q] && relax2(ed[q], du, cv[q], dist, bm_next, pl);
+#pragma unroll
+      for (int q = 0; q < SU; q++) push_next(push[q], ed[q].x, rp, ax.heavy, nxt, lq_out, hq_out, hb_out);
     }
     if (lane == 0) my_edges += b - a;
   }
@@ -128,33 +155,40 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
     unsigned idx = base + lane;
     uint32_t start = 0, deg = 0, du = 0;
     if (idx < lcount) {
-      int32_t u = lq_in[idx];
-      start = rp[u];
-      deg = rp[u + 1] - start;
-      du = __ldcg(dist + u);
+      int32_t u = ld_stream_i32(lq_in + idx, pf);
+      start = ld_stream_u32(rp + u, pf);
+      deg = ld_stream_u32(rp + u + 1, pf) - start;
+      du = ld_l2_u32(dist + u, pl);
     }
     uint32_t incl = warp_incl_scan_u32(deg);
     uint32_t excl = incl - deg;
     uint32_t total = __shfl_sync(FULL, incl, 31);
-    for (uint32_t k0 = 0; k0 < total; k0 += 32) {
-      uint32_t k = k0 + lane;
-      int j = 0;
+    for (uint32_t k0 = 0; k0 < total; k0 += 32 * SU) {
+      uint2 ed[SU];
+      uint32_t od[SU];
+      bool act[SU], push[SU];
 #pragma unroll
-      for (int s = 16; s; s >>= 1) {
-        uint32_t ex = __shfl_sync(FULL, excl, j + s);
-        if (ex <= k) j += s;
+      for (int q = 0; q < SU; q++) {
+        uint32_t k = k0 + q * 32 + lane;
+        int j = 0;
+#pragma unroll
+        for (int s = 16; s; s >>= 1) {
+          uint32_t ex = __shfl_sync(FULL, excl, j + s);
+          if (ex <= k) j += s;
+        }
+        uint32_t os = __shfl_sync(FULL, start, j);
+        uint32_t oe = __shfl_sync(FULL, excl, j);
+        od[q] = __shfl_sync(FULL, du, j);
+        act[q] = k < total;
+        ed[q] = act[q] ? ld_stream_u2(adj + os + (k - oe), pf) : make_uint2(0, 0);
       }
-      uint32_t os = __shfl_sync(FULL, start, j);
-      uint32_t oe = __shfl_sync(FULL, excl, j);
-      uint32_t od = __shfl_sync(FULL, du, j);
-      bool push = false;
-      uint32_t v = 0;
-      if (k < total) {
-        uint2 ed = adj[os + (k - oe)];
-        v = ed.x;
-        push = relax(ed, od, dist, mark, stamp);
-      }
-      push_next(push, v, rp, nxt, lq_out, hq_out, hb_out);
+      uint32_t cv[SU];
+#pragma unroll
+      for (int q = 0; q < SU; q++) cv[q] = act[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
+#pragma unroll
+      for (int q = 0; q < SU; q++) push[q] = act[q] && relax2(ed[q], od[q], cv[q], dist, bm_next, pl);
+#pragma unroll
+      for (int q = 0; q < SU; q++) push_next(push[q], ed[q].x, rp, ax.heavy, nxt, lq_out, hq_out, hb_out);
     }
     if (lane == 0) my_edges += total;
   }
@@ -170,15 +204,15 @@ __global__ void __launch_bounds__(256) k_sssp_local(const int32_t* __restrict__ 
                                                     const int32_t* __restrict__ teptr, const uint2* __restrict__ tedges,
                                                     const int32_t* __restrict__ titers, int64_t ntiles,
                                                     const uint32_t* __restrict__ rp, uint32_t* __restrict__ dist,
-                                                    uint32_t* __restrict__ mark, SsspQueues qs, SsspState* __restrict__ st) {
+                                                    SsspAux ax, SsspQueues qs, SsspState* __restrict__ st) {
   __shared__ uint32_t sd[256];
   const unsigned t = st->iter;
   if (st->stop) return;
   SsspCtr* nxt = &st->ctr[(t + 1) % 3];
-  int32_t* lq_out = qs.lq[(t + 1) & 1];
-  int32_t* hq_out = qs.hq[(t + 1) & 1];
-  uint32_t* hb_out = qs.hb[(t + 1) & 1];
-  const unsigned stamp = t + 1;
+  int32_t* lq_out = (t & 1) ? qs.lq[0] : qs.lq[1];
+  int32_t* hq_out = (t & 1) ? qs.hq[0] : qs.hq[1];
+  uint32_t* hb_out = (t & 1) ? qs.hb[0] : qs.hb[1];
+  uint32_t* bm_next = (t & 1) ? ax.bm[0] : ax.bm[1];
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     int a = tptr[tile], nm = tptr[tile + 1] - a;
     int ea = teptr[tile], ne = teptr[tile + 1] - ea;
@@ -211,10 +245,10 @@ __global__ void __launch_bounds__(256) k_sssp_local(const int32_t* __restrict__ 
         uint32_t nd = sd[i];
         if (nd < __ldcg(dist + v)) {
           uint32_t old = atomicMin(dist + v, nd);
-          push = nd < old && atomicMax(mark + v, stamp) < stamp;
+          push = nd < old && !(atomicOr(bm_next + (v >> 5), 1u << (v & 31)) & (1u << (v & 31)));
         }
       }
-      push_next(push, v, rp, nxt, lq_out, hq_out, hb_out);
+      push_next(push, v, rp, ax.heavy, nxt, lq_out, hq_out, hb_out);
     }
     __syncthreads();
   }
@@ -229,15 +263,15 @@ __global__ void __launch_bounds__(256) k_sssp_local(const int32_t* __restrict__ 
 __global__ void __launch_bounds__(256) k_sssp_merge(const int32_t* __restrict__ gptr, const int32_t* __restrict__ gslots,
                                                     const int32_t* __restrict__ ginptr, const uint2* __restrict__ gin,
                                                     int64_t ngroups, int merge_min, const uint32_t* __restrict__ rp,
-                                                    uint32_t* __restrict__ dist, uint32_t* __restrict__ mark,
+                                                    uint32_t* __restrict__ dist, SsspAux ax,
                                                     SsspQueues qs, SsspState* __restrict__ st) {
   const unsigned t = st->iter;
   if (st->stop) return;
   SsspCtr* nxt = &st->ctr[(t + 1) % 3];
-  int32_t* lq_out = qs.lq[(t + 1) & 1];
-  int32_t* hq_out = qs.hq[(t + 1) & 1];
-  uint32_t* hb_out = qs.hb[(t + 1) & 1];
-  const unsigned stamp = t + 1;
+  int32_t* lq_out = (t & 1) ? qs.lq[0] : qs.lq[1];
+  int32_t* hq_out = (t & 1) ? qs.hq[0] : qs.hq[1];
+  uint32_t* hb_out = (t & 1) ? qs.hb[0] : qs.hb[1];
+  uint32_t* bm_next = (t & 1) ? ax.bm[0] : ax.bm[1];
   const unsigned lane = lane_id();
   int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -276,11 +310,11 @@ __global__ void __launch_bounds__(256) k_sssp_merge(const int32_t* __restrict__ 
         uint32_t old = dist[s];
         if (old != mval) {
           dist[s] = mval;
-          push = mval < old && atomicMax(mark + s, stamp) < stamp;
+          push = mval < old && !(atomicOr(bm_next + (s >> 5), 1u << (s & 31)) & (1u << (s & 31)));
           if (mval > old) atomicAdd(&st->raised, 1u);
         }
       }
-      push_next(push, s, rp, nxt, lq_out, hq_out, hb_out);
+      push_next(push, s, rp, ax.heavy, nxt, lq_out, hq_out, hb_out);
     }
   }
 }
@@ -321,6 +355,18 @@ __global__ void k_sssp_init(uint32_t* __restrict__ dist, const int32_t* __restri
   st->active = nslots;
 }
 
+// bitmap of slots whose out-degree exceeds HEAVY_DEG (push-time class test)
+__global__ void k_heavy_bitmap(const uint32_t* __restrict__ rp, int64_t n, uint32_t* __restrict__ hb) {
+  for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w * 32 < n; w += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t bits = 0;
+    for (int b = 0; b < 32; b++) {
+      int64_t v = w * 32 + b;
+      if (v < n && rp[v + 1] - rp[v] > HEAVY_DEG) bits |= 1u << b;
+    }
+    hb[w] = bits;
+  }
+}
+
 // R36: max out-degree vertex of the canonical input, ties to the lowest id
 __global__ void k_argmax_deg(const int64_t* __restrict__ rp, int64_t n, unsigned long long* __restrict__ out) {
   unsigned long long best = 0;
@@ -348,7 +394,7 @@ int64_t default_source(gx_graph* g) {
 }
 
 // ---------------------------------------------------------------- driver
-void run_sssp_tpv_iter(gx_graph* g, SsspQueues qs, SsspState* st, int& launches);  // tpv.cu
+void run_sssp_tpv_iter(gx_graph* g, SsspQueues qs, SsspState* st, int& launches);  // tpv.cu (uses SsspAux via g)
 void ensure_tpv(gx_graph* g);                                                    // tpv.cu
 
 void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
@@ -366,7 +412,8 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   if (mapping == GX_MAP_TPV) ensure_tpv(g);
   int64_t ns = d.n_slots;
   r.dist.alloc(c, sizeof(uint32_t) * ns);
-  r.mark.alloc(c, sizeof(uint32_t) * ns);
+  const int64_t nwords = (ns + 31) / 32;
+  r.mark.alloc(c, sizeof(uint32_t) * 3 * nwords);   // bm[0], bm[1], heavy
   for (int i = 0; i < 2; i++) {
     r.q[i].alloc(c, sizeof(int32_t) * ns);
     r.hq[i].alloc(c, sizeof(int32_t) * ns);
@@ -380,6 +427,13 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     qs.hb[i] = r.hbase[i].as<uint32_t>();
   }
   SsspState* st = r.st.as<SsspState>();
+  SsspAux ax;
+  ax.bm[0] = r.mark.as<uint32_t>();
+  ax.bm[1] = r.mark.as<uint32_t>() + nwords;
+  ax.heavy = r.mark.as<uint32_t>() + 2 * nwords;
+  ax.nwords = nwords;
+  k_heavy_bitmap<<<grid_for(c, ns), 256, 0, s>>>(d.rp.as<uint32_t>(), ns, r.mark.as<uint32_t>() + 2 * nwords);
+  CUDA_OK(cudaGetLastError());
   // source copies: owner slot + replica slots
   std::vector<int32_t> srcs;
   if (d.identity) {
@@ -399,7 +453,7 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   CUDA_OK(cudaEventCreate(&e1));
   CUDA_OK(cudaEventRecord(e0, s));
   CUDA_OK(cudaMemsetAsync(r.dist.p, 0xFF, sizeof(uint32_t) * ns, s));
-  CUDA_OK(cudaMemsetAsync(r.mark.p, 0, sizeof(uint32_t) * ns, s));
+  CUDA_OK(cudaMemsetAsync(r.mark.p, 0, sizeof(uint32_t) * 2 * nwords, s));
   CUDA_OK(cudaMemsetAsync(r.st.p, 0, sizeof(SsspState), s));
   k_sssp_init<<<1, 32, 0, s>>>(r.dist.as<uint32_t>(), dsrc.as<int32_t>(), (int)srcs.size(), d.rp.as<uint32_t>(),
                                qs, st);
@@ -420,20 +474,20 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
       run_sssp_tpv_iter(g, qs, st, nl);
     } else {
       k_sssp_lb<<<grid_lb, 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), r.dist.as<uint32_t>(),
-                                        r.mark.as<uint32_t>(), qs, st);
+                                        ax, qs, st);
       nl++;
     }
     kt.end();
     if (d.n_tiles && g->knobs.smem) {
       k_sssp_local<<<grid_local, 256, 0, s>>>(d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(), d.t_eptr.as<int32_t>(),
                                               d.t_edges.as<uint2>(), d.t_iters.as<int32_t>(), d.n_tiles,
-                                              d.rp.as<uint32_t>(), r.dist.as<uint32_t>(), r.mark.as<uint32_t>(), qs, st);
+                                              d.rp.as<uint32_t>(), r.dist.as<uint32_t>(), ax, qs, st);
       nl++;
     }
     if (d.n_groups) {
       k_sssp_merge<<<grid_merge, 256, 0, s>>>(d.gptr.as<int32_t>(), d.gslots.as<int32_t>(), d.g_in_ptr.as<int32_t>(),
                                               d.g_in.as<uint2>(), d.n_groups, merge_min ? 1 : 0, d.rp.as<uint32_t>(),
-                                              r.dist.as<uint32_t>(), r.mark.as<uint32_t>(), qs, st);
+                                              r.dist.as<uint32_t>(), ax, qs, st);
       nl++;
     }
     k_sssp_advance<<<1, 1, 0, s>>>(st, o.max_iters);
