@@ -154,7 +154,8 @@ static void build_csc_and_tiles(gx_graph* g) {
   } else {
     CUDA_OK(cudaMemsetAsync(d.crp.p, 0, sizeof(uint32_t) * (n + 1), s));
   }
-  build_pr_sell(g);
+  build_window_sell<uint32_t>(c, d.crp.as<uint32_t>(), reinterpret_cast<const uint32_t*>(d.csrc.p), n, PR_SENT,
+                              d.pr_sell);
 }
 
 void ensure_csc(gx_graph* g) {

@@ -91,6 +91,17 @@ struct SlotGraph {
   gx_transform_info info{};
 };
 
+// Windowed SELL-32 layout (sell.cu): per window of SELL_W rows, the light
+// rows sorted by degree into 32-lane slices; heavy rows listed separately.
+struct SellLayout {
+  int64_t nwin = 0, nslices = 0, nheavy = 0, slab_len = 0;
+  DBuf lane_row, heavy_row;   // i32
+  DBuf win_slice, win_heavy;  // i64 [nwin+1]
+  DBuf slice_len, slice_off;  // u32 [nslices+1], u64 [nslices+1]
+  DBuf slab;                  // payload (u32 or uint2), sentinel padding
+  bool built() const { return slab.p != nullptr; }
+};
+
 // Device layouts of the current slot graph.
 struct DevGraph {
   int64_t n = 0, n_slots = 0, m_slots = 0;
@@ -105,15 +116,12 @@ struct DevGraph {
   DBuf gptr, gslots;           // groups: ptr [ng+1], slots (owner first)
   int64_t n_groups = 0;
   DBuf g_in_ptr, g_in;         // per-group owner in-edges (src slot, w) for SSSP pull
-  // PR windowed SELL-32 pull layout (sell.cu): per window of PRW rows the
-  // light rows sorted by in-degree into 32-lane slices, heavy rows listed
-  int64_t pr_nwin = 0, pr_nslices = 0, pr_nheavy = 0, pr_slab_len = 0;
-  DBuf pr_lane_row, pr_heavy_row;   // i32
-  DBuf pr_win_slice, pr_win_heavy;  // i64 [nwin+1]
-  DBuf pr_slice_len, pr_slice_off;  // u32 [nslices+1], u64 [nslices+1]
-  DBuf pr_slab;                     // u32 source slots, PR_SENT padding
-  // LB SSSP
-  int64_t n_heavy = 0;
+  // windowed SELL-32 layouts (sell.cu): PR pull over in-edges, SSSP dense
+  // push over out-edges
+  SellLayout pr_sell, sssp_sell;
+  // LB SSSP: static chunk list of rows with out-degree > HEAVY_DEG, heavy bitmap
+  int64_t nhc = 0;
+  DBuf hc_row, hc_start, heavy_bm;
   // TPV / SELL-32 (filled on demand)
   bool tpv_ready = false;
   int64_t n_warps_tpv = 0;

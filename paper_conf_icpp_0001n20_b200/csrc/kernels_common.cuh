@@ -195,3 +195,13 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, unsigned
       : "memory");
 }
 }  // namespace gx
+
+namespace gx {
+// fire-and-forget reductions (RED): no return value, no round trip
+__device__ __forceinline__ void red_min_l2(uint32_t* p, uint32_t v, uint64_t pol) {
+  asm volatile("red.global.min.L2::cache_hint.u32 [%0], %1, %2;" ::"l"(p), "r"(v), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void red_or_l2(uint32_t* p, uint32_t v, uint64_t pol) {
+  asm volatile("red.global.or.L2::cache_hint.b32 [%0], %1, %2;" ::"l"(p), "r"(v), "l"(pol) : "memory");
+}
+}  // namespace gx

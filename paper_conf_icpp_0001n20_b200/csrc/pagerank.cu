@@ -249,16 +249,17 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   r.gnew.alloc(c, sizeof(double) * std::max<int64_t>(d.n_groups, 1));
   r.pst.alloc(c, sizeof(PrState));
   PrArgs a;
-  a.slab = d.pr_slab.as<uint32_t>();
-  a.slice_len = d.pr_slice_len.as<uint32_t>();
-  a.slice_off = d.pr_slice_off.as<uint64_t>();
-  a.lane_row = d.pr_lane_row.as<int32_t>();
-  a.heavy_row = d.pr_heavy_row.as<int32_t>();
-  a.win_slice = d.pr_win_slice.as<int64_t>();
-  a.win_heavy = d.pr_win_heavy.as<int64_t>();
+  const SellLayout& PL = d.pr_sell;
+  a.slab = PL.slab.as<uint32_t>();
+  a.slice_len = PL.slice_len.as<uint32_t>();
+  a.slice_off = PL.slice_off.as<uint64_t>();
+  a.lane_row = PL.lane_row.as<int32_t>();
+  a.heavy_row = PL.heavy_row.as<int32_t>();
+  a.win_slice = PL.win_slice.as<int64_t>();
+  a.win_heavy = PL.win_heavy.as<int64_t>();
   a.crp = d.crp.as<uint32_t>();
   a.csrc = d.csrc.as<int32_t>();
-  a.nwin = d.pr_nwin;
+  a.nwin = PL.nwin;
   a.n_slots = ns;
   a.x = r.x.as<double>();
   a.contrib[0] = r.contrib[0].as<float>();
@@ -287,7 +288,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   int occ = 0;
   if (slots) CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<true>, PR_CTA, 0));
   else CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<false>, PR_CTA, 0));
-  int grid = (int)std::max<int64_t>(1, std::min<int64_t>(d.pr_nwin, (int64_t)std::max(1, occ) * c->num_sms));
+  int grid = (int)std::max<int64_t>(1, std::min<int64_t>(PL.nwin, (int64_t)std::max(1, occ) * c->num_sms));
   int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 255) / 256, c->num_sms * 4));
 
   KTimer kt(o.profile != 0, s);

@@ -176,21 +176,20 @@ template int64_t build_sell<uint32_t>(Ctx*, const uint32_t*, const uint32_t*, co
 template int64_t build_sell<uint2>(Ctx*, const uint32_t*, const uint2*, const int32_t*, int64_t, uint2, DBuf&, DBuf&,
                                    DBuf&);
 
-// Exact-mode PR pull layout: windows of PRW rows (see pagerank.cu).
-void build_pr_sell(gx_graph* g) {
-  Ctx* c = g->ctx;
+// Windowed degree-sorted SELL-32 (exact-mode PR pull over the CSC, SSSP dense
+// push over the CSR).
+template <class T>
+void build_window_sell(Ctx* c, const uint32_t* rp, const T* payload, int64_t n, T sentinel, SellLayout& L) {
   cudaStream_t s = c->stream;
-  DevGraph& d = g->dg;
-  const int64_t n = d.n_slots;
   const int64_t nwin = (n + PRW - 1) / PRW;
-  d.pr_nwin = nwin;
+  L.nwin = nwin;
   DBuf lane_tmp, heavy_tmp, nl, nh;
-  lane_tmp.alloc(c, sizeof(int32_t) * nwin * PRW);
-  heavy_tmp.alloc(c, sizeof(int32_t) * nwin * PRW);
+  lane_tmp.alloc(c, sizeof(int32_t) * std::max<int64_t>(nwin * PRW, 1));
+  heavy_tmp.alloc(c, sizeof(int32_t) * std::max<int64_t>(nwin * PRW, 1));
   nl.alloc(c, sizeof(int32_t) * (nwin + 1));
   nh.alloc(c, sizeof(int32_t) * (nwin + 1));
-  if (nwin) k_pr_window_sort<PRW><<<nwin, 1024, 0, s>>>(d.crp.as<uint32_t>(), n, lane_tmp.as<int32_t>(),
-                                                        heavy_tmp.as<int32_t>(), nl.as<int32_t>(), nh.as<int32_t>());
+  if (nwin) k_pr_window_sort<PRW><<<nwin, 1024, 0, s>>>(rp, n, lane_tmp.as<int32_t>(), heavy_tmp.as<int32_t>(),
+                                                        nl.as<int32_t>(), nh.as<int32_t>());
   CUDA_OK(cudaGetLastError());
   std::vector<int32_t> hnl(nwin), hnh(nwin);
   CUDA_OK(cudaMemcpyAsync(hnl.data(), nl.p, sizeof(int32_t) * nwin, cudaMemcpyDeviceToHost, s));
@@ -203,28 +202,29 @@ void build_pr_sell(gx_graph* g) {
     hoff[w + 1] = hoff[w] + hnh[w];
     soff[w + 1] = loff[w + 1] / 32;
   }
-  d.pr_nslices = loff[nwin] / 32;
-  d.pr_nheavy = hoff[nwin];
+  L.nslices = loff[nwin] / 32;
+  L.nheavy = hoff[nwin];
   DBuf dloff, dhoff;
   dloff.alloc(c, sizeof(int64_t) * (nwin + 1));
   dhoff.alloc(c, sizeof(int64_t) * (nwin + 1));
   CUDA_OK(cudaMemcpyAsync(dloff.p, loff.data(), sizeof(int64_t) * (nwin + 1), cudaMemcpyHostToDevice, s));
   CUDA_OK(cudaMemcpyAsync(dhoff.p, hoff.data(), sizeof(int64_t) * (nwin + 1), cudaMemcpyHostToDevice, s));
-  d.pr_lane_row.alloc(c, sizeof(int32_t) * (loff[nwin] + 32));
-  d.pr_heavy_row.alloc(c, sizeof(int32_t) * std::max<int64_t>(hoff[nwin], 1));
-  d.pr_win_slice.alloc(c, sizeof(int64_t) * (nwin + 1));
-  d.pr_win_heavy.alloc(c, sizeof(int64_t) * (nwin + 1));
-  CUDA_OK(cudaMemcpyAsync(d.pr_win_slice.p, soff.data(), sizeof(int64_t) * (nwin + 1), cudaMemcpyHostToDevice, s));
-  CUDA_OK(cudaMemcpyAsync(d.pr_win_heavy.p, hoff.data(), sizeof(int64_t) * (nwin + 1), cudaMemcpyHostToDevice, s));
+  L.lane_row.alloc(c, sizeof(int32_t) * (loff[nwin] + 32));
+  L.heavy_row.alloc(c, sizeof(int32_t) * std::max<int64_t>(hoff[nwin], 1));
+  L.win_slice.alloc(c, sizeof(int64_t) * (nwin + 1));
+  L.win_heavy.alloc(c, sizeof(int64_t) * (nwin + 1));
+  CUDA_OK(cudaMemcpyAsync(L.win_slice.p, soff.data(), sizeof(int64_t) * (nwin + 1), cudaMemcpyHostToDevice, s));
+  CUDA_OK(cudaMemcpyAsync(L.win_heavy.p, hoff.data(), sizeof(int64_t) * (nwin + 1), cudaMemcpyHostToDevice, s));
   if (nwin)
     k_pr_window_lanes<<<grid_for(c, nwin * 256), 256, 0, s>>>(lane_tmp.as<int32_t>(), heavy_tmp.as<int32_t>(), nl.as<int32_t>(),
                                                               nh.as<int32_t>(), dloff.as<int64_t>(), dhoff.as<int64_t>(), nwin,
-                                                              PRW, d.pr_lane_row.as<int32_t>(), d.pr_heavy_row.as<int32_t>());
+                                                              PRW, L.lane_row.as<int32_t>(), L.heavy_row.as<int32_t>());
   CUDA_OK(cudaGetLastError());
-  d.pr_slab_len = build_sell<uint32_t>(c, d.crp.as<uint32_t>(), reinterpret_cast<const uint32_t*>(d.csrc.p),
-                                       d.pr_lane_row.as<int32_t>(), d.pr_nslices, PR_SENT, d.pr_slice_len,
-                                       d.pr_slice_off, d.pr_slab);
+  L.slab_len = build_sell<T>(c, rp, payload, L.lane_row.as<int32_t>(), L.nslices, sentinel, L.slice_len, L.slice_off, L.slab);
   CUDA_OK(cudaStreamSynchronize(s));
 }
+
+template void build_window_sell<uint32_t>(Ctx*, const uint32_t*, const uint32_t*, int64_t, uint32_t, SellLayout&);
+template void build_window_sell<uint2>(Ctx*, const uint32_t*, const uint2*, int64_t, uint2, SellLayout&);
 
 }  // namespace gx

@@ -3,18 +3,19 @@
 // The paper's primary kernel is vertex-centric neighbour enumeration with a
 // "main fixed-point loop repeatedly calling the primary kernel" (PAPER.md
 // P@15381, P@40883).  Here each iteration relaxes the out-edges of the active
-// slots with atomicMin (exact integer arithmetic, bit-exact with Dijkstra on
+// slots with atomic min (exact integer arithmetic, bit-exact with Dijkstra on
 // G_L, Theorem E1), then runs the §3 shared-memory pass over the subgraph
 // tiles, then the §2.4 confluence (P@28309) of replica groups.
 //
-// LB mapping (best exact kernel): frontier queues, one persistent grid;
-//   heavy slots (out-degree > HEAVY_DEG) are split into HCHUNK-edge work
-//   items fetched with one atomic per warp; light slots are taken 32 at a
-//   time per warp and their edges are distributed over the lanes by a warp
-//   prefix scan (every lane relaxes one edge per round: coalesced 8-byte
-//   {col, w} loads, no divergence from degree skew).  Newly improved slots
-//   are deduplicated with a 1-bit-per-slot bitmap (atomicOr) and appended with
-//   warp-aggregated atomics.
+// LB mapping (best exact kernel): the frontier is a bitmap.  Each warp
+// compacts the set bits of 32 bitmap words (1024 slots) into shared memory
+// and spreads the out-edges of 32 slots at a time over its lanes by a warp
+// prefix scan (coalesced 8-byte {col, w} loads, no divergence from degree
+// skew); slots with out-degree > HEAVY_DEG are relaxed from a static list of
+// 1024-edge chunks.  A relaxation is fire-and-forget: red.min on dist and
+// red.or on the next-frontier bitmap -- no return values, queues or counters,
+// so nothing serialises on atomic round trips.  dist and the bitmaps carry
+// L2 evict_last, the edge stream evict_first.
 // TPV mapping (the paper's thread-per-vertex, §2/§4 layouts): tpv.cu.
 #include <algorithm>
 #include <chrono>
@@ -24,58 +25,26 @@
 #include "kernels_common.cuh"
 #include "ktimer.h"
 #include "sssp_common.cuh"
+#include <cub/cub.cuh>
+#include <cstdlib>
 
 namespace gx {
 
 // ---------------------------------------------------------------- helpers
-// L2 residency: dist is the only vector gathered at
-// random, so its loads / atomics carry evict_last; the edge stream, queues
-// and row offsets carry evict_first.  Frontier dedupe uses 1-bit-per-slot
-// bitmaps (2 MB at 16M slots, always L2 resident), double-buffered by
-// iteration parity: iteration t sets bits of bm[(t+1)&1] and clears bm[t&1].
-struct SsspAux {
-  uint32_t* bm[2];             // "already in the next frontier" bitmaps
-  const uint32_t* heavy;       // bitmap: out-degree > HEAVY_DEG
-  int64_t nwords;
-};
-
-__device__ __forceinline__ void push_next(bool push, uint32_t v, const uint32_t* __restrict__ rp,
-                                          const uint32_t* __restrict__ heavybm, SsspCtr* nxt,
-                                          int32_t* __restrict__ lq_out, int32_t* __restrict__ hq_out,
-                                          uint32_t* __restrict__ hb_out) {
-  unsigned bal = __ballot_sync(FULL, push);
-  if (!bal) return;
-  const bool heavy = push && ((__ldg(heavybm + (v >> 5)) >> (v & 31)) & 1u);
-  unsigned lb = __ballot_sync(FULL, push && !heavy);
-  if (lb) {
-    unsigned leader = __ffs(lb) - 1, base = 0;
-    if (lane_id() == leader) base = atomicAdd(&nxt->lcount, (unsigned)__popc(lb));
-    base = __shfl_sync(FULL, base, leader);
-    if (push && !heavy) st_stream_i32(lq_out + base + __popc(lb & lanemask_lt()), (int32_t)v, l2_evict_first());
-  }
-  if (heavy) {
-    uint32_t vdeg = rp[v + 1] - rp[v];
-    unsigned long long add = (1ull << 32) | (unsigned long long)((vdeg + HCHUNK - 1) / HCHUNK);
-    unsigned long long old = atomicAdd(&nxt->hpack, add);
-    hq_out[old >> 32] = (int32_t)v;
-    hb_out[old >> 32] = (uint32_t)(old & 0xffffffffull);
-  }
+__device__ __forceinline__ bool bit_of(const uint32_t* __restrict__ bm, uint32_t v) {
+  return (__ldcg(bm + (v >> 5)) >> (v & 31)) & 1u;
 }
 
-// relax one edge given the (possibly stale, never smaller) current distance
-// `cur` of its head; returns true iff the head must join the next frontier
-__device__ __forceinline__ bool relax2(uint2 ed, uint32_t du, uint32_t cur, uint32_t* __restrict__ dist,
-                                       uint32_t* __restrict__ bm_next, uint64_t pl) {
+// relax one edge given the (possibly stale, never smaller within a sweep)
+// distance `cur` of its head
+__device__ __forceinline__ void relax_red(uint2 ed, uint32_t du, uint32_t cur, uint32_t* __restrict__ dist,
+                                          uint32_t* __restrict__ bm_next, uint64_t pl) {
   uint32_t nd = du + ed.y;
   if (nd < du) nd = INF - 1;  // saturate (never the fixed point)
   if (nd < cur) {
-    uint32_t old = atom_min_l2(dist + ed.x, nd, pl);
-    if (nd < old) {
-      uint32_t bit = 1u << (ed.x & 31);
-      if (!(atom_or_l2(bm_next + (ed.x >> 5), bit, pl) & bit)) return true;
-    }
+    red_min_l2(dist + ed.x, nd, pl);
+    red_or_l2(bm_next + (ed.x >> 5), 1u << (ed.x & 31), pl);
   }
-  return false;
 }
 
 __device__ __forceinline__ void clear_bitmap(uint32_t* bm, int64_t nwords) {
@@ -84,149 +53,146 @@ __device__ __forceinline__ void clear_bitmap(uint32_t* bm, int64_t nwords) {
 }
 
 // ---------------------------------------------------------------- LB sweep
-constexpr int SU = 4;  // edges in flight per lane per round
+constexpr int SU = 4;         // edges in flight per lane per round
+constexpr int SB_WARPS = 8;   // warps per CTA
 
 __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj,
-                                                 uint32_t* __restrict__ dist, SsspAux ax,
-                                                 SsspQueues qs, SsspState* __restrict__ st) {
+                                                 uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st) {
+  __shared__ int32_t s_v[SB_WARPS][1024];
   __shared__ unsigned long long sh[32];
   const unsigned t = st->iter;
   if (st->stop) return;
-  const bool odd = t & 1;
-  SsspCtr* cur = &st->ctr[t % 3];
-  SsspCtr* nxt = &st->ctr[(t + 1) % 3];
-  const int32_t* lq_in = odd ? qs.lq[1] : qs.lq[0];
-  int32_t* lq_out = odd ? qs.lq[0] : qs.lq[1];
-  const int32_t* hq_in = odd ? qs.hq[1] : qs.hq[0];
-  const uint32_t* hb_in = odd ? qs.hb[1] : qs.hb[0];
-  int32_t* hq_out = odd ? qs.hq[0] : qs.hq[1];
-  uint32_t* hb_out = odd ? qs.hb[0] : qs.hb[1];
-  const unsigned lcount = cur->lcount;
-  const unsigned long long hp = cur->hpack;
-  const unsigned hcount = (unsigned)(hp >> 32), hchunks = (unsigned)(hp & 0xffffffffull);
-  const unsigned lane = lane_id();
+  const uint32_t* __restrict__ bm_cur = ax.bm[t % 3];
+  uint32_t* bm_next = ax.bm[(t + 1) % 3];
+  clear_bitmap(ax.bm[(t + 2) % 3], ax.nwords);
+  const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
   const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
-  uint32_t* bm_next = odd ? ax.bm[0] : ax.bm[1];
-  clear_bitmap(odd ? ax.bm[1] : ax.bm[0], ax.nwords);
-  unsigned long long my_edges = 0;
+  const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  unsigned long long my_edges = 0, my_act = 0;
 
-  // heavy slots: HCHUNK-edge work items
-  while (true) {
-    unsigned c = 0;
-    if (lane == 0) c = atomicAdd(&cur->hcursor, 1u);
-    c = __shfl_sync(FULL, c, 0);
-    if (c >= hchunks) break;
-    int lo = 0, hi = (int)hcount - 1;
-    while (lo < hi) {
-      int mid = (lo + hi + 1) >> 1;
-      if (hb_in[mid] <= c) lo = mid;
-      else hi = mid - 1;
-    }
-    int32_t u = hq_in[lo];
-    uint32_t du = ld_l2_u32(dist + u, pl);
-    uint32_t a = rp[u] + (c - hb_in[lo]) * HCHUNK;
-    uint32_t b = min(a + (uint32_t)HCHUNK, rp[u + 1]);
+  // heavy slots: static 1024-edge chunks of rows with out-degree > HEAVY_DEG
+  for (int64_t c = gw; c < ax.nhc; c += nw) {
+    const int32_t u = ax.hc_row[c];
+    if (!bit_of(bm_cur, (uint32_t)u)) continue;       // warp-uniform
+    const uint32_t a = ax.hc_start[c];
+    const uint32_t b = min(a + HCHUNK, rp[u + 1]);
+    if (a == rp[u] && lane == 0) my_act++;
+    const uint32_t du = ld_l2_u32(dist + u, pl);
     for (uint32_t e0 = a; e0 < b; e0 += 32 * SU) {
       uint2 ed[SU];
-      bool act[SU], push[SU];
+      bool ok[SU];
 #pragma unroll
       for (int q = 0; q < SU; q++) {
         uint32_t e = e0 + q * 32 + lane;
-        act[q] = e < b;
-        ed[q] = act[q] ? ld_stream_u2(adj + e, pf) : make_uint2(0, 0);
+        ok[q] = e < b;
+        ed[q] = ok[q] ? ld_stream_u2(adj + e, pf) : make_uint2(0, 0);
       }
       uint32_t cv[SU];
 #pragma unroll
-      for (int q = 0; q < SU; q++) cv[q] = act[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
+      for (int q = 0; q < SU; q++) cv[q] = ok[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
 #pragma unroll
-      for (int q = 0; q < SU; q++) push[q] = act[q] && relax2(ed[q], du, cv[q], dist, bm_next, pl);
-#pragma unroll
-      for (int q = 0; q < SU; q++) push_next(push[q], ed[q].x, rp, ax.heavy, nxt, lq_out, hq_out, hb_out);
+      for (int q = 0; q < SU; q++)
+        if (ok[q]) relax_red(ed[q], du, cv[q], dist, bm_next, pl);
     }
     if (lane == 0) my_edges += b - a;
   }
 
-  // light slots: 32 per warp, edges spread over lanes by a prefix scan
-  while (true) {
-    unsigned base = 0;
-    if (lane == 0) base = atomicAdd(&cur->lcursor, 32u);
-    base = __shfl_sync(FULL, base, 0);
-    if (base >= lcount) break;
-    unsigned idx = base + lane;
-    uint32_t start = 0, deg = 0, du = 0;
-    if (idx < lcount) {
-      int32_t u = ld_stream_i32(lq_in + idx, pf);
-      start = ld_stream_u32(rp + u, pf);
-      deg = ld_stream_u32(rp + u + 1, pf) - start;
-      du = ld_l2_u32(dist + u, pl);
+  // light slots: compact the frontier bits of 32 words, 32 slots per round
+  int32_t* sv = s_v[wib];
+  for (int64_t wb = gw * 32; wb < ax.nwords; wb += nw * 32) {
+    const int64_t wi = wb + lane;
+    uint32_t word = wi < ax.nwords ? (__ldcg(bm_cur + wi) & ~__ldg(ax.heavy + wi)) : 0u;
+    const uint32_t cnt = __popc(word);
+    const uint32_t incl = warp_incl_scan_u32(cnt);
+    const uint32_t total = __shfl_sync(FULL, incl, 31);
+    if (total == 0) continue;
+    uint32_t k = incl - cnt;
+    while (word) {
+      const int b = __ffs(word) - 1;
+      sv[k++] = (int32_t)(wi * 32 + b);
+      word &= word - 1;
     }
-    uint32_t incl = warp_incl_scan_u32(deg);
-    uint32_t excl = incl - deg;
-    uint32_t total = __shfl_sync(FULL, incl, 31);
-    for (uint32_t k0 = 0; k0 < total; k0 += 32 * SU) {
-      uint2 ed[SU];
-      uint32_t od[SU];
-      bool act[SU], push[SU];
-#pragma unroll
-      for (int q = 0; q < SU; q++) {
-        uint32_t k = k0 + q * 32 + lane;
-        int j = 0;
-#pragma unroll
-        for (int s = 16; s; s >>= 1) {
-          uint32_t ex = __shfl_sync(FULL, excl, j + s);
-          if (ex <= k) j += s;
-        }
-        uint32_t os = __shfl_sync(FULL, start, j);
-        uint32_t oe = __shfl_sync(FULL, excl, j);
-        od[q] = __shfl_sync(FULL, du, j);
-        act[q] = k < total;
-        ed[q] = act[q] ? ld_stream_u2(adj + os + (k - oe), pf) : make_uint2(0, 0);
+    __syncwarp();
+    if (lane == 0) my_act += total;
+    for (uint32_t base = 0; base < total; base += 32) {
+      const uint32_t idx = base + lane;
+      uint32_t start = 0, deg = 0, du = 0;
+      if (idx < total) {
+        const int32_t u = sv[idx];
+        start = rp[u];
+        deg = rp[u + 1] - start;
+        du = ld_l2_u32(dist + u, pl);
       }
-      uint32_t cv[SU];
+      const uint32_t dincl = warp_incl_scan_u32(deg);
+      const uint32_t dexcl = dincl - deg;
+      const uint32_t dtot = __shfl_sync(FULL, dincl, 31);
+      for (uint32_t k0 = 0; k0 < dtot; k0 += 32 * SU) {
+        uint2 ed[SU];
+        uint32_t od[SU];
+        bool ok[SU];
 #pragma unroll
-      for (int q = 0; q < SU; q++) cv[q] = act[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
+        for (int q = 0; q < SU; q++) {
+          const uint32_t kk = k0 + q * 32 + lane;
+          int j = 0;
 #pragma unroll
-      for (int q = 0; q < SU; q++) push[q] = act[q] && relax2(ed[q], od[q], cv[q], dist, bm_next, pl);
+          for (int sft = 16; sft; sft >>= 1) {
+            uint32_t ex = __shfl_sync(FULL, dexcl, j + sft);
+            if (ex <= kk) j += sft;
+          }
+          const uint32_t os = __shfl_sync(FULL, start, j);
+          const uint32_t oe = __shfl_sync(FULL, dexcl, j);
+          od[q] = __shfl_sync(FULL, du, j);
+          ok[q] = kk < dtot;
+          ed[q] = ok[q] ? ld_stream_u2(adj + os + (kk - oe), pf) : make_uint2(0, 0);
+        }
+        uint32_t cv[SU];
 #pragma unroll
-      for (int q = 0; q < SU; q++) push_next(push[q], ed[q].x, rp, ax.heavy, nxt, lq_out, hq_out, hb_out);
+        for (int q = 0; q < SU; q++) cv[q] = ok[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
+#pragma unroll
+        for (int q = 0; q < SU; q++)
+          if (ok[q]) relax_red(ed[q], od[q], cv[q], dist, bm_next, pl);
+      }
+      if (lane == 0) my_edges += dtot;
     }
-    if (lane == 0) my_edges += total;
+    __syncwarp();
   }
-  unsigned long long tot = block_sum_u64(my_edges, sh);
-  if (threadIdx.x == 0 && tot) atomicAdd(&st->edges, tot);
+  unsigned long long e = block_sum_u64(my_edges, sh);
+  __syncthreads();
+  unsigned long long a2 = block_sum_u64(my_act, sh);
+  if (threadIdx.x == 0) {
+    if (e) atomicAdd(&st->edges, e);
+    if (a2) atomicAdd(&st->active[t % 3], (unsigned)a2);
+  }
 }
 
 // ---------------------------------------------------------------- §3 local pass
 // One CTA per subgraph tile: member distances staged in shared memory,
 // relaxed t times over the tile's local edges (P@32188-32416, reading R28),
-// improvements written back with atomicMin and pushed to the next frontier.
+// improvements written back with atomic min and added to the next frontier.
 __global__ void __launch_bounds__(256) k_sssp_local(const int32_t* __restrict__ tptr, const int32_t* __restrict__ tmem,
                                                     const int32_t* __restrict__ teptr, const uint2* __restrict__ tedges,
                                                     const int32_t* __restrict__ titers, int64_t ntiles,
-                                                    const uint32_t* __restrict__ rp, uint32_t* __restrict__ dist,
-                                                    SsspAux ax, SsspQueues qs, SsspState* __restrict__ st) {
+                                                    uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st) {
   __shared__ uint32_t sd[256];
   const unsigned t = st->iter;
   if (st->stop) return;
-  SsspCtr* nxt = &st->ctr[(t + 1) % 3];
-  int32_t* lq_out = (t & 1) ? qs.lq[0] : qs.lq[1];
-  int32_t* hq_out = (t & 1) ? qs.hq[0] : qs.hq[1];
-  uint32_t* hb_out = (t & 1) ? qs.hb[0] : qs.hb[1];
-  uint32_t* bm_next = (t & 1) ? ax.bm[0] : ax.bm[1];
+  uint32_t* bm_next = ax.bm[(t + 1) % 3];
+  const uint64_t pl = l2_evict_last();
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    int a = tptr[tile], nm = tptr[tile + 1] - a;
-    int ea = teptr[tile], ne = teptr[tile + 1] - ea;
-    for (int i = threadIdx.x; i < nm; i += blockDim.x) sd[i] = __ldcg(dist + tmem[a + i]);
+    const int a = tptr[tile], nm = tptr[tile + 1] - a;
+    const int ea = teptr[tile], ne = teptr[tile + 1] - ea;
+    for (int i = threadIdx.x; i < nm; i += blockDim.x) sd[i] = ld_l2_u32(dist + tmem[a + i], pl);
     __syncthreads();
-    int iters = titers[tile];
+    const int iters = titers[tile];
     for (int r = 0; r < iters; r++) {
       int ch = 0;
       for (int i = threadIdx.x; i < ne; i += blockDim.x) {
-        uint2 p = tedges[ea + i];
-        uint32_t src = p.x & 0xff, dst = (p.x >> 8) & 0xff, w = p.y;
-        uint32_t du = sd[src];
+        const uint2 p = tedges[ea + i];
+        const uint32_t src = p.x & 0xff, dst = (p.x >> 8) & 0xff;
+        const uint32_t du = sd[src];
         if (du != INF) {
-          uint32_t nd = du + w;
+          uint32_t nd = du + p.y;
           if (nd < du) nd = INF - 1;
           if (nd < sd[dst]) {
             atomicMin(&sd[dst], nd);
@@ -236,19 +202,13 @@ __global__ void __launch_bounds__(256) k_sssp_local(const int32_t* __restrict__ 
       }
       if (!__syncthreads_or(ch)) break;
     }
-    for (int i0 = 0; i0 < nm; i0 += blockDim.x) {
-      int i = i0 + threadIdx.x;
-      bool push = false;
-      uint32_t v = 0;
-      if (i < nm) {
-        v = (uint32_t)tmem[a + i];
-        uint32_t nd = sd[i];
-        if (nd < __ldcg(dist + v)) {
-          uint32_t old = atomicMin(dist + v, nd);
-          push = nd < old && !(atomicOr(bm_next + (v >> 5), 1u << (v & 31)) & (1u << (v & 31)));
-        }
+    for (int i = threadIdx.x; i < nm; i += blockDim.x) {
+      const uint32_t v = (uint32_t)tmem[a + i];
+      const uint32_t nd = sd[i];
+      if (nd < ld_l2_u32(dist + v, pl)) {
+        red_min_l2(dist + v, nd, pl);
+        red_or_l2(bm_next + (v >> 5), 1u << (v & 31), pl);
       }
-      push_next(push, v, rp, ax.heavy, nxt, lq_out, hq_out, hb_out);
     }
     __syncthreads();
   }
@@ -262,35 +222,30 @@ __global__ void __launch_bounds__(256) k_sssp_local(const int32_t* __restrict__ 
 // frontier.
 __global__ void __launch_bounds__(256) k_sssp_merge(const int32_t* __restrict__ gptr, const int32_t* __restrict__ gslots,
                                                     const int32_t* __restrict__ ginptr, const uint2* __restrict__ gin,
-                                                    int64_t ngroups, int merge_min, const uint32_t* __restrict__ rp,
-                                                    uint32_t* __restrict__ dist, SsspAux ax,
-                                                    SsspQueues qs, SsspState* __restrict__ st) {
+                                                    int64_t ngroups, int merge_min, uint32_t* __restrict__ dist,
+                                                    SsspAux ax, SsspState* __restrict__ st) {
   const unsigned t = st->iter;
   if (st->stop) return;
-  SsspCtr* nxt = &st->ctr[(t + 1) % 3];
-  int32_t* lq_out = (t & 1) ? qs.lq[0] : qs.lq[1];
-  int32_t* hq_out = (t & 1) ? qs.hq[0] : qs.hq[1];
-  uint32_t* hb_out = (t & 1) ? qs.hb[0] : qs.hb[1];
-  uint32_t* bm_next = (t & 1) ? ax.bm[0] : ax.bm[1];
+  uint32_t* bm_next = ax.bm[(t + 1) % 3];
   const unsigned lane = lane_id();
-  int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t gi = warp; gi < ngroups; gi += nw) {
-    int a = gptr[gi], b = gptr[gi + 1];
-    int32_t o = gslots[a];
+    const int a = gptr[gi], b = gptr[gi + 1];
+    const int32_t o = gslots[a];
     uint32_t best = INF;
     for (int e = ginptr[gi] + lane; e < ginptr[gi + 1]; e += 32) {
-      uint2 iv = gin[e];
-      uint32_t dp = dist[iv.x];
+      const uint2 iv = gin[e];
+      const uint32_t dp = __ldcg(dist + iv.x);
       if (dp != INF) best = min(best, dp + iv.y);
     }
     best = warp_min_u32(best);
-    uint32_t own = min(dist[o], best);
+    const uint32_t own = min(__ldcg(dist + o), best);
     unsigned long long sum = 0;
     unsigned cnt = 0;
     uint32_t mn = INF;
     for (int i = a + lane; i < b; i += 32) {
-      uint32_t val = (i == a) ? own : dist[gslots[i]];
+      const uint32_t val = (i == a) ? own : __ldcg(dist + gslots[i]);
       if (val != INF) {
         sum += val;
         cnt++;
@@ -300,59 +255,63 @@ __global__ void __launch_bounds__(256) k_sssp_merge(const int32_t* __restrict__ 
     sum = warp_sum_u64(sum);
     cnt = __reduce_add_sync(FULL, cnt);
     mn = warp_min_u32(mn);
-    uint32_t mval = merge_min ? mn : (cnt ? (uint32_t)(sum / cnt) : INF);
-    for (int i0 = a; i0 < b; i0 += 32) {
-      int i = i0 + lane;
-      bool push = false;
-      uint32_t s = 0;
-      if (i < b) {
-        s = (uint32_t)gslots[i];
-        uint32_t old = dist[s];
-        if (old != mval) {
-          dist[s] = mval;
-          push = mval < old && !(atomicOr(bm_next + (s >> 5), 1u << (s & 31)) & (1u << (s & 31)));
-          if (mval > old) atomicAdd(&st->raised, 1u);
-        }
+    const uint32_t mval = merge_min ? mn : (cnt ? (uint32_t)(sum / cnt) : INF);
+    for (int i = a + lane; i < b; i += 32) {
+      const uint32_t sl = (uint32_t)gslots[i];
+      const uint32_t old = __ldcg(dist + sl);
+      if (old != mval) {
+        dist[sl] = mval;
+        if (mval < old) atomicOr(bm_next + (sl >> 5), 1u << (sl & 31));
+        else atomicAdd(&st->raised, 1u);
       }
-      push_next(push, s, rp, ax.heavy, nxt, lq_out, hq_out, hb_out);
     }
   }
 }
 
+// end of iteration t: the frontier of t was empty => converged
 __global__ void k_sssp_advance(SsspState* __restrict__ st, int max_iters) {
   if (st->stop) return;
-  unsigned t = st->iter;
-  SsspCtr* n1 = &st->ctr[(t + 1) % 3];
-  SsspCtr* n2 = &st->ctr[(t + 2) % 3];
-  n2->lcount = 0;
-  n2->lcursor = 0;
-  n2->hpack = 0;
-  n2->hcursor = 0;
-  st->active += (unsigned long long)n1->lcount + (n1->hpack >> 32);
+  const unsigned t = st->iter;
+  const unsigned act = st->active[t % 3];
+  st->act_total += act;
+  st->active[(t + 2) % 3] = 0;
+  if (act == 0) {
+    st->stop = 1;
+    return;
+  }
   st->iter = t + 1;
-  bool empty = n1->lcount == 0 && (n1->hpack >> 32) == 0;
-  if (empty) st->stop = 1;           // converged
-  else if ((int)(t + 1) >= max_iters) st->stop = 2;
+  if ((int)(t + 1) >= max_iters) st->stop = 2;
 }
 
 __global__ void k_sssp_init(uint32_t* __restrict__ dist, const int32_t* __restrict__ slots, int nslots,
-                            const uint32_t* __restrict__ rp, SsspQueues qs, SsspState* __restrict__ st) {
+                            uint32_t* __restrict__ bm0) {
   // all copies of the source start at 0 (P@28609: copies begin equal)
   if (threadIdx.x != 0 || blockIdx.x != 0) return;
   for (int i = 0; i < nslots; i++) {
-    int32_t s = slots[i];
+    const int32_t s = slots[i];
     dist[s] = 0;
-    uint32_t deg = rp[s + 1] - rp[s];
-    if (deg > HEAVY_DEG) {
-      unsigned long long old = st->ctr[0].hpack;
-      st->ctr[0].hpack = old + ((1ull << 32) | ((deg + HCHUNK - 1) / HCHUNK));
-      qs.hq[0][old >> 32] = s;
-      qs.hb[0][old >> 32] = (uint32_t)(old & 0xffffffffull);
-    } else {
-      qs.lq[0][st->ctr[0].lcount++] = s;
+    bm0[s >> 5] |= 1u << (s & 31);
+  }
+}
+
+// static chunk list of heavy rows: chunk count per row, then fill
+__global__ void k_heavy_chunks_count(const uint32_t* __restrict__ rp, int64_t n, uint32_t* __restrict__ cnt) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t d = rp[v + 1] - rp[v];
+    cnt[v] = d > HEAVY_DEG ? (d + HCHUNK - 1) / HCHUNK : 0u;
+  }
+}
+__global__ void k_heavy_chunks_fill(const uint32_t* __restrict__ rp, int64_t n, const uint32_t* __restrict__ off,
+                                    int32_t* __restrict__ hrow, uint32_t* __restrict__ hstart) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t d = rp[v + 1] - rp[v];
+    if (d <= HEAVY_DEG) continue;
+    const uint32_t k = (d + HCHUNK - 1) / HCHUNK, o = off[v];
+    for (uint32_t i = 0; i < k; i++) {
+      hrow[o + i] = (int32_t)v;
+      hstart[o + i] = rp[v] + i * HCHUNK;
     }
   }
-  st->active = nslots;
 }
 
 // bitmap of slots whose out-degree exceeds HEAVY_DEG (push-time class test)
@@ -394,46 +353,66 @@ int64_t default_source(gx_graph* g) {
 }
 
 // ---------------------------------------------------------------- driver
-void run_sssp_tpv_iter(gx_graph* g, SsspQueues qs, SsspState* st, int& launches);  // tpv.cu (uses SsspAux via g)
-void ensure_tpv(gx_graph* g);                                                    // tpv.cu
+void run_sssp_tpv_iter(gx_graph* g, SsspAux ax, SsspState* st, uint32_t* dist, int& launches);  // tpv.cu
+void ensure_tpv(gx_graph* g);                                                                  // tpv.cu
+
+static void ensure_heavy_chunks(gx_graph* g) {
+  DevGraph& d = g->dg;
+  if (d.hc_row.p) return;
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  const int64_t ns = d.n_slots;
+  DBuf cnt, off, tmp;
+  cnt.alloc(c, sizeof(uint32_t) * (ns + 1));
+  off.alloc(c, sizeof(uint32_t) * (ns + 1));
+  CUDA_OK(cudaMemsetAsync(cnt.p, 0, sizeof(uint32_t) * (ns + 1), s));
+  k_heavy_chunks_count<<<grid_for(c, ns), 256, 0, s>>>(d.rp.as<uint32_t>(), ns, cnt.as<uint32_t>());
+  size_t tb = 0;
+  CUDA_OK(cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt.as<uint32_t>(), off.as<uint32_t>(), ns + 1, s));
+  tmp.alloc(c, tb);
+  CUDA_OK(cub::DeviceScan::ExclusiveSum(tmp.p, tb, cnt.as<uint32_t>(), off.as<uint32_t>(), ns + 1, s));
+  uint32_t nhc = 0;
+  CUDA_OK(cudaMemcpyAsync(&nhc, off.as<uint32_t>() + ns, 4, cudaMemcpyDeviceToHost, s));
+  CUDA_OK(cudaStreamSynchronize(s));
+  d.nhc = nhc;
+  d.hc_row.alloc(c, sizeof(int32_t) * std::max<uint32_t>(nhc, 1));
+  d.hc_start.alloc(c, sizeof(uint32_t) * std::max<uint32_t>(nhc, 1));
+  k_heavy_chunks_fill<<<grid_for(c, ns), 256, 0, s>>>(d.rp.as<uint32_t>(), ns, off.as<uint32_t>(), d.hc_row.as<int32_t>(),
+                                                      d.hc_start.as<uint32_t>());
+  d.heavy_bm.alloc(c, sizeof(uint32_t) * ((ns + 31) / 32));
+  k_heavy_bitmap<<<grid_for(c, ns), 256, 0, s>>>(d.rp.as<uint32_t>(), ns, d.heavy_bm.as<uint32_t>());
+  CUDA_OK(cudaGetLastError());
+  CUDA_OK(cudaStreamSynchronize(s));
+}
 
 void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   Ctx* c = g->ctx;
   cudaStream_t s = c->stream;
   DevGraph& d = g->dg;
   RunState& r = g->rs;
-  int64_t src = o.source < 0 ? default_source(g) : o.source;
+  const int64_t src = o.source < 0 ? default_source(g) : o.source;
   GX_CHECK_ARG(g->n > 0, "empty graph");
   GX_CHECK_ARG(src >= 0 && src < g->n, "source out of range");
   if ((double)(g->n - 1) * (double)d.max_w >= 4294967295.0)
     GX_THROW(GX_E_UNSUPPORTED, "(n-1)*max(w) >= 2^32-1 would overflow uint32 distances");
   int mapping = o.mapping;
-  if (mapping == GX_MAP_AUTO) mapping = (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
+  if (mapping == GX_MAP_AUTO)
+    mapping = (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
   if (mapping == GX_MAP_TPV) ensure_tpv(g);
-  int64_t ns = d.n_slots;
-  r.dist.alloc(c, sizeof(uint32_t) * ns);
+  ensure_heavy_chunks(g);
+  const int64_t ns = d.n_slots;
   const int64_t nwords = (ns + 31) / 32;
-  r.mark.alloc(c, sizeof(uint32_t) * 3 * nwords);   // bm[0], bm[1], heavy
-  for (int i = 0; i < 2; i++) {
-    r.q[i].alloc(c, sizeof(int32_t) * ns);
-    r.hq[i].alloc(c, sizeof(int32_t) * ns);
-    r.hbase[i].alloc(c, sizeof(uint32_t) * ns);
-  }
+  r.dist.alloc(c, sizeof(uint32_t) * ns);
+  r.mark.alloc(c, sizeof(uint32_t) * 3 * nwords);   // frontier bitmaps bm[0..2]
   r.st.alloc(c, sizeof(SsspState));
-  SsspQueues qs;
-  for (int i = 0; i < 2; i++) {
-    qs.lq[i] = r.q[i].as<int32_t>();
-    qs.hq[i] = r.hq[i].as<int32_t>();
-    qs.hb[i] = r.hbase[i].as<uint32_t>();
-  }
   SsspState* st = r.st.as<SsspState>();
   SsspAux ax;
-  ax.bm[0] = r.mark.as<uint32_t>();
-  ax.bm[1] = r.mark.as<uint32_t>() + nwords;
-  ax.heavy = r.mark.as<uint32_t>() + 2 * nwords;
+  for (int i = 0; i < 3; i++) ax.bm[i] = r.mark.as<uint32_t>() + i * nwords;
+  ax.heavy = d.heavy_bm.as<uint32_t>();
   ax.nwords = nwords;
-  k_heavy_bitmap<<<grid_for(c, ns), 256, 0, s>>>(d.rp.as<uint32_t>(), ns, r.mark.as<uint32_t>() + 2 * nwords);
-  CUDA_OK(cudaGetLastError());
+  ax.hc_row = d.hc_row.as<int32_t>();
+  ax.hc_start = d.hc_start.as<uint32_t>();
+  ax.nhc = d.nhc;
   // source copies: owner slot + replica slots
   std::vector<int32_t> srcs;
   if (d.identity) {
@@ -453,48 +432,46 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   CUDA_OK(cudaEventCreate(&e1));
   CUDA_OK(cudaEventRecord(e0, s));
   CUDA_OK(cudaMemsetAsync(r.dist.p, 0xFF, sizeof(uint32_t) * ns, s));
-  CUDA_OK(cudaMemsetAsync(r.mark.p, 0, sizeof(uint32_t) * 2 * nwords, s));
+  CUDA_OK(cudaMemsetAsync(r.mark.p, 0, sizeof(uint32_t) * 3 * nwords, s));
   CUDA_OK(cudaMemsetAsync(r.st.p, 0, sizeof(SsspState), s));
-  k_sssp_init<<<1, 32, 0, s>>>(r.dist.as<uint32_t>(), dsrc.as<int32_t>(), (int)srcs.size(), d.rp.as<uint32_t>(),
-                               qs, st);
+  k_sssp_init<<<1, 32, 0, s>>>(r.dist.as<uint32_t>(), dsrc.as<int32_t>(), (int)srcs.size(), ax.bm[0]);
   CUDA_OK(cudaGetLastError());
   int launches = 4;
 
   int occ = 0;
   CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sssp_lb, 256, 0));
-  int grid_lb = std::max(1, occ) * c->num_sms;
-  int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 8));
-  int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 7) / 8, (int64_t)c->num_sms * 8));
-  bool merge_min = g->knobs.merge_op == GX_MERGE_MIN;
+  const int grid_lb = std::max(1, occ) * c->num_sms;
+  const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 8));
+  const int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 7) / 8, (int64_t)c->num_sms * 8));
+  const bool merge_min = g->knobs.merge_op == GX_MERGE_MIN;
 
   KTimer kt(o.profile != 0, s);
   auto one_iter = [&](int& nl) {
     kt.begin();
     if (mapping == GX_MAP_TPV) {
-      run_sssp_tpv_iter(g, qs, st, nl);
+      run_sssp_tpv_iter(g, ax, st, r.dist.as<uint32_t>(), nl);
     } else {
-      k_sssp_lb<<<grid_lb, 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), r.dist.as<uint32_t>(),
-                                        ax, qs, st);
+      k_sssp_lb<<<grid_lb, 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), r.dist.as<uint32_t>(), ax, st);
       nl++;
     }
     kt.end();
     if (d.n_tiles && g->knobs.smem) {
       k_sssp_local<<<grid_local, 256, 0, s>>>(d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(), d.t_eptr.as<int32_t>(),
                                               d.t_edges.as<uint2>(), d.t_iters.as<int32_t>(), d.n_tiles,
-                                              d.rp.as<uint32_t>(), r.dist.as<uint32_t>(), ax, qs, st);
+                                              r.dist.as<uint32_t>(), ax, st);
       nl++;
     }
     if (d.n_groups) {
       k_sssp_merge<<<grid_merge, 256, 0, s>>>(d.gptr.as<int32_t>(), d.gslots.as<int32_t>(), d.g_in_ptr.as<int32_t>(),
-                                              d.g_in.as<uint2>(), d.n_groups, merge_min ? 1 : 0, d.rp.as<uint32_t>(),
-                                              r.dist.as<uint32_t>(), ax, qs, st);
+                                              d.g_in.as<uint2>(), d.n_groups, merge_min ? 1 : 0, r.dist.as<uint32_t>(),
+                                              ax, st);
       nl++;
     }
     k_sssp_advance<<<1, 1, 0, s>>>(st, o.max_iters);
     nl++;
   };
 
-  int batch = std::max(1, o.check_every);
+  const int batch = std::max(1, o.check_every);
   cudaGraphExec_t gexec = nullptr;
   int per_batch_launches = 0;
   if (o.use_graphs && !o.profile) {
@@ -506,7 +483,6 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     CUDA_OK(cudaGraphDestroy(graph));
   }
   SsspState hst;
-  int done_iters = 0;
   while (true) {
     if (gexec) {
       CUDA_OK(cudaGraphLaunch(gexec, s));
@@ -515,7 +491,6 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
       for (int i = 0; i < batch; i++) one_iter(launches);
     }
     CUDA_OK(cudaGetLastError());
-    done_iters += batch;
     CUDA_OK(cudaMemcpyAsync(&hst, st, sizeof(SsspState), cudaMemcpyDeviceToHost, s));
     CUDA_OK(cudaStreamSynchronize(s));
     if (hst.stop) break;
@@ -527,14 +502,15 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   if (gexec) cudaGraphExecDestroy(gexec);
   cudaEventDestroy(e0);
   cudaEventDestroy(e1);
-  info.iterations = (int32_t)hst.iter;
+  // iterations that processed a non-empty frontier
+  info.iterations = (int32_t)(hst.stop == 1 ? hst.iter : hst.iter);
   info.converged = hst.stop == 1;
   info.loop_ms = ms;
   info.edges_scanned = (int64_t)hst.edges;
-  info.vertices_active = (int64_t)hst.active;
-  // bytes model: 12 B per scanned edge ({col,w} 8 + dist 4) +
-  // 14 B per processed slot (row_ptr 8 + dist 4 + queue 2*... ~2)
-  info.bytes_model = 12 * (int64_t)hst.edges + 14 * (int64_t)hst.active;
+  info.vertices_active = (int64_t)hst.act_total;
+  // bytes model: 12 B per relaxed edge ({col,w} 8 + dist gather 4)
+  // + 12 B per frontier slot (row_ptr 8 + dist 4)
+  info.bytes_model = 12 * (int64_t)hst.edges + 12 * (int64_t)hst.act_total;
   info.kernel_launches = launches;
   info.sweep_launches = kt.launches();
   info.sweep_ms = kt.total_ms();

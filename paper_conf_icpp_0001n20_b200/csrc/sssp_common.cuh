@@ -1,37 +1,31 @@
-// sssp_common.cuh -- frontier state shared by the SSSP / BC sweep kernels.
+// sssp_common.cuh -- frontier state shared by the SSSP sweep kernels.
 #pragma once
 #include <cstdint>
 
 namespace gx {
 
-constexpr uint32_t HEAVY_DEG = 256;  // out-degree above which a slot is split into work items
-constexpr uint32_t HCHUNK = 1024;    // edges per heavy work item (32 per lane)
+constexpr uint32_t HEAVY_DEG = 256;  // out-degree above which a slot is split into static chunks
+constexpr uint32_t HCHUNK = 1024;    // edges per heavy chunk
 
-// Per-iteration frontier counters, triple-buffered by iteration (t % 3): the
-// sweep of iteration t reads ctr[t%3], appends to ctr[(t+1)%3], and the
-// advance kernel clears ctr[(t+2)%3], so no host round trip is needed.
-struct SsspCtr {
-  unsigned int lcount;        // light queue length
-  unsigned int lcursor;       // light work cursor (entries handed out)
-  unsigned long long hpack;   // heavy queue: (count << 32) | total chunks
-  unsigned int hcursor;       // heavy chunk cursor
-  unsigned int pad;
-};
-
+// Device-side loop state.  The frontier is a 1-bit-per-slot bitmap,
+// triple-buffered by iteration (bm[t%3] current, bm[(t+1)%3] next,
+// bm[(t+2)%3] being cleared), so one iteration needs no host round trip.
 struct SsspState {
-  unsigned int iter;          // current iteration t
-  unsigned int stop;          // 0 running, 1 converged (empty frontier), 2 max_iters
-  SsspCtr ctr[3];
-  unsigned long long edges;   // edges relaxed, all iterations
-  unsigned long long active;  // frontier entries, all iterations
-  unsigned int raised;        // merges that raised a copy (diagnostic)
-  unsigned int pad;
+  unsigned int iter;            // current iteration t
+  unsigned int stop;            // 0 running, 1 converged (empty frontier), 2 max_iters
+  unsigned int active[3];       // slots in the frontier of iteration t (counted by its sweep)
+  unsigned int raised;          // merges that raised a copy (diagnostic)
+  unsigned long long edges;     // edges relaxed, all iterations
+  unsigned long long act_total; // frontier entries, all iterations
 };
 
-struct SsspQueues {
-  int32_t* lq[2];             // light frontier (slot ids), by iteration parity
-  int32_t* hq[2];             // heavy frontier slots
-  uint32_t* hb[2];            // heavy frontier: first chunk index of each entry
+struct SsspAux {
+  uint32_t* bm[3];              // frontier bitmaps
+  const uint32_t* heavy;        // bitmap: out-degree > HEAVY_DEG
+  int64_t nwords;
+  const int32_t* hc_row;        // static heavy chunk list: row
+  const uint32_t* hc_start;     //                          first edge
+  int64_t nhc;
 };
 
 }  // namespace gx
