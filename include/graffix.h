@@ -189,6 +189,12 @@ gx_status gx_graph_upload_csr(gx_ctx* ctx, gx_graph** out, int64_t n, int64_t m,
                               const int64_t* row_ptr, const int32_t* col, const uint32_t* w,
                               uint32_t flags);
 void gx_graph_destroy(gx_graph* g);
+
+/* Host-only graph: canonicalised as above, no device memory.  gx_transform
+ * and the gx_export_* calls work on it (the transforms are host code);
+ * gx_run / gx_download return GX_E_STATE.  Used by the CPU test suite. */
+gx_status gx_graph_create_host(gx_graph** out, int64_t n, int64_t m, const int64_t* row_ptr,
+                               const int32_t* col, const uint32_t* w, uint32_t flags);
 gx_status gx_graph_info(gx_graph* g, int64_t* n, int64_t* m);
 
 /* Paper defaults, all techniques OFF (= exact mode). */

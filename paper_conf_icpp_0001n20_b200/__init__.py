@@ -156,6 +156,18 @@ class Graph:
         _check(lib().gx_graph_upload_csr(ctx._h, C.byref(h), n, m, _ptr(row_ptr), _ptr(col), _ptr(w), flags))
         return cls(ctx, h)
 
+    @classmethod
+    def host_only(cls, row_ptr, col, w=None, validate: bool = False):
+        """Host-only graph (no device): canonicalise + transform + export.
+        Runs on a machine without a GPU; run()/download() raise GX_E_STATE."""
+        row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+        col = np.ascontiguousarray(col, dtype=np.int32)
+        w = None if w is None else np.ascontiguousarray(w, dtype=np.uint32)
+        h = C.c_void_p()
+        _check(lib().gx_graph_create_host(C.byref(h), int(row_ptr.shape[0]) - 1, int(col.shape[0]), _ptr(row_ptr),
+                                          _ptr(col), _ptr(w), GX_VALIDATE if validate else 0))
+        return cls(None, h)
+
     def transform(self, knobs: Knobs | None = None) -> dict:
         info = GxTransformInfo()
         k = knobs.to_c() if knobs is not None else None

@@ -31,7 +31,7 @@ EXPORTED = [
     "gx_abi_version", "gx_last_error", "gx_ctx_create", "gx_get_nccl_unique_id", "gx_ctx_create_dist",
     "gx_set_allocator", "gx_ctx_destroy", "gx_ctx_stream", "gx_graph_upload_csr", "gx_graph_destroy",
     "gx_graph_info", "gx_knobs_default", "gx_transform", "gx_export_sizes", "gx_export_transformed",
-    "gx_run", "gx_run_ex", "gx_run_opts_default", "gx_download", "gx_sync",
+    "gx_run", "gx_run_ex", "gx_run_opts_default", "gx_download", "gx_sync", "gx_graph_create_host",
 ]
 
 
@@ -117,6 +117,7 @@ def lib():
         "gx_run_opts_default": ([C.POINTER(GxRunOpts)], C.c_int),
         "gx_download": ([P, i32, P, i64, u32], C.c_int),
         "gx_sync": ([P], C.c_int),
+        "gx_graph_create_host": ([C.POINTER(P), i64, i64, P, P, P, u32], C.c_int),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)

@@ -234,8 +234,34 @@ gx_status gx_graph_upload_csr(gx_ctx* ctx, gx_graph** out, int64_t n, int64_t m,
 
 void gx_graph_destroy(gx_graph* g) {
   if (!g) return;
-  cudaSetDevice(g->ctx->device);
+  if (g->ctx) cudaSetDevice(g->ctx->device);
   delete g;  // DBuf destructors release device memory on the ctx stream
+}
+
+gx_status gx_graph_create_host(gx_graph** out, int64_t n, int64_t m, const int64_t* row_ptr, const int32_t* col,
+                               const uint32_t* w, uint32_t flags) {
+  GX_API_BEGIN
+  GX_CHECK_ARG(out, "out is NULL");
+  *out = nullptr;
+  GX_CHECK_ARG(n >= 0 && m >= 0 && row_ptr, "bad n/m/row_ptr");
+  GX_CHECK_ARG(m == 0 || col, "col is NULL");
+  GX_CHECK_ARG(!(flags & GX_PTRS_DEVICE), "host-only graphs take host pointers");
+  GX_CHECK_ARG(row_ptr[0] == 0 && row_ptr[n] == m, "row_ptr[0] must be 0 and row_ptr[n] == m");
+  for (int64_t u = 0; u < n; u++)
+    if (row_ptr[u + 1] < row_ptr[u]) GX_THROW(GX_E_INVALID, "row_ptr not monotone");
+  if (flags & GX_VALIDATE)
+    for (int64_t e = 0; e < m; e++) {
+      if (col[e] < 0 || col[e] >= n) GX_THROW(GX_E_INVALID, "col out of range");
+      if (w && w[e] == 0) GX_THROW(GX_E_INVALID, "weight 0");
+    }
+  gx_graph* g = new gx_graph();
+  gx_knobs_default(&g->knobs);
+  canonicalize_host(n, row_ptr, col, w, g->host);
+  g->host_valid = true;
+  g->n = n;
+  g->m = g->host.m;
+  *out = g;
+  GX_API_END
 }
 
 gx_status gx_graph_info(gx_graph* g, int64_t* n, int64_t* m) {
@@ -300,14 +326,14 @@ gx_status gx_transform(gx_graph* g, const gx_knobs* knobs, gx_transform_info* in
   gx_knobs_default(&k);
   if (knobs) k = *knobs;
   check_knobs(k);
-  CUDA_OK(cudaSetDevice(g->ctx->device));
+  if (g->ctx) CUDA_OK(cudaSetDevice(g->ctx->device));
   auto t0 = std::chrono::steady_clock::now();
   bool exact = !k.coalesce && !k.smem && !k.degree_norm;
   if (exact) {
     g->sg = SlotGraph();
     g->transformed = false;
     g->knobs = k;
-    build_device_exact(g);
+    if (g->ctx) build_device_exact(g);
     g->sg.info.n_slots = g->n;
     g->sg.info.m_slots = g->m;
   } else {
@@ -317,7 +343,7 @@ gx_status gx_transform(gx_graph* g, const gx_knobs* knobs, gx_transform_info* in
     g->sg = std::move(sg);
     g->transformed = true;
     g->knobs = k;
-    build_device_slots(g);
+    if (g->ctx) build_device_slots(g);
   }
   g->rs = RunState();
   auto t1 = std::chrono::steady_clock::now();
@@ -402,6 +428,7 @@ gx_status gx_run_ex(gx_graph* g, const gx_run_opts* opts, gx_run_info* info) {
   GX_API_BEGIN
   GX_CHECK_ARG(g && opts, "NULL argument");
   GX_CHECK_ARG(opts->struct_size == sizeof(gx_run_opts), "gx_run_opts.struct_size mismatch");
+  if (!g->ctx) GX_THROW(GX_E_STATE, "host-only graph: no device to run on");
   CUDA_OK(cudaSetDevice(g->ctx->device));
   gx_run_opts o = *opts;
   if (o.max_iters <= 0) o.max_iters = 1000000;
@@ -438,6 +465,7 @@ gx_status gx_run(gx_graph* g, gx_algo algo, int64_t source, int32_t max_iters, d
 gx_status gx_download(gx_graph* g, int32_t kind, void* out, int64_t count, uint32_t flags) {
   GX_API_BEGIN
   GX_CHECK_ARG(g && out, "NULL argument");
+  if (!g->ctx) GX_THROW(GX_E_STATE, "host-only graph: nothing has run");
   CUDA_OK(cudaSetDevice(g->ctx->device));
   gx::download(g, kind, out, count, flags);
   GX_API_END

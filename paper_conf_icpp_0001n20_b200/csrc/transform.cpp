@@ -1,0 +1,677 @@
+// transform.cpp -- the three Graffix transforms on the host (SURVEY.md §8(a)
+// A1-A3, A5-A6, A8-A9), producing the slot graph the sweeps run on.
+//
+//   §2 coalescing (Alg 2, PAPER.md P@16373-18419): BFS-forest levels, cursor
+//      renumbering into an isomorph with k-aligned levels (holes), bounded
+//      replication of well-connected (vertex, chunk) pairs into the holes.
+//   §3 memory latency (P@29857-32416): clustering coefficient on the
+//      undirected view, CC-raising sibling edges under a global budget, and
+//      disjoint {c} + N(c) subgraphs processed t ~ 2*diam times in shared memory.
+//   §4 divergence (P@33145-35029): degree buckets, warps in bucket order,
+//      2-hop padding towards ceil(0.85 * warp max).
+// Readings R1..R44 decide every tie;
+// thresholds are compared in integer ppm.  The oracle (oracle/transform.py)
+// implements the same readings independently; tests compare the exports.
+#include <omp.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <numeric>
+#include <unordered_map>
+
+#include "gx_internal.h"
+
+namespace gx {
+namespace {
+
+int64_t ppm(double x) { return (int64_t)std::floor(x * 1e6 + 0.5); }
+
+struct Edge {
+  int32_t dst;
+  uint32_t w;
+  uint8_t added;
+};
+
+// Working slot graph: one row vector per slot.
+struct Work {
+  int64_t n = 0, n_slots = 0;
+  std::vector<std::vector<Edge>> rows;
+  std::vector<int32_t> slot_to_orig;
+  std::vector<uint8_t> kind;
+  std::vector<int32_t> owner;  // orig -> owner slot
+  int64_t n_holes = 0, n_repl = 0, added_coal = 0;
+};
+
+void identity(const HostCSR& g, Work& W) {
+  W.n = g.n;
+  W.n_slots = g.n;
+  W.rows.assign(g.n, {});
+  W.slot_to_orig.resize(g.n);
+  W.kind.assign(g.n, OWNER);
+  W.owner.resize(g.n);
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int64_t u = 0; u < g.n; u++) {
+    W.slot_to_orig[u] = (int32_t)u;
+    W.owner[u] = (int32_t)u;
+    auto& r = W.rows[u];
+    r.reserve(g.rp[u + 1] - g.rp[u]);
+    for (int64_t e = g.rp[u]; e < g.rp[u + 1]; e++) r.push_back({g.col[e], g.w[e], ADD_NONE});
+  }
+}
+
+// ---------------------------------------------------------------- §2
+// Alg 2 l.2-6 with R3-R5: sources in (out-degree desc, id asc) order, a source
+// starts a reachability BFS if not yet visited; level = multi-source BFS
+// distance from the source set.
+void bfs_forest(const HostCSR& g, std::vector<int32_t>& sources, std::vector<int32_t>& level) {
+  const int64_t n = g.n;
+  std::vector<int32_t> order(n);
+  std::iota(order.begin(), order.end(), 0);
+  std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
+    return (g.rp[a + 1] - g.rp[a]) > (g.rp[b + 1] - g.rp[b]);
+  });
+  std::vector<uint8_t> vis(n, 0);
+  std::vector<int32_t> stack;
+  sources.clear();
+  for (int32_t s : order) {
+    if (vis[s]) continue;
+    sources.push_back(s);
+    vis[s] = 1;
+    stack.push_back(s);
+    while (!stack.empty()) {
+      int32_t u = stack.back();
+      stack.pop_back();
+      for (int64_t e = g.rp[u]; e < g.rp[u + 1]; e++) {
+        int32_t v = g.col[e];
+        if (!vis[v]) {
+          vis[v] = 1;
+          stack.push_back(v);
+        }
+      }
+    }
+  }
+  level.assign(n, -1);
+  std::vector<int32_t> fr(sources), nx;
+  for (int32_t s : sources) level[s] = 0;
+  int32_t lv = 0;
+  while (!fr.empty()) {
+    nx.clear();
+    for (int32_t u : fr)
+      for (int64_t e = g.rp[u]; e < g.rp[u + 1]; e++) {
+        int32_t v = g.col[e];
+        if (level[v] < 0) {
+          level[v] = lv + 1;
+          nx.push_back(v);
+        }
+      }
+    fr.swap(nx);
+    lv++;
+  }
+}
+
+// RenumberVertex (Alg 2 l.10-20), cursor reading R6-R8, pad R9.
+void renumber(const HostCSR& g, int k, std::vector<int32_t>& nw, int64_t& n_slots,
+              std::vector<std::pair<int64_t, int64_t>>& ranges) {
+  const int64_t n = g.n;
+  std::vector<int32_t> sources, level;
+  bfs_forest(g, sources, level);
+  nw.assign(n, -1);
+  for (size_t i = 0; i < sources.size(); i++) nw[sources[i]] = (int32_t)i;
+  int64_t gid = (int64_t)sources.size();
+  ranges.clear();
+  ranges.push_back({0, gid});
+  std::vector<int32_t> cur(sources), nxt;
+  std::vector<int64_t> cursor;
+  int32_t i = 0;
+  while (true) {
+    const int64_t start = (gid + k - 1) / k * k;
+    std::vector<int32_t> parents(cur);
+    std::sort(parents.begin(), parents.end(), [&](int32_t a, int32_t b) { return nw[a] < nw[b]; });
+    cursor.assign(parents.size(), 0);
+    for (size_t p = 0; p < parents.size(); p++) cursor[p] = g.rp[parents[p]];
+    nxt.clear();
+    int64_t gid2 = start;
+    // rounds: each parent numbers its next unnumbered level-(i+1) neighbour;
+    // parents that exhausted their rows drop out of later rounds
+    std::vector<size_t> live(parents.size());
+    std::iota(live.begin(), live.end(), 0);
+    while (true) {
+      bool assigned = false;
+      size_t keep = 0;
+      for (size_t li = 0; li < live.size(); li++) {
+        const size_t p = live[li];
+        const int32_t par = parents[p];
+        int64_t c = cursor[p];
+        const int64_t end = g.rp[par + 1];
+        while (c < end && !(level[g.col[c]] == i + 1 && nw[g.col[c]] == -1)) c++;
+        if (c < end) {
+          nw[g.col[c]] = (int32_t)gid2++;
+          nxt.push_back(g.col[c]);
+          c++;
+          assigned = true;
+        }
+        cursor[p] = c;
+        if (c < end) live[keep++] = p;
+      }
+      live.resize(keep);
+      if (!assigned) break;
+    }
+    if (nxt.empty()) break;
+    ranges.push_back({start, gid2});
+    gid = gid2;
+    cur.swap(nxt);
+    i++;
+  }
+  n_slots = n > 0 ? (gid + k - 1) / k * k : 0;
+}
+
+// Renumber + ReplicateVertex (Alg 2 l.21-35), readings R10-R18.
+void coalesce(const HostCSR& g, int k, int64_t theta_ppm, Work& W) {
+  const int64_t n = g.n;
+  std::vector<int32_t> nw;
+  std::vector<std::pair<int64_t, int64_t>> ranges;
+  int64_t n_slots = 0;
+  renumber(g, k, nw, n_slots, ranges);
+  W.n = n;
+  W.n_slots = n_slots;
+  W.slot_to_orig.assign(n_slots, -1);
+  W.kind.assign(n_slots, HOLE);
+  W.owner = nw;
+  W.rows.assign(n_slots, {});
+  for (int64_t u = 0; u < n; u++) {
+    W.slot_to_orig[nw[u]] = (int32_t)u;
+    W.kind[nw[u]] = OWNER;
+  }
+  // renumbered original adjacency (pre-move), CSR order
+  std::vector<std::vector<Edge>> radj(n_slots);
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int64_t u = 0; u < n; u++) {
+    auto& r = radj[nw[u]];
+    r.reserve(g.rp[u + 1] - g.rp[u]);
+    for (int64_t e = g.rp[u]; e < g.rp[u + 1]; e++) r.push_back({nw[g.col[e]], g.w[e], ADD_NONE});
+  }
+  std::vector<int32_t> nonhole((n_slots + k - 1) / k, 0);
+  for (int64_t s = 0; s < n_slots; s++)
+    if (W.kind[s] != HOLE) nonhole[s / k]++;
+  // level of each chunk (levels are chunk-aligned from level 1 on)
+  struct Asg {
+    int32_t s;
+    int64_t C;
+    int64_t hole;
+  };
+  std::vector<Asg> asg;
+  // chunk -> level index, for chunks of levels >= 1 whose previous level has holes
+  const int64_t nchunks = (int64_t)nonhole.size();
+  std::vector<int32_t> chunk_lv(nchunks, -1);
+  for (size_t li = 1; li < ranges.size(); li++) {
+    const int64_t holes = ranges[li].first - ranges[li - 1].second;
+    if (holes <= 0) continue;
+    for (int64_t C = ranges[li].first / k; C <= (ranges[li].second - 1) / k; C++) chunk_lv[C] = (int32_t)li;
+  }
+  // count (slot, chunk) pairs over edges into those chunks
+  std::vector<std::pair<int64_t, int32_t>> pairs;  // (C, s)
+  for (int64_t s = 0; s < n_slots; s++)
+    for (const Edge& e : radj[s]) {
+      const int64_t C = e.dst / k;
+      if (chunk_lv[C] >= 0) pairs.push_back({C, (int32_t)s});
+    }
+  std::sort(pairs.begin(), pairs.end());
+  // candidates per level: (-count, s, C)
+  std::vector<std::vector<std::tuple<int64_t, int32_t, int64_t>>> cands(ranges.size());
+  for (size_t a = 0; a < pairs.size();) {
+    size_t b = a;
+    while (b < pairs.size() && pairs[b] == pairs[a]) b++;
+    const int64_t cnt = (int64_t)(b - a);
+    const int64_t C = pairs[a].first;
+    if (cnt * 1000000 >= theta_ppm * (int64_t)nonhole[C]) cands[chunk_lv[C]].push_back({-cnt, pairs[a].second, C});
+    a = b;
+  }
+  for (size_t li = 1; li < ranges.size(); li++) {
+    const int64_t h0 = ranges[li - 1].second, h1 = ranges[li].first;
+    if (h1 <= h0) continue;
+    auto& cl = cands[li];
+    std::sort(cl.begin(), cl.end());
+    int64_t h = h0;
+    for (auto& c : cl) {
+      if (h >= h1) break;
+      asg.push_back({std::get<1>(c), std::get<2>(c), h++});
+    }
+  }
+  // owner rows start as the renumbered rows
+  for (int64_t s = 0; s < n_slots; s++) W.rows[s] = radj[s];
+  int64_t added = 0;
+  for (const Asg& a : asg) {
+    const auto& orow = radj[a.s];
+    std::vector<int32_t> nplus;
+    nplus.reserve(orow.size());
+    for (const Edge& e : orow) nplus.push_back(e.dst);
+    std::sort(nplus.begin(), nplus.end());
+    std::vector<Edge> moved;
+    for (const Edge& e : orow)
+      if (e.dst / k == a.C) moved.push_back(e);
+    auto& own = W.rows[a.s];
+    own.erase(std::remove_if(own.begin(), own.end(), [&](const Edge& e) { return e.dst / k == a.C; }), own.end());
+    // 2-hop edges into chunk C with the minimum path weight (R16, R17)
+    std::unordered_map<int32_t, uint32_t> best;
+    for (const Edge& ev : orow)
+      for (const Edge& eq : radj[ev.dst]) {
+        const int32_t q = eq.dst;
+        if (q / k != a.C || q == a.s || W.kind[q] == HOLE) continue;
+        if (std::binary_search(nplus.begin(), nplus.end(), q)) continue;
+        const uint32_t w = ev.w + eq.w;
+        auto it = best.find(q);
+        if (it == best.end() || w < it->second) best[q] = w;
+      }
+    std::vector<Edge> row = moved;
+    for (auto& kv : best) row.push_back({kv.first, kv.second, ADD_COALESCE});
+    W.rows[a.hole] = std::move(row);
+    W.kind[a.hole] = REPLICA;
+    W.slot_to_orig[a.hole] = W.slot_to_orig[a.s];
+    added += (int64_t)best.size();
+  }
+  int64_t holes_left = 0;
+  for (int64_t s = 0; s < n_slots; s++) holes_left += W.kind[s] == HOLE;
+  W.n_repl = (int64_t)asg.size();
+  W.n_holes = holes_left + W.n_repl;
+  W.added_coal = added;
+}
+
+// ---------------------------------------------------------------- §3
+// Mutable logical graph (original ids) with its undirected view U.
+struct Logical {
+  int64_t n;
+  std::vector<std::vector<std::pair<int32_t, uint32_t>>> out;  // sorted by dst
+  std::vector<std::vector<int32_t>> N;                         // sorted neighbours in U
+  std::vector<int64_t> T;                                      // triangles at each vertex
+
+  int64_t d(int32_t c) const { return (int64_t)N[c].size(); }
+  int64_t P(int32_t c) const { int64_t x = d(c); return x * (x - 1) / 2; }
+  bool high(int32_t c, int64_t th) const { return (__int128)T[c] * 1000000 > (__int128)th * P(c); }
+  bool adj(int32_t a, int32_t b) const { return std::binary_search(N[a].begin(), N[a].end(), b); }
+  const uint32_t* outw(int32_t a, int32_t b) const {
+    auto& r = out[a];
+    auto it = std::lower_bound(r.begin(), r.end(), std::make_pair(b, 0u),
+                               [](const std::pair<int32_t, uint32_t>& x, const std::pair<int32_t, uint32_t>& y) {
+                                 return x.first < y.first;
+                               });
+    return (it != r.end() && it->first == b) ? &it->second : nullptr;
+  }
+  bool eligible(int32_t c, int32_t a, int32_t b) const { return outw(a, c) && outw(c, b); }  // R23
+  static int64_t inter(const std::vector<int32_t>& x, const std::vector<int32_t>& y) {
+    int64_t r = 0;
+    size_t i = 0, j = 0;
+    while (i < x.size() && j < y.size()) {
+      if (x[i] < y[j]) i++;
+      else if (x[i] > y[j]) j++;
+      else { r++; i++; j++; }
+    }
+    return r;
+  }
+  void link(int32_t a, int32_t b, uint32_t w) {
+    const bool fresh = !adj(a, b);
+    auto& r = out[a];
+    auto it = std::lower_bound(r.begin(), r.end(), std::make_pair(b, 0u),
+                               [](const std::pair<int32_t, uint32_t>& x, const std::pair<int32_t, uint32_t>& y) {
+                                 return x.first < y.first;
+                               });
+    r.insert(it, {b, w});
+    if (fresh) {
+      // common neighbours gain a triangle; a and b gain |common| each
+      int64_t cnt = 0;
+      size_t i = 0, j = 0;
+      const auto &x = N[a], &y = N[b];
+      while (i < x.size() && j < y.size()) {
+        if (x[i] < y[j]) i++;
+        else if (x[i] > y[j]) j++;
+        else { T[x[i]]++; cnt++; i++; j++; }
+      }
+      T[a] += cnt;
+      T[b] += cnt;
+      N[a].insert(std::lower_bound(N[a].begin(), N[a].end(), b), b);
+      N[b].insert(std::lower_bound(N[b].begin(), N[b].end(), a), a);
+    }
+  }
+};
+
+void build_logical(const Work& W, Logical& L) {
+  const int64_t n = W.n;
+  L.n = n;
+  L.out.assign(n, {});
+  for (int64_t s = 0; s < W.n_slots; s++) {
+    if (W.kind[s] == HOLE) continue;
+    const int32_t u = W.slot_to_orig[s];
+    for (const Edge& e : W.rows[s]) L.out[u].push_back({W.slot_to_orig[e.dst], e.w});
+  }
+  std::vector<std::vector<int32_t>> inn(n);
+  for (int64_t u = 0; u < n; u++) {
+    std::sort(L.out[u].begin(), L.out[u].end());
+    for (auto& e : L.out[u]) inn[e.first].push_back((int32_t)u);
+  }
+  L.N.assign(n, {});
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int64_t u = 0; u < n; u++) {
+    auto& v = L.N[u];
+    v.reserve(L.out[u].size() + inn[u].size());
+    for (auto& e : L.out[u]) v.push_back(e.first);
+    for (int32_t x : inn[u]) v.push_back(x);
+    std::sort(v.begin(), v.end());
+    v.erase(std::unique(v.begin(), v.end()), v.end());
+  }
+  // triangles: forward algorithm over the degree-ordered orientation
+  L.T.assign(n, 0);
+  std::vector<std::vector<int32_t>> fwd(n);
+  auto rank_less = [&](int32_t a, int32_t b) {
+    return L.N[a].size() < L.N[b].size() || (L.N[a].size() == L.N[b].size() && a < b);
+  };
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int64_t u = 0; u < n; u++) {
+    for (int32_t v : L.N[u])
+      if (rank_less((int32_t)u, v)) fwd[u].push_back(v);
+    std::sort(fwd[u].begin(), fwd[u].end());
+  }
+  std::vector<int64_t> tl(n, 0);
+#pragma omp parallel
+  {
+    std::vector<int64_t> loc;  // per-thread counts for vertices touched
+#pragma omp for schedule(dynamic, 1024)
+    for (int64_t u = 0; u < n; u++) {
+      for (int32_t v : fwd[u]) {
+        const auto &x = fwd[u], &y = fwd[v];
+        size_t i = 0, j = 0;
+        while (i < x.size() && j < y.size()) {
+          if (x[i] < y[j]) i++;
+          else if (x[i] > y[j]) j++;
+          else {
+            const int32_t w = x[i];
+#pragma omp atomic
+            tl[u]++;
+#pragma omp atomic
+            tl[v]++;
+#pragma omp atomic
+            tl[w]++;
+            i++;
+            j++;
+          }
+        }
+      }
+    }
+  }
+  L.T.swap(tl);
+}
+
+struct SmemOut {
+  std::vector<std::tuple<int32_t, int32_t, uint32_t>> added;
+  std::vector<std::tuple<int32_t, std::vector<int32_t>, int32_t>> tiles;
+};
+
+// CC edge insertion: case 1 (R22) then case 2 (R24, R25); budget in directed edges (R26)
+void cc_edges(Logical& L, int64_t th, int64_t budget, SmemOut& out) {
+  const int64_t n = L.n;
+  int64_t rem = budget;
+  auto linkable = [&](int32_t c, int32_t a, int32_t b) {
+    return !L.adj(a, b) && (L.eligible(c, a, b) || L.eligible(c, b, a));
+  };
+  auto do_link = [&](int32_t c, int32_t a, int32_t b) {
+    const int32_t xs[2] = {a, b}, ys[2] = {b, a};
+    for (int q = 0; q < 2; q++) {
+      if (rem <= 0) return;
+      const int32_t x = xs[q], y = ys[q];
+      if (L.eligible(c, x, y) && !L.outw(x, y)) {
+        const uint32_t w = *L.outw(x, c) + *L.outw(c, y);
+        L.link(x, y, w);
+        out.added.push_back({x, y, w});
+        rem--;
+      }
+    }
+  };
+  // case 1
+  std::vector<std::pair<int64_t, int32_t>> cands;
+  for (int64_t c = 0; c < n; c++) {
+    if (L.d((int32_t)c) >= 2 && !L.high((int32_t)c, th)) {
+      const int64_t need = (int64_t)(((__int128)th * L.P((int32_t)c)) / 1000000) + 1 - L.T[c];
+      cands.push_back({need, (int32_t)c});
+    }
+  }
+  std::sort(cands.begin(), cands.end());
+  for (auto& cn : cands) {
+    if (rem <= 0) break;
+    const int32_t c = cn.second;
+    const int64_t P = L.P(c);
+    const int64_t need = (int64_t)(((__int128)th * P) / 1000000) + 1 - L.T[c];
+    if (need <= 0) continue;
+    if (P - L.T[c] < need) continue;
+    const std::vector<int32_t> Nc = L.N[c];
+    std::vector<std::tuple<int64_t, int32_t, int32_t>> pairs;
+    for (size_t i = 0; i < Nc.size(); i++)
+      for (size_t j = i + 1; j < Nc.size(); j++) {
+        const int32_t a = Nc[i], b = Nc[j];
+        if (linkable(c, a, b)) pairs.push_back({-Logical::inter(L.N[a], L.N[b]), a, b});
+      }
+    if ((int64_t)pairs.size() < need) continue;
+    std::sort(pairs.begin(), pairs.end());
+    for (auto& p : pairs) {
+      if (rem <= 0 || L.high(c, th)) break;
+      const int32_t a = std::get<1>(p), b = std::get<2>(p);
+      if (linkable(c, a, b)) do_link(c, a, b);
+    }
+  }
+  // case 2
+  if (rem > 0) {
+    std::vector<int32_t> highs;
+    for (int64_t c = 0; c < n; c++)
+      if (L.high((int32_t)c, th)) highs.push_back((int32_t)c);
+    std::sort(highs.begin(), highs.end(), [&](int32_t x, int32_t y) {
+      const __int128 lhs = (__int128)L.T[x] * L.P(y), rhs = (__int128)L.T[y] * L.P(x);
+      if (lhs != rhs) return lhs > rhs;
+      return x < y;
+    });
+    while (rem > 0) {
+      bool any = false;
+      for (int32_t c : highs) {
+        if (rem <= 0) break;
+        const std::vector<int32_t> Nc = L.N[c];
+        std::unordered_map<int32_t, int64_t> intdeg;
+        for (int32_t a : Nc) intdeg[a] = Logical::inter(L.N[a], Nc);
+        std::vector<int32_t> sib(Nc);
+        std::sort(sib.begin(), sib.end(), [&](int32_t x, int32_t y) {
+          return intdeg[x] != intdeg[y] ? intdeg[x] < intdeg[y] : x < y;
+        });
+        bool done = false;
+        for (int32_t a : sib) {
+          int32_t best = -1;
+          for (int32_t b : Nc) {
+            if (b == a || !linkable(c, a, b)) continue;
+            if (best < 0 || intdeg[b] < intdeg[best] || (intdeg[b] == intdeg[best] && b < best)) best = b;
+          }
+          if (best >= 0) {
+            do_link(c, std::min(a, best), std::max(a, best));
+            done = true;
+            break;
+          }
+        }
+        any |= done;
+      }
+      if (!any) break;
+    }
+  }
+}
+
+// disjoint shared-memory subgraphs (R27, R28)
+void subgraphs(const Logical& L, int64_t th, int smax, int smem_iters, SmemOut& out) {
+  const int64_t n = L.n;
+  std::vector<int32_t> cs;
+  for (int64_t c = 0; c < n; c++)
+    if (L.high((int32_t)c, th) && 1 + L.d((int32_t)c) <= smax) cs.push_back((int32_t)c);
+  std::sort(cs.begin(), cs.end(), [&](int32_t x, int32_t y) {
+    const __int128 lhs = (__int128)L.T[x] * L.P(y), rhs = (__int128)L.T[y] * L.P(x);
+    if (lhs != rhs) return lhs > rhs;
+    if (L.d(x) != L.d(y)) return L.d(x) > L.d(y);
+    return x < y;
+  });
+  std::vector<uint8_t> used(n, 0);
+  for (int32_t c : cs) {
+    bool free = !used[c];
+    for (int32_t v : L.N[c]) free = free && !used[v];
+    if (!free) continue;
+    std::vector<int32_t> S(L.N[c]);
+    S.push_back(c);
+    std::sort(S.begin(), S.end());
+    for (int32_t v : S) used[v] = 1;
+    const int64_t d = L.d(c);
+    const bool clique = L.T[c] == d * (d - 1) / 2;
+    const int32_t t = smem_iters > 0 ? smem_iters : 2 * (clique ? 1 : 2);
+    out.tiles.push_back({c, std::move(S), t});
+  }
+}
+
+// ---------------------------------------------------------------- §4
+int bucket_of(int64_t d) {
+  int b = 0;
+  while (d) {
+    b++;
+    d >>= 1;
+  }
+  return b;  // R30: 0 for d = 0, else 1 + floor(log2 d)
+}
+
+void degnorm(Work& W, int64_t th, int64_t f, bool combined, std::vector<int32_t>& sched, int64_t& added) {
+  const int64_t ns = W.n_slots;
+  std::vector<int64_t> deg(ns);
+  for (int64_t s = 0; s < ns; s++) deg[s] = (int64_t)W.rows[s].size();
+  std::vector<int32_t> order;
+  if (combined) {
+    order.resize(ns);
+    std::iota(order.begin(), order.end(), 0);
+  } else {
+    for (int64_t s = 0; s < ns; s++)
+      if (W.kind[s] != HOLE) order.push_back((int32_t)s);
+    std::stable_sort(order.begin(), order.end(),
+                     [&](int32_t a, int32_t b) { return bucket_of(deg[a]) > bucket_of(deg[b]); });
+  }
+  // pre-§4 logical out adjacency
+  std::vector<std::vector<std::pair<int32_t, uint32_t>>> lout(W.n);
+  for (int64_t s = 0; s < ns; s++) {
+    if (W.kind[s] == HOLE) continue;
+    for (const Edge& e : W.rows[s]) lout[W.slot_to_orig[s]].push_back({W.slot_to_orig[e.dst], e.w});
+  }
+  for (auto& r : lout) std::sort(r.begin(), r.end());
+  std::vector<std::vector<Edge>> adds(ns);
+  const int64_t nwarps = ((int64_t)order.size() + 31) / 32;
+#pragma omp parallel for schedule(dynamic, 64)
+  for (int64_t wi = 0; wi < nwarps; wi++) {
+    const int64_t b0 = wi * 32, b1 = std::min<int64_t>(b0 + 32, (int64_t)order.size());
+    int64_t M = 0;
+    for (int64_t i = b0; i < b1; i++) M = std::max(M, deg[order[i]]);
+    const int64_t target = (f * M + 999999) / 1000000;
+    for (int64_t i = b0; i < b1; i++) {
+      const int32_t s = order[i];
+      const int64_t d = deg[s];
+      if (W.kind[s] != OWNER || !(0 < d && d < M)) continue;
+      if (!((M - d) * 1000000 < th * M)) continue;
+      if (d >= target) continue;
+      const int32_t u = W.slot_to_orig[s];
+      const auto& ou = lout[u];
+      std::unordered_map<int32_t, uint32_t> best;
+      for (const auto& ex : ou)
+        for (const auto& eq : lout[ex.first]) {
+          const int32_t q = eq.first;
+          if (q == u) continue;
+          if (std::binary_search(ou.begin(), ou.end(), std::make_pair(q, 0u),
+                                 [](const std::pair<int32_t, uint32_t>& x, const std::pair<int32_t, uint32_t>& y) {
+                                   return x.first < y.first;
+                                 }))
+            continue;
+          const uint32_t w = ex.second + eq.second;
+          auto it = best.find(q);
+          if (it == best.end() || w < it->second) best[q] = w;
+        }
+      std::vector<std::pair<uint32_t, int32_t>> cand;
+      cand.reserve(best.size());
+      for (auto& kv : best) cand.push_back({kv.second, kv.first});
+      std::sort(cand.begin(), cand.end());
+      const int64_t take = std::min<int64_t>(target - d, (int64_t)cand.size());
+      for (int64_t j = 0; j < take; j++) adds[s].push_back({W.owner[cand[j].second], cand[j].first, ADD_DEGNORM});
+    }
+  }
+  added = 0;
+  for (int64_t s = 0; s < ns; s++) {
+    added += (int64_t)adds[s].size();
+    for (auto& e : adds[s]) W.rows[s].push_back(e);
+  }
+  sched = order;
+}
+
+}  // namespace
+
+void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out) {
+  auto t0 = std::chrono::steady_clock::now();
+  Work W;
+  if (k.coalesce) coalesce(g, k.chunk_k, ppm(k.replicate_threshold), W);
+  else identity(g, W);
+  SmemOut sm;
+  if (k.smem) {
+    Logical L;
+    build_logical(W, L);
+    const int64_t th = ppm(k.cc_threshold);
+    const int64_t budget = k.added_edge_budget >= 0 ? k.added_edge_budget : g.m / 100;
+    cc_edges(L, th, budget, sm);
+    subgraphs(L, th, k.smem_max_nodes, k.smem_iters, sm);
+    for (auto& e : sm.added)
+      W.rows[W.owner[std::get<0>(e)]].push_back({W.owner[std::get<1>(e)], std::get<2>(e), ADD_SMEM});
+  }
+  std::vector<int32_t> sched;
+  int64_t added_dn = 0;
+  if (k.degree_norm) degnorm(W, ppm(k.degsim_threshold), ppm(k.degree_target), k.coalesce != 0, sched, added_dn);
+
+  // assemble the slot CSR, rows sorted by destination slot (R11)
+  out = SlotGraph();
+  out.n = W.n;
+  out.n_slots = W.n_slots;
+  out.rp.assign(W.n_slots + 1, 0);
+  for (int64_t s = 0; s < W.n_slots; s++) out.rp[s + 1] = out.rp[s] + (int64_t)W.rows[s].size();
+  out.m_slots = out.rp[W.n_slots];
+  out.col.resize(out.m_slots);
+  out.w.resize(out.m_slots);
+  out.added.resize(out.m_slots);
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int64_t s = 0; s < W.n_slots; s++) {
+    auto& r = W.rows[s];
+    std::sort(r.begin(), r.end(), [](const Edge& a, const Edge& b) { return a.dst < b.dst; });
+    int64_t o = out.rp[s];
+    for (const Edge& e : r) {
+      out.col[o] = e.dst;
+      out.w[o] = e.w;
+      out.added[o] = e.added;
+      o++;
+    }
+  }
+  out.slot_to_orig = W.slot_to_orig;
+  out.kind = W.kind;
+  out.owner_slot = W.owner;
+  out.sched = sched;
+  out.tile_ptr.assign(1, 0);
+  for (auto& t : sm.tiles) {
+    out.tile_centre.push_back(std::get<0>(t));
+    for (int32_t v : std::get<1>(t)) out.tile_members.push_back(v);
+    out.tile_ptr.push_back((int64_t)out.tile_members.size());
+    out.tile_iters.push_back(std::get<2>(t));
+  }
+  gx_transform_info& I = out.info;
+  std::memset(&I, 0, sizeof(I));
+  I.n_slots = W.n_slots;
+  I.m_slots = out.m_slots;
+  I.n_holes = W.n_holes;
+  I.n_replicas = W.n_repl;
+  I.holes_filled = W.n_repl;
+  I.edges_added_coalesce = W.added_coal;
+  I.edges_added_smem = (int64_t)sm.added.size();
+  I.edges_added_degnorm = added_dn;
+  I.n_subgraphs = (int64_t)sm.tiles.size();
+  I.subgraph_vertices = (int64_t)out.tile_members.size();
+  // extra space (Table 5 analogue): added slots and edges relative to n + m
+  I.extra_space_pct = 100.0 * (double)((W.n_slots - W.n) + (out.m_slots - g.m)) / (double)std::max<int64_t>(1, g.n + g.m);
+  I.transform_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+}
+
+}  // namespace gx
