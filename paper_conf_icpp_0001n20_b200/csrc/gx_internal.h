@@ -122,14 +122,15 @@ struct DevGraph {
   // LB SSSP: static chunk list of rows with out-degree > HEAVY_DEG, heavy bitmap
   int64_t nhc = 0;
   DBuf hc_row, hc_start, heavy_bm;
-  // TPV / SELL-32 (filled on demand)
+  // TPV (paper's thread-per-vertex mapping, tpv.cu): lanes = the §4 schedule
+  // (or slot order), SELL-32 slabs of out-edges (SSSP) and in-edges (PR)
   bool tpv_ready = false;
-  int64_t n_warps_tpv = 0;
-  DBuf sched;                  // i32 [lanes]
-  DBuf sell_off;               // u64 [warps+1] slab offsets (in edges)
-  DBuf sell_adj;               // uint2 slabs, col = -1 padding
-  DBuf csell_off, csell_src;   // PR pull slabs (in-edges), src = -1 padding
-  int64_t sell_lanes = 0;
+  int64_t tpv_nslices = 0;
+  DBuf sched;                  // i32 [schedule length] (host sched uploaded)
+  DBuf tpv_lane_row;           // i32 [nslices*32 + 32], -1 = idle lane
+  DBuf tpv_out_len, tpv_out_off, tpv_out_slab;   // u32, u64, uint2 {dst, w}
+  DBuf tpv_in_len, tpv_in_off, tpv_in_slab;      // u32, u64, u32 src
+  int64_t tpv_out_slab_len = 0, tpv_in_slab_len = 0;
   // §3 tiles
   int64_t n_tiles = 0;
   DBuf t_ptr, t_members, t_eptr, t_edges, t_iters;  // local CSR per tile

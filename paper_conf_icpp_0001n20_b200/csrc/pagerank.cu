@@ -54,6 +54,12 @@ struct PrArgs {
   double* gnew;
   double base, damp, invN;
   PrState* st;
+  // TPV mapping (tpv.cu): lane-per-slot slabs of in-edges in schedule order
+  const int32_t* tpv_lane_row;
+  const uint32_t* tpv_len;
+  const uint64_t* tpv_off;
+  const uint32_t* tpv_slab;
+  int64_t tpv_nslices;
 };
 
 template <bool SLOTS>
@@ -169,6 +175,54 @@ __global__ void __launch_bounds__(PR_CTA) k_pr_sell(PrArgs a) {
   }
 }
 
+// The paper's thread-per-vertex pull (tpv.cu): lane = slot of the schedule,
+// each lane sums its own in-edges from the SELL-32 slab and finalises its
+// slot; a warp lasts as long as its longest row (what §4 normalises).
+template <bool SLOTS>
+__global__ void __launch_bounds__(256) k_pr_tpv(PrArgs a) {
+  __shared__ double s_red[32];
+  PrState* st = a.st;
+  if (st->stop) return;
+  const unsigned t = st->iter;
+  const float* __restrict__ cin = a.contrib[t & 1];
+  float* cout = a.contrib[(t + 1) & 1];
+  const double addc = a.base + a.damp * st->dang[t % 3] * a.invN;
+  double my_delta = 0, my_dang = 0;
+  const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
+  const unsigned lane = lane_id();
+  const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t sl = gw; sl < a.tpv_nslices; sl += nw) {
+    const int32_t row = a.tpv_lane_row[sl * 32 + lane];
+    const uint32_t L = a.tpv_len[sl];
+    const uint32_t* p = a.tpv_slab + a.tpv_off[sl] + lane;
+    double acc = 0.0;
+    uint32_t j = 0;
+    for (; j + PR_U <= L; j += PR_U) {
+      uint32_t e[PR_U];
+#pragma unroll
+      for (int u = 0; u < PR_U; u++) e[u] = row >= 0 ? ld_stream_u32(p + 32 * (j + u), pf) : PR_SENT;
+      float v[PR_U];
+#pragma unroll
+      for (int u = 0; u < PR_U; u++) v[u] = e[u] != PR_SENT ? ld_keep_f32(cin + e[u], pl) : 0.0f;
+#pragma unroll
+      for (int u = 0; u < PR_U; u++) acc += (double)v[u];
+    }
+    for (; j < L; j++) {
+      uint32_t e = row >= 0 ? ld_stream_u32(p + 32 * j, pf) : PR_SENT;
+      if (e != PR_SENT) acc += (double)ld_keep_f32(cin + e, pl);
+    }
+    if (row >= 0) pr_finalize<SLOTS>(a, row, acc, __ldcs(a.x + row), __ldcs(a.D + row), addc, cout, my_delta, my_dang);
+  }
+  double dsum = block_sum_f64(my_delta, s_red);
+  __syncthreads();
+  double gsum = block_sum_f64(my_dang, s_red);
+  if (threadIdx.x == 0) {
+    if (dsum != 0.0) atomicAdd(&st->delta[(t + 1) % 3], dsum);
+    if (gsum != 0.0) atomicAdd(&st->dang[(t + 1) % 3], gsum);
+  }
+}
+
 // §2.4 confluence: every copy <- mean(owner's new value, replicas' carried
 // values) (P@28609, mirror reading R19); next contrib for all copies.
 __global__ void k_pr_merge(PrArgs a, const int32_t* __restrict__ gptr, const int32_t* __restrict__ gslots,
@@ -233,7 +287,7 @@ __global__ void k_pr_init(PrArgs a, int64_t n_slots, double x0) {
 }
 
 void ensure_csc(gx_graph* g);  // devgraph.cu
-void run_pagerank_tpv_iter(gx_graph* g, void* args, int& launches);  // tpv.cu (pull over SELL slabs)
+void ensure_tpv(gx_graph* g);  // tpv.cu
 
 void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   Ctx* c = g->ctx;
@@ -273,6 +327,17 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   a.invN = 1.0 / (double)g->n;
   a.st = r.pst.as<PrState>();
   const bool slots = !d.identity;
+  int mapping = o.mapping;
+  if (mapping == GX_MAP_AUTO)
+    mapping = (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
+  if (mapping == GX_MAP_TPV) {
+    ensure_tpv(g);
+    a.tpv_lane_row = d.tpv_lane_row.as<int32_t>();
+    a.tpv_len = d.tpv_in_len.as<uint32_t>();
+    a.tpv_off = d.tpv_in_off.as<uint64_t>();
+    a.tpv_slab = d.tpv_in_slab.as<uint32_t>();
+    a.tpv_nslices = d.tpv_nslices;
+  }
 
   cudaEvent_t e0, e1;
   CUDA_OK(cudaEventCreate(&e0));
@@ -290,12 +355,20 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   else CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<false>, PR_CTA, 0));
   int grid = (int)std::max<int64_t>(1, std::min<int64_t>(PL.nwin, (int64_t)std::max(1, occ) * c->num_sms));
   int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 255) / 256, c->num_sms * 4));
+  int occt = 0;
+  CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occt, k_pr_tpv<true>, 256, 0));
+  const int grid_tpv = std::max(1, occt) * c->num_sms;
 
   KTimer kt(o.profile != 0, s);
   auto one_iter = [&](int& nl) {
     kt.begin();
-    if (slots) k_pr_sell<true><<<grid, PR_CTA, 0, s>>>(a);
-    else k_pr_sell<false><<<grid, PR_CTA, 0, s>>>(a);
+    if (mapping == GX_MAP_TPV) {
+      if (slots) k_pr_tpv<true><<<grid_tpv, 256, 0, s>>>(a);
+      else k_pr_tpv<false><<<grid_tpv, 256, 0, s>>>(a);
+    } else {
+      if (slots) k_pr_sell<true><<<grid, PR_CTA, 0, s>>>(a);
+      else k_pr_sell<false><<<grid, PR_CTA, 0, s>>>(a);
+    }
     kt.end();
     nl++;
     if (d.n_groups) {

@@ -166,6 +166,61 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
   }
 }
 
+// ---------------------------------------------------------------- TPV sweep
+// The paper's mapping (tpv.cu): one warp per 32-slot slice of the schedule,
+// lane = slot; a lane whose slot is in the frontier walks its row in the
+// SELL-32 slab (one coalesced 256-byte load per column).  The warp runs as
+// long as its longest active row -- the divergence that §4 normalises.
+__global__ void __launch_bounds__(256) k_sssp_tpv(const int32_t* __restrict__ lane_row, const uint32_t* __restrict__ slen,
+                                                  const uint64_t* __restrict__ soff, const uint2* __restrict__ slab,
+                                                  int64_t nslices, uint32_t* __restrict__ dist, SsspAux ax,
+                                                  SsspState* __restrict__ st) {
+  __shared__ unsigned long long sh[32];
+  const unsigned t = st->iter;
+  if (st->stop) return;
+  const uint32_t* __restrict__ bm_cur = ax.bm[t % 3];
+  uint32_t* bm_next = ax.bm[(t + 1) % 3];
+  clear_bitmap(ax.bm[(t + 2) % 3], ax.nwords);
+  const unsigned lane = lane_id();
+  const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
+  const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  unsigned long long my_edges = 0, my_act = 0;
+  for (int64_t sl = gw; sl < nslices; sl += nw) {
+    const int32_t row = lane_row[sl * 32 + lane];
+    const bool act = row >= 0 && bit_of(bm_cur, (uint32_t)row);
+    if (!__any_sync(FULL, act)) continue;
+    my_act += act;
+    const uint32_t du = act ? ld_l2_u32(dist + row, pl) : 0u;
+    const uint32_t L = slen[sl];
+    const uint2* p = slab + soff[sl] + lane;
+    for (uint32_t j = 0; j < L; j += SU) {
+      uint2 ed[SU];
+      bool ok[SU];
+#pragma unroll
+      for (int q = 0; q < SU; q++) {
+        ed[q] = (act && j + q < L) ? ld_stream_u2(p + 32 * (j + q), pf) : make_uint2(0xFFFFFFFFu, 0u);
+        ok[q] = ed[q].x != 0xFFFFFFFFu;
+      }
+      uint32_t cv[SU];
+#pragma unroll
+      for (int q = 0; q < SU; q++) cv[q] = ok[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
+#pragma unroll
+      for (int q = 0; q < SU; q++) {
+        if (ok[q]) relax_red(ed[q], du, cv[q], dist, bm_next, pl);
+        my_edges += ok[q];
+      }
+    }
+  }
+  unsigned long long e = block_sum_u64(my_edges, sh);
+  __syncthreads();
+  unsigned long long a2 = block_sum_u64(my_act, sh);
+  if (threadIdx.x == 0) {
+    if (e) atomicAdd(&st->edges, e);
+    if (a2) atomicAdd(&st->active[t % 3], (unsigned)a2);
+  }
+}
+
 // ---------------------------------------------------------------- §3 local pass
 // One CTA per subgraph tile: member distances staged in shared memory,
 // relaxed t times over the tile's local edges (P@32188-32416, reading R28),
@@ -353,7 +408,7 @@ int64_t default_source(gx_graph* g) {
 }
 
 // ---------------------------------------------------------------- driver
-void run_sssp_tpv_iter(gx_graph* g, SsspAux ax, SsspState* st, uint32_t* dist, int& launches);  // tpv.cu
+
 void ensure_tpv(gx_graph* g);                                                                  // tpv.cu
 
 static void ensure_heavy_chunks(gx_graph* g) {
@@ -441,6 +496,9 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   int occ = 0;
   CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sssp_lb, 256, 0));
   const int grid_lb = std::max(1, occ) * c->num_sms;
+  int occt = 0;
+  CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occt, k_sssp_tpv, 256, 0));
+  const int grid_tpv = std::max(1, occt) * c->num_sms;
   const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 8));
   const int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 7) / 8, (int64_t)c->num_sms * 8));
   const bool merge_min = g->knobs.merge_op == GX_MERGE_MIN;
@@ -449,7 +507,10 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   auto one_iter = [&](int& nl) {
     kt.begin();
     if (mapping == GX_MAP_TPV) {
-      run_sssp_tpv_iter(g, ax, st, r.dist.as<uint32_t>(), nl);
+      k_sssp_tpv<<<grid_tpv, 256, 0, s>>>(d.tpv_lane_row.as<int32_t>(), d.tpv_out_len.as<uint32_t>(),
+                                          d.tpv_out_off.as<uint64_t>(), d.tpv_out_slab.as<uint2>(), d.tpv_nslices,
+                                          r.dist.as<uint32_t>(), ax, st);
+      nl++;
     } else {
       k_sssp_lb<<<grid_lb, 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), r.dist.as<uint32_t>(), ax, st);
       nl++;

@@ -5,7 +5,4 @@ namespace gx {
 void run_scc(gx_graph*, const gx_run_opts&, gx_run_info&) { GX_THROW(GX_E_UNSUPPORTED, "SCC not built yet"); }
 void run_mst(gx_graph*, const gx_run_opts&, gx_run_info&) { GX_THROW(GX_E_UNSUPPORTED, "MST not built yet"); }
 void run_bc(gx_graph*, const gx_run_opts&, gx_run_info&) { GX_THROW(GX_E_UNSUPPORTED, "BC not built yet"); }
-struct SsspQueues;
-struct SsspState;
-void ensure_tpv(gx_graph*) { GX_THROW(GX_E_UNSUPPORTED, "TPV mapping not built yet"); }
 }  // namespace gx

@@ -1,0 +1,117 @@
+"""GPU parity of the transformed-graph sweeps with the oracle (SURVEY.md
+§8(a) A2-A11): every Graffix knob, both sweep mappings (LB and the paper's
+thread-per-vertex TPV), replica merges (mean / min) and the §3 local pass.
+
+* SSSP: bit-exact with Dijkstra on G_L (the oracle's definition on the
+  transformed graph), which Theorem E1 makes equal to Dijkstra on G.
+* PageRank: L1 <= 1e-6 against the oracle's PageRank of G_L (Theorem E3).
+"""
+import numpy as np
+import pytest
+
+import graphgen
+from golden_io import load
+from gpu_util import ctx, upload
+from oracle import algos as A
+from oracle import transform as T
+from oracle.graph import from_raw, graph_to_edgelist, sssp_source
+
+pytestmark = pytest.mark.gpu
+
+GRAPHS = {
+    "rmat12": lambda: graphgen.rmat(12),
+    "road48": lambda: graphgen.road(48),
+    "uniform": lambda: graphgen.uniform(3000, 30000),
+    "fig1_4": lambda: load("fig1_4.txt")[0],
+}
+KNOBS = {
+    "coal": T.Knobs(coalesce=True, chunk_k=16, replicate_threshold=0.4),
+    "coal_k4": T.Knobs(coalesce=True, chunk_k=4, replicate_threshold=0.2),
+    "smem": T.Knobs(smem=True, cc_threshold=0.3, added_edge_budget=200),
+    "degnorm": T.Knobs(degree_norm=True, degsim_threshold=0.5),
+    "all": T.Knobs(coalesce=True, chunk_k=8, replicate_threshold=0.3, smem=True, cc_threshold=0.3,
+                   degree_norm=True, degsim_threshold=0.5),
+}
+
+
+def knobs_c(kn, merge_op=0):
+    import paper_conf_icpp_0001n20_b200 as gx
+    d = {f: getattr(kn, f) for f in kn.__dataclass_fields__}
+    d["merge_op"] = merge_op
+    return gx.Knobs(**d)
+
+
+@pytest.mark.parametrize("gname", list(GRAPHS))
+@pytest.mark.parametrize("kname", list(KNOBS))
+@pytest.mark.parametrize("mapping", ["auto", "lb", "tpv"])
+def test_sssp_transformed_bit_exact(gname, kname, mapping):
+    raw = GRAPHS[gname]()
+    g = from_raw(raw)
+    kn = KNOBS[kname]
+    tg = T.transform(g, kn)
+    s = sssp_source(g)
+    want = A.sssp_dijkstra(tg.logical(), s)
+    assert np.array_equal(want, A.sssp_dijkstra(graph_to_edgelist(g), s))     # E1
+    G = upload(raw)
+    info = G.transform(knobs_c(kn))
+    assert info["n_replicas"] == tg.info["n_replicas"]
+    r = G.run("sssp", source=-1, mapping=mapping)
+    assert r["converged"] == 1
+    got = G.download("dist")
+    assert np.array_equal(got, want), f"{int(np.sum(got != want))} mismatches"
+
+
+@pytest.mark.parametrize("gname", list(GRAPHS))
+@pytest.mark.parametrize("kname", list(KNOBS))
+@pytest.mark.parametrize("mapping", ["lb", "tpv"])
+def test_pagerank_transformed_l1(gname, kname, mapping):
+    raw = GRAPHS[gname]()
+    g = from_raw(raw)
+    kn = KNOBS[kname]
+    tg = T.transform(g, kn)
+    want, _ = A.pagerank(tg.logical(), tol=1e-14)
+    G = upload(raw)
+    G.transform(knobs_c(kn))
+    G.run("pagerank", tol=1e-11, max_iters=5000, mapping=mapping)
+    got = G.download("rank")
+    assert np.abs(got - want).sum() <= 1e-6
+
+
+@pytest.mark.parametrize("gname", ["road48", "rmat12"])
+def test_merge_min_sssp(gname):
+    raw = GRAPHS[gname]()
+    g = from_raw(raw)
+    kn = T.Knobs(coalesce=True, chunk_k=4, replicate_threshold=0.0)
+    G = upload(raw)
+    G.transform(knobs_c(kn, merge_op=1))
+    G.run("sssp")
+    assert np.array_equal(G.download("dist"), A.sssp_dijkstra(graph_to_edgelist(g), sssp_source(g)))
+
+
+def test_device_transform_export_matches_oracle():
+    raw = graphgen.rmat(11)
+    kn = KNOBS["all"]
+    G = upload(raw)
+    G.transform(knobs_c(kn))
+    ex = G.export()
+    tg = T.transform(from_raw(raw), kn)
+    rp, col, w, ad = tg.csr()
+    assert ex["n_slots"] == tg.n_slots
+    assert np.array_equal(ex["row_ptr"], rp) and np.array_equal(ex["col"], col)
+    assert np.array_equal(ex["w"].astype(np.int64), w) and np.array_equal(ex["slot_kind"], tg.slot_kind)
+
+
+def test_inaccuracy_reporting():
+    """Inaccuracy per knob (P@40990): SSSP exact at convergence (E1), PR not."""
+    from oracle.metrics import inaccuracy
+    raw = graphgen.rmat(12)
+    G = upload(raw)
+    G.run("sssp")
+    d0 = G.download("dist")
+    G.run("pagerank", tol=1e-12)
+    x0 = G.download("rank")
+    G.transform(knobs_c(KNOBS["all"]))
+    G.run("sssp")
+    G.run("pagerank", tol=1e-12)
+    assert inaccuracy(G.download("dist"), d0)["inacc_pct"] == 0.0
+    assert inaccuracy(G.download("rank"), x0)["inacc_pct"] > 0.0
