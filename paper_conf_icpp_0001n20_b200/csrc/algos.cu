@@ -1,0 +1,487 @@
+// algos.cu -- the paper's other algorithms (PAPER.md P@36969: SSSP, MST, SCC,
+// PR, BC) on the logical graph G_L: every slot edge
+// with its source folded into the owner vertex (replica rows are part of the
+// owner's adjacency, reading R19 "owner broadcast"), including every edge the
+// transforms added.  Results are per original vertex.
+//
+//  * SCC: colouring (max-id forward propagation, backward closure from the
+//    colour roots), repeated on the unassigned vertices; label = min original
+//    id of the component (R38).  Bit-exact.
+//  * MST: Boruvka on the undirected view ({u,v} weighs the lighter direction,
+//    R39) with 64-bit (weight, edge) keys; minimum spanning forest weight.
+//  * BC: Brandes (Alg 1, Eq 1-2, P@12652-14843), unweighted, directed, over
+//    the caller's source sample (R37): level-synchronous forward pass with
+//    fp64 sigma (atomicAdd, P@14089), backward delta pass per level.
+#include <algorithm>
+#include <chrono>
+#include <cub/cub.cuh>
+
+#include "gx_internal.h"
+#include "kernels_common.cuh"
+
+namespace gx {
+
+// ---------------------------------------------------------------- G_L
+__global__ void k_esrc(const uint32_t* __restrict__ rp, int64_t n, uint32_t* __restrict__ esrc) {
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t u = warp; u < n; u += nw)
+    for (uint32_t e = rp[u] + lane_id(); e < rp[u + 1]; e += 32) esrc[e] = (uint32_t)u;
+}
+
+void ensure_logical(gx_graph* g) {
+  DevGraph& d = g->dg;
+  if (d.lg_ready) return;
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  const int64_t n = g->n;
+  if (!d.identity) {
+    const SlotGraph& sg = g->sg;
+    std::vector<uint32_t> rp(n + 1, 0);
+    for (int64_t sl = 0; sl < sg.n_slots; sl++)
+      if (sg.kind[sl] != HOLE) rp[sg.slot_to_orig[sl] + 1] += (uint32_t)(sg.rp[sl + 1] - sg.rp[sl]);
+    for (int64_t u = 0; u < n; u++) rp[u + 1] += rp[u];
+    std::vector<uint2> adj(std::max<uint32_t>(rp[n], 1));
+    std::vector<uint32_t> cur(rp.begin(), rp.end() - 1);
+    for (int64_t sl = 0; sl < sg.n_slots; sl++) {
+      if (sg.kind[sl] == HOLE) continue;
+      const int32_t u = sg.slot_to_orig[sl];
+      for (int64_t e = sg.rp[sl]; e < sg.rp[sl + 1]; e++)
+        adj[cur[u]++] = make_uint2((uint32_t)sg.slot_to_orig[sg.col[e]], sg.w[e]);
+    }
+    d.lg_m = rp[n];
+    d.lg_rp.alloc(c, sizeof(uint32_t) * (n + 1));
+    d.lg_adj.alloc(c, sizeof(uint2) * adj.size());
+    CUDA_OK(cudaMemcpyAsync(d.lg_rp.p, rp.data(), sizeof(uint32_t) * (n + 1), cudaMemcpyHostToDevice, s));
+    CUDA_OK(cudaMemcpyAsync(d.lg_adj.p, adj.data(), sizeof(uint2) * adj.size(), cudaMemcpyHostToDevice, s));
+    CUDA_OK(cudaStreamSynchronize(s));
+  } else {
+    d.lg_m = d.m_slots;
+  }
+  const uint32_t* rp = d.identity ? d.rp.as<uint32_t>() : d.lg_rp.as<uint32_t>();
+  d.lg_esrc.alloc(c, sizeof(uint32_t) * std::max<int64_t>(d.lg_m, 1));
+  if (n) k_esrc<<<grid_for(c, n * 32), 256, 0, s>>>(rp, n, d.lg_esrc.as<uint32_t>());
+  CUDA_OK(cudaGetLastError());
+  d.lg_ready = true;
+}
+
+struct LG {
+  const uint32_t* rp;
+  const uint2* adj;
+  const uint32_t* esrc;
+  int64_t n, m;
+};
+
+static LG logical(gx_graph* g) {
+  ensure_logical(g);
+  DevGraph& d = g->dg;
+  LG L;
+  L.rp = d.identity ? d.rp.as<uint32_t>() : d.lg_rp.as<uint32_t>();
+  L.adj = d.identity ? d.adj.as<uint2>() : d.lg_adj.as<uint2>();
+  L.esrc = d.lg_esrc.as<uint32_t>();
+  L.n = g->n;
+  L.m = d.lg_m;
+  return L;
+}
+
+#define GRID_STRIDE(i, n) for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < (n); i += (int64_t)gridDim.x * blockDim.x)
+
+// ---------------------------------------------------------------- SCC
+__global__ void k_scc_color_init(const int32_t* __restrict__ label, uint32_t* __restrict__ color,
+                                 uint8_t* __restrict__ vis, int64_t n) {
+  GRID_STRIDE(v, n) {
+    if (label[v] < 0) color[v] = (uint32_t)v;
+    vis[v] = 0;
+  }
+}
+// forward max-colour propagation over the edges of unassigned vertices
+__global__ void k_scc_fw(LG L, const int32_t* __restrict__ label, uint32_t* __restrict__ color, int* __restrict__ changed) {
+  int ch = 0;
+  GRID_STRIDE(e, L.m) {
+    const uint32_t u = L.esrc[e], v = L.adj[e].x;
+    if (label[u] < 0 && label[v] < 0) {
+      const uint32_t cu = __ldcg(color + u);
+      if (cu > __ldcg(color + v)) {
+        atomicMax(color + v, cu);
+        ch = 1;
+      }
+    }
+  }
+  if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
+}
+__global__ void k_scc_roots(const int32_t* __restrict__ label, const uint32_t* __restrict__ color,
+                            uint8_t* __restrict__ vis, int64_t n) {
+  GRID_STRIDE(v, n) if (label[v] < 0 && color[v] == (uint32_t)v) vis[v] = 1;
+}
+// backward closure inside each colour: u joins if it reaches a member
+__global__ void k_scc_bw(LG L, const int32_t* __restrict__ label, const uint32_t* __restrict__ color,
+                         uint8_t* __restrict__ vis, int* __restrict__ changed) {
+  int ch = 0;
+  GRID_STRIDE(e, L.m) {
+    const uint32_t u = L.esrc[e], v = L.adj[e].x;
+    if (label[u] < 0 && !vis[u] && vis[v] && color[u] == color[v]) {
+      vis[u] = 1;
+      ch = 1;
+    }
+  }
+  if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
+}
+__global__ void k_scc_assign(int32_t* __restrict__ label, const uint32_t* __restrict__ color,
+                             const uint8_t* __restrict__ vis, int64_t n, unsigned long long* __restrict__ left) {
+  unsigned long long c = 0;
+  GRID_STRIDE(v, n) {
+    if (label[v] < 0) {
+      if (vis[v]) label[v] = (int32_t)color[v];
+      else c++;
+    }
+  }
+  c = warp_sum_u64(c);
+  if (lane_id() == 0 && c) atomicAdd(left, c);
+}
+__global__ void k_scc_min(const int32_t* __restrict__ label, int32_t* __restrict__ smin, int64_t n) {
+  GRID_STRIDE(v, n) atomicMin(smin + label[v], (int32_t)v);
+}
+__global__ void k_scc_final(const int32_t* __restrict__ label, const int32_t* __restrict__ smin,
+                            int32_t* __restrict__ out, int64_t n) {
+  GRID_STRIDE(v, n) out[v] = smin[label[v]];
+}
+
+void run_scc(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  LG L = logical(g);
+  RunState& r = g->rs;
+  const int64_t n = L.n;
+  GX_CHECK_ARG(n > 0, "empty graph");
+  r.label.alloc(c, sizeof(int32_t) * n);
+  r.label2.alloc(c, sizeof(int32_t) * n);
+  r.comp.alloc(c, sizeof(uint32_t) * n);
+  r.changed.alloc(c, 64);
+  DBuf vis;
+  vis.alloc(c, n);
+  int32_t* label = r.label.as<int32_t>();
+  uint32_t* color = r.comp.as<uint32_t>();
+  int* changed = r.changed.as<int>();
+  unsigned long long* left = reinterpret_cast<unsigned long long*>(r.changed.as<char>() + 8);
+  const int gn = grid_for(c, n), ge = grid_for(c, std::max<int64_t>(L.m, 1));
+  cudaEvent_t e0, e1;
+  CUDA_OK(cudaEventCreate(&e0));
+  CUDA_OK(cudaEventCreate(&e1));
+  CUDA_OK(cudaEventRecord(e0, s));
+  CUDA_OK(cudaMemsetAsync(label, 0xFF, sizeof(int32_t) * n, s));
+  int launches = 0, rounds = 0;
+  int64_t edges = 0;
+  while (true) {
+    k_scc_color_init<<<gn, 256, 0, s>>>(label, color, vis.as<uint8_t>(), n);
+    launches++;
+    for (;;) {
+      int h = 0;
+      CUDA_OK(cudaMemsetAsync(changed, 0, 4, s));
+      k_scc_fw<<<ge, 256, 0, s>>>(L, label, color, changed);
+      launches++;
+      rounds++;
+      edges += L.m;
+      CUDA_OK(cudaMemcpyAsync(&h, changed, 4, cudaMemcpyDeviceToHost, s));
+      CUDA_OK(cudaStreamSynchronize(s));
+      if (!h) break;
+    }
+    k_scc_roots<<<gn, 256, 0, s>>>(label, color, vis.as<uint8_t>(), n);
+    launches++;
+    for (;;) {
+      int h = 0;
+      CUDA_OK(cudaMemsetAsync(changed, 0, 4, s));
+      k_scc_bw<<<ge, 256, 0, s>>>(L, label, color, vis.as<uint8_t>(), changed);
+      launches++;
+      rounds++;
+      edges += L.m;
+      CUDA_OK(cudaMemcpyAsync(&h, changed, 4, cudaMemcpyDeviceToHost, s));
+      CUDA_OK(cudaStreamSynchronize(s));
+      if (!h) break;
+    }
+    unsigned long long hl = 0;
+    CUDA_OK(cudaMemsetAsync(left, 0, 8, s));
+    k_scc_assign<<<gn, 256, 0, s>>>(label, color, vis.as<uint8_t>(), n, left);
+    launches++;
+    CUDA_OK(cudaMemcpyAsync(&hl, left, 8, cudaMemcpyDeviceToHost, s));
+    CUDA_OK(cudaStreamSynchronize(s));
+    if (hl == 0) break;
+  }
+  DBuf smin;
+  smin.alloc(c, sizeof(int32_t) * n);
+  CUDA_OK(cudaMemsetAsync(smin.p, 0x7F, sizeof(int32_t) * n, s));
+  k_scc_min<<<gn, 256, 0, s>>>(label, smin.as<int32_t>(), n);
+  k_scc_final<<<gn, 256, 0, s>>>(label, smin.as<int32_t>(), r.label2.as<int32_t>(), n);
+  launches += 2;
+  CUDA_OK(cudaEventRecord(e1, s));
+  CUDA_OK(cudaEventSynchronize(e1));
+  float ms = 0;
+  CUDA_OK(cudaEventElapsedTime(&ms, e0, e1));
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  info.iterations = rounds;
+  info.converged = 1;
+  info.loop_ms = ms;
+  info.edges_scanned = edges;
+  info.bytes_model = edges * 16;  // esrc 4 + {dst,w} 8 + 2 label/colour gathers
+  info.kernel_launches = launches;
+  r.have[GX_SCC] = true;
+}
+
+// ---------------------------------------------------------------- MST
+__global__ void k_mst_best(LG L, const uint32_t* __restrict__ comp, unsigned long long* __restrict__ best,
+                           int* __restrict__ any) {
+  int a = 0;
+  GRID_STRIDE(e, L.m) {
+    const uint32_t u = L.esrc[e];
+    const uint2 ed = L.adj[e];
+    const uint32_t cu = comp[u], cv = comp[ed.x];
+    if (cu != cv) {
+      const unsigned long long key = ((unsigned long long)ed.y << 32) | (unsigned long long)e;
+      atomicMin(best + cu, key);
+      atomicMin(best + cv, key);
+      a = 1;
+    }
+  }
+  if (__syncthreads_or(a) && threadIdx.x == 0) *any = 1;
+}
+__global__ void k_mst_hook(LG L, const uint32_t* __restrict__ comp, const unsigned long long* __restrict__ best,
+                           uint32_t* __restrict__ parent, int64_t n) {
+  GRID_STRIDE(cc, n) {
+    parent[cc] = (uint32_t)cc;
+    if (comp[cc] != (uint32_t)cc || best[cc] == ~0ull) continue;
+    const uint32_t e = (uint32_t)(best[cc] & 0xffffffffull);
+    const uint32_t cu = comp[L.esrc[e]], cv = comp[L.adj[e].x];
+    parent[cc] = cu == (uint32_t)cc ? cv : cu;
+  }
+}
+__global__ void k_mst_resolve(const uint32_t* __restrict__ comp, const unsigned long long* __restrict__ best,
+                              uint32_t* __restrict__ parent, int64_t n, unsigned long long* __restrict__ wsum) {
+  unsigned long long w = 0;
+  GRID_STRIDE(cc, n) {
+    if (comp[cc] != (uint32_t)cc || best[cc] == ~0ull) continue;
+    const uint32_t o = parent[cc];
+    const bool mutual = parent[o] == (uint32_t)cc;
+    if (!(mutual && (uint32_t)cc < o)) w += best[cc] >> 32;   // each chosen edge once
+  }
+  w = warp_sum_u64(w);
+  if (lane_id() == 0 && w) atomicAdd(wsum, w);
+}
+__global__ void k_mst_root(const uint32_t* __restrict__ comp, const unsigned long long* __restrict__ best,
+                           uint32_t* __restrict__ parent, int64_t n) {
+  GRID_STRIDE(cc, n) {
+    if (comp[cc] != (uint32_t)cc || best[cc] == ~0ull) continue;
+    const uint32_t o = parent[cc];
+    if (parent[o] == (uint32_t)cc && (uint32_t)cc < o) parent[cc] = (uint32_t)cc;
+  }
+}
+__global__ void k_mst_jump(uint32_t* __restrict__ parent, int64_t n, int* __restrict__ changed) {
+  int ch = 0;
+  GRID_STRIDE(cc, n) {
+    const uint32_t p = parent[cc], pp = parent[p];
+    if (p != pp) {
+      parent[cc] = pp;
+      ch = 1;
+    }
+  }
+  if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
+}
+__global__ void k_mst_relabel(uint32_t* __restrict__ comp, const uint32_t* __restrict__ parent, int64_t n) {
+  GRID_STRIDE(v, n) comp[v] = parent[comp[v]];
+}
+__global__ void k_iota_u32(uint32_t* __restrict__ a, int64_t n) { GRID_STRIDE(i, n) a[i] = (uint32_t)i; }
+
+void run_mst(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  LG L = logical(g);
+  RunState& r = g->rs;
+  const int64_t n = L.n;
+  GX_CHECK_ARG(n > 0, "empty graph");
+  GX_CHECK_ARG(L.m < (int64_t(1) << 32), "too many edges for 32-bit edge keys");
+  r.comp.alloc(c, sizeof(uint32_t) * n);
+  r.mst_best.alloc(c, sizeof(unsigned long long) * n);
+  r.changed.alloc(c, 64);
+  DBuf parent;
+  parent.alloc(c, sizeof(uint32_t) * n);
+  uint32_t* comp = r.comp.as<uint32_t>();
+  unsigned long long* best = r.mst_best.as<unsigned long long>();
+  int* flag = r.changed.as<int>();
+  unsigned long long* wsum = reinterpret_cast<unsigned long long*>(r.changed.as<char>() + 8);
+  const int gn = grid_for(c, n), ge = grid_for(c, std::max<int64_t>(L.m, 1));
+  cudaEvent_t e0, e1;
+  CUDA_OK(cudaEventCreate(&e0));
+  CUDA_OK(cudaEventCreate(&e1));
+  CUDA_OK(cudaEventRecord(e0, s));
+  k_iota_u32<<<gn, 256, 0, s>>>(comp, n);
+  CUDA_OK(cudaMemsetAsync(wsum, 0, 8, s));
+  int launches = 1, rounds = 0;
+  int64_t edges = 0;
+  while (true) {
+    int h = 0;
+    CUDA_OK(cudaMemsetAsync(best, 0xFF, sizeof(unsigned long long) * n, s));
+    CUDA_OK(cudaMemsetAsync(flag, 0, 4, s));
+    k_mst_best<<<ge, 256, 0, s>>>(L, comp, best, flag);
+    edges += L.m;
+    rounds++;
+    launches++;
+    CUDA_OK(cudaMemcpyAsync(&h, flag, 4, cudaMemcpyDeviceToHost, s));
+    CUDA_OK(cudaStreamSynchronize(s));
+    if (!h) break;
+    k_mst_hook<<<gn, 256, 0, s>>>(L, comp, best, parent.as<uint32_t>(), n);
+    k_mst_resolve<<<gn, 256, 0, s>>>(comp, best, parent.as<uint32_t>(), n, wsum);
+    k_mst_root<<<gn, 256, 0, s>>>(comp, best, parent.as<uint32_t>(), n);
+    launches += 3;
+    for (;;) {
+      int ch = 0;
+      CUDA_OK(cudaMemsetAsync(flag, 0, 4, s));
+      k_mst_jump<<<gn, 256, 0, s>>>(parent.as<uint32_t>(), n, flag);
+      launches++;
+      CUDA_OK(cudaMemcpyAsync(&ch, flag, 4, cudaMemcpyDeviceToHost, s));
+      CUDA_OK(cudaStreamSynchronize(s));
+      if (!ch) break;
+    }
+    k_mst_relabel<<<gn, 256, 0, s>>>(comp, parent.as<uint32_t>(), n);
+    launches++;
+  }
+  unsigned long long W = 0;
+  CUDA_OK(cudaMemcpyAsync(&W, wsum, 8, cudaMemcpyDeviceToHost, s));
+  CUDA_OK(cudaEventRecord(e1, s));
+  CUDA_OK(cudaEventSynchronize(e1));
+  float ms = 0;
+  CUDA_OK(cudaEventElapsedTime(&ms, e0, e1));
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  r.mst_weight = W;
+  info.iterations = rounds;
+  info.converged = 1;
+  info.loop_ms = ms;
+  info.edges_scanned = edges;
+  info.bytes_model = edges * 20;  // esrc 4 + {dst,w} 8 + 2 comp gathers
+  info.kernel_launches = launches;
+  r.have[GX_MST] = true;
+}
+
+// ---------------------------------------------------------------- BC
+// forward: warp per frontier vertex; a head joins level L+1 by CAS and
+// accumulates sigma from every level-L predecessor (P@14089).
+__global__ void k_bc_fwd(LG L, const int32_t* __restrict__ q, int64_t q0, int64_t q1, int32_t lvl,
+                         int32_t* __restrict__ level, double* __restrict__ sigma, int32_t* __restrict__ qout,
+                         unsigned int* __restrict__ qtail) {
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t i = q0 + warp; i < q1; i += nw) {
+    const int32_t u = q[i];
+    const double su = sigma[u];
+    for (uint32_t e = L.rp[u] + lane_id(); e < L.rp[u + 1]; e += 32) {
+      const uint32_t w = L.adj[e].x;
+      int32_t lw = __ldcg(level + w);
+      if (lw < 0) {
+        if (atomicCAS(level + w, -1, lvl + 1) == -1) {
+          const unsigned pos = atomicAdd(qtail, 1u);
+          qout[pos] = (int32_t)w;
+        }
+        lw = lvl + 1;
+      }
+      if (lw == lvl + 1) atomicAdd(sigma + w, su);
+    }
+  }
+}
+// backward: delta(v) = sum_{v->w, level w = level v + 1} sigma_v / sigma_w (1 + delta_w)  (Eq 1)
+__global__ void k_bc_bwd(LG L, const int32_t* __restrict__ q, int64_t q0, int64_t q1, int32_t lvl, int32_t src,
+                         const int32_t* __restrict__ level, const double* __restrict__ sigma, double* __restrict__ delta,
+                         double* __restrict__ bc) {
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t i = q0 + warp; i < q1; i += nw) {
+    const int32_t v = q[i];
+    double acc = 0.0;
+    for (uint32_t e = L.rp[v] + lane_id(); e < L.rp[v + 1]; e += 32) {
+      const uint32_t w = L.adj[e].x;
+      if (level[w] == lvl + 1) acc += (1.0 + delta[w]) / sigma[w];
+    }
+    acc = warp_sum_f64(acc) * sigma[v];
+    if (lane_id() == 0) {
+      delta[v] = acc;
+      if (v != src) bc[v] += acc;   // Eq 2
+    }
+  }
+}
+
+void run_bc(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  LG L = logical(g);
+  RunState& r = g->rs;
+  const int64_t n = L.n;
+  GX_CHECK_ARG(n > 0, "empty graph");
+  GX_CHECK_ARG(o.bc_sources != nullptr && o.n_bc_sources > 0, "BC needs bc_sources (reading R37)");
+  for (int64_t i = 0; i < o.n_bc_sources; i++)
+    GX_CHECK_ARG(o.bc_sources[i] >= 0 && o.bc_sources[i] < n, "BC source out of range");
+  r.level.alloc(c, sizeof(int32_t) * n);
+  r.sigma.alloc(c, sizeof(double) * n);
+  r.delta.alloc(c, sizeof(double) * n);
+  r.bc.alloc(c, sizeof(double) * n);
+  r.changed.alloc(c, 64);
+  DBuf q;
+  q.alloc(c, sizeof(int32_t) * n);
+  unsigned int* qtail = r.changed.as<unsigned int>();
+  const int gn = grid_for(c, n);
+  const int gw = c->num_sms * 16;
+  cudaEvent_t e0, e1;
+  CUDA_OK(cudaEventCreate(&e0));
+  CUDA_OK(cudaEventCreate(&e1));
+  CUDA_OK(cudaEventRecord(e0, s));
+  CUDA_OK(cudaMemsetAsync(r.bc.p, 0, sizeof(double) * n, s));
+  int launches = 0, rounds = 0;
+  int64_t edges = 0;
+  for (int64_t si = 0; si < o.n_bc_sources; si++) {
+    const int32_t src = (int32_t)o.bc_sources[si];
+    CUDA_OK(cudaMemsetAsync(r.level.p, 0xFF, sizeof(int32_t) * n, s));
+    CUDA_OK(cudaMemsetAsync(r.sigma.p, 0, sizeof(double) * n, s));
+    CUDA_OK(cudaMemsetAsync(r.delta.p, 0, sizeof(double) * n, s));
+    const int32_t zero = 0;
+    const double one = 1.0;
+    const unsigned int tail1 = 1;
+    CUDA_OK(cudaMemcpyAsync(r.level.as<int32_t>() + src, &zero, 4, cudaMemcpyHostToDevice, s));
+    CUDA_OK(cudaMemcpyAsync(r.sigma.as<double>() + src, &one, 8, cudaMemcpyHostToDevice, s));
+    CUDA_OK(cudaMemcpyAsync(q.as<int32_t>(), &src, 4, cudaMemcpyHostToDevice, s));
+    CUDA_OK(cudaMemcpyAsync(qtail, &tail1, 4, cudaMemcpyHostToDevice, s));
+    std::vector<int64_t> off{0, 1};
+    for (int32_t lvl = 0;; lvl++) {
+      const int64_t q0 = off[lvl], q1 = off[lvl + 1];
+      if (q1 == q0) break;
+      k_bc_fwd<<<gw, 256, 0, s>>>(L, q.as<int32_t>(), q0, q1, lvl, r.level.as<int32_t>(), r.sigma.as<double>(),
+                                  q.as<int32_t>(), qtail);
+      launches++;
+      rounds++;
+      unsigned int t = 0;
+      CUDA_OK(cudaMemcpyAsync(&t, qtail, 4, cudaMemcpyDeviceToHost, s));
+      CUDA_OK(cudaStreamSynchronize(s));
+      off.push_back(t);
+    }
+    // levels 0..D: off[l]..off[l+1]
+    const int32_t D = (int32_t)off.size() - 2;
+    for (int32_t lvl = D - 1; lvl >= 0; lvl--) {
+      k_bc_bwd<<<gw, 256, 0, s>>>(L, q.as<int32_t>(), off[lvl], off[lvl + 1], lvl, src, r.level.as<int32_t>(),
+                                  r.sigma.as<double>(), r.delta.as<double>(), r.bc.as<double>());
+      launches++;
+    }
+    edges += 2 * L.m;  // upper bound: every reached row scanned forward and backward
+  }
+  (void)gn;
+  CUDA_OK(cudaEventRecord(e1, s));
+  CUDA_OK(cudaEventSynchronize(e1));
+  float ms = 0;
+  CUDA_OK(cudaEventElapsedTime(&ms, e0, e1));
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  info.iterations = rounds;
+  info.converged = 1;
+  info.loop_ms = ms;
+  info.edges_scanned = edges;
+  info.bytes_model = edges * 20;
+  info.kernel_launches = launches;
+  r.have[GX_BC] = true;
+}
+
+}  // namespace gx

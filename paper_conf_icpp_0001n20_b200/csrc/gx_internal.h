@@ -131,6 +131,11 @@ struct DevGraph {
   DBuf tpv_out_len, tpv_out_off, tpv_out_slab;   // u32, u64, uint2 {dst, w}
   DBuf tpv_in_len, tpv_in_off, tpv_in_slab;      // u32, u64, u32 src
   int64_t tpv_out_slab_len = 0, tpv_in_slab_len = 0;
+  // logical graph G_L over original ids (replica rows folded into their
+  // owner): SCC / MST / BC (algos.cu); in exact mode it aliases rp / adj
+  bool lg_ready = false;
+  DBuf lg_rp, lg_adj, lg_esrc;  // u32 [n+1], uint2 {dst, w} [m_L], u32 [m_L]
+  int64_t lg_m = 0;
   // §3 tiles
   int64_t n_tiles = 0;
   DBuf t_ptr, t_members, t_eptr, t_edges, t_iters;  // local CSR per tile

@@ -91,7 +91,11 @@ void download(gx_graph* g, int kind, void* out, int64_t count, uint32_t flags) {
     case GX_OUT_BC_F64:
       if (!r.have[GX_BC]) GX_THROW(GX_E_STATE, "BC has not run on this graph");
       GX_CHECK_ARG(count == g->n, "count must be n");
-      gather_out<double>(g, r.bc, out, count, flags);
+      // BC runs on G_L over original ids (algos.cu): no owner gather
+      CUDA_OK(cudaMemcpyAsync(out, r.bc.p, sizeof(double) * count,
+                              (flags & GX_PTRS_DEVICE) ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
+                              g->ctx->stream));
+      CUDA_OK(cudaStreamSynchronize(g->ctx->stream));
       break;
     case GX_OUT_MST_WEIGHT_U64:
       if (!r.have[GX_MST]) GX_THROW(GX_E_STATE, "MST has not run on this graph");
