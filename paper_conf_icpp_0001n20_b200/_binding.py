@@ -13,7 +13,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libgraffix.so")
+LIB_PATH = os.environ.get("GX_LIB_PATH") or os.path.join(_HERE, "libgraffix.so")
 
 GX_OK, GX_E_INVALID, GX_E_STATE, GX_E_OOM, GX_E_CUDA, GX_E_NCCL, GX_E_UNSUPPORTED = range(7)
 STATUS_NAMES = ["GX_OK", "GX_E_INVALID", "GX_E_STATE", "GX_E_OOM", "GX_E_CUDA", "GX_E_NCCL",

@@ -12,11 +12,12 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-OUT = os.path.join(HERE, "libgraffix.so")
-OBJ = os.path.join(HERE, "build")
+OUT = os.environ.get("GX_BUILD_OUT") or os.path.join(HERE, "libgraffix.so")
+OBJ = os.environ.get("GX_BUILD_OBJ") or os.path.join(HERE, "build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-fopenmp,-O3", "-I" + os.path.join(HERE, "..", "include")]
+COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-fopenmp,-O3", "-I" + os.path.join(HERE, "..", "include")] + \
+    os.environ.get("GX_NVCC_EXTRA", "").split()
 
 
 def _sources():

@@ -82,7 +82,10 @@ __device__ __forceinline__ void pr_finalize(const PrArgs& a, int64_t v, double y
   if (!Dv) my_dang += xn;
 }
 
-constexpr int PR_CTA = 256;
+#ifndef GX_PR_CTA
+#define GX_PR_CTA 256
+#endif
+constexpr int PR_CTA = GX_PR_CTA;
 constexpr int PR_U = 8;   // gathers in flight per lane
 
 template <bool SLOTS>

@@ -15,6 +15,7 @@
 #include <cub/cub.cuh>
 
 #include <algorithm>
+#include <cstdlib>
 
 #include "gx_internal.h"
 #include "kernels_common.cuh"
@@ -29,7 +30,8 @@ namespace gx {
 template <int WR>
 __global__ void __launch_bounds__(1024) k_pr_window_sort(const uint32_t* __restrict__ crp, int64_t n,
                                                          int32_t* __restrict__ lane_tmp, int32_t* __restrict__ heavy_tmp,
-                                                         int32_t* __restrict__ nlight, int32_t* __restrict__ nheavy) {
+                                                         int32_t* __restrict__ nlight, int32_t* __restrict__ nheavy,
+                                                         uint32_t heavy_thr) {
   __shared__ uint32_t key[WR];
   const int64_t w = blockIdx.x;
   const int64_t base = w * WR;
@@ -38,9 +40,9 @@ __global__ void __launch_bounds__(1024) k_pr_window_sort(const uint32_t* __restr
     uint32_t k = 0xFFFFFFFFu;  // beyond n: sorts last
     if (r < n) {
       uint32_t d = crp[r + 1] - crp[r];
-      uint32_t cls = d > PR_HEAVY ? 1u : 0u;
-      uint32_t dd = d > PR_HEAVY ? 0u : (PR_HEAVY - d);
-      k = (cls << 31) | (dd << 12) | (uint32_t)i;   // WR <= 4096, PR_HEAVY < 2^19
+      uint32_t cls = d > heavy_thr ? 1u : 0u;
+      uint32_t dd = d > heavy_thr ? 0u : (heavy_thr - d);
+      k = (cls << 31) | (dd << 12) | (uint32_t)i;   // WR <= 4096, heavy_thr < 2^19
     }
     key[i] = k;
   }
@@ -188,8 +190,10 @@ void build_window_sell(Ctx* c, const uint32_t* rp, const T* payload, int64_t n, 
   heavy_tmp.alloc(c, sizeof(int32_t) * std::max<int64_t>(nwin * PRW, 1));
   nl.alloc(c, sizeof(int32_t) * (nwin + 1));
   nh.alloc(c, sizeof(int32_t) * (nwin + 1));
+  uint32_t heavy_thr = PR_HEAVY;
+  if (const char* e = getenv("GX_PR_HEAVY")) heavy_thr = (uint32_t)std::max(1, std::min(atoi(e), 1 << 18));
   if (nwin) k_pr_window_sort<PRW><<<nwin, 1024, 0, s>>>(rp, n, lane_tmp.as<int32_t>(), heavy_tmp.as<int32_t>(),
-                                                        nl.as<int32_t>(), nh.as<int32_t>());
+                                                        nl.as<int32_t>(), nh.as<int32_t>(), heavy_thr);
   CUDA_OK(cudaGetLastError());
   std::vector<int32_t> hnl(nwin), hnh(nwin);
   CUDA_OK(cudaMemcpyAsync(hnl.data(), nl.p, sizeof(int32_t) * nwin, cudaMemcpyDeviceToHost, s));

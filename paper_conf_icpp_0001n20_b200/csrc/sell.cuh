@@ -3,8 +3,11 @@
 #include "gx_internal.h"
 
 namespace gx {
-constexpr int PRW = 2048;               // rows per window (one CTA per window in the PR pull)
-constexpr uint32_t PR_HEAVY = 256;      // degree above which a row is processed warp-per-row
+#ifndef GX_PRW
+#define GX_PRW 1024
+#endif
+constexpr int PRW = GX_PRW;             // rows per window (one CTA per window in the PR pull)
+constexpr uint32_t PR_HEAVY = 64;       // degree above which a row is processed warp-per-row (swept: 64 best)
 template <class T>
 int64_t build_sell(Ctx* c, const uint32_t* rp, const T* payload, const int32_t* lane_row, int64_t nslices, T sentinel,
                    DBuf& slice_len, DBuf& slice_off, DBuf& slab);

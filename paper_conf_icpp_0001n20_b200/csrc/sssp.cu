@@ -27,6 +27,7 @@
 #include "sssp_common.cuh"
 #include <cub/cub.cuh>
 #include <cstdlib>
+#include <cstring>
 
 namespace gx {
 
@@ -69,7 +70,9 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
   const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
   const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  unsigned long long my_edges = 0, my_act = 0;
+  const uint32_t tau = st->tau;   // near-far: frontier slots with dist >= tau wait
+  unsigned long long my_edges = 0, my_act = 0, my_def = 0;
+  uint32_t my_min = INF;
 
   // heavy slots: static 1024-edge chunks of rows with out-degree > HEAVY_DEG
   for (int64_t c = gw; c < ax.nhc; c += nw) {
@@ -77,8 +80,16 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
     if (!bit_of(bm_cur, (uint32_t)u)) continue;       // warp-uniform
     const uint32_t a = ax.hc_start[c];
     const uint32_t b = min(a + HCHUNK, rp[u + 1]);
-    if (a == rp[u] && lane == 0) my_act++;
     const uint32_t du = ld_l2_u32(dist + u, pl);
+    if (du >= tau) {                                   // deferred to a later bucket
+      if (a == rp[u] && lane == 0) {
+        red_or_l2(bm_next + (u >> 5), 1u << (u & 31), pl);
+        my_def++;
+        my_min = min(my_min, du);
+      }
+      continue;
+    }
+    if (a == rp[u] && lane == 0) my_act++;
     for (uint32_t e0 = a; e0 < b; e0 += 32 * SU) {
       uint2 ed[SU];
       bool ok[SU];
@@ -114,15 +125,21 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
       word &= word - 1;
     }
     __syncwarp();
-    if (lane == 0) my_act += total;
     for (uint32_t base = 0; base < total; base += 32) {
       const uint32_t idx = base + lane;
       uint32_t start = 0, deg = 0, du = 0;
       if (idx < total) {
         const int32_t u = sv[idx];
-        start = rp[u];
-        deg = rp[u + 1] - start;
         du = ld_l2_u32(dist + u, pl);
+        if (du >= tau) {                               // deferred to a later bucket
+          red_or_l2(bm_next + (u >> 5), 1u << (u & 31), pl);
+          my_def++;
+          my_min = min(my_min, du);
+        } else {
+          start = rp[u];
+          deg = rp[u + 1] - start;
+          my_act++;
+        }
       }
       const uint32_t dincl = warp_incl_scan_u32(deg);
       const uint32_t dexcl = dincl - deg;
@@ -160,9 +177,14 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
   unsigned long long e = block_sum_u64(my_edges, sh);
   __syncthreads();
   unsigned long long a2 = block_sum_u64(my_act, sh);
+  __syncthreads();
+  unsigned long long d2 = block_sum_u64(my_def, sh);
+  my_min = warp_min_u32(my_min);
+  if (lane == 0 && my_min != INF) atomicMin(&st->mindef[t % 3], my_min);
   if (threadIdx.x == 0) {
     if (e) atomicAdd(&st->edges, e);
     if (a2) atomicAdd(&st->active[t % 3], (unsigned)a2);
+    if (d2) atomicAdd(&st->deferred[t % 3], (unsigned)d2);
   }
 }
 
@@ -327,12 +349,19 @@ __global__ void __launch_bounds__(256) k_sssp_merge(const int32_t* __restrict__ 
 __global__ void k_sssp_advance(SsspState* __restrict__ st, int max_iters) {
   if (st->stop) return;
   const unsigned t = st->iter;
-  const unsigned act = st->active[t % 3];
+  const unsigned act = st->active[t % 3], def = st->deferred[t % 3];
   st->act_total += act;
   st->active[(t + 2) % 3] = 0;
-  if (act == 0) {
+  st->deferred[(t + 2) % 3] = 0;
+  st->mindef[(t + 2) % 3] = INF;
+  if (act == 0 && def == 0) {
     st->stop = 1;
     return;
+  }
+  if (act == 0) {
+    // the current bucket drained: move the threshold past the nearest waiting slot
+    const unsigned long long nt = (unsigned long long)st->mindef[t % 3] + st->delta;
+    st->tau = nt >= INF ? INF : (unsigned)nt;
   }
   st->iter = t + 1;
   if ((int)(t + 1) >= max_iters) st->stop = 2;
@@ -411,6 +440,16 @@ int64_t default_source(gx_graph* g) {
 
 void ensure_tpv(gx_graph* g);                                                                  // tpv.cu
 
+// Near-far bucket width: a multiple of the mean edge weight scaled down by the
+// mean degree (delta-stepping's Delta ~ w / d heuristic), at least 1.
+static unsigned sssp_delta(const DevGraph& d) {
+  if (d.n_slots == 0 || d.m_slots == 0) return 0u;
+  const double avg_deg = (double)d.m_slots / (double)d.n_slots;
+  const double avg_w = 0.5 * (1.0 + (double)d.max_w);
+  const double delta = 8.0 * avg_w / std::max(1.0, avg_deg);
+  return (unsigned)std::max(1.0, delta);
+}
+
 static void ensure_heavy_chunks(gx_graph* g) {
   DevGraph& d = g->dg;
   if (d.hc_row.p) return;
@@ -488,7 +527,17 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   CUDA_OK(cudaEventRecord(e0, s));
   CUDA_OK(cudaMemsetAsync(r.dist.p, 0xFF, sizeof(uint32_t) * ns, s));
   CUDA_OK(cudaMemsetAsync(r.mark.p, 0, sizeof(uint32_t) * 3 * nwords, s));
-  CUDA_OK(cudaMemsetAsync(r.st.p, 0, sizeof(SsspState), s));
+  {
+    // near-far bucket width (LB mapping only; 0 = plain frontier Bellman-Ford)
+    static SsspState init;
+    std::memset(&init, 0, sizeof(init));
+    unsigned delta = mapping == GX_MAP_LB ? sssp_delta(d) : 0u;
+    if (const char* e = getenv("GX_SSSP_DELTA")) delta = (unsigned)std::max(0, atoi(e));
+    init.delta = delta;
+    init.tau = delta ? delta : INF;
+    for (int i = 0; i < 3; i++) init.mindef[i] = INF;
+    CUDA_OK(cudaMemcpyAsync(r.st.p, &init, sizeof(SsspState), cudaMemcpyHostToDevice, s));
+  }
   k_sssp_init<<<1, 32, 0, s>>>(r.dist.as<uint32_t>(), dsrc.as<int32_t>(), (int)srcs.size(), ax.bm[0]);
   CUDA_OK(cudaGetLastError());
   int launches = 4;

@@ -13,7 +13,11 @@ constexpr uint32_t HCHUNK = 1024;    // edges per heavy chunk
 struct SsspState {
   unsigned int iter;            // current iteration t
   unsigned int stop;            // 0 running, 1 converged (empty frontier), 2 max_iters
-  unsigned int active[3];       // slots in the frontier of iteration t (counted by its sweep)
+  unsigned int active[3];       // frontier slots processed in iteration t
+  unsigned int deferred[3];     // frontier slots with dist >= tau carried to t+1 (near-far)
+  unsigned int mindef[3];       // smallest deferred distance
+  unsigned int tau;             // near-far threshold: only dist < tau is relaxed
+  unsigned int delta;           // bucket width (0 = plain Bellman-Ford frontier)
   unsigned int raised;          // merges that raised a copy (diagnostic)
   unsigned long long edges;     // edges relaxed, all iterations
   unsigned long long act_total; // frontier entries, all iterations
