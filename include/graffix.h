@@ -132,7 +132,9 @@ typedef struct {
   int64_t n_bc_sources;
   int32_t profile;         /* 1 => eager launches with a CUDA event pair around every
                               main sweep kernel (sweep_ms / sweep_launches below)   */
-  int32_t pad_;
+  int32_t sim_ranks;       /* > 1 on a single-GPU context: run the 1-D partitioned
+                              path with this many simulated ranks (exchange by a
+                              device reduction instead of NCCL); LB mapping only    */
 } gx_run_opts;
 
 /* Transformed-graph export (debug / parity path).  Two-call protocol: call
@@ -223,6 +225,12 @@ gx_status gx_run_opts_default(gx_run_opts* o);
  * merge) into `out` (host or device per flags).  count = n, or 1 for MST.
  * Errors: GX_E_STATE (that algorithm has not run), GX_E_INVALID (count). */
 gx_status gx_download(gx_graph* g, int32_t kind, void* out, int64_t count, uint32_t flags);
+
+/* 1-D partition used by the multi-GPU path: bounds[0..P]
+ * over rows [0,n) of the host CSR row_ptr, balancing (edges + rows) per rank,
+ * each interior bound rounded to a multiple of `align` (the PR window, 1024).
+ * Host-only; no device needed.  Errors: GX_E_INVALID (P < 1, align < 1). */
+gx_status gx_partition_rows(int64_t n, const int64_t* row_ptr, int32_t P, int64_t align, int64_t* bounds);
 
 /* Synchronise the context stream (host wait). */
 gx_status gx_sync(gx_ctx* ctx);

@@ -69,8 +69,17 @@ class Context:
     @classmethod
     def distributed(cls, device: int, rank: int, world: int, group=None, stream=None):
         """One context per rank; the NCCL id is broadcast with torch.distributed."""
+        import glob
+        import os
+
         import torch
         import torch.distributed as dist
+        if not os.environ.get("GX_NCCL_LIB"):
+            # torch's bundled NCCL (SURVEY.md §5: avoid mixing two libnccl copies)
+            cands = glob.glob(os.path.join(os.path.dirname(torch.__file__), "..", "nvidia", "nccl", "lib",
+                                           "libnccl.so.2"))
+            if cands:
+                os.environ["GX_NCCL_LIB"] = os.path.realpath(cands[0])
         uid = torch.zeros(128, dtype=torch.uint8)
         if rank == 0:
             buf = (C.c_uint8 * 128)()
@@ -176,7 +185,7 @@ class Graph:
 
     def run(self, algo: str = "sssp", source: int = -1, max_iters: int = 0, tol: float = 1e-9,
             mapping: str = "auto", damping: float = 0.85, check_every: int = 8, use_graphs: bool = True,
-            bc_sources=None, profile: bool = False) -> dict:
+            bc_sources=None, profile: bool = False, sim_ranks: int = 0) -> dict:
         o = GxRunOpts()
         _check(lib().gx_run_opts_default(C.byref(o)))
         o.algo = ALGOS[algo]
@@ -188,6 +197,7 @@ class Graph:
         o.check_every = int(check_every)
         o.use_graphs = int(bool(use_graphs))
         o.profile = int(bool(profile))
+        o.sim_ranks = int(sim_ranks)
         keep = None
         if bc_sources is not None:
             keep = np.ascontiguousarray(bc_sources, dtype=np.int64)

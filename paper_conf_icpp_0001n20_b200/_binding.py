@@ -32,6 +32,7 @@ EXPORTED = [
     "gx_set_allocator", "gx_ctx_destroy", "gx_ctx_stream", "gx_graph_upload_csr", "gx_graph_destroy",
     "gx_graph_info", "gx_knobs_default", "gx_transform", "gx_export_sizes", "gx_export_transformed",
     "gx_run", "gx_run_ex", "gx_run_opts_default", "gx_download", "gx_sync", "gx_graph_create_host",
+    "gx_partition_rows",
 ]
 
 
@@ -61,7 +62,7 @@ class GxRunOpts(C.Structure):
     _fields_ = [("struct_size", C.c_uint32), ("algo", C.c_int32), ("source", C.c_int64),
                 ("max_iters", C.c_int32), ("mapping", C.c_int32), ("tol", C.c_double), ("damping", C.c_double),
                 ("check_every", C.c_int32), ("use_graphs", C.c_int32), ("bc_sources", C.c_void_p),
-                ("n_bc_sources", C.c_int64), ("profile", C.c_int32), ("pad_", C.c_int32)]
+                ("n_bc_sources", C.c_int64), ("profile", C.c_int32), ("sim_ranks", C.c_int32)]
 
 
 class GxExportSizes(C.Structure):
@@ -118,6 +119,7 @@ def lib():
         "gx_download": ([P, i32, P, i64, u32], C.c_int),
         "gx_sync": ([P], C.c_int),
         "gx_graph_create_host": ([C.POINTER(P), i64, i64, P, P, P, u32], C.c_int),
+        "gx_partition_rows": ([i64, P, i32, i64, P], C.c_int),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -130,6 +132,14 @@ def lib():
 def _check(st: int):
     if st != GX_OK:
         raise GraffixError(st, lib().gx_last_error().decode(errors="replace"))
+
+
+def partition_rows(row_ptr, P: int, align: int = 1024):
+    """Rank bounds of the 1-D partition (gx_partition_rows)."""
+    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    out = np.empty(P + 1, dtype=np.int64)
+    _check(lib().gx_partition_rows(int(row_ptr.shape[0]) - 1, _ptr(row_ptr), int(P), int(align), _ptr(out)))
+    return out
 
 
 def _ptr(a) -> C.c_void_p:

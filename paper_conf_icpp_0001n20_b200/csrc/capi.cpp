@@ -472,3 +472,15 @@ gx_status gx_download(gx_graph* g, int32_t kind, void* out, int64_t count, uint3
 }
 
 }  // extern "C"
+
+#include "dist.h"
+
+extern "C" gx_status gx_partition_rows(int64_t n, const int64_t* row_ptr, int32_t P, int64_t align, int64_t* bounds) {
+  GX_API_BEGIN
+  GX_CHECK_ARG(n >= 0 && row_ptr && bounds, "NULL argument");
+  GX_CHECK_ARG(P >= 1 && align >= 1, "P and align must be >= 1");
+  std::vector<int64_t> rp(row_ptr, row_ptr + n + 1);
+  std::vector<int64_t> b = gx::partition_rows(rp, n, P, align);
+  std::memcpy(bounds, b.data(), sizeof(int64_t) * (P + 1));
+  GX_API_END
+}

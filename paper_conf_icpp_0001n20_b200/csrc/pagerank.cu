@@ -22,6 +22,7 @@
 #include "kernels_common.cuh"
 #include "ktimer.h"
 #include "sell.cuh"
+#include "dist.h"
 
 namespace gx {
 
@@ -45,6 +46,7 @@ struct PrArgs {
   const uint32_t* crp;
   const int32_t* csrc;
   int64_t nwin;
+  int64_t win_lo, win_hi;  // this rank's windows (dist.h); [0, nwin) on one rank
   int64_t n_slots;
   double* x;
   float* contrib[2];
@@ -102,7 +104,7 @@ __global__ void __launch_bounds__(PR_CTA) k_pr_sell(PrArgs a) {
   const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
   const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
   constexpr unsigned NWARP = PR_CTA / 32;
-  for (int64_t w = blockIdx.x; w < a.nwin; w += gridDim.x) {
+  for (int64_t w = a.win_lo + blockIdx.x; w < a.win_hi; w += gridDim.x) {
     const int64_t base = w * PRW;
     const int nrows = (int)min((int64_t)PRW, a.n_slots - base);
     for (int i = threadIdx.x; i < PRW; i += PR_CTA) s_y[i] = 0.0;
@@ -292,6 +294,128 @@ __global__ void k_pr_init(PrArgs a, int64_t n_slots, double x0) {
 void ensure_csc(gx_graph* g);  // devgraph.cu
 void ensure_tpv(gx_graph* g);  // tpv.cu
 
+__global__ void k_mask_outside(double* __restrict__ x, int64_t n, int64_t lo, int64_t hi) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    if (i < lo || i >= hi) x[i] = 0.0;
+}
+
+// 1-D partitioned PageRank (dist.h): each rank pulls the windows of its own
+// row range and writes x / next contrib for those rows only; the exchange sums
+// the owned contrib slices (zero elsewhere, so the sum is exact), the L1 delta
+// and the dangling mass, and the owners' new values of replicated vertices;
+// the §2.4 merge then runs identically on every rank.
+static void run_pagerank_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, const PrArgs& a0, int P,
+                              bool sim) {
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  DevGraph& d = g->dg;
+  RunState& r = g->rs;
+  const int64_t ns = d.n_slots, ng = std::max<int64_t>(d.n_groups, 1);
+  const std::vector<int64_t> bounds = partition_rows_dev(c, d.crp.as<uint32_t>(), ns, P, PRW_ALIGN);
+  const int nloc = sim ? P : 1;
+  struct Rank {
+    DBuf x, c0, c1, gnew, st;
+    PrArgs a;
+    int64_t lo, hi;
+  };
+  std::vector<Rank> R(nloc);
+  cudaEvent_t e0, e1;
+  CUDA_OK(cudaEventCreate(&e0));
+  CUDA_OK(cudaEventCreate(&e1));
+  CUDA_OK(cudaEventRecord(e0, s));
+  for (int p = 0; p < nloc; p++) {
+    Rank& K = R[p];
+    DBuf& x = p == 0 ? r.x : K.x;
+    DBuf& c0 = p == 0 ? r.contrib[0] : K.c0;
+    DBuf& c1 = p == 0 ? r.contrib[1] : K.c1;
+    DBuf& gn = p == 0 ? r.gnew : K.gnew;
+    DBuf& st = p == 0 ? r.pst : K.st;
+    x.alloc(c, sizeof(double) * ns);
+    c0.alloc(c, sizeof(float) * ns);
+    c1.alloc(c, sizeof(float) * ns);
+    gn.alloc(c, sizeof(double) * ng);
+    st.alloc(c, sizeof(PrState));
+    K.a = a0;
+    K.a.x = x.as<double>();
+    K.a.contrib[0] = c0.as<float>();
+    K.a.contrib[1] = c1.as<float>();
+    K.a.gnew = gn.as<double>();
+    K.a.st = st.as<PrState>();
+    const int rank = sim ? p : c->rank;
+    K.lo = bounds[rank];
+    K.hi = bounds[rank + 1];
+    K.a.win_lo = K.lo / PRW;
+    K.a.win_hi = (K.hi + PRW - 1) / PRW;
+    CUDA_OK(cudaMemsetAsync(st.p, 0, sizeof(PrState), s));
+    if (d.identity) k_pr_init<false><<<grid_for(c, ns), 256, 0, s>>>(K.a, ns, 1.0 / (double)g->n);
+    else k_pr_init<true><<<grid_for(c, ns), 256, 0, s>>>(K.a, ns, 1.0 / (double)g->n);
+  }
+  Exch X;
+  X.c = c;
+  X.P = P;
+  X.sim = sim;
+  int occ = 0;
+  CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<true>, PR_CTA, 0));
+  const int grid = (int)std::max<int64_t>(1, (int64_t)std::max(1, occ) * c->num_sms);
+  const int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 255) / 256, c->num_sms * 4));
+  int launches = nloc, t = 0;
+  PrState h;
+  for (;; t++) {
+    std::vector<float*> cn;
+    std::vector<double*> dl, dg, gl;
+    for (int p = 0; p < nloc; p++) {
+      PrArgs& A = R[p].a;
+      float* cnext = A.contrib[(t + 1) & 1];
+      CUDA_OK(cudaMemsetAsync(cnext, 0, sizeof(float) * ns, s));
+      if (d.n_groups) CUDA_OK(cudaMemsetAsync(A.gnew, 0, sizeof(double) * ng, s));
+      if (d.identity) k_pr_sell<false><<<grid, PR_CTA, 0, s>>>(A);
+      else k_pr_sell<true><<<grid, PR_CTA, 0, s>>>(A);
+      launches++;
+      cn.push_back(cnext);
+      dl.push_back(&A.st->delta[0]);
+      dg.push_back(&A.st->dang[0]);
+      gl.push_back(A.gnew);
+    }
+    X.sum_f32(cn, ns);                                  // the exchange
+    X.sum_f64(dl, 3);
+    X.sum_f64(dg, 3);
+    if (d.n_groups) X.sum_f64(gl, d.n_groups);
+    for (int p = 0; p < nloc; p++) {
+      if (d.n_groups) {
+        k_pr_merge<<<grid_merge, 256, 0, s>>>(R[p].a, d.gptr.as<int32_t>(), d.gslots.as<int32_t>(), d.n_groups);
+        launches++;
+      }
+      k_pr_advance<<<1, 1, 0, s>>>(R[p].a.st, o.tol, o.max_iters);
+      launches++;
+    }
+    CUDA_OK(cudaMemcpyAsync(&h, R[0].a.st, sizeof(PrState), cudaMemcpyDeviceToHost, s));
+    CUDA_OK(cudaStreamSynchronize(s));
+    if (h.stop) break;
+  }
+  // assemble x: each slot from the rank that owns it
+  std::vector<double*> xl;
+  for (int p = 0; p < nloc; p++) {
+    k_mask_outside<<<grid_for(c, ns), 256, 0, s>>>(R[p].a.x, ns, R[p].lo, R[p].hi);
+    xl.push_back(R[p].a.x);
+  }
+  X.sum_f64(xl, ns);
+  CUDA_OK(cudaEventRecord(e1, s));
+  CUDA_OK(cudaEventSynchronize(e1));
+  float ms = 0;
+  CUDA_OK(cudaEventElapsedTime(&ms, e0, e1));
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  info.iterations = (int32_t)h.iter;
+  info.converged = h.stop == 1;
+  info.loop_ms = ms;
+  info.last_delta = h.last_delta;
+  info.edges_scanned = (int64_t)h.iter * d.m_slots;
+  info.vertices_active = (int64_t)h.iter * ns;
+  info.bytes_model = (int64_t)h.iter * (8 * d.m_slots + 24 * ns);
+  info.kernel_launches = launches;
+  r.have[GX_PAGERANK] = true;
+}
+
 void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   Ctx* c = g->ctx;
   cudaStream_t s = c->stream;
@@ -317,6 +441,8 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   a.crp = d.crp.as<uint32_t>();
   a.csrc = d.csrc.as<int32_t>();
   a.nwin = PL.nwin;
+  a.win_lo = 0;
+  a.win_hi = PL.nwin;
   a.n_slots = ns;
   a.x = r.x.as<double>();
   a.contrib[0] = r.contrib[0].as<float>();
@@ -330,6 +456,16 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   a.invN = 1.0 / (double)g->n;
   a.st = r.pst.as<PrState>();
   const bool slots = !d.identity;
+  {
+    const bool sim = c->world == 1 && o.sim_ranks > 1;
+    const int P = sim ? o.sim_ranks : c->world;
+    if (P > 1) {
+      GX_CHECK_ARG(P <= 8, "at most 8 ranks");
+      GX_CHECK_ARG(o.mapping != GX_MAP_TPV, "the partitioned path uses the LB mapping");
+      run_pagerank_dist(g, o, info, a, P, sim);
+      return;
+    }
+  }
   int mapping = o.mapping;
   if (mapping == GX_MAP_AUTO)
     mapping = (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;

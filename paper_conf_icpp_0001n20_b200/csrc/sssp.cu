@@ -25,6 +25,8 @@
 #include "kernels_common.cuh"
 #include "ktimer.h"
 #include "sssp_common.cuh"
+#include "dist.h"
+#include "sell.cuh"
 #include <cub/cub.cuh>
 #include <cstdlib>
 #include <cstring>
@@ -58,7 +60,8 @@ constexpr int SU = 4;         // edges in flight per lane per round
 constexpr int SB_WARPS = 8;   // warps per CTA
 
 __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj,
-                                                 uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st) {
+                                                 uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st,
+                                                 int64_t row_lo, int64_t row_hi) {
   __shared__ int32_t s_v[SB_WARPS][1024];
   __shared__ unsigned long long sh[32];
   const unsigned t = st->iter;
@@ -77,6 +80,7 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
   // heavy slots: static 1024-edge chunks of rows with out-degree > HEAVY_DEG
   for (int64_t c = gw; c < ax.nhc; c += nw) {
     const int32_t u = ax.hc_row[c];
+    if (u < row_lo || u >= row_hi) continue;          // another rank's rows (dist.h)
     if (!bit_of(bm_cur, (uint32_t)u)) continue;       // warp-uniform
     const uint32_t a = ax.hc_start[c];
     const uint32_t b = min(a + HCHUNK, rp[u + 1]);
@@ -111,9 +115,10 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
 
   // light slots: compact the frontier bits of 32 words, 32 slots per round
   int32_t* sv = s_v[wib];
-  for (int64_t wb = gw * 32; wb < ax.nwords; wb += nw * 32) {
+  const int64_t w_lo = row_lo >> 5, w_hi = min((row_hi + 31) >> 5, ax.nwords);   // ranges are 32-aligned
+  for (int64_t wb = w_lo + gw * 32; wb < w_hi; wb += nw * 32) {
     const int64_t wi = wb + lane;
-    uint32_t word = wi < ax.nwords ? (__ldcg(bm_cur + wi) & ~__ldg(ax.heavy + wi)) : 0u;
+    uint32_t word = wi < w_hi ? (__ldcg(bm_cur + wi) & ~__ldg(ax.heavy + wi)) : 0u;
     const uint32_t cnt = __popc(word);
     const uint32_t incl = warp_incl_scan_u32(cnt);
     const uint32_t total = __shfl_sync(FULL, incl, 31);
@@ -479,6 +484,157 @@ static void ensure_heavy_chunks(gx_graph* g) {
   CUDA_OK(cudaStreamSynchronize(s));
 }
 
+// owned slots whose distance dropped in this iteration (any rank's relaxation,
+// visible after the allreduce) join this rank's next frontier
+__global__ void k_frontier_diff(const uint32_t* __restrict__ dist, const uint32_t* __restrict__ dold, SsspAux ax,
+                                const SsspState* __restrict__ st, int64_t lo, int64_t hi) {
+  if (st->stop) return;
+  uint32_t* bm_next = ax.bm[(st->iter + 1) % 3];
+  const int64_t w_lo = lo >> 5, w_hi = min((hi + 31) >> 5, ax.nwords);
+  for (int64_t w = w_lo + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < w_hi; w += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t bits = 0;
+    for (int b = 0; b < 32; b++) {
+      const int64_t v = w * 32 + b;
+      if (v >= lo && v < hi && dist[v] < dold[v]) bits |= 1u << b;
+    }
+    if (bits) bm_next[w] |= bits;
+  }
+}
+
+struct SsspRank {
+  DBuf dist, mark, st, dold;
+  SsspAux ax;
+  int64_t lo = 0, hi = 0;
+};
+
+// 1-D partitioned SSSP (dist.h): each rank relaxes the frontier slots of its
+// own range; after every sweep dist is allreduced with min, the owners rebuild
+// their next frontier from the distances that dropped, and the frontier
+// counters are allreduced so every rank takes the same near-far decision.
+static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, int P, bool sim, int64_t src,
+                          unsigned delta) {
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  DevGraph& d = g->dg;
+  RunState& r = g->rs;
+  const int64_t ns = d.n_slots, nwords = (ns + 31) / 32;
+  const std::vector<int64_t> bounds = partition_rows_dev(c, d.rp.as<uint32_t>(), ns, P, PRW_ALIGN);
+  const int nloc = sim ? P : 1;
+  std::vector<SsspRank> R(nloc);
+  std::vector<int32_t> srcs{d.identity ? (int32_t)src : g->sg.owner_slot[src]};
+  if (!d.identity)
+    for (int64_t sl = 0; sl < g->sg.n_slots; sl++)
+      if (g->sg.kind[sl] == REPLICA && g->sg.slot_to_orig[sl] == src) srcs.push_back((int32_t)sl);
+  DBuf dsrc;
+  dsrc.alloc(c, sizeof(int32_t) * srcs.size());
+  CUDA_OK(cudaMemcpyAsync(dsrc.p, srcs.data(), sizeof(int32_t) * srcs.size(), cudaMemcpyHostToDevice, s));
+  SsspState init;
+  std::memset(&init, 0, sizeof(init));
+  init.delta = delta;
+  init.tau = delta ? delta : INF;
+  for (int i = 0; i < 3; i++) init.mindef[i] = INF;
+  cudaEvent_t e0, e1;
+  CUDA_OK(cudaEventCreate(&e0));
+  CUDA_OK(cudaEventCreate(&e1));
+  CUDA_OK(cudaEventRecord(e0, s));
+  for (int p = 0; p < nloc; p++) {
+    SsspRank& K = R[p];
+    DBuf& dist = p == 0 ? r.dist : K.dist;
+    DBuf& mark = p == 0 ? r.mark : K.mark;
+    DBuf& st = p == 0 ? r.st : K.st;
+    dist.alloc(c, sizeof(uint32_t) * ns);
+    mark.alloc(c, sizeof(uint32_t) * 3 * nwords);
+    st.alloc(c, sizeof(SsspState));
+    K.dold.alloc(c, sizeof(uint32_t) * ns);
+    for (int i = 0; i < 3; i++) K.ax.bm[i] = mark.as<uint32_t>() + i * nwords;
+    K.ax.heavy = d.heavy_bm.as<uint32_t>();
+    K.ax.nwords = nwords;
+    K.ax.hc_row = d.hc_row.as<int32_t>();
+    K.ax.hc_start = d.hc_start.as<uint32_t>();
+    K.ax.nhc = d.nhc;
+    const int rank = sim ? p : c->rank;
+    K.lo = bounds[rank];
+    K.hi = bounds[rank + 1];
+    CUDA_OK(cudaMemsetAsync(dist.p, 0xFF, sizeof(uint32_t) * ns, s));
+    CUDA_OK(cudaMemsetAsync(mark.p, 0, sizeof(uint32_t) * 3 * nwords, s));
+    CUDA_OK(cudaMemcpyAsync(st.p, &init, sizeof(SsspState), cudaMemcpyHostToDevice, s));
+    k_sssp_init<<<1, 32, 0, s>>>(dist.as<uint32_t>(), dsrc.as<int32_t>(), (int)srcs.size(), K.ax.bm[0]);
+  }
+  auto D = [&](int p) { return (p == 0 ? r.dist : R[p].dist).as<uint32_t>(); };
+  auto S = [&](int p) { return (p == 0 ? r.st : R[p].st).as<SsspState>(); };
+  Exch X;
+  X.c = c;
+  X.P = P;
+  X.sim = sim;
+  int occ = 0;
+  CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sssp_lb, 256, 0));
+  const int grid_lb = std::max(1, occ) * c->num_sms;
+  const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 8));
+  const int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 7) / 8, (int64_t)c->num_sms * 8));
+  const bool merge_min = g->knobs.merge_op == GX_MERGE_MIN;
+  int launches = 0;
+  SsspState hst;
+  std::vector<uint32_t*> dl, al, fl, ml;
+  for (int p = 0; p < nloc; p++) {
+    dl.push_back(D(p));
+    al.push_back(&S(p)->active[0]);
+    fl.push_back(&S(p)->deferred[0]);
+    ml.push_back(&S(p)->mindef[0]);
+  }
+  for (;;) {
+    for (int p = 0; p < nloc; p++) {
+      CUDA_OK(cudaMemcpyAsync(R[p].dold.p, D(p), sizeof(uint32_t) * ns, cudaMemcpyDeviceToDevice, s));
+      k_sssp_lb<<<grid_lb, 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), D(p), R[p].ax, S(p), R[p].lo, R[p].hi);
+      launches++;
+      if (d.n_tiles && g->knobs.smem) {
+        k_sssp_local<<<grid_local, 256, 0, s>>>(d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(), d.t_eptr.as<int32_t>(),
+                                                d.t_edges.as<uint2>(), d.t_iters.as<int32_t>(), d.n_tiles, D(p), R[p].ax,
+                                                S(p));
+        launches++;
+      }
+    }
+    X.min_u32(dl, ns);                                  // the exchange
+    for (int p = 0; p < nloc; p++) {
+      if (d.n_groups) {
+        k_sssp_merge<<<grid_merge, 256, 0, s>>>(d.gptr.as<int32_t>(), d.gslots.as<int32_t>(), d.g_in_ptr.as<int32_t>(),
+                                                d.g_in.as<uint2>(), d.n_groups, merge_min ? 1 : 0, D(p), R[p].ax, S(p));
+        launches++;
+      }
+      k_frontier_diff<<<grid_for(c, nwords), 256, 0, s>>>(D(p), R[p].dold.as<uint32_t>(), R[p].ax, S(p), R[p].lo,
+                                                           R[p].hi);
+      launches++;
+    }
+    X.sum_u32(al, 3);
+    X.sum_u32(fl, 3);
+    X.min_u32(ml, 3);
+    for (int p = 0; p < nloc; p++) k_sssp_advance<<<1, 1, 0, s>>>(S(p), o.max_iters), launches++;
+    CUDA_OK(cudaMemcpyAsync(&hst, S(0), sizeof(SsspState), cudaMemcpyDeviceToHost, s));
+    CUDA_OK(cudaStreamSynchronize(s));
+    if (hst.stop) break;
+  }
+  unsigned long long edges = 0;
+  for (int p = 0; p < nloc; p++) {
+    SsspState h;
+    CUDA_OK(cudaMemcpyAsync(&h, S(p), sizeof(SsspState), cudaMemcpyDeviceToHost, s));
+    CUDA_OK(cudaStreamSynchronize(s));
+    edges += h.edges;
+  }
+  CUDA_OK(cudaEventRecord(e1, s));
+  CUDA_OK(cudaEventSynchronize(e1));
+  float ms = 0;
+  CUDA_OK(cudaEventElapsedTime(&ms, e0, e1));
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  info.iterations = (int32_t)hst.iter;
+  info.converged = hst.stop == 1;
+  info.loop_ms = ms;
+  info.edges_scanned = (int64_t)edges;
+  info.vertices_active = (int64_t)hst.act_total;
+  info.bytes_model = 12 * (int64_t)edges + 12 * (int64_t)hst.act_total;
+  info.kernel_launches = launches;
+  r.have[GX_SSSP] = true;
+}
+
 void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   Ctx* c = g->ctx;
   cudaStream_t s = c->stream;
@@ -489,6 +645,17 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   GX_CHECK_ARG(src >= 0 && src < g->n, "source out of range");
   if ((double)(g->n - 1) * (double)d.max_w >= 4294967295.0)
     GX_THROW(GX_E_UNSUPPORTED, "(n-1)*max(w) >= 2^32-1 would overflow uint32 distances");
+  const bool sim = c->world == 1 && o.sim_ranks > 1;
+  const int P = sim ? o.sim_ranks : c->world;
+  if (P > 1) {
+    GX_CHECK_ARG(P <= 8, "at most 8 ranks");
+    GX_CHECK_ARG(o.mapping != GX_MAP_TPV, "the partitioned path uses the LB mapping");
+    ensure_heavy_chunks(g);
+    unsigned delta = sssp_delta(d);
+    if (const char* e = getenv("GX_SSSP_DELTA")) delta = (unsigned)std::max(0, atoi(e));
+    run_sssp_dist(g, o, info, P, sim, src, delta);
+    return;
+  }
   int mapping = o.mapping;
   if (mapping == GX_MAP_AUTO)
     mapping = (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
@@ -561,7 +728,7 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
                                           r.dist.as<uint32_t>(), ax, st);
       nl++;
     } else {
-      k_sssp_lb<<<grid_lb, 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), r.dist.as<uint32_t>(), ax, st);
+      k_sssp_lb<<<grid_lb, 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), r.dist.as<uint32_t>(), ax, st, 0, ns);
       nl++;
     }
     kt.end();
