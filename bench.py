@@ -225,8 +225,15 @@ def main():
     dom = max(kern, key=lambda k: kern[k]["ms_total"])
     dk = kern[dom]
     achieved = dk["gbs"]
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "latest", "traffic.json")
+    if os.path.exists(tpath):
+        tj = json.load(open(tpath))
+        if dom in tj:
+            traffic = tj[dom]["traffic_bytes_per_launch"]
     roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
-                "frac": achieved / peak if achieved else None, "traffic": None, "peak_source": peak_src,
+                "frac": achieved / peak if achieved else None, "traffic": traffic,
+                "traffic_unit": "bytes/launch (ncu dram read+write, profiles/latest)", "peak_source": peak_src,
                 "bytes_per_launch": dk["bytes"] / max(dk["launches"], 1),
                 "us_per_launch": 1e3 * dk["ms_total"] / max(dk["launches"], 1)}
 
