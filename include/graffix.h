@@ -54,7 +54,8 @@ typedef enum {
 typedef enum { GX_SSSP = 1, GX_PAGERANK = 2, GX_SCC = 3, GX_MST = 4, GX_BC = 5 } gx_algo;
 
 /* Confluence operator (§2.4, P@28421-28736): the paper's algorithm-agnostic
- * arithmetic mean, or the algorithm-aware min (SSSP only). */
+ * arithmetic mean, or the algorithm-aware one (SSSP: min of the copies;
+ * PageRank: the owner's new value broadcast to its replicas). */
 typedef enum { GX_MERGE_MEAN = 0, GX_MERGE_MIN = 1 } gx_merge;
 
 /* Sweep mapping.  LB: edge-balanced warp-cooperative kernels (the best exact
@@ -106,7 +107,9 @@ typedef struct {
 } gx_transform_info;
 
 typedef struct {
-  int32_t iterations, converged;
+  int32_t iterations;
+  int32_t converged;       /* 1 fixed point reached (SSSP: empty frontier; PR: delta < tol),
+                              0 max_iters hit, 2 PR stopped at the fp32-contrib noise floor */
   double loop_ms;          /* device time of init + fixed-point loop (CUDA events) */
   double last_delta;       /* PR: final L1 delta                                   */
   int64_t edges_scanned;   /* edges relaxed / gathered over all iterations         */

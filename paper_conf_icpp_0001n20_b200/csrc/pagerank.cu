@@ -30,8 +30,11 @@ struct PrState {
   double delta[3];   // L1 change of x_{t+1}, accumulated into [(t+1)%3]
   double dang[3];    // sum of x_t over dangling vertices, [t%3]
   unsigned iter;
-  unsigned stop;     // 1 converged, 2 max_iters
+  unsigned stop;     // 1 converged (delta < tol), 2 max_iters, 3 at the fp32-contrib noise floor
   double last_delta;
+  double best_delta; // smallest delta so far (stagnation test)
+  unsigned stall;    // iterations since best_delta last improved by >= 1 %
+  unsigned pad;
 };
 
 struct PrArgs {
@@ -56,6 +59,7 @@ struct PrArgs {
   double* gnew;
   double base, damp, invN;
   PrState* st;
+  int merge_bcast;       // 1: algorithm-aware merge (owner broadcast), else mean
   // TPV mapping (tpv.cu): lane-per-slot slabs of in-edges in schedule order
   const int32_t* tpv_lane_row;
   const uint32_t* tpv_len;
@@ -243,7 +247,10 @@ __global__ void k_pr_merge(PrArgs a, const int32_t* __restrict__ gptr, const int
     int32_t o = gslots[b];
     double s = a.gnew[g];
     for (int i = b + 1; i < e; i++) s += a.x[gslots[i]];
-    double mean = s / (double)(e - b);
+    // GX_MERGE_MEAN: the paper's algorithm-agnostic mean (P@28609) over the
+    // owner's new value and the replicas' carried values; the algorithm-aware
+    // alternative (P@28421) for PR broadcasts the owner's new value (R54)
+    double mean = a.merge_bcast ? a.gnew[g] : s / (double)(e - b);
     my_delta += fabs(mean - a.x[o]);
     uint32_t Dv = a.D[o];
     float c = Dv ? (float)(mean / (double)Dv) : 0.0f;
@@ -270,7 +277,17 @@ __global__ void k_pr_advance(PrState* st, double tol, int max_iters) {
   st->delta[(t + 2) % 3] = 0.0;
   st->dang[(t + 2) % 3] = 0.0;
   st->iter = t + 1;
+  // contrib is stored in fp32: once the iterate reaches the fixed point of the
+  // rounded map it may cycle at a delta floor ~1e-8..1e-9 (R55).
+  // 32 iterations without a 1 % improvement below 1e-6 ends the loop there.
+  if (t == 0 || dl < 0.99 * st->best_delta) {
+    st->best_delta = dl;
+    st->stall = 0;
+  } else {
+    st->stall++;
+  }
   if (dl < tol) st->stop = 1;
+  else if (st->stall >= 32 && st->best_delta < 1e-6) st->stop = 3;
   else if ((int)(t + 1) >= max_iters) st->stop = 2;
 }
 
@@ -406,7 +423,7 @@ static void run_pagerank_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& in
   cudaEventDestroy(e0);
   cudaEventDestroy(e1);
   info.iterations = (int32_t)h.iter;
-  info.converged = h.stop == 1;
+  info.converged = h.stop == 1 ? 1 : (h.stop == 3 ? 2 : 0);   // 2 = fp32 noise floor (R55)
   info.loop_ms = ms;
   info.last_delta = h.last_delta;
   info.edges_scanned = (int64_t)h.iter * d.m_slots;
@@ -455,6 +472,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   a.base = (1.0 - o.damping) / (double)g->n;
   a.invN = 1.0 / (double)g->n;
   a.st = r.pst.as<PrState>();
+  a.merge_bcast = g->knobs.merge_op == GX_MERGE_MIN ? 1 : 0;
   const bool slots = !d.identity;
   {
     const bool sim = c->world == 1 && o.sim_ranks > 1;
@@ -549,7 +567,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   cudaEventDestroy(e0);
   cudaEventDestroy(e1);
   info.iterations = (int32_t)h.iter;
-  info.converged = h.stop == 1;
+  info.converged = h.stop == 1 ? 1 : (h.stop == 3 ? 2 : 0);   // 2 = fp32 noise floor (R55)
   info.loop_ms = ms;
   info.last_delta = h.last_delta;
   info.edges_scanned = (int64_t)h.iter * d.m_slots;

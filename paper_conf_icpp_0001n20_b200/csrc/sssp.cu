@@ -261,9 +261,17 @@ __global__ void __launch_bounds__(256) k_sssp_local(const int32_t* __restrict__ 
   if (st->stop) return;
   uint32_t* bm_next = ax.bm[(t + 1) % 3];
   const uint64_t pl = l2_evict_last();
+  const uint32_t* bm_cur = ax.bm[t % 3];
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int a = tptr[tile], nm = tptr[tile + 1] - a;
     const int ea = teptr[tile], ne = teptr[tile + 1] - ea;
+    // only tiles touched by this iteration: a member in the frontier or improved by the sweep
+    int touched = 0;
+    for (int i = threadIdx.x; i < nm; i += blockDim.x) {
+      const uint32_t v = (uint32_t)tmem[a + i];
+      touched |= (int)(((__ldcg(bm_cur + (v >> 5)) | __ldcg(bm_next + (v >> 5))) >> (v & 31)) & 1u);
+    }
+    if (!__syncthreads_or(touched)) continue;
     for (int i = threadIdx.x; i < nm; i += blockDim.x) sd[i] = ld_l2_u32(dist + tmem[a + i], pl);
     __syncthreads();
     const int iters = titers[tile];
@@ -447,10 +455,12 @@ void ensure_tpv(gx_graph* g);                                                   
 
 // Near-far bucket width: a multiple of the mean edge weight scaled down by the
 // mean degree (delta-stepping's Delta ~ w / d heuristic), at least 1.
-static unsigned sssp_delta(const DevGraph& d) {
+// (the input graph's maximum weight: added 2-hop edges must not change Delta)
+static unsigned sssp_delta(const gx_graph* g) {
+  const DevGraph& d = g->dg;
   if (d.n_slots == 0 || d.m_slots == 0) return 0u;
-  const double avg_deg = (double)d.m_slots / (double)d.n_slots;
-  const double avg_w = 0.5 * (1.0 + (double)d.max_w);
+  const double avg_deg = (double)g->m / (double)std::max<int64_t>(1, g->n);
+  const double avg_w = 0.5 * (1.0 + (double)g->max_w);
   const double delta = 8.0 * avg_w / std::max(1.0, avg_deg);
   return (unsigned)std::max(1.0, delta);
 }
@@ -651,7 +661,7 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     GX_CHECK_ARG(P <= 8, "at most 8 ranks");
     GX_CHECK_ARG(o.mapping != GX_MAP_TPV, "the partitioned path uses the LB mapping");
     ensure_heavy_chunks(g);
-    unsigned delta = sssp_delta(d);
+    unsigned delta = sssp_delta(g);
     if (const char* e = getenv("GX_SSSP_DELTA")) delta = (unsigned)std::max(0, atoi(e));
     run_sssp_dist(g, o, info, P, sim, src, delta);
     return;
@@ -698,7 +708,7 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     // near-far bucket width (LB mapping only; 0 = plain frontier Bellman-Ford)
     static SsspState init;
     std::memset(&init, 0, sizeof(init));
-    unsigned delta = mapping == GX_MAP_LB ? sssp_delta(d) : 0u;
+    unsigned delta = mapping == GX_MAP_LB ? sssp_delta(g) : 0u;
     if (const char* e = getenv("GX_SSSP_DELTA")) delta = (unsigned)std::max(0, atoi(e));
     init.delta = delta;
     init.tau = delta ? delta : INF;

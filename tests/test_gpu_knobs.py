@@ -115,3 +115,16 @@ def test_inaccuracy_reporting():
     G.run("pagerank", tol=1e-12)
     assert inaccuracy(G.download("dist"), d0)["inacc_pct"] == 0.0
     assert inaccuracy(G.download("rank"), x0)["inacc_pct"] > 0.0
+
+
+@pytest.mark.parametrize("gname", ["road48", "rmat12"])
+def test_pagerank_aware_merge_same_fixed_point(gname):
+    """Algorithm-aware merge for PR (owner broadcast, R54) reaches the same G_L
+    fixed point as the paper's mean merge (Theorem E3)."""
+    raw = GRAPHS[gname]()
+    kn = T.Knobs(coalesce=True, chunk_k=4, replicate_threshold=0.0)
+    want, _ = A.pagerank(T.transform(from_raw(raw), kn).logical(), tol=1e-14)
+    G = upload(raw)
+    G.transform(knobs_c(kn, merge_op=1))
+    r = G.run("pagerank", tol=1e-11, max_iters=5000, mapping="lb")
+    assert np.abs(G.download("rank") - want).sum() <= 1e-6
