@@ -113,12 +113,18 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
     if (lane == 0) my_edges += b - a;
   }
 
-  // light slots: compact the frontier bits of 32 words, 32 slots per round
+  // light slots: each warp compacts the frontier bits of 32 bitmap words into
+  // shared memory and relaxes them 32 slots per round.  The words of a warp
+  // are strided by the warp count (word = lo + gw + nw * j), so frontiers that
+  // cluster in id space (e.g. after the §2 BFS renumbering) still spread over
+  // all warps, while sparse random frontiers still batch up to 1024 slots.
   int32_t* sv = s_v[wib];
   const int64_t w_lo = row_lo >> 5, w_hi = min((row_hi + 31) >> 5, ax.nwords);   // ranges are 32-aligned
-  for (int64_t wb = w_lo + gw * 32; wb < w_hi; wb += nw * 32) {
-    const int64_t wi = wb + lane;
-    uint32_t word = wi < w_hi ? (__ldcg(bm_cur + wi) & ~__ldg(ax.heavy + wi)) : 0u;
+  const int64_t my_words = (w_hi - w_lo - gw + nw - 1) / nw;                       // words owned by this warp
+  for (int64_t j0 = 0; j0 < my_words; j0 += 32) {
+    const int64_t jj = j0 + lane;
+    const int64_t wi = w_lo + gw + nw * jj;
+    uint32_t word = jj < my_words ? (__ldcg(bm_cur + wi) & ~__ldg(ax.heavy + wi)) : 0u;
     const uint32_t cnt = __popc(word);
     const uint32_t incl = warp_incl_scan_u32(cnt);
     const uint32_t total = __shfl_sync(FULL, incl, 31);
@@ -132,8 +138,9 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
     __syncwarp();
     for (uint32_t base = 0; base < total; base += 32) {
       const uint32_t idx = base + lane;
+      const bool mine = idx < total;
       uint32_t start = 0, deg = 0, du = 0;
-      if (idx < total) {
+      if (mine) {
         const int32_t u = sv[idx];
         du = ld_l2_u32(dist + u, pl);
         if (du >= tau) {                               // deferred to a later bucket
