@@ -58,25 +58,21 @@ __global__ void k_max_u32(const uint32_t* __restrict__ w, int64_t m, unsigned in
   if ((threadIdx.x & 31) == 0 && mx) atomicMax(out, mx);
 }
 
-// key = (dst << 32) | src for every out-edge; src found by each row owner
-__global__ void k_csc_keys(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj, int64_t n,
-                           uint64_t* __restrict__ keys) {
-  // one warp per row: rows of any length stay coalesced
+// (dst key, src value) per out-edge, plus the in-degree histogram; one warp
+// per row keeps rows of any length coalesced
+__global__ void k_csc_pairs(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj, int64_t n,
+                            uint32_t* __restrict__ key, uint32_t* __restrict__ val, uint32_t* __restrict__ cnt) {
   int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   int lane = threadIdx.x & 31;
   int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t u = warp; u < n; u += nw) {
     uint32_t a = rp[u], b = rp[u + 1];
-    for (uint32_t e = a + lane; e < b; e += 32) keys[e] = ((uint64_t)adj[e].x << 32) | (uint64_t)u;
-  }
-}
-
-__global__ void k_csc_split(const uint64_t* __restrict__ keys, int64_t m, int32_t* __restrict__ csrc,
-                            uint32_t* __restrict__ cnt) {
-  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x) {
-    uint64_t k = keys[e];
-    csrc[e] = (int32_t)(k & 0xffffffffu);
-    atomicAdd(&cnt[k >> 32], 1u);
+    for (uint32_t e = a + lane; e < b; e += 32) {
+      const uint32_t v = adj[e].x;
+      key[e] = v;
+      val[e] = (uint32_t)u;
+      atomicAdd(&cnt[v], 1u);
+    }
   }
 }
 
@@ -128,24 +124,26 @@ static void build_csc_and_tiles(gx_graph* g) {
   d.crp.alloc(c, sizeof(uint32_t) * (n + 1));
   d.csrc.alloc(c, sizeof(int32_t) * std::max<int64_t>(m, 1));
   if (m > 0) {
-    DBuf keys, keys2, tmp;
-    keys.alloc(c, sizeof(uint64_t) * m);
-    keys2.alloc(c, sizeof(uint64_t) * m);
-    k_csc_keys<<<grid_for(c, n * 32), 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), n,
-                                                   keys.as<uint64_t>());
+    // stable LSD radix sort of 32-bit dst keys carrying the src as payload:
+    // edges enter in src order, so each CSC row comes out sorted by source
+    DBuf k0, k1, v0, v1, tmp, cnt;
+    k0.alloc(c, sizeof(uint32_t) * m);
+    k1.alloc(c, sizeof(uint32_t) * m);
+    v0.alloc(c, sizeof(uint32_t) * m);
+    v1.alloc(c, sizeof(uint32_t) * m);
+    cnt.alloc(c, sizeof(uint32_t) * (n + 1));
+    CUDA_OK(cudaMemsetAsync(cnt.p, 0, sizeof(uint32_t) * (n + 1), s));
+    k_csc_pairs<<<grid_for(c, n * 32), 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), n, k0.as<uint32_t>(),
+                                                    v0.as<uint32_t>(), cnt.as<uint32_t>());
     CUDA_OK(cudaGetLastError());
     int bits = 1;
     while ((int64_t(1) << bits) < n) bits++;
     size_t tb = 0;
-    cub::DoubleBuffer<uint64_t> db(keys.as<uint64_t>(), keys2.as<uint64_t>());
-    CUDA_OK(cub::DeviceRadixSort::SortKeys(nullptr, tb, db, (int64_t)m, 0, 32 + bits, s));
+    cub::DoubleBuffer<uint32_t> dk(k0.as<uint32_t>(), k1.as<uint32_t>()), dv(v0.as<uint32_t>(), v1.as<uint32_t>());
+    CUDA_OK(cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv, (int64_t)m, 0, bits, s));
     tmp.alloc(c, tb);
-    CUDA_OK(cub::DeviceRadixSort::SortKeys(tmp.p, tb, db, (int64_t)m, 0, 32 + bits, s));
-    DBuf cnt;
-    cnt.alloc(c, sizeof(uint32_t) * (n + 1));
-    CUDA_OK(cudaMemsetAsync(cnt.p, 0, sizeof(uint32_t) * (n + 1), s));
-    k_csc_split<<<grid_for(c, m), 256, 0, s>>>(db.Current(), m, d.csrc.as<int32_t>(), cnt.as<uint32_t>());
-    CUDA_OK(cudaGetLastError());
+    CUDA_OK(cub::DeviceRadixSort::SortPairs(tmp.p, tb, dk, dv, (int64_t)m, 0, bits, s));
+    CUDA_OK(cudaMemcpyAsync(d.csrc.p, dv.Current(), sizeof(uint32_t) * m, cudaMemcpyDeviceToDevice, s));
     size_t sb = 0;
     CUDA_OK(cub::DeviceScan::ExclusiveSum(nullptr, sb, cnt.as<uint32_t>(), d.crp.as<uint32_t>(), n + 1, s));
     DBuf t2;
