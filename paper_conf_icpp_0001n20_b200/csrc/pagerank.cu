@@ -232,6 +232,92 @@ __global__ void __launch_bounds__(256) k_pr_tpv(PrArgs a) {
   }
 }
 
+// §3 shared-memory pass for PR (P@32188-32416; SURVEY A7 "PR store"): after
+// the sweep, each subgraph tile iterates its members t times in shared
+// memory, x_v <- (1-d)/N + d (ext_v + sum_{u in S, u->v} x_u / D_u + dang/N),
+// where ext_v = y_v - sum_{u in S, u->v} contrib_u is the inflow from outside
+// the tile (y_v recovered from the sweep's x_v).  Members that are replicated
+// or not owners keep their sweep values and act as external sources.  The
+// fixed point is unchanged (Theorem E3); delta grows by |x_loc - x_sweep|
+// (an upper bound of the true change), dangling mass by the exact change.
+template <bool SLOTS>
+__global__ void __launch_bounds__(256) k_pr_local(PrArgs a, const int32_t* __restrict__ tptr,
+                                                  const int32_t* __restrict__ tmem, const int32_t* __restrict__ teptr,
+                                                  const uint2* __restrict__ tedges, const int32_t* __restrict__ titers,
+                                                  int64_t ntiles) {
+  __shared__ double xs[256], xn[256], ext[256];
+  __shared__ uint32_t Ds[256];
+  __shared__ uint8_t fixed[256];
+  __shared__ double s_red[32];
+  PrState* st = a.st;
+  if (st->stop) return;
+  const unsigned t = st->iter;
+  const float* __restrict__ cin = a.contrib[t & 1];
+  float* cout = a.contrib[(t + 1) & 1];
+  const double addc = a.base + a.damp * st->dang[t % 3] * a.invN;
+  double my_delta = 0, my_dang = 0;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int b0 = tptr[tile], nm = tptr[tile + 1] - b0;
+    const int e0 = teptr[tile], ne = teptr[tile + 1] - e0;
+    for (int i = threadIdx.x; i < nm; i += blockDim.x) {
+      const int32_t v = tmem[b0 + i];
+      bool fx = SLOTS && (a.kind[v] != OWNER || (a.gid && a.gid[v] >= 0));
+      fixed[i] = fx;
+      xs[i] = a.x[v];
+      Ds[i] = a.D[v];
+      ext[i] = fx ? 0.0 : (xs[i] - addc) / a.damp;    // y_v of the sweep
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < nm; i += blockDim.x) {
+      if (fixed[i]) continue;
+      double sub = 0.0;
+      for (int e = 0; e < ne; e++) {
+        const uint2 p = tedges[e0 + e];
+        const int s = p.x & 0xff, d = (p.x >> 8) & 0xff;
+        if (d == i && !fixed[s]) sub += (double)cin[tmem[b0 + s]];
+      }
+      ext[i] -= sub;
+    }
+    __syncthreads();
+    const int iters = titers[tile];
+    for (int r = 0; r < iters; r++) {
+      for (int i = threadIdx.x; i < nm; i += blockDim.x) {
+        if (fixed[i]) {
+          xn[i] = xs[i];
+          continue;
+        }
+        double in = ext[i];
+        for (int e = 0; e < ne; e++) {
+          const uint2 p = tedges[e0 + e];
+          const int s = p.x & 0xff, d = (p.x >> 8) & 0xff;
+          if (d == i && !fixed[s] && Ds[s]) in += xs[s] / (double)Ds[s];
+        }
+        xn[i] = addc + a.damp * in;
+      }
+      __syncthreads();
+      for (int i = threadIdx.x; i < nm; i += blockDim.x) xs[i] = xn[i];
+      __syncthreads();
+    }
+    for (int i = threadIdx.x; i < nm; i += blockDim.x) {
+      if (fixed[i]) continue;
+      const int32_t v = tmem[b0 + i];
+      const double old = a.x[v];
+      a.x[v] = xs[i];
+      cout[v] = Ds[i] ? (float)(xs[i] / (double)Ds[i]) : 0.0f;
+      my_delta += fabs(xs[i] - old);
+      if (!Ds[i]) my_dang += xs[i] - old;
+    }
+    __syncthreads();
+  }
+  double dsum = block_sum_f64(my_delta, s_red);
+  __syncthreads();
+  double gsum = block_sum_f64(my_dang, s_red);
+  if (threadIdx.x == 0) {
+    if (dsum != 0.0) atomicAdd(&st->delta[(t + 1) % 3], dsum);
+    if (gsum != 0.0) atomicAdd(&st->dang[(t + 1) % 3], gsum);
+  }
+}
+
 // §2.4 confluence: every copy <- mean(owner's new value, replicas' carried
 // values) (P@28609, mirror reading R19); next contrib for all copies.
 __global__ void k_pr_merge(PrArgs a, const int32_t* __restrict__ gptr, const int32_t* __restrict__ gslots,
@@ -528,6 +614,18 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     }
     kt.end();
     nl++;
+    if (d.n_tiles && g->knobs.smem) {
+      const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 8));
+      if (slots)
+        k_pr_local<true><<<grid_local, 256, 0, s>>>(a, d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(),
+                                                    d.t_eptr.as<int32_t>(), d.t_edges.as<uint2>(), d.t_iters.as<int32_t>(),
+                                                    d.n_tiles);
+      else
+        k_pr_local<false><<<grid_local, 256, 0, s>>>(a, d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(),
+                                                     d.t_eptr.as<int32_t>(), d.t_edges.as<uint2>(),
+                                                     d.t_iters.as<int32_t>(), d.n_tiles);
+      nl++;
+    }
     if (d.n_groups) {
       k_pr_merge<<<grid_merge, 256, 0, s>>>(a, d.gptr.as<int32_t>(), d.gslots.as<int32_t>(), d.n_groups);
       nl++;
