@@ -20,6 +20,7 @@
 #include <algorithm>
 #include <chrono>
 #include <cmath>
+#include <cstdio>
 
 #include "gx_internal.h"
 #include "kernels_common.cuh"
@@ -50,6 +51,24 @@ __device__ __forceinline__ void relax_red(uint2 ed, uint32_t du, uint32_t cur, u
   }
 }
 
+// near-far relaxation: a head whose new distance is below tau joins the next
+// frontier, otherwise the far pile (far_min tracks its smallest distance)
+__device__ __forceinline__ void relax_nf(uint2 ed, uint32_t du, uint32_t cur, uint32_t* __restrict__ dist,
+                                         uint32_t* __restrict__ bm_next, uint32_t* __restrict__ far, uint32_t tau,
+                                         uint32_t& far_min, uint64_t pl) {
+  uint32_t nd = du + ed.y;
+  if (nd < du) nd = INF - 1;
+  if (nd < cur) {
+    red_min_l2(dist + ed.x, nd, pl);
+    if (nd < tau) {
+      red_or_l2(bm_next + (ed.x >> 5), 1u << (ed.x & 31), pl);
+    } else {
+      red_or_l2(far + (ed.x >> 5), 1u << (ed.x & 31), pl);
+      far_min = min(far_min, nd);
+    }
+  }
+}
+
 __device__ __forceinline__ void clear_bitmap(uint32_t* bm, int64_t nwords) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nwords; i += (int64_t)gridDim.x * blockDim.x)
     bm[i] = 0u;
@@ -73,8 +92,9 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
   const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
   const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const uint32_t tau = st->tau;   // near-far: frontier slots with dist >= tau wait
-  unsigned long long my_edges = 0, my_act = 0, my_def = 0;
+  const uint32_t tau = st->tau;   // near-far: relaxations to dist >= tau go to the far pile
+  if (blockIdx.x == 0 && threadIdx.x == 0) st->split = 0;   // the split kernel of t-1 is done
+  unsigned long long my_edges = 0, my_act = 0;
   uint32_t my_min = INF;
 
   // heavy slots: static 1024-edge chunks of rows with out-degree > HEAVY_DEG
@@ -85,14 +105,6 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
     const uint32_t a = ax.hc_start[c];
     const uint32_t b = min(a + HCHUNK, rp[u + 1]);
     const uint32_t du = ld_l2_u32(dist + u, pl);
-    if (du >= tau) {                                   // deferred to a later bucket
-      if (a == rp[u] && lane == 0) {
-        red_or_l2(bm_next + (u >> 5), 1u << (u & 31), pl);
-        my_def++;
-        my_min = min(my_min, du);
-      }
-      continue;
-    }
     if (a == rp[u] && lane == 0) my_act++;
     for (uint32_t e0 = a; e0 < b; e0 += 32 * SU) {
       uint2 ed[SU];
@@ -108,7 +120,7 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
       for (int q = 0; q < SU; q++) cv[q] = ok[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
 #pragma unroll
       for (int q = 0; q < SU; q++)
-        if (ok[q]) relax_red(ed[q], du, cv[q], dist, bm_next, pl);
+        if (ok[q]) relax_nf(ed[q], du, cv[q], dist, bm_next, ax.far, tau, my_min, pl);
     }
     if (lane == 0) my_edges += b - a;
   }
@@ -143,15 +155,9 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
       if (mine) {
         const int32_t u = sv[idx];
         du = ld_l2_u32(dist + u, pl);
-        if (du >= tau) {                               // deferred to a later bucket
-          red_or_l2(bm_next + (u >> 5), 1u << (u & 31), pl);
-          my_def++;
-          my_min = min(my_min, du);
-        } else {
-          start = rp[u];
-          deg = rp[u + 1] - start;
-          my_act++;
-        }
+        start = rp[u];
+        deg = rp[u + 1] - start;
+        my_act++;
       }
       const uint32_t dincl = warp_incl_scan_u32(deg);
       const uint32_t dexcl = dincl - deg;
@@ -180,7 +186,7 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
         for (int q = 0; q < SU; q++) cv[q] = ok[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
 #pragma unroll
         for (int q = 0; q < SU; q++)
-          if (ok[q]) relax_red(ed[q], od[q], cv[q], dist, bm_next, pl);
+          if (ok[q]) relax_nf(ed[q], od[q], cv[q], dist, bm_next, ax.far, tau, my_min, pl);
       }
       if (lane == 0) my_edges += dtot;
     }
@@ -189,14 +195,11 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
   unsigned long long e = block_sum_u64(my_edges, sh);
   __syncthreads();
   unsigned long long a2 = block_sum_u64(my_act, sh);
-  __syncthreads();
-  unsigned long long d2 = block_sum_u64(my_def, sh);
   my_min = warp_min_u32(my_min);
-  if (lane == 0 && my_min != INF) atomicMin(&st->mindef[t % 3], my_min);
+  if (lane == 0 && my_min != INF) atomicMin(&st->far_min, my_min);
   if (threadIdx.x == 0) {
     if (e) atomicAdd(&st->edges, e);
     if (a2) atomicAdd(&st->active[t % 3], (unsigned)a2);
-    if (d2) atomicAdd(&st->deferred[t % 3], (unsigned)d2);
   }
 }
 
@@ -369,22 +372,52 @@ __global__ void __launch_bounds__(256) k_sssp_merge(const int32_t* __restrict__ 
 __global__ void k_sssp_advance(SsspState* __restrict__ st, int max_iters) {
   if (st->stop) return;
   const unsigned t = st->iter;
-  const unsigned act = st->active[t % 3], def = st->deferred[t % 3];
+  const unsigned act = st->active[t % 3];
   st->act_total += act;
   st->active[(t + 2) % 3] = 0;
-  st->deferred[(t + 2) % 3] = 0;
-  st->mindef[(t + 2) % 3] = INF;
-  if (act == 0 && def == 0) {
-    st->stop = 1;
-    return;
-  }
   if (act == 0) {
-    // the current bucket drained: move the threshold past the nearest waiting slot
-    const unsigned long long nt = (unsigned long long)st->mindef[t % 3] + st->delta;
+    if (st->far_min == INF) {   // near frontier and far pile both empty
+      st->stop = 1;
+      return;
+    }
+    // the bucket drained: raise the threshold past the nearest far slot and
+    // let k_sssp_split move the far slots below it into the next frontier
+    const unsigned long long nt = (unsigned long long)st->far_min + st->delta;
     st->tau = nt >= INF ? INF : (unsigned)nt;
+    st->far_min = INF;
+    st->split = 1;
   }
   st->iter = t + 1;
   if ((int)(t + 1) >= max_iters) st->stop = 2;
+}
+
+// near-far refill (after k_sssp_advance raised tau): far slots of this rank's
+// range with dist < tau join the frontier of the new iteration; the rest stay
+// and re-establish far_min
+__global__ void k_sssp_split(const uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st, int64_t lo,
+                             int64_t hi) {
+  if (st->stop || !st->split) return;
+  const uint32_t tau = st->tau;
+  uint32_t* bm_cur = ax.bm[st->iter % 3];
+  uint32_t my_min = INF;
+  const int64_t w_lo = lo >> 5, w_hi = min((hi + 31) >> 5, ax.nwords);
+  for (int64_t w = w_lo + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < w_hi; w += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t bits = ax.far[w];
+    if (!bits) continue;
+    uint32_t move = 0, keep = bits;
+    while (bits) {
+      const int b = __ffs(bits) - 1;
+      bits &= bits - 1;
+      const uint32_t d = dist[w * 32 + b];
+      if (d < tau) move |= 1u << b;
+      else my_min = min(my_min, d);
+    }
+    keep &= ~move;
+    ax.far[w] = keep;
+    if (move) bm_cur[w] |= move;
+  }
+  my_min = warp_min_u32(my_min);
+  if (lane_id() == 0 && my_min != INF) atomicMin(&st->far_min, my_min);
 }
 
 __global__ void k_sssp_init(uint32_t* __restrict__ dist, const int32_t* __restrict__ slots, int nslots,
@@ -502,20 +535,34 @@ static void ensure_heavy_chunks(gx_graph* g) {
 }
 
 // owned slots whose distance dropped in this iteration (any rank's relaxation,
-// visible after the allreduce) join this rank's next frontier
+// visible after the allreduce) join this rank's next frontier, or its far
+// pile when the new distance is at or above the near-far threshold
 __global__ void k_frontier_diff(const uint32_t* __restrict__ dist, const uint32_t* __restrict__ dold, SsspAux ax,
-                                const SsspState* __restrict__ st, int64_t lo, int64_t hi) {
+                                SsspState* __restrict__ st, int64_t lo, int64_t hi) {
   if (st->stop) return;
   uint32_t* bm_next = ax.bm[(st->iter + 1) % 3];
+  const uint32_t tau = st->tau;
+  uint32_t my_min = INF;
   const int64_t w_lo = lo >> 5, w_hi = min((hi + 31) >> 5, ax.nwords);
   for (int64_t w = w_lo + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < w_hi; w += (int64_t)gridDim.x * blockDim.x) {
-    uint32_t bits = 0;
+    uint32_t near = 0, far = 0;
     for (int b = 0; b < 32; b++) {
       const int64_t v = w * 32 + b;
-      if (v >= lo && v < hi && dist[v] < dold[v]) bits |= 1u << b;
+      if (v < lo || v >= hi) continue;
+      const uint32_t nd = dist[v];
+      if (nd >= dold[v]) continue;
+      if (nd < tau) {
+        near |= 1u << b;
+      } else {
+        far |= 1u << b;
+        my_min = min(my_min, nd);
+      }
     }
-    if (bits) bm_next[w] |= bits;
+    if (near) bm_next[w] |= near;
+    if (far) ax.far[w] |= far;
   }
+  my_min = warp_min_u32(my_min);
+  if (lane_id() == 0 && my_min != INF) atomicMin(&st->far_min, my_min);
 }
 
 struct SsspRank {
@@ -549,7 +596,7 @@ static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, 
   std::memset(&init, 0, sizeof(init));
   init.delta = delta;
   init.tau = delta ? delta : INF;
-  for (int i = 0; i < 3; i++) init.mindef[i] = INF;
+  init.far_min = INF;
   cudaEvent_t e0, e1;
   CUDA_OK(cudaEventCreate(&e0));
   CUDA_OK(cudaEventCreate(&e1));
@@ -560,10 +607,11 @@ static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, 
     DBuf& mark = p == 0 ? r.mark : K.mark;
     DBuf& st = p == 0 ? r.st : K.st;
     dist.alloc(c, sizeof(uint32_t) * ns);
-    mark.alloc(c, sizeof(uint32_t) * 3 * nwords);
+    mark.alloc(c, sizeof(uint32_t) * 4 * nwords);
     st.alloc(c, sizeof(SsspState));
     K.dold.alloc(c, sizeof(uint32_t) * ns);
     for (int i = 0; i < 3; i++) K.ax.bm[i] = mark.as<uint32_t>() + i * nwords;
+    K.ax.far = mark.as<uint32_t>() + 3 * nwords;
     K.ax.heavy = d.heavy_bm.as<uint32_t>();
     K.ax.nwords = nwords;
     K.ax.hc_row = d.hc_row.as<int32_t>();
@@ -573,7 +621,7 @@ static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, 
     K.lo = bounds[rank];
     K.hi = bounds[rank + 1];
     CUDA_OK(cudaMemsetAsync(dist.p, 0xFF, sizeof(uint32_t) * ns, s));
-    CUDA_OK(cudaMemsetAsync(mark.p, 0, sizeof(uint32_t) * 3 * nwords, s));
+    CUDA_OK(cudaMemsetAsync(mark.p, 0, sizeof(uint32_t) * 4 * nwords, s));
     CUDA_OK(cudaMemcpyAsync(st.p, &init, sizeof(SsspState), cudaMemcpyHostToDevice, s));
     k_sssp_init<<<1, 32, 0, s>>>(dist.as<uint32_t>(), dsrc.as<int32_t>(), (int)srcs.size(), K.ax.bm[0]);
   }
@@ -591,12 +639,11 @@ static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, 
   const bool merge_min = g->knobs.merge_op == GX_MERGE_MIN;
   int launches = 0;
   SsspState hst;
-  std::vector<uint32_t*> dl, al, fl, ml;
+  std::vector<uint32_t*> dl, al, fl;
   for (int p = 0; p < nloc; p++) {
     dl.push_back(D(p));
     al.push_back(&S(p)->active[0]);
-    fl.push_back(&S(p)->deferred[0]);
-    ml.push_back(&S(p)->mindef[0]);
+    fl.push_back(&S(p)->far_min);
   }
   for (;;) {
     for (int p = 0; p < nloc; p++) {
@@ -622,9 +669,12 @@ static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, 
       launches++;
     }
     X.sum_u32(al, 3);
-    X.sum_u32(fl, 3);
-    X.min_u32(ml, 3);
-    for (int p = 0; p < nloc; p++) k_sssp_advance<<<1, 1, 0, s>>>(S(p), o.max_iters), launches++;
+    X.min_u32(fl, 1);                                   // every rank takes the same bucket decision
+    for (int p = 0; p < nloc; p++) {
+      k_sssp_advance<<<1, 1, 0, s>>>(S(p), o.max_iters);
+      k_sssp_split<<<grid_for(c, nwords), 256, 0, s>>>(D(p), R[p].ax, S(p), R[p].lo, R[p].hi);
+      launches += 2;
+    }
     CUDA_OK(cudaMemcpyAsync(&hst, S(0), sizeof(SsspState), cudaMemcpyDeviceToHost, s));
     CUDA_OK(cudaStreamSynchronize(s));
     if (hst.stop) break;
@@ -681,11 +731,12 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   const int64_t ns = d.n_slots;
   const int64_t nwords = (ns + 31) / 32;
   r.dist.alloc(c, sizeof(uint32_t) * ns);
-  r.mark.alloc(c, sizeof(uint32_t) * 3 * nwords);   // frontier bitmaps bm[0..2]
+  r.mark.alloc(c, sizeof(uint32_t) * 4 * nwords);   // frontier bitmaps bm[0..2] + far pile
   r.st.alloc(c, sizeof(SsspState));
   SsspState* st = r.st.as<SsspState>();
   SsspAux ax;
   for (int i = 0; i < 3; i++) ax.bm[i] = r.mark.as<uint32_t>() + i * nwords;
+  ax.far = r.mark.as<uint32_t>() + 3 * nwords;
   ax.heavy = d.heavy_bm.as<uint32_t>();
   ax.nwords = nwords;
   ax.hc_row = d.hc_row.as<int32_t>();
@@ -710,7 +761,7 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   CUDA_OK(cudaEventCreate(&e1));
   CUDA_OK(cudaEventRecord(e0, s));
   CUDA_OK(cudaMemsetAsync(r.dist.p, 0xFF, sizeof(uint32_t) * ns, s));
-  CUDA_OK(cudaMemsetAsync(r.mark.p, 0, sizeof(uint32_t) * 3 * nwords, s));
+  CUDA_OK(cudaMemsetAsync(r.mark.p, 0, sizeof(uint32_t) * 4 * nwords, s));
   {
     // near-far bucket width (LB mapping only; 0 = plain frontier Bellman-Ford)
     static SsspState init;
@@ -719,7 +770,7 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     if (const char* e = getenv("GX_SSSP_DELTA")) delta = (unsigned)std::max(0, atoi(e));
     init.delta = delta;
     init.tau = delta ? delta : INF;
-    for (int i = 0; i < 3; i++) init.mindef[i] = INF;
+    init.far_min = INF;
     CUDA_OK(cudaMemcpyAsync(r.st.p, &init, sizeof(SsspState), cudaMemcpyHostToDevice, s));
   }
   k_sssp_init<<<1, 32, 0, s>>>(r.dist.as<uint32_t>(), dsrc.as<int32_t>(), (int)srcs.size(), ax.bm[0]);
@@ -735,6 +786,7 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 8));
   const int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 7) / 8, (int64_t)c->num_sms * 8));
   const bool merge_min = g->knobs.merge_op == GX_MERGE_MIN;
+  const int grid_split = grid_for(c, nwords);
 
   KTimer kt(o.profile != 0, s);
   auto one_iter = [&](int& nl) {
@@ -763,6 +815,10 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     }
     k_sssp_advance<<<1, 1, 0, s>>>(st, o.max_iters);
     nl++;
+    if (mapping == GX_MAP_LB) {
+      k_sssp_split<<<grid_split, 256, 0, s>>>(r.dist.as<uint32_t>(), ax, st, 0, ns);
+      nl++;
+    }
   };
 
   const int batch = std::max(1, o.check_every);
@@ -777,10 +833,21 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     CUDA_OK(cudaGraphDestroy(graph));
   }
   SsspState hst;
+  // GX_SSSP_TRACE (profile runs): one stderr line per iteration --
+  // iteration, frontier size, cumulative edges, tau, far_min, sweep-kernel ms
+  const bool trace = o.profile && getenv("GX_SSSP_TRACE");
   while (true) {
     if (gexec) {
       CUDA_OK(cudaGraphLaunch(gexec, s));
       launches += per_batch_launches;
+    } else if (trace) {
+      one_iter(launches);
+      CUDA_OK(cudaMemcpyAsync(&hst, st, sizeof(SsspState), cudaMemcpyDeviceToHost, s));
+      CUDA_OK(cudaStreamSynchronize(s));
+      float kms = 0;
+      cudaEventElapsedTime(&kms, kt.ev[kt.ev.size() - 2], kt.ev.back());
+      fprintf(stderr, "sssp-trace t=%u act=%u edges=%llu tau=%u far_min=%u split=%u sweep_ms=%.4f\n", hst.iter - 1,
+              hst.active[(hst.iter - 1) % 3], hst.edges, hst.tau, hst.far_min, hst.split, kms);
     } else {
       for (int i = 0; i < batch; i++) one_iter(launches);
     }

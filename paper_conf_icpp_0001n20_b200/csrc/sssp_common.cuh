@@ -14,10 +14,12 @@ struct SsspState {
   unsigned int iter;            // current iteration t
   unsigned int stop;            // 0 running, 1 converged (empty frontier), 2 max_iters
   unsigned int active[3];       // frontier slots processed in iteration t
-  unsigned int deferred[3];     // frontier slots with dist >= tau carried to t+1 (near-far)
-  unsigned int mindef[3];       // smallest deferred distance
-  unsigned int tau;             // near-far threshold: only dist < tau is relaxed
+  unsigned int deferred[3];     // (unused, kept for layout)
+  unsigned int mindef[3];       // (unused, kept for layout)
+  unsigned int tau;             // near-far threshold: relaxations to dist >= tau go to the far pile
   unsigned int delta;           // bucket width (0 = plain Bellman-Ford frontier)
+  unsigned int far_min;         // upper bound of the smallest distance in the far pile (INF = empty)
+  unsigned int split;           // 1: the near frontier drained, refill it from the far pile
   unsigned int raised;          // merges that raised a copy (diagnostic)
   unsigned long long edges;     // edges relaxed, all iterations
   unsigned long long act_total; // frontier entries, all iterations
@@ -25,6 +27,7 @@ struct SsspState {
 
 struct SsspAux {
   uint32_t* bm[3];              // frontier bitmaps
+  uint32_t* far;                // near-far: slots waiting for a later bucket
   const uint32_t* heavy;        // bitmap: out-degree > HEAVY_DEG
   int64_t nwords;
   const int32_t* hc_row;        // static heavy chunk list: row
