@@ -92,10 +92,16 @@ __device__ __forceinline__ void pr_finalize(const PrArgs& a, int64_t v, double y
 #define GX_PR_CTA 256
 #endif
 constexpr int PR_CTA = GX_PR_CTA;
-constexpr int PR_U = 8;   // gathers in flight per lane
+#ifndef GX_PR_U
+#define GX_PR_U 8
+#endif
+#ifndef GX_PR_MINB
+#define GX_PR_MINB 1
+#endif
+constexpr int PR_U = GX_PR_U;   // gathers in flight per lane
 
 template <bool SLOTS>
-__global__ void __launch_bounds__(PR_CTA) k_pr_sell(PrArgs a) {
+__global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell(PrArgs a) {
   __shared__ double s_y[PRW];
   __shared__ double s_red[32];
   PrState* st = a.st;
