@@ -42,12 +42,13 @@ __device__ __forceinline__ bool bit_of(const uint32_t* __restrict__ bm, uint32_t
 // relax one edge given the (possibly stale, never smaller within a sweep)
 // distance `cur` of its head
 __device__ __forceinline__ void relax_red(uint2 ed, uint32_t du, uint32_t cur, uint32_t* __restrict__ dist,
-                                          uint32_t* __restrict__ bm_next, uint64_t pl) {
+                                          uint32_t* __restrict__ bm_next, uint32_t& npush, uint64_t pl) {
   uint32_t nd = du + ed.y;
   if (nd < du) nd = INF - 1;  // saturate (never the fixed point)
   if (nd < cur) {
     red_min_l2(dist + ed.x, nd, pl);
     red_or_l2(bm_next + (ed.x >> 5), 1u << (ed.x & 31), pl);
+    npush++;
   }
 }
 
@@ -55,17 +56,53 @@ __device__ __forceinline__ void relax_red(uint2 ed, uint32_t du, uint32_t cur, u
 // frontier, otherwise the far pile (far_min tracks its smallest distance)
 __device__ __forceinline__ void relax_nf(uint2 ed, uint32_t du, uint32_t cur, uint32_t* __restrict__ dist,
                                          uint32_t* __restrict__ bm_next, uint32_t* __restrict__ far, uint32_t tau,
-                                         uint32_t& far_min, uint64_t pl) {
+                                         uint32_t& far_min, uint32_t& npush, uint64_t pl) {
   uint32_t nd = du + ed.y;
   if (nd < du) nd = INF - 1;
   if (nd < cur) {
     red_min_l2(dist + ed.x, nd, pl);
     if (nd < tau) {
       red_or_l2(bm_next + (ed.x >> 5), 1u << (ed.x & 31), pl);
+      npush++;
     } else {
       red_or_l2(far + (ed.x >> 5), 1u << (ed.x & 31), pl);
       far_min = min(far_min, nd);
     }
+  }
+}
+
+// Block-level reduction of a sweep's per-thread counters: one atomic of each
+// kind per CTA (same-address atomics from every warp would serialise in L2).
+// Every thread of the CTA must call it.
+__device__ __forceinline__ void flush_counters(SsspState* st, unsigned t, unsigned long long edges,
+                                               unsigned long long act, uint32_t push, uint32_t fmin) {
+  __shared__ unsigned long long s_e[32], s_a[32];
+  __shared__ uint32_t s_p[32], s_m[32];
+  edges = warp_sum_u64(edges);
+  act = warp_sum_u64(act);
+  push = __reduce_add_sync(FULL, push);
+  fmin = warp_min_u32(fmin);
+  const unsigned w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  if (lane_id() == 0) {
+    s_e[w] = edges;
+    s_a[w] = act;
+    s_p[w] = push;
+    s_m[w] = fmin;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long e = 0, a = 0;
+    uint32_t p = 0, m = INF;
+    for (unsigned i = 0; i < nw; i++) {
+      e += s_e[i];
+      a += s_a[i];
+      p += s_p[i];
+      m = min(m, s_m[i]);
+    }
+    if (e) atomicAdd(&st->edges, e);
+    if (a) atomicAdd(&st->active[t % 3], (unsigned)a);
+    if (p) atomicAdd(&st->pushed[t % 3], p);
+    if (m != INF) atomicMin(&st->far_min, m);
   }
 }
 
@@ -82,7 +119,6 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
                                                  uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st,
                                                  int64_t row_lo, int64_t row_hi) {
   __shared__ int32_t s_v[SB_WARPS][1024];
-  __shared__ unsigned long long sh[32];
   const unsigned t = st->iter;
   if (st->stop) return;
   const uint32_t* __restrict__ bm_cur = ax.bm[t % 3];
@@ -95,7 +131,7 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
   const uint32_t tau = st->tau;   // near-far: relaxations to dist >= tau go to the far pile
   if (blockIdx.x == 0 && threadIdx.x == 0) st->split = 0;   // the split kernel of t-1 is done
   unsigned long long my_edges = 0, my_act = 0;
-  uint32_t my_min = INF;
+  uint32_t my_min = INF, my_push = 0;
 
   // heavy slots: static 1024-edge chunks of rows with out-degree > HEAVY_DEG
   for (int64_t c = gw; c < ax.nhc; c += nw) {
@@ -120,7 +156,7 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
       for (int q = 0; q < SU; q++) cv[q] = ok[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
 #pragma unroll
       for (int q = 0; q < SU; q++)
-        if (ok[q]) relax_nf(ed[q], du, cv[q], dist, bm_next, ax.far, tau, my_min, pl);
+        if (ok[q]) relax_nf(ed[q], du, cv[q], dist, bm_next, ax.far, tau, my_min, my_push, pl);
     }
     if (lane == 0) my_edges += b - a;
   }
@@ -186,21 +222,13 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
         for (int q = 0; q < SU; q++) cv[q] = ok[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
 #pragma unroll
         for (int q = 0; q < SU; q++)
-          if (ok[q]) relax_nf(ed[q], od[q], cv[q], dist, bm_next, ax.far, tau, my_min, pl);
+          if (ok[q]) relax_nf(ed[q], od[q], cv[q], dist, bm_next, ax.far, tau, my_min, my_push, pl);
       }
       if (lane == 0) my_edges += dtot;
     }
     __syncwarp();
   }
-  unsigned long long e = block_sum_u64(my_edges, sh);
-  __syncthreads();
-  unsigned long long a2 = block_sum_u64(my_act, sh);
-  my_min = warp_min_u32(my_min);
-  if (lane == 0 && my_min != INF) atomicMin(&st->far_min, my_min);
-  if (threadIdx.x == 0) {
-    if (e) atomicAdd(&st->edges, e);
-    if (a2) atomicAdd(&st->active[t % 3], (unsigned)a2);
-  }
+  flush_counters(st, t, my_edges, my_act, my_push, my_min);
 }
 
 // ---------------------------------------------------------------- TPV sweep
@@ -212,7 +240,6 @@ __global__ void __launch_bounds__(256) k_sssp_tpv(const int32_t* __restrict__ la
                                                   const uint64_t* __restrict__ soff, const uint2* __restrict__ slab,
                                                   int64_t nslices, uint32_t* __restrict__ dist, SsspAux ax,
                                                   SsspState* __restrict__ st) {
-  __shared__ unsigned long long sh[32];
   const unsigned t = st->iter;
   if (st->stop) return;
   const uint32_t* __restrict__ bm_cur = ax.bm[t % 3];
@@ -223,6 +250,7 @@ __global__ void __launch_bounds__(256) k_sssp_tpv(const int32_t* __restrict__ la
   const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   unsigned long long my_edges = 0, my_act = 0;
+  uint32_t my_push = 0;
   for (int64_t sl = gw; sl < nslices; sl += nw) {
     const int32_t row = lane_row[sl * 32 + lane];
     const bool act = row >= 0 && bit_of(bm_cur, (uint32_t)row);
@@ -244,18 +272,12 @@ __global__ void __launch_bounds__(256) k_sssp_tpv(const int32_t* __restrict__ la
       for (int q = 0; q < SU; q++) cv[q] = ok[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
 #pragma unroll
       for (int q = 0; q < SU; q++) {
-        if (ok[q]) relax_red(ed[q], du, cv[q], dist, bm_next, pl);
+        if (ok[q]) relax_red(ed[q], du, cv[q], dist, bm_next, my_push, pl);
         my_edges += ok[q];
       }
     }
   }
-  unsigned long long e = block_sum_u64(my_edges, sh);
-  __syncthreads();
-  unsigned long long a2 = block_sum_u64(my_act, sh);
-  if (threadIdx.x == 0) {
-    if (e) atomicAdd(&st->edges, e);
-    if (a2) atomicAdd(&st->active[t % 3], (unsigned)a2);
-  }
+  flush_counters(st, t, my_edges, my_act, my_push, INF);
 }
 
 // ---------------------------------------------------------------- §3 local pass
@@ -272,6 +294,7 @@ __global__ void __launch_bounds__(256) k_sssp_local(const int32_t* __restrict__ 
   uint32_t* bm_next = ax.bm[(t + 1) % 3];
   const uint64_t pl = l2_evict_last();
   const uint32_t* bm_cur = ax.bm[t % 3];
+  uint32_t my_push = 0;
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int a = tptr[tile], nm = tptr[tile + 1] - a;
     const int ea = teptr[tile], ne = teptr[tile + 1] - ea;
@@ -308,10 +331,12 @@ __global__ void __launch_bounds__(256) k_sssp_local(const int32_t* __restrict__ 
       if (nd < ld_l2_u32(dist + v, pl)) {
         red_min_l2(dist + v, nd, pl);
         red_or_l2(bm_next + (v >> 5), 1u << (v & 31), pl);
+        my_push++;
       }
     }
     __syncthreads();
   }
+  flush_counters(st, t, 0, 0, my_push, INF);
 }
 
 // ---------------------------------------------------------------- §2.4 merge
@@ -330,6 +355,7 @@ __global__ void __launch_bounds__(256) k_sssp_merge(const int32_t* __restrict__ 
   const unsigned lane = lane_id();
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  uint32_t my_push = 0;
   for (int64_t gi = warp; gi < ngroups; gi += nw) {
     const int a = gptr[gi], b = gptr[gi + 1];
     const int32_t o = gslots[a];
@@ -361,23 +387,30 @@ __global__ void __launch_bounds__(256) k_sssp_merge(const int32_t* __restrict__ 
       const uint32_t old = __ldcg(dist + sl);
       if (old != mval) {
         dist[sl] = mval;
-        if (mval < old) atomicOr(bm_next + (sl >> 5), 1u << (sl & 31));
-        else atomicAdd(&st->raised, 1u);
+        if (mval < old) {
+          atomicOr(bm_next + (sl >> 5), 1u << (sl & 31));
+          my_push++;
+        } else {
+          atomicAdd(&st->raised, 1u);
+        }
       }
     }
   }
+  flush_counters(st, t, 0, 0, my_push, INF);
 }
 
-// end of iteration t: the frontier of t was empty => converged
+// end of iteration t: no bit was set in the next frontier and the far pile is
+// empty => converged (every decreased slot has been relaxed)
 __global__ void k_sssp_advance(SsspState* __restrict__ st, int max_iters) {
   if (st->stop) return;
   const unsigned t = st->iter;
-  const unsigned act = st->active[t % 3];
-  st->act_total += act;
+  st->act_total += st->active[t % 3];
   st->active[(t + 2) % 3] = 0;
-  if (act == 0) {
-    if (st->far_min == INF) {   // near frontier and far pile both empty
+  st->pushed[(t + 2) % 3] = 0;
+  if (st->pushed[t % 3] == 0) {  // the next frontier is empty
+    if (st->far_min == INF) {    // ... and so is the far pile
       st->stop = 1;
+      st->iter = t + 1;
       return;
     }
     // the bucket drained: raise the threshold past the nearest far slot and
@@ -416,8 +449,7 @@ __global__ void k_sssp_split(const uint32_t* __restrict__ dist, SsspAux ax, Sssp
     ax.far[w] = keep;
     if (move) bm_cur[w] |= move;
   }
-  my_min = warp_min_u32(my_min);
-  if (lane_id() == 0 && my_min != INF) atomicMin(&st->far_min, my_min);
+  flush_counters(st, 0, 0, 0, 0, my_min);
 }
 
 __global__ void k_sssp_init(uint32_t* __restrict__ dist, const int32_t* __restrict__ slots, int nslots,
@@ -542,7 +574,7 @@ __global__ void k_frontier_diff(const uint32_t* __restrict__ dist, const uint32_
   if (st->stop) return;
   uint32_t* bm_next = ax.bm[(st->iter + 1) % 3];
   const uint32_t tau = st->tau;
-  uint32_t my_min = INF;
+  uint32_t my_min = INF, my_push = 0;
   const int64_t w_lo = lo >> 5, w_hi = min((hi + 31) >> 5, ax.nwords);
   for (int64_t w = w_lo + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < w_hi; w += (int64_t)gridDim.x * blockDim.x) {
     uint32_t near = 0, far = 0;
@@ -560,9 +592,9 @@ __global__ void k_frontier_diff(const uint32_t* __restrict__ dist, const uint32_
     }
     if (near) bm_next[w] |= near;
     if (far) ax.far[w] |= far;
+    my_push += __popc(near);
   }
-  my_min = warp_min_u32(my_min);
-  if (lane_id() == 0 && my_min != INF) atomicMin(&st->far_min, my_min);
+  flush_counters(st, st->iter, 0, 0, my_push, my_min);
 }
 
 struct SsspRank {
@@ -668,7 +700,7 @@ static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, 
                                                            R[p].hi);
       launches++;
     }
-    X.sum_u32(al, 3);
+    X.sum_u32(al, 6);                                   // active[3] + pushed[3]
     X.min_u32(fl, 1);                                   // every rank takes the same bucket decision
     for (int p = 0; p < nloc; p++) {
       k_sssp_advance<<<1, 1, 0, s>>>(S(p), o.max_iters);

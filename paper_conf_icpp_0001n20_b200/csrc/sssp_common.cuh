@@ -14,8 +14,8 @@ struct SsspState {
   unsigned int iter;            // current iteration t
   unsigned int stop;            // 0 running, 1 converged (empty frontier), 2 max_iters
   unsigned int active[3];       // frontier slots processed in iteration t
-  unsigned int deferred[3];     // (unused, kept for layout)
-  unsigned int mindef[3];       // (unused, kept for layout)
+  unsigned int pushed[3];       // next-frontier bits set in iteration t (0 => the next frontier is empty);
+                                // contiguous with active[] so one allreduce sums both (dist.h)
   unsigned int tau;             // near-far threshold: relaxations to dist >= tau go to the far pile
   unsigned int delta;           // bucket width (0 = plain Bellman-Ford frontier)
   unsigned int far_min;         // upper bound of the smallest distance in the far pile (INF = empty)
