@@ -133,32 +133,45 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
   unsigned long long my_edges = 0, my_act = 0;
   uint32_t my_min = INF, my_push = 0;
 
-  // heavy slots: static 1024-edge chunks of rows with out-degree > HEAVY_DEG
-  for (int64_t c = gw; c < ax.nhc; c += nw) {
-    const int32_t u = ax.hc_row[c];
-    if (u < row_lo || u >= row_hi) continue;          // another rank's rows (dist.h)
-    if (!bit_of(bm_cur, (uint32_t)u)) continue;       // warp-uniform
-    const uint32_t a = ax.hc_start[c];
-    const uint32_t b = min(a + HCHUNK, rp[u + 1]);
-    const uint32_t du = ld_l2_u32(dist + u, pl);
-    if (a == rp[u] && lane == 0) my_act++;
-    for (uint32_t e0 = a; e0 < b; e0 += 32 * SU) {
-      uint2 ed[SU];
-      bool ok[SU];
-#pragma unroll
-      for (int q = 0; q < SU; q++) {
-        uint32_t e = e0 + q * 32 + lane;
-        ok[q] = e < b;
-        ed[q] = ok[q] ? ld_stream_u2(adj + e, pf) : make_uint2(0, 0);
-      }
-      uint32_t cv[SU];
-#pragma unroll
-      for (int q = 0; q < SU; q++) cv[q] = ok[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
-#pragma unroll
-      for (int q = 0; q < SU; q++)
-        if (ok[q]) relax_nf(ed[q], du, cv[q], dist, bm_next, ax.far, tau, my_min, my_push, pl);
+  // heavy slots: static 1024-edge chunks of rows with out-degree > HEAVY_DEG.
+  // This warp owns chunks gw + nw*k; its lanes test 32 of them at once (one
+  // round of dependent loads instead of 32) and the warp relaxes the active ones.
+  const int64_t my_chunks = ax.nhc > gw ? (ax.nhc - gw + nw - 1) / nw : 0;
+  for (int64_t k0 = 0; k0 < my_chunks; k0 += 32) {
+    const int64_t kc = k0 + lane;
+    int32_t uc = -1;
+    if (kc < my_chunks) {
+      uc = ax.hc_row[gw + nw * kc];
+      if (uc < row_lo || uc >= row_hi || !bit_of(bm_cur, (uint32_t)uc)) uc = -1;   // another rank's rows (dist.h)
     }
-    if (lane == 0) my_edges += b - a;
+    unsigned todo = __ballot_sync(FULL, uc >= 0);
+    while (todo) {
+      const int l = __ffs(todo) - 1;
+      todo &= todo - 1;
+      const int64_t c = gw + nw * (k0 + l);
+      const int32_t u = __shfl_sync(FULL, uc, l);
+      const uint32_t a = ax.hc_start[c];
+      const uint32_t b = min(a + HCHUNK, rp[u + 1]);
+      const uint32_t du = ld_l2_u32(dist + u, pl);
+      if (a == rp[u] && lane == 0) my_act++;
+      for (uint32_t e0 = a; e0 < b; e0 += 32 * SU) {
+        uint2 ed[SU];
+        bool ok[SU];
+#pragma unroll
+        for (int q = 0; q < SU; q++) {
+          uint32_t e = e0 + q * 32 + lane;
+          ok[q] = e < b;
+          ed[q] = ok[q] ? ld_stream_u2(adj + e, pf) : make_uint2(0, 0);
+        }
+        uint32_t cv[SU];
+#pragma unroll
+        for (int q = 0; q < SU; q++) cv[q] = ok[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
+#pragma unroll
+        for (int q = 0; q < SU; q++)
+          if (ok[q]) relax_nf(ed[q], du, cv[q], dist, bm_next, ax.far, tau, my_min, my_push, pl);
+      }
+      if (lane == 0) my_edges += b - a;
+    }
   }
 
   // light slots: each warp compacts the frontier bits of 32 bitmap words into
