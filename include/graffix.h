@@ -138,7 +138,26 @@ typedef struct {
   int32_t sim_ranks;       /* > 1 on a single-GPU context: run the 1-D partitioned
                               path with this many simulated ranks (exchange by a
                               device reduction instead of NCCL); LB mapping only    */
+  int32_t pr_schedule;     /* PR update schedule on one GPU (SURVEY §8(c) Theorem E3:
+                              every schedule has the same fixed point x*):
+                              GX_PR_JACOBI (default) = sweep t reads only x_t (two
+                              contrib buffers, the oracle's iteration order);
+                              GX_PR_ASYNC = one contrib buffer updated in place, a
+                              row reads whichever of x_t / x_{t+1} its sources hold
+                              (asynchronous vertex-centric kernels, P@15381): half
+                              the contrib footprint, but the lagged dangling term
+                              slows convergence (RMAT-24: 52 vs 22 iterations,
+                              DESIGN.md).  The multi-GPU path is Jacobi.          */
+  int32_t merge_every;     /* §2.4 confluence cadence (P@28188-28736):
+                              1 (default) = after every iteration; c > 1 = after
+                              every c-th iteration and once more whenever the
+                              sweep alone has reached its fixed point; 0 = only
+                              then ("merge at the end").  Every cadence ends at a
+                              merged fixed point (Theorems E1/E3).                */
 } gx_run_opts;
+
+#define GX_PR_JACOBI 0
+#define GX_PR_ASYNC 1
 
 /* Transformed-graph export (debug / parity path).  Two-call protocol: call
  * gx_export_sizes, allocate host arrays of those sizes, call

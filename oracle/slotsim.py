@@ -26,9 +26,25 @@ def _merge_int(vals):
     return sum(fin) // len(fin)
 
 
+def _merge_now(it: int, merge_every: int, sweep_fixed: bool) -> bool:
+    """Merge cadence, P@28188: "The merging or the confluence may be done after
+    a certain number of iterations or at the end of the overall computation"
+    (Graffix's default: after every iteration).  merge_every = c: c == 1 every
+    iteration; c > 1 after every c-th iteration (1-based) and after any
+    iteration whose sweep changed nothing (so the run ends merged); c == 0 only
+    "at the end": after the first iteration whose sweep changed nothing."""
+    if merge_every == 1:
+        return True
+    if merge_every > 1 and it % merge_every == 0:
+        return True
+    return sweep_fixed
+
+
 def sssp_slots(tg: TransformedGraph, source: int, max_iters: int = 100000,
-               merge: str = "mean", local_pass: bool = True):
-    """Returns (dist per original vertex, iterations)."""
+               merge: str = "mean", local_pass: bool = True, merge_every: int = 1):
+    """Returns (dist per original vertex, iterations).  With merge_every == 0
+    the run ends right after its single final merge (values pushed by that
+    merge are not relaxed further)."""
     groups = tg.groups()
     dist = [INF32] * tg.n_slots
     o = int(tg.owner_slot[source])
@@ -55,21 +71,27 @@ def sssp_slots(tg: TransformedGraph, source: int, max_iters: int = 100000,
                         for (q, w, _) in tg.rows[s]:
                             if q in ms and new[s] + w < new[q]:
                                 new[q] = new[s] + w
-        for own, copies in groups.items():
-            mval = _merge_int([new[c] for c in copies]) if merge == "mean" else min(new[c] for c in copies)
-            for c in copies:
-                new[c] = mval
-        if new == dist:
+        merged = bool(groups) and _merge_now(it, merge_every, new == dist)
+        if merged:
+            for own, copies in groups.items():
+                mval = _merge_int([new[c] for c in copies]) if merge == "mean" else min(new[c] for c in copies)
+                for c in copies:
+                    new[c] = mval
+        if merge_every == 0 and merged:
+            dist = new
+            break
+        if new == dist and (merged or not groups):
             break
         dist = new
     return np.asarray([dist[int(tg.owner_slot[v])] for v in range(tg.n)], dtype=np.uint32), it
 
 
 def pagerank_slots(tg: TransformedGraph, damping: float = 0.85, tol: float = 1e-13,
-                   max_iters: int = 100000):
+                   max_iters: int = 100000, merge_every: int = 1):
     """Mirror-replica PageRank on slots: each copy divides by D (the total
     logical out-degree); replicas carry the last merged value.  Returns
-    (x per original vertex, iterations)."""
+    (x per original vertex, iterations).  Merge cadence as in _merge_now, with
+    "the sweep changed nothing" read as delta < tol."""
     N = tg.n
     groups = tg.groups()
     D = tg.divisor().astype(np.float64)
@@ -88,10 +110,15 @@ def pagerank_slots(tg: TransformedGraph, damping: float = 0.85, tol: float = 1e-
         dang = x[owners][D[owners] == 0].sum()
         xn = x.copy()
         xn[owners] = (1.0 - damping) / N + damping * (y[owners] + dang / N)
-        for own, copies in groups.items():
-            xn[copies] = xn[copies].mean()
+        sweep_fixed = np.abs(xn[owners] - x[owners]).sum() < tol
+        merged = bool(groups) and _merge_now(it, merge_every, sweep_fixed)
+        if merged:
+            for own, copies in groups.items():
+                xn[copies] = xn[copies].mean()
         delta = np.abs(xn[owners] - x[owners]).sum()
         x = xn
-        if delta < tol:
+        if merge_every == 0 and merged:
+            break
+        if delta < tol and (merged or not groups):
             break
     return x[owners], it

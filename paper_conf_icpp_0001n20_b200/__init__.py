@@ -185,7 +185,8 @@ class Graph:
 
     def run(self, algo: str = "sssp", source: int = -1, max_iters: int = 0, tol: float = 1e-9,
             mapping: str = "auto", damping: float = 0.85, check_every: int = 8, use_graphs: bool = True,
-            bc_sources=None, profile: bool = False, sim_ranks: int = 0) -> dict:
+            bc_sources=None, profile: bool = False, sim_ranks: int = 0, pr_schedule: str = "jacobi",
+            merge_every: int = 1) -> dict:
         o = GxRunOpts()
         _check(lib().gx_run_opts_default(C.byref(o)))
         o.algo = ALGOS[algo]
@@ -198,6 +199,8 @@ class Graph:
         o.use_graphs = int(bool(use_graphs))
         o.profile = int(bool(profile))
         o.sim_ranks = int(sim_ranks)
+        o.pr_schedule = {"jacobi": 0, "async": 1}[pr_schedule]
+        o.merge_every = int(merge_every)
         keep = None
         if bc_sources is not None:
             keep = np.ascontiguousarray(bc_sources, dtype=np.int64)

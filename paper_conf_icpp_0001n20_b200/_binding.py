@@ -62,7 +62,8 @@ class GxRunOpts(C.Structure):
     _fields_ = [("struct_size", C.c_uint32), ("algo", C.c_int32), ("source", C.c_int64),
                 ("max_iters", C.c_int32), ("mapping", C.c_int32), ("tol", C.c_double), ("damping", C.c_double),
                 ("check_every", C.c_int32), ("use_graphs", C.c_int32), ("bc_sources", C.c_void_p),
-                ("n_bc_sources", C.c_int64), ("profile", C.c_int32), ("sim_ranks", C.c_int32)]
+                ("n_bc_sources", C.c_int64), ("profile", C.c_int32), ("sim_ranks", C.c_int32),
+                ("pr_schedule", C.c_int32), ("merge_every", C.c_int32)]
 
 
 class GxExportSizes(C.Structure):

@@ -303,6 +303,8 @@ gx_status gx_run_opts_default(gx_run_opts* o) {
   o->damping = 0.85;
   o->check_every = 8;
   o->use_graphs = 1;
+  o->pr_schedule = GX_PR_JACOBI;
+  o->merge_every = 1;
   return GX_OK;
 }
 
@@ -434,6 +436,8 @@ gx_status gx_run_ex(gx_graph* g, const gx_run_opts* opts, gx_run_info* info) {
   if (o.max_iters <= 0) o.max_iters = 1000000;
   if (o.check_every <= 0) o.check_every = 8;
   GX_CHECK_ARG(o.mapping >= GX_MAP_AUTO && o.mapping <= GX_MAP_TPV, "mapping invalid");
+  GX_CHECK_ARG(o.pr_schedule == GX_PR_JACOBI || o.pr_schedule == GX_PR_ASYNC, "pr_schedule invalid");
+  GX_CHECK_ARG(o.merge_every >= 0, "merge_every must be >= 0");
   gx_run_info ri;
   std::memset(&ri, 0, sizeof(ri));
   switch (o.algo) {

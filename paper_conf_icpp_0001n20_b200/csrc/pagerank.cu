@@ -17,6 +17,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdlib>
+#include <cstring>
 
 #include "gx_internal.h"
 #include "kernels_common.cuh"
@@ -34,6 +35,9 @@ struct PrState {
   double last_delta;
   double best_delta; // smallest delta so far (stagnation test)
   unsigned stall;    // iterations since best_delta last improved by >= 1 %
+  unsigned merge_every;  // §2.4 cadence (gx_run_opts.merge_every)
+  unsigned do_merge;     // iteration `iter` ends with a merge (set by k_pr_advance)
+  unsigned force;        // the sweep reached its fixed point without a merge: merge next
   unsigned pad;
 };
 
@@ -68,14 +72,29 @@ struct PrArgs {
   int64_t tpv_nslices;
 };
 
+// contrib gather: read-only (.nc) in a Jacobi sweep; in the asynchronous
+// schedule the buffer is written by the same sweep, so the load goes through
+// L2 (.cg) and returns either the old or the new value of the source.
+template <bool ASYNC>
+__device__ __forceinline__ float ld_contrib(const float* p, uint64_t pol) {
+  if (ASYNC) {
+    float v;
+    asm("ld.global.cg.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
+    return v;
+  }
+  return ld_keep_f32(p, pol);
+}
+
 template <bool SLOTS>
 __device__ __forceinline__ void pr_finalize(const PrArgs& a, int64_t v, double y, double xo, uint32_t Dv, double addc,
-                                            float* cout, double& my_delta, double& my_dang) {
+                                            float* cout, double& my_delta, double& my_dang, bool merge_now) {
   if (SLOTS) {
     if (a.kind[v] != OWNER) return;  // holes stay 0; replicas are set by the merge
   }
   double xn = addc + a.damp * y;
-  if (SLOTS && a.gid) {
+  // a replicated owner hands its new value to the merge; in an iteration
+  // without a merge (cadence N2) it updates its own copy only
+  if (SLOTS && a.gid && merge_now) {
     int g = a.gid[v];
     if (g >= 0) {
       a.gnew[g] = xn;
@@ -100,16 +119,17 @@ constexpr int PR_CTA = GX_PR_CTA;
 #endif
 constexpr int PR_U = GX_PR_U;   // gathers in flight per lane
 
-template <bool SLOTS>
+template <bool SLOTS, bool ASYNC>
 __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell(PrArgs a) {
   __shared__ double s_y[PRW];
   __shared__ double s_red[32];
   PrState* st = a.st;
   if (st->stop) return;
   const unsigned t = st->iter;
-  const float* __restrict__ cin = a.contrib[t & 1];
+  const float* cin = a.contrib[t & 1];
   float* cout = a.contrib[(t + 1) & 1];
   const double addc = a.base + a.damp * st->dang[t % 3] * a.invN;
+  const bool merge_now = st->do_merge != 0;
   double my_delta = 0, my_dang = 0;
   const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
   const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
@@ -133,13 +153,13 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell(PrArgs a) {
         for (int u = 0; u < PR_U; u++) e[u] = ld_stream_u32(p + 32 * (j + u), pf);
         float v[PR_U];
 #pragma unroll
-        for (int u = 0; u < PR_U; u++) v[u] = e[u] != PR_SENT ? ld_keep_f32(cin + e[u], pl) : 0.0f;
+        for (int u = 0; u < PR_U; u++) v[u] = e[u] != PR_SENT ? ld_contrib<ASYNC>(cin + e[u], pl) : 0.0f;
 #pragma unroll
         for (int u = 0; u < PR_U; u++) acc += (double)v[u];
       }
       for (; j < L; j++) {
         uint32_t e = ld_stream_u32(p + 32 * j, pf);
-        if (e != PR_SENT) acc += (double)ld_keep_f32(cin + e, pl);
+        if (e != PR_SENT) acc += (double)ld_contrib<ASYNC>(cin + e, pl);
       }
       if (row >= 0) s_y[row - base] = acc;
     }
@@ -154,7 +174,7 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell(PrArgs a) {
 #pragma unroll
         for (int u = 0; u < 4; u++) {
           uint32_t ee = e + 32 * u;
-          v[u] = ee < e1 ? ld_keep_f32(cin + ld_stream_i32(a.csrc + ee, pf), pl) : 0.0f;
+          v[u] = ee < e1 ? ld_contrib<ASYNC>(cin + ld_stream_i32(a.csrc + ee, pf), pl) : 0.0f;
         }
 #pragma unroll
         for (int u = 0; u < 4; u++) acc += (double)v[u];
@@ -176,7 +196,7 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell(PrArgs a) {
 #pragma unroll
       for (int u = 0; u < 4; u++) {
         int i = i0 + u * PR_CTA;
-        if (i < nrows) pr_finalize<SLOTS>(a, base + i, s_y[i], xo[u], Dv[u], addc, cout, my_delta, my_dang);
+        if (i < nrows) pr_finalize<SLOTS>(a, base + i, s_y[i], xo[u], Dv[u], addc, cout, my_delta, my_dang, merge_now);
       }
     }
     __syncthreads();
@@ -193,15 +213,16 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell(PrArgs a) {
 // The paper's thread-per-vertex pull (tpv.cu): lane = slot of the schedule,
 // each lane sums its own in-edges from the SELL-32 slab and finalises its
 // slot; a warp lasts as long as its longest row (what §4 normalises).
-template <bool SLOTS>
+template <bool SLOTS, bool ASYNC>
 __global__ void __launch_bounds__(256) k_pr_tpv(PrArgs a) {
   __shared__ double s_red[32];
   PrState* st = a.st;
   if (st->stop) return;
   const unsigned t = st->iter;
-  const float* __restrict__ cin = a.contrib[t & 1];
+  const float* cin = a.contrib[t & 1];
   float* cout = a.contrib[(t + 1) & 1];
   const double addc = a.base + a.damp * st->dang[t % 3] * a.invN;
+  const bool merge_now = st->do_merge != 0;
   double my_delta = 0, my_dang = 0;
   const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
   const unsigned lane = lane_id();
@@ -219,15 +240,16 @@ __global__ void __launch_bounds__(256) k_pr_tpv(PrArgs a) {
       for (int u = 0; u < PR_U; u++) e[u] = row >= 0 ? ld_stream_u32(p + 32 * (j + u), pf) : PR_SENT;
       float v[PR_U];
 #pragma unroll
-      for (int u = 0; u < PR_U; u++) v[u] = e[u] != PR_SENT ? ld_keep_f32(cin + e[u], pl) : 0.0f;
+      for (int u = 0; u < PR_U; u++) v[u] = e[u] != PR_SENT ? ld_contrib<ASYNC>(cin + e[u], pl) : 0.0f;
 #pragma unroll
       for (int u = 0; u < PR_U; u++) acc += (double)v[u];
     }
     for (; j < L; j++) {
       uint32_t e = row >= 0 ? ld_stream_u32(p + 32 * j, pf) : PR_SENT;
-      if (e != PR_SENT) acc += (double)ld_keep_f32(cin + e, pl);
+      if (e != PR_SENT) acc += (double)ld_contrib<ASYNC>(cin + e, pl);
     }
-    if (row >= 0) pr_finalize<SLOTS>(a, row, acc, __ldcs(a.x + row), __ldcs(a.D + row), addc, cout, my_delta, my_dang);
+    if (row >= 0) pr_finalize<SLOTS>(a, row, acc, __ldcs(a.x + row), __ldcs(a.D + row), addc, cout, my_delta, my_dang,
+                                      merge_now);
   }
   double dsum = block_sum_f64(my_delta, s_red);
   __syncthreads();
@@ -258,7 +280,7 @@ __global__ void __launch_bounds__(256) k_pr_local(PrArgs a, const int32_t* __res
   PrState* st = a.st;
   if (st->stop) return;
   const unsigned t = st->iter;
-  const float* __restrict__ cin = a.contrib[t & 1];
+  const float* cin = a.contrib[t & 1];
   float* cout = a.contrib[(t + 1) & 1];
   const double addc = a.base + a.damp * st->dang[t % 3] * a.invN;
   double my_delta = 0, my_dang = 0;
@@ -333,6 +355,15 @@ __global__ void k_pr_merge(PrArgs a, const int32_t* __restrict__ gptr, const int
   if (st->stop) return;
   const unsigned t = st->iter;
   float* cout = a.contrib[(t + 1) & 1];
+  if (!st->do_merge) {
+    // iteration without a merge (cadence N2): replicas carry their values, and
+    // under Jacobi their contributions must be carried into the next buffer
+    const float* cin = a.contrib[t & 1];
+    if (cin == cout) return;
+    for (int64_t g = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; g < ngroups; g += (int64_t)gridDim.x * blockDim.x)
+      for (int i = gptr[g] + 1; i < gptr[g + 1]; i++) cout[gslots[i]] = cin[gslots[i]];
+    return;
+  }
   double my_delta = 0, my_dang = 0;
   for (int64_t g = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; g < ngroups; g += (int64_t)gridDim.x * blockDim.x) {
     int b = gptr[g], e = gptr[g + 1];
@@ -361,6 +392,16 @@ __global__ void k_pr_merge(PrArgs a, const int32_t* __restrict__ gptr, const int
   }
 }
 
+// loop state at iteration 0 (host copy: the merge cadence fields)
+static void pr_state_init(PrState* dst, int merge_every, cudaStream_t s) {
+  static PrState init;
+  std::memset(&init, 0, sizeof(init));
+  init.merge_every = (unsigned)merge_every;
+  init.do_merge = merge_every == 1 ? 1u : 0u;   // iteration 0 merges iff (0 + 1) % c == 0
+  // pageable source: the copy is staged before cudaMemcpyAsync returns
+  CUDA_OK(cudaMemcpyAsync(dst, &init, sizeof(PrState), cudaMemcpyHostToDevice, s));
+}
+
 __global__ void k_pr_advance(PrState* st, double tol, int max_iters) {
   if (st->stop) return;
   unsigned t = st->iter;
@@ -378,9 +419,26 @@ __global__ void k_pr_advance(PrState* st, double tol, int max_iters) {
   } else {
     st->stall++;
   }
-  if (dl < tol) st->stop = 1;
-  else if (st->stall >= 32 && st->best_delta < 1e-6) st->stop = 3;
-  else if ((int)(t + 1) >= max_iters) st->stop = 2;
+  // merge cadence (P@28188 "after a certain number of iterations or at the
+  // end of the overall computation"; gx_run_opts.merge_every = c):
+  // c = 1 every iteration; c > 1 every c-th iteration, and a converged sweep
+  // that did not merge merges in one more iteration before stopping; c = 0
+  // only that final merge, after which the run ends.
+  const unsigned c = st->merge_every;
+  const bool merged = st->do_merge != 0;
+  if (c == 0 && merged) {
+    st->stop = 1;
+    return;
+  }
+  const unsigned done = dl < tol ? 1u : (st->stall >= 32 && st->best_delta < 1e-6) ? 3u : 0u;
+  if (done) {
+    if (c == 1 || merged) st->stop = done;
+    else st->force = 1;
+  } else if ((int)(t + 1) >= max_iters) {
+    st->stop = 2;
+  }
+  st->do_merge = (c == 1 || (c > 1 && (t + 2) % c == 0) || st->force) ? 1u : 0u;
+  if (st->do_merge) st->force = 0;
 }
 
 template <bool SLOTS>
@@ -393,7 +451,7 @@ __global__ void k_pr_init(PrArgs a, int64_t n_slots, double x0) {
     uint32_t Dv = a.D[v];
     a.x[v] = xv;
     a.contrib[0][v] = (k != HOLE && Dv) ? (float)(xv / (double)Dv) : 0.0f;
-    a.contrib[1][v] = 0.0f;
+    if (a.contrib[1] != a.contrib[0]) a.contrib[1][v] = 0.0f;
     if (k == OWNER && !Dv) my_dang += xv;
   }
   double gsum = block_sum_f64(my_dang, s_red);
@@ -455,7 +513,7 @@ static void run_pagerank_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& in
     K.hi = bounds[rank + 1];
     K.a.win_lo = K.lo / PRW;
     K.a.win_hi = (K.hi + PRW - 1) / PRW;
-    CUDA_OK(cudaMemsetAsync(st.p, 0, sizeof(PrState), s));
+    pr_state_init(st.as<PrState>(), 1, s);
     if (d.identity) k_pr_init<false><<<grid_for(c, ns), 256, 0, s>>>(K.a, ns, 1.0 / (double)g->n);
     else k_pr_init<true><<<grid_for(c, ns), 256, 0, s>>>(K.a, ns, 1.0 / (double)g->n);
   }
@@ -464,7 +522,7 @@ static void run_pagerank_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& in
   X.P = P;
   X.sim = sim;
   int occ = 0;
-  CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<true>, PR_CTA, 0));
+  CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<true, false>, PR_CTA, 0));
   const int grid = (int)std::max<int64_t>(1, (int64_t)std::max(1, occ) * c->num_sms);
   const int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 255) / 256, c->num_sms * 4));
   int launches = nloc, t = 0;
@@ -477,8 +535,8 @@ static void run_pagerank_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& in
       float* cnext = A.contrib[(t + 1) & 1];
       CUDA_OK(cudaMemsetAsync(cnext, 0, sizeof(float) * ns, s));
       if (d.n_groups) CUDA_OK(cudaMemsetAsync(A.gnew, 0, sizeof(double) * ng, s));
-      if (d.identity) k_pr_sell<false><<<grid, PR_CTA, 0, s>>>(A);
-      else k_pr_sell<true><<<grid, PR_CTA, 0, s>>>(A);
+      if (d.identity) k_pr_sell<false, false><<<grid, PR_CTA, 0, s>>>(A);
+      else k_pr_sell<true, false><<<grid, PR_CTA, 0, s>>>(A);
       launches++;
       cn.push_back(cnext);
       dl.push_back(&A.st->delta[0]);
@@ -535,7 +593,11 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   int64_t ns = d.n_slots;
   r.x.alloc(c, sizeof(double) * ns);
   r.contrib[0].alloc(c, sizeof(float) * ns);
-  r.contrib[1].alloc(c, sizeof(float) * ns);
+  const bool sim_ = c->world == 1 && o.sim_ranks > 1;
+  // the asynchronous schedule keeps ONE contrib buffer (read and written in
+  // place by the sweep); Jacobi and the partitioned path need two
+  const bool async = o.pr_schedule == GX_PR_ASYNC && c->world == 1 && !sim_;
+  if (!async) r.contrib[1].alloc(c, sizeof(float) * ns);
   r.gnew.alloc(c, sizeof(double) * std::max<int64_t>(d.n_groups, 1));
   r.pst.alloc(c, sizeof(PrState));
   PrArgs a;
@@ -555,7 +617,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   a.n_slots = ns;
   a.x = r.x.as<double>();
   a.contrib[0] = r.contrib[0].as<float>();
-  a.contrib[1] = r.contrib[1].as<float>();
+  a.contrib[1] = async ? a.contrib[0] : r.contrib[1].as<float>();
   a.D = d.D.as<uint32_t>();
   a.kind = d.identity ? nullptr : d.kind.as<uint8_t>();
   a.gid = d.n_groups ? d.gid.as<int32_t>() : nullptr;
@@ -572,6 +634,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     if (P > 1) {
       GX_CHECK_ARG(P <= 8, "at most 8 ranks");
       GX_CHECK_ARG(o.mapping != GX_MAP_TPV, "the partitioned path uses the LB mapping");
+      GX_CHECK_ARG(o.merge_every == 1 || !d.n_groups, "the partitioned path merges after every iteration");
       run_pagerank_dist(g, o, info, a, P, sim);
       return;
     }
@@ -592,7 +655,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   CUDA_OK(cudaEventCreate(&e0));
   CUDA_OK(cudaEventCreate(&e1));
   CUDA_OK(cudaEventRecord(e0, s));
-  CUDA_OK(cudaMemsetAsync(r.pst.p, 0, sizeof(PrState), s));
+  pr_state_init(a.st, d.n_groups ? o.merge_every : 1, s);
   int gi = grid_for(c, ns);
   if (slots) k_pr_init<true><<<gi, 256, 0, s>>>(a, ns, 1.0 / (double)g->n);
   else k_pr_init<false><<<gi, 256, 0, s>>>(a, ns, 1.0 / (double)g->n);
@@ -600,23 +663,33 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   int launches = 1;
 
   int occ = 0;
-  if (slots) CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<true>, PR_CTA, 0));
-  else CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<false>, PR_CTA, 0));
+  if (slots) CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<true, false>, PR_CTA, 0));
+  else CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<false, false>, PR_CTA, 0));
   int grid = (int)std::max<int64_t>(1, std::min<int64_t>(PL.nwin, (int64_t)std::max(1, occ) * c->num_sms));
   int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 255) / 256, c->num_sms * 4));
   int occt = 0;
-  CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occt, k_pr_tpv<true>, 256, 0));
+  CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occt, k_pr_tpv<true, false>, 256, 0));
   const int grid_tpv = std::max(1, occt) * c->num_sms;
 
   KTimer kt(o.profile != 0, s);
   auto one_iter = [&](int& nl) {
     kt.begin();
     if (mapping == GX_MAP_TPV) {
-      if (slots) k_pr_tpv<true><<<grid_tpv, 256, 0, s>>>(a);
-      else k_pr_tpv<false><<<grid_tpv, 256, 0, s>>>(a);
+      if (async) {
+        if (slots) k_pr_tpv<true, true><<<grid_tpv, 256, 0, s>>>(a);
+        else k_pr_tpv<false, true><<<grid_tpv, 256, 0, s>>>(a);
+      } else {
+        if (slots) k_pr_tpv<true, false><<<grid_tpv, 256, 0, s>>>(a);
+        else k_pr_tpv<false, false><<<grid_tpv, 256, 0, s>>>(a);
+      }
     } else {
-      if (slots) k_pr_sell<true><<<grid, PR_CTA, 0, s>>>(a);
-      else k_pr_sell<false><<<grid, PR_CTA, 0, s>>>(a);
+      if (async) {
+        if (slots) k_pr_sell<true, true><<<grid, PR_CTA, 0, s>>>(a);
+        else k_pr_sell<false, true><<<grid, PR_CTA, 0, s>>>(a);
+      } else {
+        if (slots) k_pr_sell<true, false><<<grid, PR_CTA, 0, s>>>(a);
+        else k_pr_sell<false, false><<<grid, PR_CTA, 0, s>>>(a);
+      }
     }
     kt.end();
     nl++;

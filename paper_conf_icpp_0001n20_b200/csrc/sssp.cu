@@ -363,7 +363,7 @@ __global__ void __launch_bounds__(256) k_sssp_merge(const int32_t* __restrict__ 
                                                     int64_t ngroups, int merge_min, uint32_t* __restrict__ dist,
                                                     SsspAux ax, SsspState* __restrict__ st) {
   const unsigned t = st->iter;
-  if (st->stop) return;
+  if (st->stop || !st->do_merge) return;
   uint32_t* bm_next = ax.bm[(t + 1) % 3];
   const unsigned lane = lane_id();
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -412,11 +412,31 @@ __global__ void __launch_bounds__(256) k_sssp_merge(const int32_t* __restrict__ 
   flush_counters(st, t, 0, 0, my_push, INF);
 }
 
+// merge cadence c != 1 (P@28188: "after a certain number of iterations or at
+// the end of the overall computation"): decided once per iteration,
+// before the merge kernel, from the sweep's counters.  c > 1: merge after
+// every c-th iteration and whenever the sweep alone reached its fixed point
+// (so the run still ends at a merged fixed point); c = 0: only then, and that
+// merge ends the run (copies keep the mean; what it pushes is not relaxed).
+__global__ void k_sssp_merge_decide(SsspState* __restrict__ st) {
+  if (st->stop) return;
+  const unsigned t = st->iter, c = st->merge_every;
+  const bool fixed = st->pushed[t % 3] == 0 && st->far_min == INF;
+  st->do_merge = ((c > 1 && ((t + 1) % c == 0 || fixed)) || (c == 0 && fixed)) ? 1u : 0u;
+  st->final_merge = (c == 0 && fixed) ? 1u : 0u;
+}
+
 // end of iteration t: no bit was set in the next frontier and the far pile is
 // empty => converged (every decreased slot has been relaxed)
 __global__ void k_sssp_advance(SsspState* __restrict__ st, int max_iters) {
   if (st->stop) return;
   const unsigned t = st->iter;
+  if (st->final_merge) {
+    st->act_total += st->active[t % 3];
+    st->stop = 1;
+    st->iter = t + 1;
+    return;
+  }
   st->act_total += st->active[t % 3];
   st->active[(t + 2) % 3] = 0;
   st->pushed[(t + 2) % 3] = 0;
@@ -642,6 +662,8 @@ static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, 
   init.delta = delta;
   init.tau = delta ? delta : INF;
   init.far_min = INF;
+  init.merge_every = 1;
+  init.do_merge = 1;
   cudaEvent_t e0, e1;
   CUDA_OK(cudaEventCreate(&e0));
   CUDA_OK(cudaEventCreate(&e1));
@@ -762,6 +784,7 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   if (P > 1) {
     GX_CHECK_ARG(P <= 8, "at most 8 ranks");
     GX_CHECK_ARG(o.mapping != GX_MAP_TPV, "the partitioned path uses the LB mapping");
+    GX_CHECK_ARG(o.merge_every == 1 || !d.n_groups, "the partitioned path merges after every iteration");
     ensure_heavy_chunks(g);
     unsigned delta = sssp_delta(g);
     if (const char* e = getenv("GX_SSSP_DELTA")) delta = (unsigned)std::max(0, atoi(e));
@@ -816,6 +839,8 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     init.delta = delta;
     init.tau = delta ? delta : INF;
     init.far_min = INF;
+    init.merge_every = d.n_groups ? (unsigned)o.merge_every : 1u;
+    init.do_merge = init.merge_every == 1 ? 1u : 0u;
     CUDA_OK(cudaMemcpyAsync(r.st.p, &init, sizeof(SsspState), cudaMemcpyHostToDevice, s));
   }
   k_sssp_init<<<1, 32, 0, s>>>(r.dist.as<uint32_t>(), dsrc.as<int32_t>(), (int)srcs.size(), ax.bm[0]);
@@ -853,6 +878,10 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
       nl++;
     }
     if (d.n_groups) {
+      if (o.merge_every != 1) {
+        k_sssp_merge_decide<<<1, 1, 0, s>>>(st);
+        nl++;
+      }
       k_sssp_merge<<<grid_merge, 256, 0, s>>>(d.gptr.as<int32_t>(), d.gslots.as<int32_t>(), d.g_in_ptr.as<int32_t>(),
                                               d.g_in.as<uint2>(), d.n_groups, merge_min ? 1 : 0, r.dist.as<uint32_t>(),
                                               ax, st);

@@ -23,6 +23,10 @@ struct SsspState {
   unsigned int raised;          // merges that raised a copy (diagnostic)
   unsigned long long edges;     // edges relaxed, all iterations
   unsigned long long act_total; // frontier entries, all iterations
+  unsigned int merge_every;     // §2.4 cadence c (gx_run_opts.merge_every; 1 when there are no replicas)
+  unsigned int do_merge;        // iteration `iter` ends with a merge
+  unsigned int final_merge;     // c = 0: this iteration's merge ends the run
+  unsigned int pad;
 };
 
 struct SsspAux {

@@ -128,3 +128,54 @@ def test_pagerank_aware_merge_same_fixed_point(gname):
     G.transform(knobs_c(kn, merge_op=1))
     r = G.run("pagerank", tol=1e-11, max_iters=5000, mapping="lb")
     assert np.abs(G.download("rank") - want).sum() <= 1e-6
+
+
+# ---------------------------------------------------------------- PR schedule + merge cadence (N2)
+@pytest.mark.parametrize("gname", list(GRAPHS))
+@pytest.mark.parametrize("kname", ["coal", "smem", "all"])
+@pytest.mark.parametrize("schedule", ["jacobi", "async"])
+def test_pagerank_schedules_same_fixed_point(gname, kname, schedule):
+    """Jacobi (two contrib buffers) and the asynchronous in-place schedule
+    reach the same G_L PageRank (Theorem E3: any schedule)."""
+    raw = GRAPHS[gname]()
+    kn = KNOBS[kname]
+    want, _ = A.pagerank(T.transform(from_raw(raw), kn).logical(), tol=1e-14)
+    G = upload(raw)
+    G.transform(knobs_c(kn))
+    G.run("pagerank", tol=1e-11, max_iters=5000, mapping="lb", pr_schedule=schedule)
+    assert np.abs(G.download("rank") - want).sum() <= 1e-6
+
+
+@pytest.mark.parametrize("gname", ["road48", "rmat12", "fig1_4"])
+@pytest.mark.parametrize("c", [2, 3, 0])
+@pytest.mark.parametrize("mapping", ["lb", "tpv"])
+def test_sssp_merge_cadence(gname, c, mapping):
+    """c > 1 ends at the merged fixed point (= Dijkstra, E1); c = 0 ("merge at
+    the end", P@28188) is bit-exact with the oracle's end-only loop."""
+    from oracle import slotsim as S
+    raw = GRAPHS[gname]()
+    g = from_raw(raw)
+    kn = T.Knobs(coalesce=True, chunk_k=4, replicate_threshold=0.0)
+    tg = T.transform(g, kn)
+    s = sssp_source(g)
+    want = A.sssp_dijkstra(graph_to_edgelist(g), s) if c else S.sssp_slots(tg, s, merge_every=0, local_pass=False)[0]
+    G = upload(raw)
+    G.transform(knobs_c(kn))
+    G.run("sssp", mapping=mapping, merge_every=c)
+    got = G.download("dist")
+    assert np.array_equal(got, want), f"{int(np.sum(got != want))} mismatches"
+
+
+@pytest.mark.parametrize("gname", ["road48", "rmat12"])
+@pytest.mark.parametrize("c", [2, 0])
+@pytest.mark.parametrize("schedule", ["jacobi", "async"])
+def test_pagerank_merge_cadence(gname, c, schedule):
+    from oracle import slotsim as S
+    raw = GRAPHS[gname]()
+    kn = T.Knobs(coalesce=True, chunk_k=4, replicate_threshold=0.0)
+    tg = T.transform(from_raw(raw), kn)
+    want = A.pagerank(tg.logical(), tol=1e-14)[0] if c else S.pagerank_slots(tg, tol=1e-14, merge_every=0)[0]
+    G = upload(raw)
+    G.transform(knobs_c(kn))
+    G.run("pagerank", tol=1e-12, max_iters=20000, mapping="lb", pr_schedule=schedule, merge_every=c)
+    assert np.abs(G.download("rank") - want).sum() <= 1e-6

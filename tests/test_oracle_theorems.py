@@ -61,3 +61,111 @@ def test_E1_on_rmat_with_all_knobs():
     s = int(np.argmax(g.outdeg()))
     d_slot, _ = S.sssp_slots(tg, s)
     assert np.array_equal(d_slot, A.sssp_dijkstra(graph_to_edgelist(g), s))
+
+
+# ---------------------------------------------------------------- merge cadence (P@28188)
+from scipy.sparse import csr_matrix                      # noqa: E402
+from scipy.sparse.csgraph import dijkstra as sp_dijkstra  # noqa: E402
+
+from oracle.graph import INF32                            # noqa: E402
+from oracle.transform import HOLE, REPLICA                # noqa: E402
+
+CAD_KNOBS = [T.Knobs(coalesce=True, chunk_k=4, replicate_threshold=0.0),
+             T.Knobs(coalesce=True, chunk_k=2, replicate_threshold=0.0, smem=True, cc_threshold=0.2,
+                     added_edge_budget=10)]
+
+
+def _slot_multi_source_dijkstra(tg, source):
+    """Independent pin for the no-merge fixed point: shortest paths in the SLOT
+    graph (replica slots have no in-edges) from every copy of the source
+    (copies start equal, P@28609), by scipy's Dijkstra."""
+    rp, col, w, _ = tg.csr()
+    A = csr_matrix((w.astype(np.float64), col, rp), shape=(tg.n_slots, tg.n_slots))
+    o = int(tg.owner_slot[source])
+    srcs = tg.groups().get(o, [o])
+    D = sp_dijkstra(A, directed=True, indices=srcs, min_only=True)
+    return np.where(np.isinf(D), INF32, D).astype(np.int64)
+
+
+@settings(max_examples=40, deadline=None)
+@given(seed=st.integers(0, 10**6), n=st.integers(3, 24), p=st.floats(0.1, 0.4),
+       ki=st.integers(0, len(CAD_KNOBS) - 1), c=st.integers(2, 4))
+def test_cadence_c_gt_1_ends_at_merged_fixed_point(seed, n, p, ki, c):
+    """Merging every c-th iteration (plus once at a sweep fixed point) still
+    ends at the G_L solution: Dijkstra(G) exactly (E1), PR(G_L) (E3)."""
+    g = rand_graph(seed, n, p)
+    tg = T.transform(g, CAD_KNOBS[ki])
+    src = seed % n
+    d, _ = S.sssp_slots(tg, src, merge_every=c)
+    assert np.array_equal(d, A.sssp_dijkstra(graph_to_edgelist(g), src))
+    x, _ = S.pagerank_slots(tg, merge_every=c)
+    xL, _ = A.pagerank(tg.logical())
+    assert np.abs(x - xL).sum() < 1e-9
+
+
+@settings(max_examples=40, deadline=None)
+@given(seed=st.integers(0, 10**6), n=st.integers(3, 24), p=st.floats(0.1, 0.4),
+       ki=st.integers(0, len(CAD_KNOBS) - 1))
+def test_cadence_end_only_sssp_is_mean_of_slot_shortest_paths(seed, n, p, ki):
+    """Merge only at the end (c = 0): each vertex ends with the floor mean
+    (INF copies excluded, R19) of its copies' slot-graph shortest paths."""
+    g = rand_graph(seed, n, p)
+    tg = T.transform(g, CAD_KNOBS[ki])
+    src = seed % n
+    d, _ = S.sssp_slots(tg, src, merge_every=0)
+    ds = _slot_multi_source_dijkstra(tg, src)
+    groups = tg.groups()
+    for v in range(n):
+        o = int(tg.owner_slot[v])
+        fin = [int(ds[c]) for c in groups.get(o, [o]) if ds[c] != INF32]
+        want = sum(fin) // len(fin) if fin else INF32
+        assert int(d[v]) == want
+
+
+def test_cadence_end_only_sssp_can_be_inexact():
+    """The end-only merge is the one schedule under which SSSP is inexact
+    (reading R42): some seeded graph shows a non-zero difference."""
+    seen = 0
+    for seed in range(60):
+        g = rand_graph(seed, 16, 0.15)
+        tg = T.transform(g, CAD_KNOBS[0])
+        if not tg.groups():
+            continue
+        d, _ = S.sssp_slots(tg, 0, merge_every=0)
+        seen += int(not np.array_equal(d, A.sssp_dijkstra(graph_to_edgelist(g), 0)))
+    assert seen > 0
+
+
+@settings(max_examples=30, deadline=None)
+@given(seed=st.integers(0, 10**6), n=st.integers(3, 20), p=st.floats(0.1, 0.4))
+def test_cadence_end_only_pagerank_dense_solve(seed, n, p):
+    """c = 0 for PR: the no-merge fixed point solves a linear system in which
+    replicas keep x0 = 1/N (dense solve, independent of the iteration), then
+    one merge takes the mean of the owner and its replicas' carried values."""
+    g = rand_graph(seed, n, p)
+    tg = T.transform(g, CAD_KNOBS[0])
+    x, _ = S.pagerank_slots(tg, merge_every=0)
+    N, d = tg.n, 0.85
+    Dv = tg.divisor().astype(np.float64)
+    owners = [int(tg.owner_slot[v]) for v in range(N)]
+    idx = {o: i for i, o in enumerate(owners)}
+    M = np.zeros((N, N))
+    b = np.full(N, (1 - d) / N)
+    for s, row in enumerate(tg.rows):
+        if tg.slot_kind[s] == HOLE or not row:
+            continue
+        for (q, _, _) in row:
+            if q not in idx:
+                continue
+            if tg.slot_kind[s] == REPLICA:          # constant inflow from x0
+                b[idx[q]] += d * (1.0 / N) / Dv[s]
+            else:
+                M[idx[q], idx[s]] += d / Dv[s]
+    for o in owners:                                 # dangling mass spread uniformly
+        if Dv[o] == 0:
+            M[:, idx[o]] += d / N
+    xf = np.linalg.solve(np.eye(N) - M, b)
+    want = xf.copy()
+    for o, copies in tg.groups().items():
+        want[idx[o]] = (xf[idx[o]] + (len(copies) - 1) / N) / len(copies)
+    assert np.abs(x - want).sum() < 1e-9
