@@ -140,14 +140,18 @@ typedef struct {
                               device reduction instead of NCCL); LB mapping only    */
   int32_t pr_schedule;     /* PR update schedule on one GPU (SURVEY §8(c) Theorem E3:
                               every schedule has the same fixed point x*):
-                              GX_PR_JACOBI (default) = sweep t reads only x_t (two
-                              contrib buffers, the oracle's iteration order);
-                              GX_PR_ASYNC = one contrib buffer updated in place, a
-                              row reads whichever of x_t / x_{t+1} its sources hold
-                              (asynchronous vertex-centric kernels, P@15381): half
-                              the contrib footprint, but the lagged dangling term
-                              slows convergence (RMAT-24: 52 vs 22 iterations,
-                              DESIGN.md).  The multi-GPU path is Jacobi.          */
+                              GX_PR_ASYNC (default) = one contrib buffer updated in
+                              place, a row reads whichever of x_t / x_{t+1} its
+                              sources hold (asynchronous vertex-centric kernels,
+                              P@15381), half the contrib footprint;
+                              GX_PR_JACOBI = sweep t reads only x_t (two contrib
+                              buffers, the oracle's iteration order).
+                              Both scale iteration t's inputs by 1/sum(x_t) (lazy
+                              normalisation; the fixed point sums to 1), without
+                              which the asynchronous schedule and the §3 local
+                              pass lose mass that decays only at rate d per
+                              iteration (RMAT-24: async 14 iterations, Jacobi 22;
+                              DESIGN.md R56).  The multi-GPU path is Jacobi.     */
   int32_t merge_every;     /* §2.4 confluence cadence (P@28188-28736):
                               1 (default) = after every iteration; c > 1 = after
                               every c-th iteration and once more whenever the

@@ -185,7 +185,7 @@ class Graph:
 
     def run(self, algo: str = "sssp", source: int = -1, max_iters: int = 0, tol: float = 1e-9,
             mapping: str = "auto", damping: float = 0.85, check_every: int = 8, use_graphs: bool = True,
-            bc_sources=None, profile: bool = False, sim_ranks: int = 0, pr_schedule: str = "jacobi",
+            bc_sources=None, profile: bool = False, sim_ranks: int = 0, pr_schedule: str = "async",
             merge_every: int = 1) -> dict:
         o = GxRunOpts()
         _check(lib().gx_run_opts_default(C.byref(o)))

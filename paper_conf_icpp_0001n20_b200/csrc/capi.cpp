@@ -303,7 +303,7 @@ gx_status gx_run_opts_default(gx_run_opts* o) {
   o->damping = 0.85;
   o->check_every = 8;
   o->use_graphs = 1;
-  o->pr_schedule = GX_PR_JACOBI;
+  o->pr_schedule = GX_PR_ASYNC;
   o->merge_every = 1;
   return GX_OK;
 }

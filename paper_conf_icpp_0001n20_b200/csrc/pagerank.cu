@@ -30,6 +30,8 @@ namespace gx {
 struct PrState {
   double delta[3];   // L1 change of x_{t+1}, accumulated into [(t+1)%3]
   double dang[3];    // sum of x_t over dangling vertices, [t%3]
+  double mass[3];    // sum of x_{t+1} over the vertices (owners), accumulated into [(t+1)%3]
+  double scale;      // 1 / sum(x_t): lazy normalisation of iteration t's inputs (see k_pr_advance)
   unsigned iter;
   unsigned stop;     // 1 converged (delta < tol), 2 max_iters, 3 at the fp32-contrib noise floor
   double last_delta;
@@ -38,7 +40,8 @@ struct PrState {
   unsigned merge_every;  // §2.4 cadence (gx_run_opts.merge_every)
   unsigned do_merge;     // iteration `iter` ends with a merge (set by k_pr_advance)
   unsigned force;        // the sweep reached its fixed point without a merge: merge next
-  unsigned pad;
+  unsigned normalize;    // lazy normalisation on (off for the end-only merge, whose
+                         // intermediate no-merge fixed point does not sum to 1)
 };
 
 struct PrArgs {
@@ -72,6 +75,22 @@ struct PrArgs {
   int64_t tpv_nslices;
 };
 
+// one atomic of each kind per CTA: L1 delta, dangling mass and total mass of
+// the values this CTA wrote in iteration t
+__device__ __forceinline__ void pr_flush(PrState* st, unsigned t, double my_delta, double my_dang, double my_mass,
+                                         double* s_red) {
+  double dsum = block_sum_f64(my_delta, s_red);
+  __syncthreads();
+  double gsum = block_sum_f64(my_dang, s_red);
+  __syncthreads();
+  double msum = block_sum_f64(my_mass, s_red);
+  if (threadIdx.x == 0) {
+    if (dsum != 0.0) atomicAdd(&st->delta[(t + 1) % 3], dsum);
+    if (gsum != 0.0) atomicAdd(&st->dang[(t + 1) % 3], gsum);
+    if (msum != 0.0) atomicAdd(&st->mass[(t + 1) % 3], msum);
+  }
+}
+
 // contrib gather: read-only (.nc) in a Jacobi sweep; in the asynchronous
 // schedule the buffer is written by the same sweep, so the load goes through
 // L2 (.cg) and returns either the old or the new value of the source.
@@ -87,11 +106,12 @@ __device__ __forceinline__ float ld_contrib(const float* p, uint64_t pol) {
 
 template <bool SLOTS>
 __device__ __forceinline__ void pr_finalize(const PrArgs& a, int64_t v, double y, double xo, uint32_t Dv, double addc,
-                                            float* cout, double& my_delta, double& my_dang, bool merge_now) {
+                                            float* cout, double& my_delta, double& my_dang, bool merge_now, double sc,
+                                            double& my_mass) {
   if (SLOTS) {
     if (a.kind[v] != OWNER) return;  // holes stay 0; replicas are set by the merge
   }
-  double xn = addc + a.damp * y;
+  double xn = addc + a.damp * sc * y;
   // a replicated owner hands its new value to the merge; in an iteration
   // without a merge (cadence N2) it updates its own copy only
   if (SLOTS && a.gid && merge_now) {
@@ -102,7 +122,8 @@ __device__ __forceinline__ void pr_finalize(const PrArgs& a, int64_t v, double y
     }
   }
   __stcs(a.x + v, xn);
-  my_delta += fabs(xn - xo);
+  my_delta += fabs(xn - sc * xo);
+  my_mass += xn;
   __stcs(cout + v, Dv ? (float)(xn / (double)Dv) : 0.0f);
   if (!Dv) my_dang += xn;
 }
@@ -128,9 +149,10 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell(PrArgs a) {
   const unsigned t = st->iter;
   const float* cin = a.contrib[t & 1];
   float* cout = a.contrib[(t + 1) & 1];
-  const double addc = a.base + a.damp * st->dang[t % 3] * a.invN;
+  const double sc = st->scale;
+  const double addc = a.base + a.damp * sc * st->dang[t % 3] * a.invN;
   const bool merge_now = st->do_merge != 0;
-  double my_delta = 0, my_dang = 0;
+  double my_delta = 0, my_dang = 0, my_mass = 0;
   const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
   const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
   constexpr unsigned NWARP = PR_CTA / 32;
@@ -196,18 +218,119 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell(PrArgs a) {
 #pragma unroll
       for (int u = 0; u < 4; u++) {
         int i = i0 + u * PR_CTA;
-        if (i < nrows) pr_finalize<SLOTS>(a, base + i, s_y[i], xo[u], Dv[u], addc, cout, my_delta, my_dang, merge_now);
+        if (i < nrows) pr_finalize<SLOTS>(a, base + i, s_y[i], xo[u], Dv[u], addc, cout, my_delta, my_dang, merge_now, sc,
+                                              my_mass);
       }
     }
     __syncthreads();
   }
-  double dsum = block_sum_f64(my_delta, s_red);
-  __syncthreads();
-  double gsum = block_sum_f64(my_dang, s_red);
+  pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
+}
+
+// v2 of the windowed SELL pull: (1) the window's x and D are bulk-copied
+// (cp.async.bulk, one elected thread) into shared memory while the warps
+// gather, so the fused update never waits on DRAM; (2) warps take work items
+// -- heavy rows first, then the slices in their descending-length order --
+// from a shared counter (longest-processing-time first), instead of a fixed
+// round robin that leaves the warps with the longest slices as stragglers at
+// the window barrier; (3) every row is written exactly once (lane_row and
+// heavy_row partition the window), so s_y needs no zeroing pass.
+template <bool SLOTS, bool ASYNC>
+__global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell2(PrArgs a) {
+  __shared__ double s_y[PRW];
+  __shared__ __align__(128) double s_x[PRW];
+  __shared__ __align__(128) uint32_t s_D[PRW];
+  __shared__ double s_red[32];
+  __shared__ __align__(8) uint64_t bar;
+  __shared__ int s_next;
+  PrState* st = a.st;
+  if (st->stop) return;
+  const unsigned t = st->iter;
+  const float* cin = a.contrib[t & 1];
+  float* cout = a.contrib[(t + 1) & 1];
+  const double sc = st->scale;
+  const double addc = a.base + a.damp * sc * st->dang[t % 3] * a.invN;
+  const bool merge_now = st->do_merge != 0;
+  double my_delta = 0, my_dang = 0, my_mass = 0;
+  const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
+  const unsigned lane = lane_id();
   if (threadIdx.x == 0) {
-    if (dsum != 0.0) atomicAdd(&st->delta[(t + 1) % 3], dsum);
-    if (gsum != 0.0) atomicAdd(&st->dang[(t + 1) % 3], gsum);
+    mbar_init(&bar, 1);
+    mbar_fence_init();
+    s_next = 0;
   }
+  __syncthreads();
+  unsigned phase = 0;
+  for (int64_t w = a.win_lo + blockIdx.x; w < a.win_hi; w += gridDim.x) {
+    const int64_t base = w * PRW;
+    const int nrows = (int)min((int64_t)PRW, a.n_slots - base);
+    const bool bulk = nrows == PRW;
+    if (bulk && threadIdx.x == 0) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      mbar_expect_tx(&bar, PRW * 12);
+      tma_load_1d(s_x, a.x + base, PRW * 8, &bar, pf);
+      tma_load_1d(s_D, a.D + base, PRW * 4, &bar, pf);
+    }
+    const int64_t s0 = a.win_slice[w], h0 = a.win_heavy[w];
+    const int nh = (int)(a.win_heavy[w + 1] - h0), nit = nh + (int)(a.win_slice[w + 1] - s0);
+    for (;;) {
+      int it = 0;
+      if (lane == 0) it = atomicAdd(&s_next, 1);
+      it = __shfl_sync(FULL, it, 0);
+      if (it >= nit) break;
+      if (it < nh) {   // heavy row: warp-per-row over the CSC
+        const int32_t r = a.heavy_row[h0 + it];
+        const uint32_t e0 = a.crp[r], e1 = a.crp[r + 1];
+        double acc = 0.0;
+        for (uint32_t e = e0 + lane; e < e1; e += 32 * 4) {
+          float v[4];
+#pragma unroll
+          for (int u = 0; u < 4; u++) {
+            uint32_t ee = e + 32 * u;
+            v[u] = ee < e1 ? ld_contrib<ASYNC>(cin + ld_stream_i32(a.csrc + ee, pf), pl) : 0.0f;
+          }
+#pragma unroll
+          for (int u = 0; u < 4; u++) acc += (double)v[u];
+        }
+        acc = warp_sum_f64(acc);
+        if (lane == 0) s_y[r - base] = acc;
+        continue;
+      }
+      const int64_t sl = s0 + (it - nh);   // light slice: lane-per-row
+      const uint32_t L = a.slice_len[sl];
+      const uint32_t* p = a.slab + a.slice_off[sl] + lane;
+      const int32_t row = a.lane_row[sl * 32 + lane];
+      double acc = 0.0;
+      uint32_t j = 0;
+      for (; j + PR_U <= L; j += PR_U) {
+        uint32_t e[PR_U];
+#pragma unroll
+        for (int u = 0; u < PR_U; u++) e[u] = ld_stream_u32(p + 32 * (j + u), pf);
+        float v[PR_U];
+#pragma unroll
+        for (int u = 0; u < PR_U; u++) v[u] = e[u] != PR_SENT ? ld_contrib<ASYNC>(cin + e[u], pl) : 0.0f;
+#pragma unroll
+        for (int u = 0; u < PR_U; u++) acc += (double)v[u];
+      }
+      for (; j < L; j++) {
+        uint32_t e = ld_stream_u32(p + 32 * j, pf);
+        if (e != PR_SENT) acc += (double)ld_contrib<ASYNC>(cin + e, pl);
+      }
+      if (row >= 0) s_y[row - base] = acc;
+    }
+    if (bulk) mbar_wait(&bar, phase);
+    phase ^= bulk ? 1u : 0u;
+    __syncthreads();
+    if (threadIdx.x == 0) s_next = 0;    // published by the barrier below
+    for (int i = threadIdx.x; i < nrows; i += PR_CTA) {
+      const double xo = bulk ? s_x[i] : __ldcs(a.x + base + i);
+      const uint32_t Dv = bulk ? s_D[i] : __ldcs(a.D + base + i);
+      pr_finalize<SLOTS>(a, base + i, s_y[i], xo, Dv, addc, cout, my_delta, my_dang, merge_now, sc,
+                                              my_mass);
+    }
+    __syncthreads();
+  }
+  pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
 }
 
 // The paper's thread-per-vertex pull (tpv.cu): lane = slot of the schedule,
@@ -221,9 +344,10 @@ __global__ void __launch_bounds__(256) k_pr_tpv(PrArgs a) {
   const unsigned t = st->iter;
   const float* cin = a.contrib[t & 1];
   float* cout = a.contrib[(t + 1) & 1];
-  const double addc = a.base + a.damp * st->dang[t % 3] * a.invN;
+  const double sc = st->scale;
+  const double addc = a.base + a.damp * sc * st->dang[t % 3] * a.invN;
   const bool merge_now = st->do_merge != 0;
-  double my_delta = 0, my_dang = 0;
+  double my_delta = 0, my_dang = 0, my_mass = 0;
   const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
   const unsigned lane = lane_id();
   const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -249,15 +373,9 @@ __global__ void __launch_bounds__(256) k_pr_tpv(PrArgs a) {
       if (e != PR_SENT) acc += (double)ld_contrib<ASYNC>(cin + e, pl);
     }
     if (row >= 0) pr_finalize<SLOTS>(a, row, acc, __ldcs(a.x + row), __ldcs(a.D + row), addc, cout, my_delta, my_dang,
-                                      merge_now);
+                                      merge_now, sc, my_mass);
   }
-  double dsum = block_sum_f64(my_delta, s_red);
-  __syncthreads();
-  double gsum = block_sum_f64(my_dang, s_red);
-  if (threadIdx.x == 0) {
-    if (dsum != 0.0) atomicAdd(&st->delta[(t + 1) % 3], dsum);
-    if (gsum != 0.0) atomicAdd(&st->dang[(t + 1) % 3], gsum);
-  }
+  pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
 }
 
 // §3 shared-memory pass for PR (P@32188-32416; SURVEY A7 "PR store"): after
@@ -282,8 +400,9 @@ __global__ void __launch_bounds__(256) k_pr_local(PrArgs a, const int32_t* __res
   const unsigned t = st->iter;
   const float* cin = a.contrib[t & 1];
   float* cout = a.contrib[(t + 1) & 1];
-  const double addc = a.base + a.damp * st->dang[t % 3] * a.invN;
-  double my_delta = 0, my_dang = 0;
+  const double sc = st->scale;
+  const double addc = a.base + a.damp * sc * st->dang[t % 3] * a.invN;
+  double my_delta = 0, my_dang = 0, my_mass = 0;
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int b0 = tptr[tile], nm = tptr[tile + 1] - b0;
     const int e0 = teptr[tile], ne = teptr[tile + 1] - e0;
@@ -293,7 +412,7 @@ __global__ void __launch_bounds__(256) k_pr_local(PrArgs a, const int32_t* __res
       fixed[i] = fx;
       xs[i] = a.x[v];
       Ds[i] = a.D[v];
-      ext[i] = fx ? 0.0 : (xs[i] - addc) / a.damp;    // y_v of the sweep
+      ext[i] = fx ? 0.0 : (xs[i] - addc) / a.damp;    // sc * y_v of the sweep
     }
     __syncthreads();
     for (int i = threadIdx.x; i < nm; i += blockDim.x) {
@@ -304,7 +423,7 @@ __global__ void __launch_bounds__(256) k_pr_local(PrArgs a, const int32_t* __res
         const int s = p.x & 0xff, d = (p.x >> 8) & 0xff;
         if (d == i && !fixed[s]) sub += (double)cin[tmem[b0 + s]];
       }
-      ext[i] -= sub;
+      ext[i] -= sc * sub;
     }
     __syncthreads();
     const int iters = titers[tile];
@@ -333,17 +452,12 @@ __global__ void __launch_bounds__(256) k_pr_local(PrArgs a, const int32_t* __res
       a.x[v] = xs[i];
       cout[v] = Ds[i] ? (float)(xs[i] / (double)Ds[i]) : 0.0f;
       my_delta += fabs(xs[i] - old);
+      my_mass += xs[i] - old;
       if (!Ds[i]) my_dang += xs[i] - old;
     }
     __syncthreads();
   }
-  double dsum = block_sum_f64(my_delta, s_red);
-  __syncthreads();
-  double gsum = block_sum_f64(my_dang, s_red);
-  if (threadIdx.x == 0) {
-    if (dsum != 0.0) atomicAdd(&st->delta[(t + 1) % 3], dsum);
-    if (gsum != 0.0) atomicAdd(&st->dang[(t + 1) % 3], gsum);
-  }
+  pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
 }
 
 // §2.4 confluence: every copy <- mean(owner's new value, replicas' carried
@@ -364,17 +478,19 @@ __global__ void k_pr_merge(PrArgs a, const int32_t* __restrict__ gptr, const int
       for (int i = gptr[g] + 1; i < gptr[g + 1]; i++) cout[gslots[i]] = cin[gslots[i]];
     return;
   }
-  double my_delta = 0, my_dang = 0;
+  const double sc = st->scale;   // carried values are on the scale of x_t
+  double my_delta = 0, my_dang = 0, my_mass = 0;
   for (int64_t g = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; g < ngroups; g += (int64_t)gridDim.x * blockDim.x) {
     int b = gptr[g], e = gptr[g + 1];
     int32_t o = gslots[b];
     double s = a.gnew[g];
-    for (int i = b + 1; i < e; i++) s += a.x[gslots[i]];
+    for (int i = b + 1; i < e; i++) s += sc * a.x[gslots[i]];
     // GX_MERGE_MEAN: the paper's algorithm-agnostic mean (P@28609) over the
     // owner's new value and the replicas' carried values; the algorithm-aware
     // alternative (P@28421) for PR broadcasts the owner's new value (R54)
     double mean = a.merge_bcast ? a.gnew[g] : s / (double)(e - b);
-    my_delta += fabs(mean - a.x[o]);
+    my_delta += fabs(mean - sc * a.x[o]);
+    my_mass += mean;
     uint32_t Dv = a.D[o];
     float c = Dv ? (float)(mean / (double)Dv) : 0.0f;
     for (int i = b; i < e; i++) {
@@ -383,13 +499,7 @@ __global__ void k_pr_merge(PrArgs a, const int32_t* __restrict__ gptr, const int
     }
     if (!Dv) my_dang += mean;
   }
-  double dsum = block_sum_f64(my_delta, s_red);
-  __syncthreads();
-  double gsum = block_sum_f64(my_dang, s_red);
-  if (threadIdx.x == 0) {
-    if (dsum != 0.0) atomicAdd(&st->delta[(t + 1) % 3], dsum);
-    if (gsum != 0.0) atomicAdd(&st->dang[(t + 1) % 3], gsum);
-  }
+  pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
 }
 
 // loop state at iteration 0 (host copy: the merge cadence fields)
@@ -397,6 +507,8 @@ static void pr_state_init(PrState* dst, int merge_every, cudaStream_t s) {
   static PrState init;
   std::memset(&init, 0, sizeof(init));
   init.merge_every = (unsigned)merge_every;
+  init.scale = 1.0;    // x0 = 1/N on every vertex sums to 1
+  init.normalize = merge_every != 0 ? 1u : 0u;
   init.do_merge = merge_every == 1 ? 1u : 0u;   // iteration 0 merges iff (0 + 1) % c == 0
   // pageable source: the copy is staged before cudaMemcpyAsync returns
   CUDA_OK(cudaMemcpyAsync(dst, &init, sizeof(PrState), cudaMemcpyHostToDevice, s));
@@ -407,8 +519,15 @@ __global__ void k_pr_advance(PrState* st, double tol, int max_iters) {
   unsigned t = st->iter;
   double dl = st->delta[(t + 1) % 3];
   st->last_delta = dl;
+  // lazy normalisation: the next iteration scales its inputs by 1 / sum(x).
+  // Jacobi conserves the mass (sum x = 1) by itself; the asynchronous schedule
+  // and the §3 local pass do not, and a mass defect decays only at rate d per
+  // iteration (R56).  The fixed point is unchanged (it has sum 1).
+  const double ms = st->mass[(t + 1) % 3];
+  st->scale = (st->normalize && ms > 0.0) ? 1.0 / ms : 1.0;
   st->delta[(t + 2) % 3] = 0.0;
   st->dang[(t + 2) % 3] = 0.0;
+  st->mass[(t + 2) % 3] = 0.0;
   st->iter = t + 1;
   // contrib is stored in fp32: once the iterate reaches the fixed point of the
   // rounded map it may cycle at a delta floor ~1e-8..1e-9 (R55).
@@ -529,7 +648,7 @@ static void run_pagerank_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& in
   PrState h;
   for (;; t++) {
     std::vector<float*> cn;
-    std::vector<double*> dl, dg, gl;
+    std::vector<double*> dl, dg, gl, ml;
     for (int p = 0; p < nloc; p++) {
       PrArgs& A = R[p].a;
       float* cnext = A.contrib[(t + 1) & 1];
@@ -541,11 +660,13 @@ static void run_pagerank_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& in
       cn.push_back(cnext);
       dl.push_back(&A.st->delta[0]);
       dg.push_back(&A.st->dang[0]);
+      ml.push_back(&A.st->mass[0]);
       gl.push_back(A.gnew);
     }
     X.sum_f32(cn, ns);                                  // the exchange
     X.sum_f64(dl, 3);
     X.sum_f64(dg, 3);
+    X.sum_f64(ml, 3);
     if (d.n_groups) X.sum_f64(gl, d.n_groups);
     for (int p = 0; p < nloc; p++) {
       if (d.n_groups) {
@@ -662,8 +783,11 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   CUDA_OK(cudaGetLastError());
   int launches = 1;
 
+  // GX_PR_KERNEL=1 selects the round-1 kernel (A/B experiments)
+  const bool v2 = !(getenv("GX_PR_KERNEL") && atoi(getenv("GX_PR_KERNEL")) == 1);
   int occ = 0;
-  if (slots) CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<true, false>, PR_CTA, 0));
+  if (v2) CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell2<true, false>, PR_CTA, 0));
+  else if (slots) CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<true, false>, PR_CTA, 0));
   else CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<false, false>, PR_CTA, 0));
   int grid = (int)std::max<int64_t>(1, std::min<int64_t>(PL.nwin, (int64_t)std::max(1, occ) * c->num_sms));
   int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 255) / 256, c->num_sms * 4));
@@ -683,7 +807,15 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
         else k_pr_tpv<false, false><<<grid_tpv, 256, 0, s>>>(a);
       }
     } else {
-      if (async) {
+      if (v2) {
+        if (async) {
+          if (slots) k_pr_sell2<true, true><<<grid, PR_CTA, 0, s>>>(a);
+          else k_pr_sell2<false, true><<<grid, PR_CTA, 0, s>>>(a);
+        } else {
+          if (slots) k_pr_sell2<true, false><<<grid, PR_CTA, 0, s>>>(a);
+          else k_pr_sell2<false, false><<<grid, PR_CTA, 0, s>>>(a);
+        }
+      } else if (async) {
         if (slots) k_pr_sell<true, true><<<grid, PR_CTA, 0, s>>>(a);
         else k_pr_sell<false, true><<<grid, PR_CTA, 0, s>>>(a);
       } else {
