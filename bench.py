@@ -215,7 +215,7 @@ def main():
     # dominant kernel roofline (live CUDA events around each sweep launch)
     peak, peak_src = peaks()
     kern = {}
-    for name, idx in (("k_sssp_lb", 0), ("k_pr_sell", 1)):
+    for name, idx in (("k_sssp_lb", 0), ("k_pr_sell2", 1)):
         ms = sum(r[idx]["sweep_ms"] for r in runs)
         nl = sum(r[idx]["sweep_launches"] for r in runs)
         by = sum(r[idx]["sweep_bytes"] for r in runs)
