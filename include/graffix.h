@@ -97,7 +97,21 @@ typedef struct {
   int32_t degree_norm;           /* §4 on/off (P@33145)                               */
   double degsim_threshold;       /* degreeSim < theta_d (strict), default 0.3         */
   double degree_target;          /* "degree-normalisation factor", default 0.85       */
+  int32_t added_weight_rule;     /* weight of every added edge standing for a 2-hop
+                                    path with hop weights w1, w2:
+                                    GX_W_SUM (default) w1 + w2 (P@34493, reading R17:
+                                    never shorter than the path, SSSP stays exact);
+                                    GX_W_MAX max(w1, w2), GX_W_MEAN max(1, (w1+w2)/2)
+                                    ("one can choose an alternative", P@34692)        */
+  int32_t sibling_undirected;    /* §3: 0 (default) sibling edges only along directed
+                                    2-paths a->c->b (R23); 1 any two neighbours of c
+                                    in the undirected CC view (P@29950), both
+                                    directions, hop weights = lighter direction       */
 } gx_knobs;
+
+#define GX_W_SUM 0
+#define GX_W_MAX 1
+#define GX_W_MEAN 2
 
 typedef struct {
   int64_t n_slots, n_holes, n_replicas, holes_filled;

@@ -54,6 +54,27 @@ class Knobs:
     degree_norm: bool = False
     degsim_threshold: float = 0.3        # best near 0.3 (P@55324)
     degree_target: float = 0.85          # 85% of warp max (P@55220)
+    added_weight: str = "sum"            # N3: weight rule of every added edge (combine())
+    sibling_undirected: bool = False     # N3: §3 sibling edges on the undirected CC view
+
+
+WEIGHT_RULES = ("sum", "max", "mean")
+
+
+def combine(w1: int, w2: int, rule: str = "sum") -> int:
+    """Weight of an added edge u->q that stands for the 2-hop path u->v->q
+    with hop weights w1, w2.  P@34493 sets it to the sum ("sum", reading R17,
+    the default: the edge is never shorter than the path it replaces) and
+    P@34692 allows "an alternative method to set up the edge-weights"
+    (SURVEY N3): "max" = the heavier hop, "mean" = floor((w1 + w2) / 2),
+    at least 1.  Any rule but "sum" can shorten distances (inexact SSSP)."""
+    if rule == "sum":
+        return w1 + w2
+    if rule == "max":
+        return max(w1, w2)
+    if rule == "mean":
+        return max(1, (w1 + w2) // 2)
+    raise ValueError(rule)
 
 
 @dataclass
@@ -226,7 +247,7 @@ def renumber(g: Graph, k: int):
     return np.asarray(new, np.int64), n_slots, ranges, sources
 
 
-def coalesce(g: Graph, k: int, theta_ppm: int) -> TransformedGraph:
+def coalesce(g: Graph, k: int, theta_ppm: int, rule: str = "sum") -> TransformedGraph:
     """§2: renumber into an isomorph, then ReplicateVertex (Alg 2 l.21-35).
 
     Replication (P@17298-18419, P@23832-27600, readings R10-R18):
@@ -242,7 +263,8 @@ def coalesce(g: Graph, k: int, theta_ppm: int) -> TransformedGraph:
       * per assignment (n, C, hole): every edge n->p with chunk(p) = C moves to
         the hole's row (l.32-34); the hole gets n->q for every non-hole q in C
         with q not in N+(n) + {n} reachable as n->v->q, weight
-        min_v w(n,v)+w(v,q) (l.35; R16, R17), using n's pre-move edges;
+        min_v combine(w(n,v), w(v,q)) (l.35; R16, R17; sum by default),
+        using n's pre-move edges;
       * replicas have no in-edges (R18).
     """
     new, n_slots, ranges, sources = renumber(g, k)
@@ -294,8 +316,9 @@ def coalesce(g: Graph, k: int, theta_ppm: int) -> TransformedGraph:
         for (v, wv) in orig_row:
             for (q, wq) in radj[v]:
                 if q // k == C and q not in nplus and q != s and kind[q] != HOLE:
-                    if q not in best or wv + wq < best[q]:
-                        best[q] = wv + wq
+                    wc = combine(wv, wq, rule)
+                    if q not in best or wc < best[q]:
+                        best[q] = wc
         rows[h] = moved + [[q, w, ADD_COALESCE] for q, w in sorted(best.items())]
         kind[h] = REPLICA
         slot_to_orig[h] = slot_to_orig[s]
@@ -345,9 +368,18 @@ class _Logical:
         # strict >, CC = 0 when d < 2 (reading R21)
         return self.T[c] * 1_000_000 > th * self.P(c)
 
-    def eligible(self, c, a, b):
-        """Directed sibling edge a->b for centre c (reading R23)."""
+    def eligible(self, c, a, b, undirected=False):
+        """Sibling edge a->b for centre c: along a directed 2-path a->c->b
+        (reading R23); with undirected=True (N3, the CC view P@29950) any
+        two neighbours of c in U."""
+        if undirected:
+            return a in self.N[c] and b in self.N[c]
         return (c in self.out[a]) and (b in self.out[c])
+
+    def wU(self, a, b):
+        """Weight of the pair {a, b} in U: the lighter existing direction."""
+        ws = [x for x in (self.out[a].get(b), self.out[b].get(a)) if x is not None]
+        return min(ws)
 
     def link(self, a, b, w):
         """Insert a->b into G_L; keep N and triangle counts current."""
@@ -364,7 +396,7 @@ class _Logical:
             self.N[b].add(a)
 
 
-def cc_edges(tg: TransformedGraph, cc_ppm: int, budget: int):
+def cc_edges(tg: TransformedGraph, cc_ppm: int, budget: int, rule: str = "sum", undirected: bool = False):
     """§3 edge insertion (P@30608-32051), readings R21-R26.  PARITY UNPINNED
     beyond invariants (the selection rules are readings).
 
@@ -381,7 +413,9 @@ def cc_edges(tg: TransformedGraph, cc_ppm: int, budget: int):
     to its lowest-internal-degree linkable partner (ties: id).  Stops when
     the budget is 0 or a pass links nothing.
     Linking {a, b} inserts a->b if eligible then b->a if eligible (a < b),
-    each costing 1 unit of budget, weight w(x,c) + w(c,y) (sum rule R17).
+    each costing 1 unit of budget, weight combine(w(x,c), w(c,y)) (sum rule
+    R17 by default).  undirected=True (N3): every pair of U-neighbours of c
+    is eligible in both directions, hop weights taken in U (wU).
     Returns the list of added (a, b, w)."""
     L = _Logical(tg)
     n = tg.n
@@ -389,14 +423,17 @@ def cc_edges(tg: TransformedGraph, cc_ppm: int, budget: int):
     rem = [budget]
 
     def linkable(c, a, b):
-        return b not in L.N[a] and (L.eligible(c, a, b) or L.eligible(c, b, a))
+        return b not in L.N[a] and (L.eligible(c, a, b, undirected) or L.eligible(c, b, a, undirected))
 
     def do_link(c, a, b):
         for (x, y) in ((a, b), (b, a)):
             if rem[0] <= 0:
                 return
-            if L.eligible(c, x, y) and y not in L.out[x]:
-                w = L.out[x][c] + L.out[c][y]
+            if L.eligible(c, x, y, undirected) and y not in L.out[x]:
+                if undirected:
+                    w = combine(L.wU(x, c), L.wU(c, y), rule)
+                else:
+                    w = combine(L.out[x][c], L.out[c][y], rule)
                 L.link(x, y, w)
                 added.append((x, y, w))
                 rem[0] -= 1
@@ -506,7 +543,7 @@ def subgraphs(L: _Logical, n: int, cc_ppm: int, smax: int, smem_iters: int):
 def apply_smem(tg: TransformedGraph, knobs: Knobs, m_orig: int):
     cc_ppm = ppm(knobs.cc_threshold)
     budget = knobs.added_edge_budget if knobs.added_edge_budget >= 0 else m_orig // 100
-    added, L = cc_edges(tg, cc_ppm, budget)
+    added, L = cc_edges(tg, cc_ppm, budget, knobs.added_weight, knobs.sibling_undirected)
     for (a, b, w) in added:
         tg.rows[int(tg.owner_slot[a])].append([int(tg.owner_slot[b]), w, ADD_SMEM])
     tg.tiles = subgraphs(L, tg.n, cc_ppm, knobs.smem_max_nodes, knobs.smem_iters)
@@ -533,7 +570,7 @@ def apply_degnorm(tg: TransformedGraph, knobs: Knobs, combined: bool):
     (M - d) * 1e6 < theta_ppm * M (degreeSim < theta, R32) whose d < target =
     ceil(f_ppm * M / 1e6) gets up to target - d edges v->q to logical 2-hop
     out-neighbours q not in N+(v) + {v} (non-hole), ordered by
-    (min_x w(v,x)+w(x,q), q asc); candidates come from the graph before any
+    (min_x combine(w(v,x), w(x,q)), q asc); candidates come from the graph before any
     §4 addition.  Replica slots are not padded (reading)."""
     th = ppm(knobs.degsim_threshold)
     f = ppm(knobs.degree_target)
@@ -570,8 +607,9 @@ def apply_degnorm(tg: TransformedGraph, knobs: Knobs, combined: bool):
                 for q, wq in lout[x].items():
                     if q == u or q in lout[u]:
                         continue
-                    if q not in best or wx + wq < best[q]:
-                        best[q] = wx + wq
+                    wc = combine(wx, wq, knobs.added_weight)
+                    if q not in best or wc < best[q]:
+                        best[q] = wc
             cand = sorted(best.items(), key=lambda kv: (kv[1], kv[0]))[:target - d]
             for q, w in cand:
                 adds.append((s, int(tg.owner_slot[q]), w))
@@ -586,7 +624,7 @@ def transform(g: Graph, knobs: Knobs | None = None) -> TransformedGraph:
     """TransformGraph (Alg 2 l.1-9) extended with §3 and §4 (composition R34)."""
     knobs = knobs or Knobs()
     if knobs.coalesce:
-        tg = coalesce(g, knobs.chunk_k, ppm(knobs.replicate_threshold))
+        tg = coalesce(g, knobs.chunk_k, ppm(knobs.replicate_threshold), knobs.added_weight)
     else:
         tg = identity(g)
         tg.info.update(n_holes=0, n_replicas=0, holes_filled=0, edges_added_coalesce=0)

@@ -42,12 +42,17 @@ class Knobs:
     degree_norm: bool = False
     degsim_threshold: float = 0.3
     degree_target: float = 0.85
+    added_weight: str = "sum"          # N3: "sum" | "max" | "mean" (gx_knobs.added_weight_rule)
+    sibling_undirected: bool = False   # N3: §3 sibling edges on the undirected CC view
 
     def to_c(self) -> GxKnobs:
         k = GxKnobs()
         _check(lib().gx_knobs_default(C.byref(k)))
         for f in fields(self):
             v = getattr(self, f.name)
+            if f.name == "added_weight":
+                k.added_weight_rule = {"sum": 0, "max": 1, "mean": 2}[v]
+                continue
             setattr(k, f.name, int(v) if isinstance(v, bool) else v)
         return k
 

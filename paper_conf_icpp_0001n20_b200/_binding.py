@@ -41,7 +41,7 @@ class GxKnobs(C.Structure):
                 ("replicate_threshold", C.c_double), ("merge_op", C.c_int32), ("smem", C.c_int32),
                 ("cc_threshold", C.c_double), ("added_edge_budget", C.c_int64), ("smem_iters", C.c_int32),
                 ("smem_max_nodes", C.c_int32), ("degree_norm", C.c_int32), ("degsim_threshold", C.c_double),
-                ("degree_target", C.c_double)]
+                ("degree_target", C.c_double), ("added_weight_rule", C.c_int32), ("sibling_undirected", C.c_int32)]
 
 
 class GxTransformInfo(C.Structure):

@@ -288,6 +288,8 @@ gx_status gx_knobs_default(gx_knobs* k) {
   k->degree_norm = 0;
   k->degsim_threshold = 0.3;
   k->degree_target = 0.85;
+  k->added_weight_rule = GX_W_SUM;
+  k->sibling_undirected = 0;
   return GX_OK;
 }
 
@@ -319,6 +321,8 @@ static void check_knobs(const gx_knobs& k) {
   GX_CHECK_ARG(k.smem_max_nodes >= 2 && k.smem_max_nodes <= 255, "smem_max_nodes must be in 2..255");
   GX_CHECK_ARG(k.merge_op == GX_MERGE_MEAN || k.merge_op == GX_MERGE_MIN, "merge_op invalid");
   GX_CHECK_ARG(k.smem_iters >= 0, "smem_iters must be >= 0");
+  GX_CHECK_ARG(k.added_weight_rule >= GX_W_SUM && k.added_weight_rule <= GX_W_MEAN, "added_weight_rule invalid");
+  GX_CHECK_ARG(k.sibling_undirected == 0 || k.sibling_undirected == 1, "sibling_undirected must be 0 or 1");
 }
 
 gx_status gx_transform(gx_graph* g, const gx_knobs* knobs, gx_transform_info* info) {

@@ -25,6 +25,17 @@
 namespace gx {
 namespace {
 
+// Weight of an added edge standing for the 2-hop path with hop weights w1, w2
+// (gx_knobs.added_weight_rule): the sum (P@34493, R17) or one of
+// the "alternative" rules P@34692 allows.
+uint32_t combine_w(uint32_t w1, uint32_t w2, int rule) {
+  switch (rule) {
+    case GX_W_MAX: return std::max(w1, w2);
+    case GX_W_MEAN: return std::max<uint32_t>(1u, (uint32_t)(((uint64_t)w1 + w2) / 2));
+    default: return w1 + w2;
+  }
+}
+
 int64_t ppm(double x) { return (int64_t)std::floor(x * 1e6 + 0.5); }
 
 struct Edge {
@@ -167,7 +178,7 @@ void renumber(const HostCSR& g, int k, std::vector<int32_t>& nw, int64_t& n_slot
 }
 
 // Renumber + ReplicateVertex (Alg 2 l.21-35), readings R10-R18.
-void coalesce(const HostCSR& g, int k, int64_t theta_ppm, Work& W) {
+void coalesce(const HostCSR& g, int k, int64_t theta_ppm, int wrule, Work& W) {
   const int64_t n = g.n;
   std::vector<int32_t> nw;
   std::vector<std::pair<int64_t, int64_t>> ranges;
@@ -259,7 +270,7 @@ void coalesce(const HostCSR& g, int k, int64_t theta_ppm, Work& W) {
         const int32_t q = eq.dst;
         if (q / k != a.C || q == a.s || W.kind[q] == HOLE) continue;
         if (std::binary_search(nplus.begin(), nplus.end(), q)) continue;
-        const uint32_t w = ev.w + eq.w;
+        const uint32_t w = combine_w(ev.w, eq.w, wrule);
         auto it = best.find(q);
         if (it == best.end() || w < it->second) best[q] = w;
       }
@@ -297,7 +308,17 @@ struct Logical {
                                });
     return (it != r.end() && it->first == b) ? &it->second : nullptr;
   }
-  bool eligible(int32_t c, int32_t a, int32_t b) const { return outw(a, c) && outw(c, b); }  // R23
+  // sibling edge a->b for centre c: along a directed 2-path (R23), or any two
+  // U-neighbours of c with the undirected variant (N3, P@29950)
+  bool eligible(int32_t c, int32_t a, int32_t b, bool und) const {
+    return und ? (adj(c, a) && adj(c, b)) : (outw(a, c) && outw(c, b));
+  }
+  // weight of the pair {a, b} in U: the lighter existing direction
+  uint32_t wU(int32_t a, int32_t b) const {
+    const uint32_t* x = outw(a, b);
+    const uint32_t* y = outw(b, a);
+    return x && y ? std::min(*x, *y) : (x ? *x : *y);
+  }
   static int64_t inter(const std::vector<int32_t>& x, const std::vector<int32_t>& y) {
     int64_t r = 0;
     size_t i = 0, j = 0;
@@ -406,19 +427,19 @@ struct SmemOut {
 };
 
 // CC edge insertion: case 1 (R22) then case 2 (R24, R25); budget in directed edges (R26)
-void cc_edges(Logical& L, int64_t th, int64_t budget, SmemOut& out) {
+void cc_edges(Logical& L, int64_t th, int64_t budget, int wrule, bool und, SmemOut& out) {
   const int64_t n = L.n;
   int64_t rem = budget;
   auto linkable = [&](int32_t c, int32_t a, int32_t b) {
-    return !L.adj(a, b) && (L.eligible(c, a, b) || L.eligible(c, b, a));
+    return !L.adj(a, b) && (L.eligible(c, a, b, und) || L.eligible(c, b, a, und));
   };
   auto do_link = [&](int32_t c, int32_t a, int32_t b) {
     const int32_t xs[2] = {a, b}, ys[2] = {b, a};
     for (int q = 0; q < 2; q++) {
       if (rem <= 0) return;
       const int32_t x = xs[q], y = ys[q];
-      if (L.eligible(c, x, y) && !L.outw(x, y)) {
-        const uint32_t w = *L.outw(x, c) + *L.outw(c, y);
+      if (L.eligible(c, x, y, und) && !L.outw(x, y)) {
+        const uint32_t w = und ? combine_w(L.wU(x, c), L.wU(c, y), wrule) : combine_w(*L.outw(x, c), *L.outw(c, y), wrule);
         L.link(x, y, w);
         out.added.push_back({x, y, w});
         rem--;
@@ -535,7 +556,7 @@ int bucket_of(int64_t d) {
   return b;  // R30: 0 for d = 0, else 1 + floor(log2 d)
 }
 
-void degnorm(Work& W, int64_t th, int64_t f, bool combined, std::vector<int32_t>& sched, int64_t& added) {
+void degnorm(Work& W, int64_t th, int64_t f, bool combined, int wrule, std::vector<int32_t>& sched, int64_t& added) {
   const int64_t ns = W.n_slots;
   std::vector<int64_t> deg(ns);
   for (int64_t s = 0; s < ns; s++) deg[s] = (int64_t)W.rows[s].size();
@@ -582,7 +603,7 @@ void degnorm(Work& W, int64_t th, int64_t f, bool combined, std::vector<int32_t>
                                    return x.first < y.first;
                                  }))
             continue;
-          const uint32_t w = ex.second + eq.second;
+          const uint32_t w = combine_w(ex.second, eq.second, wrule);
           auto it = best.find(q);
           if (it == best.end() || w < it->second) best[q] = w;
         }
@@ -607,7 +628,7 @@ void degnorm(Work& W, int64_t th, int64_t f, bool combined, std::vector<int32_t>
 void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out) {
   auto t0 = std::chrono::steady_clock::now();
   Work W;
-  if (k.coalesce) coalesce(g, k.chunk_k, ppm(k.replicate_threshold), W);
+  if (k.coalesce) coalesce(g, k.chunk_k, ppm(k.replicate_threshold), k.added_weight_rule, W);
   else identity(g, W);
   SmemOut sm;
   if (k.smem) {
@@ -615,14 +636,15 @@ void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out) {
     build_logical(W, L);
     const int64_t th = ppm(k.cc_threshold);
     const int64_t budget = k.added_edge_budget >= 0 ? k.added_edge_budget : g.m / 100;
-    cc_edges(L, th, budget, sm);
+    cc_edges(L, th, budget, k.added_weight_rule, k.sibling_undirected != 0, sm);
     subgraphs(L, th, k.smem_max_nodes, k.smem_iters, sm);
     for (auto& e : sm.added)
       W.rows[W.owner[std::get<0>(e)]].push_back({W.owner[std::get<1>(e)], std::get<2>(e), ADD_SMEM});
   }
   std::vector<int32_t> sched;
   int64_t added_dn = 0;
-  if (k.degree_norm) degnorm(W, ppm(k.degsim_threshold), ppm(k.degree_target), k.coalesce != 0, sched, added_dn);
+  if (k.degree_norm)
+    degnorm(W, ppm(k.degsim_threshold), ppm(k.degree_target), k.coalesce != 0, k.added_weight_rule, sched, added_dn);
 
   // assemble the slot CSR, rows sorted by destination slot (R11)
   out = SlotGraph();

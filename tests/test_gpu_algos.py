@@ -23,7 +23,12 @@ KNOBS = {
     "exact": None,
     "all": T.Knobs(coalesce=True, chunk_k=8, replicate_threshold=0.3, smem=True, cc_threshold=0.3,
                    degree_norm=True, degsim_threshold=0.5),
+    # N3: undirected sibling edges + max-weight rule (may merge SCCs, lighten the MST)
+    "n3": T.Knobs(coalesce=True, chunk_k=8, replicate_threshold=0.3, smem=True, cc_threshold=0.3,
+                  added_edge_budget=400, sibling_undirected=True, degree_norm=True, degsim_threshold=0.5,
+                  added_weight="max"),
 }
+E2_HOLDS = {"exact", "all"}     # directed 2-path edges preserve reachability
 
 
 def setup(gname, kname):
@@ -47,7 +52,8 @@ def test_scc_bit_exact(gname, kname):
     want = A.scc_tarjan(el)
     assert np.array_equal(got.astype(np.int64), want)
     # Theorem E2: the transforms preserve reachability -> same SCCs as G
-    assert np.array_equal(want, A.scc_tarjan(graph_to_edgelist(g)))
+    if kname in E2_HOLDS:
+        assert np.array_equal(want, A.scc_tarjan(graph_to_edgelist(g)))
 
 
 @pytest.mark.parametrize("gname", list(GRAPHS))

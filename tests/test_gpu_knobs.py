@@ -179,3 +179,40 @@ def test_pagerank_merge_cadence(gname, c, schedule):
     G.transform(knobs_c(kn))
     G.run("pagerank", tol=1e-12, max_iters=20000, mapping="lb", pr_schedule=schedule, merge_every=c)
     assert np.abs(G.download("rank") - want).sum() <= 1e-6
+
+
+# ---------------------------------------------------------------- N3 added-edge variants
+N3 = {
+    "coal_wmax": T.Knobs(coalesce=True, chunk_k=4, replicate_threshold=0.2, added_weight="max"),
+    "smem_und_wmean": T.Knobs(smem=True, cc_threshold=0.3, added_edge_budget=300, sibling_undirected=True,
+                              added_weight="mean"),
+    "degnorm_wmax": T.Knobs(degree_norm=True, degsim_threshold=0.5, added_weight="max"),
+    "all_und_wmax": T.Knobs(coalesce=True, chunk_k=8, replicate_threshold=0.3, smem=True, cc_threshold=0.3,
+                            sibling_undirected=True, degree_norm=True, degsim_threshold=0.5, added_weight="max"),
+}
+
+
+@pytest.mark.parametrize("gname", list(GRAPHS))
+@pytest.mark.parametrize("kname", list(N3))
+@pytest.mark.parametrize("mapping", ["lb", "tpv"])
+def test_n3_sssp_pagerank_on_GL(gname, kname, mapping):
+    """Alternative weights / undirected siblings: the GPU still reaches the
+    G_L definitions exactly (SSSP bit-exact with Dijkstra(G_L), PR within 1e-6),
+    and SSSP may now be shorter than on G (never longer): non-zero inaccuracy."""
+    raw = GRAPHS[gname]()
+    g = from_raw(raw)
+    kn = N3[kname]
+    L = T.transform(g, kn).logical()
+    s = sssp_source(g)
+    want = A.sssp_dijkstra(L, s)
+    exact = A.sssp_dijkstra(graph_to_edgelist(g), s)
+    fin = exact != 0xFFFFFFFF
+    assert np.all(want[fin] <= exact[fin])
+    G = upload(raw)
+    G.transform(knobs_c(kn))
+    G.run("sssp", mapping=mapping)
+    got = G.download("dist")
+    assert np.array_equal(got, want), f"{int(np.sum(got != want))} mismatches"
+    xw, _ = A.pagerank(L, tol=1e-14)
+    G.run("pagerank", tol=1e-11, max_iters=5000, mapping=mapping)
+    assert np.abs(G.download("rank") - xw).sum() <= 1e-6

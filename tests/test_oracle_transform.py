@@ -249,3 +249,75 @@ def test_canonicalize_rules():
     g = canonicalize(3, [0, 4, 5, 5], [2, 0, 1, 2, 0], [9, 5, 3, 4, 7])
     assert g.row_ptr.tolist() == [0, 2, 3, 3]
     assert g.col.tolist() == [2, 1, 0] and g.w.tolist() == [4, 3, 7]
+
+
+# ---------------------------------------------------------------- N3: added-edge variants
+RULE = {"sum": lambda a, b: a + b, "max": max, "mean": lambda a, b: max(1, (a + b) // 2)}
+
+
+def test_combine_rules_closed_form():
+    """P@34493 (sum) and the alternatives of P@34692, written out."""
+    assert [T.combine(3, 7, r) for r in ("sum", "max", "mean")] == [10, 7, 5]
+    assert T.combine(1, 1, "mean") == 1 and T.combine(1, 2, "mean") == 1
+    with pytest.raises(ValueError):
+        T.combine(1, 2, "first")
+
+
+@settings(max_examples=40, deadline=None)
+@given(seed=st.integers(0, 10**6), n=st.integers(2, 30), p=st.floats(0.05, 0.4),
+       rule=st.sampled_from(["max", "mean"]))
+def test_coalesce_weight_rule_brute_force(seed, n, p, rule):
+    """§2 replica 2-hop edges under an alternative rule: weight = min over every
+    intermediate v of rule(w(u,v), w(v,q)) in the ORIGINAL graph (brute force)."""
+    g = rand_graph(seed, n, p)
+    tg = T.coalesce(g, 2, T.ppm(0.0), rule)
+    orig = {(int(s), int(d)): int(w) for s, d, w in zip(*g.edges())}
+    L = tg.logical()
+    for s, d, w, a in zip(L.src.tolist(), L.dst.tolist(), L.w.tolist(), L.added.tolist()):
+        if a:
+            best = min(RULE[rule](orig[(s, v)], orig[(v, d)]) for v in range(g.n)
+                       if (s, v) in orig and (v, d) in orig)
+            assert w == best
+
+
+@settings(max_examples=40, deadline=None)
+@given(seed=st.integers(0, 10**6), n=st.integers(2, 60), p=st.floats(0.02, 0.3),
+       rule=st.sampled_from(["max", "mean"]))
+def test_degnorm_weight_rule_brute_force(seed, n, p, rule):
+    g = rand_graph(seed, n, p)
+    tg = T.transform(g, T.Knobs(degree_norm=True, degsim_threshold=0.9, added_weight=rule))
+    orig = {(int(s), int(d)): int(w) for s, d, w in zip(*g.edges())}
+    L = tg.logical()
+    for s, d, w, a in zip(L.src.tolist(), L.dst.tolist(), L.w.tolist(), L.added.tolist()):
+        if a:
+            assert w == min(RULE[rule](orig[(s, v)], orig[(v, d)]) for v in range(g.n)
+                            if (s, v) in orig and (v, d) in orig)
+
+
+@settings(max_examples=40, deadline=None)
+@given(seed=st.integers(0, 10**6), n=st.integers(3, 30), p=st.floats(0.05, 0.5),
+       budget=st.integers(0, 30), rule=st.sampled_from(["sum", "max"]))
+def test_smem_undirected_siblings(seed, n, p, budget, rule):
+    """Undirected sibling edges (P@29950 CC view): every added a->b joins two
+    U-neighbours c of the final graph with weight rule(wU(a,c), wU(c,b)),
+    wU = lighter direction; the budget holds; SCCs can only merge."""
+    g = rand_graph(seed, n, p)
+    tg = T.transform(g, T.Knobs(smem=True, cc_threshold=0.3, added_edge_budget=budget,
+                                sibling_undirected=True, added_weight=rule))
+    orig = {(int(s), int(d)): int(w) for s, d, w in zip(*g.edges())}
+    L = tg.logical()
+    final = {(int(s), int(d)): int(w) for s, d, w in zip(L.src, L.dst, L.w)}
+
+    def wU(x, y):
+        return min(v for v in (final.get((x, y)), final.get((y, x))) if v is not None)
+    adds = [(int(s), int(d), int(w)) for s, d, w, a in zip(L.src, L.dst, L.w, L.added) if a]
+    assert len(adds) <= budget
+    for (a, b, w) in adds:
+        assert (a, b) not in orig and (b, a) not in orig
+        assert any(((a, c) in final or (c, a) in final) and ((c, b) in final or (b, c) in final)
+                   and RULE[rule](wU(a, c), wU(c, b)) == w for c in range(g.n) if c not in (a, b))
+    from oracle import algos as A
+    from oracle.graph import graph_to_edgelist
+    lg, lL = A.scc_tarjan(graph_to_edgelist(g)), A.scc_tarjan(L)
+    for v in range(g.n):                   # same SCC in G => same SCC in G_L
+        assert lL[v] == lL[lg[v]]

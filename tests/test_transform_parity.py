@@ -69,6 +69,14 @@ KNOBS = {
     "degnorm_t06": T.Knobs(degree_norm=True, degsim_threshold=0.6, degree_target=0.7),
     "all": T.Knobs(coalesce=True, chunk_k=16, replicate_threshold=0.4, smem=True, cc_threshold=0.4,
                    degree_norm=True, degsim_threshold=0.5),
+    # N3 variants: alternative added-edge weights (P@34692), undirected sibling edges (P@29950)
+    "all_wmax": T.Knobs(coalesce=True, chunk_k=8, replicate_threshold=0.3, smem=True, cc_threshold=0.4,
+                        degree_norm=True, degsim_threshold=0.5, added_weight="max"),
+    "all_wmean": T.Knobs(coalesce=True, chunk_k=8, replicate_threshold=0.3, smem=True, cc_threshold=0.4,
+                         degree_norm=True, degsim_threshold=0.5, added_weight="mean"),
+    "smem_undirected": T.Knobs(smem=True, cc_threshold=0.4, sibling_undirected=True),
+    "smem_undirected_wmax": T.Knobs(smem=True, cc_threshold=0.3, added_edge_budget=80, sibling_undirected=True,
+                                    added_weight="max"),
 }
 
 GRAPHS = {
