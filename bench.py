@@ -217,7 +217,9 @@ def main():
     kern = {}
     for name, idx in (("k_sssp_lb", 0), ("k_pr_sell2", 1)):
         ms = sum(r[idx]["sweep_ms"] for r in runs)
-        nl = sum(r[idx]["sweep_launches"] for r in runs)
+        # sweeps that did work (a CUDA-graph / eager batch may launch a few
+        # more that return at once after convergence; their ~3 us stay in ms)
+        nl = sum(r[idx]["iterations"] for r in runs)
         by = sum(r[idx]["sweep_bytes"] for r in runs)
         kern[name] = {"ms_total": ms, "launches": nl, "bytes": by,
                       "gbs": by / (ms * 1e-3) / 1e9 if ms > 0 else None,
@@ -236,6 +238,15 @@ def main():
                 "traffic_unit": "bytes/launch (ncu dram read+write, profiles/latest)", "peak_source": peak_src,
                 "bytes_per_launch": dk["bytes"] / max(dk["launches"], 1),
                 "us_per_launch": 1e3 * dk["ms_total"] / max(dk["launches"], 1)}
+    if dom == "k_pr_sell2":
+        # the ceiling this kernel actually meets: random 4-byte contrib gathers
+        # through L1TEX (~1 wavefront/clk/SM); peak = tools/microbench4.cu LSU
+        # gathers from a 64 MB L2-resident vector (profiles/r1b)
+        gathers = sum(b["edges_scanned"] for _, b in runs)
+        g_rate = gathers / (dk["ms_total"] * 1e-3) / 1e9
+        roofline["secondary"] = {"bound": "l1tex random-gather wavefronts", "achieved": g_rate, "peak": 273.5,
+                                 "unit": "Ggather/s", "frac": g_rate / 273.5,
+                                 "peak_source": "measured, profiles/r1b/microbench4_tma_gather.txt"}
 
     a0, b0 = runs[-1]
     per_algo = {

@@ -393,6 +393,7 @@ __global__ void __launch_bounds__(256) k_pr_local(PrArgs a, const int32_t* __res
                                                   int64_t ntiles) {
   __shared__ double xs[256], xn[256], ext[256];
   __shared__ uint32_t Ds[256];
+  __shared__ int32_t smem_id[256];
   __shared__ uint8_t fixed[256];
   __shared__ double s_red[32];
   PrState* st = a.st;
@@ -412,18 +413,33 @@ __global__ void __launch_bounds__(256) k_pr_local(PrArgs a, const int32_t* __res
       fixed[i] = fx;
       xs[i] = a.x[v];
       Ds[i] = a.D[v];
-      ext[i] = fx ? 0.0 : (xs[i] - addc) / a.damp;    // sc * y_v of the sweep
+      smem_id[i] = v;
     }
     __syncthreads();
+    // external inflow of each member, gathered from the CSC with the values
+    // the contrib buffer holds now (sources outside the tile, or members that
+    // keep their values); scaled like the sweep's inputs.  Under the
+    // asynchronous schedule the sweep's own inputs are unknown (old or new), so
+    // recovering it as y_v - (in-tile part) would mix the two and can stall.
     for (int i = threadIdx.x; i < nm; i += blockDim.x) {
-      if (fixed[i]) continue;
-      double sub = 0.0;
-      for (int e = 0; e < ne; e++) {
-        const uint2 p = tedges[e0 + e];
-        const int s = p.x & 0xff, d = (p.x >> 8) & 0xff;
-        if (d == i && !fixed[s]) sub += (double)cin[tmem[b0 + s]];
+      if (fixed[i]) {
+        ext[i] = 0.0;
+        continue;
       }
-      ext[i] -= sc * sub;
+      const int32_t v = smem_id[i];
+      double in = 0.0;
+      for (uint32_t e = a.crp[v]; e < a.crp[v + 1]; e++) {
+        const int32_t u = a.csrc[e];
+        int lo = 0, hi = nm;   // members are sorted slot ids
+        while (lo < hi) {
+          const int mid = (lo + hi) >> 1;
+          if (smem_id[mid] < u) lo = mid + 1;
+          else hi = mid;
+        }
+        const bool inside = lo < nm && smem_id[lo] == u && !fixed[lo];
+        if (!inside) in += (double)cin[u];
+      }
+      ext[i] = sc * in;
     }
     __syncthreads();
     const int iters = titers[tile];

@@ -22,6 +22,8 @@
 #include <cmath>
 #include <cstdio>
 
+#include <cooperative_groups.h>
+
 #include "gx_internal.h"
 #include "kernels_common.cuh"
 #include "ktimer.h"
@@ -33,6 +35,7 @@
 #include <cstring>
 
 namespace gx {
+namespace cg = cooperative_groups;
 
 // ---------------------------------------------------------------- helpers
 __device__ __forceinline__ bool bit_of(const uint32_t* __restrict__ bm, uint32_t v) {
@@ -115,9 +118,9 @@ __device__ __forceinline__ void clear_bitmap(uint32_t* bm, int64_t nwords) {
 constexpr int SU = 4;         // edges in flight per lane per round
 constexpr int SB_WARPS = 8;   // warps per CTA
 
-__global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj,
-                                                 uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st,
-                                                 int64_t row_lo, int64_t row_hi) {
+__device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj,
+                                            uint32_t* __restrict__ dist, const SsspAux& ax, SsspState* __restrict__ st,
+                                            int64_t row_lo, int64_t row_hi) {
   __shared__ int32_t s_v[SB_WARPS][1024];
   const unsigned t = st->iter;
   if (st->stop) return;
@@ -244,6 +247,12 @@ __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp
   flush_counters(st, t, my_edges, my_act, my_push, my_min);
 }
 
+__global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj,
+                                                 uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st,
+                                                 int64_t row_lo, int64_t row_hi) {
+  sssp_lb_dev(rp, adj, dist, ax, st, row_lo, row_hi);
+}
+
 // ---------------------------------------------------------------- TPV sweep
 // The paper's mapping (tpv.cu): one warp per 32-slot slice of the schedule,
 // lane = slot; a lane whose slot is in the frontier walks its row in the
@@ -297,10 +306,10 @@ __global__ void __launch_bounds__(256) k_sssp_tpv(const int32_t* __restrict__ la
 // One CTA per subgraph tile: member distances staged in shared memory,
 // relaxed t times over the tile's local edges (P@32188-32416, reading R28),
 // improvements written back with atomic min and added to the next frontier.
-__global__ void __launch_bounds__(256) k_sssp_local(const int32_t* __restrict__ tptr, const int32_t* __restrict__ tmem,
-                                                    const int32_t* __restrict__ teptr, const uint2* __restrict__ tedges,
-                                                    const int32_t* __restrict__ titers, int64_t ntiles,
-                                                    uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st) {
+__device__ __forceinline__ void sssp_local_dev(const int32_t* __restrict__ tptr, const int32_t* __restrict__ tmem,
+                                               const int32_t* __restrict__ teptr, const uint2* __restrict__ tedges,
+                                               const int32_t* __restrict__ titers, int64_t ntiles,
+                                               uint32_t* __restrict__ dist, const SsspAux& ax, SsspState* __restrict__ st) {
   __shared__ uint32_t sd[256];
   const unsigned t = st->iter;
   if (st->stop) return;
@@ -352,16 +361,23 @@ __global__ void __launch_bounds__(256) k_sssp_local(const int32_t* __restrict__ 
   flush_counters(st, t, 0, 0, my_push, INF);
 }
 
+__global__ void __launch_bounds__(256) k_sssp_local(const int32_t* __restrict__ tptr, const int32_t* __restrict__ tmem,
+                                                    const int32_t* __restrict__ teptr, const uint2* __restrict__ tedges,
+                                                    const int32_t* __restrict__ titers, int64_t ntiles,
+                                                    uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st) {
+  sssp_local_dev(tptr, tmem, teptr, tedges, titers, ntiles, dist, ax, st);
+}
+
 // ---------------------------------------------------------------- §2.4 merge
 // One warp per confluence group.  The owner first re-pulls its in-edges (the
 // Jacobi step a merge may have undone), then all
 // copies take the mean (floor of the exact 64-bit mean, INF copies excluded,
 // reading R19) or the min (GX_MERGE_MIN).  Copies that decrease re-enter the
 // frontier.
-__global__ void __launch_bounds__(256) k_sssp_merge(const int32_t* __restrict__ gptr, const int32_t* __restrict__ gslots,
-                                                    const int32_t* __restrict__ ginptr, const uint2* __restrict__ gin,
-                                                    int64_t ngroups, int merge_min, uint32_t* __restrict__ dist,
-                                                    SsspAux ax, SsspState* __restrict__ st) {
+__device__ __forceinline__ void sssp_merge_dev(const int32_t* __restrict__ gptr, const int32_t* __restrict__ gslots,
+                                               const int32_t* __restrict__ ginptr, const uint2* __restrict__ gin,
+                                               int64_t ngroups, int merge_min, uint32_t* __restrict__ dist,
+                                               const SsspAux& ax, SsspState* __restrict__ st) {
   const unsigned t = st->iter;
   if (st->stop || !st->do_merge) return;
   uint32_t* bm_next = ax.bm[(t + 1) % 3];
@@ -412,23 +428,31 @@ __global__ void __launch_bounds__(256) k_sssp_merge(const int32_t* __restrict__ 
   flush_counters(st, t, 0, 0, my_push, INF);
 }
 
+__global__ void __launch_bounds__(256) k_sssp_merge(const int32_t* __restrict__ gptr, const int32_t* __restrict__ gslots,
+                                                    const int32_t* __restrict__ ginptr, const uint2* __restrict__ gin,
+                                                    int64_t ngroups, int merge_min, uint32_t* __restrict__ dist,
+                                                    SsspAux ax, SsspState* __restrict__ st) {
+  sssp_merge_dev(gptr, gslots, ginptr, gin, ngroups, merge_min, dist, ax, st);
+}
+
 // merge cadence c != 1 (P@28188: "after a certain number of iterations or at
 // the end of the overall computation"): decided once per iteration,
 // before the merge kernel, from the sweep's counters.  c > 1: merge after
 // every c-th iteration and whenever the sweep alone reached its fixed point
 // (so the run still ends at a merged fixed point); c = 0: only then, and that
 // merge ends the run (copies keep the mean; what it pushes is not relaxed).
-__global__ void k_sssp_merge_decide(SsspState* __restrict__ st) {
+__device__ __forceinline__ void sssp_merge_decide_dev(SsspState* __restrict__ st) {
   if (st->stop) return;
   const unsigned t = st->iter, c = st->merge_every;
   const bool fixed = st->pushed[t % 3] == 0 && st->far_min == INF;
   st->do_merge = ((c > 1 && ((t + 1) % c == 0 || fixed)) || (c == 0 && fixed)) ? 1u : 0u;
   st->final_merge = (c == 0 && fixed) ? 1u : 0u;
 }
+__global__ void k_sssp_merge_decide(SsspState* __restrict__ st) { sssp_merge_decide_dev(st); }
 
 // end of iteration t: no bit was set in the next frontier and the far pile is
 // empty => converged (every decreased slot has been relaxed)
-__global__ void k_sssp_advance(SsspState* __restrict__ st, int max_iters) {
+__device__ __forceinline__ void sssp_advance_dev(SsspState* __restrict__ st, int max_iters) {
   if (st->stop) return;
   const unsigned t = st->iter;
   if (st->final_merge) {
@@ -456,12 +480,13 @@ __global__ void k_sssp_advance(SsspState* __restrict__ st, int max_iters) {
   st->iter = t + 1;
   if ((int)(t + 1) >= max_iters) st->stop = 2;
 }
+__global__ void k_sssp_advance(SsspState* __restrict__ st, int max_iters) { sssp_advance_dev(st, max_iters); }
 
 // near-far refill (after k_sssp_advance raised tau): far slots of this rank's
 // range with dist < tau join the frontier of the new iteration; the rest stay
 // and re-establish far_min
-__global__ void k_sssp_split(const uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st, int64_t lo,
-                             int64_t hi) {
+__device__ __forceinline__ void sssp_split_dev(const uint32_t* __restrict__ dist, const SsspAux& ax,
+                                               SsspState* __restrict__ st, int64_t lo, int64_t hi) {
   if (st->stop || !st->split) return;
   const uint32_t tau = st->tau;
   uint32_t* bm_cur = ax.bm[st->iter % 3];
@@ -483,6 +508,64 @@ __global__ void k_sssp_split(const uint32_t* __restrict__ dist, SsspAux ax, Sssp
     if (move) bm_cur[w] |= move;
   }
   flush_counters(st, 0, 0, 0, 0, my_min);
+}
+__global__ void k_sssp_split(const uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st, int64_t lo,
+                             int64_t hi) {
+  sssp_split_dev(dist, ax, st, lo, hi);
+}
+
+// ---------------------------------------------------------------- persistent loop
+// The whole fixed-point loop of the LB mapping in ONE cooperative launch:
+// every phase of an iteration (sweep, §3 local pass, §2.4 merge, advance,
+// near-far refill) runs on the resident grid, separated by grid-wide
+// barriers, instead of 3-5 kernel launches per iteration.  What it removes is
+// the per-iteration fixed cost (launch gaps, kernel prologues), which is what
+// bounds high-diameter graphs: a road grid needs ~10^4 iterations whose
+// frontiers are a few thousand slots.  grid.sync() is a gpu-scope
+// release/acquire (MEMBAR.GPU + CCTL.IVALL in SASS), so every phase sees the
+// previous phase's writes; the loop state is read only after a barrier.
+struct SsspLoop {
+  const uint32_t* rp;
+  const uint2* adj;
+  uint32_t* dist;
+  SsspAux ax;
+  SsspState* st;
+  int64_t n_slots;
+  const int32_t *tptr, *tmem, *teptr, *titers;
+  const uint2* tedges;
+  int64_t ntiles;
+  const int32_t *gptr, *gslots, *ginptr;
+  const uint2* gin;
+  int64_t ngroups;
+  int merge_min, cadence, max_iters;
+};
+
+__global__ void __launch_bounds__(256) k_sssp_persist(SsspLoop a) {
+  cg::grid_group grid = cg::this_grid();
+  const bool lead = blockIdx.x == 0 && threadIdx.x == 0;
+  for (;;) {
+    if (*(volatile unsigned*)&a.st->stop) break;
+    sssp_lb_dev(a.rp, a.adj, a.dist, a.ax, a.st, 0, a.n_slots);
+    grid.sync();
+    if (a.ntiles) {
+      sssp_local_dev(a.tptr, a.tmem, a.teptr, a.tedges, a.titers, a.ntiles, a.dist, a.ax, a.st);
+      grid.sync();
+    }
+    if (a.ngroups) {
+      if (a.cadence) {
+        if (lead) sssp_merge_decide_dev(a.st);
+        grid.sync();
+      }
+      sssp_merge_dev(a.gptr, a.gslots, a.ginptr, a.gin, a.ngroups, a.merge_min, a.dist, a.ax, a.st);
+      grid.sync();
+    }
+    if (lead) sssp_advance_dev(a.st, a.max_iters);
+    grid.sync();
+    if (*(volatile unsigned*)&a.st->split) {
+      sssp_split_dev(a.dist, a.ax, a.st, 0, a.n_slots);
+      grid.sync();
+    }
+  }
 }
 
 __global__ void k_sssp_init(uint32_t* __restrict__ dist, const int32_t* __restrict__ slots, int nslots,
@@ -910,7 +993,46 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   // GX_SSSP_TRACE (profile runs): one stderr line per iteration --
   // iteration, frontier size, cumulative edges, tau, far_min, sweep-kernel ms
   const bool trace = o.profile && getenv("GX_SSSP_TRACE");
-  while (true) {
+  // LB mapping: the whole loop as one cooperative launch (k_sssp_persist);
+  // GX_SSSP_PERSIST=0 selects the per-kernel loop below (A/B, tracing)
+  int occp = 0, coop = 0;
+  CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occp, k_sssp_persist, 256, 0));
+  CUDA_OK(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, c->device));
+  const char* pe = getenv("GX_SSSP_PERSIST");
+  const bool persist = mapping == GX_MAP_LB && coop && occp > 0 && !trace && !(pe && atoi(pe) == 0);
+  if (persist) {
+    SsspLoop L;
+    L.rp = d.rp.as<uint32_t>();
+    L.adj = d.adj.as<uint2>();
+    L.dist = r.dist.as<uint32_t>();
+    L.ax = ax;
+    L.st = st;
+    L.n_slots = ns;
+    const bool tiles = d.n_tiles && g->knobs.smem;
+    L.tptr = d.t_ptr.as<int32_t>();
+    L.tmem = d.t_members.as<int32_t>();
+    L.teptr = d.t_eptr.as<int32_t>();
+    L.titers = d.t_iters.as<int32_t>();
+    L.tedges = d.t_edges.as<uint2>();
+    L.ntiles = tiles ? d.n_tiles : 0;
+    L.gptr = d.gptr.as<int32_t>();
+    L.gslots = d.gslots.as<int32_t>();
+    L.ginptr = d.g_in_ptr.as<int32_t>();
+    L.gin = d.g_in.as<uint2>();
+    L.ngroups = d.n_groups;
+    L.merge_min = merge_min ? 1 : 0;
+    L.cadence = o.merge_every != 1 ? 1 : 0;
+    L.max_iters = o.max_iters;
+    void* args[] = {&L};
+    kt.begin();
+    CUDA_OK(cudaLaunchCooperativeKernel((void*)k_sssp_persist, dim3((unsigned)(occp * c->num_sms)), dim3(256), args,
+                                        0, s));
+    kt.end();
+    launches += 1;
+    CUDA_OK(cudaMemcpyAsync(&hst, st, sizeof(SsspState), cudaMemcpyDeviceToHost, s));
+    CUDA_OK(cudaStreamSynchronize(s));
+  }
+  while (!persist) {
     if (gexec) {
       CUDA_OK(cudaGraphLaunch(gexec, s));
       launches += per_batch_launches;

@@ -16,6 +16,8 @@
 
 #include <algorithm>
 #include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cmath>
 #include <numeric>
 #include <unordered_map>
@@ -627,17 +629,30 @@ void degnorm(Work& W, int64_t th, int64_t f, bool combined, int wrule, std::vect
 
 void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out) {
   auto t0 = std::chrono::steady_clock::now();
+  // GX_TRANSFORM_TRACE=1: per-phase host times on stderr
+  const bool trace = getenv("GX_TRANSFORM_TRACE") != nullptr;
+  auto tp = t0;
+  auto phase = [&](const char* name) {
+    if (!trace) return;
+    auto now = std::chrono::steady_clock::now();
+    fprintf(stderr, "transform %-12s %8.1f ms\n", name, std::chrono::duration<double, std::milli>(now - tp).count());
+    tp = now;
+  };
   Work W;
   if (k.coalesce) coalesce(g, k.chunk_k, ppm(k.replicate_threshold), k.added_weight_rule, W);
   else identity(g, W);
+  phase(k.coalesce ? "coalesce" : "identity");
   SmemOut sm;
   if (k.smem) {
     Logical L;
     build_logical(W, L);
+    phase("logical+tri");
     const int64_t th = ppm(k.cc_threshold);
     const int64_t budget = k.added_edge_budget >= 0 ? k.added_edge_budget : g.m / 100;
     cc_edges(L, th, budget, k.added_weight_rule, k.sibling_undirected != 0, sm);
+    phase("cc_edges");
     subgraphs(L, th, k.smem_max_nodes, k.smem_iters, sm);
+    phase("subgraphs");
     for (auto& e : sm.added)
       W.rows[W.owner[std::get<0>(e)]].push_back({W.owner[std::get<1>(e)], std::get<2>(e), ADD_SMEM});
   }
@@ -645,6 +660,7 @@ void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out) {
   int64_t added_dn = 0;
   if (k.degree_norm)
     degnorm(W, ppm(k.degsim_threshold), ppm(k.degree_target), k.coalesce != 0, k.added_weight_rule, sched, added_dn);
+  phase("degnorm");
 
   // assemble the slot CSR, rows sorted by destination slot (R11)
   out = SlotGraph();
@@ -679,6 +695,7 @@ void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out) {
     out.tile_ptr.push_back((int64_t)out.tile_members.size());
     out.tile_iters.push_back(std::get<2>(t));
   }
+  phase("assemble");
   gx_transform_info& I = out.info;
   std::memset(&I, 0, sizeof(I));
   I.n_slots = W.n_slots;

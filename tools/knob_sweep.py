@@ -51,6 +51,9 @@ def graph_for(cfg, small):
     if cfg == "c4":
         n, m = ((1 << 22, 1 << 26) if small else (1 << 24, 1 << 28))
         return graphgen.uniform(n, m), f"uniform{n}x{m}"
+    if cfg == "c5":
+        s = 24 if small else 26
+        return graphgen.rmat(s), f"rmat{s}"
     raise ValueError(cfg)
 
 
@@ -69,12 +72,29 @@ def points(cfg):
                 for b in (0,)] + [(f"coalesce road t{t}", K(coalesce=True, replicate_threshold=t)) for t in (0.4, 0.6)]
     if cfg == "c4":
         return [(f"degnorm t{t}", K(degree_norm=True, degsim_threshold=t)) for t in (0.0, 0.1, 0.2, 0.3, 0.4, 0.5)]
+    if cfg == "c5":
+        return [("all three", K(coalesce=True, smem=True, degree_norm=True)),
+                ("all three aware-merge", K(coalesce=True, smem=True, degree_norm=True, merge_op=1))]
     raise ValueError(cfg)
+
+
+def c5_partitioned(G, tag, base):
+    """C5: the 1-D partitioned path at P = 1, 2, 4, 8 -- simulated ranks on one
+    GPU (each rank's sweep + the exchange as a device reduction), so these
+    times are the partitioned algorithm's cost on one device, not scaling."""
+    for P in (1, 2, 4, 8):
+        row = dict(base, knob=tag, P=P, note="simulated ranks on 1 GPU")
+        for algo in ("sssp", "pagerank"):
+            kw = {"tol": 1e-9} if algo == "pagerank" else {}
+            r = G.run(algo, mapping="lb", sim_ranks=P if P > 1 else 0, **kw)
+            row[f"{algo}_ms"] = r["loop_ms"]
+            row[f"{algo}_iters"] = r["iterations"]
+        print(json.dumps(row), flush=True)
 
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--config", default="c1", choices=["c1", "c2", "c3", "c4"])
+    ap.add_argument("--config", default="c1", choices=["c1", "c2", "c3", "c4", "c5"])
     ap.add_argument("--scale-down", action="store_true")
     ap.add_argument("--budgets", default="0,0.1,0.5,1,2,5")
     a = ap.parse_args()
@@ -90,6 +110,8 @@ def main():
     d0 = G.download("dist")
     G.run("pagerank", mapping="lb", tol=1e-9)
     x0 = G.download("rank")
+    if a.config == "c5":
+        c5_partitioned(G, "exact", {"graph": gname, "n": G.n, "m": m, "config": "c5"})
     pts = points(a.config)
     if a.config == "c3":
         pts = [(f"smem t0.5 budget {b}%", gx.Knobs(smem=True, cc_threshold=0.5, added_edge_budget=int(float(b) / 100 * m)))
@@ -122,6 +144,8 @@ def main():
             else:
                 row["pr_inacc_pct"] = inacc(G.download("rank"), x0)
         print(json.dumps(row), flush=True)
+        if a.config == "c5":
+            c5_partitioned(G, name, base)
         G.transform(None)
 
 
