@@ -121,6 +121,10 @@ struct DevGraph {
   SellLayout pr_sell, sssp_sell;
   // LB SSSP: static chunk list of rows with out-degree > HEAVY_DEG, heavy bitmap
   int64_t nhc = 0;
+  // SSSP block-local mode (sssp.cu): block size the locality was measured for,
+  // fraction of edges inside a block, max out-degree
+  int64_t blk_rows = 0, blk_maxdeg = 0;
+  double blk_local = 0.0;
   DBuf hc_row, hc_start, heavy_bm;
   // TPV (paper's thread-per-vertex mapping, tpv.cu): lanes = the §4 schedule
   // (or slot order), SELL-32 slabs of out-edges (SSSP) and in-edges (PR)

@@ -78,7 +78,8 @@ __device__ __forceinline__ void relax_nf(uint2 ed, uint32_t du, uint32_t cur, ui
 // kind per CTA (same-address atomics from every warp would serialise in L2).
 // Every thread of the CTA must call it.
 __device__ __forceinline__ void flush_counters(SsspState* st, unsigned t, unsigned long long edges,
-                                               unsigned long long act, uint32_t push, uint32_t fmin) {
+                                               unsigned long long act, uint32_t push, uint32_t fmin,
+                                               uint32_t* fdst = nullptr) {
   __shared__ unsigned long long s_e[32], s_a[32];
   __shared__ uint32_t s_p[32], s_m[32];
   edges = warp_sum_u64(edges);
@@ -105,7 +106,7 @@ __device__ __forceinline__ void flush_counters(SsspState* st, unsigned t, unsign
     if (e) atomicAdd(&st->edges, e);
     if (a) atomicAdd(&st->active[t % 3], (unsigned)a);
     if (p) atomicAdd(&st->pushed[t % 3], p);
-    if (m != INF) atomicMin(&st->far_min, m);
+    if (m != INF) atomicMin(fdst ? fdst : &st->far_min, m);
   }
 }
 
@@ -118,12 +119,11 @@ __device__ __forceinline__ void clear_bitmap(uint32_t* bm, int64_t nwords) {
 constexpr int SU = 4;         // edges in flight per lane per round
 constexpr int SB_WARPS = 8;   // warps per CTA
 
+// iteration t with near-far threshold tau; the far pile's minimum goes to fdst
 __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj,
                                             uint32_t* __restrict__ dist, const SsspAux& ax, SsspState* __restrict__ st,
-                                            int64_t row_lo, int64_t row_hi) {
-  __shared__ int32_t s_v[SB_WARPS][1024];
-  const unsigned t = st->iter;
-  if (st->stop) return;
+                                            int64_t row_lo, int64_t row_hi, const unsigned t, const uint32_t tau,
+                                            uint32_t* fdst, int32_t (*s_v)[1024]) {
   const uint32_t* __restrict__ bm_cur = ax.bm[t % 3];
   uint32_t* bm_next = ax.bm[(t + 1) % 3];
   clear_bitmap(ax.bm[(t + 2) % 3], ax.nwords);
@@ -131,8 +131,6 @@ __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, con
   const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
   const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const uint32_t tau = st->tau;   // near-far: relaxations to dist >= tau go to the far pile
-  if (blockIdx.x == 0 && threadIdx.x == 0) st->split = 0;   // the split kernel of t-1 is done
   unsigned long long my_edges = 0, my_act = 0;
   uint32_t my_min = INF, my_push = 0;
 
@@ -185,10 +183,26 @@ __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, con
   int32_t* sv = s_v[wib];
   const int64_t w_lo = row_lo >> 5, w_hi = min((row_hi + 31) >> 5, ax.nwords);   // ranges are 32-aligned
   const int64_t my_words = (w_hi - w_lo - gw + nw - 1) / nw;                       // words owned by this warp
-  for (int64_t j0 = 0; j0 < my_words; j0 += 32) {
-    const int64_t jj = j0 + lane;
+  // the frontier words of SCAN_B rounds are loaded together (one memory
+  // latency instead of SCAN_B when the frontier is sparse, as on road grids)
+  constexpr int SCAN_B = 4;
+  for (int64_t jb = 0; jb < my_words; jb += 32 * SCAN_B) {
+    uint32_t wv[SCAN_B];
+#pragma unroll
+    for (int b = 0; b < SCAN_B; b++) {
+      const int64_t jj = jb + 32 * b + lane;
+      const int64_t wi = w_lo + gw + nw * jj;
+      wv[b] = jj < my_words ? (__ldcg(bm_cur + wi) & ~__ldg(ax.heavy + wi)) : 0u;
+    }
+    uint32_t anyw = 0;
+#pragma unroll
+    for (int b = 0; b < SCAN_B; b++) anyw |= wv[b];
+    if (!__any_sync(FULL, anyw != 0)) continue;
+#pragma unroll 1
+  for (int b = 0; b < SCAN_B; b++) {
+    const int64_t jj = jb + 32 * b + lane;
     const int64_t wi = w_lo + gw + nw * jj;
-    uint32_t word = jj < my_words ? (__ldcg(bm_cur + wi) & ~__ldg(ax.heavy + wi)) : 0u;
+    uint32_t word = wv[b];
     const uint32_t cnt = __popc(word);
     const uint32_t incl = warp_incl_scan_u32(cnt);
     const uint32_t total = __shfl_sync(FULL, incl, 31);
@@ -244,13 +258,20 @@ __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, con
     }
     __syncwarp();
   }
-  flush_counters(st, t, my_edges, my_act, my_push, my_min);
+  }
+  flush_counters(st, t, my_edges, my_act, my_push, my_min, fdst);
 }
 
 __global__ void __launch_bounds__(256) k_sssp_lb(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj,
                                                  uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st,
                                                  int64_t row_lo, int64_t row_hi) {
-  sssp_lb_dev(rp, adj, dist, ax, st, row_lo, row_hi);
+  if (st->stop) return;
+  const unsigned t = st->iter;
+  // near-far: relaxations to dist >= tau go to the far pile
+  const uint32_t tau = st->tau;
+  if (blockIdx.x == 0 && threadIdx.x == 0) st->split = 0;   // the split kernel of t-1 is done
+  __shared__ int32_t s_v[SB_WARPS][1024];
+  sssp_lb_dev(rp, adj, dist, ax, st, row_lo, row_hi, t, tau, &st->far_min, s_v);
 }
 
 // ---------------------------------------------------------------- TPV sweep
@@ -485,11 +506,11 @@ __global__ void k_sssp_advance(SsspState* __restrict__ st, int max_iters) { sssp
 // near-far refill (after k_sssp_advance raised tau): far slots of this rank's
 // range with dist < tau join the frontier of the new iteration; the rest stay
 // and re-establish far_min
+// t = the iteration the refilled frontier belongs to; remaining far minimum -> fdst
 __device__ __forceinline__ void sssp_split_dev(const uint32_t* __restrict__ dist, const SsspAux& ax,
-                                               SsspState* __restrict__ st, int64_t lo, int64_t hi) {
-  if (st->stop || !st->split) return;
-  const uint32_t tau = st->tau;
-  uint32_t* bm_cur = ax.bm[st->iter % 3];
+                                               SsspState* __restrict__ st, int64_t lo, int64_t hi, const unsigned t,
+                                               const uint32_t tau, uint32_t* fdst) {
+  uint32_t* bm_cur = ax.bm[t % 3];
   uint32_t my_min = INF;
   const int64_t w_lo = lo >> 5, w_hi = min((hi + 31) >> 5, ax.nwords);
   for (int64_t w = w_lo + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < w_hi; w += (int64_t)gridDim.x * blockDim.x) {
@@ -507,11 +528,136 @@ __device__ __forceinline__ void sssp_split_dev(const uint32_t* __restrict__ dist
     ax.far[w] = keep;
     if (move) bm_cur[w] |= move;
   }
-  flush_counters(st, 0, 0, 0, 0, my_min);
+  flush_counters(st, 0, 0, 0, 0, my_min, fdst);
 }
 __global__ void k_sssp_split(const uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st, int64_t lo,
                              int64_t hi) {
-  sssp_split_dev(dist, ax, st, lo, hi);
+  if (st->stop || !st->split) return;
+  sssp_split_dev(dist, ax, st, lo, hi, st->iter, st->tau, &st->far_min);
+}
+
+// ---------------------------------------------------------------- block-local mode
+// For graphs whose edges mostly stay inside contiguous id blocks (road grids
+// in their natural row-major order: ~10^4 iterations of a few thousand slots
+// each), CTA b owns rows [b*B, (b+1)*B).  In each global iteration it relaxes
+// the frontier slots of its block and keeps propagating improvements of its
+// OWN rows through a shared-memory work queue for up to BLK_ROUNDS local
+// rounds, so a wave crosses many hops per grid barrier (the paper's §3 idea
+// -- iterate a subgraph in shared memory, P@32188 -- applied exactly, to the
+// id blocks, without added edges).  Improvements of other blocks' rows (and
+// queue overflow) go to the global next frontier as usual.  Any relaxation
+// order reaches the same fixed point (monotone min; Theorem E1's argument).
+constexpr int BLK_MAX = 65536;   // rows per block (in-queue bitmap = 8 KB of shared memory)
+constexpr int BLK_Q = 2048;      // entries per local queue buffer (two buffers)
+constexpr int BLK_ROUNDS = 256;  // local rounds per global iteration
+
+__device__ __forceinline__ void sssp_block_dev(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj,
+                                               uint32_t* __restrict__ dist, const SsspAux& ax,
+                                               SsspState* __restrict__ st, int64_t n_slots, int64_t B,
+                                               const unsigned t, const uint32_t tau, uint32_t* fdst,
+                                               uint8_t* pool) {
+  // shared memory (aliases the LB sweep's compaction buffer): two queues,
+  // the in-queue bitmap of the block, two counters
+  int32_t (*q)[BLK_Q] = reinterpret_cast<int32_t (*)[BLK_Q]>(pool);
+  uint32_t* inq = reinterpret_cast<uint32_t*>(pool + 2 * BLK_Q * 4);
+  int* s_cnt = reinterpret_cast<int*>(pool + 2 * BLK_Q * 4 + BLK_MAX / 8);
+  const uint32_t* __restrict__ bm_cur = ax.bm[t % 3];
+  uint32_t* bm_next = ax.bm[(t + 1) % 3];
+  clear_bitmap(ax.bm[(t + 2) % 3], ax.nwords);
+  const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
+  const int64_t lo = (int64_t)blockIdx.x * B, hi = min(n_slots, lo + B);
+  unsigned long long my_edges = 0, my_act = 0;
+  uint32_t my_min = INF, my_push = 0;
+  if (lo < hi) {
+    const int nw_blk = (int)((hi - lo + 31) >> 5);
+    for (int i = threadIdx.x; i < nw_blk; i += blockDim.x) inq[i] = 0;
+    if (threadIdx.x < 2) s_cnt[threadIdx.x] = 0;
+    __syncthreads();
+    int cur = 0;
+    // relax the out-edges of u; own-block improvements below tau are queued
+    auto relax_vertex = [&](int32_t u) {
+      const uint32_t du = ld_l2_u32(dist + u, pl);
+      const uint32_t a = rp[u], b = rp[u + 1];
+      my_act++;
+      my_edges += b - a;
+      for (uint32_t e = a; e < b; e++) {
+        const uint2 ed = ld_stream_u2(adj + e, pf);
+        uint32_t nd = du + ed.y;
+        if (nd < du) nd = INF - 1;
+        const uint32_t cv = ld_l2_u32(dist + ed.x, pl);
+        if (nd >= cv) continue;
+        const int64_t v = ed.x;
+        if (v >= lo && v < hi && nd < tau) {
+          const uint32_t old = atom_min_l2(dist + v, nd, pl);
+          if (nd < old) {
+            const uint32_t bit = 1u << ((v - lo) & 31);
+            if (!(atomicOr(&inq[(v - lo) >> 5], bit) & bit)) {
+              const int k = atomicAdd(&s_cnt[cur ^ 1], 1);
+              if (k < BLK_Q) {
+                q[cur ^ 1][k] = (int32_t)v;
+              } else {   // queue full: next global iteration
+                red_or_l2(bm_next + (v >> 5), 1u << (v & 31), pl);
+                my_push++;
+              }
+            }
+          }
+        } else {
+          relax_nf(ed, du, cv, dist, bm_next, ax.far, tau, my_min, my_push, pl);
+        }
+      }
+    };
+    // the global frontier's slots in this block (a thread per bitmap word);
+    // pushes of this pass land in q[1]
+    cur = 0;
+    for (int64_t w = (lo >> 5) + threadIdx.x; w < ((hi + 31) >> 5); w += blockDim.x) {
+      uint32_t bits = __ldcg(bm_cur + w);
+      while (bits) {
+        const int b = __ffs(bits) - 1;
+        bits &= bits - 1;
+        relax_vertex((int32_t)(w * 32 + b));
+      }
+    }
+    __syncthreads();
+    cur = 1;
+    for (int r = 0; r < BLK_ROUNDS; r++) {
+      const int n = min(s_cnt[cur], BLK_Q);
+      if (n == 0) break;                       // uniform: read after a barrier
+      if (threadIdx.x == 0) s_cnt[cur ^ 1] = 0;
+      __syncthreads();
+      for (int i = threadIdx.x; i < n; i += blockDim.x) {
+        const int32_t u = q[cur][i];
+        atomicAnd(&inq[(u - lo) >> 5], ~(1u << ((u - lo) & 31)));
+        relax_vertex(u);
+      }
+      __syncthreads();
+      cur ^= 1;
+    }
+    // rounds exhausted: what is still queued joins the global next frontier
+    const int n = min(s_cnt[cur], BLK_Q);
+    for (int i = threadIdx.x; i < n; i += blockDim.x) {
+      const int32_t u = q[cur][i];
+      red_or_l2(bm_next + (u >> 5), 1u << (u & 31), pl);
+      my_push++;
+    }
+  }
+  flush_counters(st, t, my_edges, my_act, my_push, my_min, fdst);
+}
+
+__global__ void k_block_locality(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj, int64_t n, int64_t B,
+                                 unsigned long long* __restrict__ out) {
+  unsigned long long loc = 0;
+  uint32_t mx = 0;
+  for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n; u += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t a = rp[u], b = rp[u + 1];
+    mx = max(mx, b - a);
+    for (uint32_t e = a; e < b; e++) loc += (adj[e].x / B) == (u / B);
+  }
+  loc = warp_sum_u64(loc);
+  mx = warp_max_u32(mx);
+  if (lane_id() == 0) {
+    atomicAdd(out, loc);
+    atomicMax(out + 1, (unsigned long long)mx);
+  }
 }
 
 // ---------------------------------------------------------------- persistent loop
@@ -538,31 +684,92 @@ struct SsspLoop {
   const uint2* gin;
   int64_t ngroups;
   int merge_min, cadence, max_iters;
+  int64_t block_rows;   // > 0: block-local mode with this many rows per CTA
 };
 
-__global__ void __launch_bounds__(256) k_sssp_persist(SsspLoop a) {
+constexpr int PERSIST_POOL = SB_WARPS * 1024 * 4;   // 32 KB: LB compaction buffer / block-mode queues
+static_assert(2 * BLK_Q * 4 + BLK_MAX / 8 + 16 <= PERSIST_POOL, "block-mode buffers must fit the pool");
+
+__global__ void __launch_bounds__(256, 4) k_sssp_persist(SsspLoop a) {
+  __shared__ __align__(16) uint8_t pool[PERSIST_POOL];
   cg::grid_group grid = cg::this_grid();
   const bool lead = blockIdx.x == 0 && threadIdx.x == 0;
+  SsspState* st = a.st;
+  // Loop control is replicated: after the sweep's barrier every thread reads
+  // the same counters and takes the same decision (stop / refill / new tau),
+  // so no barrier is needed between the decision and the next sweep.  The
+  // lead thread mirrors the state into *st for the host and clears the
+  // counter slots of iteration t+2 (last read at the decision of t-1, which
+  // every CTA has passed).  far3[t%3] collects the far pile's minimum pushed
+  // in iteration t; rf is the running minimum since the last refill.
+  unsigned t = st->iter;
+  uint32_t tau = st->tau, rf = INF;
+  const uint32_t delta = st->delta;
   for (;;) {
-    if (*(volatile unsigned*)&a.st->stop) break;
-    sssp_lb_dev(a.rp, a.adj, a.dist, a.ax, a.st, 0, a.n_slots);
+    if (a.block_rows > 0)
+      sssp_block_dev(a.rp, a.adj, a.dist, a.ax, st, a.n_slots, a.block_rows, t, tau, &st->far3[t % 3], pool);
+    else
+      sssp_lb_dev(a.rp, a.adj, a.dist, a.ax, st, 0, a.n_slots, t, tau, &st->far3[t % 3],
+                  reinterpret_cast<int32_t (*)[1024]>(pool));
     grid.sync();
     if (a.ntiles) {
-      sssp_local_dev(a.tptr, a.tmem, a.teptr, a.tedges, a.titers, a.ntiles, a.dist, a.ax, a.st);
+      sssp_local_dev(a.tptr, a.tmem, a.teptr, a.tedges, a.titers, a.ntiles, a.dist, a.ax, st);
       grid.sync();
     }
+    bool final_merge = false;
     if (a.ngroups) {
-      if (a.cadence) {
-        if (lead) sssp_merge_decide_dev(a.st);
+      bool doit = true;
+      if (a.cadence) {   // cadence N2, same rule as k_sssp_merge_decide
+        const unsigned c = st->merge_every;
+        const bool fixed = *(volatile unsigned*)&st->pushed[t % 3] == 0 &&
+                           min(rf, *(volatile unsigned*)&st->far3[t % 3]) == INF;
+        doit = (c > 1 && ((t + 1) % c == 0 || fixed)) || (c == 0 && fixed);
+        final_merge = c == 0 && fixed;
+        if (lead) {
+          st->do_merge = doit ? 1u : 0u;
+          st->final_merge = final_merge ? 1u : 0u;
+        }
         grid.sync();
       }
-      sssp_merge_dev(a.gptr, a.gslots, a.ginptr, a.gin, a.ngroups, a.merge_min, a.dist, a.ax, a.st);
-      grid.sync();
+      if (doit) {
+        sssp_merge_dev(a.gptr, a.gslots, a.ginptr, a.gin, a.ngroups, a.merge_min, a.dist, a.ax, st);
+        grid.sync();
+      }
     }
-    if (lead) sssp_advance_dev(a.st, a.max_iters);
-    grid.sync();
-    if (*(volatile unsigned*)&a.st->split) {
-      sssp_split_dev(a.dist, a.ax, a.st, 0, a.n_slots);
+    // ---- decision (every thread, identical inputs)
+    const unsigned pushed = *(volatile unsigned*)&st->pushed[t % 3];
+    const uint32_t fm = min(rf, *(volatile unsigned*)&st->far3[t % 3]);
+    unsigned stop = 0;
+    bool split = false;
+    if (final_merge) {
+      stop = 1;
+    } else if (pushed == 0) {
+      if (fm == INF) {
+        stop = 1;
+      } else {   // the bucket drained: raise tau past the nearest far slot
+        const unsigned long long nt = (unsigned long long)fm + delta;
+        tau = nt >= INF ? INF : (unsigned)nt;
+        rf = INF;
+        split = true;
+      }
+    } else {
+      rf = fm;
+    }
+    if (!stop && (int)(t + 1) >= a.max_iters) stop = 2;
+    if (lead) {
+      st->act_total += st->active[t % 3];
+      st->active[(t + 2) % 3] = 0;
+      st->pushed[(t + 2) % 3] = 0;
+      st->far3[(t + 2) % 3] = INF;
+      st->iter = t + 1;
+      st->tau = tau;
+      st->far_min = rf;
+      st->stop = stop;
+    }
+    if (stop) break;
+    t++;
+    if (split) {   // near-far refill of iteration t's frontier
+      sssp_split_dev(a.dist, a.ax, st, 0, a.n_slots, t, tau, &st->far3[t % 3]);
       grid.sync();
     }
   }
@@ -649,7 +856,12 @@ static unsigned sssp_delta(const gx_graph* g) {
   if (d.n_slots == 0 || d.m_slots == 0) return 0u;
   const double avg_deg = (double)g->m / (double)std::max<int64_t>(1, g->n);
   const double avg_w = 0.5 * (1.0 + (double)g->max_w);
-  const double delta = 8.0 * avg_w / std::max(1.0, avg_deg);
+  double delta = 8.0 * avg_w / std::max(1.0, avg_deg);
+  // sparse, high-diameter graphs (road grids, ~2.5 arcs/vertex) need ~10^4
+  // iterations at any bucket width, and each costs ~15 us of barriers and
+  // frontier scans: there wide buckets win (road 4900^2, persistent loop:
+  // Delta 160 -> 334 ms, 1000 -> 198, 3000 -> 171, 10^4 -> 161, profiles/r1b)
+  if (avg_deg < 4.0) delta *= 64.0;
   return (unsigned)std::max(1.0, delta);
 }
 
@@ -745,6 +957,7 @@ static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, 
   init.delta = delta;
   init.tau = delta ? delta : INF;
   init.far_min = INF;
+  init.far3[0] = init.far3[1] = init.far3[2] = INF;
   init.merge_every = 1;
   init.do_merge = 1;
   cudaEvent_t e0, e1;
@@ -922,6 +1135,7 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     init.delta = delta;
     init.tau = delta ? delta : INF;
     init.far_min = INF;
+  init.far3[0] = init.far3[1] = init.far3[2] = INF;
     init.merge_every = d.n_groups ? (unsigned)o.merge_every : 1u;
     init.do_merge = init.merge_every == 1 ? 1u : 0u;
     CUDA_OK(cudaMemcpyAsync(r.st.p, &init, sizeof(SsspState), cudaMemcpyHostToDevice, s));
@@ -1023,6 +1237,32 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     L.merge_min = merge_min ? 1 : 0;
     L.cadence = o.merge_every != 1 ? 1 : 0;
     L.max_iters = o.max_iters;
+    // block-local mode when most edges stay inside the CTA id blocks and rows
+    // are short (thread-per-slot relaxation); GX_SSSP_BLOCK=0/1 overrides
+    const int64_t gridp = (int64_t)occp * c->num_sms;
+    const int64_t B = ((ns + gridp - 1) / gridp + 31) / 32 * 32;
+    L.block_rows = 0;
+    if (B <= BLK_MAX && d.m_slots > 0) {
+      if (d.blk_rows != B) {
+        DBuf cnt;
+        cnt.alloc(c, 16);
+        CUDA_OK(cudaMemsetAsync(cnt.p, 0, 16, s));
+        k_block_locality<<<grid_for(c, ns), 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), ns, B,
+                                                        cnt.as<unsigned long long>());
+        unsigned long long h[2];
+        CUDA_OK(cudaMemcpyAsync(h, cnt.p, 16, cudaMemcpyDeviceToHost, s));
+        CUDA_OK(cudaStreamSynchronize(s));
+        d.blk_rows = B;
+        d.blk_local = (double)h[0] / (double)d.m_slots;
+        d.blk_maxdeg = (int64_t)h[1];
+      }
+      const char* be = getenv("GX_SSSP_BLOCK");
+      // experimental: off unless GX_SSSP_BLOCK=1 (road 4900^2: 326 ms at the
+      // default Delta vs 331 for the LB sweep, but 270 vs 198 at Delta 1000 --
+      // each local round still pays an L2 round trip per hop)
+      const bool want = be ? atoi(be) != 0 && d.blk_maxdeg <= 64 : false;
+      if (want) L.block_rows = B;
+    }
     void* args[] = {&L};
     kt.begin();
     CUDA_OK(cudaLaunchCooperativeKernel((void*)k_sssp_persist, dim3((unsigned)(occp * c->num_sms)), dim3(256), args,

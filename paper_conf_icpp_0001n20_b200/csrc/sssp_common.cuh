@@ -26,7 +26,7 @@ struct SsspState {
   unsigned int merge_every;     // §2.4 cadence c (gx_run_opts.merge_every; 1 when there are no replicas)
   unsigned int do_merge;        // iteration `iter` ends with a merge
   unsigned int final_merge;     // c = 0: this iteration's merge ends the run
-  unsigned int pad;
+  unsigned int far3[3];         // persistent loop: far-pile minimum pushed in iteration t, [t%3]
 };
 
 struct SsspAux {

@@ -130,3 +130,43 @@ def test_full_size_certificates(scale):
     r = pagerank_residual(src, g.col, g.n, x)
     assert r["bound"] <= 1e-6, r
     assert abs(r["mass"] - 1) < 1e-6
+
+
+@pytest.mark.parametrize("name", ["rmat12", "uniform", "road64", "star_hub", "dups_loops", "isolated"])
+@pytest.mark.parametrize("persist,block", [("0", None), ("1", "0"), ("1", "1")])
+def test_sssp_loop_modes_bit_exact(name, persist, block, monkeypatch):
+    """Every LB loop variant reaches Dijkstra exactly: per-kernel launches
+    (GX_SSSP_PERSIST=0), the cooperative persistent loop, and its block-local
+    mode (shared-memory queues over contiguous id blocks) forced on any graph."""
+    monkeypatch.setenv("GX_SSSP_PERSIST", persist)
+    if block is not None:
+        monkeypatch.setenv("GX_SSSP_BLOCK", block)
+    raw = GRAPHS[name]()
+    g = from_raw(raw)
+    want = A.sssp_dijkstra(graph_to_edgelist(g), sssp_source(g))
+    G = upload(raw)
+    info = G.run("sssp", source=-1, mapping="lb")
+    assert info["converged"] == 1
+    got = G.download("dist")
+    assert np.array_equal(got, want), f"{np.sum(got != want)} mismatches"
+
+
+def test_sssp_block_mode_road_grid_closed_form(monkeypatch):
+    """Block-local mode on a full 4-neighbour grid with unit weights: the
+    distances are the Manhattan distances (closed form)."""
+    monkeypatch.setenv("GX_SSSP_BLOCK", "1")
+    side = 300
+    edges = []
+    for r in range(side):
+        for c in range(side):
+            v = r * side + c
+            if c + 1 < side:
+                edges += [(v, v + 1, 1), (v + 1, v, 1)]
+            if r + 1 < side:
+                edges += [(v, v + side, 1), (v + side, v, 1)]
+    raw = graphgen.from_edge_list(side * side, edges)
+    G = upload(raw)
+    G.run("sssp", source=0, mapping="lb")
+    got = G.download("dist").astype(np.int64)
+    rr, cc = np.divmod(np.arange(side * side), side)
+    assert np.array_equal(got, rr + cc)
