@@ -27,6 +27,18 @@
 namespace gx {
 namespace {
 
+// GX_TRANSFORM_TRACE=1: sub-phase times on stderr
+struct PhaseTimer {
+  bool on = getenv("GX_TRANSFORM_TRACE") != nullptr;
+  std::chrono::steady_clock::time_point t = std::chrono::steady_clock::now();
+  void operator()(const char* name) {
+    if (!on) return;
+    auto now = std::chrono::steady_clock::now();
+    fprintf(stderr, "  %-22s %8.1f ms\n", name, std::chrono::duration<double, std::milli>(now - t).count());
+    t = now;
+  }
+};
+
 // Weight of an added edge standing for the 2-hop path with hop weights w1, w2
 // (gx_knobs.added_weight_rule): the sum (P@34493, R17) or one of
 // the "alternative" rules P@34692 allows.
@@ -128,7 +140,9 @@ void renumber(const HostCSR& g, int k, std::vector<int32_t>& nw, int64_t& n_slot
               std::vector<std::pair<int64_t, int64_t>>& ranges) {
   const int64_t n = g.n;
   std::vector<int32_t> sources, level;
+  PhaseTimer pt;
   bfs_forest(g, sources, level);
+  pt("bfs_forest+levels");
   nw.assign(n, -1);
   for (size_t i = 0; i < sources.size(); i++) nw[sources[i]] = (int32_t)i;
   int64_t gid = (int64_t)sources.size();
@@ -177,6 +191,7 @@ void renumber(const HostCSR& g, int k, std::vector<int32_t>& nw, int64_t& n_slot
     i++;
   }
   n_slots = n > 0 ? (gid + k - 1) / k * k : 0;
+  pt("cursor numbering");
 }
 
 // Renumber + ReplicateVertex (Alg 2 l.21-35), readings R10-R18.
@@ -186,6 +201,7 @@ void coalesce(const HostCSR& g, int k, int64_t theta_ppm, int wrule, Work& W) {
   std::vector<std::pair<int64_t, int64_t>> ranges;
   int64_t n_slots = 0;
   renumber(g, k, nw, n_slots, ranges);
+  PhaseTimer pt;
   W.n = n;
   W.n_slots = n_slots;
   W.slot_to_orig.assign(n_slots, -1);
@@ -204,6 +220,7 @@ void coalesce(const HostCSR& g, int k, int64_t theta_ppm, int wrule, Work& W) {
     r.reserve(g.rp[u + 1] - g.rp[u]);
     for (int64_t e = g.rp[u]; e < g.rp[u + 1]; e++) r.push_back({nw[g.col[e]], g.w[e], ADD_NONE});
   }
+  pt("relabelled adjacency");
   std::vector<int32_t> nonhole((n_slots + k - 1) / k, 0);
   for (int64_t s = 0; s < n_slots; s++)
     if (W.kind[s] != HOLE) nonhole[s / k]++;
@@ -222,28 +239,53 @@ void coalesce(const HostCSR& g, int k, int64_t theta_ppm, int wrule, Work& W) {
     if (holes <= 0) continue;
     for (int64_t C = ranges[li].first / k; C <= (ranges[li].second - 1) / k; C++) chunk_lv[C] = (int32_t)li;
   }
-  // count (slot, chunk) pairs over edges into those chunks
-  std::vector<std::pair<int64_t, int32_t>> pairs;  // (C, s)
-  for (int64_t s = 0; s < n_slots; s++)
-    for (const Edge& e : radj[s]) {
-      const int64_t C = e.dst / k;
-      if (chunk_lv[C] >= 0) pairs.push_back({C, (int32_t)s});
+  // candidates (-count, s, C) per level: count the chunks of each row (rows
+  // are short), in parallel over slots; since a level has h <= k-1 holes only
+  // the h smallest candidates of each level matter, and the global h smallest
+  // are among every thread's h smallest -- each thread keeps a bounded list
+  using Cand = std::tuple<int64_t, int32_t, int64_t>;
+  const size_t nlv = ranges.size();
+  std::vector<int64_t> lv_holes(nlv, 0);
+  for (size_t li = 1; li < nlv; li++) lv_holes[li] = std::max<int64_t>(0, ranges[li].first - ranges[li - 1].second);
+  const int nth = omp_get_max_threads();
+  std::vector<std::vector<std::vector<Cand>>> loc(nth, std::vector<std::vector<Cand>>(nlv));
+#pragma omp parallel
+  {
+    auto& L = loc[omp_get_thread_num()];
+    std::vector<int64_t> cs;
+#pragma omp for schedule(dynamic, 4096)
+    for (int64_t s = 0; s < n_slots; s++) {
+      cs.clear();
+      for (const Edge& e : radj[s]) {
+        const int64_t C = e.dst / k;
+        if (chunk_lv[C] >= 0) cs.push_back(C);
+      }
+      if (cs.empty()) continue;
+      std::sort(cs.begin(), cs.end());
+      for (size_t a = 0; a < cs.size();) {
+        size_t b = a;
+        while (b < cs.size() && cs[b] == cs[a]) b++;
+        const int64_t cnt = (int64_t)(b - a), C = cs[a];
+        a = b;
+        if (cnt * 1000000 < theta_ppm * (int64_t)nonhole[C]) continue;
+        auto& v = L[chunk_lv[C]];
+        const size_t h = (size_t)lv_holes[chunk_lv[C]];
+        const Cand c{-cnt, (int32_t)s, C};
+        if (v.size() < h) {
+          v.insert(std::upper_bound(v.begin(), v.end(), c), c);
+        } else if (c < v.back()) {
+          v.pop_back();
+          v.insert(std::upper_bound(v.begin(), v.end(), c), c);
+        }
+      }
     }
-  std::sort(pairs.begin(), pairs.end());
-  // candidates per level: (-count, s, C)
-  std::vector<std::vector<std::tuple<int64_t, int32_t, int64_t>>> cands(ranges.size());
-  for (size_t a = 0; a < pairs.size();) {
-    size_t b = a;
-    while (b < pairs.size() && pairs[b] == pairs[a]) b++;
-    const int64_t cnt = (int64_t)(b - a);
-    const int64_t C = pairs[a].first;
-    if (cnt * 1000000 >= theta_ppm * (int64_t)nonhole[C]) cands[chunk_lv[C]].push_back({-cnt, pairs[a].second, C});
-    a = b;
   }
-  for (size_t li = 1; li < ranges.size(); li++) {
+  pt("replica candidates");
+  for (size_t li = 1; li < nlv; li++) {
     const int64_t h0 = ranges[li - 1].second, h1 = ranges[li].first;
     if (h1 <= h0) continue;
-    auto& cl = cands[li];
+    std::vector<Cand> cl;
+    for (int th = 0; th < nth; th++) cl.insert(cl.end(), loc[th][li].begin(), loc[th][li].end());
     std::sort(cl.begin(), cl.end());
     int64_t h = h0;
     for (auto& c : cl) {
@@ -357,30 +399,55 @@ struct Logical {
   }
 };
 
+// G_L out-adjacency (original ids, sorted by destination): the owner slot's
+// row of every vertex in parallel, then the replica rows appended
+void logical_out(const Work& W, std::vector<std::vector<std::pair<int32_t, uint32_t>>>& out) {
+  const int64_t n = W.n;
+  out.assign(n, {});
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int64_t u = 0; u < n; u++) {
+    const auto& row = W.rows[W.owner[u]];
+    auto& r = out[u];
+    r.reserve(row.size());
+    for (const Edge& e : row) r.push_back({W.slot_to_orig[e.dst], e.w});
+  }
+  for (int64_t s = 0; s < W.n_slots; s++) {
+    if (W.kind[s] != REPLICA) continue;
+    auto& r = out[W.slot_to_orig[s]];
+    for (const Edge& e : W.rows[s]) r.push_back({W.slot_to_orig[e.dst], e.w});
+  }
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int64_t u = 0; u < n; u++) std::sort(out[u].begin(), out[u].end());
+}
+
 void build_logical(const Work& W, Logical& L) {
+  PhaseTimer pt;
   const int64_t n = W.n;
   L.n = n;
-  L.out.assign(n, {});
-  for (int64_t s = 0; s < W.n_slots; s++) {
-    if (W.kind[s] == HOLE) continue;
-    const int32_t u = W.slot_to_orig[s];
-    for (const Edge& e : W.rows[s]) L.out[u].push_back({W.slot_to_orig[e.dst], e.w});
-  }
-  std::vector<std::vector<int32_t>> inn(n);
-  for (int64_t u = 0; u < n; u++) {
-    std::sort(L.out[u].begin(), L.out[u].end());
-    for (auto& e : L.out[u]) inn[e.first].push_back((int32_t)u);
-  }
+  logical_out(W, L.out);
+  // in-adjacency by counting (CSC of G_L)
+  std::vector<int64_t> ip(n + 1, 0);
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int64_t u = 0; u < n; u++)
+    for (auto& e : L.out[u]) __atomic_fetch_add(&ip[e.first + 1], 1, __ATOMIC_RELAXED);
+  for (int64_t v = 0; v < n; v++) ip[v + 1] += ip[v];
+  std::vector<int32_t> isrc(ip[n]);
+  std::vector<int64_t> cur(ip.begin(), ip.end() - 1);
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int64_t u = 0; u < n; u++)
+    for (auto& e : L.out[u]) isrc[__atomic_fetch_add(&cur[e.first], 1, __ATOMIC_RELAXED)] = (int32_t)u;
+  pt("logical out+in");
   L.N.assign(n, {});
 #pragma omp parallel for schedule(dynamic, 4096)
   for (int64_t u = 0; u < n; u++) {
     auto& v = L.N[u];
-    v.reserve(L.out[u].size() + inn[u].size());
+    v.reserve(L.out[u].size() + (ip[u + 1] - ip[u]));
     for (auto& e : L.out[u]) v.push_back(e.first);
-    for (int32_t x : inn[u]) v.push_back(x);
+    for (int64_t i = ip[u]; i < ip[u + 1]; i++) v.push_back(isrc[i]);
     std::sort(v.begin(), v.end());
     v.erase(std::unique(v.begin(), v.end()), v.end());
   }
+  pt("undirected N");
   // triangles: forward algorithm over the degree-ordered orientation
   L.T.assign(n, 0);
   std::vector<std::vector<int32_t>> fwd(n);
@@ -393,6 +460,7 @@ void build_logical(const Work& W, Logical& L) {
       if (rank_less((int32_t)u, v)) fwd[u].push_back(v);
     std::sort(fwd[u].begin(), fwd[u].end());
   }
+  pt("forward lists");
   std::vector<int64_t> tl(n, 0);
 #pragma omp parallel
   {
@@ -421,6 +489,7 @@ void build_logical(const Work& W, Logical& L) {
     }
   }
   L.T.swap(tl);
+  pt("triangles");
 }
 
 struct SmemOut {
@@ -559,6 +628,7 @@ int bucket_of(int64_t d) {
 }
 
 void degnorm(Work& W, int64_t th, int64_t f, bool combined, int wrule, std::vector<int32_t>& sched, int64_t& added) {
+  PhaseTimer pt;
   const int64_t ns = W.n_slots;
   std::vector<int64_t> deg(ns);
   for (int64_t s = 0; s < ns; s++) deg[s] = (int64_t)W.rows[s].size();
@@ -573,12 +643,9 @@ void degnorm(Work& W, int64_t th, int64_t f, bool combined, int wrule, std::vect
                      [&](int32_t a, int32_t b) { return bucket_of(deg[a]) > bucket_of(deg[b]); });
   }
   // pre-§4 logical out adjacency
-  std::vector<std::vector<std::pair<int32_t, uint32_t>>> lout(W.n);
-  for (int64_t s = 0; s < ns; s++) {
-    if (W.kind[s] == HOLE) continue;
-    for (const Edge& e : W.rows[s]) lout[W.slot_to_orig[s]].push_back({W.slot_to_orig[e.dst], e.w});
-  }
-  for (auto& r : lout) std::sort(r.begin(), r.end());
+  std::vector<std::vector<std::pair<int32_t, uint32_t>>> lout;
+  logical_out(W, lout);
+  pt("order + logical out");
   std::vector<std::vector<Edge>> adds(ns);
   const int64_t nwarps = ((int64_t)order.size() + 31) / 32;
 #pragma omp parallel for schedule(dynamic, 64)
@@ -595,7 +662,8 @@ void degnorm(Work& W, int64_t th, int64_t f, bool combined, int wrule, std::vect
       if (d >= target) continue;
       const int32_t u = W.slot_to_orig[s];
       const auto& ou = lout[u];
-      std::unordered_map<int32_t, uint32_t> best;
+      // logical 2-hop out-neighbours q not in N+(u) + {u}, min combined weight
+      std::vector<std::pair<int32_t, uint32_t>> two;
       for (const auto& ex : ou)
         for (const auto& eq : lout[ex.first]) {
           const int32_t q = eq.first;
@@ -605,18 +673,18 @@ void degnorm(Work& W, int64_t th, int64_t f, bool combined, int wrule, std::vect
                                    return x.first < y.first;
                                  }))
             continue;
-          const uint32_t w = combine_w(ex.second, eq.second, wrule);
-          auto it = best.find(q);
-          if (it == best.end() || w < it->second) best[q] = w;
+          two.push_back({q, combine_w(ex.second, eq.second, wrule)});
         }
+      std::sort(two.begin(), two.end());   // by q, then weight: the first of each q is its minimum
       std::vector<std::pair<uint32_t, int32_t>> cand;
-      cand.reserve(best.size());
-      for (auto& kv : best) cand.push_back({kv.second, kv.first});
+      for (size_t i = 0; i < two.size(); i++)
+        if (i == 0 || two[i].first != two[i - 1].first) cand.push_back({two[i].second, two[i].first});
       std::sort(cand.begin(), cand.end());
       const int64_t take = std::min<int64_t>(target - d, (int64_t)cand.size());
       for (int64_t j = 0; j < take; j++) adds[s].push_back({W.owner[cand[j].second], cand[j].first, ADD_DEGNORM});
     }
   }
+  pt("padding candidates");
   added = 0;
   for (int64_t s = 0; s < ns; s++) {
     added += (int64_t)adds[s].size();
