@@ -292,6 +292,14 @@ void build_device_slots(gx_graph* g) {
     up(d.t_eptr, teptr.data(), sizeof(int32_t) * teptr.size());
     up(d.t_edges, tedges.data(), sizeof(uint2) * tedges.size());
     up(d.t_iters, titers.data(), sizeof(int32_t) * titers.size());
+    // slot -> tile map and the touched-tile scratch of the SSSP local pass
+    std::vector<int32_t> st(sg.n_slots, -1);
+    for (int64_t t = 0; t < nt; t++)
+      for (int32_t i = tp[t]; i < tp[t + 1]; i++) st[tmem[i]] = (int32_t)t;
+    up(d.slot_tile, st.data(), sizeof(int32_t) * st.size());
+    std::vector<uint32_t> zero((nt + 31) / 32, 0u);
+    up(d.tile_mark, zero.data(), sizeof(uint32_t) * zero.size());
+    d.tile_list.alloc(c, sizeof(int32_t) * nt);
   }
   if (!sg.sched.empty()) up(d.sched, sg.sched.data(), sizeof(int32_t) * sg.sched.size());
   CUDA_OK(cudaStreamSynchronize(s));  // host vectors go out of scope

@@ -143,6 +143,7 @@ struct DevGraph {
   // §3 tiles
   int64_t n_tiles = 0;
   DBuf t_ptr, t_members, t_eptr, t_edges, t_iters;  // local CSR per tile
+  DBuf slot_tile, tile_mark, tile_list;              // slot -> tile (-1), touched-tile bitmap / list (SSSP)
   int64_t t_max_members = 0, t_max_edges = 0;
 };
 

@@ -378,6 +378,10 @@ __global__ void __launch_bounds__(256) k_pr_tpv(PrArgs a) {
   pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
 }
 
+// 64 threads per tile: tiles average a handful of members (S_max 64), so
+// small CTAs let ~24 tiles per SM progress at once (was 8 with 256 threads)
+constexpr int PRL_THREADS = 64;
+
 // §3 shared-memory pass for PR (P@32188-32416; SURVEY A7 "PR store"): after
 // the sweep, each subgraph tile iterates its members t times in shared
 // memory, x_v <- (1-d)/N + d (ext_v + sum_{u in S, u->v} x_u / D_u + dang/N),
@@ -387,7 +391,7 @@ __global__ void __launch_bounds__(256) k_pr_tpv(PrArgs a) {
 // fixed point is unchanged (Theorem E3); delta grows by |x_loc - x_sweep|
 // (an upper bound of the true change), dangling mass by the exact change.
 template <bool SLOTS>
-__global__ void __launch_bounds__(256) k_pr_local(PrArgs a, const int32_t* __restrict__ tptr,
+__global__ void __launch_bounds__(PRL_THREADS) k_pr_local(PrArgs a, const int32_t* __restrict__ tptr,
                                                   const int32_t* __restrict__ tmem, const int32_t* __restrict__ teptr,
                                                   const uint2* __restrict__ tedges, const int32_t* __restrict__ titers,
                                                   int64_t ntiles) {
@@ -842,13 +846,13 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     kt.end();
     nl++;
     if (d.n_tiles && g->knobs.smem) {
-      const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 8));
+      const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 24));
       if (slots)
-        k_pr_local<true><<<grid_local, 256, 0, s>>>(a, d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(),
+        k_pr_local<true><<<grid_local, PRL_THREADS, 0, s>>>(a, d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(),
                                                     d.t_eptr.as<int32_t>(), d.t_edges.as<uint2>(), d.t_iters.as<int32_t>(),
                                                     d.n_tiles);
       else
-        k_pr_local<false><<<grid_local, 256, 0, s>>>(a, d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(),
+        k_pr_local<false><<<grid_local, PRL_THREADS, 0, s>>>(a, d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(),
                                                      d.t_eptr.as<int32_t>(), d.t_edges.as<uint2>(),
                                                      d.t_iters.as<int32_t>(), d.n_tiles);
       nl++;

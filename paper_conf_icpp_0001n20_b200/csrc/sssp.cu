@@ -327,10 +327,39 @@ __global__ void __launch_bounds__(256) k_sssp_tpv(const int32_t* __restrict__ la
 // One CTA per subgraph tile: member distances staged in shared memory,
 // relaxed t times over the tile's local edges (P@32188-32416, reading R28),
 // improvements written back with atomic min and added to the next frontier.
+// Touched-tile list (tlist != nullptr): the tiles with a member in the current
+// or the next frontier, collected by sssp_tiles_collect_dev, so the pass costs
+// O(touched tiles) instead of a scan of every tile per iteration (a road grid
+// has ~4e5 tiles and ~1e4 iterations).
+__device__ __forceinline__ void sssp_tiles_collect_dev(const SsspAux& ax, SsspState* __restrict__ st, unsigned t,
+                                                       const int32_t* __restrict__ slot_tile,
+                                                       uint32_t* __restrict__ tmark, int32_t* __restrict__ tlist) {
+  const uint32_t* bm_cur = ax.bm[t % 3];
+  const uint32_t* bm_next = ax.bm[(t + 1) % 3];
+  for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < ax.nwords; w += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t bits = __ldcg(bm_cur + w) | __ldcg(bm_next + w);
+    while (bits) {
+      const int b = __ffs(bits) - 1;
+      bits &= bits - 1;
+      const int32_t tl = slot_tile[w * 32 + b];
+      if (tl < 0) continue;
+      const uint32_t bit = 1u << (tl & 31);
+      if (!(atomicOr(tmark + (tl >> 5), bit) & bit)) tlist[atomicAdd(&st->tiles_n[t % 3], 1u)] = tl;
+    }
+  }
+}
+__global__ void k_sssp_tiles_collect(SsspAux ax, SsspState* __restrict__ st, const int32_t* __restrict__ slot_tile,
+                                     uint32_t* __restrict__ tmark, int32_t* __restrict__ tlist) {
+  if (st->stop) return;
+  sssp_tiles_collect_dev(ax, st, st->iter, slot_tile, tmark, tlist);
+}
+
 __device__ __forceinline__ void sssp_local_dev(const int32_t* __restrict__ tptr, const int32_t* __restrict__ tmem,
                                                const int32_t* __restrict__ teptr, const uint2* __restrict__ tedges,
                                                const int32_t* __restrict__ titers, int64_t ntiles,
-                                               uint32_t* __restrict__ dist, const SsspAux& ax, SsspState* __restrict__ st) {
+                                               uint32_t* __restrict__ dist, const SsspAux& ax, SsspState* __restrict__ st,
+                                               const int32_t* __restrict__ tlist = nullptr,
+                                               uint32_t* __restrict__ tmark = nullptr) {
   __shared__ uint32_t sd[256];
   const unsigned t = st->iter;
   if (st->stop) return;
@@ -338,16 +367,22 @@ __device__ __forceinline__ void sssp_local_dev(const int32_t* __restrict__ tptr,
   const uint64_t pl = l2_evict_last();
   const uint32_t* bm_cur = ax.bm[t % 3];
   uint32_t my_push = 0;
-  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+  const int64_t nwork = tlist ? (int64_t)*(volatile unsigned*)&st->tiles_n[t % 3] : ntiles;
+  for (int64_t wi = blockIdx.x; wi < nwork; wi += gridDim.x) {
+    const int64_t tile = tlist ? tlist[wi] : wi;
     const int a = tptr[tile], nm = tptr[tile + 1] - a;
     const int ea = teptr[tile], ne = teptr[tile + 1] - ea;
-    // only tiles touched by this iteration: a member in the frontier or improved by the sweep
-    int touched = 0;
-    for (int i = threadIdx.x; i < nm; i += blockDim.x) {
-      const uint32_t v = (uint32_t)tmem[a + i];
-      touched |= (int)(((__ldcg(bm_cur + (v >> 5)) | __ldcg(bm_next + (v >> 5))) >> (v & 31)) & 1u);
+    if (tlist) {
+      if (threadIdx.x == 0) atomicAnd(tmark + (tile >> 5), ~(1u << (tile & 31)));   // listed once per iteration
+    } else {
+      // only tiles touched by this iteration: a member in the frontier or improved by the sweep
+      int touched = 0;
+      for (int i = threadIdx.x; i < nm; i += blockDim.x) {
+        const uint32_t v = (uint32_t)tmem[a + i];
+        touched |= (int)(((__ldcg(bm_cur + (v >> 5)) | __ldcg(bm_next + (v >> 5))) >> (v & 31)) & 1u);
+      }
+      if (!__syncthreads_or(touched)) continue;
     }
-    if (!__syncthreads_or(touched)) continue;
     for (int i = threadIdx.x; i < nm; i += blockDim.x) sd[i] = ld_l2_u32(dist + tmem[a + i], pl);
     __syncthreads();
     const int iters = titers[tile];
@@ -385,8 +420,9 @@ __device__ __forceinline__ void sssp_local_dev(const int32_t* __restrict__ tptr,
 __global__ void __launch_bounds__(256) k_sssp_local(const int32_t* __restrict__ tptr, const int32_t* __restrict__ tmem,
                                                     const int32_t* __restrict__ teptr, const uint2* __restrict__ tedges,
                                                     const int32_t* __restrict__ titers, int64_t ntiles,
-                                                    uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st) {
-  sssp_local_dev(tptr, tmem, teptr, tedges, titers, ntiles, dist, ax, st);
+                                                    uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st,
+                                                    const int32_t* __restrict__ tlist, uint32_t* __restrict__ tmark) {
+  sssp_local_dev(tptr, tmem, teptr, tedges, titers, ntiles, dist, ax, st, tlist, tmark);
 }
 
 // ---------------------------------------------------------------- §2.4 merge
@@ -485,6 +521,7 @@ __device__ __forceinline__ void sssp_advance_dev(SsspState* __restrict__ st, int
   st->act_total += st->active[t % 3];
   st->active[(t + 2) % 3] = 0;
   st->pushed[(t + 2) % 3] = 0;
+  st->tiles_n[(t + 2) % 3] = 0;
   if (st->pushed[t % 3] == 0) {  // the next frontier is empty
     if (st->far_min == INF) {    // ... and so is the far pile
       st->stop = 1;
@@ -685,6 +722,9 @@ struct SsspLoop {
   int64_t ngroups;
   int merge_min, cadence, max_iters;
   int64_t block_rows;   // > 0: block-local mode with this many rows per CTA
+  const int32_t* slot_tile;
+  uint32_t* tmark;
+  int32_t* tlist;
 };
 
 constexpr int PERSIST_POOL = SB_WARPS * 1024 * 4;   // 32 KB: LB compaction buffer / block-mode queues
@@ -713,7 +753,9 @@ __global__ void __launch_bounds__(256, 4) k_sssp_persist(SsspLoop a) {
                   reinterpret_cast<int32_t (*)[1024]>(pool));
     grid.sync();
     if (a.ntiles) {
-      sssp_local_dev(a.tptr, a.tmem, a.teptr, a.tedges, a.titers, a.ntiles, a.dist, a.ax, st);
+      sssp_tiles_collect_dev(a.ax, st, t, a.slot_tile, a.tmark, a.tlist);
+      grid.sync();
+      sssp_local_dev(a.tptr, a.tmem, a.teptr, a.tedges, a.titers, a.ntiles, a.dist, a.ax, st, a.tlist, a.tmark);
       grid.sync();
     }
     bool final_merge = false;
@@ -761,6 +803,7 @@ __global__ void __launch_bounds__(256, 4) k_sssp_persist(SsspLoop a) {
       st->active[(t + 2) % 3] = 0;
       st->pushed[(t + 2) % 3] = 0;
       st->far3[(t + 2) % 3] = INF;
+      st->tiles_n[(t + 2) % 3] = 0;
       st->iter = t + 1;
       st->tau = tau;
       st->far_min = rf;
@@ -1016,7 +1059,7 @@ static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, 
       if (d.n_tiles && g->knobs.smem) {
         k_sssp_local<<<grid_local, 256, 0, s>>>(d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(), d.t_eptr.as<int32_t>(),
                                                 d.t_edges.as<uint2>(), d.t_iters.as<int32_t>(), d.n_tiles, D(p), R[p].ax,
-                                                S(p));
+                                                S(p), nullptr, nullptr);
         launches++;
       }
     }
@@ -1073,7 +1116,10 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   const int64_t src = o.source < 0 ? default_source(g) : o.source;
   GX_CHECK_ARG(g->n > 0, "empty graph");
   GX_CHECK_ARG(src >= 0 && src < g->n, "source out of range");
-  if ((double)(g->n - 1) * (double)d.max_w >= 4294967295.0)
+  // the bound uses the INPUT graph's weights: an added edge stands for a path
+  // at least as long (sum rule) or is lighter than both hops (max / mean
+  // rules), so no distance exceeds (n-1) * max w of the input
+  if ((double)(g->n - 1) * (double)g->max_w >= 4294967295.0)
     GX_THROW(GX_E_UNSUPPORTED, "(n-1)*max(w) >= 2^32-1 would overflow uint32 distances");
   const bool sim = c->world == 1 && o.sim_ranks > 1;
   const int P = sim ? o.sim_ranks : c->world;
@@ -1169,10 +1215,13 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     }
     kt.end();
     if (d.n_tiles && g->knobs.smem) {
+      k_sssp_tiles_collect<<<grid_for(c, nwords), 256, 0, s>>>(ax, st, d.slot_tile.as<int32_t>(),
+                                                               d.tile_mark.as<uint32_t>(), d.tile_list.as<int32_t>());
       k_sssp_local<<<grid_local, 256, 0, s>>>(d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(), d.t_eptr.as<int32_t>(),
                                               d.t_edges.as<uint2>(), d.t_iters.as<int32_t>(), d.n_tiles,
-                                              r.dist.as<uint32_t>(), ax, st);
-      nl++;
+                                              r.dist.as<uint32_t>(), ax, st, d.tile_list.as<int32_t>(),
+                                              d.tile_mark.as<uint32_t>());
+      nl += 2;
     }
     if (d.n_groups) {
       if (o.merge_every != 1) {
@@ -1229,6 +1278,9 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     L.titers = d.t_iters.as<int32_t>();
     L.tedges = d.t_edges.as<uint2>();
     L.ntiles = tiles ? d.n_tiles : 0;
+    L.slot_tile = d.slot_tile.as<int32_t>();
+    L.tmark = d.tile_mark.as<uint32_t>();
+    L.tlist = d.tile_list.as<int32_t>();
     L.gptr = d.gptr.as<int32_t>();
     L.gslots = d.gslots.as<int32_t>();
     L.ginptr = d.g_in_ptr.as<int32_t>();

@@ -27,6 +27,7 @@ struct SsspState {
   unsigned int do_merge;        // iteration `iter` ends with a merge
   unsigned int final_merge;     // c = 0: this iteration's merge ends the run
   unsigned int far3[3];         // persistent loop: far-pile minimum pushed in iteration t, [t%3]
+  unsigned int tiles_n[3];      // §3 tiles touched in iteration t (list length), [t%3]
 };
 
 struct SsspAux {
