@@ -107,29 +107,53 @@ def test_device_pointer_upload_and_download():
     assert np.array_equal(out.cpu().numpy().view(np.uint32), want)
 
 
-@pytest.mark.parametrize("scale", [24])
-def test_full_size_certificates(scale):
-    """BASELINE.json's target config (RMAT-24, exact mode) in bench.py's launch
-    configuration: SSSP checked by the O(m) certificate, PR by the residual
-    bound r/(1-d) (oracle.metrics), both on the canonical graph."""
+FULL = {   # BASELINE.json's configurations at their full sizes
+    "T24_rmat24": (lambda: graphgen.rmat(24), None),
+    "C3_road4900": (lambda: graphgen.road(4900), None),
+    "C4_uniform16M_256M": (lambda: graphgen.uniform(1 << 24, 1 << 28), None),
+    "C2_rmat22_coalesce": (lambda: graphgen.rmat(22), dict(coalesce=True, chunk_k=16, replicate_threshold=0.6)),
+}
+
+
+@pytest.mark.parametrize("cfg", list(FULL))
+def test_full_size_certificates(cfg):
+    """BASELINE.json's configurations at full size, in bench.py's launch
+    configuration (LB mapping, persistent SSSP loop, asynchronous PR): SSSP
+    checked by the O(m) certificate on the ORIGINAL graph (Theorem E1 makes
+    the transformed run's distances equal to G's), PR by the residual bound
+    r/(1-d) on the graph it ran on (G, or G_L for a transformed run)."""
+    import paper_conf_icpp_0001n20_b200 as gx
     from oracle.graph import canonicalize_sorted
     from oracle.metrics import pagerank_residual, sssp_certificate
     ctx()
-    raw = graphgen.rmat(scale)
+    make, knobs = FULL[cfg]
+    raw = make()
     G = upload(raw)
     g = canonicalize_sorted(raw.n, raw.row_ptr, raw.col, raw.w)
     del raw
+    if knobs:
+        G.transform(gx.Knobs(**knobs))
     s = sssp_source(g)
-    G.run("sssp", source=-1, mapping="lb")
+    r = G.run("sssp", source=-1, mapping="lb")
+    assert r["converged"] == 1
     dist = G.download("dist")
     cert = sssp_certificate(g, s, dist)
     assert cert["ok"], cert
     info = G.run("pagerank", tol=1e-9, mapping="lb")
     x = G.download("rank")
-    src = np.repeat(np.arange(g.n, dtype=np.int32), np.diff(g.row_ptr))
-    r = pagerank_residual(src, g.col, g.n, x)
-    assert r["bound"] <= 1e-6, r
-    assert abs(r["mass"] - 1) < 1e-6
+    if knobs:   # G_L of the transformed run (replica rows folded into the owner)
+        ex = G.export()
+        keep = ex["slot_kind"] != 2
+        o = ex["slot_to_orig"]
+        src = np.repeat(o, np.diff(ex["row_ptr"]))
+        dst = o[ex["col"]]
+        del ex, keep
+    else:
+        src = np.repeat(np.arange(g.n, dtype=np.int32), np.diff(g.row_ptr))
+        dst = g.col
+    res = pagerank_residual(src, dst, g.n, x)
+    assert res["bound"] <= 1e-6, res
+    assert abs(res["mass"] - 1) < 1e-6
 
 
 @pytest.mark.parametrize("name", ["rmat12", "uniform", "road64", "star_hub", "dups_loops", "isolated"])

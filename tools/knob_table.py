@@ -7,6 +7,10 @@ for f in sorted(glob.glob(sys.argv[1] + "/*.jsonl")):
     print("==", f.split("/")[-1])
     for line in open(f):
         d = json.loads(line)
+        if "P" in d:
+            print(f"  [{d['knob']}] P={d['P']} ({d['note']}): SSSP {d['sssp_ms']:.2f} ms ({d['sssp_iters']} it) | "
+                  f"PR {d['pagerank_ms']:.2f} ms ({d['pagerank_iters']} it)")
+            continue
         if d["knob"] == "exact":
             print(f"  {d['graph']} exact: SSSP lb {d['sssp_lb_ms']:.2f} ms tpv {d['sssp_tpv_ms']:.2f} | PR lb {d['pr_lb_ms']:.2f} tpv {d['pr_tpv_ms']:.2f} ({d['pr_iters']} it)")
             continue
