@@ -36,7 +36,9 @@ WORKLOADS = {
     "c2": dict(scale=22, desc="C2: RMAT-22, exact mode, SSSP + PageRank"),
     "c1": dict(scale=14, desc="C1: RMAT-14, exact mode, SSSP + PageRank"),
 }
-CPU_SAMPLE_SCALE = 17   # bounded oracle sample: same generator at 1/128 of T24
+CPU_SAMPLE_SCALE = 17
+PR_KERNELS = {1: "k_pr_sell2", 2: "k_pr_tpv", 3: "k_pr_pb"}   # gx_mapping -> PR sweep kernel
+MAPPING_NAMES = {0: "auto", 1: "lb", 2: "tpv", 3: "pb"}   # bounded oracle sample: same generator at 1/128 of T24
 
 
 def peaks():
@@ -142,6 +144,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--pr-mapping", default="auto", choices=["auto", "lb", "tpv", "pb"],
+                    help="PageRank sweep mapping (auto = the blocked pull on one GPU at these sizes)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -170,7 +174,7 @@ def main():
 
     def step(profile):
         a = G.run("sssp", source=-1, mapping="lb", profile=profile)
-        b = G.run("pagerank", tol=1e-9, mapping="lb", profile=profile)
+        b = G.run("pagerank", tol=1e-9, mapping=args.pr_mapping, profile=profile)
         return a, b
 
     for _ in range(args.warmup):
@@ -215,7 +219,8 @@ def main():
     # dominant kernel roofline (live CUDA events around each sweep launch)
     peak, peak_src = peaks()
     kern = {}
-    for name, idx in (("k_sssp_lb", 0), ("k_pr_sell2", 1)):
+    pr_kernel = PR_KERNELS.get(runs[-1][1].get("mapping_used", 1), "k_pr_sell2")
+    for name, idx in (("k_sssp_lb", 0), (pr_kernel, 1)):
         ms = sum(r[idx]["sweep_ms"] for r in runs)
         # sweeps that did work (a CUDA-graph / eager batch may launch a few
         # more that return at once after convergence; their ~3 us stay in ms)
@@ -277,7 +282,7 @@ def main():
             e0.record(stream)
             G2 = gx.Graph.upload(ctx, hrp.numpy(), hcol.numpy(), hw.numpy().view(np.uint32), canonical=True)
             a = G2.run("sssp", source=-1, mapping="lb")
-            b = G2.run("pagerank", tol=1e-9, mapping="lb")
+            b = G2.run("pagerank", tol=1e-9, mapping=args.pr_mapping)
             G2.download("dist", out=hdist.numpy().view(np.uint32))
             G2.download("rank", out=hrank.numpy())
             e1.record(stream)
@@ -308,7 +313,9 @@ def main():
                 "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
                 "scaling": "strong" if world > 1 else "weak", "vs_baseline": None, "dtype": "u32/f64", "data": "synthetic",
                 "config": {"workload": wl["desc"], "graph": f"rmat{wl['scale']}", "n": n, "m": m,
-                           "knobs": "exact", "mapping": "lb", "l2": "flushed between steps (256 MiB write)",
+                           "knobs": "exact",
+                           "mapping": {"sssp": MAPPING_NAMES.get(runs[-1][0].get("mapping_used", 1), "lb"),
+                                       "pagerank": MAPPING_NAMES.get(runs[-1][1].get("mapping_used", 1), "?")}, "l2": "flushed between steps (256 MiB write)",
                            "parallelism": f"1-D partitioned x{world} (NCCL)" if world > 1 else "single"},
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
                 "clocks": clocks, "per_algo": per_algo, "kernels": kern}

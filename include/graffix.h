@@ -61,8 +61,15 @@ typedef enum { GX_MERGE_MEAN = 0, GX_MERGE_MIN = 1 } gx_merge;
 /* Sweep mapping.  LB: edge-balanced warp-cooperative kernels (the best exact
  * kernels).  TPV: the paper's vertex-centric mapping, one thread per slot
  * (P@15381), lanes of a warp = 32 consecutive entries of the §4 schedule,
- * edges in SELL-32 slabs.  AUTO = LB in exact mode, TPV when §2 or §4 is on. */
-typedef enum { GX_MAP_AUTO = 0, GX_MAP_LB = 1, GX_MAP_TPV = 2 } gx_mapping;
+ * edges in SELL-32 slabs.  PB (PageRank only; other algorithms run LB):
+ * propagation-blocked pull -- the x_u/D_u terms of the sum in P@36969 are
+ * streamed along the edges in (source block, sink block) segments and summed
+ * in shared memory, so no random global gathers remain; single GPU,
+ * asynchronous schedule.  AUTO = PB for PageRank on one GPU when the graph
+ * spans at least GX_PB_MIN_BLOCKS blocks of 16384 slots and no §3 tiles are
+ * present, else LB in exact mode and TPV when §2 or §4 is on. */
+typedef enum { GX_MAP_AUTO = 0, GX_MAP_LB = 1, GX_MAP_TPV = 2, GX_MAP_PB = 3 } gx_mapping;
+#define GX_PB_MIN_BLOCKS 64
 
 /* upload / download flags */
 #define GX_PTRS_HOST 0u       /* pointers are host memory (pageable or pinned)   */
@@ -133,6 +140,7 @@ typedef struct {
   int32_t sweep_launches;  /* profile: launches of the main sweep kernel            */
   double sweep_ms;         /* profile: summed CUDA-event time of the main sweep kernel */
   int64_t sweep_bytes;     /* algorithmic bytes moved by the main sweep kernel       */
+  int32_t mapping_used;    /* gx_mapping the sweeps ran with (AUTO resolved)         */
 } gx_run_info;
 
 typedef struct {

@@ -22,7 +22,7 @@ GX_SSSP, GX_PAGERANK, GX_SCC, GX_MST, GX_BC = 1, 2, 3, 4, 5
 ALGOS = {"sssp": GX_SSSP, "pagerank": GX_PAGERANK, "pr": GX_PAGERANK, "scc": GX_SCC, "mst": GX_MST,
          "bc": GX_BC}
 GX_MERGE_MEAN, GX_MERGE_MIN = 0, 1
-GX_MAP_AUTO, GX_MAP_LB, GX_MAP_TPV = 0, 1, 2
+GX_MAP_AUTO, GX_MAP_LB, GX_MAP_TPV, GX_MAP_PB = 0, 1, 2, 3
 GX_PTRS_HOST, GX_PTRS_DEVICE, GX_VALIDATE, GX_CANONICAL = 0, 1, 2, 4
 GX_OUT_DIST_U32, GX_OUT_RANK_F64, GX_OUT_LABEL_I32, GX_OUT_BC_F64, GX_OUT_MST_WEIGHT_U64 = 1, 2, 3, 4, 5
 
@@ -55,7 +55,7 @@ class GxRunInfo(C.Structure):
     _fields_ = [("iterations", C.c_int32), ("converged", C.c_int32), ("loop_ms", C.c_double),
                 ("last_delta", C.c_double), ("edges_scanned", C.c_int64), ("bytes_model", C.c_int64),
                 ("vertices_active", C.c_int64), ("kernel_launches", C.c_int32), ("sweep_launches", C.c_int32),
-                ("sweep_ms", C.c_double), ("sweep_bytes", C.c_int64)]
+                ("sweep_ms", C.c_double), ("sweep_bytes", C.c_int64), ("mapping_used", C.c_int32)]
 
 
 class GxRunOpts(C.Structure):

@@ -156,6 +156,119 @@ static void build_csc_and_tiles(gx_graph* g) {
                               d.pr_sell);
 }
 
+// ---- propagation-blocked PR layout (PbLayout, gx_internal.h) ----
+// key = bin(v) * nb + block(u) per out-edge (sink-bin major), payload = the
+// two local indices; histogram of keys for the segment offsets
+__global__ void k_pb_pairs(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj, int64_t n, uint32_t nb,
+                           uint32_t* __restrict__ key, uint32_t* __restrict__ val, uint32_t* __restrict__ cnt) {
+  int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  int lane = threadIdx.x & 31;
+  int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t u = warp; u < n; u += nw) {
+    const uint32_t a = rp[u], b = rp[u + 1];
+    const uint32_t bu = (uint32_t)(u / PB_R), lu = (uint32_t)(u % PB_R);
+    for (uint32_t e = a + lane; e < b; e += 32) {
+      const uint32_t v = adj[e].x;
+      const uint32_t k = (v / PB_R) * nb + bu;
+      key[e] = k;
+      val[e] = lu | ((v % PB_R) << 16);
+      atomicAdd(&cnt[k], 1u);
+    }
+  }
+}
+
+// segment lengths padded to a multiple of PB_PAD (16-byte aligned u16 runs)
+__global__ void k_pb_padcnt(const uint32_t* __restrict__ cnt, uint32_t* __restrict__ pc, int64_t nk) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nk; i += (int64_t)gridDim.x * blockDim.x)
+    pc[i] = i + 1 < nk ? (cnt[i] + PB_PAD - 1) / PB_PAD * PB_PAD : 0u;
+}
+
+// element i of the sorted order (key k) -> padded position P2[k] + (i - P[k])
+__global__ void k_pb_place(const uint32_t* __restrict__ key, const uint32_t* __restrict__ pay,
+                           const uint32_t* __restrict__ P, const uint32_t* __restrict__ P2, uint16_t* __restrict__ sl,
+                           uint16_t* __restrict__ dl, int64_t m) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t k = key[i], p = pay[i];
+    const uint32_t pos = P2[k] + ((uint32_t)i - P[k]);
+    sl[pos] = (uint16_t)(p & 0xffffu);
+    dl[pos] = (uint16_t)(p >> 16);
+  }
+}
+
+// q[s*nb + b] = start of segment (s, b) = P2[b*nb + s]; row nb = bin ends
+__global__ void k_pb_transpose(const uint32_t* __restrict__ P2, uint32_t* __restrict__ q, int64_t nb) {
+  const int64_t tot = (nb + 1) * nb;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < tot; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t s = i / nb, b = i % nb;
+    q[i] = s < nb ? P2[b * nb + s] : P2[(b + 1) * nb];
+  }
+}
+
+void ensure_pb(gx_graph* g) {
+  DevGraph& d = g->dg;
+  PbLayout& L = d.pr_pb;
+  if (L.built()) return;
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  const int64_t n = d.n_slots, m = d.m_slots;
+  const int64_t nb = std::max<int64_t>(1, (n + PB_R - 1) / PB_R);
+  const int64_t nk = nb * nb + 1;
+  if (nb * nb >= (int64_t(1) << 32)) GX_THROW(GX_E_UNSUPPORTED, "graph too large for the blocked PR layout");
+  L.nb = nb;
+  DBuf P, P2, cnt, pc;
+  cnt.alloc(c, sizeof(uint32_t) * nk);
+  pc.alloc(c, sizeof(uint32_t) * nk);
+  P.alloc(c, sizeof(uint32_t) * nk);
+  P2.alloc(c, sizeof(uint32_t) * nk);
+  CUDA_OK(cudaMemsetAsync(cnt.p, 0, sizeof(uint32_t) * nk, s));
+  DBuf k0, k1, v0, v1, tmp;
+  cub::DoubleBuffer<uint32_t> dk, dv;
+  if (m > 0) {
+    k0.alloc(c, sizeof(uint32_t) * m);
+    k1.alloc(c, sizeof(uint32_t) * m);
+    v0.alloc(c, sizeof(uint32_t) * m);
+    v1.alloc(c, sizeof(uint32_t) * m);
+    k_pb_pairs<<<grid_for(c, n * 32), 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), n, (uint32_t)nb,
+                                                   k0.as<uint32_t>(), v0.as<uint32_t>(), cnt.as<uint32_t>());
+    CUDA_OK(cudaGetLastError());
+    int bits = 1;
+    while ((int64_t(1) << bits) < nb * nb) bits++;
+    size_t tb = 0;
+    dk = cub::DoubleBuffer<uint32_t>(k0.as<uint32_t>(), k1.as<uint32_t>());
+    dv = cub::DoubleBuffer<uint32_t>(v0.as<uint32_t>(), v1.as<uint32_t>());
+    CUDA_OK(cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv, (int64_t)m, 0, bits, s));
+    tmp.alloc(c, tb);
+    CUDA_OK(cub::DeviceRadixSort::SortPairs(tmp.p, tb, dk, dv, (int64_t)m, 0, bits, s));
+  }
+  k_pb_padcnt<<<grid_for(c, nk), 256, 0, s>>>(cnt.as<uint32_t>(), pc.as<uint32_t>(), nk);
+  size_t sb = 0;
+  CUDA_OK(cub::DeviceScan::ExclusiveSum(nullptr, sb, cnt.as<uint32_t>(), P.as<uint32_t>(), nk, s));
+  DBuf t2;
+  t2.alloc(c, sb);
+  CUDA_OK(cub::DeviceScan::ExclusiveSum(t2.p, sb, cnt.as<uint32_t>(), P.as<uint32_t>(), nk, s));
+  CUDA_OK(cub::DeviceScan::ExclusiveSum(t2.p, sb, pc.as<uint32_t>(), P2.as<uint32_t>(), nk, s));
+  uint32_t mp = 0;
+  CUDA_OK(cudaMemcpyAsync(&mp, P2.as<uint32_t>() + nb * nb, 4, cudaMemcpyDeviceToHost, s));
+  CUDA_OK(cudaStreamSynchronize(s));
+  if ((int64_t)mp < m || mp >= 0xfffffff0u) GX_THROW(GX_E_UNSUPPORTED, "padded edge count overflows 32 bits");
+  L.m_pad = mp;
+  const int64_t mm = std::max<int64_t>(mp, 8);
+  L.src_loc.alloc(c, sizeof(uint16_t) * mm);
+  L.dst_loc.alloc(c, sizeof(uint16_t) * mm);
+  L.val.alloc(c, sizeof(float) * mm);
+  // padding entries: source index PB_R (a zero term in shared memory), sink 0
+  launch_fill_u32(c, L.src_loc.as<uint32_t>(), (uint32_t)PB_R * 0x10001u, mm / 2);   // mm is a multiple of 8
+  CUDA_OK(cudaMemsetAsync(L.dst_loc.p, 0, sizeof(uint16_t) * mm, s));
+  CUDA_OK(cudaMemsetAsync(L.val.p, 0, sizeof(float) * mm, s));
+  if (m > 0)
+    k_pb_place<<<grid_for(c, m), 256, 0, s>>>(dk.Current(), dv.Current(), P.as<uint32_t>(), P2.as<uint32_t>(),
+                                              L.src_loc.as<uint16_t>(), L.dst_loc.as<uint16_t>(), m);
+  L.q.alloc(c, sizeof(uint32_t) * (nb + 1) * nb);
+  k_pb_transpose<<<grid_for(c, (nb + 1) * nb), 256, 0, s>>>(P2.as<uint32_t>(), L.q.as<uint32_t>(), nb);
+  CUDA_OK(cudaGetLastError());
+  CUDA_OK(cudaStreamSynchronize(s));   // temporaries are freed on return
+}
+
 void ensure_csc(gx_graph* g) {
   if (g->dg.crp.p) return;
   build_csc_and_tiles(g);

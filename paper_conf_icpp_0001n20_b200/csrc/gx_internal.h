@@ -102,6 +102,26 @@ struct SellLayout {
   bool built() const { return slab.p != nullptr; }
 };
 
+// Propagation-blocked PR layout (pagerank.cu k_pr_pb): slots are cut into
+// blocks of PB_R rows; the edges u->v are grouped by (sink bin(v), source
+// block(u)) into segments, sink-bin major, each edge stored as the two 16-bit
+// local indices u%PB_R, v%PB_R; every segment is padded to a multiple of
+// PB_PAD entries (source index PB_R = a zero term, sink 0), so all runs are
+// 16-byte aligned.  q[s*nb + b] = start of segment (block s -> bin b),
+// q[nb*nb + b] = end of bin b: bin b's in-edges are the contiguous range
+// [q[b], q[nb*nb + b]); segment (s, b) = [q[s*nb + b], q[(s+1)*nb + b]).
+// val f32[m_pad] carries x_u/D_u along every edge (written by the source
+// block's scatter, read by the sink bin).
+constexpr int PB_R = 16384;
+constexpr int PB_PAD = 8;
+struct PbLayout {
+  int64_t nb = 0, m_pad = 0;
+  DBuf q;                       // u32 [(nb+1)*nb]
+  DBuf src_loc, dst_loc;        // u16 [m_pad]
+  DBuf val;                     // f32 [m_pad]
+  bool built() const { return q.p != nullptr; }
+};
+
 // Device layouts of the current slot graph.
 struct DevGraph {
   int64_t n = 0, n_slots = 0, m_slots = 0;
@@ -119,6 +139,7 @@ struct DevGraph {
   // windowed SELL-32 layouts (sell.cu): PR pull over in-edges, SSSP dense
   // push over out-edges
   SellLayout pr_sell, sssp_sell;
+  PbLayout pr_pb;              // propagation-blocked PR (built on first use)
   // LB SSSP: static chunk list of rows with out-degree > HEAVY_DEG, heavy bitmap
   int64_t nhc = 0;
   // SSSP block-local mode (sssp.cu): block size the locality was measured for,

@@ -42,6 +42,7 @@ struct PrState {
   unsigned force;        // the sweep reached its fixed point without a merge: merge next
   unsigned normalize;    // lazy normalisation on (off for the end-only merge, whose
                          // intermediate no-merge fixed point does not sum to 1)
+  unsigned pb_next[3];   // blocked mapping: next sink bin of iteration t, [t%3]
 };
 
 struct PrArgs {
@@ -333,6 +334,272 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell2(PrArgs a) {
   pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
 }
 
+// ---------------------------------------------------------------------------
+// Propagation-blocked pull (GX_MAP_PB; PbLayout in gx_internal.h).  The sum
+// of P@36969, y_v = sum_{u->v} x_u / D_u, is computed without any random
+// global gather: every edge carries its term x_u/D_u in val[] (f32), laid out
+// sink-bin major in (sink bin, source block) segments of PB_R-slot blocks.
+// One CTA per SM claims sink bins in ascending order and, for bin b:
+//   (1) streams the bin's contiguous range of val + 16-bit sink index with
+//       16-byte loads and adds each term into a shared-memory accumulator of
+//       its sink row (unsigned 64-bit fixed point, 2^-56 units, kept as two
+//       32-bit words: exact, so the sum does not depend on the order); meanwhile the bin's
+//       x / D rows and block b's scatter segments are bulk-prefetched into L2;
+//   (2) runs the PR update of the bin's rows (x, delta, dangling and total
+//       mass as in pr_finalize) and keeps the new x/D of every row in shared
+//       memory;
+//   (3) scatters those terms along block b's out-edges: nb segments (one per
+//       sink bin), each a 16-byte aligned run read with one 16-byte load of
+//       source indices per lane and written as two float4 per lane.
+// Bins later in the same sweep read the terms (3) just wrote, earlier bins
+// read them next sweep: the asynchronous in-place schedule of the LB kernel
+// (Theorem E3 fixes the limit; any mix of old and new terms is a valid
+// chaotic-relaxation step).  Per edge and sweep: 4 + 2 bytes read in (1), 2
+// read + 4 written in (3), all streaming -- 12 B against the 8 B of the
+// gather pull, at HBM rate instead of the L1TEX random-sector rate.
+// One CTA per SM (measured: two CTAs of half the rows, PB_R = 8192, are 18 %
+// slower -- twice the segments, each half as long)
+constexpr int PB_THREADS = 1024;
+constexpr int PB_CTAS_PER_SM = 1;
+constexpr int PB_CH = 4 * PB_THREADS;   // (1): elements per bulk-copied chunk (4 per thread)
+constexpr int PB_NST = 4;          // (1): ring stages (3 chunks in flight while one is consumed)
+constexpr size_t PB_STAGE = (size_t)PB_CH * 6;
+// dynamic smem: acc_lo u32[R] (reused as the f32 terms s_c after the update)
+// | 8 zero words (s_c[R..R+7], the padding entries' source) | acc_hi u32[R] | ring
+constexpr size_t PB_RING_OFF = (size_t)PB_R * 8 + 32;
+constexpr size_t PB_SMEM = PB_RING_OFF + PB_NST * PB_STAGE;
+
+struct PbArgs {
+  const uint32_t* q;
+  const uint16_t* src_loc;
+  const uint16_t* dst_loc;
+  float* val;
+  int64_t nb;
+};
+
+__device__ __forceinline__ float4 ld_cg_f4(const float* p) {
+  float4 v;
+  asm volatile("ld.global.cg.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ void l2_prefetch_bulk(const void* p, uint32_t bytes) {
+  if (bytes >= 16) asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes & ~15u) : "memory");
+}
+// fixed-point accumulation with the one native shared-memory atomic (32-bit
+// ATOMS.ADD; 64-bit and float adds compile to CAS loops): a term t >= 0 is
+// v = rn(t * 2^56) (quantum 1.4e-17, at most ~7e-18 per edge), split into
+// 32-bit halves; the low half is added with a returning atomic and a carry
+// out of it (rare: the low word holds up to 6e-8 of rank) goes to the high word.
+__device__ __forceinline__ void pb_add4(uint32_t* lo, uint32_t* hi, uint2 r, float4 t4) {
+  const uint32_t rr[4] = {r.x & 0xffffu, r.x >> 16, r.y & 0xffffu, r.y >> 16};
+  const float tt[4] = {t4.x, t4.y, t4.z, t4.w};
+  unsigned long long v[4];
+  uint32_t old[4];
+#pragma unroll
+  for (int i = 0; i < 4; i++) v[i] = __float2ull_rn(tt[i] * 0x1p56f);
+  // the returning atomics are independent: issue them back to back
+#pragma unroll
+  for (int i = 0; i < 4; i++) old[i] = atomicAdd(&lo[rr[i]], (uint32_t)v[i]);
+#pragma unroll
+  for (int i = 0; i < 4; i++) {
+    const uint32_t vl = (uint32_t)v[i];
+    const uint32_t vh = (uint32_t)(v[i] >> 32) + (old[i] + vl < old[i] ? 1u : 0u);
+    if (vh) atomicAdd(&hi[rr[i]], vh);
+  }
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void pb_put8(float* dst, const float* s_c, uint4 w) {
+  float4 o0, o1;
+  o0.x = s_c[w.x & 0xffffu]; o0.y = s_c[w.x >> 16];
+  o0.z = s_c[w.y & 0xffffu]; o0.w = s_c[w.y >> 16];
+  o1.x = s_c[w.z & 0xffffu]; o1.y = s_c[w.z >> 16];
+  o1.z = s_c[w.w & 0xffffu]; o1.w = s_c[w.w >> 16];
+  __stcg(reinterpret_cast<float4*>(dst), o0);
+  __stcg(reinterpret_cast<float4*>(dst) + 1, o1);
+}
+
+// the PR update of one row (pr_finalize) returning the row's next term x/D;
+// false when the row is not recomputed here (hole, replica, or an owner that
+// hands its value to the merge) -- its term is then the stored contrib
+template <bool SLOTS>
+__device__ __forceinline__ bool pb_update(const PrArgs& a, int64_t v, double y, double xo, uint32_t Dv, double addc,
+                                          bool merge_now, double sc, double& my_delta, double& my_dang,
+                                          double& my_mass, float& c) {
+  if (SLOTS) {
+    if (a.kind[v] != OWNER) return false;
+  }
+  const double xn = addc + a.damp * sc * y;
+  if (SLOTS && a.gid && merge_now) {
+    const int g = a.gid[v];
+    if (g >= 0) {
+      a.gnew[g] = xn;
+      return false;
+    }
+  }
+  __stcs(a.x + v, xn);
+  my_delta += fabs(xn - sc * xo);
+  my_mass += xn;
+  c = Dv ? (float)(xn / (double)Dv) : 0.0f;
+  __stcg(a.contrib[0] + v, c);
+  if (!Dv) my_dang += xn;
+  return true;
+}
+
+template <bool SLOTS>
+__global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, PbArgs p) {
+  extern __shared__ __align__(16) unsigned char pb_smem[];
+  uint32_t* acc_lo = reinterpret_cast<uint32_t*>(pb_smem);
+  uint32_t* acc_hi = acc_lo + PB_R + 8;
+  float* s_c = reinterpret_cast<float*>(acc_lo);   // terms, written over acc_lo by (2)
+  unsigned char* ring = pb_smem + PB_RING_OFF;
+  __shared__ double s_red[32];
+  __shared__ int s_bin;
+  __shared__ __align__(8) uint64_t full[PB_NST], empty[PB_NST];
+  PrState* st = a.st;
+  if (st->stop) return;
+  const unsigned t = st->iter;
+  const double sc = st->scale;
+  const double addc = a.base + a.damp * sc * st->dang[t % 3] * a.invN;
+  const bool merge_now = st->do_merge != 0;
+  double my_delta = 0, my_dang = 0, my_mass = 0;
+  const uint64_t pf = l2_evict_first();
+  const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
+  constexpr unsigned NW = PB_THREADS / 32;
+  const int64_t nb = p.nb;
+  const uint32_t* qend = p.q + nb * nb;
+  const double inv_fix = 1.0 / 72057594037927936.0;   // 2^-56
+  if (threadIdx.x < 8) acc_lo[PB_R + threadIdx.x] = 0u;  // s_c[R..R+7] = 0.0f
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < PB_NST; i++) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], NW);
+    }
+    mbar_fence_init();
+  }
+  uint32_t g = 0;   // chunks this CTA has consumed (ring position), same in every thread
+  for (;;) {
+    if (threadIdx.x == 0) s_bin = (int)atomicAdd(&st->pb_next[t % 3], 1u);
+    for (int i = threadIdx.x; i < PB_R / 4; i += PB_THREADS) {
+      reinterpret_cast<uint4*>(acc_lo)[i] = make_uint4(0, 0, 0, 0);
+      reinterpret_cast<uint4*>(acc_hi)[i] = make_uint4(0, 0, 0, 0);
+    }
+    __syncthreads();
+    const int64_t b = s_bin;
+    if (b >= nb) break;
+    const int64_t base = b * PB_R;
+    const int nrows = (int)min((int64_t)PB_R, a.n_slots - base);
+    const uint32_t* r0 = p.q + b * nb;   // block b's scatter segments: [r0[j], r1[j])
+    const uint32_t* r1 = r0 + nb;
+    // (1) the bin's in-edges: one contiguous range, bulk-copied chunk by chunk
+    // into a PB_NST-stage shared-memory ring (one thread issues; each warp
+    // releases a stage when it has added its part)
+    const uint32_t E0 = __ldg(p.q + b), E1 = __ldg(qend + b);
+    const uint32_t nch = (E1 - E0 + PB_CH - 1) / PB_CH;
+    auto issue = [&](uint32_t c) {   // thread 0 only
+      const uint32_t gc = g + c, stg = gc % PB_NST;
+      if (gc >= PB_NST) mbar_wait(&empty[stg], ((gc / PB_NST) - 1) & 1);
+      const uint32_t e = E0 + c * PB_CH, n = min((uint32_t)PB_CH, E1 - e);
+      unsigned char* dst = ring + stg * PB_STAGE;
+      mbar_expect_tx(&full[stg], n * 6);
+      tma_load_1d(dst, p.val + e, n * 4, &full[stg], pf);
+      tma_load_1d(dst + PB_CH * 4, p.dst_loc + e, n * 2, &full[stg], pf);
+    };
+    if (threadIdx.x == 0) {
+      for (uint32_t c = 0; c < nch && c < PB_NST; c++) issue(c);
+      // L2 prefetch for (2) and (3)
+      l2_prefetch_bulk(a.x + base, (uint32_t)nrows * 8u);
+      l2_prefetch_bulk(a.D + base, (uint32_t)nrows * 4u);
+    }
+    for (int64_t j = threadIdx.x; j < nb; j += PB_THREADS) {
+      const uint32_t lo = __ldg(r0 + j), hi = __ldg(r1 + j);
+      if (hi > lo) l2_prefetch_bulk(p.src_loc + lo, (hi - lo) * 2u);
+    }
+    for (uint32_t c = 0; c < nch; c++) {
+      const uint32_t gc = g + c, stg = gc % PB_NST;
+      const uint32_t n = min((uint32_t)PB_CH, E1 - (E0 + c * PB_CH));
+      mbar_wait(&full[stg], (gc / PB_NST) & 1);
+      const unsigned char* src = ring + stg * PB_STAGE;
+      const uint32_t i = 4u * threadIdx.x;
+      if (i < n) {
+        const float4 tv = *reinterpret_cast<const float4*>(src + 4 * i);
+        const uint2 rv = *reinterpret_cast<const uint2*>(src + PB_CH * 4 + 2 * i);
+        pb_add4(acc_lo, acc_hi, rv, tv);
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[stg]);
+      if (threadIdx.x == 0 && c + PB_NST < nch) issue(c + PB_NST);
+    }
+    g += nch;
+    __syncthreads();
+    // (2) the PR update of the bin's rows
+    for (int i0 = threadIdx.x; i0 < nrows; i0 += PB_THREADS * 4) {
+      double xo[4];
+      uint32_t Dv[4];
+#pragma unroll
+      for (int u = 0; u < 4; u++) {
+        const int i = i0 + u * PB_THREADS;
+        xo[u] = i < nrows ? __ldcs(a.x + base + i) : 0.0;
+        Dv[u] = i < nrows ? __ldcs(a.D + base + i) : 0u;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; u++) {
+        const int i = i0 + u * PB_THREADS;
+        if (i < nrows) {
+          const int64_t v = base + i;
+          float c = 0.0f;
+          const unsigned long long fx = ((unsigned long long)acc_hi[i] << 32) | acc_lo[i];
+          if (!pb_update<SLOTS>(a, v, (double)fx * inv_fix, xo[u], Dv[u], addc, merge_now, sc, my_delta, my_dang,
+                                my_mass, c))
+            c = __ldcg(a.contrib[0] + v);
+          s_c[i] = c;
+        }
+      }
+    }
+    __syncthreads();
+    // (3) scatter the new terms along block b's segments, 4 segments per step
+    for (int64_t j0 = (int64_t)warp * 32; j0 < nb; j0 += 32 * NW) {
+      const int64_t j = j0 + lane;
+      const uint32_t lo = j < nb ? __ldg(r0 + j) : 0u, hi = j < nb ? __ldg(r1 + j) : 0u;
+      const int kn = (int)min((int64_t)32, nb - j0);
+      for (int k = 0; k < kn; k += 4) {
+        uint32_t ee[4], hh[4];
+        uint4 w[4];
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+          ee[u] = __shfl_sync(FULL, lo, k + u) + 8u * lane;
+          hh[u] = __shfl_sync(FULL, hi, k + u);
+          if (ee[u] < hh[u]) w[u] = ld_stream_v4(reinterpret_cast<const uint32_t*>(p.src_loc + ee[u]), pf);
+        }
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+          if (ee[u] < hh[u]) pb_put8(p.val + ee[u], s_c, w[u]);
+          for (uint32_t e = ee[u] + 256u; e < hh[u]; e += 256u)
+            pb_put8(p.val + e, s_c, ld_stream_v4(reinterpret_cast<const uint32_t*>(p.src_loc + e), pf));
+        }
+      }
+    }
+    __syncthreads();   // s_c (= acc_lo) is zeroed for the next bin
+  }
+  pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
+}
+
+// val[] <- the initial terms contrib_0[u] along every edge (CTA per sink bin;
+// the source block of each segment is found by walking the bin's row of q)
+__global__ void k_pb_init_val(PbArgs p, const float* __restrict__ contrib, int64_t n_slots) {
+  for (int64_t b = blockIdx.x; b < p.nb; b += gridDim.x) {
+    for (int64_t s = 0; s < p.nb; s++) {
+      const uint32_t e0 = p.q[s * p.nb + b], e1 = p.q[(s + 1) * p.nb + b];
+      const float* cb = contrib + s * PB_R;
+      for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) {
+        const uint32_t sl = p.src_loc[e];
+        p.val[e] = sl < PB_R && s * PB_R + sl < n_slots ? __ldg(cb + sl) : 0.0f;
+      }
+    }
+  }
+}
+
 // The paper's thread-per-vertex pull (tpv.cu): lane = slot of the schedule,
 // each lane sums its own in-edges from the SELL-32 slab and finalises its
 // slot; a warp lasts as long as its longest row (what §4 normalises).
@@ -546,6 +813,7 @@ __global__ void k_pr_advance(PrState* st, double tol, int max_iters) {
   const double ms = st->mass[(t + 1) % 3];
   st->scale = (st->normalize && ms > 0.0) ? 1.0 / ms : 1.0;
   st->delta[(t + 2) % 3] = 0.0;
+  st->pb_next[(t + 2) % 3] = 0u;
   st->dang[(t + 2) % 3] = 0.0;
   st->mass[(t + 2) % 3] = 0.0;
   st->iter = t + 1;
@@ -598,6 +866,7 @@ __global__ void k_pr_init(PrArgs a, int64_t n_slots, double x0) {
 }
 
 void ensure_csc(gx_graph* g);  // devgraph.cu
+void ensure_pb(gx_graph* g);   // devgraph.cu
 void ensure_tpv(gx_graph* g);  // tpv.cu
 
 __global__ void k_mask_outside(double* __restrict__ x, int64_t n, int64_t lo, int64_t hi) {
@@ -721,6 +990,7 @@ static void run_pagerank_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& in
   info.vertices_active = (int64_t)h.iter * ns;
   info.bytes_model = (int64_t)h.iter * (8 * d.m_slots + 24 * ns);
   info.kernel_launches = launches;
+  info.mapping_used = GX_MAP_LB;
   r.have[GX_PAGERANK] = true;
 }
 
@@ -781,8 +1051,28 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     }
   }
   int mapping = o.mapping;
-  if (mapping == GX_MAP_AUTO)
-    mapping = (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
+  const bool tiles = d.n_tiles && g->knobs.smem;
+  if (mapping == GX_MAP_AUTO) {
+    const bool pb_ok = async && !tiles && (ns + PB_R - 1) / PB_R >= GX_PB_MIN_BLOCKS && !getenv("GX_NO_PB");
+    mapping = pb_ok ? GX_MAP_PB
+                    : (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
+  }
+  GX_CHECK_ARG(mapping != GX_MAP_PB || async, "the blocked mapping runs the asynchronous schedule");
+  PbArgs pb{};
+  if (mapping == GX_MAP_PB) {
+    ensure_pb(g);
+    pb.q = d.pr_pb.q.as<uint32_t>();
+    pb.src_loc = d.pr_pb.src_loc.as<uint16_t>();
+    pb.dst_loc = d.pr_pb.dst_loc.as<uint16_t>();
+    pb.val = d.pr_pb.val.as<float>();
+    pb.nb = d.pr_pb.nb;
+    static bool attr = false;
+    if (!attr) {
+      CUDA_OK(cudaFuncSetAttribute(k_pr_pb<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
+      CUDA_OK(cudaFuncSetAttribute(k_pr_pb<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
+      attr = true;
+    }
+  }
   if (mapping == GX_MAP_TPV) {
     ensure_tpv(g);
     a.tpv_lane_row = d.tpv_lane_row.as<int32_t>();
@@ -800,8 +1090,10 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   int gi = grid_for(c, ns);
   if (slots) k_pr_init<true><<<gi, 256, 0, s>>>(a, ns, 1.0 / (double)g->n);
   else k_pr_init<false><<<gi, 256, 0, s>>>(a, ns, 1.0 / (double)g->n);
+  if (mapping == GX_MAP_PB) k_pb_init_val<<<(int)std::min<int64_t>(pb.nb, c->num_sms * 8), 256, 0, s>>>(pb, a.contrib[0], ns);
   CUDA_OK(cudaGetLastError());
-  int launches = 1;
+  int launches = mapping == GX_MAP_PB ? 2 : 1;
+  const int grid_pb = (int)std::max<int64_t>(1, std::min<int64_t>(pb.nb, (int64_t)c->num_sms * PB_CTAS_PER_SM));
 
   // GX_PR_KERNEL=1 selects the round-1 kernel (A/B experiments)
   const bool v2 = !(getenv("GX_PR_KERNEL") && atoi(getenv("GX_PR_KERNEL")) == 1);
@@ -818,7 +1110,10 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   KTimer kt(o.profile != 0, s);
   auto one_iter = [&](int& nl) {
     kt.begin();
-    if (mapping == GX_MAP_TPV) {
+    if (mapping == GX_MAP_PB) {
+      if (slots) k_pr_pb<true><<<grid_pb, PB_THREADS, PB_SMEM, s>>>(a, pb);
+      else k_pr_pb<false><<<grid_pb, PB_THREADS, PB_SMEM, s>>>(a, pb);
+    } else if (mapping == GX_MAP_TPV) {
       if (async) {
         if (slots) k_pr_tpv<true, true><<<grid_tpv, 256, 0, s>>>(a);
         else k_pr_tpv<false, true><<<grid_tpv, 256, 0, s>>>(a);
@@ -845,7 +1140,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     }
     kt.end();
     nl++;
-    if (d.n_tiles && g->knobs.smem) {
+    if (tiles) {
       const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 24));
       if (slots)
         k_pr_local<true><<<grid_local, PRL_THREADS, 0, s>>>(a, d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(),
@@ -904,10 +1199,15 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   // bytes model: 8 B per in-edge (source id 4 + contrib gather 4) and
   // 24 B per slot (x read 8 + x write 8 + contrib write 4 + D 4)
   info.bytes_model = (int64_t)h.iter * (8 * d.m_slots + 24 * ns);
+  // blocked mapping (k_pr_pb): 12 B per edge (val 4 + sink index 2 read, source
+  // index 2 read + val 4 written) and 28 B per slot (x r/w 16, D 4, contrib
+  // write 4, the bin's segment offsets ~4)
+  if (mapping == GX_MAP_PB) info.bytes_model = (int64_t)h.iter * (12 * d.m_slots + 28 * ns);
   info.kernel_launches = launches;
   info.sweep_launches = kt.launches();
   info.sweep_ms = kt.total_ms();
   info.sweep_bytes = info.bytes_model;
+  info.mapping_used = mapping;
   r.have[GX_PAGERANK] = true;
 }
 

@@ -1133,7 +1133,7 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     run_sssp_dist(g, o, info, P, sim, src, delta);
     return;
   }
-  int mapping = o.mapping;
+  int mapping = o.mapping == GX_MAP_PB ? GX_MAP_LB : o.mapping;   // PB is a PageRank mapping
   if (mapping == GX_MAP_AUTO)
     mapping = (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
   if (mapping == GX_MAP_TPV) ensure_tpv(g);
@@ -1364,6 +1364,7 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   info.sweep_launches = kt.launches();
   info.sweep_ms = kt.total_ms();
   info.sweep_bytes = info.bytes_model;
+  info.mapping_used = mapping;
   r.have[GX_SSSP] = true;
 }
 

@@ -49,18 +49,54 @@ def test_sssp_exact_bit_exact(name, mode):
 
 
 @pytest.mark.parametrize("name", list(GRAPHS))
-def test_pagerank_exact_l1(name):
+@pytest.mark.parametrize("mapping", ["lb", "pb"])
+def test_pagerank_exact_l1(name, mapping):
     raw = GRAPHS[name]()
     g = from_raw(raw)
     want, _ = A.pagerank(graph_to_edgelist(g), tol=1e-14)
     G = upload(raw)
-    info = G.run("pagerank", tol=1e-10, max_iters=5000, mapping="lb")
+    info = G.run("pagerank", tol=1e-10, max_iters=5000, mapping=mapping)
     got = G.download("rank")
     # fp32 contrib: the delta floor sits near 1e-10 on some graphs;
     # parity is the L1 bar either way
     l1 = np.abs(got - want).sum()
     assert l1 <= 1e-6, l1
     assert abs(got.sum() - 1.0) < 1e-6
+
+
+PB_GRAPHS = {   # several 16384-slot blocks each, ragged last block
+    "rmat17": lambda: graphgen.rmat(17),
+    "uniform_ragged": lambda: graphgen.uniform(100003, 1600000),
+    "road300": lambda: graphgen.road(300),
+    "hub_rows": lambda: graphgen.from_edge_list(
+        40000, [(v, 7, 1) for v in range(40000) if v != 7] + [(7, v, 1) for v in range(0, 40000, 5)]
+        + [(v, (v * 31 + 11) % 40000, 1) for v in range(40000)]),
+}
+
+
+@pytest.mark.parametrize("name", list(PB_GRAPHS))
+def test_pagerank_blocked_multiblock(name):
+    """The propagation-blocked pull (GX_MAP_PB) across several source blocks /
+    sink bins, incl. a ragged last block, in-hub and out-hub rows, dangling
+    vertices: L1 <= 1e-6 against the oracle; the LB kernel agrees too."""
+    raw = PB_GRAPHS[name]()
+    g = from_raw(raw)
+    want, _ = A.pagerank(graph_to_edgelist(g), tol=1e-14)
+    G = upload(raw)
+    info = G.run("pagerank", tol=1e-10, max_iters=5000, mapping="pb")
+    got = G.download("rank")
+    assert info["converged"] >= 1
+    assert np.abs(got - want).sum() <= 1e-6
+    assert abs(got.sum() - 1.0) < 1e-6
+    G.run("pagerank", tol=1e-10, max_iters=5000, mapping="lb")
+    assert np.abs(G.download("rank") - want).sum() <= 1e-6
+
+
+def test_pagerank_blocked_needs_async():
+    import paper_conf_icpp_0001n20_b200 as gx
+    G = upload(graphgen.rmat(10))
+    with pytest.raises(gx.GraffixError):
+        G.run("pagerank", mapping="pb", pr_schedule="jacobi")
 
 
 def test_sssp_max_iters_not_an_error():
@@ -139,7 +175,7 @@ def test_full_size_certificates(cfg):
     dist = G.download("dist")
     cert = sssp_certificate(g, s, dist)
     assert cert["ok"], cert
-    info = G.run("pagerank", tol=1e-9, mapping="lb")
+    info = G.run("pagerank", tol=1e-9)   # AUTO: the blocked pull at these sizes (bench.py's default)
     x = G.download("rank")
     if knobs:   # G_L of the transformed run (replica rows folded into the owner)
         ex = G.export()

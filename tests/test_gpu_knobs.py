@@ -63,7 +63,7 @@ def test_sssp_transformed_bit_exact(gname, kname, mapping):
 
 @pytest.mark.parametrize("gname", list(GRAPHS))
 @pytest.mark.parametrize("kname", list(KNOBS))
-@pytest.mark.parametrize("mapping", ["lb", "tpv"])
+@pytest.mark.parametrize("mapping", ["lb", "tpv", "pb"])
 def test_pagerank_transformed_l1(gname, kname, mapping):
     raw = GRAPHS[gname]()
     g = from_raw(raw)
@@ -168,7 +168,7 @@ def test_sssp_merge_cadence(gname, c, mapping):
 
 @pytest.mark.parametrize("gname", ["road48", "rmat12"])
 @pytest.mark.parametrize("c", [2, 0])
-@pytest.mark.parametrize("schedule", ["jacobi", "async"])
+@pytest.mark.parametrize("schedule", ["jacobi", "async", "async_pb"])
 def test_pagerank_merge_cadence(gname, c, schedule):
     from oracle import slotsim as S
     raw = GRAPHS[gname]()
@@ -177,7 +177,9 @@ def test_pagerank_merge_cadence(gname, c, schedule):
     want = A.pagerank(tg.logical(), tol=1e-14)[0] if c else S.pagerank_slots(tg, tol=1e-14, merge_every=0)[0]
     G = upload(raw)
     G.transform(knobs_c(kn))
-    G.run("pagerank", tol=1e-12, max_iters=20000, mapping="lb", pr_schedule=schedule, merge_every=c)
+    mapping = "pb" if schedule == "async_pb" else "lb"
+    G.run("pagerank", tol=1e-12, max_iters=20000, mapping=mapping, pr_schedule=schedule.split("_")[0],
+          merge_every=c)
     assert np.abs(G.download("rank") - want).sum() <= 1e-6
 
 
