@@ -447,6 +447,41 @@ __device__ __forceinline__ bool pb_update(const PrArgs& a, int64_t v, double y, 
   return true;
 }
 
+// (3): the terms s_c[0..PB_R) of one source block along its nb segments
+// [r0[j], r1[j]) (16-byte aligned runs of 8-entry groups), 4 segments per warp
+// step: one 16-byte load of source indices and two float4 stores per lane.
+// lo0 / hi0 = the bounds of segment threadIdx.x (already loaded by the caller).
+__device__ __forceinline__ void pb_scatter(const PbArgs& p, const float* s_c, const uint32_t* r0, const uint32_t* r1,
+                                           uint32_t lo0, uint32_t hi0, uint64_t pf) {
+  const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
+  constexpr unsigned NW = PB_THREADS / 32;
+  static_assert(32 * NW == PB_THREADS, "segment j0 + lane of the first pass is thread j");
+  const int64_t nb = p.nb;
+  for (int64_t j0 = (int64_t)warp * 32; j0 < nb; j0 += 32 * NW) {
+    const int64_t j = j0 + lane;
+    const bool first = j0 < 32 * NW;
+    const uint32_t lo = first ? lo0 : j < nb ? __ldg(r0 + j) : 0u;
+    const uint32_t hi = first ? hi0 : j < nb ? __ldg(r1 + j) : 0u;
+    const int kn = (int)min((int64_t)32, nb - j0);
+    for (int k = 0; k < kn; k += 4) {
+      uint32_t ee[4], hh[4];
+      uint4 w[4];
+#pragma unroll
+      for (int u = 0; u < 4; u++) {
+        ee[u] = __shfl_sync(FULL, lo, k + u) + 8u * lane;
+        hh[u] = __shfl_sync(FULL, hi, k + u);
+        if (ee[u] < hh[u]) w[u] = ld_stream_v4(reinterpret_cast<const uint32_t*>(p.src_loc + ee[u]), pf);
+      }
+#pragma unroll
+      for (int u = 0; u < 4; u++) {
+        if (ee[u] < hh[u]) pb_put8(p.val + ee[u], s_c, w[u]);
+        for (uint32_t e = ee[u] + 256u; e < hh[u]; e += 256u)
+          pb_put8(p.val + e, s_c, ld_stream_v4(reinterpret_cast<const uint32_t*>(p.src_loc + e), pf));
+      }
+    }
+  }
+}
+
 template <bool SLOTS>
 __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, PbArgs p) {
   extern __shared__ __align__(16) unsigned char pb_smem[];
@@ -479,6 +514,16 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
     mbar_fence_init();
   }
   uint32_t g = 0;   // chunks this CTA has consumed (ring position), same in every thread
+  // (1)'s producer (thread 0): chunk c of the range [e_lo, e_hi) into ring slot gc
+  auto issue = [&](uint32_t gc, uint32_t e_lo, uint32_t e_hi, uint32_t c) {
+    const uint32_t stg = gc % PB_NST;
+    if (gc >= PB_NST) mbar_wait(&empty[stg], ((gc / PB_NST) - 1) & 1);
+    const uint32_t e = e_lo + c * PB_CH, n = min((uint32_t)PB_CH, e_hi - e);
+    unsigned char* dst = ring + stg * PB_STAGE;
+    mbar_expect_tx(&full[stg], n * 6);
+    tma_load_1d(dst, p.val + e, n * 4, &full[stg], pf);
+    tma_load_1d(dst + PB_CH * 4, p.dst_loc + e, n * 2, &full[stg], pf);
+  };
   for (;;) {
     if (threadIdx.x == 0) s_bin = (int)atomicAdd(&st->pb_next[t % 3], 1u);
     for (int i = threadIdx.x; i < PB_R / 4; i += PB_THREADS) {
@@ -494,26 +539,25 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
     const uint32_t* r1 = r0 + nb;
     // (1) the bin's in-edges: one contiguous range, bulk-copied chunk by chunk
     // into a PB_NST-stage shared-memory ring (one thread issues; each warp
-    // releases a stage when it has added its part)
+    // releases a stage when it has added its part).  (Claiming the next bin
+    // and starting its first chunks during (3) was measured 15 % slower: the
+    // claiming warp's delay holds the whole CTA at the end of (3).)
     const uint32_t E0 = __ldg(p.q + b), E1 = __ldg(qend + b);
     const uint32_t nch = (E1 - E0 + PB_CH - 1) / PB_CH;
-    auto issue = [&](uint32_t c) {   // thread 0 only
-      const uint32_t gc = g + c, stg = gc % PB_NST;
-      if (gc >= PB_NST) mbar_wait(&empty[stg], ((gc / PB_NST) - 1) & 1);
-      const uint32_t e = E0 + c * PB_CH, n = min((uint32_t)PB_CH, E1 - e);
-      unsigned char* dst = ring + stg * PB_STAGE;
-      mbar_expect_tx(&full[stg], n * 6);
-      tma_load_1d(dst, p.val + e, n * 4, &full[stg], pf);
-      tma_load_1d(dst + PB_CH * 4, p.dst_loc + e, n * 2, &full[stg], pf);
-    };
     if (threadIdx.x == 0) {
-      for (uint32_t c = 0; c < nch && c < PB_NST; c++) issue(c);
+      for (uint32_t c = 0; c < nch && c < PB_NST; c++) issue(g + c, E0, E1, c);
       // L2 prefetch for (2) and (3)
       l2_prefetch_bulk(a.x + base, (uint32_t)nrows * 8u);
       l2_prefetch_bulk(a.D + base, (uint32_t)nrows * 4u);
     }
+    // (3)'s first PB_THREADS segment bounds stay in registers
+    uint32_t lo0 = 0, hi0 = 0;
     for (int64_t j = threadIdx.x; j < nb; j += PB_THREADS) {
       const uint32_t lo = __ldg(r0 + j), hi = __ldg(r1 + j);
+      if (j == threadIdx.x) {
+        lo0 = lo;
+        hi0 = hi;
+      }
       if (hi > lo) l2_prefetch_bulk(p.src_loc + lo, (hi - lo) * 2u);
     }
     for (uint32_t c = 0; c < nch; c++) {
@@ -529,7 +573,7 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
       }
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stg]);
-      if (threadIdx.x == 0 && c + PB_NST < nch) issue(c + PB_NST);
+      if (threadIdx.x == 0 && c + PB_NST < nch) issue(gc + PB_NST, E0, E1, c + PB_NST);
     }
     g += nch;
     __syncthreads();
@@ -558,45 +602,30 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
       }
     }
     __syncthreads();
-    // (3) scatter the new terms along block b's segments, 4 segments per step
-    for (int64_t j0 = (int64_t)warp * 32; j0 < nb; j0 += 32 * NW) {
-      const int64_t j = j0 + lane;
-      const uint32_t lo = j < nb ? __ldg(r0 + j) : 0u, hi = j < nb ? __ldg(r1 + j) : 0u;
-      const int kn = (int)min((int64_t)32, nb - j0);
-      for (int k = 0; k < kn; k += 4) {
-        uint32_t ee[4], hh[4];
-        uint4 w[4];
-#pragma unroll
-        for (int u = 0; u < 4; u++) {
-          ee[u] = __shfl_sync(FULL, lo, k + u) + 8u * lane;
-          hh[u] = __shfl_sync(FULL, hi, k + u);
-          if (ee[u] < hh[u]) w[u] = ld_stream_v4(reinterpret_cast<const uint32_t*>(p.src_loc + ee[u]), pf);
-        }
-#pragma unroll
-        for (int u = 0; u < 4; u++) {
-          if (ee[u] < hh[u]) pb_put8(p.val + ee[u], s_c, w[u]);
-          for (uint32_t e = ee[u] + 256u; e < hh[u]; e += 256u)
-            pb_put8(p.val + e, s_c, ld_stream_v4(reinterpret_cast<const uint32_t*>(p.src_loc + e), pf));
-        }
-      }
-    }
+    // (3) scatter the new terms along block b's segments
+    pb_scatter(p, s_c, r0, r1, lo0, hi0, pf);
     __syncthreads();   // s_c (= acc_lo) is zeroed for the next bin
   }
   pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
 }
 
-// val[] <- the initial terms contrib_0[u] along every edge (CTA per sink bin;
-// the source block of each segment is found by walking the bin's row of q)
-__global__ void k_pb_init_val(PbArgs p, const float* __restrict__ contrib, int64_t n_slots) {
+// val[] <- the initial terms contrib_0[u] along every edge: (3) for every
+// source block with s_c = contrib_0 of the block
+__global__ void __launch_bounds__(PB_THREADS, 1) k_pb_init_val(PbArgs p, const float* __restrict__ contrib,
+                                                               int64_t n_slots) {
+  extern __shared__ __align__(16) float pb_init_s[];
+  float* s_c = pb_init_s;   // PB_R + 8 floats
+  const uint64_t pf = l2_evict_first();
+  if (threadIdx.x < 8) s_c[PB_R + threadIdx.x] = 0.0f;
   for (int64_t b = blockIdx.x; b < p.nb; b += gridDim.x) {
-    for (int64_t s = 0; s < p.nb; s++) {
-      const uint32_t e0 = p.q[s * p.nb + b], e1 = p.q[(s + 1) * p.nb + b];
-      const float* cb = contrib + s * PB_R;
-      for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) {
-        const uint32_t sl = p.src_loc[e];
-        p.val[e] = sl < PB_R && s * PB_R + sl < n_slots ? __ldg(cb + sl) : 0.0f;
-      }
-    }
+    const int64_t base = b * PB_R;
+    for (int i = threadIdx.x; i < PB_R; i += PB_THREADS) s_c[i] = base + i < n_slots ? contrib[base + i] : 0.0f;
+    const uint32_t* r0 = p.q + b * p.nb;
+    const uint32_t* r1 = r0 + p.nb;
+    const uint32_t lo0 = threadIdx.x < p.nb ? r0[threadIdx.x] : 0u, hi0 = threadIdx.x < p.nb ? r1[threadIdx.x] : 0u;
+    __syncthreads();
+    pb_scatter(p, s_c, r0, r1, lo0, hi0, pf);
+    __syncthreads();
   }
 }
 
@@ -1070,6 +1099,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     if (!attr) {
       CUDA_OK(cudaFuncSetAttribute(k_pr_pb<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
       CUDA_OK(cudaFuncSetAttribute(k_pr_pb<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
+      CUDA_OK(cudaFuncSetAttribute(k_pb_init_val, cudaFuncAttributeMaxDynamicSharedMemorySize, (PB_R + 8) * 4));
       attr = true;
     }
   }
@@ -1090,7 +1120,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   int gi = grid_for(c, ns);
   if (slots) k_pr_init<true><<<gi, 256, 0, s>>>(a, ns, 1.0 / (double)g->n);
   else k_pr_init<false><<<gi, 256, 0, s>>>(a, ns, 1.0 / (double)g->n);
-  if (mapping == GX_MAP_PB) k_pb_init_val<<<(int)std::min<int64_t>(pb.nb, c->num_sms * 8), 256, 0, s>>>(pb, a.contrib[0], ns);
+  if (mapping == GX_MAP_PB) k_pb_init_val<<<(int)std::min<int64_t>(pb.nb, c->num_sms * 2), PB_THREADS, (PB_R + 8) * 4, s>>>(pb, a.contrib[0], ns);
   CUDA_OK(cudaGetLastError());
   int launches = mapping == GX_MAP_PB ? 2 : 1;
   const int grid_pb = (int)std::max<int64_t>(1, std::min<int64_t>(pb.nb, (int64_t)c->num_sms * PB_CTAS_PER_SM));
