@@ -1229,14 +1229,14 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   // bytes model: 8 B per in-edge (source id 4 + contrib gather 4) and
   // 24 B per slot (x read 8 + x write 8 + contrib write 4 + D 4)
   info.bytes_model = (int64_t)h.iter * (8 * d.m_slots + 24 * ns);
-  // blocked mapping (k_pr_pb): 12 B per edge (val 4 + sink index 2 read, source
-  // index 2 read + val 4 written) and 28 B per slot (x r/w 16, D 4, contrib
-  // write 4, the bin's segment offsets ~4)
-  if (mapping == GX_MAP_PB) info.bytes_model = (int64_t)h.iter * (12 * d.m_slots + 28 * ns);
   info.kernel_launches = launches;
   info.sweep_launches = kt.launches();
   info.sweep_ms = kt.total_ms();
-  info.sweep_bytes = info.bytes_model;
+  // the bytes the sweep kernel's own encoding moves: the blocked mapping
+  // (k_pr_pb) streams 12 B per edge (val 4 + sink index 2 read, source index 2
+  // read + val 4 written) and 28 B per slot (x r/w 16, D 4, contrib write 4,
+  // segment offsets ~4) instead of the pull's 8 B gather per edge
+  info.sweep_bytes = mapping == GX_MAP_PB ? (int64_t)h.iter * (12 * d.m_slots + 28 * ns) : info.bytes_model;
   info.mapping_used = mapping;
   r.have[GX_PAGERANK] = true;
 }
