@@ -452,14 +452,13 @@ __device__ __forceinline__ bool pb_update(const PrArgs& a, int64_t v, double y, 
 // step: one 16-byte load of source indices and two float4 stores per lane.
 // lo0 / hi0 = the bounds of segment threadIdx.x (already loaded by the caller).
 __device__ __forceinline__ void pb_scatter(const PbArgs& p, const float* s_c, const uint32_t* r0, const uint32_t* r1,
-                                           uint32_t lo0, uint32_t hi0, uint64_t pf) {
-  const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
-  constexpr unsigned NW = PB_THREADS / 32;
-  static_assert(32 * NW == PB_THREADS, "segment j0 + lane of the first pass is thread j");
+                                           uint32_t lo0, uint32_t hi0, uint64_t pf, unsigned warp = threadIdx.x >> 5,
+                                           unsigned NW = PB_THREADS / 32, bool cached = true) {
+  const unsigned lane = lane_id();
   const int64_t nb = p.nb;
   for (int64_t j0 = (int64_t)warp * 32; j0 < nb; j0 += 32 * NW) {
     const int64_t j = j0 + lane;
-    const bool first = j0 < 32 * NW;
+    const bool first = cached && j0 < 32 * NW;   // then segment j is thread j's (lo0, hi0)
     const uint32_t lo = first ? lo0 : j < nb ? __ldg(r0 + j) : 0u;
     const uint32_t hi = first ? hi0 : j < nb ? __ldg(r1 + j) : 0u;
     const int kn = (int)min((int64_t)32, nb - j0);
@@ -609,6 +608,131 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
   pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
 }
 
+// Warp-specialised variant (GX_PB_KERNEL=2): the CTA's warps are split into
+// group A (PB2_NA warps: phase (1) of bin b_k, plain 16-byte loads, 16 terms
+// per thread in flight) and group B (the rest: phase (3) of bin b_{k-1}) that
+// run at the same time on separate shared-memory arrays (acc vs s_c), so one
+// bin's stream and the previous bin's scatter overlap on every SM; then all
+// warps run (2) for b_k, which zeroes acc as it reads it and fills s_c.
+#ifndef GX_PB2_NA
+#define GX_PB2_NA 20
+#endif
+constexpr int PB2_NA = GX_PB2_NA;
+constexpr size_t PB2_SMEM = (size_t)PB_R * 8 + 32 + (size_t)(PB_R + 8) * 4;
+
+__device__ __forceinline__ void pb_add8(uint32_t* lo, uint32_t* hi, uint4 r, float4 v0, float4 v1) {
+  pb_add4(lo, hi, make_uint2(r.x, r.y), v0);
+  pb_add4(lo, hi, make_uint2(r.z, r.w), v1);
+}
+
+template <bool SLOTS>
+__global__ void __launch_bounds__(PB_THREADS, 1) k_pr_pb2(PrArgs a, PbArgs p) {
+  extern __shared__ __align__(16) unsigned char pb_smem[];
+  uint32_t* acc_lo = reinterpret_cast<uint32_t*>(pb_smem);
+  uint32_t* acc_hi = acc_lo + PB_R + 8;
+  float* s_c = reinterpret_cast<float*>(acc_hi + PB_R);   // PB_R + 8 terms (last 8 = 0)
+  __shared__ double s_red[32];
+  __shared__ int s_bin;
+  PrState* st = a.st;
+  if (st->stop) return;
+  const unsigned t = st->iter;
+  const double sc = st->scale;
+  const double addc = a.base + a.damp * sc * st->dang[t % 3] * a.invN;
+  const bool merge_now = st->do_merge != 0;
+  double my_delta = 0, my_dang = 0, my_mass = 0;
+  const uint64_t pf = l2_evict_first();
+  const unsigned warp = threadIdx.x >> 5;
+  const bool grpA = warp < (unsigned)PB2_NA;
+  const int64_t nb = p.nb;
+  const uint32_t* qend = p.q + nb * nb;
+  const double inv_fix = 1.0 / 72057594037927936.0;   // 2^-56
+  if (threadIdx.x < 8) s_c[PB_R + threadIdx.x] = 0.0f;
+  for (int i = threadIdx.x; i < PB_R / 4; i += PB_THREADS) {
+    reinterpret_cast<uint4*>(acc_lo)[i] = make_uint4(0, 0, 0, 0);
+    reinterpret_cast<uint4*>(acc_hi)[i] = make_uint4(0, 0, 0, 0);
+  }
+  if (threadIdx.x == 0) s_bin = (int)atomicAdd(&st->pb_next[t % 3], 1u);
+  __syncthreads();
+  int64_t bcur = s_bin, bprev = nb;
+  while (bcur < nb || bprev < nb) {
+    if (grpA) {
+      if (bcur < nb) {
+        const int64_t base = bcur * PB_R;
+        const int nrows = (int)min((int64_t)PB_R, a.n_slots - base);
+        const unsigned ta = threadIdx.x;
+        if (ta == 0) {
+          l2_prefetch_bulk(a.x + base, (uint32_t)nrows * 8u);
+          l2_prefetch_bulk(a.D + base, (uint32_t)nrows * 4u);
+        }
+        const uint32_t* r0 = p.q + bcur * nb;
+        for (int64_t j = ta; j < nb; j += PB2_NA * 32) {   // next slot's scatter segments
+          const uint32_t lo = __ldg(r0 + j), hi = __ldg(r0 + nb + j);
+          if (hi > lo) l2_prefetch_bulk(p.src_loc + lo, (hi - lo) * 2u);
+        }
+        // (1) the bin's contiguous in-edge range
+        const uint32_t E0 = __ldg(p.q + bcur), E1 = __ldg(qend + bcur);
+        constexpr uint32_t STEP = 8u * PB2_NA * 32;
+        for (uint32_t e = E0 + 8u * ta; e < E1; e += 2 * STEP) {
+          const bool two = e + STEP < E1;
+          const uint4 ra = ld_stream_v4(reinterpret_cast<const uint32_t*>(p.dst_loc + e), pf);
+          const float4 va0 = ld_cg_f4(p.val + e), va1 = ld_cg_f4(p.val + e + 4);
+          uint4 rb = make_uint4(0, 0, 0, 0);
+          float4 vb0 = make_float4(0, 0, 0, 0), vb1 = vb0;
+          if (two) {
+            rb = ld_stream_v4(reinterpret_cast<const uint32_t*>(p.dst_loc + e + STEP), pf);
+            vb0 = ld_cg_f4(p.val + e + STEP);
+            vb1 = ld_cg_f4(p.val + e + STEP + 4);
+          }
+          pb_add8(acc_lo, acc_hi, ra, va0, va1);
+          pb_add8(acc_lo, acc_hi, rb, vb0, vb1);
+        }
+      }
+    } else if (bprev < nb) {
+      // (3) of the previous bin
+      const uint32_t* r0 = p.q + bprev * nb;
+      pb_scatter(p, s_c, r0, r0 + nb, 0u, 0u, pf, warp - PB2_NA, PB_THREADS / 32 - PB2_NA, false);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) s_bin = (int)atomicAdd(&st->pb_next[t % 3], 1u);
+    if (bcur < nb) {
+      // (2) the PR update of bin bcur: acc -> s_c, acc zeroed for the next bin
+      const int64_t base = bcur * PB_R;
+      const int nrows = (int)min((int64_t)PB_R, a.n_slots - base);
+      for (int i0 = threadIdx.x; i0 < PB_R; i0 += PB_THREADS * 4) {
+        double xo[4];
+        uint32_t Dv[4];
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+          const int i = i0 + u * PB_THREADS;
+          xo[u] = i < nrows ? __ldcs(a.x + base + i) : 0.0;
+          Dv[u] = i < nrows ? __ldcs(a.D + base + i) : 0u;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+          const int i = i0 + u * PB_THREADS;
+          if (i < nrows) {
+            const int64_t v = base + i;
+            const unsigned long long fx = ((unsigned long long)acc_hi[i] << 32) | acc_lo[i];
+            float c = 0.0f;
+            if (!pb_update<SLOTS>(a, v, (double)fx * inv_fix, xo[u], Dv[u], addc, merge_now, sc, my_delta, my_dang,
+                                  my_mass, c))
+              c = __ldcg(a.contrib[0] + v);
+            s_c[i] = c;
+          }
+          if (i < PB_R) {
+            acc_lo[i] = 0u;
+            acc_hi[i] = 0u;
+          }
+        }
+      }
+    }
+    __syncthreads();
+    bprev = bcur;
+    bcur = bcur < nb ? (int64_t)s_bin : nb;
+  }
+  pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
+}
+
 // val[] <- the initial terms contrib_0[u] along every edge: (3) for every
 // source block with s_c = contrib_0 of the block
 __global__ void __launch_bounds__(PB_THREADS, 1) k_pb_init_val(PbArgs p, const float* __restrict__ contrib,
@@ -674,26 +798,34 @@ __global__ void __launch_bounds__(256) k_pr_tpv(PrArgs a) {
   pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
 }
 
-// 64 threads per tile: tiles average a handful of members (S_max 64), so
-// small CTAs let ~24 tiles per SM progress at once (was 8 with 256 threads)
-constexpr int PRL_THREADS = 64;
+// 128 threads (4 warps) per tile.  Round 1 ran one thread per member and
+// rescanned all of the tile's edges for every member in every local
+// iteration (O(members x edges)); a hub member's CSC in-list was also walked by
+// a single thread.  Now: warp-per-member external inflow, and the tile's edges
+// regrouped by sink member in shared memory once per tile (a deterministic
+// counting sort, one warp, __match_any_sync ranks), so a local iteration costs
+// O(edges / threads).
+constexpr int PRL_THREADS = 128;
 
 // §3 shared-memory pass for PR (P@32188-32416; SURVEY A7 "PR store"): after
 // the sweep, each subgraph tile iterates its members t times in shared
 // memory, x_v <- (1-d)/N + d (ext_v + sum_{u in S, u->v} x_u / D_u + dang/N),
-// where ext_v = y_v - sum_{u in S, u->v} contrib_u is the inflow from outside
-// the tile (y_v recovered from the sweep's x_v).  Members that are replicated
-// or not owners keep their sweep values and act as external sources.  The
-// fixed point is unchanged (Theorem E3); delta grows by |x_loc - x_sweep|
-// (an upper bound of the true change), dangling mass by the exact change.
+// where ext_v is the inflow from outside the tile (gathered from the CSC with
+// the current contrib values).  Members that are replicated or not owners
+// keep their sweep values and act as external sources.  The fixed point is
+// unchanged (Theorem E3); delta grows by |x_loc - x_sweep| (an upper bound of
+// the true change), dangling mass by the exact change.
+// Dynamic shared memory: t_max_edges bytes (source member per in-edge).
 template <bool SLOTS>
 __global__ void __launch_bounds__(PRL_THREADS) k_pr_local(PrArgs a, const int32_t* __restrict__ tptr,
                                                   const int32_t* __restrict__ tmem, const int32_t* __restrict__ teptr,
                                                   const uint2* __restrict__ tedges, const int32_t* __restrict__ titers,
                                                   int64_t ntiles) {
-  __shared__ double xs[256], xn[256], ext[256];
+  extern __shared__ uint8_t in_src[];
+  __shared__ double xs[256], xn[256], ext[256], cs[256];
   __shared__ uint32_t Ds[256];
   __shared__ int32_t smem_id[256];
+  __shared__ int in_ptr[257], cur[256];
   __shared__ uint8_t fixed[256];
   __shared__ double s_red[32];
   PrState* st = a.st;
@@ -704,6 +836,8 @@ __global__ void __launch_bounds__(PRL_THREADS) k_pr_local(PrArgs a, const int32_
   const double sc = st->scale;
   const double addc = a.base + a.damp * sc * st->dang[t % 3] * a.invN;
   double my_delta = 0, my_dang = 0, my_mass = 0;
+  const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
+  constexpr unsigned NW = PRL_THREADS / 32;
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int b0 = tptr[tile], nm = tptr[tile + 1] - b0;
     const int e0 = teptr[tile], ne = teptr[tile + 1] - e0;
@@ -714,47 +848,72 @@ __global__ void __launch_bounds__(PRL_THREADS) k_pr_local(PrArgs a, const int32_
       xs[i] = a.x[v];
       Ds[i] = a.D[v];
       smem_id[i] = v;
+      cur[i] = 0;
     }
     __syncthreads();
-    // external inflow of each member, gathered from the CSC with the values
-    // the contrib buffer holds now (sources outside the tile, or members that
-    // keep their values); scaled like the sweep's inputs.  Under the
-    // asynchronous schedule the sweep's own inputs are unknown (old or new), so
-    // recovering it as y_v - (in-tile part) would mix the two and can stall.
-    for (int i = threadIdx.x; i < nm; i += blockDim.x) {
-      if (fixed[i]) {
-        ext[i] = 0.0;
-        continue;
+    // in-degree of every member inside the tile
+    for (int e = threadIdx.x; e < ne; e += blockDim.x) atomicAdd(&cur[(tedges[e0 + e].x >> 8) & 0xff], 1);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      int acc = 0;
+      for (int i = 0; i < nm; i++) {
+        in_ptr[i] = acc;
+        acc += cur[i];
+        cur[i] = in_ptr[i];
       }
-      const int32_t v = smem_id[i];
+      in_ptr[nm] = acc;
+    }
+    __syncthreads();
+    // edges regrouped by sink member, in tile-edge order within a sink (one
+    // warp, 32 edges per step; lanes with the same sink ranked by match_any)
+    if (warp == 0) {
+      for (int c0 = 0; c0 < ne; c0 += 32) {
+        const int e = c0 + (int)lane;
+        const bool ok = e < ne;
+        const uint32_t px = ok ? tedges[e0 + e].x : 0u;
+        const int d = ok ? (int)((px >> 8) & 0xff) : 256 + (int)lane;
+        const unsigned same = __match_any_sync(FULL, d);
+        const int rank = __popc(same & lanemask_lt());
+        if (ok) in_src[cur[d] + rank] = (uint8_t)(px & 0xff);
+        __syncwarp();
+        if (ok && rank == 0) cur[d] += __popc(same);
+        __syncwarp();
+      }
+    }
+    // external inflow, warp per member, from the CSC with the values the
+    // contrib buffer holds now (sources outside the tile, or members that keep
+    // their values); scaled like the sweep's inputs
+    for (int i = warp; i < nm; i += NW) {
       double in = 0.0;
-      for (uint32_t e = a.crp[v]; e < a.crp[v + 1]; e++) {
-        const int32_t u = a.csrc[e];
-        int lo = 0, hi = nm;   // members are sorted slot ids
-        while (lo < hi) {
-          const int mid = (lo + hi) >> 1;
-          if (smem_id[mid] < u) lo = mid + 1;
-          else hi = mid;
+      if (!fixed[i]) {
+        const int32_t v = smem_id[i];
+        for (uint32_t e = a.crp[v] + lane; e < a.crp[v + 1]; e += 32) {
+          const int32_t u = a.csrc[e];
+          int lo = 0, hi = nm;   // members are sorted slot ids
+          while (lo < hi) {
+            const int mid = (lo + hi) >> 1;
+            if (smem_id[mid] < u) lo = mid + 1;
+            else hi = mid;
+          }
+          const bool inside = lo < nm && smem_id[lo] == u && !fixed[lo];
+          if (!inside) in += (double)cin[u];
         }
-        const bool inside = lo < nm && smem_id[lo] == u && !fixed[lo];
-        if (!inside) in += (double)cin[u];
       }
-      ext[i] = sc * in;
+      in = warp_sum_f64(in);
+      if (lane == 0) ext[i] = sc * in;
     }
     __syncthreads();
     const int iters = titers[tile];
     for (int r = 0; r < iters; r++) {
+      for (int i = threadIdx.x; i < nm; i += blockDim.x) cs[i] = (!fixed[i] && Ds[i]) ? xs[i] / (double)Ds[i] : 0.0;
+      __syncthreads();
       for (int i = threadIdx.x; i < nm; i += blockDim.x) {
         if (fixed[i]) {
           xn[i] = xs[i];
           continue;
         }
         double in = ext[i];
-        for (int e = 0; e < ne; e++) {
-          const uint2 p = tedges[e0 + e];
-          const int s = p.x & 0xff, d = (p.x >> 8) & 0xff;
-          if (d == i && !fixed[s] && Ds[s]) in += xs[s] / (double)Ds[s];
-        }
+        for (int k = in_ptr[i]; k < in_ptr[i + 1]; k++) in += cs[in_src[k]];
         xn[i] = addc + a.damp * in;
       }
       __syncthreads();
@@ -1026,11 +1185,22 @@ static void run_pagerank_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& in
 void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   Ctx* c = g->ctx;
   cudaStream_t s = c->stream;
-  ensure_csc(g);
   DevGraph& d = g->dg;
   RunState& r = g->rs;
   GX_CHECK_ARG(g->n > 0, "empty graph");
   int64_t ns = d.n_slots;
+  // sweep mapping (one GPU); the blocked pull needs no CSC unless the §3 local
+  // pass runs (it gathers the tiles' external inflow from the CSC)
+  const int P_ranks = (c->world == 1 && o.sim_ranks > 1) ? o.sim_ranks : c->world;
+  const bool async_ = o.pr_schedule == GX_PR_ASYNC && P_ranks == 1;
+  const bool tiles = d.n_tiles && g->knobs.smem;
+  int mapping = o.mapping;
+  if (mapping == GX_MAP_AUTO) {
+    const bool pb_ok = async_ && !tiles && (ns + PB_R - 1) / PB_R >= GX_PB_MIN_BLOCKS && !getenv("GX_NO_PB");
+    mapping = pb_ok ? GX_MAP_PB
+                    : (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
+  }
+  if (P_ranks > 1 || mapping != GX_MAP_PB || tiles) ensure_csc(g);
   r.x.alloc(c, sizeof(double) * ns);
   r.contrib[0].alloc(c, sizeof(float) * ns);
   const bool sim_ = c->world == 1 && o.sim_ranks > 1;
@@ -1073,18 +1243,11 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     const int P = sim ? o.sim_ranks : c->world;
     if (P > 1) {
       GX_CHECK_ARG(P <= 8, "at most 8 ranks");
-      GX_CHECK_ARG(o.mapping != GX_MAP_TPV, "the partitioned path uses the LB mapping");
+      GX_CHECK_ARG(o.mapping != GX_MAP_TPV && o.mapping != GX_MAP_PB, "the partitioned path uses the LB mapping");
       GX_CHECK_ARG(o.merge_every == 1 || !d.n_groups, "the partitioned path merges after every iteration");
       run_pagerank_dist(g, o, info, a, P, sim);
       return;
     }
-  }
-  int mapping = o.mapping;
-  const bool tiles = d.n_tiles && g->knobs.smem;
-  if (mapping == GX_MAP_AUTO) {
-    const bool pb_ok = async && !tiles && (ns + PB_R - 1) / PB_R >= GX_PB_MIN_BLOCKS && !getenv("GX_NO_PB");
-    mapping = pb_ok ? GX_MAP_PB
-                    : (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
   }
   GX_CHECK_ARG(mapping != GX_MAP_PB || async, "the blocked mapping runs the asynchronous schedule");
   PbArgs pb{};
@@ -1100,6 +1263,8 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
       CUDA_OK(cudaFuncSetAttribute(k_pr_pb<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
       CUDA_OK(cudaFuncSetAttribute(k_pr_pb<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
       CUDA_OK(cudaFuncSetAttribute(k_pb_init_val, cudaFuncAttributeMaxDynamicSharedMemorySize, (PB_R + 8) * 4));
+      CUDA_OK(cudaFuncSetAttribute(k_pr_pb2<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB2_SMEM));
+      CUDA_OK(cudaFuncSetAttribute(k_pr_pb2<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB2_SMEM));
       attr = true;
     }
   }
@@ -1123,6 +1288,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   if (mapping == GX_MAP_PB) k_pb_init_val<<<(int)std::min<int64_t>(pb.nb, c->num_sms * 2), PB_THREADS, (PB_R + 8) * 4, s>>>(pb, a.contrib[0], ns);
   CUDA_OK(cudaGetLastError());
   int launches = mapping == GX_MAP_PB ? 2 : 1;
+  const bool pb_v2 = getenv("GX_PB_KERNEL") && atoi(getenv("GX_PB_KERNEL")) == 2;
   const int grid_pb = (int)std::max<int64_t>(1, std::min<int64_t>(pb.nb, (int64_t)c->num_sms * PB_CTAS_PER_SM));
 
   // GX_PR_KERNEL=1 selects the round-1 kernel (A/B experiments)
@@ -1140,7 +1306,10 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   KTimer kt(o.profile != 0, s);
   auto one_iter = [&](int& nl) {
     kt.begin();
-    if (mapping == GX_MAP_PB) {
+    if (mapping == GX_MAP_PB && pb_v2) {
+      if (slots) k_pr_pb2<true><<<grid_pb, PB_THREADS, PB2_SMEM, s>>>(a, pb);
+      else k_pr_pb2<false><<<grid_pb, PB_THREADS, PB2_SMEM, s>>>(a, pb);
+    } else if (mapping == GX_MAP_PB) {
       if (slots) k_pr_pb<true><<<grid_pb, PB_THREADS, PB_SMEM, s>>>(a, pb);
       else k_pr_pb<false><<<grid_pb, PB_THREADS, PB_SMEM, s>>>(a, pb);
     } else if (mapping == GX_MAP_TPV) {
@@ -1171,13 +1340,14 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     kt.end();
     nl++;
     if (tiles) {
-      const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 24));
+      const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 16));
+      const size_t prl_smem = (size_t)std::max<int64_t>(d.t_max_edges, 16);
       if (slots)
-        k_pr_local<true><<<grid_local, PRL_THREADS, 0, s>>>(a, d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(),
+        k_pr_local<true><<<grid_local, PRL_THREADS, prl_smem, s>>>(a, d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(),
                                                     d.t_eptr.as<int32_t>(), d.t_edges.as<uint2>(), d.t_iters.as<int32_t>(),
                                                     d.n_tiles);
       else
-        k_pr_local<false><<<grid_local, PRL_THREADS, 0, s>>>(a, d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(),
+        k_pr_local<false><<<grid_local, PRL_THREADS, prl_smem, s>>>(a, d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(),
                                                      d.t_eptr.as<int32_t>(), d.t_edges.as<uint2>(),
                                                      d.t_iters.as<int32_t>(), d.n_tiles);
       nl++;
