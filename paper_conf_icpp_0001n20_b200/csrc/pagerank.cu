@@ -358,7 +358,10 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell2(PrArgs a) {
 // read + 4 written in (3), all streaming -- 12 B against the 8 B of the
 // gather pull, at HBM rate instead of the L1TEX random-sector rate.
 // One CTA per SM (measured: two CTAs of half the rows, PB_R = 8192, are 18 %
-// slower -- twice the segments, each half as long)
+// slower -- twice the segments, each half as long; a warp-specialised CTA
+// running one bin's (1) beside the previous bin's (3) on separate warps was
+// 5 % slower per sweep and needed 17 sweeps instead of 15, the scatter lagging
+// one bin behind -- profiles/README.md "third session")
 constexpr int PB_THREADS = 1024;
 constexpr int PB_CTAS_PER_SM = 1;
 constexpr int PB_CH = 4 * PB_THREADS;   // (1): elements per bulk-copied chunk (4 per thread)
@@ -604,131 +607,6 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
     // (3) scatter the new terms along block b's segments
     pb_scatter(p, s_c, r0, r1, lo0, hi0, pf);
     __syncthreads();   // s_c (= acc_lo) is zeroed for the next bin
-  }
-  pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
-}
-
-// Warp-specialised variant (GX_PB_KERNEL=2): the CTA's warps are split into
-// group A (PB2_NA warps: phase (1) of bin b_k, plain 16-byte loads, 16 terms
-// per thread in flight) and group B (the rest: phase (3) of bin b_{k-1}) that
-// run at the same time on separate shared-memory arrays (acc vs s_c), so one
-// bin's stream and the previous bin's scatter overlap on every SM; then all
-// warps run (2) for b_k, which zeroes acc as it reads it and fills s_c.
-#ifndef GX_PB2_NA
-#define GX_PB2_NA 20
-#endif
-constexpr int PB2_NA = GX_PB2_NA;
-constexpr size_t PB2_SMEM = (size_t)PB_R * 8 + 32 + (size_t)(PB_R + 8) * 4;
-
-__device__ __forceinline__ void pb_add8(uint32_t* lo, uint32_t* hi, uint4 r, float4 v0, float4 v1) {
-  pb_add4(lo, hi, make_uint2(r.x, r.y), v0);
-  pb_add4(lo, hi, make_uint2(r.z, r.w), v1);
-}
-
-template <bool SLOTS>
-__global__ void __launch_bounds__(PB_THREADS, 1) k_pr_pb2(PrArgs a, PbArgs p) {
-  extern __shared__ __align__(16) unsigned char pb_smem[];
-  uint32_t* acc_lo = reinterpret_cast<uint32_t*>(pb_smem);
-  uint32_t* acc_hi = acc_lo + PB_R + 8;
-  float* s_c = reinterpret_cast<float*>(acc_hi + PB_R);   // PB_R + 8 terms (last 8 = 0)
-  __shared__ double s_red[32];
-  __shared__ int s_bin;
-  PrState* st = a.st;
-  if (st->stop) return;
-  const unsigned t = st->iter;
-  const double sc = st->scale;
-  const double addc = a.base + a.damp * sc * st->dang[t % 3] * a.invN;
-  const bool merge_now = st->do_merge != 0;
-  double my_delta = 0, my_dang = 0, my_mass = 0;
-  const uint64_t pf = l2_evict_first();
-  const unsigned warp = threadIdx.x >> 5;
-  const bool grpA = warp < (unsigned)PB2_NA;
-  const int64_t nb = p.nb;
-  const uint32_t* qend = p.q + nb * nb;
-  const double inv_fix = 1.0 / 72057594037927936.0;   // 2^-56
-  if (threadIdx.x < 8) s_c[PB_R + threadIdx.x] = 0.0f;
-  for (int i = threadIdx.x; i < PB_R / 4; i += PB_THREADS) {
-    reinterpret_cast<uint4*>(acc_lo)[i] = make_uint4(0, 0, 0, 0);
-    reinterpret_cast<uint4*>(acc_hi)[i] = make_uint4(0, 0, 0, 0);
-  }
-  if (threadIdx.x == 0) s_bin = (int)atomicAdd(&st->pb_next[t % 3], 1u);
-  __syncthreads();
-  int64_t bcur = s_bin, bprev = nb;
-  while (bcur < nb || bprev < nb) {
-    if (grpA) {
-      if (bcur < nb) {
-        const int64_t base = bcur * PB_R;
-        const int nrows = (int)min((int64_t)PB_R, a.n_slots - base);
-        const unsigned ta = threadIdx.x;
-        if (ta == 0) {
-          l2_prefetch_bulk(a.x + base, (uint32_t)nrows * 8u);
-          l2_prefetch_bulk(a.D + base, (uint32_t)nrows * 4u);
-        }
-        const uint32_t* r0 = p.q + bcur * nb;
-        for (int64_t j = ta; j < nb; j += PB2_NA * 32) {   // next slot's scatter segments
-          const uint32_t lo = __ldg(r0 + j), hi = __ldg(r0 + nb + j);
-          if (hi > lo) l2_prefetch_bulk(p.src_loc + lo, (hi - lo) * 2u);
-        }
-        // (1) the bin's contiguous in-edge range
-        const uint32_t E0 = __ldg(p.q + bcur), E1 = __ldg(qend + bcur);
-        constexpr uint32_t STEP = 8u * PB2_NA * 32;
-        for (uint32_t e = E0 + 8u * ta; e < E1; e += 2 * STEP) {
-          const bool two = e + STEP < E1;
-          const uint4 ra = ld_stream_v4(reinterpret_cast<const uint32_t*>(p.dst_loc + e), pf);
-          const float4 va0 = ld_cg_f4(p.val + e), va1 = ld_cg_f4(p.val + e + 4);
-          uint4 rb = make_uint4(0, 0, 0, 0);
-          float4 vb0 = make_float4(0, 0, 0, 0), vb1 = vb0;
-          if (two) {
-            rb = ld_stream_v4(reinterpret_cast<const uint32_t*>(p.dst_loc + e + STEP), pf);
-            vb0 = ld_cg_f4(p.val + e + STEP);
-            vb1 = ld_cg_f4(p.val + e + STEP + 4);
-          }
-          pb_add8(acc_lo, acc_hi, ra, va0, va1);
-          pb_add8(acc_lo, acc_hi, rb, vb0, vb1);
-        }
-      }
-    } else if (bprev < nb) {
-      // (3) of the previous bin
-      const uint32_t* r0 = p.q + bprev * nb;
-      pb_scatter(p, s_c, r0, r0 + nb, 0u, 0u, pf, warp - PB2_NA, PB_THREADS / 32 - PB2_NA, false);
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) s_bin = (int)atomicAdd(&st->pb_next[t % 3], 1u);
-    if (bcur < nb) {
-      // (2) the PR update of bin bcur: acc -> s_c, acc zeroed for the next bin
-      const int64_t base = bcur * PB_R;
-      const int nrows = (int)min((int64_t)PB_R, a.n_slots - base);
-      for (int i0 = threadIdx.x; i0 < PB_R; i0 += PB_THREADS * 4) {
-        double xo[4];
-        uint32_t Dv[4];
-#pragma unroll
-        for (int u = 0; u < 4; u++) {
-          const int i = i0 + u * PB_THREADS;
-          xo[u] = i < nrows ? __ldcs(a.x + base + i) : 0.0;
-          Dv[u] = i < nrows ? __ldcs(a.D + base + i) : 0u;
-        }
-#pragma unroll
-        for (int u = 0; u < 4; u++) {
-          const int i = i0 + u * PB_THREADS;
-          if (i < nrows) {
-            const int64_t v = base + i;
-            const unsigned long long fx = ((unsigned long long)acc_hi[i] << 32) | acc_lo[i];
-            float c = 0.0f;
-            if (!pb_update<SLOTS>(a, v, (double)fx * inv_fix, xo[u], Dv[u], addc, merge_now, sc, my_delta, my_dang,
-                                  my_mass, c))
-              c = __ldcg(a.contrib[0] + v);
-            s_c[i] = c;
-          }
-          if (i < PB_R) {
-            acc_lo[i] = 0u;
-            acc_hi[i] = 0u;
-          }
-        }
-      }
-    }
-    __syncthreads();
-    bprev = bcur;
-    bcur = bcur < nb ? (int64_t)s_bin : nb;
   }
   pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
 }
@@ -1263,8 +1141,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
       CUDA_OK(cudaFuncSetAttribute(k_pr_pb<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
       CUDA_OK(cudaFuncSetAttribute(k_pr_pb<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
       CUDA_OK(cudaFuncSetAttribute(k_pb_init_val, cudaFuncAttributeMaxDynamicSharedMemorySize, (PB_R + 8) * 4));
-      CUDA_OK(cudaFuncSetAttribute(k_pr_pb2<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB2_SMEM));
-      CUDA_OK(cudaFuncSetAttribute(k_pr_pb2<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB2_SMEM));
+
       attr = true;
     }
   }
@@ -1288,7 +1165,6 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   if (mapping == GX_MAP_PB) k_pb_init_val<<<(int)std::min<int64_t>(pb.nb, c->num_sms * 2), PB_THREADS, (PB_R + 8) * 4, s>>>(pb, a.contrib[0], ns);
   CUDA_OK(cudaGetLastError());
   int launches = mapping == GX_MAP_PB ? 2 : 1;
-  const bool pb_v2 = getenv("GX_PB_KERNEL") && atoi(getenv("GX_PB_KERNEL")) == 2;
   const int grid_pb = (int)std::max<int64_t>(1, std::min<int64_t>(pb.nb, (int64_t)c->num_sms * PB_CTAS_PER_SM));
 
   // GX_PR_KERNEL=1 selects the round-1 kernel (A/B experiments)
@@ -1306,10 +1182,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   KTimer kt(o.profile != 0, s);
   auto one_iter = [&](int& nl) {
     kt.begin();
-    if (mapping == GX_MAP_PB && pb_v2) {
-      if (slots) k_pr_pb2<true><<<grid_pb, PB_THREADS, PB2_SMEM, s>>>(a, pb);
-      else k_pr_pb2<false><<<grid_pb, PB_THREADS, PB2_SMEM, s>>>(a, pb);
-    } else if (mapping == GX_MAP_PB) {
+    if (mapping == GX_MAP_PB) {
       if (slots) k_pr_pb<true><<<grid_pb, PB_THREADS, PB_SMEM, s>>>(a, pb);
       else k_pr_pb<false><<<grid_pb, PB_THREADS, PB_SMEM, s>>>(a, pb);
     } else if (mapping == GX_MAP_TPV) {
