@@ -345,7 +345,7 @@ gx_status gx_transform(gx_graph* g, const gx_knobs* knobs, gx_transform_info* in
   } else {
     ensure_host(g);
     SlotGraph sg;
-    transform_host(g->host, k, sg);
+    transform_host(g->host, k, sg, getenv("GX_TRANSFORM_HOST") ? nullptr : g->ctx);
     g->sg = std::move(sg);
     g->transformed = true;
     g->knobs = k;

@@ -137,12 +137,17 @@ void bfs_forest(const HostCSR& g, std::vector<int32_t>& sources, std::vector<int
 
 // RenumberVertex (Alg 2 l.10-20), cursor reading R6-R8, pad R9.
 void renumber(const HostCSR& g, int k, std::vector<int32_t>& nw, int64_t& n_slots,
-              std::vector<std::pair<int64_t, int64_t>>& ranges) {
+              std::vector<std::pair<int64_t, int64_t>>& ranges, Ctx* dev) {
   const int64_t n = g.n;
   std::vector<int32_t> sources, level;
   PhaseTimer pt;
-  bfs_forest(g, sources, level);
-  pt("bfs_forest+levels");
+  if (dev) {
+    gpu_bfs_forest(dev, n, g.rp.data(), g.col.data(), sources, level);   // N1 (gtransform.cu)
+    pt("bfs_forest+levels (GPU)");
+  } else {
+    bfs_forest(g, sources, level);
+    pt("bfs_forest+levels");
+  }
   nw.assign(n, -1);
   for (size_t i = 0; i < sources.size(); i++) nw[sources[i]] = (int32_t)i;
   int64_t gid = (int64_t)sources.size();
@@ -195,12 +200,12 @@ void renumber(const HostCSR& g, int k, std::vector<int32_t>& nw, int64_t& n_slot
 }
 
 // Renumber + ReplicateVertex (Alg 2 l.21-35), readings R10-R18.
-void coalesce(const HostCSR& g, int k, int64_t theta_ppm, int wrule, Work& W) {
+void coalesce(const HostCSR& g, int k, int64_t theta_ppm, int wrule, Work& W, Ctx* dev) {
   const int64_t n = g.n;
   std::vector<int32_t> nw;
   std::vector<std::pair<int64_t, int64_t>> ranges;
   int64_t n_slots = 0;
-  renumber(g, k, nw, n_slots, ranges);
+  renumber(g, k, nw, n_slots, ranges, dev);
   PhaseTimer pt;
   W.n = n;
   W.n_slots = n_slots;
@@ -420,7 +425,7 @@ void logical_out(const Work& W, std::vector<std::vector<std::pair<int32_t, uint3
   for (int64_t u = 0; u < n; u++) std::sort(out[u].begin(), out[u].end());
 }
 
-void build_logical(const Work& W, Logical& L) {
+void build_logical(const Work& W, Logical& L, Ctx* dev) {
   PhaseTimer pt;
   const int64_t n = W.n;
   L.n = n;
@@ -448,6 +453,19 @@ void build_logical(const Work& W, Logical& L) {
     v.erase(std::unique(v.begin(), v.end()), v.end());
   }
   pt("undirected N");
+  if (dev) {
+    // N1: the forward-algorithm triangle count on the graph's device
+    std::vector<int64_t> np(n + 1, 0);
+    for (int64_t u = 0; u < n; u++) np[u + 1] = np[u] + (int64_t)L.N[u].size();
+    std::vector<int32_t> nc(std::max<int64_t>(np[n], 1));
+#pragma omp parallel for schedule(dynamic, 4096)
+    for (int64_t u = 0; u < n; u++) std::copy(L.N[u].begin(), L.N[u].end(), nc.begin() + np[u]);
+    pt("flatten U");
+    L.T.assign(n, 0);
+    gpu_triangles(dev, n, np.data(), nc.data(), L.T.data());
+    pt("triangles (GPU)");
+    return;
+  }
   // triangles: forward algorithm over the degree-ordered orientation
   L.T.assign(n, 0);
   std::vector<std::vector<int32_t>> fwd(n);
@@ -695,7 +713,7 @@ void degnorm(Work& W, int64_t th, int64_t f, bool combined, int wrule, std::vect
 
 }  // namespace
 
-void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out) {
+void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out, Ctx* dev) {
   auto t0 = std::chrono::steady_clock::now();
   // GX_TRANSFORM_TRACE=1: per-phase host times on stderr
   const bool trace = getenv("GX_TRANSFORM_TRACE") != nullptr;
@@ -707,13 +725,13 @@ void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out) {
     tp = now;
   };
   Work W;
-  if (k.coalesce) coalesce(g, k.chunk_k, ppm(k.replicate_threshold), k.added_weight_rule, W);
+  if (k.coalesce) coalesce(g, k.chunk_k, ppm(k.replicate_threshold), k.added_weight_rule, W, dev);
   else identity(g, W);
   phase(k.coalesce ? "coalesce" : "identity");
   SmemOut sm;
   if (k.smem) {
     Logical L;
-    build_logical(W, L);
+    build_logical(W, L, dev);
     phase("logical+tri");
     const int64_t th = ppm(k.cc_threshold);
     const int64_t budget = k.added_edge_budget >= 0 ? k.added_edge_budget : g.m / 100;

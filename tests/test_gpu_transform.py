@@ -1,0 +1,89 @@
+"""GPU-resident preprocessing: with a device context the
+§3 triangle counts (the clustering coefficients of P@29857 that drive the CC
+edge insertion and the subgraph selection) and the §2 source order,
+reachability forest and multi-source BFS levels (Alg 2 l.2-6) are computed on
+the GPU (gtransform.cu).  The exported transformed graph must be bit-identical to
+the oracle's and to the host-only library path (no device), element by
+element -- the triangle counts feed integer decisions only."""
+import numpy as np
+import pytest
+
+import graphgen
+from golden_io import load
+from gpu_util import ctx, upload
+from oracle import transform as T
+from test_transform_parity import assert_same, oracle_export
+
+pytestmark = pytest.mark.gpu
+
+GRAPHS = {
+    "rmat12": lambda: graphgen.rmat(12),
+    "road48": lambda: graphgen.road(48),
+    "uniform": lambda: graphgen.uniform(3000, 30000),
+    "fig1_4": lambda: load("fig1_4.txt")[0],
+    "clique_hub": lambda: graphgen.from_edge_list(
+        300, [(a, b, 1 + (a * b) % 5) for a in range(40) for b in range(40) if a != b]
+        + [(0, v, 2) for v in range(40, 300)] + [(v, (v * 13) % 300, 3) for v in range(40, 300)]),
+}
+KNOBS = {
+    "smem": T.Knobs(smem=True, cc_threshold=0.3, added_edge_budget=200),
+    "smem_und": T.Knobs(smem=True, cc_threshold=0.3, added_edge_budget=300, sibling_undirected=True),
+    "all": T.Knobs(coalesce=True, chunk_k=8, replicate_threshold=0.3, smem=True, cc_threshold=0.3,
+                   degree_norm=True, degsim_threshold=0.5),
+}
+
+
+def _knobs(gx, kn):
+    return gx.Knobs(**{f: getattr(kn, f) for f in kn.__dataclass_fields__})
+
+
+@pytest.mark.parametrize("gname", list(GRAPHS))
+@pytest.mark.parametrize("kname", list(KNOBS))
+def test_device_transform_matches_oracle(gname, kname):
+    import paper_conf_icpp_0001n20_b200 as gx
+    raw = GRAPHS[gname]()
+    kn = KNOBS[kname]
+    G = upload(raw)
+    info = G.transform(_knobs(gx, kn))
+    assert_same(G.export(), oracle_export(raw, kn), info)
+
+
+@pytest.mark.parametrize("scale", [16, 18])
+@pytest.mark.parametrize("kname", ["smem", "coalesce_smem"])
+def test_device_transform_matches_host_library(scale, kname):
+    """Larger RMAT (many triangles, hub rows): device path vs the host-only
+    library path, whose transforms are pinned to the oracle on CPU."""
+    import paper_conf_icpp_0001n20_b200 as gx
+    ctx()
+    raw = graphgen.rmat(scale)
+    kn = {"smem": T.Knobs(smem=True, cc_threshold=0.5),
+          "coalesce_smem": T.Knobs(coalesce=True, chunk_k=16, replicate_threshold=0.4, smem=True,
+                                   cc_threshold=0.5)}[kname]
+    G = upload(raw)
+    info = G.transform(_knobs(gx, kn))
+    H = gx.Graph.host_only(raw.row_ptr, raw.col, raw.w)
+    hinfo = H.transform(_knobs(gx, kn))
+    a, b = G.export(), H.export()
+    for k in ("row_ptr", "col", "w", "edge_added", "slot_to_orig", "slot_kind", "sched", "tile_ptr",
+              "tile_members", "tile_centre", "tile_iters"):
+        assert np.array_equal(np.asarray(a[k]), np.asarray(b[k])), k
+    for k in ("n_slots", "n_replicas", "n_holes", "edges_added_coalesce", "edges_added_smem", "n_subgraphs",
+              "subgraph_vertices"):
+        assert info[k] == hinfo[k], k
+    assert info["n_subgraphs"] > 0
+
+
+def test_device_levels_road_grid():
+    """High-diameter graph (hundreds of BFS levels): the coalescing
+    renumbering from device levels equals the host-only library's."""
+    import paper_conf_icpp_0001n20_b200 as gx
+    ctx()
+    raw = graphgen.road(200)
+    kn = T.Knobs(coalesce=True, chunk_k=16, replicate_threshold=0.4)
+    G = upload(raw)
+    G.transform(_knobs(gx, kn))
+    H = gx.Graph.host_only(raw.row_ptr, raw.col, raw.w)
+    H.transform(_knobs(gx, kn))
+    a, b = G.export(), H.export()
+    for k in ("row_ptr", "col", "slot_to_orig", "slot_kind"):
+        assert np.array_equal(np.asarray(a[k]), np.asarray(b[k])), k
