@@ -367,6 +367,10 @@ constexpr int PB_CTAS_PER_SM = 1;
 constexpr int PB_CH = 4 * PB_THREADS;   // (1): elements per bulk-copied chunk (4 per thread)
 constexpr int PB_NST = 4;          // (1): ring stages (3 chunks in flight while one is consumed)
 constexpr size_t PB_STAGE = (size_t)PB_CH * 6;
+#ifndef GX_PB_SEGU
+#define GX_PB_SEGU 2    // measured: 1: 824, 2: 818, 4: 863, 8: 942 us per sweep (RMAT-24)
+#endif
+constexpr int PB_SEGU = GX_PB_SEGU;   // (3): segments in flight per warp step (16-byte load each per lane)
 // dynamic smem: acc_lo u32[R] (reused as the f32 terms s_c after the update)
 // | 8 zero words (s_c[R..R+7], the padding entries' source) | acc_hi u32[R] | ring
 constexpr size_t PB_RING_OFF = (size_t)PB_R * 8 + 32;
@@ -445,7 +449,9 @@ __device__ __forceinline__ bool pb_update(const PrArgs& a, int64_t v, double y, 
   my_delta += fabs(xn - sc * xo);
   my_mass += xn;
   c = Dv ? (float)(xn / (double)Dv) : 0.0f;
-  __stcg(a.contrib[0] + v, c);
+  // the stored contrib is read by the merge / local pass / merge carry only
+  // (slot graphs); in exact mode the terms live in val[] alone
+  if (SLOTS) __stcg(a.contrib[0] + v, c);
   if (!Dv) my_dang += xn;
   return true;
 }
@@ -465,17 +471,17 @@ __device__ __forceinline__ void pb_scatter(const PbArgs& p, const float* s_c, co
     const uint32_t lo = first ? lo0 : j < nb ? __ldg(r0 + j) : 0u;
     const uint32_t hi = first ? hi0 : j < nb ? __ldg(r1 + j) : 0u;
     const int kn = (int)min((int64_t)32, nb - j0);
-    for (int k = 0; k < kn; k += 4) {
-      uint32_t ee[4], hh[4];
-      uint4 w[4];
+    for (int k = 0; k < kn; k += PB_SEGU) {
+      uint32_t ee[PB_SEGU], hh[PB_SEGU];
+      uint4 w[PB_SEGU];
 #pragma unroll
-      for (int u = 0; u < 4; u++) {
+      for (int u = 0; u < PB_SEGU; u++) {
         ee[u] = __shfl_sync(FULL, lo, k + u) + 8u * lane;
         hh[u] = __shfl_sync(FULL, hi, k + u);
         if (ee[u] < hh[u]) w[u] = ld_stream_v4(reinterpret_cast<const uint32_t*>(p.src_loc + ee[u]), pf);
       }
 #pragma unroll
-      for (int u = 0; u < 4; u++) {
+      for (int u = 0; u < PB_SEGU; u++) {
         if (ee[u] < hh[u]) pb_put8(p.val + ee[u], s_c, w[u]);
         for (uint32_t e = ee[u] + 256u; e < hh[u]; e += 256u)
           pb_put8(p.val + e, s_c, ld_stream_v4(reinterpret_cast<const uint32_t*>(p.src_loc + e), pf));
