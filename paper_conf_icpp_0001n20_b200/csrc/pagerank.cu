@@ -365,8 +365,15 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell2(PrArgs a) {
 constexpr int PB_THREADS = 1024;
 constexpr int PB_CTAS_PER_SM = 1;
 constexpr int PB_CH = 4 * PB_THREADS;   // (1): elements per bulk-copied chunk (4 per thread)
-constexpr int PB_NST = 4;          // (1): ring stages (3 chunks in flight while one is consumed)
+#ifndef GX_PB_NST
+#define GX_PB_NST 4
+#endif
+constexpr int PB_NST = GX_PB_NST;  // (1): ring stages (NST - 1 chunks in flight while one is consumed)
 constexpr size_t PB_STAGE = (size_t)PB_CH * 6;
+#ifndef GX_PB_CPT
+#define GX_PB_CPT 1
+#endif
+constexpr int PB_CPT = GX_PB_CPT;     // (1): ring chunks consumed per turn (4 terms each per thread)
 #ifndef GX_PB_SEGU
 #define GX_PB_SEGU 2    // measured: 1: 824, 2: 818, 4: 863, 8: 942 us per sweep (RMAT-24)
 #endif
@@ -568,20 +575,38 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
       }
       if (hi > lo) l2_prefetch_bulk(p.src_loc + lo, (hi - lo) * 2u);
     }
-    for (uint32_t c = 0; c < nch; c++) {
-      const uint32_t gc = g + c, stg = gc % PB_NST;
-      const uint32_t n = min((uint32_t)PB_CH, E1 - (E0 + c * PB_CH));
-      mbar_wait(&full[stg], (gc / PB_NST) & 1);
-      const unsigned char* src = ring + stg * PB_STAGE;
+    for (uint32_t c = 0; c < nch; c += PB_CPT) {
+      float4 tv[PB_CPT];
+      uint2 rv[PB_CPT];
+      bool ok[PB_CPT];
       const uint32_t i = 4u * threadIdx.x;
-      if (i < n) {
-        const float4 tv = *reinterpret_cast<const float4*>(src + 4 * i);
-        const uint2 rv = *reinterpret_cast<const uint2*>(src + PB_CH * 4 + 2 * i);
-        pb_add4(acc_lo, acc_hi, rv, tv);
+#pragma unroll
+      for (int q = 0; q < PB_CPT; q++) {
+        const uint32_t cc = c + q, gc = g + cc, stg = gc % PB_NST;
+        ok[q] = false;
+        if (cc < nch) {
+          const uint32_t n = min((uint32_t)PB_CH, E1 - (E0 + cc * PB_CH));
+          mbar_wait(&full[stg], (gc / PB_NST) & 1);
+          const unsigned char* src = ring + stg * PB_STAGE;
+          ok[q] = i < n;
+          if (ok[q]) {
+            tv[q] = *reinterpret_cast<const float4*>(src + 4 * i);
+            rv[q] = *reinterpret_cast<const uint2*>(src + PB_CH * 4 + 2 * i);
+          }
+        }
       }
+#pragma unroll
+      for (int q = 0; q < PB_CPT; q++)
+        if (ok[q]) pb_add4(acc_lo, acc_hi, rv[q], tv[q]);
       __syncwarp();
-      if (lane == 0) mbar_arrive(&empty[stg]);
-      if (threadIdx.x == 0 && c + PB_NST < nch) issue(gc + PB_NST, E0, E1, c + PB_NST);
+#pragma unroll
+      for (int q = 0; q < PB_CPT; q++) {
+        const uint32_t cc = c + q, gc = g + cc;
+        if (cc < nch) {
+          if (lane == 0) mbar_arrive(&empty[gc % PB_NST]);
+          if (threadIdx.x == 0 && cc + PB_NST < nch) issue(gc + PB_NST, E0, E1, cc + PB_NST);
+        }
+      }
     }
     g += nch;
     __syncthreads();
