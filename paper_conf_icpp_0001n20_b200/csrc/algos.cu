@@ -228,22 +228,37 @@ void run_scc(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
 }
 
 // ---------------------------------------------------------------- MST
-__global__ void k_mst_best(LG L, const uint32_t* __restrict__ comp, unsigned long long* __restrict__ best,
-                           int* __restrict__ any) {
+// min (weight, edge) key of every component over the active edges (all edges
+// in round 1, then the compacted cross-component list): the current best is
+// read first, so the atomic is skipped for the (late-round: nearly all) keys
+// that cannot win -- Boruvka's later rounds hit a handful of components and
+// unconditional atomics on them serialise at L2
+__global__ void k_mst_best(LG L, const uint32_t* __restrict__ act, int64_t na, const uint32_t* __restrict__ comp,
+                           unsigned long long* __restrict__ best, int* __restrict__ any) {
   int a = 0;
-  GRID_STRIDE(e, L.m) {
+  GRID_STRIDE(i, na) {
+    const uint32_t e = act ? act[i] : (uint32_t)i;
     const uint32_t u = L.esrc[e];
     const uint2 ed = L.adj[e];
     const uint32_t cu = comp[u], cv = comp[ed.x];
     if (cu != cv) {
       const unsigned long long key = ((unsigned long long)ed.y << 32) | (unsigned long long)e;
-      atomicMin(best + cu, key);
-      atomicMin(best + cv, key);
+      if (key < __ldcg(best + cu)) atomicMin(best + cu, key);
+      if (key < __ldcg(best + cv)) atomicMin(best + cv, key);
       a = 1;
     }
   }
   if (__syncthreads_or(a) && threadIdx.x == 0) *any = 1;
 }
+// the edges still joining two components after the round's merges
+struct MstCross {
+  const uint32_t* esrc;
+  const uint2* adj;
+  const uint32_t* comp;
+  __device__ __forceinline__ bool operator()(const uint32_t& e) const {
+    return comp[esrc[e]] != comp[adj[e].x];
+  }
+};
 __global__ void k_mst_hook(LG L, const uint32_t* __restrict__ comp, const unsigned long long* __restrict__ best,
                            uint32_t* __restrict__ parent, int64_t n) {
   GRID_STRIDE(cc, n) {
@@ -307,7 +322,7 @@ void run_mst(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   unsigned long long* best = r.mst_best.as<unsigned long long>();
   int* flag = r.changed.as<int>();
   unsigned long long* wsum = reinterpret_cast<unsigned long long*>(r.changed.as<char>() + 8);
-  const int gn = grid_for(c, n), ge = grid_for(c, std::max<int64_t>(L.m, 1));
+  const int gn = grid_for(c, n);
   cudaEvent_t e0, e1;
   CUDA_OK(cudaEventCreate(&e0));
   CUDA_OK(cudaEventCreate(&e1));
@@ -316,12 +331,18 @@ void run_mst(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   CUDA_OK(cudaMemsetAsync(wsum, 0, 8, s));
   int launches = 1, rounds = 0;
   int64_t edges = 0;
+  // active-edge lists (cub::DeviceSelect keeps edge order): round r scans only
+  // the edges that still join two components
+  DBuf act[2], nsel, stmp;
+  int64_t na = L.m;
+  const uint32_t* al = nullptr;
+  int cur = 0;
   while (true) {
     int h = 0;
     CUDA_OK(cudaMemsetAsync(best, 0xFF, sizeof(unsigned long long) * n, s));
     CUDA_OK(cudaMemsetAsync(flag, 0, 4, s));
-    k_mst_best<<<ge, 256, 0, s>>>(L, comp, best, flag);
-    edges += L.m;
+    k_mst_best<<<grid_for(c, std::max<int64_t>(na, 1)), 256, 0, s>>>(L, al, na, comp, best, flag);
+    edges += na;
     rounds++;
     launches++;
     CUDA_OK(cudaMemcpyAsync(&h, flag, 4, cudaMemcpyDeviceToHost, s));
@@ -342,6 +363,34 @@ void run_mst(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     }
     k_mst_relabel<<<gn, 256, 0, s>>>(comp, parent.as<uint32_t>(), n);
     launches++;
+    // compact the cross-component edges for the next round
+    if (!act[0].p) {
+      act[0].alloc(c, sizeof(uint32_t) * std::max<int64_t>(L.m, 1));
+      act[1].alloc(c, sizeof(uint32_t) * std::max<int64_t>(L.m, 1));
+      nsel.alloc(c, 8);
+    }
+    MstCross pred{L.esrc, L.adj, comp};
+    size_t tb = 0;
+    if (al) {
+      CUDA_OK(cub::DeviceSelect::If(nullptr, tb, al, act[cur ^ 1].as<uint32_t>(), nsel.as<int64_t>(), na, pred, s));
+    } else {
+      cub::CountingInputIterator<uint32_t> all(0);
+      CUDA_OK(cub::DeviceSelect::If(nullptr, tb, all, act[cur ^ 1].as<uint32_t>(), nsel.as<int64_t>(), na, pred, s));
+    }
+    stmp.alloc(c, tb);
+    if (al) {
+      CUDA_OK(cub::DeviceSelect::If(stmp.p, tb, al, act[cur ^ 1].as<uint32_t>(), nsel.as<int64_t>(), na, pred, s));
+    } else {
+      cub::CountingInputIterator<uint32_t> all(0);
+      CUDA_OK(cub::DeviceSelect::If(stmp.p, tb, all, act[cur ^ 1].as<uint32_t>(), nsel.as<int64_t>(), na, pred, s));
+    }
+    launches++;
+    int64_t hn = 0;
+    CUDA_OK(cudaMemcpyAsync(&hn, nsel.p, 8, cudaMemcpyDeviceToHost, s));
+    CUDA_OK(cudaStreamSynchronize(s));
+    cur ^= 1;
+    al = act[cur].as<uint32_t>();
+    na = hn;
   }
   unsigned long long W = 0;
   CUDA_OK(cudaMemcpyAsync(&W, wsum, 8, cudaMemcpyDeviceToHost, s));
