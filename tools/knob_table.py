@@ -12,9 +12,13 @@ for f in sorted(glob.glob(sys.argv[1] + "/*.jsonl")):
                   f"PR {d['pagerank_ms']:.2f} ms ({d['pagerank_iters']} it)")
             continue
         if d["knob"] == "exact":
-            print(f"  {d['graph']} exact: SSSP lb {d['sssp_lb_ms']:.2f} ms tpv {d['sssp_tpv_ms']:.2f} | PR lb {d['pr_lb_ms']:.2f} tpv {d['pr_tpv_ms']:.2f} ({d['pr_iters']} it)")
+            pbx = f" pb {d['pr_pb_ms']:.2f}" if "pr_pb_ms" in d else ""
+            print(f"  {d['graph']} exact: SSSP lb {d['sssp_lb_ms']:.2f} ms tpv {d['sssp_tpv_ms']:.2f} | PR lb {d['pr_lb_ms']:.2f} tpv {d['pr_tpv_ms']:.2f}{pbx} ({d['pr_iters']} it)")
             continue
         print(f"  {d['knob']:30s} tr {d['transform_s']:5.1f}s +{d['extra_space_pct']:5.2f}% | SSSP tpv {d['sssp_tpv_ms']:7.2f} "
               f"({d['sssp_tpv_speedup_same_mapping']:.2f}x) lb {d['sssp_lb_ms']:6.2f} ({d['sssp_lb_speedup_same_mapping']:.2f}x) "
               f"inacc {d['sssp_inacc_pct']:.2f}% | PR tpv {d['pagerank_tpv_ms']:7.2f} ({d['pagerank_tpv_speedup_same_mapping']:.2f}x) "
-              f"lb {d['pagerank_lb_ms']:6.2f} ({d['pagerank_lb_speedup_same_mapping']:.2f}x) inacc {d['pr_inacc_pct']:.2f}% it {d['pr_lb_iters']}")
+              f"lb {d['pagerank_lb_ms']:6.2f} ({d['pagerank_lb_speedup_same_mapping']:.2f}x)"
+              + (f" pb {d['pagerank_pb_ms']:6.2f} ({d['pagerank_pb_speedup_same_mapping']:.2f}x, "
+                 f"{d['pagerank_pb_speedup_vs_best_exact']:.2f}x best)" if "pagerank_pb_ms" in d else "")
+              + f" inacc {d['pr_inacc_pct']:.2f}% it {d['pr_lb_iters']}")
