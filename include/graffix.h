@@ -66,10 +66,10 @@ typedef enum { GX_MERGE_MEAN = 0, GX_MERGE_MIN = 1 } gx_merge;
  * streamed along the edges in (source block, sink block) segments and summed
  * in shared memory, so no random global gathers remain; single GPU,
  * asynchronous schedule.  AUTO = PB for PageRank on one GPU when the graph
- * spans at least GX_PB_MIN_BLOCKS blocks of 16384 slots and no §3 tiles are
- * present, else LB in exact mode and TPV when §2 or §4 is on. */
+ * spans at least GX_PB_MIN_BINS_PER_SM blocks of 16384 slots per SM and no §3
+ * tiles are present, else LB in exact mode and TPV when §2 or §4 is on. */
 typedef enum { GX_MAP_AUTO = 0, GX_MAP_LB = 1, GX_MAP_TPV = 2, GX_MAP_PB = 3 } gx_mapping;
-#define GX_PB_MIN_BLOCKS 64
+#define GX_PB_MIN_BINS_PER_SM 3
 
 /* upload / download flags */
 #define GX_PTRS_HOST 0u       /* pointers are host memory (pageable or pinned)   */

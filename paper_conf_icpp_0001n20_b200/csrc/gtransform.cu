@@ -296,3 +296,194 @@ void gpu_bfs_forest(Ctx* c, int64_t n, const int64_t* rp, const int32_t* col, st
 }
 
 }  // namespace gx
+
+namespace gx {
+
+// ---------------------------------------------------------------- §4 padding
+// Candidates of the degree normalisation (P@33654-35029, readings R32/R33):
+// for a padded vertex u, the logical 2-hop out-neighbours q not in N+(u) and
+// not u, each with its lightest combined weight, ordered by (weight, id); the
+// first `take` of them become edges.  Two segmented radix sorts per batch of
+// queries: (q, w) keys to keep each q's minimum, then (w, q) keys.
+__device__ __forceinline__ uint32_t combine_w_dev(uint32_t w1, uint32_t w2, int rule) {
+  if (rule == GX_W_MAX) return max(w1, w2);
+  if (rule == GX_W_MEAN) return max(1u, (uint32_t)(((uint64_t)w1 + w2) / 2));
+  return w1 + w2;
+}
+
+// upper bound of query i's candidates: sum of |N+(x)| over x in N+(u)
+__global__ void k_pad_count(const int64_t* __restrict__ lp, const int32_t* __restrict__ ld,
+                            const int32_t* __restrict__ qu, int64_t nq, uint64_t* __restrict__ cnt) {
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const unsigned lane = threadIdx.x & 31;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t i = warp; i < nq; i += nw) {
+    const int32_t u = qu[i];
+    unsigned long long c = 0;
+    for (int64_t e = lp[u] + lane; e < lp[u + 1]; e += 32) {
+      const int32_t x = ld[e];
+      c += (unsigned long long)(lp[x + 1] - lp[x]);
+    }
+    for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(FULL, c, o);
+    if (lane == 0) cnt[i] = c;
+  }
+}
+
+// (q << 32 | w) per 2-hop path u -> x -> q; excluded q (u itself or an out-
+// neighbour of u) become the sentinel ~0 (sorted last)
+__global__ void k_pad_fill(const int64_t* __restrict__ lp, const int32_t* __restrict__ ld,
+                           const uint32_t* __restrict__ lw, const int32_t* __restrict__ qu, int64_t nq,
+                           const uint64_t* __restrict__ off, uint64_t base, int rule,
+                           unsigned long long* __restrict__ keys) {
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const unsigned lane = threadIdx.x & 31;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t i = warp; i < nq; i += nw) {
+    const int32_t u = qu[i];
+    const int64_t ua = lp[u], ub = lp[u + 1];
+    uint64_t o = off[i] - base;
+    for (int64_t ex = ua; ex < ub; ex++) {
+      const int32_t x = ld[ex];
+      const uint32_t w1 = lw[ex];
+      const int64_t xa = lp[x], xb = lp[x + 1];
+      for (int64_t eq = xa + lane; eq < xb; eq += 32) {
+        const int32_t q = ld[eq];
+        bool keep = q != u;
+        if (keep) {   // q in N+(u)?  (rows sorted by destination)
+          int64_t lo = ua, hi = ub;
+          while (lo < hi) {
+            const int64_t mid = (lo + hi) >> 1;
+            if (ld[mid] < q) lo = mid + 1;
+            else hi = mid;
+          }
+          keep = !(lo < ub && ld[lo] == q);
+        }
+        keys[o + (eq - xa)] = keep ? (((unsigned long long)(uint32_t)q << 32) | combine_w_dev(w1, lw[eq], rule))
+                                   : ~0ull;
+      }
+      o += (uint64_t)(xb - xa);
+    }
+  }
+}
+
+// first (q, w) of each q -> (w << 32 | q); repeats and sentinels -> ~0
+__global__ void k_pad_dedupe(const unsigned long long* __restrict__ in, unsigned long long* __restrict__ out,
+                             const uint64_t* __restrict__ off, int64_t nq, uint64_t base) {
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const unsigned lane = threadIdx.x & 31;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t i = warp; i < nq; i += nw) {
+    const uint64_t a = off[i] - base, b = off[i + 1] - base;
+    for (uint64_t j = a + lane; j < b; j += 32) {
+      const unsigned long long k = in[j];
+      const bool first = k != ~0ull && (j == a || (in[j - 1] >> 32) != (k >> 32));
+      out[j] = first ? (((k & 0xffffffffull) << 32) | (k >> 32)) : ~0ull;
+    }
+  }
+}
+
+// the first take_i keys of every sorted segment (~0 where fewer exist)
+__global__ void k_pad_take(const unsigned long long* __restrict__ k, const uint64_t* __restrict__ off, uint64_t base,
+                           const int64_t* __restrict__ tptr, int64_t nq, unsigned long long* __restrict__ out) {
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const unsigned lane = threadIdx.x & 31;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t i = warp; i < nq; i += nw) {
+    const uint64_t a = off[i] - base, len = off[i + 1] - off[i];
+    const int64_t t0 = tptr[i], t = tptr[i + 1] - t0;
+    for (int64_t j = lane; j < t; j += 32) out[t0 - tptr[0] + j] = (uint64_t)j < len ? k[a + j] : ~0ull;
+  }
+}
+
+// queries (vertex qu[i], at most qtake[i] edges); lout = G_L out-adjacency as
+// CSR sorted by destination (host).  Out: for query i the chosen (w << 32 | q)
+// keys in [rptr[i], rptr[i+1]) of rkeys, in (weight, id) order.
+void gpu_pad_candidates(Ctx* c, int64_t n, const int64_t* lp, const int32_t* ld, const uint32_t* lw, int64_t nq,
+                        const int32_t* qu, const int32_t* qtake, int rule, std::vector<int64_t>& rptr,
+                        std::vector<uint64_t>& rkeys) {
+  cudaStream_t s = c->stream;
+  rptr.assign(nq + 1, 0);
+  rkeys.clear();
+  if (nq == 0) return;
+  const int64_t m = lp[n];
+  DBuf dlp, dld, dlw, dqu, cnt, off, tmp, k0, k1, sb, kout;
+  dlp.alloc(c, sizeof(int64_t) * (n + 1));
+  dld.alloc(c, sizeof(int32_t) * std::max<int64_t>(m, 1));
+  dlw.alloc(c, sizeof(uint32_t) * std::max<int64_t>(m, 1));
+  dqu.alloc(c, sizeof(int32_t) * nq);
+  CUDA_OK(cudaMemcpyAsync(dlp.p, lp, sizeof(int64_t) * (n + 1), cudaMemcpyHostToDevice, s));
+  if (m) {
+    CUDA_OK(cudaMemcpyAsync(dld.p, ld, sizeof(int32_t) * m, cudaMemcpyHostToDevice, s));
+    CUDA_OK(cudaMemcpyAsync(dlw.p, lw, sizeof(uint32_t) * m, cudaMemcpyHostToDevice, s));
+  }
+  CUDA_OK(cudaMemcpyAsync(dqu.p, qu, sizeof(int32_t) * nq, cudaMemcpyHostToDevice, s));
+  cnt.alloc(c, sizeof(uint64_t) * (nq + 1));
+  off.alloc(c, sizeof(uint64_t) * (nq + 1));
+  CUDA_OK(cudaMemsetAsync(cnt.p, 0, sizeof(uint64_t) * (nq + 1), s));
+  const int grid = c->num_sms * 16;
+  k_pad_count<<<grid, 256, 0, s>>>(dlp.as<int64_t>(), dld.as<int32_t>(), dqu.as<int32_t>(), nq, cnt.as<uint64_t>());
+  CUDA_OK(cudaGetLastError());
+  size_t tb = 0;
+  CUDA_OK(cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt.as<uint64_t>(), off.as<uint64_t>(), nq + 1, s));
+  tmp.alloc(c, tb);
+  CUDA_OK(cub::DeviceScan::ExclusiveSum(tmp.p, tb, cnt.as<uint64_t>(), off.as<uint64_t>(), nq + 1, s));
+  // output slots per query: qtake[i] (the caller's upper bound)
+  std::vector<int64_t> htp(nq + 1, 0);
+  for (int64_t i = 0; i < nq; i++) htp[i + 1] = htp[i] + std::max<int32_t>(qtake[i], 0);
+  DBuf dtp;
+  dtp.alloc(c, sizeof(int64_t) * (nq + 1));
+  CUDA_OK(cudaMemcpyAsync(dtp.p, htp.data(), sizeof(int64_t) * (nq + 1), cudaMemcpyHostToDevice, s));
+  std::vector<uint64_t> hoff(nq + 1);
+  CUDA_OK(cudaMemcpyAsync(hoff.data(), off.p, sizeof(uint64_t) * (nq + 1), cudaMemcpyDeviceToHost, s));
+  CUDA_OK(cudaStreamSynchronize(s));
+  // batches of queries with at most B candidate keys (segmented sorts take int sizes)
+  const uint64_t B = uint64_t(1) << 28;
+  std::vector<uint64_t> hk;
+  int64_t i0 = 0;
+  while (i0 < nq) {
+    int64_t i1 = i0 + 1;
+    while (i1 < nq && hoff[i1 + 1] - hoff[i0] <= B) i1++;
+    const uint64_t base = hoff[i0], tot = hoff[i1] - base;
+    const int64_t bq = i1 - i0;
+    k0.alloc(c, sizeof(uint64_t) * std::max<uint64_t>(tot, 1));
+    k1.alloc(c, sizeof(uint64_t) * std::max<uint64_t>(tot, 1));
+    sb.alloc(c, sizeof(int64_t) * (bq + 1));
+    std::vector<int64_t> seg(bq + 1);
+    for (int64_t i = 0; i <= bq; i++) seg[i] = (int64_t)(hoff[i0 + i] - base);
+    CUDA_OK(cudaMemcpyAsync(sb.p, seg.data(), sizeof(int64_t) * (bq + 1), cudaMemcpyHostToDevice, s));
+    if (tot) {
+      k_pad_fill<<<grid, 256, 0, s>>>(dlp.as<int64_t>(), dld.as<int32_t>(), dlw.as<uint32_t>(), dqu.as<int32_t>() + i0,
+                                      bq, off.as<uint64_t>() + i0, base, rule, k0.as<unsigned long long>());
+      CUDA_OK(cudaGetLastError());
+      size_t t1 = 0;
+      const int64_t* b0 = sb.as<int64_t>();
+      CUDA_OK(cub::DeviceSegmentedSort::SortKeys(nullptr, t1, k0.as<uint64_t>(), k1.as<uint64_t>(), (int)tot,
+                                                 (int)bq, b0, b0 + 1, s));
+      tmp.alloc(c, t1);
+      CUDA_OK(cub::DeviceSegmentedSort::SortKeys(tmp.p, t1, k0.as<uint64_t>(), k1.as<uint64_t>(), (int)tot, (int)bq,
+                                                 b0, b0 + 1, s));
+      k_pad_dedupe<<<grid, 256, 0, s>>>(k1.as<unsigned long long>(), k0.as<unsigned long long>(),
+                                        off.as<uint64_t>() + i0, bq, base);
+      CUDA_OK(cudaGetLastError());
+      CUDA_OK(cub::DeviceSegmentedSort::SortKeys(tmp.p, t1, k0.as<uint64_t>(), k1.as<uint64_t>(), (int)tot, (int)bq,
+                                                 b0, b0 + 1, s));
+      // only the first take_i keys of each segment travel back
+      const int64_t nt = htp[i1] - htp[i0];
+      kout.alloc(c, sizeof(uint64_t) * std::max<int64_t>(nt, 1));
+      k_pad_take<<<grid, 256, 0, s>>>(k1.as<unsigned long long>(), off.as<uint64_t>() + i0, base,
+                                      dtp.as<int64_t>() + i0, bq, kout.as<unsigned long long>());
+      CUDA_OK(cudaGetLastError());
+      hk.resize(nt);
+      if (nt) CUDA_OK(cudaMemcpyAsync(hk.data(), kout.p, sizeof(uint64_t) * nt, cudaMemcpyDeviceToHost, s));
+      CUDA_OK(cudaStreamSynchronize(s));
+    }
+    for (int64_t i = i0; i < i1; i++) {
+      if (tot)
+        for (int64_t j = htp[i] - htp[i0]; j < htp[i + 1] - htp[i0] && hk[j] != ~0ull; j++) rkeys.push_back(hk[j]);
+      rptr[i + 1] = (int64_t)rkeys.size();
+    }
+    i0 = i1;
+  }
+}
+
+}  // namespace gx

@@ -210,6 +210,9 @@ void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out, Ctx* de
 void gpu_triangles(Ctx* c, int64_t n, const int64_t* np, const int32_t* nc, int64_t* T);
 void gpu_bfs_forest(Ctx* c, int64_t n, const int64_t* rp, const int32_t* col, std::vector<int32_t>& sources,
                     std::vector<int32_t>& level);
+void gpu_pad_candidates(Ctx* c, int64_t n, const int64_t* lp, const int32_t* ld, const uint32_t* lw, int64_t nq,
+                        const int32_t* qu, const int32_t* qtake, int rule, std::vector<int64_t>& rptr,
+                        std::vector<uint64_t>& rkeys);
 void build_device_exact(gx_graph* g);
 void build_device_slots(gx_graph* g);
 void build_tpv(gx_graph* g);

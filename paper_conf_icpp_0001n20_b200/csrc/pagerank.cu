@@ -1105,7 +1105,11 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   const bool tiles = d.n_tiles && g->knobs.smem;
   int mapping = o.mapping;
   if (mapping == GX_MAP_AUTO) {
-    const bool pb_ok = async_ && !tiles && (ns + PB_R - 1) / PB_R >= GX_PB_MIN_BLOCKS && !getenv("GX_NO_PB");
+    // one CTA per SM claims sink bins: with fewer than ~3 bins per SM the last
+    // wave leaves most SMs idle (RMAT-22, 256 bins: 5.5 ms vs LB 4.5 ms;
+    // RMAT-24, 1024 bins: 12.2 vs 16.1 ms)
+    const bool pb_ok = async_ && !tiles && (ns + PB_R - 1) / PB_R >= (int64_t)GX_PB_MIN_BINS_PER_SM * c->num_sms &&
+                       !getenv("GX_NO_PB");
     mapping = pb_ok ? GX_MAP_PB
                     : (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
   }

@@ -645,7 +645,8 @@ int bucket_of(int64_t d) {
   return b;  // R30: 0 for d = 0, else 1 + floor(log2 d)
 }
 
-void degnorm(Work& W, int64_t th, int64_t f, bool combined, int wrule, std::vector<int32_t>& sched, int64_t& added) {
+void degnorm(Work& W, int64_t th, int64_t f, bool combined, int wrule, std::vector<int32_t>& sched, int64_t& added,
+             Ctx* dev) {
   PhaseTimer pt;
   const int64_t ns = W.n_slots;
   std::vector<int64_t> deg(ns);
@@ -666,6 +667,45 @@ void degnorm(Work& W, int64_t th, int64_t f, bool combined, int wrule, std::vect
   pt("order + logical out");
   std::vector<std::vector<Edge>> adds(ns);
   const int64_t nwarps = ((int64_t)order.size() + 31) / 32;
+  if (dev) {
+    // N1: the padded slots are found here (per-warp M and target), their
+    // candidates ranked on the device (gtransform.cu gpu_pad_candidates)
+    std::vector<int32_t> qs, qu, qtake;
+    for (int64_t wi = 0; wi < nwarps; wi++) {
+      const int64_t b0 = wi * 32, b1 = std::min<int64_t>(b0 + 32, (int64_t)order.size());
+      int64_t M = 0;
+      for (int64_t i = b0; i < b1; i++) M = std::max(M, deg[order[i]]);
+      const int64_t target = (f * M + 999999) / 1000000;
+      for (int64_t i = b0; i < b1; i++) {
+        const int32_t s = order[i];
+        const int64_t d = deg[s];
+        if (W.kind[s] != OWNER || !(0 < d && d < M)) continue;
+        if (!((M - d) * 1000000 < th * M)) continue;
+        if (d >= target) continue;
+        qs.push_back(s);
+        qu.push_back(W.slot_to_orig[s]);
+        qtake.push_back((int32_t)(target - d));
+      }
+    }
+    std::vector<int64_t> lp(W.n + 1, 0);
+    for (int64_t u = 0; u < W.n; u++) lp[u + 1] = lp[u] + (int64_t)lout[u].size();
+    std::vector<int32_t> ld(std::max<int64_t>(lp[W.n], 1));
+    std::vector<uint32_t> lw(std::max<int64_t>(lp[W.n], 1));
+#pragma omp parallel for schedule(dynamic, 4096)
+    for (int64_t u = 0; u < W.n; u++)
+      for (size_t j = 0; j < lout[u].size(); j++) {
+        ld[lp[u] + j] = lout[u][j].first;
+        lw[lp[u] + j] = lout[u][j].second;
+      }
+    std::vector<int64_t> rptr;
+    std::vector<uint64_t> rkeys;
+    gpu_pad_candidates(dev, W.n, lp.data(), ld.data(), lw.data(), (int64_t)qs.size(), qu.data(), qtake.data(), wrule,
+                       rptr, rkeys);
+    for (size_t i = 0; i < qs.size(); i++)
+      for (int64_t j = rptr[i]; j < rptr[i + 1]; j++)
+        adds[qs[i]].push_back({W.owner[(int32_t)(rkeys[j] & 0xffffffffull)], (uint32_t)(rkeys[j] >> 32), ADD_DEGNORM});
+    pt("padding candidates (GPU)");
+  } else {
 #pragma omp parallel for schedule(dynamic, 64)
   for (int64_t wi = 0; wi < nwarps; wi++) {
     const int64_t b0 = wi * 32, b1 = std::min<int64_t>(b0 + 32, (int64_t)order.size());
@@ -703,6 +743,7 @@ void degnorm(Work& W, int64_t th, int64_t f, bool combined, int wrule, std::vect
     }
   }
   pt("padding candidates");
+  }
   added = 0;
   for (int64_t s = 0; s < ns; s++) {
     added += (int64_t)adds[s].size();
@@ -745,7 +786,8 @@ void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out, Ctx* de
   std::vector<int32_t> sched;
   int64_t added_dn = 0;
   if (k.degree_norm)
-    degnorm(W, ppm(k.degsim_threshold), ppm(k.degree_target), k.coalesce != 0, k.added_weight_rule, sched, added_dn);
+    degnorm(W, ppm(k.degsim_threshold), ppm(k.degree_target), k.coalesce != 0, k.added_weight_rule, sched, added_dn,
+            dev);
   phase("degnorm");
 
   // assemble the slot CSR, rows sorted by destination slot (R11)

@@ -1,8 +1,9 @@
 """GPU-resident preprocessing: with a device context the
 §3 triangle counts (the clustering coefficients of P@29857 that drive the CC
 edge insertion and the subgraph selection) and the §2 source order,
-reachability forest and multi-source BFS levels (Alg 2 l.2-6) are computed on
-the GPU (gtransform.cu).  The exported transformed graph must be bit-identical to
+reachability forest and multi-source BFS levels (Alg 2 l.2-6) and the §4
+padding candidates (2-hop out-neighbours ranked by (weight, id), P@33654) are
+computed on the GPU (gtransform.cu).  The exported transformed graph must be bit-identical to
 the oracle's and to the host-only library path (no device), element by
 element -- the triangle counts feed integer decisions only."""
 import numpy as np
@@ -49,7 +50,7 @@ def test_device_transform_matches_oracle(gname, kname):
 
 
 @pytest.mark.parametrize("scale", [16, 18])
-@pytest.mark.parametrize("kname", ["smem", "coalesce_smem"])
+@pytest.mark.parametrize("kname", ["smem", "coalesce_smem", "degnorm", "degnorm_wmax", "all"])
 def test_device_transform_matches_host_library(scale, kname):
     """Larger RMAT (many triangles, hub rows): device path vs the host-only
     library path, whose transforms are pinned to the oracle on CPU."""
@@ -58,7 +59,11 @@ def test_device_transform_matches_host_library(scale, kname):
     raw = graphgen.rmat(scale)
     kn = {"smem": T.Knobs(smem=True, cc_threshold=0.5),
           "coalesce_smem": T.Knobs(coalesce=True, chunk_k=16, replicate_threshold=0.4, smem=True,
-                                   cc_threshold=0.5)}[kname]
+                                   cc_threshold=0.5),
+          "degnorm": T.Knobs(degree_norm=True, degsim_threshold=0.5),
+          "degnorm_wmax": T.Knobs(degree_norm=True, degsim_threshold=0.4, added_weight="max"),
+          "all": T.Knobs(coalesce=True, chunk_k=16, replicate_threshold=0.4, smem=True, cc_threshold=0.5,
+                         degree_norm=True, degsim_threshold=0.4)}[kname]
     G = upload(raw)
     info = G.transform(_knobs(gx, kn))
     H = gx.Graph.host_only(raw.row_ptr, raw.col, raw.w)
@@ -67,10 +72,10 @@ def test_device_transform_matches_host_library(scale, kname):
     for k in ("row_ptr", "col", "w", "edge_added", "slot_to_orig", "slot_kind", "sched", "tile_ptr",
               "tile_members", "tile_centre", "tile_iters"):
         assert np.array_equal(np.asarray(a[k]), np.asarray(b[k])), k
-    for k in ("n_slots", "n_replicas", "n_holes", "edges_added_coalesce", "edges_added_smem", "n_subgraphs",
-              "subgraph_vertices"):
+    for k in ("n_slots", "n_replicas", "n_holes", "edges_added_coalesce", "edges_added_smem", "edges_added_degnorm",
+              "n_subgraphs", "subgraph_vertices"):
         assert info[k] == hinfo[k], k
-    assert info["n_subgraphs"] > 0
+    assert info["n_subgraphs"] > 0 or info["edges_added_degnorm"] > 0
 
 
 def test_device_levels_road_grid():

@@ -11,6 +11,10 @@ for f in sorted(glob.glob(sys.argv[1] + "/*.jsonl")):
             print(f"  [{d['knob']}] P={d['P']} ({d['note']}): SSSP {d['sssp_ms']:.2f} ms ({d['sssp_iters']} it) | "
                   f"PR {d['pagerank_ms']:.2f} ms ({d['pagerank_iters']} it)")
             continue
+        if "sssp_lb_ms" not in d and "pagerank_lb_ms" not in d:   # other tools' lines (algos_c4)
+            print("  " + ", ".join(f"{k}={v:.3g}" if isinstance(v, float) else f"{k}={v}" for k, v in d.items()
+                                   if k not in ("config", "graph", "n", "m")))
+            continue
         if d["knob"] == "exact":
             pbx = f" pb {d['pr_pb_ms']:.2f}" if "pr_pb_ms" in d else ""
             print(f"  {d['graph']} exact: SSSP lb {d['sssp_lb_ms']:.2f} ms tpv {d['sssp_tpv_ms']:.2f} | PR lb {d['pr_lb_ms']:.2f} tpv {d['pr_tpv_ms']:.2f}{pbx} ({d['pr_iters']} it)")
