@@ -128,6 +128,9 @@ struct DevGraph {
   bool identity = true;        // exact mode: slot == original id, no holes
   uint32_t max_w = 1;
   DBuf rp, adj;                // out-CSR: u32 [n_slots+1], uint2 {col, w} [m_slots]
+  DBuf adjp;                   // packed out-edges col << adjp_wbits | w (sssp.cu), when they fit 32 bits
+  uint32_t adjp_wbits = 0;
+  bool adjp_tried = false;
   DBuf crp, csrc;              // in-CSC:  u32 [n_slots+1], i32 [m_slots]
   DBuf D;                      // u32 [n_slots]: logical out-degree (PR divisor)
   DBuf owner;                  // i32 [n]: original id -> owner slot

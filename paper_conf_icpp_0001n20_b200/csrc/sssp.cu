@@ -162,7 +162,7 @@ __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, con
         for (int q = 0; q < SU; q++) {
           uint32_t e = e0 + q * 32 + lane;
           ok[q] = e < b;
-          ed[q] = ok[q] ? ld_stream_u2(adj + e, pf) : make_uint2(0, 0);
+          ed[q] = ok[q] ? ld_edge(adj, ax, e, pf) : make_uint2(0, 0);
         }
         uint32_t cv[SU];
 #pragma unroll
@@ -245,7 +245,7 @@ __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, con
           const uint32_t oe = __shfl_sync(FULL, dexcl, j);
           od[q] = __shfl_sync(FULL, du, j);
           ok[q] = kk < dtot;
-          ed[q] = ok[q] ? ld_stream_u2(adj + os + (kk - oe), pf) : make_uint2(0, 0);
+          ed[q] = ok[q] ? ld_edge(adj, ax, os + (kk - oe), pf) : make_uint2(0, 0);
         }
         uint32_t cv[SU];
 #pragma unroll
@@ -618,7 +618,7 @@ __device__ __forceinline__ void sssp_block_dev(const uint32_t* __restrict__ rp, 
       my_act++;
       my_edges += b - a;
       for (uint32_t e = a; e < b; e++) {
-        const uint2 ed = ld_stream_u2(adj + e, pf);
+        const uint2 ed = ld_edge(adj, ax, e, pf);
         uint32_t nd = du + ed.y;
         if (nd < du) nd = INF - 1;
         const uint32_t cv = ld_l2_u32(dist + ed.x, pl);
@@ -711,7 +711,7 @@ struct SsspLoop {
   const uint32_t* rp;
   const uint2* adj;
   uint32_t* dist;
-  SsspAux ax;
+  SsspAux ax{};
   SsspState* st;
   int64_t n_slots;
   const int32_t *tptr, *tmem, *teptr, *titers;
@@ -908,6 +908,45 @@ static unsigned sssp_delta(const gx_graph* g) {
   return (unsigned)std::max(1.0, delta);
 }
 
+__global__ void k_adj_wmax(const uint2* __restrict__ adj, int64_t m, unsigned int* __restrict__ out) {
+  unsigned int mx = 0;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x)
+    mx = max(mx, adj[e].y);
+  mx = warp_max_u32(mx);
+  if ((threadIdx.x & 31) == 0 && mx) atomicMax(out, mx);
+}
+__global__ void k_adj_pack(const uint2* __restrict__ adj, int64_t m, uint32_t wb, uint32_t* __restrict__ out) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x) {
+    const uint2 v = adj[e];
+    out[e] = (v.x << wb) | v.y;
+  }
+}
+
+// {dst, w} packed into one u32 when the slot ids and the largest weight fit
+// (RMAT-24: 24 + 7 bits): the relaxation stream halves (8 -> 4 B per edge)
+static void ensure_packed_adj(gx_graph* g) {
+  DevGraph& d = g->dg;
+  if (d.adjp_tried) return;
+  d.adjp_tried = true;
+  if (getenv("GX_SSSP_NO_PACK") || d.m_slots == 0) return;
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  DBuf mx;
+  mx.alloc(c, 4);
+  CUDA_OK(cudaMemsetAsync(mx.p, 0, 4, s));
+  k_adj_wmax<<<grid_for(c, d.m_slots), 256, 0, s>>>(d.adj.as<uint2>(), d.m_slots, mx.as<unsigned int>());
+  unsigned int wmax = 0;
+  CUDA_OK(cudaMemcpyAsync(&wmax, mx.p, 4, cudaMemcpyDeviceToHost, s));
+  CUDA_OK(cudaStreamSynchronize(s));
+  uint32_t wb = 1;
+  while (wb < 32 && (wmax >> wb)) wb++;
+  if (wb >= 16 || d.n_slots > (int64_t(1) << (32 - wb))) return;
+  d.adjp.alloc(c, sizeof(uint32_t) * d.m_slots);
+  k_adj_pack<<<grid_for(c, d.m_slots), 256, 0, s>>>(d.adj.as<uint2>(), d.m_slots, wb, d.adjp.as<uint32_t>());
+  CUDA_OK(cudaGetLastError());
+  d.adjp_wbits = wb;
+}
+
 static void ensure_heavy_chunks(gx_graph* g) {
   DevGraph& d = g->dg;
   if (d.hc_row.p) return;
@@ -970,7 +1009,7 @@ __global__ void k_frontier_diff(const uint32_t* __restrict__ dist, const uint32_
 
 struct SsspRank {
   DBuf dist, mark, st, dold;
-  SsspAux ax;
+  SsspAux ax{};
   int64_t lo = 0, hi = 0;
 };
 
@@ -1144,7 +1183,7 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   r.mark.alloc(c, sizeof(uint32_t) * 4 * nwords);   // frontier bitmaps bm[0..2] + far pile
   r.st.alloc(c, sizeof(SsspState));
   SsspState* st = r.st.as<SsspState>();
-  SsspAux ax;
+  SsspAux ax{};
   for (int i = 0; i < 3; i++) ax.bm[i] = r.mark.as<uint32_t>() + i * nwords;
   ax.far = r.mark.as<uint32_t>() + 3 * nwords;
   ax.heavy = d.heavy_bm.as<uint32_t>();
@@ -1152,6 +1191,11 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   ax.hc_row = d.hc_row.as<int32_t>();
   ax.hc_start = d.hc_start.as<uint32_t>();
   ax.nhc = d.nhc;
+  if (mapping == GX_MAP_LB) {
+    ensure_packed_adj(g);
+    ax.adjp = d.adjp.as<uint32_t>();
+    ax.wbits = d.adjp_wbits;
+  }
   // source copies: owner slot + replica slots
   std::vector<int32_t> srcs;
   if (d.identity) {
@@ -1363,7 +1407,8 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   info.kernel_launches = launches;
   info.sweep_launches = kt.launches();
   info.sweep_ms = kt.total_ms();
-  info.sweep_bytes = info.bytes_model;
+  // packed edges: {dst, w} in 4 bytes instead of 8
+  info.sweep_bytes = ax.adjp ? 8 * (int64_t)hst.edges + 12 * (int64_t)hst.act_total : info.bytes_model;
   info.mapping_used = mapping;
   r.have[GX_SSSP] = true;
 }

@@ -38,6 +38,22 @@ struct SsspAux {
   const int32_t* hc_row;        // static heavy chunk list: row
   const uint32_t* hc_start;     //                          first edge
   int64_t nhc;
+  // packed out-edges (null: use the uint2 {dst, w} array): dst << wbits | w in
+  // one u32 when n' <= 2^(32 - wbits) -- 4 bytes per relaxed edge instead of 8
+  const uint32_t* adjp;
+  uint32_t wbits;
 };
+// the out-edge e as {dst, w}
+__device__ __forceinline__ uint2 ld_edge(const uint2* __restrict__ adj, const SsspAux& ax, uint32_t e, uint64_t pol) {
+  if (ax.adjp) {
+    uint32_t v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(ax.adjp + e), "l"(pol));
+    return make_uint2(v >> ax.wbits, v & ((1u << ax.wbits) - 1u));
+  }
+  uint2 v;
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0, %1}, [%2], %3;" : "=r"(v.x), "=r"(v.y) : "l"(adj + e),
+      "l"(pol));
+  return v;
+}
 
 }  // namespace gx
