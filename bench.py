@@ -307,7 +307,7 @@ def main():
             t = float(tt.item())
         e2e = {"value": e2e_edges / (t * 1e-3) / 1e9, "unit": UNIT, "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": d2h, "ms_per_step": t / len(e2e_ms),
-               "note": "upload of canonical pinned CSR (GX_CANONICAL) + device CSC build + SSSP + PR + download dist, rank"}
+               "note": "upload of canonical pinned CSR (GX_CANONICAL) + device layouts (SSSP heavy chunks, blocked-PR segments) + SSSP + PR + download dist, rank"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
