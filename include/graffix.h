@@ -68,7 +68,14 @@ typedef enum { GX_MERGE_MEAN = 0, GX_MERGE_MIN = 1 } gx_merge;
  * asynchronous schedule.  AUTO = PB for PageRank on one GPU when the graph
  * spans at least GX_PB_MIN_BINS_PER_SM blocks of 16384 slots per SM and no §3
  * tiles are present, else LB in exact mode and TPV when §2 or §4 is on. */
-typedef enum { GX_MAP_AUTO = 0, GX_MAP_LB = 1, GX_MAP_TPV = 2, GX_MAP_PB = 3 } gx_mapping;
+/* VNS (the paper's second workload P@11477-11746: Graffix
+ * layouts under another engine's mapping): Tigr-style virtual node splitting
+ * on our own kernels -- every slot's out-row is cut into virtual nodes of at
+ * most K edges (env GX_VNS_K, default 8), one thread per virtual node in the
+ * TPV lane order (§4 schedule or slot order), so a warp's longest row is
+ * bounded by K.  SSSP; PageRank runs TPV under it (a pull row cannot be split
+ * without a combine step). */
+typedef enum { GX_MAP_AUTO = 0, GX_MAP_LB = 1, GX_MAP_TPV = 2, GX_MAP_PB = 3, GX_MAP_VNS = 4 } gx_mapping;
 #define GX_PB_MIN_BINS_PER_SM 3
 
 /* upload / download flags */

@@ -17,14 +17,14 @@ from dataclasses import dataclass, fields
 
 import numpy as np
 
-from ._binding import (ALGOS, ALLOC_FN, GX_CANONICAL, GX_MAP_AUTO, GX_MAP_LB, GX_MAP_PB, GX_MAP_TPV, GX_OUT_BC_F64,
+from ._binding import (ALGOS, ALLOC_FN, GX_CANONICAL, GX_MAP_AUTO, GX_MAP_LB, GX_MAP_PB, GX_MAP_TPV, GX_MAP_VNS, GX_OUT_BC_F64,
                        GX_OUT_DIST_U32, GX_OUT_LABEL_I32, GX_OUT_MST_WEIGHT_U64, GX_OUT_RANK_F64,
                        GX_PTRS_DEVICE, GX_PTRS_HOST, GX_VALIDATE, RELEASE_FN, GraffixError, GxExport,
                        GxExportSizes, GxKnobs, GxRunInfo, GxRunOpts, GxTransformInfo, _check, _ptr, lib)
 
 __all__ = ["Context", "Graph", "Knobs", "GraffixError", "lib", "MAPPINGS"]
 
-MAPPINGS = {"auto": GX_MAP_AUTO, "lb": GX_MAP_LB, "tpv": GX_MAP_TPV, "pb": GX_MAP_PB}
+MAPPINGS = {"auto": GX_MAP_AUTO, "lb": GX_MAP_LB, "tpv": GX_MAP_TPV, "pb": GX_MAP_PB, "vns": GX_MAP_VNS}
 
 
 @dataclass

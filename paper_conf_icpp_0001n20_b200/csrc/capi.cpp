@@ -439,7 +439,7 @@ gx_status gx_run_ex(gx_graph* g, const gx_run_opts* opts, gx_run_info* info) {
   gx_run_opts o = *opts;
   if (o.max_iters <= 0) o.max_iters = 1000000;
   if (o.check_every <= 0) o.check_every = 8;
-  GX_CHECK_ARG(o.mapping >= GX_MAP_AUTO && o.mapping <= GX_MAP_PB, "mapping invalid");
+  GX_CHECK_ARG(o.mapping >= GX_MAP_AUTO && o.mapping <= GX_MAP_VNS, "mapping invalid");
   GX_CHECK_ARG(o.pr_schedule == GX_PR_JACOBI || o.pr_schedule == GX_PR_ASYNC, "pr_schedule invalid");
   GX_CHECK_ARG(o.merge_every >= 0, "merge_every must be >= 0");
   gx_run_info ri;

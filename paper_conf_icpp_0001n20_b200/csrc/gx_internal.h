@@ -159,6 +159,12 @@ struct DevGraph {
   DBuf tpv_out_len, tpv_out_off, tpv_out_slab;   // u32, u64, uint2 {dst, w}
   DBuf tpv_in_len, tpv_in_off, tpv_in_slab;      // u32, u64, u32 src
   int64_t tpv_out_slab_len = 0, tpv_in_slab_len = 0;
+  // VNS (N4, tpv.cu): virtual nodes of <= vns_k out-edges in TPV lane order;
+  // lanes carry their slot (for dist / frontier) and their edge chunk (slabs)
+  bool vns_ready = false;
+  int64_t vns_nslices = 0, vns_nv = 0;
+  int vns_k = 0;
+  DBuf vns_lane_slot, vns_len, vns_off, vns_slab;
   // logical graph G_L over original ids (replica rows folded into their
   // owner): SCC / MST / BC (algos.cu); in exact mode it aliases rp / adj
   bool lg_ready = false;

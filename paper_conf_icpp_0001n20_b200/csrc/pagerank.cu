@@ -1113,6 +1113,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     mapping = pb_ok ? GX_MAP_PB
                     : (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
   }
+  if (mapping == GX_MAP_VNS) mapping = GX_MAP_TPV;   // a pull row is not split (graffix.h)
   if (P_ranks > 1 || mapping != GX_MAP_PB || tiles) ensure_csc(g);
   r.x.alloc(c, sizeof(double) * ns);
   r.contrib[0].alloc(c, sizeof(float) * ns);
@@ -1156,7 +1157,8 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     const int P = sim ? o.sim_ranks : c->world;
     if (P > 1) {
       GX_CHECK_ARG(P <= 8, "at most 8 ranks");
-      GX_CHECK_ARG(o.mapping != GX_MAP_TPV && o.mapping != GX_MAP_PB, "the partitioned path uses the LB mapping");
+      GX_CHECK_ARG(o.mapping != GX_MAP_TPV && o.mapping != GX_MAP_PB && o.mapping != GX_MAP_VNS,
+                   "the partitioned path uses the LB mapping");
       GX_CHECK_ARG(o.merge_every == 1 || !d.n_groups, "the partitioned path merges after every iteration");
       run_pagerank_dist(g, o, info, a, P, sim);
       return;

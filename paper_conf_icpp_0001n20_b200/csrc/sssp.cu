@@ -890,6 +890,7 @@ int64_t default_source(gx_graph* g) {
 // ---------------------------------------------------------------- driver
 
 void ensure_tpv(gx_graph* g);                                                                  // tpv.cu
+void ensure_vns(gx_graph* g);                                                                  // tpv.cu
 
 // Near-far bucket width: a multiple of the mean edge weight scaled down by the
 // mean degree (delta-stepping's Delta ~ w / d heuristic), at least 1.
@@ -1164,7 +1165,7 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   const int P = sim ? o.sim_ranks : c->world;
   if (P > 1) {
     GX_CHECK_ARG(P <= 8, "at most 8 ranks");
-    GX_CHECK_ARG(o.mapping != GX_MAP_TPV, "the partitioned path uses the LB mapping");
+    GX_CHECK_ARG(o.mapping != GX_MAP_TPV && o.mapping != GX_MAP_VNS, "the partitioned path uses the LB mapping");
     GX_CHECK_ARG(o.merge_every == 1 || !d.n_groups, "the partitioned path merges after every iteration");
     ensure_heavy_chunks(g);
     unsigned delta = sssp_delta(g);
@@ -1176,6 +1177,7 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   if (mapping == GX_MAP_AUTO)
     mapping = (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
   if (mapping == GX_MAP_TPV) ensure_tpv(g);
+  if (mapping == GX_MAP_VNS) ensure_vns(g);
   ensure_heavy_chunks(g);
   const int64_t ns = d.n_slots;
   const int64_t nwords = (ns + 31) / 32;
@@ -1251,6 +1253,12 @@ void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     if (mapping == GX_MAP_TPV) {
       k_sssp_tpv<<<grid_tpv, 256, 0, s>>>(d.tpv_lane_row.as<int32_t>(), d.tpv_out_len.as<uint32_t>(),
                                           d.tpv_out_off.as<uint64_t>(), d.tpv_out_slab.as<uint2>(), d.tpv_nslices,
+                                          r.dist.as<uint32_t>(), ax, st);
+      nl++;
+    } else if (mapping == GX_MAP_VNS) {
+      // the TPV sweep over virtual nodes: lane -> its slot (dist, frontier), slab -> its <= K edges
+      k_sssp_tpv<<<grid_tpv, 256, 0, s>>>(d.vns_lane_slot.as<int32_t>(), d.vns_len.as<uint32_t>(),
+                                          d.vns_off.as<uint64_t>(), d.vns_slab.as<uint2>(), d.vns_nslices,
                                           r.dist.as<uint32_t>(), ax, st);
       nl++;
     } else {

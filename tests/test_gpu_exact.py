@@ -92,6 +92,22 @@ def test_pagerank_blocked_multiblock(name):
     assert np.abs(G.download("rank") - want).sum() <= 1e-6
 
 
+@pytest.mark.parametrize("name", ["rmat12", "star_hub", "road64", "dups_loops", "isolated", "single"])
+@pytest.mark.parametrize("k", ["1", "3", "8", "64"])
+def test_sssp_virtual_node_splitting(name, k, monkeypatch):
+    """N4: Tigr-style virtual node splitting (rows cut into <= K-edge virtual
+    nodes, one thread each) reaches the same Dijkstra distances."""
+    monkeypatch.setenv("GX_VNS_K", k)
+    raw = GRAPHS[name]()
+    g = from_raw(raw)
+    s = sssp_source(g)
+    want = A.sssp_dijkstra(graph_to_edgelist(g), s)
+    G = upload(raw)
+    info = G.run("sssp", source=-1, mapping="vns")
+    assert info["converged"] == 1 and info["mapping_used"] == 4
+    assert np.array_equal(G.download("dist"), want)
+
+
 def test_pagerank_blocked_needs_async():
     import paper_conf_icpp_0001n20_b200 as gx
     G = upload(graphgen.rmat(10))

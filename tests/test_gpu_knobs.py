@@ -43,7 +43,7 @@ def knobs_c(kn, merge_op=0):
 
 @pytest.mark.parametrize("gname", list(GRAPHS))
 @pytest.mark.parametrize("kname", list(KNOBS))
-@pytest.mark.parametrize("mapping", ["auto", "lb", "tpv"])
+@pytest.mark.parametrize("mapping", ["auto", "lb", "tpv", "vns"])
 def test_sssp_transformed_bit_exact(gname, kname, mapping):
     raw = GRAPHS[gname]()
     g = from_raw(raw)
