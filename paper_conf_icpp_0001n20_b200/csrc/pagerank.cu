@@ -364,7 +364,18 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell2(PrArgs a) {
 // one bin behind -- profiles/README.md "third session")
 constexpr int PB_THREADS = 1024;
 constexpr int PB_CTAS_PER_SM = 1;
-constexpr int PB_CH = 4 * PB_THREADS;   // (1): elements per bulk-copied chunk (4 per thread)
+#ifndef GX_PB_PRODUCER
+#define GX_PB_PRODUCER 1    // measured: 774 vs 813 us per sweep (RMAT-24)
+#endif
+#ifndef GX_PB_EPT
+#define GX_PB_EPT 4
+#endif
+constexpr int PB_EPT = GX_PB_EPT;   // (1): terms per consumer thread per chunk (multiple of 4)
+// (1): with a producer warp the last warp only issues the ring's bulk copies
+// and the other 31 consume; else thread 0 issues between its own chunks
+constexpr bool PB_PRODUCER = GX_PB_PRODUCER != 0;
+constexpr int PB_CONSUMERS = PB_PRODUCER ? PB_THREADS - 32 : PB_THREADS;
+constexpr int PB_CH = PB_EPT * PB_CONSUMERS;   // (1): elements per bulk-copied chunk
 #ifndef GX_PB_NST
 #define GX_PB_NST 4
 #endif
@@ -524,7 +535,7 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
   if (threadIdx.x == 0) {
     for (int i = 0; i < PB_NST; i++) {
       mbar_init(&full[i], 1);
-      mbar_init(&empty[i], NW);
+      mbar_init(&empty[i], PB_CONSUMERS / 32);
     }
     mbar_fence_init();
   }
@@ -560,7 +571,8 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
     const uint32_t E0 = __ldg(p.q + b), E1 = __ldg(qend + b);
     const uint32_t nch = (E1 - E0 + PB_CH - 1) / PB_CH;
     if (threadIdx.x == 0) {
-      for (uint32_t c = 0; c < nch && c < PB_NST; c++) issue(g + c, E0, E1, c);
+      if (!PB_PRODUCER)
+        for (uint32_t c = 0; c < nch && c < PB_NST; c++) issue(g + c, E0, E1, c);
       // L2 prefetch for (2) and (3)
       l2_prefetch_bulk(a.x + base, (uint32_t)nrows * 8u);
       l2_prefetch_bulk(a.D + base, (uint32_t)nrows * 4u);
@@ -575,36 +587,47 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
       }
       if (hi > lo) l2_prefetch_bulk(p.src_loc + lo, (hi - lo) * 2u);
     }
+    if (PB_PRODUCER && threadIdx.x >= PB_CONSUMERS) {
+      if (threadIdx.x == PB_CONSUMERS)
+        for (uint32_t c = 0; c < nch; c++) issue(g + c, E0, E1, c);
+    } else
     for (uint32_t c = 0; c < nch; c += PB_CPT) {
-      float4 tv[PB_CPT];
-      uint2 rv[PB_CPT];
-      bool ok[PB_CPT];
-      const uint32_t i = 4u * threadIdx.x;
+      constexpr int G4 = PB_EPT / 4;
+      float4 tv[PB_CPT][G4];
+      uint2 rv[PB_CPT][G4];
+      bool ok[PB_CPT][G4];
 #pragma unroll
       for (int q = 0; q < PB_CPT; q++) {
         const uint32_t cc = c + q, gc = g + cc, stg = gc % PB_NST;
-        ok[q] = false;
+#pragma unroll
+        for (int h = 0; h < G4; h++) ok[q][h] = false;
         if (cc < nch) {
           const uint32_t n = min((uint32_t)PB_CH, E1 - (E0 + cc * PB_CH));
           mbar_wait(&full[stg], (gc / PB_NST) & 1);
           const unsigned char* src = ring + stg * PB_STAGE;
-          ok[q] = i < n;
-          if (ok[q]) {
-            tv[q] = *reinterpret_cast<const float4*>(src + 4 * i);
-            rv[q] = *reinterpret_cast<const uint2*>(src + PB_CH * 4 + 2 * i);
+#pragma unroll
+          for (int h = 0; h < G4; h++) {
+            const uint32_t i = 4u * (threadIdx.x + h * PB_CONSUMERS);
+            ok[q][h] = i < n;
+            if (ok[q][h]) {
+              tv[q][h] = *reinterpret_cast<const float4*>(src + 4 * i);
+              rv[q][h] = *reinterpret_cast<const uint2*>(src + PB_CH * 4 + 2 * i);
+            }
           }
         }
       }
 #pragma unroll
       for (int q = 0; q < PB_CPT; q++)
-        if (ok[q]) pb_add4(acc_lo, acc_hi, rv[q], tv[q]);
+#pragma unroll
+        for (int h = 0; h < G4; h++)
+          if (ok[q][h]) pb_add4(acc_lo, acc_hi, rv[q][h], tv[q][h]);
       __syncwarp();
 #pragma unroll
       for (int q = 0; q < PB_CPT; q++) {
         const uint32_t cc = c + q, gc = g + cc;
         if (cc < nch) {
           if (lane == 0) mbar_arrive(&empty[gc % PB_NST]);
-          if (threadIdx.x == 0 && cc + PB_NST < nch) issue(gc + PB_NST, E0, E1, cc + PB_NST);
+          if (!PB_PRODUCER && threadIdx.x == 0 && cc + PB_NST < nch) issue(gc + PB_NST, E0, E1, cc + PB_NST);
         }
       }
     }
