@@ -460,6 +460,197 @@ __global__ void k_bc_bwd(LG L, const int32_t* __restrict__ q, int64_t q0, int64_
   }
 }
 
+// ---- batched Brandes: BCB sources at a time, per-vertex state interleaved
+// ([v][b]: levels 16 B, sigma / coef / delta 32 B each), so one sector gather
+// of a neighbour serves the whole batch and a vertex's edges are read once per
+// level at which any source of the batch reaches it.  Per source the
+// arithmetic is that of k_bc_fwd / k_bc_bwd: sigma sums are exact integers
+// (order-free), each coef / delta is the same lane-strided sum + warp
+// reduction, and bc[v] adds the batch's deltas in source order at the end.
+constexpr int BCB = 4;
+
+__global__ void k_bcb_seed(const int32_t* __restrict__ src, int nb, int32_t* __restrict__ level4,
+                           double* __restrict__ sigma4, int32_t* __restrict__ qlev) {
+  const int b = threadIdx.x;
+  if (b < nb) {
+    const int32_t s = src[b];
+    level4[(int64_t)s * BCB + b] = 0;
+    sigma4[(int64_t)s * BCB + b] = 1.0;
+    qlev[s] = 0;
+  }
+}
+
+__global__ void k_bcb_fwd(LG L, const int32_t* __restrict__ q, int64_t q0, int64_t q1, int32_t lvl,
+                          int32_t* __restrict__ level4, double* __restrict__ sigma4, int32_t* __restrict__ qlev,
+                          int32_t* __restrict__ qout, unsigned int* __restrict__ qtail) {
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t i = q0 + warp; i < q1; i += nw) {
+    const int32_t u = q[i];
+    const int4 lu = *reinterpret_cast<const int4*>(level4 + (int64_t)u * BCB);
+    const int lus[BCB] = {lu.x, lu.y, lu.z, lu.w};
+    double su[BCB];
+    unsigned m = 0;
+#pragma unroll
+    for (int b = 0; b < BCB; b++) {
+      if (lus[b] == lvl) m |= 1u << b;
+      su[b] = sigma4[(int64_t)u * BCB + b];
+    }
+    for (uint32_t e = L.rp[u] + lane_id(); e < L.rp[u + 1]; e += 32) {
+      const uint32_t w = L.adj[e].x;
+      int32_t* lw4 = level4 + (int64_t)w * BCB;
+      const int4 lw = __ldcg(reinterpret_cast<const int4*>(lw4));
+      const int lws[BCB] = {lw.x, lw.y, lw.z, lw.w};
+      bool claimed = false;
+#pragma unroll
+      for (int b = 0; b < BCB; b++) {
+        if (!(m >> b & 1u)) continue;
+        int l = lws[b];
+        if (l < 0) {
+          if (atomicCAS(lw4 + b, -1, lvl + 1) == -1) claimed = true;
+          l = lvl + 1;   // a failed CAS lost to this level's other writer
+        }
+        if (l == lvl + 1) atomicAdd(sigma4 + (int64_t)w * BCB + b, su[b]);
+      }
+      if (claimed && atomicExch(qlev + w, lvl + 1) != lvl + 1) qout[atomicAdd(qtail, 1u)] = (int32_t)w;
+    }
+  }
+}
+
+__global__ void k_bcb_bwd(LG L, const int32_t* __restrict__ q, int64_t q0, int64_t q1, int32_t lvl,
+                          const int32_t* __restrict__ level4, const double* __restrict__ sigma4,
+                          double* __restrict__ coef4, double* __restrict__ delta4) {
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t i = q0 + warp; i < q1; i += nw) {
+    const int32_t v = q[i];
+    const int4 lv = *reinterpret_cast<const int4*>(level4 + (int64_t)v * BCB);
+    const int lvs[BCB] = {lv.x, lv.y, lv.z, lv.w};
+    unsigned m = 0;
+#pragma unroll
+    for (int b = 0; b < BCB; b++)
+      if (lvs[b] == lvl) m |= 1u << b;
+    double acc[BCB] = {0.0, 0.0, 0.0, 0.0};
+    for (uint32_t e = L.rp[v] + lane_id(); e < L.rp[v + 1]; e += 32) {
+      const uint32_t w = L.adj[e].x;
+      const int4 lw = *reinterpret_cast<const int4*>(level4 + (int64_t)w * BCB);
+      const int lws[BCB] = {lw.x, lw.y, lw.z, lw.w};
+      unsigned hit = 0;
+#pragma unroll
+      for (int b = 0; b < BCB; b++)
+        if ((m >> b & 1u) && lws[b] == lvl + 1) hit |= 1u << b;
+      if (hit) {
+        const double2 c01 = *reinterpret_cast<const double2*>(coef4 + (int64_t)w * BCB);
+        const double2 c23 = *reinterpret_cast<const double2*>(coef4 + (int64_t)w * BCB + 2);
+        const double cs[BCB] = {c01.x, c01.y, c23.x, c23.y};
+#pragma unroll
+        for (int b = 0; b < BCB; b++)
+          if (hit >> b & 1u) acc[b] += cs[b];
+      }
+    }
+#pragma unroll
+    for (int b = 0; b < BCB; b++) {
+      if (!(m >> b & 1u)) continue;   // warp-uniform
+      const double sv = sigma4[(int64_t)v * BCB + b];
+      const double d = warp_sum_f64(acc[b]) * sv;
+      if (lane_id() == 0) {
+        coef4[(int64_t)v * BCB + b] = (1.0 + d) / sv;
+        delta4[(int64_t)v * BCB + b] = d;
+      }
+    }
+  }
+}
+
+// Eq 2 for the batch: bc[v] += delta_b(v) for b in source order, v != s_b
+__global__ void k_bcb_acc(const double* __restrict__ delta4, const int32_t* __restrict__ src, int nb, int64_t n,
+                          double* __restrict__ bc) {
+  GRID_STRIDE(v, n) {
+    double x = bc[v];
+    for (int b = 0; b < nb; b++)
+      if ((int32_t)v != src[b]) x += delta4[v * BCB + b];
+    bc[v] = x;
+  }
+}
+
+static void run_bc_batched(gx_graph* g, const gx_run_opts& o, gx_run_info& info, LG L) {
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  RunState& r = g->rs;
+  const int64_t n = L.n;
+  r.bc.alloc(c, sizeof(double) * n);
+  r.changed.alloc(c, 64);
+  DBuf level4, sigma4, coef4, delta4, qlev, q, dsrc;
+  level4.alloc(c, sizeof(int32_t) * BCB * n);
+  sigma4.alloc(c, sizeof(double) * BCB * n);
+  coef4.alloc(c, sizeof(double) * BCB * n);
+  delta4.alloc(c, sizeof(double) * BCB * n);
+  qlev.alloc(c, sizeof(int32_t) * n);
+  q.alloc(c, sizeof(int32_t) * BCB * n);   // a vertex is queued at most once per level it has for some source
+  dsrc.alloc(c, sizeof(int32_t) * BCB);
+  unsigned int* qtail = r.changed.as<unsigned int>();
+  const int gw = c->num_sms * 16;
+  cudaEvent_t e0, e1;
+  CUDA_OK(cudaEventCreate(&e0));
+  CUDA_OK(cudaEventCreate(&e1));
+  CUDA_OK(cudaEventRecord(e0, s));
+  CUDA_OK(cudaMemsetAsync(r.bc.p, 0, sizeof(double) * n, s));
+  int launches = 0, rounds = 0;
+  int64_t edges = 0;
+  for (int64_t s0 = 0; s0 < o.n_bc_sources; s0 += BCB) {
+    const int nbat = (int)std::min<int64_t>(BCB, o.n_bc_sources - s0);
+    int32_t hs[BCB];
+    for (int b = 0; b < nbat; b++) hs[b] = (int32_t)o.bc_sources[s0 + b];
+    std::vector<int32_t> q0v;
+    for (int b = 0; b < nbat; b++)
+      if (std::find(q0v.begin(), q0v.end(), hs[b]) == q0v.end()) q0v.push_back(hs[b]);
+    CUDA_OK(cudaMemsetAsync(level4.p, 0xFF, sizeof(int32_t) * BCB * n, s));
+    CUDA_OK(cudaMemsetAsync(qlev.p, 0xFF, sizeof(int32_t) * n, s));
+    CUDA_OK(cudaMemsetAsync(sigma4.p, 0, sizeof(double) * BCB * n, s));
+    CUDA_OK(cudaMemsetAsync(delta4.p, 0, sizeof(double) * BCB * n, s));
+    CUDA_OK(cudaMemcpyAsync(dsrc.p, hs, sizeof(int32_t) * nbat, cudaMemcpyHostToDevice, s));
+    CUDA_OK(cudaMemcpyAsync(q.p, q0v.data(), sizeof(int32_t) * q0v.size(), cudaMemcpyHostToDevice, s));
+    const unsigned int tail0 = (unsigned int)q0v.size();
+    CUDA_OK(cudaMemcpyAsync(qtail, &tail0, 4, cudaMemcpyHostToDevice, s));
+    k_bcb_seed<<<1, 32, 0, s>>>(dsrc.as<int32_t>(), nbat, level4.as<int32_t>(), sigma4.as<double>(), qlev.as<int32_t>());
+    launches++;
+    std::vector<int64_t> off{0, (int64_t)q0v.size()};
+    for (int32_t lvl = 0;; lvl++) {
+      const int64_t a = off[lvl], b = off[lvl + 1];
+      if (b == a) break;
+      k_bcb_fwd<<<gw, 256, 0, s>>>(L, q.as<int32_t>(), a, b, lvl, level4.as<int32_t>(), sigma4.as<double>(),
+                                   qlev.as<int32_t>(), q.as<int32_t>(), qtail);
+      launches++;
+      rounds++;
+      unsigned int t = 0;
+      CUDA_OK(cudaMemcpyAsync(&t, qtail, 4, cudaMemcpyDeviceToHost, s));
+      CUDA_OK(cudaStreamSynchronize(s));
+      off.push_back(t);
+    }
+    const int32_t D = (int32_t)off.size() - 2;
+    for (int32_t lvl = D; lvl >= 0; lvl--) {
+      k_bcb_bwd<<<gw, 256, 0, s>>>(L, q.as<int32_t>(), off[lvl], off[lvl + 1], lvl, level4.as<int32_t>(),
+                                   sigma4.as<double>(), coef4.as<double>(), delta4.as<double>());
+      launches++;
+    }
+    k_bcb_acc<<<grid_for(c, n), 256, 0, s>>>(delta4.as<double>(), dsrc.as<int32_t>(), nbat, n, r.bc.as<double>());
+    launches++;
+    edges += 2 * L.m * nbat;   // per source, as the single-source path counts
+  }
+  CUDA_OK(cudaEventRecord(e1, s));
+  CUDA_OK(cudaEventSynchronize(e1));
+  float ms = 0;
+  CUDA_OK(cudaEventElapsedTime(&ms, e0, e1));
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  info.iterations = rounds;
+  info.converged = 1;
+  info.loop_ms = ms;
+  info.edges_scanned = edges;
+  info.bytes_model = edges * 20;
+  info.kernel_launches = launches;
+  r.have[GX_BC] = true;
+}
+
 void run_bc(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   Ctx* c = g->ctx;
   cudaStream_t s = c->stream;
@@ -470,6 +661,10 @@ void run_bc(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   GX_CHECK_ARG(o.bc_sources != nullptr && o.n_bc_sources > 0, "BC needs bc_sources (reading R37)");
   for (int64_t i = 0; i < o.n_bc_sources; i++)
     GX_CHECK_ARG(o.bc_sources[i] >= 0 && o.bc_sources[i] < n, "BC source out of range");
+  if (!getenv("GX_BC_SINGLE")) {   // batched sources (default); GX_BC_SINGLE=1: one source at a time
+    run_bc_batched(g, o, info, L);
+    return;
+  }
   r.level.alloc(c, sizeof(int32_t) * n);
   r.sigma.alloc(c, sizeof(double) * n);
   r.delta.alloc(c, sizeof(double) * n);
