@@ -35,6 +35,7 @@ WORKLOADS = {
                               "SSSP (R36 source, int weights 1..100) + PageRank (d=0.85, tol 1e-9)"),
     "c2": dict(scale=22, desc="C2: RMAT-22, exact mode, SSSP + PageRank"),
     "c1": dict(scale=14, desc="C1: RMAT-14, exact mode, SSSP + PageRank"),
+    "c5": dict(scale=26, desc="C5 on one GPU: RMAT-26 (the paper's rmat26, P@35940), exact mode, SSSP + PageRank"),
 }
 CPU_SAMPLE_SCALE = 17
 PR_KERNELS = {1: "k_pr_sell2", 2: "k_pr_tpv", 3: "k_pr_pb"}   # gx_mapping -> PR sweep kernel

@@ -270,7 +270,8 @@ gx_status gx_export_transformed(gx_graph* g, gx_export_t* out);
 /* Run one algorithm to its fixed point on the transformed graph.  Not
  * converging within max_iters is not an error (converged = 0).
  * Errors: GX_E_STATE (no graph), GX_E_INVALID (source out of range),
- * GX_E_UNSUPPORTED ((n-1)*max(w) >= 2^32-1 for SSSP). */
+ * GX_E_UNSUPPORTED (SSSP: a shortest-path length reached 2^32-2, the saturation
+ * value of the uint32 distances, reading R51; the result is then not valid). */
 gx_status gx_run(gx_graph* g, gx_algo algo, int64_t source, int32_t max_iters, double tol,
                  gx_run_info* info);
 gx_status gx_run_ex(gx_graph* g, const gx_run_opts* opts, gx_run_info* info);

@@ -137,12 +137,18 @@ def test_errors():
     from paper_conf_icpp_0001n20_b200 import Graph
     with pytest.raises(GraffixError):
         Graph.upload(ctx(), raw.row_ptr, bad, raw.w, validate=True)
-    # overflow guard: (n-1) * max(w) >= 2^32 - 1
+    # overflow guard (R51): a shortest-path length reaching 2^32 - 2 is reported
     big = graphgen.from_edge_list(3, [(0, 1, 2**31), (1, 2, 2**31)])
     Gb = upload(big)
     with pytest.raises(GraffixError) as e:
         Gb.run("sssp", source=0)
     assert e.value.status == 6
+    # ... but a large static bound (n-1)*max(w) with short true distances runs:
+    # the saturated candidate 2^32-2 never wins against a real path
+    ok = graphgen.from_edge_list(4, [(0, 1, 1), (1, 2, 1), (2, 3, 1), (0, 3, 2**31), (3, 0, 2**31 + 7)])
+    Go = upload(ok)
+    Go.run("sssp", source=0)
+    assert list(Go.download("dist")) == [0, 1, 2, 3]
 
 
 def test_device_pointer_upload_and_download():
