@@ -131,6 +131,8 @@ struct DevGraph {
   DBuf adjp;                   // packed out-edges col << adjp_wbits | w (sssp.cu), when they fit 32 bits
   uint32_t adjp_wbits = 0;
   bool adjp_tried = false;
+  DBuf lh_lend;                // sssp.cu light / heavy split of adjp at lh_delta: u32 [n_slots]
+  uint32_t lh_delta = 0;
   DBuf crp, csrc;              // in-CSC:  u32 [n_slots+1], i32 [m_slots]
   DBuf D;                      // u32 [n_slots]: logical out-degree (PR divisor)
   DBuf owner;                  // i32 [n]: original id -> owner slot

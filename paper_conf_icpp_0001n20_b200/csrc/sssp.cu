@@ -123,10 +123,15 @@ constexpr int SB_WARPS = 8;   // warps per CTA
 __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj,
                                             uint32_t* __restrict__ dist, const SsspAux& ax, SsspState* __restrict__ st,
                                             int64_t row_lo, int64_t row_hi, const unsigned t, const uint32_t tau,
-                                            uint32_t* fdst, int32_t (*s_v)[1024]) {
-  const uint32_t* __restrict__ bm_cur = ax.bm[t % 3];
+                                            uint32_t* fdst, int32_t (*s_v)[1024], const int lh = 0,
+                                            const int pp = 0) {
+  // lh: 0 all edges; 1 light pass (light edges, frontier recorded in pend[pp]);
+  // 2 heavy pass (heavy edges of pend[pp], pend[pp ^ 1] cleared for the next bucket)
+  const uint32_t* __restrict__ bm_cur = lh == 2 ? ax.pend[pp] : ax.bm[t % 3];
   uint32_t* bm_next = ax.bm[(t + 1) % 3];
+  uint32_t* pend_w = lh == 1 ? ax.pend[pp] : nullptr;
   clear_bitmap(ax.bm[(t + 2) % 3], ax.nwords);
+  if (lh == 2) clear_bitmap(ax.pend[pp ^ 1], ax.nwords);
   const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
   const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
   const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -151,10 +156,16 @@ __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, con
       todo &= todo - 1;
       const int64_t c = gw + nw * (k0 + l);
       const int32_t u = __shfl_sync(FULL, uc, l);
-      const uint32_t a = ax.hc_start[c];
-      const uint32_t b = min(a + HCHUNK, rp[u + 1]);
+      uint32_t a = ax.hc_start[c];
+      uint32_t b = min(a + HCHUNK, rp[u + 1]);
       const uint32_t du = ld_l2_u32(dist + u, pl);
       if (a == rp[u] && lane == 0) my_act++;
+      if (lh) {   // the chunk's light / heavy part
+        const uint32_t le = ax.lend[u];
+        if (lh == 1) b = min(b, le);
+        else a = max(a, le);
+        if (a >= b) continue;
+      }
       for (uint32_t e0 = a; e0 < b; e0 += 32 * SU) {
         uint2 ed[SU];
         bool ok[SU];
@@ -192,7 +203,13 @@ __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, con
     for (int b = 0; b < SCAN_B; b++) {
       const int64_t jj = jb + 32 * b + lane;
       const int64_t wi = w_lo + gw + nw * jj;
-      wv[b] = jj < my_words ? (__ldcg(bm_cur + wi) & ~__ldg(ax.heavy + wi)) : 0u;
+      uint32_t raw = 0u;
+      if (jj < my_words) {
+        raw = __ldcg(bm_cur + wi);
+        // this warp owns word wi in every sweep: a plain read-modify-write
+        if (pend_w && raw) __stcg(pend_w + wi, __ldcg(pend_w + wi) | raw);
+      }
+      wv[b] = raw ? (raw & ~__ldg(ax.heavy + wi)) : 0u;
     }
     uint32_t anyw = 0;
 #pragma unroll
@@ -222,7 +239,10 @@ __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, con
         const int32_t u = sv[idx];
         du = ld_l2_u32(dist + u, pl);
         start = rp[u];
-        deg = rp[u + 1] - start;
+        uint32_t end = rp[u + 1];
+        if (lh == 1) end = ax.lend[u];
+        else if (lh == 2) start = ax.lend[u];
+        deg = end - start;
         my_act++;
       }
       const uint32_t dincl = warp_incl_scan_u32(deg);
@@ -745,12 +765,18 @@ __global__ void __launch_bounds__(256, 4) k_sssp_persist(SsspLoop a) {
   unsigned t = st->iter;
   uint32_t tau = st->tau, rf = INF;
   const uint32_t delta = st->delta;
+  // light / heavy split (ax.lend set; no tiles, merges or block mode): pend_n =
+  // frontier entries since the last heavy pass, hv = this iteration is one
+  const bool lh = a.ax.lend != nullptr;
+  unsigned pend_n = 0;
+  int pp = 0;
+  bool hv = false;
   for (;;) {
     if (a.block_rows > 0)
       sssp_block_dev(a.rp, a.adj, a.dist, a.ax, st, a.n_slots, a.block_rows, t, tau, &st->far3[t % 3], pool);
     else
       sssp_lb_dev(a.rp, a.adj, a.dist, a.ax, st, 0, a.n_slots, t, tau, &st->far3[t % 3],
-                  reinterpret_cast<int32_t (*)[1024]>(pool));
+                  reinterpret_cast<int32_t (*)[1024]>(pool), lh ? (hv ? 2 : 1) : 0, pp);
     grid.sync();
     if (a.ntiles) {
       sssp_tiles_collect_dev(a.ax, st, t, a.slot_tile, a.tmark, a.tlist);
@@ -783,8 +809,20 @@ __global__ void __launch_bounds__(256, 4) k_sssp_persist(SsspLoop a) {
     const uint32_t fm = min(rf, *(volatile unsigned*)&st->far3[t % 3]);
     unsigned stop = 0;
     bool split = false;
+    if (lh) {
+      if (hv) {
+        pend_n = 0;
+        pp ^= 1;
+      } else {
+        pend_n += *(volatile unsigned*)&st->active[t % 3];
+      }
+    }
+    hv = false;
     if (final_merge) {
       stop = 1;
+    } else if (pushed == 0 && pend_n > 0) {
+      hv = true;   // the bucket drained: relax the heavy edges of its slots
+      rf = fm;
     } else if (pushed == 0) {
       if (fm == INF) {
         stop = 1;
@@ -946,6 +984,51 @@ static void ensure_packed_adj(gx_graph* g) {
   k_adj_pack<<<grid_for(c, d.m_slots), 256, 0, s>>>(d.adj.as<uint2>(), d.m_slots, wb, d.adjp.as<uint32_t>());
   CUDA_OK(cudaGetLastError());
   d.adjp_wbits = wb;
+}
+
+// light / heavy split of the packed rows at bucket width delta: each row is
+// stably partitioned into its light edges (w < delta) then its heavy ones
+// (warp per row, ballot ranks), lend[u] = end of the light part.  The order
+// of a row's edges does not change the SSSP fixed point.
+__global__ void k_adj_lh(const uint32_t* __restrict__ rp, const uint32_t* __restrict__ in, uint32_t* __restrict__ out,
+                         uint32_t* __restrict__ lend, int64_t n, uint32_t delta, uint32_t wb) {
+  const unsigned lane = lane_id(), lt = (1u << lane) - 1u;
+  const uint32_t wm = (1u << wb) - 1u;
+  for (int64_t u = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; u < n;
+       u += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+    const uint32_t a = rp[u], b = rp[u + 1];
+    uint32_t nl = 0;
+    for (uint32_t e = a + lane; e - lane < b; e += 32)
+      nl += __popc(__ballot_sync(FULL, e < b && (in[e] & wm) < delta));
+    uint32_t li = a, hi = a + nl;
+    for (uint32_t e = a + lane; e - lane < b; e += 32) {
+      const bool ok = e < b;
+      const uint32_t v = ok ? in[e] : 0u;
+      const bool light = ok && (v & wm) < delta;
+      const unsigned bl = __ballot_sync(FULL, light), bh = __ballot_sync(FULL, ok && !light);
+      if (light) out[li + __popc(bl & lt)] = v;
+      else if (ok) out[hi + __popc(bh & lt)] = v;
+      li += __popc(bl);
+      hi += __popc(bh);
+    }
+    if (lane == 0) lend[u] = a + nl;
+  }
+}
+
+static void ensure_lh(gx_graph* g, uint32_t delta) {
+  DevGraph& d = g->dg;
+  if (d.lh_lend.p && d.lh_delta == delta) return;
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  DBuf out;
+  out.alloc(c, sizeof(uint32_t) * d.m_slots);
+  if (!d.lh_lend.p) d.lh_lend.alloc(c, sizeof(uint32_t) * std::max<int64_t>(1, d.n_slots));
+  k_adj_lh<<<c->num_sms * 8, 256, 0, s>>>(d.rp.as<uint32_t>(), d.adjp.as<uint32_t>(), out.as<uint32_t>(),
+                                          d.lh_lend.as<uint32_t>(), d.n_slots, delta, d.adjp_wbits);
+  CUDA_OK(cudaGetLastError());
+  CUDA_OK(cudaStreamSynchronize(s));
+  d.adjp = std::move(out);
+  d.lh_delta = delta;
 }
 
 static void ensure_heavy_chunks(gx_graph* g) {
@@ -1184,7 +1267,7 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
   const int64_t ns = d.n_slots;
   const int64_t nwords = (ns + 31) / 32;
   r.dist.alloc(c, sizeof(uint32_t) * ns);
-  r.mark.alloc(c, sizeof(uint32_t) * 4 * nwords);   // frontier bitmaps bm[0..2] + far pile
+  r.mark.alloc(c, sizeof(uint32_t) * 6 * nwords);   // frontier bitmaps bm[0..2] + far pile + pend[0..1]
   r.st.alloc(c, sizeof(SsspState));
   SsspState* st = r.st.as<SsspState>();
   SsspAux ax{};
@@ -1214,12 +1297,33 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
   dsrc.alloc(c, sizeof(int32_t) * srcs.size());
   CUDA_OK(cudaMemcpyAsync(dsrc.p, srcs.data(), sizeof(int32_t) * srcs.size(), cudaMemcpyHostToDevice, s));
 
+  // light / heavy split (persistent LB loop, exact mode on packed rows: no §3
+  // tiles or §2 merges, which move distances outside the sweeps); the layout
+  // is built once per bucket width, outside the timed region.  Off unless
+  // GX_SSSP_LH=1: measured on RMAT-24 it relaxes 374M edges instead of 451M but
+  // takes 72 iterations instead of 57 and 5.33 ms instead of 5.10 (Delta 12-100
+  // all slower than the default without it; profiles/r1e/lh_sweep.txt)
+  unsigned hst_delta = mapping == GX_MAP_LB ? sssp_delta(g) : 0u;
+  if (const char* e = getenv("GX_SSSP_DELTA")) hst_delta = (unsigned)std::max(0, atoi(e));
+  bool want_lh = false;
+  {
+    const char* lhe = getenv("GX_SSSP_LH");
+    const char* pe0 = getenv("GX_SSSP_PERSIST");
+    const char* be0 = getenv("GX_SSSP_BLOCK");
+    want_lh = mapping == GX_MAP_LB && ax.adjp && hst_delta > 0 && !(d.n_tiles && g->knobs.smem) && !d.n_groups &&
+              (lhe && atoi(lhe) != 0) && !(pe0 && atoi(pe0) == 0) && !(be0 && atoi(be0) != 0) &&
+              !(o.profile && getenv("GX_SSSP_TRACE"));
+    if (want_lh) {
+      ensure_lh(g, hst_delta);
+      ax.adjp = d.adjp.as<uint32_t>();   // the partitioned copy replaced the buffer
+    }
+  }
   cudaEvent_t e0, e1;
   CUDA_OK(cudaEventCreate(&e0));
   CUDA_OK(cudaEventCreate(&e1));
   CUDA_OK(cudaEventRecord(e0, s));
   CUDA_OK(cudaMemsetAsync(r.dist.p, 0xFF, sizeof(uint32_t) * ns, s));
-  CUDA_OK(cudaMemsetAsync(r.mark.p, 0, sizeof(uint32_t) * 4 * nwords, s));
+  CUDA_OK(cudaMemsetAsync(r.mark.p, 0, sizeof(uint32_t) * 6 * nwords, s));
   {
     // near-far bucket width (LB mapping only; 0 = plain frontier Bellman-Ford)
     static SsspState init;
@@ -1368,6 +1472,11 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
       // each local round still pays an L2 round trip per hop)
       const bool want = be ? atoi(be) != 0 && d.blk_maxdeg <= 64 : false;
       if (want) L.block_rows = B;
+    }
+    if (want_lh && L.block_rows == 0) {
+      L.ax.lend = d.lh_lend.as<uint32_t>();
+      L.ax.pend[0] = r.mark.as<uint32_t>() + 4 * nwords;
+      L.ax.pend[1] = r.mark.as<uint32_t>() + 5 * nwords;
     }
     void* args[] = {&L};
     kt.begin();

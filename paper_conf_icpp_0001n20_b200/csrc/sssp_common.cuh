@@ -42,6 +42,13 @@ struct SsspAux {
   // one u32 when n' <= 2^(32 - wbits) -- 4 bytes per relaxed edge instead of 8
   const uint32_t* adjp;
   uint32_t wbits;
+  // light / heavy edge split (delta-stepping's edge classes; null: off):
+  // row u's edges [rp[u], lend[u]) have w < delta, [lend[u], rp[u+1]) w >= delta.
+  // A light pass relaxes the light edges of the frontier and records it in
+  // pend[p]; a heavy pass relaxes the heavy edges of pend[p] once the bucket
+  // drained (a heavy edge from the bucket cannot land below tau, sssp.cu)
+  const uint32_t* lend;
+  uint32_t* pend[2];
 };
 // the out-edge e as {dst, w}
 __device__ __forceinline__ uint2 ld_edge(const uint2* __restrict__ adj, const SsspAux& ax, uint32_t e, uint64_t pol) {

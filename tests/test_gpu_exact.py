@@ -233,6 +233,26 @@ def test_sssp_loop_modes_bit_exact(name, persist, block, monkeypatch):
     assert np.array_equal(got, want), f"{np.sum(got != want)} mismatches"
 
 
+@pytest.mark.parametrize("name", ["rmat12", "uniform", "road64", "star_hub", "dups_loops", "isolated"])
+@pytest.mark.parametrize("delta", [None, "1", "7", "40", "1000"])
+def test_sssp_light_heavy_split_bit_exact(name, delta, monkeypatch):
+    """The persistent loop with the light / heavy edge split (GX_SSSP_LH=1:
+    rows partitioned at the bucket width, heavy edges of a bucket relaxed once
+    when it drains) reaches Dijkstra exactly at any bucket width."""
+    monkeypatch.setenv("GX_SSSP_LH", "1")
+    if delta is not None:
+        monkeypatch.setenv("GX_SSSP_DELTA", delta)
+    raw = GRAPHS[name]()
+    g = from_raw(raw)
+    want = A.sssp_dijkstra(graph_to_edgelist(g), sssp_source(g))
+    G = upload(raw)
+    for _ in range(2):   # the second run reuses the partitioned rows
+        info = G.run("sssp", source=-1, mapping="lb")
+        assert info["converged"] == 1
+        got = G.download("dist")
+        assert np.array_equal(got, want), f"{np.sum(got != want)} mismatches"
+
+
 def test_sssp_block_mode_road_grid_closed_form(monkeypatch):
     """Block-local mode on a full 4-neighbour grid with unit weights: the
     distances are the Manhattan distances (closed form)."""
