@@ -388,7 +388,11 @@ constexpr int PB_CPT = GX_PB_CPT;     // (1): ring chunks consumed per turn (4 t
 #ifndef GX_PB_SEGU
 #define GX_PB_SEGU 2    // measured: 1: 824, 2: 818, 4: 863, 8: 942 us per sweep (RMAT-24)
 #endif
-constexpr int PB_SEGU = GX_PB_SEGU;   // (3): segments in flight per warp step (16-byte load each per lane)
+constexpr int PB_SEGU = GX_PB_SEGU;
+#ifndef GX_PB_PFA
+#define GX_PB_PFA 0    // measured: 0: 773, 4: 801, 8: 813, 16: 848, 32: 876 us per sweep (profiles/r1e)
+#endif
+constexpr int PB_PFA = GX_PB_PFA;     // (1): L2 prefetch distance of the bin stream, in chunks (0: off)   // (3): segments in flight per warp step (16-byte load each per lane)
 // dynamic smem: acc_lo u32[R] (reused as the f32 terms s_c after the update)
 // | 8 zero words (s_c[R..R+7], the padding entries' source) | acc_hi u32[R] | ring
 constexpr size_t PB_RING_OFF = (size_t)PB_R * 8 + 32;
@@ -589,7 +593,14 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
     }
     if (PB_PRODUCER && threadIdx.x >= PB_CONSUMERS) {
       if (threadIdx.x == PB_CONSUMERS)
-        for (uint32_t c = 0; c < nch; c++) issue(g + c, E0, E1, c);
+        for (uint32_t c = 0; c < nch; c++) {
+          if (PB_PFA && c + PB_PFA < nch) {   // chunk c + PFA into L2 ahead of its bulk copy
+            const uint32_t e = E0 + (c + PB_PFA) * PB_CH, n = min((uint32_t)PB_CH, E1 - e);
+            l2_prefetch_bulk(p.val + e, n * 4u);
+            l2_prefetch_bulk(p.dst_loc + e, n * 2u);
+          }
+          issue(g + c, E0, E1, c);
+        }
     } else
     for (uint32_t c = 0; c < nch; c += PB_CPT) {
       constexpr int G4 = PB_EPT / 4;

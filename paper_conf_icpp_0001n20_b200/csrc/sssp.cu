@@ -116,7 +116,17 @@ __device__ __forceinline__ void clear_bitmap(uint32_t* bm, int64_t nwords) {
 }
 
 // ---------------------------------------------------------------- LB sweep
-constexpr int SU = 4;         // edges in flight per lane per round
+// measured (RMAT-24 exact, persistent loop, profiles/r1e/sssp_hint_variants.txt):
+// row_ptr loads with L2 evict_first (the gathered dist keeps the L2) and 3
+// edges in flight per lane: 5.04 -> 4.78 ms; SU 8: 5.8 ms; 5-6 CTAs/SM
+// (__launch_bounds__ min blocks, spills): 5.9-9.8 ms
+#ifndef GX_SSSP_RP_EF
+#define GX_SSSP_RP_EF 1
+#endif
+#ifndef GX_SSSP_SU
+#define GX_SSSP_SU 3
+#endif
+constexpr int SU = GX_SSSP_SU;   // edges in flight per lane per round
 constexpr int SB_WARPS = 8;   // warps per CTA
 
 // iteration t with near-far threshold tau; the far pile's minimum goes to fdst
@@ -238,8 +248,13 @@ __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, con
       if (mine) {
         const int32_t u = sv[idx];
         du = ld_l2_u32(dist + u, pl);
+#if GX_SSSP_RP_EF
+        start = ld_l2_u32(rp + u, pf);   // keep the L2 for the gathered dist
+        uint32_t end = ld_l2_u32(rp + u + 1, pf);
+#else
         start = rp[u];
         uint32_t end = rp[u + 1];
+#endif
         if (lh == 1) end = ax.lend[u];
         else if (lh == 2) start = ax.lend[u];
         deg = end - start;
@@ -750,7 +765,10 @@ struct SsspLoop {
 constexpr int PERSIST_POOL = SB_WARPS * 1024 * 4;   // 32 KB: LB compaction buffer / block-mode queues
 static_assert(2 * BLK_Q * 4 + BLK_MAX / 8 + 16 <= PERSIST_POOL, "block-mode buffers must fit the pool");
 
-__global__ void __launch_bounds__(256, 4) k_sssp_persist(SsspLoop a) {
+#ifndef GX_SSSP_MINB
+#define GX_SSSP_MINB 4
+#endif
+__global__ void __launch_bounds__(256, GX_SSSP_MINB) k_sssp_persist(SsspLoop a) {
   __shared__ __align__(16) uint8_t pool[PERSIST_POOL];
   cg::grid_group grid = cg::this_grid();
   const bool lead = blockIdx.x == 0 && threadIdx.x == 0;
