@@ -83,6 +83,8 @@ typedef enum { GX_MAP_AUTO = 0, GX_MAP_LB = 1, GX_MAP_TPV = 2, GX_MAP_PB = 3, GX
 #define GX_PTRS_DEVICE 1u     /* pointers are device memory of the ctx device    */
 #define GX_VALIDATE 2u        /* check monotone row_ptr, col range, weights >= 1 */
 #define GX_CANONICAL 4u       /* caller asserts: no self-loops, no duplicates    */
+#define GX_ASYNC_UPLOAD 8u    /* with GX_CANONICAL and host pointers, no GX_VALIDATE:
+                                 the weights are copied on a second stream; see below */
 
 /* download kinds */
 #define GX_OUT_DIST_U32 1        /* SSSP distance, 0xFFFFFFFF = unreachable [n]  */
@@ -240,6 +242,14 @@ gx_status gx_ctx_stream(gx_ctx* ctx, void** stream_out);
  * weights w (NULL => all 1; must be >= 1).  Canonicalised (reading R2): self-
  * loops dropped, a duplicate (u,v) merged into its first occurrence keeping
  * the minimum weight, row order otherwise kept -- unless GX_CANONICAL.
+ * GX_ASYNC_UPLOAD (with GX_CANONICAL, host pointers, w != NULL, no GX_VALIDATE;
+ * ignored otherwise): the call returns once row_ptr and col are queued; w is
+ * copied on a second stream behind col, so a following exact-mode PageRank on
+ * the blocked mapping (which needs only the structure) overlaps its transfer.
+ * The caller keeps row_ptr / col / w valid and unchanged until a call that
+ * joins the copy: gx_run of any other algorithm or mapping, gx_transform,
+ * gx_export_*, gx_sync or gx_graph_destroy.  Pinned host memory is needed for
+ * the copies to overlap anything.
  * Errors: GX_E_INVALID (n < 0, m < 0, with GX_VALIDATE: non-monotone row_ptr,
  * col out of [0,n), w = 0), GX_E_UNSUPPORTED (m >= 2^32 or n >= 2^31). */
 gx_status gx_graph_upload_csr(gx_ctx* ctx, gx_graph** out, int64_t n, int64_t m,

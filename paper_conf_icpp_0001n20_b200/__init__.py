@@ -17,7 +17,7 @@ from dataclasses import dataclass, fields
 
 import numpy as np
 
-from ._binding import (ALGOS, ALLOC_FN, GX_CANONICAL, GX_MAP_AUTO, GX_MAP_LB, GX_MAP_PB, GX_MAP_TPV, GX_MAP_VNS, GX_OUT_BC_F64,
+from ._binding import (ALGOS, ALLOC_FN, GX_ASYNC_UPLOAD, GX_CANONICAL, GX_MAP_AUTO, GX_MAP_LB, GX_MAP_PB, GX_MAP_TPV, GX_MAP_VNS, GX_OUT_BC_F64,
                        GX_OUT_DIST_U32, GX_OUT_LABEL_I32, GX_OUT_MST_WEIGHT_U64, GX_OUT_RANK_F64,
                        GX_PTRS_DEVICE, GX_PTRS_HOST, GX_VALIDATE, RELEASE_FN, GraffixError, GxExport,
                        GxExportSizes, GxKnobs, GxRunInfo, GxRunOpts, GxTransformInfo, _check, _ptr, lib)
@@ -155,8 +155,11 @@ class Graph:
         self.last_run: dict | None = None
 
     @classmethod
-    def upload(cls, ctx: Context, row_ptr, col, w=None, validate: bool = False, canonical: bool = False):
-        """Upload a CSR graph.  numpy arrays => host pointers; torch CUDA tensors => device."""
+    def upload(cls, ctx: Context, row_ptr, col, w=None, validate: bool = False, canonical: bool = False,
+               async_upload: bool = False):
+        """Upload a CSR graph.  numpy arrays => host pointers; torch CUDA tensors => device.
+        async_upload (GX_ASYNC_UPLOAD, with canonical host arrays): the weights are copied on a
+        second stream; the arrays are kept referenced by the Graph until it is closed."""
         dev = hasattr(row_ptr, "is_cuda") and row_ptr.is_cuda
         if not dev:
             row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
@@ -165,10 +168,13 @@ class Graph:
         n = int(row_ptr.shape[0]) - 1
         m = int(col.shape[0])
         flags = (GX_PTRS_DEVICE if dev else GX_PTRS_HOST) | (GX_VALIDATE if validate else 0) | \
-            (GX_CANONICAL if canonical else 0)
+            (GX_CANONICAL if canonical else 0) | (GX_ASYNC_UPLOAD if async_upload else 0)
         h = C.c_void_p()
         _check(lib().gx_graph_upload_csr(ctx._h, C.byref(h), n, m, _ptr(row_ptr), _ptr(col), _ptr(w), flags))
-        return cls(ctx, h)
+        G = cls(ctx, h)
+        if async_upload:
+            G._keep = (row_ptr, col, w)   # read by the copy until a joining call (include/graffix.h)
+        return G
 
     @classmethod
     def host_only(cls, row_ptr, col, w=None, validate: bool = False):

@@ -60,7 +60,7 @@ void DBuf::alloc(Ctx* c, size_t b) {
 
 // upload helpers implemented in devgraph.cu
 void device_upload_input(gx_graph* g, const int64_t* rp, const int32_t* col, const uint32_t* w,
-                         bool device_ptrs, bool validate);
+                         bool device_ptrs, bool validate, bool async = false);
 
 }  // namespace gx
 
@@ -155,12 +155,17 @@ void gx_ctx_destroy(gx_ctx* ctx) {
   if (ctx->stream) cudaStreamSynchronize(ctx->stream);
   if (ctx->nccl) gx_comm_destroy(ctx->nccl);
   if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
+  if (ctx->copy_stream) {
+    cudaStreamSynchronize(ctx->copy_stream);
+    cudaStreamDestroy(ctx->copy_stream);
+  }
   delete ctx;
 }
 
 gx_status gx_sync(gx_ctx* ctx) {
   GX_API_BEGIN
   GX_CHECK_ARG(ctx, "ctx is NULL");
+  if (ctx->copy_stream) CUDA_OK(cudaStreamSynchronize(ctx->copy_stream));
   CUDA_OK(cudaStreamSynchronize(ctx->stream));
   GX_API_END
 }
@@ -186,7 +191,7 @@ gx_status gx_graph_upload_csr(gx_ctx* ctx, gx_graph** out, int64_t n, int64_t m,
     if (flags & GX_CANONICAL) {
       g->n = n;
       g->m = m;
-      device_upload_input(g, row_ptr, col, w, dev, validate);
+      device_upload_input(g, row_ptr, col, w, dev, validate, (flags & GX_ASYNC_UPLOAD) != 0);
     } else {
       // canonicalise on the host (reading R2); device inputs come back first
       std::vector<int64_t> hrp;
@@ -235,6 +240,13 @@ gx_status gx_graph_upload_csr(gx_ctx* ctx, gx_graph** out, int64_t n, int64_t m,
 void gx_graph_destroy(gx_graph* g) {
   if (!g) return;
   if (g->ctx) cudaSetDevice(g->ctx->device);
+  if (g->pend_ev) {   // an asynchronous upload still reading host memory / writing its buffers
+    cudaEventSynchronize(g->pend_ev);
+    try {
+      resolve_pending(g);
+    } catch (...) {
+    }
+  }
   delete g;  // DBuf destructors release device memory on the ctx stream
 }
 
@@ -328,6 +340,7 @@ static void check_knobs(const gx_knobs& k) {
 gx_status gx_transform(gx_graph* g, const gx_knobs* knobs, gx_transform_info* info) {
   GX_API_BEGIN
   GX_CHECK_ARG(g, "graph is NULL");
+  resolve_pending(g);
   gx_knobs k;
   gx_knobs_default(&k);
   if (knobs) k = *knobs;
@@ -361,6 +374,7 @@ gx_status gx_transform(gx_graph* g, const gx_knobs* knobs, gx_transform_info* in
 gx_status gx_export_sizes(gx_graph* g, gx_export_sizes_t* s) {
   GX_API_BEGIN
   GX_CHECK_ARG(g && s, "NULL argument");
+  resolve_pending(g);
   if (!g->transformed) {
     ensure_host(g);
     s->n_slots = g->n;
@@ -382,6 +396,7 @@ gx_status gx_export_sizes(gx_graph* g, gx_export_sizes_t* s) {
 gx_status gx_export_transformed(gx_graph* g, gx_export_t* o) {
   GX_API_BEGIN
   GX_CHECK_ARG(g && o, "NULL argument");
+  resolve_pending(g);
   if (!g->transformed) {
     // exact mode: identity slots; rows sorted by destination (R11)
     ensure_host(g);
@@ -444,6 +459,9 @@ gx_status gx_run_ex(gx_graph* g, const gx_run_opts* opts, gx_run_info* info) {
   GX_CHECK_ARG(o.merge_every >= 0, "merge_every must be >= 0");
   gx_run_info ri;
   std::memset(&ri, 0, sizeof(ri));
+  // an asynchronous upload's weights are joined here, except for PageRank,
+  // which joins them itself unless it runs the blocked pull (structure only)
+  if (o.algo != GX_PAGERANK) resolve_pending(g);
   switch (o.algo) {
     case GX_SSSP: run_sssp(g, o, ri); break;
     case GX_PAGERANK:

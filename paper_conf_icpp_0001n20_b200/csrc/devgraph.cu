@@ -79,7 +79,7 @@ __global__ void k_csc_pairs(const uint32_t* __restrict__ rp, const uint2* __rest
 // ------------------------------------------------------------------ host side
 
 void device_upload_input(gx_graph* g, const int64_t* rp, const int32_t* col, const uint32_t* w,
-                         bool device_ptrs, bool validate) {
+                         bool device_ptrs, bool validate, bool async) {
   Ctx* c = g->ctx;
   cudaStream_t s = c->stream;
   int64_t n = g->n, m = g->m;
@@ -87,6 +87,27 @@ void device_upload_input(gx_graph* g, const int64_t* rp, const int32_t* col, con
   g->in_col.alloc(c, sizeof(int32_t) * std::max<int64_t>(m, 1));
   g->in_w.alloc(c, sizeof(uint32_t) * std::max<int64_t>(m, 1));
   cudaMemcpyKind kind = device_ptrs ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
+  if (async && !device_ptrs && !validate && w && m > 0) {
+    // row_ptr and col on the ctx stream; the weights (and their maximum) on
+    // the copy stream once col has landed, so that work needing only the
+    // structure (the blocked PageRank) overlaps their transfer
+    if (!c->copy_stream) CUDA_OK(cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
+    g->maxw_buf.alloc(c, 16);
+    CUDA_OK(cudaMemsetAsync(g->maxw_buf.p, 0, 16, s));
+    CUDA_OK(cudaMemcpyAsync(g->in_rp.p, rp, sizeof(int64_t) * (n + 1), kind, s));
+    CUDA_OK(cudaMemcpyAsync(g->in_col.p, col, sizeof(int32_t) * m, kind, s));
+    cudaEvent_t ev;
+    CUDA_OK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+    CUDA_OK(cudaEventRecord(ev, s));
+    CUDA_OK(cudaStreamWaitEvent(c->copy_stream, ev, 0));
+    CUDA_OK(cudaEventDestroy(ev));
+    CUDA_OK(cudaMemcpyAsync(g->in_w.p, w, sizeof(uint32_t) * m, kind, c->copy_stream));
+    k_max_u32<<<grid_for(c, m), 256, 0, c->copy_stream>>>(g->in_w.as<uint32_t>(), m, g->maxw_buf.as<unsigned int>());
+    CUDA_OK(cudaGetLastError());
+    g->maxw_pending = true;
+    g->max_w = 1;   // until resolve_pending
+    return;
+  }
   CUDA_OK(cudaMemcpyAsync(g->in_rp.p, rp, sizeof(int64_t) * (n + 1), kind, s));
   if (m) {
     CUDA_OK(cudaMemcpyAsync(g->in_col.p, col, sizeof(int32_t) * m, kind, s));
@@ -159,7 +180,8 @@ static void build_csc_and_tiles(gx_graph* g) {
 // ---- propagation-blocked PR layout (PbLayout, gx_internal.h) ----
 // key = bin(v) * nb + block(u) per out-edge (sink-bin major), payload = the
 // two local indices; histogram of keys for the segment offsets
-__global__ void k_pb_pairs(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj, int64_t n, uint32_t nb,
+__global__ void k_pb_pairs(const uint32_t* __restrict__ rp, const uint32_t* __restrict__ colp, uint32_t cstride,
+                           int64_t n, uint32_t nb,
                            uint32_t* __restrict__ key, uint32_t* __restrict__ val, uint32_t* __restrict__ cnt) {
   int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   int lane = threadIdx.x & 31;
@@ -168,7 +190,7 @@ __global__ void k_pb_pairs(const uint32_t* __restrict__ rp, const uint2* __restr
     const uint32_t a = rp[u], b = rp[u + 1];
     const uint32_t bu = (uint32_t)(u / PB_R), lu = (uint32_t)(u % PB_R);
     for (uint32_t e = a + lane; e < b; e += 32) {
-      const uint32_t v = adj[e].x;
+      const uint32_t v = colp[(size_t)e * cstride];
       const uint32_t k = (v / PB_R) * nb + bu;
       key[e] = k;
       val[e] = lu | ((v % PB_R) << 16);
@@ -228,7 +250,12 @@ void ensure_pb(gx_graph* g) {
     k1.alloc(c, sizeof(uint32_t) * m);
     v0.alloc(c, sizeof(uint32_t) * m);
     v1.alloc(c, sizeof(uint32_t) * m);
-    k_pb_pairs<<<grid_for(c, n * 32), 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), n, (uint32_t)nb,
+    // exact mode reads the uploaded col (not the {col, w} pairs, which an
+    // asynchronous upload may still be producing)
+    const bool ident = d.identity && g->in_col.p;
+    k_pb_pairs<<<grid_for(c, n * 32), 256, 0, s>>>(d.rp.as<uint32_t>(),
+                                                   ident ? g->in_col.as<uint32_t>() : d.adj.as<uint32_t>(),
+                                                   ident ? 1u : 2u, n, (uint32_t)nb,
                                                    k0.as<uint32_t>(), v0.as<uint32_t>(), cnt.as<uint32_t>());
     CUDA_OK(cudaGetLastError());
     int bits = 1;
@@ -269,6 +296,25 @@ void ensure_pb(gx_graph* g) {
   CUDA_OK(cudaStreamSynchronize(s));   // temporaries are freed on return
 }
 
+// join the GX_ASYNC_UPLOAD work into the ctx stream; read the weights' maximum
+void resolve_pending(gx_graph* g) {
+  if (!g->ctx) return;
+  cudaStream_t s = g->ctx->stream;
+  if (g->pend_ev) {
+    CUDA_OK(cudaStreamWaitEvent(s, g->pend_ev, 0));
+    CUDA_OK(cudaEventDestroy(g->pend_ev));
+    g->pend_ev = nullptr;
+  }
+  if (g->maxw_pending) {
+    unsigned int h = 0;
+    CUDA_OK(cudaMemcpyAsync(&h, g->maxw_buf.p, 4, cudaMemcpyDeviceToHost, s));
+    CUDA_OK(cudaStreamSynchronize(s));
+    g->max_w = std::max(1u, h);
+    if (g->dg.identity) g->dg.max_w = g->max_w;
+    g->maxw_pending = false;
+  }
+}
+
 void ensure_csc(gx_graph* g) {
   if (g->dg.crp.p) return;
   build_csc_and_tiles(g);
@@ -288,8 +334,21 @@ void build_device_exact(gx_graph* g) {
   d.rp.alloc(c, sizeof(uint32_t) * (n + 1));
   k_rp64_to_u32<<<grid_for(c, n + 1), 256, 0, s>>>(g->in_rp.as<int64_t>(), d.rp.as<uint32_t>(), n + 1);
   d.adj.alloc(c, sizeof(uint2) * std::max<int64_t>(m, 1));
-  if (m) k_interleave<<<grid_for(c, m), 256, 0, s>>>(g->in_col.as<int32_t>(), g->in_w.as<uint32_t>(),
-                                                     d.adj.as<uint2>(), m);
+  if (g->maxw_pending) {   // GX_ASYNC_UPLOAD: interleave behind the weights' copy
+    cudaEvent_t ev;
+    CUDA_OK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+    CUDA_OK(cudaEventRecord(ev, s));   // d.adj allocated
+    CUDA_OK(cudaStreamWaitEvent(c->copy_stream, ev, 0));
+    CUDA_OK(cudaEventDestroy(ev));
+    k_interleave<<<grid_for(c, m), 256, 0, c->copy_stream>>>(g->in_col.as<int32_t>(), g->in_w.as<uint32_t>(),
+                                                             d.adj.as<uint2>(), m);
+    CUDA_OK(cudaGetLastError());
+    CUDA_OK(cudaEventCreateWithFlags(&g->pend_ev, cudaEventDisableTiming));
+    CUDA_OK(cudaEventRecord(g->pend_ev, c->copy_stream));
+  } else if (m) {
+    k_interleave<<<grid_for(c, m), 256, 0, s>>>(g->in_col.as<int32_t>(), g->in_w.as<uint32_t>(), d.adj.as<uint2>(),
+                                                m);
+  }
   d.D.alloc(c, sizeof(uint32_t) * std::max<int64_t>(n, 1));
   k_outdeg<<<grid_for(c, n), 256, 0, s>>>(d.rp.as<uint32_t>(), d.D.as<uint32_t>(), n);
   CUDA_OK(cudaGetLastError());

@@ -55,6 +55,7 @@ struct DBuf {
 struct Ctx {
   int device = 0;
   cudaStream_t stream = nullptr;
+  cudaStream_t copy_stream = nullptr;   // GX_ASYNC_UPLOAD: weights H2D + {col, w} interleave (lazily created)
   bool own_stream = false;
   gx_alloc_fn alloc = nullptr;
   gx_release_fn release = nullptr;
@@ -203,6 +204,12 @@ struct gx_graph {
   gx::DBuf in_rp, in_col, in_w;   // canonical input on device (original ids)
   int64_t n = 0, m = 0;
   uint32_t max_w = 1;
+  // GX_ASYNC_UPLOAD: the weights' copy, their maximum and the {col, w}
+  // interleave run on ctx->copy_stream; pend_ev marks their end and
+  // gx::resolve_pending() joins them into the ctx stream (and reads max_w)
+  cudaEvent_t pend_ev = nullptr;
+  gx::DBuf maxw_buf;
+  bool maxw_pending = false;
   gx::SlotGraph sg;            // current transform (empty in exact mode)
   bool transformed = false;
   gx_knobs knobs{};
@@ -225,6 +232,7 @@ void gpu_pad_candidates(Ctx* c, int64_t n, const int64_t* lp, const int32_t* ld,
                         const int32_t* qu, const int32_t* qtake, int rule, std::vector<int64_t>& rptr,
                         std::vector<uint64_t>& rkeys);
 void build_device_exact(gx_graph* g);
+void resolve_pending(gx_graph* g);
 void build_device_slots(gx_graph* g);
 void build_tpv(gx_graph* g);
 void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info);

@@ -1148,7 +1148,10 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
                     : (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
   }
   if (mapping == GX_MAP_VNS) mapping = GX_MAP_TPV;   // a pull row is not split (graffix.h)
-  if (P_ranks > 1 || mapping != GX_MAP_PB || tiles) ensure_csc(g);
+  if (P_ranks > 1 || mapping != GX_MAP_PB || tiles) {
+    resolve_pending(g);   // GX_ASYNC_UPLOAD: these layouts read the {col, w} pairs
+    ensure_csc(g);
+  }
   r.x.alloc(c, sizeof(double) * ns);
   r.contrib[0].alloc(c, sizeof(float) * ns);
   const bool sim_ = c->world == 1 && o.sim_ranks > 1;

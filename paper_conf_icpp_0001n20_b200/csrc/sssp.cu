@@ -988,13 +988,17 @@ static void ensure_packed_adj(gx_graph* g) {
   if (getenv("GX_SSSP_NO_PACK") || d.m_slots == 0) return;
   Ctx* c = g->ctx;
   cudaStream_t s = c->stream;
-  DBuf mx;
-  mx.alloc(c, 4);
-  CUDA_OK(cudaMemsetAsync(mx.p, 0, 4, s));
-  k_adj_wmax<<<grid_for(c, d.m_slots), 256, 0, s>>>(d.adj.as<uint2>(), d.m_slots, mx.as<unsigned int>());
   unsigned int wmax = 0;
-  CUDA_OK(cudaMemcpyAsync(&wmax, mx.p, 4, cudaMemcpyDeviceToHost, s));
-  CUDA_OK(cudaStreamSynchronize(s));
+  if (d.identity) {
+    wmax = d.max_w;   // measured at upload
+  } else {
+    DBuf mx;
+    mx.alloc(c, 4);
+    CUDA_OK(cudaMemsetAsync(mx.p, 0, 4, s));
+    k_adj_wmax<<<grid_for(c, d.m_slots), 256, 0, s>>>(d.adj.as<uint2>(), d.m_slots, mx.as<unsigned int>());
+    CUDA_OK(cudaMemcpyAsync(&wmax, mx.p, 4, cudaMemcpyDeviceToHost, s));
+    CUDA_OK(cudaStreamSynchronize(s));
+  }
   uint32_t wb = 1;
   while (wb < 32 && (wmax >> wb)) wb++;
   if (wb >= 16 || d.n_slots > (int64_t(1) << (32 - wb))) return;
@@ -1470,7 +1474,9 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
     const int64_t gridp = (int64_t)occp * c->num_sms;
     const int64_t B = ((ns + gridp - 1) / gridp + 31) / 32 * 32;
     L.block_rows = 0;
-    if (B <= BLK_MAX && d.m_slots > 0) {
+    const char* be = getenv("GX_SSSP_BLOCK");
+    // (the locality count costs ~2 ms on RMAT-24: only when the mode is asked for)
+    if (B <= BLK_MAX && d.m_slots > 0 && be && atoi(be) != 0) {
       if (d.blk_rows != B) {
         DBuf cnt;
         cnt.alloc(c, 16);
@@ -1484,7 +1490,6 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
         d.blk_local = (double)h[0] / (double)d.m_slots;
         d.blk_maxdeg = (int64_t)h[1];
       }
-      const char* be = getenv("GX_SSSP_BLOCK");
       // experimental: off unless GX_SSSP_BLOCK=1 (road 4900^2: 326 ms at the
       // default Delta vs 331 for the LB sweep, but 270 vs 198 at Delta 1000 --
       // each local round still pays an L2 round trip per hop)

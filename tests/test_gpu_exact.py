@@ -272,3 +272,61 @@ def test_sssp_block_mode_road_grid_closed_form(monkeypatch):
     got = G.download("dist").astype(np.int64)
     rr, cc = np.divmod(np.arange(side * side), side)
     assert np.array_equal(got, rr + cc)
+
+
+def _canonical_pinned(raw):
+    """The canonical CSR of raw (a sync upload's export), in pinned host memory."""
+    import torch
+    ex = upload(raw).export()
+    return (torch.from_numpy(ex["row_ptr"]).pin_memory(), torch.from_numpy(ex["col"]).pin_memory(),
+            torch.from_numpy(ex["w"].view(np.int32)).pin_memory())
+
+
+@pytest.mark.parametrize("name", ["rmat12", "rmat14_C1", "uniform", "road64", "star_hub", "dups_loops"])
+@pytest.mark.parametrize("order", ["pr_first", "sssp_first"])
+def test_async_upload_parity(name, order):
+    """GX_ASYNC_UPLOAD (weights copied on a second stream; the blocked PageRank
+    runs on the structure while they land): SSSP bit-exact against Dijkstra and
+    PageRank within L1 1e-6 of the oracle, in either call order."""
+    import paper_conf_icpp_0001n20_b200 as gx
+    raw = GRAPHS[name]()
+    g = from_raw(raw)
+    el = graph_to_edgelist(g)
+    want_d = A.sssp_dijkstra(el, sssp_source(g))
+    want_x, _ = A.pagerank(el, tol=1e-14)
+    rp, col, w = _canonical_pinned(raw)
+    G = gx.Graph.upload(ctx(), rp.numpy(), col.numpy(), w.numpy().view(np.uint32), canonical=True,
+                        async_upload=True)
+    steps = ["pr", "sssp"] if order == "pr_first" else ["sssp", "pr"]
+    for st in steps:
+        if st == "pr":
+            G.run("pagerank", tol=1e-10, max_iters=5000, mapping="pb")
+            x = G.download("rank")
+        else:
+            info = G.run("sssp", source=-1, mapping="lb")
+            assert info["converged"] == 1
+            d = G.download("dist")
+    assert np.array_equal(d, want_d), f"{np.sum(d != want_d)} mismatches"
+    assert float(np.abs(x - want_x).sum()) <= 1e-6
+    G.close()
+
+
+def test_async_upload_close_transform_export():
+    """An asynchronous upload closed at once, or followed by a transform or an
+    export, joins the weights' copy first (no stale weights, no freed buffers)."""
+    import paper_conf_icpp_0001n20_b200 as gx
+    raw = GRAPHS["rmat12"]()
+    g = from_raw(raw)
+    rp, col, w = _canonical_pinned(raw)
+    args = (rp.numpy(), col.numpy(), w.numpy().view(np.uint32))
+    for _ in range(3):
+        gx.Graph.upload(ctx(), *args, canonical=True, async_upload=True).close()
+    G = gx.Graph.upload(ctx(), *args, canonical=True, async_upload=True)
+    ex = G.export()
+    assert np.array_equal(ex["w"].view(np.uint32), w.numpy().view(np.uint32))
+    G.close()
+    G = gx.Graph.upload(ctx(), *args, canonical=True, async_upload=True)
+    G.transform(gx.Knobs(coalesce=True))
+    G.run("sssp", source=-1)
+    assert np.array_equal(G.download("dist"), A.sssp_dijkstra(graph_to_edgelist(g), sssp_source(g)))
+    G.close()
