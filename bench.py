@@ -296,9 +296,10 @@ def main():
             G2 = gx.Graph.upload(ctx, hrp.numpy(), hcol.numpy(), hw.numpy().view(np.uint32), canonical=True,
                                  async_upload=not args.e2e_sync)
             b = G2.run("pagerank", tol=1e-9, mapping=args.pr_mapping)
-            G2.download("rank", out=hrank.numpy())
+            G2.download("rank", out=hrank.numpy(), async_copy=not args.e2e_sync)   # D2H overlaps SSSP
             a = G2.run("sssp", source=-1, mapping="lb")
             G2.download("dist", out=hdist.numpy().view(np.uint32))
+            ctx.sync()
             e1.record(stream)
             torch.cuda.synchronize()
             G2.close()
@@ -312,7 +313,7 @@ def main():
             t = float(tt.item())
         e2e = {"value": e2e_edges / (t * 1e-3) / 1e9, "unit": UNIT, "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": d2h, "ms_per_step": t / len(e2e_ms),
-               "note": "upload of canonical pinned CSR (GX_CANONICAL" + ("" if args.e2e_sync else " | GX_ASYNC_UPLOAD: weights H2D overlapping the blocked PR") + ") + device layouts (blocked-PR segments, SSSP heavy chunks) + PR + download rank + SSSP + download dist"}
+               "note": "upload of canonical pinned CSR (GX_CANONICAL" + ("" if args.e2e_sync else " | GX_ASYNC_UPLOAD: weights H2D overlapping the blocked PR; rank D2H (GX_DL_ASYNC) overlapping SSSP") + ") + device layouts (blocked-PR segments, SSSP heavy chunks) + PR + download rank + SSSP + download dist"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

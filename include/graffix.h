@@ -83,6 +83,7 @@ typedef enum { GX_MAP_AUTO = 0, GX_MAP_LB = 1, GX_MAP_TPV = 2, GX_MAP_PB = 3, GX
 #define GX_PTRS_DEVICE 1u     /* pointers are device memory of the ctx device    */
 #define GX_VALIDATE 2u        /* check monotone row_ptr, col range, weights >= 1 */
 #define GX_CANONICAL 4u       /* caller asserts: no self-loops, no duplicates    */
+#define GX_DL_ASYNC 16u       /* gx_download: see there                          */
 #define GX_ASYNC_UPLOAD 8u    /* with GX_CANONICAL and host pointers, no GX_VALIDATE:
                                  the weights are copied on a second stream; see below */
 
@@ -289,6 +290,12 @@ gx_status gx_run_opts_default(gx_run_opts* o);
 
 /* Copy a result (indexed by ORIGINAL vertex id; owner slots after the final
  * merge) into `out` (host or device per flags).  count = n, or 1 for MST.
+ * GX_DL_ASYNC (distances / ranks of an untransformed graph into host memory;
+ * ignored otherwise): the copy is queued on a second stream behind the run
+ * that produced the result and the call returns at once, so a following run
+ * of another algorithm overlaps it.  `out` is complete after gx_sync, and is
+ * also waited for by the next run that overwrites that result, by gx_transform
+ * and by gx_graph_destroy; do not read it before.  Pinned memory for overlap.
  * Errors: GX_E_STATE (that algorithm has not run), GX_E_INVALID (count). */
 gx_status gx_download(gx_graph* g, int32_t kind, void* out, int64_t count, uint32_t flags);
 

@@ -17,7 +17,7 @@ from dataclasses import dataclass, fields
 
 import numpy as np
 
-from ._binding import (ALGOS, ALLOC_FN, GX_ASYNC_UPLOAD, GX_CANONICAL, GX_MAP_AUTO, GX_MAP_LB, GX_MAP_PB, GX_MAP_TPV, GX_MAP_VNS, GX_OUT_BC_F64,
+from ._binding import (ALGOS, ALLOC_FN, GX_ASYNC_UPLOAD, GX_CANONICAL, GX_DL_ASYNC, GX_MAP_AUTO, GX_MAP_LB, GX_MAP_PB, GX_MAP_TPV, GX_MAP_VNS, GX_OUT_BC_F64,
                        GX_OUT_DIST_U32, GX_OUT_LABEL_I32, GX_OUT_MST_WEIGHT_U64, GX_OUT_RANK_F64,
                        GX_PTRS_DEVICE, GX_PTRS_HOST, GX_VALIDATE, RELEASE_FN, GraffixError, GxExport,
                        GxExportSizes, GxKnobs, GxRunInfo, GxRunOpts, GxTransformInfo, _check, _ptr, lib)
@@ -226,15 +226,17 @@ class Graph:
               "label": (GX_OUT_LABEL_I32, np.int32), "bc": (GX_OUT_BC_F64, np.float64),
               "mst_weight": (GX_OUT_MST_WEIGHT_U64, np.uint64)}
 
-    def download(self, kind: str, out=None):
+    def download(self, kind: str, out=None, async_copy: bool = False):
         """Result by original vertex id.  ``out`` may be a numpy array (pinned or
-        pageable host memory) or a torch CUDA tensor (device copy)."""
+        pageable host memory) or a torch CUDA tensor (device copy).  async_copy
+        (GX_DL_ASYNC, host ``out``): complete only after ``ctx.sync()``."""
         k, dt = self._KINDS[kind]
         count = 1 if kind == "mst_weight" else self.n
         dev = out is not None and hasattr(out, "is_cuda") and out.is_cuda
         if out is None:
             out = np.empty(count, dtype=dt)
-        _check(lib().gx_download(self._h, k, _ptr(out), count, GX_PTRS_DEVICE if dev else GX_PTRS_HOST))
+        flags = (GX_PTRS_DEVICE if dev else GX_PTRS_HOST) | (GX_DL_ASYNC if async_copy else 0)
+        _check(lib().gx_download(self._h, k, _ptr(out), count, flags))
         if kind == "mst_weight" and not dev:
             return int(out[0])
         return out

@@ -240,6 +240,12 @@ gx_status gx_graph_upload_csr(gx_ctx* ctx, gx_graph** out, int64_t n, int64_t m,
 void gx_graph_destroy(gx_graph* g) {
   if (!g) return;
   if (g->ctx) cudaSetDevice(g->ctx->device);
+  for (int k = 0; k < 8; k++)
+    if (g->dl_ev[k]) {   // an asynchronous download still writing host memory
+      cudaEventSynchronize(g->dl_ev[k]);
+      cudaEventDestroy(g->dl_ev[k]);
+      g->dl_ev[k] = nullptr;
+    }
   if (g->pend_ev) {   // an asynchronous upload still reading host memory / writing its buffers
     cudaEventSynchronize(g->pend_ev);
     try {
@@ -341,6 +347,7 @@ gx_status gx_transform(gx_graph* g, const gx_knobs* knobs, gx_transform_info* in
   GX_API_BEGIN
   GX_CHECK_ARG(g, "graph is NULL");
   resolve_pending(g);
+  join_download(g, -1);
   gx_knobs k;
   gx_knobs_default(&k);
   if (knobs) k = *knobs;
@@ -462,6 +469,9 @@ gx_status gx_run_ex(gx_graph* g, const gx_run_opts* opts, gx_run_info* info) {
   // an asynchronous upload's weights are joined here, except for PageRank,
   // which joins them itself unless it runs the blocked pull (structure only)
   if (o.algo != GX_PAGERANK) resolve_pending(g);
+  // results this run overwrites: wait for their asynchronous downloads
+  if (o.algo == GX_SSSP) join_download(g, GX_OUT_DIST_U32);
+  else if (o.algo == GX_PAGERANK) join_download(g, GX_OUT_RANK_F64);
   switch (o.algo) {
     case GX_SSSP: run_sssp(g, o, ri); break;
     case GX_PAGERANK:

@@ -208,6 +208,7 @@ struct gx_graph {
   // interleave run on ctx->copy_stream; pend_ev marks their end and
   // gx::resolve_pending() joins them into the ctx stream (and reads max_w)
   cudaEvent_t pend_ev = nullptr;
+  cudaEvent_t dl_ev[8] = {};   // GX_DL_ASYNC: end of the download of result kind k (on ctx->copy_stream)
   gx::DBuf maxw_buf;
   bool maxw_pending = false;
   gx::SlotGraph sg;            // current transform (empty in exact mode)
@@ -233,6 +234,7 @@ void gpu_pad_candidates(Ctx* c, int64_t n, const int64_t* lp, const int32_t* ld,
                         std::vector<uint64_t>& rkeys);
 void build_device_exact(gx_graph* g);
 void resolve_pending(gx_graph* g);
+void join_download(gx_graph* g, int kind);   // kind < 0: every kind
 void build_device_slots(gx_graph* g);
 void build_tpv(gx_graph* g);
 void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info);

@@ -44,11 +44,26 @@ void launch_iota_i32(Ctx* c, int32_t* a, int64_t n) {
 // Results are read from owner slots (SURVEY.md §8(b) ownership; holes and
 // replicas are never exposed), indexed by original vertex id.
 template <class T>
-static void gather_out(gx_graph* g, const DBuf& src, void* out, int64_t n, uint32_t flags) {
+static void gather_out(gx_graph* g, const DBuf& src, void* out, int64_t n, uint32_t flags, int kind) {
   Ctx* c = g->ctx;
   cudaStream_t s = c->stream;
   bool dev = flags & GX_PTRS_DEVICE;
   const T* sp = src.as<T>();
+  join_download(g, kind);   // a previous asynchronous download of this kind
+  if (g->dg.identity && !dev && (flags & GX_DL_ASYNC)) {
+    // the copy on the second stream after the producing work; the ctx stream
+    // goes on (join_download / gx_sync / destroy complete it)
+    if (!c->copy_stream) CUDA_OK(cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
+    cudaEvent_t ev;
+    CUDA_OK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+    CUDA_OK(cudaEventRecord(ev, s));
+    CUDA_OK(cudaStreamWaitEvent(c->copy_stream, ev, 0));
+    CUDA_OK(cudaEventDestroy(ev));
+    CUDA_OK(cudaMemcpyAsync(out, sp, sizeof(T) * n, cudaMemcpyDeviceToHost, c->copy_stream));
+    CUDA_OK(cudaEventCreateWithFlags(&g->dl_ev[kind], cudaEventDisableTiming));
+    CUDA_OK(cudaEventRecord(g->dl_ev[kind], c->copy_stream));
+    return;
+  }
   if (g->dg.identity) {
     CUDA_OK(cudaMemcpyAsync(out, sp, sizeof(T) * n, dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, s));
   } else {
@@ -66,18 +81,29 @@ static void gather_out(gx_graph* g, const DBuf& src, void* out, int64_t n, uint3
   CUDA_OK(cudaStreamSynchronize(s));
 }
 
+// the ctx stream waits for the asynchronous download(s) of `kind` (-1: all)
+// before it may overwrite or free their source buffers
+void join_download(gx_graph* g, int kind) {
+  for (int k = 0; k < 8; k++) {
+    if ((kind >= 0 && k != kind) || !g->dl_ev[k]) continue;
+    CUDA_OK(cudaStreamWaitEvent(g->ctx->stream, g->dl_ev[k], 0));
+    CUDA_OK(cudaEventDestroy(g->dl_ev[k]));
+    g->dl_ev[k] = nullptr;
+  }
+}
+
 void download(gx_graph* g, int kind, void* out, int64_t count, uint32_t flags) {
   RunState& r = g->rs;
   switch (kind) {
     case GX_OUT_DIST_U32:
       if (!r.have[GX_SSSP]) GX_THROW(GX_E_STATE, "SSSP has not run on this graph");
       GX_CHECK_ARG(count == g->n, "count must be n");
-      gather_out<uint32_t>(g, r.dist, out, count, flags);
+      gather_out<uint32_t>(g, r.dist, out, count, flags, kind);
       break;
     case GX_OUT_RANK_F64:
       if (!r.have[GX_PAGERANK]) GX_THROW(GX_E_STATE, "PageRank has not run on this graph");
       GX_CHECK_ARG(count == g->n, "count must be n");
-      gather_out<double>(g, r.x, out, count, flags);
+      gather_out<double>(g, r.x, out, count, flags, kind);
       break;
     case GX_OUT_LABEL_I32:
       if (!r.have[GX_SCC]) GX_THROW(GX_E_STATE, "SCC has not run on this graph");

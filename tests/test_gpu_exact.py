@@ -330,3 +330,27 @@ def test_async_upload_close_transform_export():
     G.run("sssp", source=-1)
     assert np.array_equal(G.download("dist"), A.sssp_dijkstra(graph_to_edgelist(g), sssp_source(g)))
     G.close()
+
+
+def test_async_download_overlaps_and_joins():
+    """GX_DL_ASYNC: a rank download queued behind PageRank completes at
+    ctx.sync() with the values of the run that produced it, even when the next
+    PageRank run (which overwrites the rank vector) is issued before that."""
+    import torch
+    raw = GRAPHS["rmat14_C1"]()
+    g = from_raw(raw)
+    el = graph_to_edgelist(g)
+    G = upload(raw)
+    G.run("pagerank", tol=1e-10, mapping="pb")
+    ref = G.download("rank")
+    out = torch.empty(g.n, dtype=torch.float64).pin_memory().numpy()
+    G.download("rank", out=out, async_copy=True)
+    G.run("sssp", source=-1, mapping="lb")
+    dout = torch.empty(g.n, dtype=torch.int32).pin_memory().numpy().view(np.uint32)
+    G.download("dist", out=dout, async_copy=True)
+    G.run("pagerank", tol=1e-2, mapping="pb")     # overwrites the ranks after the copy
+    ctx().sync()
+    assert np.array_equal(out, ref)
+    assert np.array_equal(dout, A.sssp_dijkstra(el, sssp_source(g)))
+    assert not np.array_equal(G.download("rank"), ref)
+    G.close()
