@@ -127,7 +127,11 @@ __device__ __forceinline__ void clear_bitmap(uint32_t* bm, int64_t nwords) {
 #define GX_SSSP_SU 3
 #endif
 constexpr int SU = GX_SSSP_SU;   // edges in flight per lane per round
-constexpr int SB_WARPS = 8;   // warps per CTA
+#ifndef GX_SSSP_TPB
+#define GX_SSSP_TPB 256
+#endif
+constexpr int PERSIST_TPB = GX_SSSP_TPB;   // threads per CTA of the persistent loop
+constexpr int SB_WARPS = PERSIST_TPB / 32 > 8 ? PERSIST_TPB / 32 : 8;   // warps per CTA (k_sssp_lb: 8)
 
 // iteration t with near-far threshold tau; the far pile's minimum goes to fdst
 __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj,
@@ -762,13 +766,13 @@ struct SsspLoop {
   int32_t* tlist;
 };
 
-constexpr int PERSIST_POOL = SB_WARPS * 1024 * 4;   // 32 KB: LB compaction buffer / block-mode queues
+constexpr int PERSIST_POOL = SB_WARPS * 1024 * 4;   // 32 KB at 256 threads: LB compaction buffer / block-mode queues
 static_assert(2 * BLK_Q * 4 + BLK_MAX / 8 + 16 <= PERSIST_POOL, "block-mode buffers must fit the pool");
 
 #ifndef GX_SSSP_MINB
-#define GX_SSSP_MINB 4
+#define GX_SSSP_MINB (1024 / GX_SSSP_TPB)
 #endif
-__global__ void __launch_bounds__(256, GX_SSSP_MINB) k_sssp_persist(SsspLoop a) {
+__global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(SsspLoop a) {
   __shared__ __align__(16) uint8_t pool[PERSIST_POOL];
   cg::grid_group grid = cg::this_grid();
   const bool lead = blockIdx.x == 0 && threadIdx.x == 0;
@@ -1439,7 +1443,7 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
   // LB mapping: the whole loop as one cooperative launch (k_sssp_persist);
   // GX_SSSP_PERSIST=0 selects the per-kernel loop below (A/B, tracing)
   int occp = 0, coop = 0;
-  CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occp, k_sssp_persist, 256, 0));
+  CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occp, k_sssp_persist, PERSIST_TPB, 0));
   CUDA_OK(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, c->device));
   const char* pe = getenv("GX_SSSP_PERSIST");
   const bool persist = mapping == GX_MAP_LB && coop && occp > 0 && !trace && !(pe && atoi(pe) == 0);
@@ -1503,7 +1507,7 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
     }
     void* args[] = {&L};
     kt.begin();
-    CUDA_OK(cudaLaunchCooperativeKernel((void*)k_sssp_persist, dim3((unsigned)(occp * c->num_sms)), dim3(256), args,
+    CUDA_OK(cudaLaunchCooperativeKernel((void*)k_sssp_persist, dim3((unsigned)(occp * c->num_sms)), dim3(PERSIST_TPB), args,
                                         0, s));
     kt.end();
     launches += 1;
