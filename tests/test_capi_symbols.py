@@ -61,3 +61,22 @@ def test_null_arguments_rejected(L):
     assert L.gx_ctx_create(None, 0, None) == 1
     assert L.gx_knobs_default(None) == 1
     assert L.gx_graph_upload_csr(None, None, 0, 0, None, None, None, 0) == 1
+
+
+def test_binding_constants_match_header():
+    """Every #define / enum value the binding mirrors equals the header's."""
+    from paper_conf_icpp_0001n20_b200 import _binding as B
+    src = open(os.path.join(ROOT, "include", "graffix.h")).read()
+    defs = {k: int(v) for k, v in re.findall(r"#define\s+(GX_[A-Z0-9_]+)\s+(\d+)u?\b", src)}
+    for k, v in re.findall(r"\b(GX_[A-Z0-9_]+)\s*=\s*(\d+)", src):
+        defs.setdefault(k, int(v))
+    checked = 0
+    for name in dir(B):
+        if name.startswith("GX_") and name in defs and isinstance(getattr(B, name), int):
+            assert getattr(B, name) == defs[name], name
+            checked += 1
+    assert checked >= 15
+    for flag in ("GX_PTRS_DEVICE", "GX_VALIDATE", "GX_CANONICAL", "GX_ASYNC_UPLOAD", "GX_DL_ASYNC"):
+        assert flag in defs and hasattr(B, flag), flag
+    flags = [defs[f] for f in ("GX_PTRS_DEVICE", "GX_VALIDATE", "GX_CANONICAL", "GX_ASYNC_UPLOAD", "GX_DL_ASYNC")]
+    assert all(f & (f - 1) == 0 for f in flags) and len(set(flags)) == len(flags)   # distinct single bits
