@@ -419,13 +419,32 @@ __device__ __forceinline__ void l2_prefetch_bulk(const void* p, uint32_t bytes) 
 // v = rn(t * 2^56) (quantum 1.4e-17, at most ~7e-18 per edge), split into
 // 32-bit halves; the low half is added with a returning atomic and a carry
 // out of it (rare: the low word holds up to 6e-8 of rank) goes to the high word.
+// rn(t * 2^56) for a term 0 <= t <= 1 with integer instructions: the same
+// value as __float2ull_rn(t * 0x1p56f) (the scaling is exact in f32, a
+// subnormal t rounds to 0 either way) without the 64-bit F2I, which issues to
+// the same MIO queue as the shared-memory atomics it feeds
+#ifndef GX_PB_IFIX
+#define GX_PB_IFIX 0    // measured slower: 713.5 (F2I.U64) vs 758 us per sweep (profiles/r1f/ifix_variants.txt)
+#endif
+__device__ __forceinline__ unsigned long long pb_fix56(float t) {
+  if (!GX_PB_IFIX) return __float2ull_rn(t * 0x1p56f);
+  const uint32_t b = __float_as_uint(t);
+  const int e = (int)(b >> 23);   // biased exponent (t >= 0)
+  const uint32_t m = (b & 0x7fffffu) | 0x800000u;
+  const int sh = e - 94;          // t * 2^56 = m * 2^(e - 127 - 23 + 56)
+  if (sh >= 0) return (unsigned long long)m << sh;
+  const int r = -sh;
+  if (e == 0 || r > 25) return 0ull;
+  const uint32_t q = m >> r, rem = m & ((1u << r) - 1u), half = 1u << (r - 1);
+  return q + ((rem > half || (rem == half && (q & 1u))) ? 1u : 0u);
+}
 __device__ __forceinline__ void pb_add4(uint32_t* lo, uint32_t* hi, uint2 r, float4 t4) {
   const uint32_t rr[4] = {r.x & 0xffffu, r.x >> 16, r.y & 0xffffu, r.y >> 16};
   const float tt[4] = {t4.x, t4.y, t4.z, t4.w};
   unsigned long long v[4];
   uint32_t old[4];
 #pragma unroll
-  for (int i = 0; i < 4; i++) v[i] = __float2ull_rn(tt[i] * 0x1p56f);
+  for (int i = 0; i < 4; i++) v[i] = pb_fix56(tt[i]);
   // the returning atomics are independent: issue them back to back
 #pragma unroll
   for (int i = 0; i < 4; i++) old[i] = atomicAdd(&lo[rr[i]], (uint32_t)v[i]);
@@ -537,9 +556,10 @@ template <int N>
 __device__ __forceinline__ void cp_async_wait() {
   asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
 }
+template <int DEPTH>
 __device__ __forceinline__ void pb_scatter_async(const PbArgs& p, const float* s_c, const uint32_t* r0,
                                                  const uint32_t* r1, uint32_t lo0, uint32_t hi0, uint64_t pf,
-                                                 uint4* stage /* this warp's PB_SDEPTH x 32 uint4 */) {
+                                                 uint4* stage /* this warp's DEPTH x 32 uint4 */) {
   const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
   constexpr unsigned NW = PB_THREADS / 32;
   const int64_t nb = p.nb;
@@ -570,7 +590,7 @@ __device__ __forceinline__ void pb_scatter_async(const PbArgs& p, const float* s
     }
     return false;
   };
-  uint32_t pe[PB_SDEPTH];
+  uint32_t pe[DEPTH];
   int pending = 0;
   bool more = true;
   auto refill = [&](int s) {
@@ -588,11 +608,11 @@ __device__ __forceinline__ void pb_scatter_async(const PbArgs& p, const float* s
     cp_async_commit();
   };
 #pragma unroll
-  for (int s = 0; s < PB_SDEPTH; s++) refill(s);
+  for (int s = 0; s < DEPTH; s++) refill(s);
   while (pending) {
 #pragma unroll
-    for (int s = 0; s < PB_SDEPTH; s++) {
-      cp_async_wait<PB_SDEPTH - 1>();
+    for (int s = 0; s < DEPTH; s++) {
+      cp_async_wait<DEPTH - 1>();
       if (pe[s] != 0xffffffffu) pb_put8(p.val + pe[s], s_c, stage[s * 32 + lane]);
       if (pending) pending--;   // stage s's step (issued in order) is consumed
       refill(s);
@@ -760,7 +780,7 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
     __syncthreads();
     // (3) scatter the new terms along block b's segments
     if (GX_PB_SASYNC) {
-      pb_scatter_async(p, s_c, r0, r1, lo0, hi0, pf, reinterpret_cast<uint4*>(ring) + warp * PB_SDEPTH * 32);
+      pb_scatter_async<PB_SDEPTH>(p, s_c, r0, r1, lo0, hi0, pf, reinterpret_cast<uint4*>(ring) + warp * PB_SDEPTH * 32);
       // the ring's next writes are the bulk copies (async proxy)
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     } else
@@ -771,8 +791,14 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
 }
 
 // val[] <- the initial terms contrib_0[u] along every edge: (3) for every
-// source block with s_c = contrib_0 of the block
-__global__ void __launch_bounds__(PB_THREADS, 1) k_pb_init_val(PbArgs p, const float* __restrict__ contrib,
+// source block with s_c = contrib_0 of the block, each warp with a
+// 2-deep cp.async staging slice after s_c
+constexpr int PB_INIT_SDEPTH = 2;
+constexpr size_t PB_INIT_SMEM = (size_t)(PB_R + 8) * 4 + (GX_PB_SASYNC ? (size_t)(PB_THREADS / 32) * PB_INIT_SDEPTH * 512 : 0);
+#ifndef GX_PB_INIT_MINB
+#define GX_PB_INIT_MINB 1    // measured: 1 and 2 (32 registers, spill) tie (profiles/r1f/init_variants.txt)
+#endif
+__global__ void __launch_bounds__(PB_THREADS, GX_PB_INIT_MINB) k_pb_init_val(PbArgs p, const float* __restrict__ contrib,
                                                                int64_t n_slots) {
   extern __shared__ __align__(16) float pb_init_s[];
   float* s_c = pb_init_s;   // PB_R + 8 floats
@@ -785,7 +811,11 @@ __global__ void __launch_bounds__(PB_THREADS, 1) k_pb_init_val(PbArgs p, const f
     const uint32_t* r1 = r0 + p.nb;
     const uint32_t lo0 = threadIdx.x < p.nb ? r0[threadIdx.x] : 0u, hi0 = threadIdx.x < p.nb ? r1[threadIdx.x] : 0u;
     __syncthreads();
-    pb_scatter(p, s_c, r0, r1, lo0, hi0, pf);
+    if (GX_PB_SASYNC)
+      pb_scatter_async<PB_INIT_SDEPTH>(p, s_c, r0, r1, lo0, hi0, pf,
+                                       reinterpret_cast<uint4*>(s_c + PB_R + 8) + (threadIdx.x >> 5) * PB_INIT_SDEPTH * 32);
+    else
+      pb_scatter(p, s_c, r0, r1, lo0, hi0, pf);
     __syncthreads();
   }
 }
@@ -1308,7 +1338,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     if (!attr) {
       CUDA_OK(cudaFuncSetAttribute(k_pr_pb<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
       CUDA_OK(cudaFuncSetAttribute(k_pr_pb<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
-      CUDA_OK(cudaFuncSetAttribute(k_pb_init_val, cudaFuncAttributeMaxDynamicSharedMemorySize, (PB_R + 8) * 4));
+      CUDA_OK(cudaFuncSetAttribute(k_pb_init_val, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_INIT_SMEM));
 
       attr = true;
     }
@@ -1330,7 +1360,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   int gi = grid_for(c, ns);
   if (slots) k_pr_init<true><<<gi, 256, 0, s>>>(a, ns, 1.0 / (double)g->n);
   else k_pr_init<false><<<gi, 256, 0, s>>>(a, ns, 1.0 / (double)g->n);
-  if (mapping == GX_MAP_PB) k_pb_init_val<<<(int)std::min<int64_t>(pb.nb, c->num_sms * 2), PB_THREADS, (PB_R + 8) * 4, s>>>(pb, a.contrib[0], ns);
+  if (mapping == GX_MAP_PB) k_pb_init_val<<<(int)std::min<int64_t>(pb.nb, c->num_sms * 2), PB_THREADS, PB_INIT_SMEM, s>>>(pb, a.contrib[0], ns);
   CUDA_OK(cudaGetLastError());
   int launches = mapping == GX_MAP_PB ? 2 : 1;
   const int grid_pb = (int)std::max<int64_t>(1, std::min<int64_t>(pb.nb, (int64_t)c->num_sms * PB_CTAS_PER_SM));
