@@ -10,7 +10,7 @@ import pytest
 import graphgen
 from gpu_util import ctx, upload
 from oracle import algos as A
-from oracle.graph import INF32, from_raw, graph_to_edgelist, sssp_source
+from oracle.graph import INF32, canonicalize_sorted, from_raw, graph_to_edgelist, sssp_source
 
 pytestmark = pytest.mark.gpu
 
@@ -90,6 +90,34 @@ def test_pagerank_blocked_multiblock(name):
     assert abs(got.sum() - 1.0) < 1e-6
     G.run("pagerank", tol=1e-10, max_iters=5000, mapping="lb")
     assert np.abs(G.download("rank") - want).sum() <= 1e-6
+
+
+def test_pagerank_blocked_more_bins_than_segment_groups():
+    """GX_MAP_PB with nb = 1025 sink bins (> 1024 = one 32-segment group per
+    warp of a 1024-thread CTA): every warp's scatter walks past its first group
+    of segment bounds (the group advance in pb_scatter / pb_scatter_async that
+    RMAT-24's nb = 1024 never reaches), with a ragged last block.  Too large for
+    the oracle's power iteration in a test, so checked by properties that hold
+    at any size: the fixed-point residual of the PR map (the oracle's update
+    rule, O3 / R35) in fp64, unit mass, and the LB mapping's ranks."""
+    n = 16384 * 1024 + 4099
+    raw = graphgen.uniform(n, 2 * n)
+    G = upload(raw)
+    info = G.run("pagerank", tol=1e-10, max_iters=5000, mapping="pb")
+    assert info["mapping_used"] == 3
+    assert info["converged"] >= 1
+    x = G.download("rank")
+    assert abs(x.sum() - 1.0) < 1e-6
+    src, dst, _ = canonicalize_sorted(raw.n, raw.row_ptr, raw.col, raw.w).edges()   # A0
+    src = np.asarray(src, dtype=np.int64)
+    dst = np.asarray(dst, dtype=np.int64)
+    dout = np.bincount(src, minlength=n).astype(np.float64)
+    dang = dout == 0
+    contrib = np.where(dang, 0.0, x / np.where(dang, 1.0, dout))
+    fx = 0.15 / n + 0.85 * (np.bincount(dst, weights=contrib[src], minlength=n) + x[dang].sum() / n)
+    assert np.abs(fx - x).sum() <= 1e-6
+    G.run("pagerank", tol=1e-10, max_iters=5000, mapping="lb")
+    assert np.abs(G.download("rank") - x).sum() <= 1e-6
 
 
 @pytest.mark.parametrize("name", ["rmat12", "star_hub", "road64", "dups_loops", "isolated", "single"])
