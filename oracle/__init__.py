@@ -22,6 +22,7 @@ Modules
                 iteration, §2.4 P@27655-28981), used to pin Theorems E1/E3.
   metrics    -- inaccuracy (P@40990-41294) and O(m) certificates.
 
-Parity status per function is stated in each docstring; functions whose
-only pins are invariants say "parity unpinned".
+Parity status per function is stated in each docstring (see DESIGN.md §3);
+every function is pinned to something other than itself (printed examples,
+hand-derived fixtures, closed forms, brute force or library routines).
 """

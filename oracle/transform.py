@@ -19,9 +19,12 @@ Parity status:
   renumber/replicate: pinned to the Fig 1-4 printed example (tests/golden)
     and to the isomorphism / 2-hop-path invariants;
   degree padding: pinned to the Fig 6 example + invariants;
-  cc_edges (case 1 / case 2 selection) and subgraph packing: PARITY UNPINNED
-    beyond invariants (budget, 2-path + sum weight, disjointness) -- the
-    selection rules R22-R28 are readings, Fig 5 cannot be recovered.
+  cc_edges (case 1 / case 2 selection) and subgraph packing: pinned to six
+    hand-derived fixtures (tests/golden/sec3_*.txt, derivations in each file,
+    P@31015 common-neighbour preference, P@31268 fewest internal edges) that
+    kill every single-decision mutant of tools/mutate_sec3.py, plus the
+    invariants (budget, 2-path + sum weight, disjointness).  Fig 5 itself
+    cannot be recovered; the selection rules R22-R28 are readings.
 """
 from __future__ import annotations
 
@@ -397,8 +400,12 @@ class _Logical:
 
 
 def cc_edges(tg: TransformedGraph, cc_ppm: int, budget: int, rule: str = "sum", undirected: bool = False):
-    """§3 edge insertion (P@30608-32051), readings R21-R26.  PARITY UNPINNED
-    beyond invariants (the selection rules are readings).
+    """§3 edge insertion (P@30608-32051), readings R21-R26.  Pinned by the
+    hand-derived fixtures S1-S6 (tests/golden/sec3_*.txt): centre order
+    (S1), pair order by common neighbours P@31015 (S2), stop at high (S2),
+    case-2 sibling / partner by fewest internal edges P@31268 (S3), case 1
+    before case 2 and case-2 centre order (S4), skip rule (S5), round-robin
+    passes (S6); tools/mutate_sec3.py shows each decision is load-bearing.
 
     Case 1 (raise near-threshold centres, R22): non-high centres with d >= 2
     in (need asc, id asc) order, need = floor(theta_ppm * P / 1e6) + 1 - T
@@ -507,7 +514,9 @@ def cc_edges(tg: TransformedGraph, cc_ppm: int, budget: int, rule: str = "sum", 
 
 def subgraphs(L: _Logical, n: int, cc_ppm: int, smax: int, smem_iters: int):
     """§3 shared-memory subgraphs (P@30023-30382, P@31631, P@32188-32416),
-    readings R27/R28.  PARITY UNPINNED beyond invariants.
+    readings R27/R28.  Pinned by the tiles of fixtures S1-S6 (centre order
+    CC desc S1, d desc S2, id asc S1/S4; t = 2 x diameter: 2 for cliques,
+    4 in S3/S4/S6).
 
     Centres: high vertices with 1 + d <= S_max, ordered (CC desc (exact
     rational), d desc, id asc); S(c) = {c} + N(c) is accepted iff disjoint from

@@ -59,14 +59,13 @@ def main():
         tp = time.time() - t0
         G = gx.Graph.upload(ctx, prp, pcol, pw)
         res = {}
-        for al, kw in (("sssp", {}), ("pagerank", {"tol": 1e-9})):
+        for al, mp, kw in (("sssp", "lb", {}), ("pagerank", "lb", {"tol": 1e-9}), ("pagerank", "pb", {"tol": 1e-9})):
             if al not in a.algos.split(","):
-                res[al] = None
                 continue
-            rs = [G.run(al, mapping="lb", **kw) for _ in range(a.reps)]
+            rs = [G.run(al, mapping=mp, **kw) for _ in range(a.reps)]
             b = min(rs, key=lambda r: r["loop_ms"])
-            res[al] = (round(b["loop_ms"], 3), b["iterations"], b["edges_scanned"])
-        print(f"order={o} permute_s={tp:.1f} sssp={res['sssp']} pagerank={res['pagerank']}", flush=True)
+            res[al + "_" + mp] = (round(b["loop_ms"], 3), b["iterations"], b["edges_scanned"])
+        print(f"order={o} permute_s={tp:.1f} " + " ".join(f"{k}={v}" for k, v in res.items()), flush=True)
         G.close()
 
 
