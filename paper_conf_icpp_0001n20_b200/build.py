@@ -6,6 +6,7 @@ from __future__ import annotations
 
 import concurrent.futures as cf
 import glob
+import hashlib
 import os
 import subprocess
 import sys
@@ -47,8 +48,20 @@ def _compile(src: str, force: bool, extra) -> str:
     return obj
 
 
+def _flags_stamp(extra) -> str:
+    """Hash of everything that changes the objects besides the sources: the
+    compiler, the arch and the full flag set (GX_NVCC_EXTRA and ``extra``)."""
+    return hashlib.sha256(repr((NVCC, ARCH, COMMON, list(extra))).encode()).hexdigest()
+
+
 def build(force: bool = False, jobs: int | None = None, extra=()) -> str:
     os.makedirs(OBJ, exist_ok=True)
+    # objects built with other flags (an A/B variant's -D...) are never reused
+    stamp_path = os.path.join(OBJ, "flags.stamp")
+    stamp = _flags_stamp(extra)
+    old = open(stamp_path).read().strip() if os.path.exists(stamp_path) else ""
+    if old != stamp:
+        force = True
     srcs = _sources()
     with cf.ThreadPoolExecutor(max_workers=jobs or min(16, os.cpu_count() or 4)) as ex:
         objs = list(ex.map(lambda s: _compile(s, force, extra), srcs))
@@ -59,6 +72,9 @@ def build(force: bool = False, jobs: int | None = None, extra=()) -> str:
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
         os.replace(tmp, OUT)
+    if old != stamp:
+        with open(stamp_path, "w") as f:
+            f.write(stamp + "\n")
     return OUT
 
 

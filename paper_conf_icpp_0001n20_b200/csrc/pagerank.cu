@@ -1334,14 +1334,11 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     pb.dst_loc = d.pr_pb.dst_loc.as<uint16_t>();
     pb.val = d.pr_pb.val.as<float>();
     pb.nb = d.pr_pb.nb;
-    static bool attr = false;
-    if (!attr) {
-      CUDA_OK(cudaFuncSetAttribute(k_pr_pb<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
-      CUDA_OK(cudaFuncSetAttribute(k_pr_pb<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
-      CUDA_OK(cudaFuncSetAttribute(k_pb_init_val, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_INIT_SMEM));
-
-      attr = true;
-    }
+    // the opt-in is per device (context): set it on every run (cheap), not
+    // once per process -- a second GPU in the same process needs it too
+    CUDA_OK(cudaFuncSetAttribute(k_pr_pb<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
+    CUDA_OK(cudaFuncSetAttribute(k_pr_pb<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
+    CUDA_OK(cudaFuncSetAttribute(k_pb_init_val, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_INIT_SMEM));
   }
   if (mapping == GX_MAP_TPV) {
     ensure_tpv(g);

@@ -46,8 +46,7 @@ __device__ __forceinline__ bool bit_of(const uint32_t* __restrict__ bm, uint32_t
 // distance `cur` of its head
 __device__ __forceinline__ void relax_red(uint2 ed, uint32_t du, uint32_t cur, uint32_t* __restrict__ dist,
                                           uint32_t* __restrict__ bm_next, uint32_t& npush, uint64_t pl) {
-  uint32_t nd = du + ed.y;
-  if (nd < du) nd = INF - 1;  // saturate (never the fixed point)
+  const uint32_t nd = sat_add(du, ed.y);   // R51
   if (nd < cur) {
     red_min_l2(dist + ed.x, nd, pl);
     red_or_l2(bm_next + (ed.x >> 5), 1u << (ed.x & 31), pl);
@@ -60,8 +59,7 @@ __device__ __forceinline__ void relax_red(uint2 ed, uint32_t du, uint32_t cur, u
 __device__ __forceinline__ void relax_nf(uint2 ed, uint32_t du, uint32_t cur, uint32_t* __restrict__ dist,
                                          uint32_t* __restrict__ bm_next, uint32_t* __restrict__ far, uint32_t tau,
                                          uint32_t& far_min, uint32_t& npush, uint64_t pl) {
-  uint32_t nd = du + ed.y;
-  if (nd < du) nd = INF - 1;
+  const uint32_t nd = sat_add(du, ed.y);
   if (nd < cur) {
     red_min_l2(dist + ed.x, nd, pl);
     if (nd < tau) {
@@ -432,8 +430,7 @@ __device__ __forceinline__ void sssp_local_dev(const int32_t* __restrict__ tptr,
         const uint32_t src = p.x & 0xff, dst = (p.x >> 8) & 0xff;
         const uint32_t du = sd[src];
         if (du != INF) {
-          uint32_t nd = du + p.y;
-          if (nd < du) nd = INF - 1;
+          const uint32_t nd = sat_add(du, p.y);
           if (nd < sd[dst]) {
             atomicMin(&sd[dst], nd);
             ch = 1;
@@ -488,7 +485,7 @@ __device__ __forceinline__ void sssp_merge_dev(const int32_t* __restrict__ gptr,
     for (int e = ginptr[gi] + lane; e < ginptr[gi + 1]; e += 32) {
       const uint2 iv = gin[e];
       const uint32_t dp = __ldcg(dist + iv.x);
-      if (dp != INF) best = min(best, dp + iv.y < dp ? INF - 1 : dp + iv.y);   // saturating (R51)
+      if (dp != INF) best = min(best, sat_add(dp, iv.y));   // saturating (R51)
     }
     best = warp_min_u32(best);
     const uint32_t own = min(__ldcg(dist + o), best);
@@ -658,8 +655,7 @@ __device__ __forceinline__ void sssp_block_dev(const uint32_t* __restrict__ rp, 
       my_edges += b - a;
       for (uint32_t e = a; e < b; e++) {
         const uint2 ed = ld_edge(adj, ax, e, pf);
-        uint32_t nd = du + ed.y;
-        if (nd < du) nd = INF - 1;
+        const uint32_t nd = sat_add(du, ed.y);
         const uint32_t cv = ld_l2_u32(dist + ed.x, pl);
         if (nd >= cv) continue;
         const int64_t v = ed.x;

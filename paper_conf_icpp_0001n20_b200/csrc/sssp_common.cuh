@@ -50,6 +50,13 @@ struct SsspAux {
   const uint32_t* lend;
   uint32_t* pend[2];
 };
+// du + w, saturated at 2^32-2 (reading R51): every sum that wraps or lands on
+// INF becomes INF-1, which k_sat_check reports as an overflow after the run
+__device__ __forceinline__ uint32_t sat_add(uint32_t du, uint32_t w) {
+  const uint32_t nd = du + w;
+  return (nd < du || nd == 0xFFFFFFFFu) ? 0xFFFFFFFEu : nd;
+}
+
 // the out-edge e as {dst, w}
 __device__ __forceinline__ uint2 ld_edge(const uint2* __restrict__ adj, const SsspAux& ax, uint32_t e, uint64_t pol) {
   if (ax.adjp) {

@@ -171,6 +171,14 @@ def test_errors():
     with pytest.raises(GraffixError) as e:
         Gb.run("sssp", source=0)
     assert e.value.status == 6
+    # a path whose length is exactly 2^32 - 1 (= INF as a sum, no wrap) is also
+    # reported, for every mapping (the sum must saturate, not vanish)
+    exact_inf = graphgen.from_edge_list(3, [(0, 1, 2**31), (1, 2, 2**31 - 1)])
+    for mp in ("lb", "tpv", "vns"):
+        Ge = upload(exact_inf)
+        with pytest.raises(GraffixError) as e:
+            Ge.run("sssp", source=0, mapping=mp)
+        assert e.value.status == 6, mp
     # ... but a large static bound (n-1)*max(w) with short true distances runs:
     # the saturated candidate 2^32-2 never wins against a real path
     ok = graphgen.from_edge_list(4, [(0, 1, 1), (1, 2, 1), (2, 3, 1), (0, 3, 2**31), (3, 0, 2**31 + 7)])
