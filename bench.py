@@ -42,6 +42,15 @@ PR_KERNELS = {1: "k_pr_sell2", 2: "k_pr_tpv", 3: "k_pr_pb"}   # gx_mapping -> PR
 MAPPING_NAMES = {0: "auto", 1: "lb", 2: "tpv", 3: "pb"}   # bounded oracle sample: same generator at 1/128 of T24
 
 
+def _free_port() -> int:
+    import socket
+    so = socket.socket()
+    so.bind(("127.0.0.1", 0))
+    port = so.getsockname()[1]
+    so.close()
+    return port
+
+
 def peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -108,6 +117,70 @@ def oracle_sample(scale=CPU_SAMPLE_SCALE):
             "n": g.n, "m": g.m}
 
 
+def inaccuracy_pct(approx, exact, inf=None):
+    """PAPER.md P@40990-41294 (reading R40): 100 * sum|a - e| / sum|e| over the
+    vertices finite in both runs (a metric on two GPU results, no oracle)."""
+    a = np.asarray(approx, dtype=np.float64)
+    e = np.asarray(exact, dtype=np.float64)
+    ok = np.ones(a.shape, bool) if inf is None else (np.asarray(approx) != inf) & (np.asarray(exact) != inf)
+    den = np.abs(e[ok]).sum()
+    return float(100.0 * np.abs(a[ok] - e[ok]).sum() / den) if den > 0 else 0.0
+
+
+def knob_points(ctx, reps=2):
+    """BASELINE metric's "speedup vs exact at inaccuracy%" (Tables 6 and 8,
+    P@42046-42906, P@43835-44682) at two paper-style settings: C2 (RMAT-22) §2
+    coalescing k=16, theta_conn=0.6 with the algorithm-aware merge; C4 (uniform
+    16M/256M) §4 degree normalisation theta_d=0.3, f=0.85.  Per algorithm: the
+    knob's best mapping vs the best exact mapping, and per mapping vs the same
+    mapping exact; inaccuracy (R40) of the knob run vs the exact run; transform
+    time and extra space (Table 5 analogue)."""
+    import graphgen
+    import paper_conf_icpp_0001n20_b200 as gx
+    U32_INF = 0xFFFFFFFF
+    cases = [
+        ("C2 rmat22 coalesce k16 theta0.6 aware-merge", lambda: graphgen.rmat(22),
+         gx.Knobs(coalesce=True, chunk_k=16, replicate_threshold=0.6, merge_op=1)),
+        ("C4 uniform16M/256M degnorm theta0.3 f0.85", lambda: graphgen.uniform(1 << 24, 1 << 28),
+         gx.Knobs(degree_norm=True, degsim_threshold=0.3, degree_target=0.85)),
+    ]
+    maps = {"sssp": ("lb", "tpv"), "pagerank": ("pb", "lb", "tpv")}
+    out = []
+    for name, mk, kn in cases:
+        t0 = time.perf_counter()
+        raw = mk()
+        G = gx.Graph.upload(ctx, raw.row_ptr, raw.col, raw.w)
+
+        def timed(algo, mp):
+            kw = {"tol": 1e-9} if algo == "pagerank" else {}
+            return min(G.run(algo, mapping=mp, **kw)["loop_ms"] for _ in range(reps))
+        ex = {a: {mp: timed(a, mp) for mp in maps[a]} for a in maps}
+        G.run("sssp", mapping="lb")
+        de = G.download("dist").copy()
+        G.run("pagerank", mapping="pb", tol=1e-9)
+        xe = G.download("rank").copy()
+        info = G.transform(kn)
+        ap = {a: {mp: timed(a, mp) for mp in maps[a]} for a in maps}
+        G.run("sssp", mapping="auto")
+        da = G.download("dist")
+        G.run("pagerank", mapping="auto", tol=1e-9)
+        xa = G.download("rank")
+        inacc = {"sssp": inaccuracy_pct(da, de, U32_INF), "pagerank": inaccuracy_pct(xa, xe)}
+        pt = {}
+        for a in maps:
+            best_e = min(ex[a].values())
+            best_k = min(ap[a].values())
+            pt[a] = {"exact_ms": ex[a], "knob_ms": ap[a],
+                     "speedup_vs_best_exact": best_e / best_k,
+                     "speedup_same_mapping": {mp: ex[a][mp] / ap[a][mp] for mp in maps[a]},
+                     "inaccuracy_pct": inacc[a]}
+        out.append({"config": name, "n": G.n, "m": G.m, "transform_s": info["transform_ms"] / 1e3,
+                    "extra_space_pct": info["extra_space_pct"], "algos": pt,
+                    "wall_s": time.perf_counter() - t0})
+        G.close()
+    return out
+
+
 def cpu_cores_used() -> int:
     return 1   # the oracle is single-threaded Python/numpy (numpy bincount is serial)
 
@@ -144,6 +217,7 @@ def main():
     ap.add_argument("--workload", default="t24", choices=list(WORKLOADS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-knobs", action="store_true", help="skip the knob speedup / inaccuracy points (~60 s)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--e2e-sync", action="store_true", help="upload without GX_ASYNC_UPLOAD")
     ap.add_argument("--pr-mapping", default="auto", choices=["auto", "lb", "tpv", "pb"],
@@ -152,10 +226,18 @@ def main():
     args.warmup = max(args.warmup, 3)
 
     rank = int(os.environ.get("RANK", "0"))
-    world = int(os.environ.get("WORLD_SIZE", "1"))
+    world = int(os.environ.get("WORLD_SIZE", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world == 0 and args.gpus > 1 and args.impl == "ours":
+        # not under torchrun: start the N ranks ourselves (one process per GPU)
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", f"--master-port={_free_port()}", os.path.abspath(__file__)] + sys.argv[1:]
+        return subprocess.call(cmd)
+    world = world or 1
     if args.impl == "reference":
         return run_reference(args, rank, world)
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: WORLD_SIZE={world} but --gpus {args.gpus}")
 
     import torch
     import torch.distributed as dist
@@ -208,28 +290,37 @@ def main():
         tt = torch.tensor([tot_ms], device="cuda")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         tot_ms = float(tt.item())
-    # SSSP relaxations are counted per rank (sum them); PR sweeps cover all m per iteration
-    sssp_edges = sum(a["edges_scanned"] for a, _ in runs)
+    # edges scanned are counted per rank (SSSP relaxations of its rows, PR
+    # in-edges of its rows per sweep): the job's total is the sum over ranks
+    edges = sum(a["edges_scanned"] + b["edges_scanned"] for a, b in runs)
     if world > 1:
-        te = torch.tensor([float(sssp_edges)], device="cuda", dtype=torch.float64)
+        te = torch.tensor([float(edges)], device="cuda", dtype=torch.float64)
         dist.all_reduce(te)
-        sssp_edges = int(te.item())
-    edges = sssp_edges + sum(b["edges_scanned"] for _, b in runs)
+        edges = int(te.item())
     value = edges / (tot_ms * 1e-3) / 1e9
     launches = sum(a["kernel_launches"] + b["kernel_launches"] for a, b in runs)
 
-    # dominant kernel roofline (live CUDA events around each sweep launch)
+    # dominant kernel roofline (live CUDA events around each sweep launch on the
+    # library's stream).  One GPU: SSSP is ONE cooperative launch per run
+    # (k_sssp_persist, the whole fixed-point loop); PageRank one launch per
+    # sweep.  N > 1: the partitioned loops (sweeps + NCCL exchange) per rank.
     peak, peak_src = peaks()
     kern = {}
     pr_kernel = PR_KERNELS.get(runs[-1][1].get("mapping_used", 1), "k_pr_sell2")
-    for name, idx in (("k_sssp_lb", 0), (pr_kernel, 1)):
-        ms = sum(r[idx]["sweep_ms"] for r in runs)
-        # sweeps that did work (a CUDA-graph / eager batch may launch a few
-        # more that return at once after convergence; their ~3 us stay in ms)
-        nl = sum(r[idx]["iterations"] for r in runs)
+    sssp_kernel = "k_sssp_persist" if world == 1 else "sssp partitioned loop (k_sssp_lb + exchange)"
+    if world > 1:
+        pr_kernel = "pagerank partitioned loop (k_pr_sell2 + exchange)"
+    for name, idx in ((sssp_kernel, 0), (pr_kernel, 1)):
+        if world == 1:
+            ms = sum(r[idx]["sweep_ms"] for r in runs)
+            nl = sum(r[idx]["sweep_launches"] for r in runs)
+        else:
+            ms = sum(r[idx]["loop_ms"] for r in runs)
+            nl = len(runs)
+        it = sum(r[idx]["iterations"] for r in runs)
         by = sum(r[idx]["bytes_model"] for r in runs)        # algorithmic (SURVEY §8(d) model)
-        enc = sum(r[idx]["sweep_bytes"] for r in runs)       # what the kernel's encoding streams
-        kern[name] = {"ms_total": ms, "launches": nl, "bytes": by, "encoding_bytes": enc,
+        enc = sum(r[idx].get("sweep_bytes", 0) or r[idx]["bytes_model"] for r in runs)   # the kernel's encoding
+        kern[name] = {"ms_total": ms, "launches": nl, "iterations": it, "bytes": by, "encoding_bytes": enc,
                       "gbs": by / (ms * 1e-3) / 1e9 if ms > 0 else None,
                       "encoding_gbs": enc / (ms * 1e-3) / 1e9 if ms > 0 else None,
                       "share_of_step": ms / tot_ms if tot_ms else None}
@@ -240,13 +331,15 @@ def main():
     tpath = os.path.join(ROOT, "profiles", "latest", "traffic.json")
     if os.path.exists(tpath):
         tj = json.load(open(tpath))
-        if dom in tj:
+        if dom in tj and tj[dom].get("graph", "rmat24") == f"rmat{wl['scale']}":
             traffic = tj[dom]["traffic_bytes_per_launch"]
+    # PR: a launch is one sweep (8 B/in-edge + 32 B/slot); SSSP: one launch is the whole loop
     roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak if achieved else None, "traffic": traffic,
                 "traffic_unit": "bytes/launch (ncu dram read+write, profiles/latest)", "peak_source": peak_src,
                 "bytes_per_launch": dk["bytes"] / max(dk["launches"], 1),
-                "us_per_launch": 1e3 * dk["ms_total"] / max(dk["launches"], 1)}
+                "us_per_launch": 1e3 * dk["ms_total"] / max(dk["launches"], 1),
+                "bytes_model": "SURVEY §8(d): PR 8 B/in-edge + 32 B/slot per sweep; SSSP 12 B/relaxed edge + 12 B/frontier slot"}
     if dk["encoding_bytes"] != dk["bytes"]:
         # k_pr_pb streams 12 B per edge where the §8(d) pull model counts 8 B
         # (it trades the random contrib gathers for streamed terms): frac above
@@ -254,15 +347,6 @@ def main():
         roofline["encoding"] = {"bytes_per_launch": dk["encoding_bytes"] / max(dk["launches"], 1),
                                 "achieved": dk["encoding_gbs"], "frac": dk["encoding_gbs"] / peak,
                                 "model": "12 B/edge + 28 B/slot (blocked pull: terms streamed along edges)"}
-    if dom == "k_pr_sell2":
-        # the ceiling this kernel actually meets: random 4-byte contrib gathers
-        # through L1TEX (~1 wavefront/clk/SM); peak = tools/microbench4.cu LSU
-        # gathers from a 64 MB L2-resident vector (profiles/r1b)
-        gathers = sum(b["edges_scanned"] for _, b in runs)
-        g_rate = gathers / (dk["ms_total"] * 1e-3) / 1e9
-        roofline["secondary"] = {"bound": "l1tex random-gather wavefronts", "achieved": g_rate, "peak": 273.5,
-                                 "unit": "Ggather/s", "frac": g_rate / 273.5,
-                                 "peak_source": "measured, profiles/r1b/microbench4_tma_gather.txt"}
 
     a0, b0 = runs[-1]
     per_algo = {
@@ -311,6 +395,9 @@ def main():
             tt = torch.tensor([t], device="cuda")
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             t = float(tt.item())
+            te = torch.tensor([float(e2e_edges)], device="cuda", dtype=torch.float64)
+            dist.all_reduce(te)
+            e2e_edges = int(te.item())
         e2e = {"value": e2e_edges / (t * 1e-3) / 1e9, "unit": UNIT, "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": d2h, "ms_per_step": t / len(e2e_ms),
                "note": "upload of canonical pinned CSR (GX_CANONICAL" + ("" if args.e2e_sync else " | GX_ASYNC_UPLOAD: weights H2D overlapping the blocked PR; rank D2H (GX_DL_ASYNC) overlapping SSSP") + ") + device layouts (blocked-PR segments, SSSP heavy chunks) + PR + download rank + SSSP + download dist"}
@@ -323,17 +410,21 @@ def main():
                          f"(n={r['n']}, m={r['m']}; same generator, 1/{1 << (24 - CPU_SAMPLE_SCALE)} of T24), "
                          f"{r['sec']:.1f} s", "host_cores": os.cpu_count()}
 
+    knobs = None
+    if rank == 0 and world == 1 and not args.no_knobs:
+        knobs = knob_points(ctx)
+
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
-                "scaling": "strong" if world > 1 else "weak", "vs_baseline": None, "dtype": "u32/f64", "data": "synthetic",
+                "scaling": "strong", "vs_baseline": None, "dtype": "u32/f64", "data": "synthetic",
                 "config": {"workload": wl["desc"], "graph": f"rmat{wl['scale']}", "n": n, "m": m,
                            "knobs": "exact",
                            "mapping": {"sssp": MAPPING_NAMES.get(runs[-1][0].get("mapping_used", 1), "lb"),
                                        "pagerank": MAPPING_NAMES.get(runs[-1][1].get("mapping_used", 1), "?")}, "l2": "flushed between steps (256 MiB write)",
                            "parallelism": f"1-D partitioned x{world} (NCCL)" if world > 1 else "single"},
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
-                "clocks": clocks, "per_algo": per_algo, "kernels": kern}
+                "clocks": clocks, "per_algo": per_algo, "kernels": kern, "knobs": knobs}
         print(json.dumps(line))
     if world > 1:
         dist.destroy_process_group()

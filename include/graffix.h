@@ -231,6 +231,37 @@ gx_status gx_get_nccl_unique_id(uint8_t out[128]);
 gx_status gx_ctx_create_dist(gx_ctx** out, int device, void* cuda_stream, int rank,
                              int world, const uint8_t id[128]);
 
+/* Hosted exchange: the same 1-D partitioned path (the paper
+ * itself is single-GPU, P@38588) with a transport supplied by the caller
+ * instead of NCCL -- e.g. torch.distributed over gloo, so that two processes
+ * sharing ONE GPU run the library's real partitioned code.  Every collective
+ * of the partitioned path is staged through a pinned host buffer owned by the
+ * context: the library copies the device data to host_buf, calls fn, and
+ * copies the part it relies on back.  fn must return 0 on success (any other
+ * value fails the run with GX_E_NCCL) and must be called collectively by
+ * every rank (same kind / count / dtype / op / offsets):
+ *   GX_COLL_ALLREDUCE       host_buf[0..count) <- reduction (op) over ranks
+ *   GX_COLL_ALLGATHERV      host_buf[offsets[r]..offsets[r+1]) <- rank r's
+ *                           values of that slice, for every r (count =
+ *                           offsets[world]; offsets has world+1 entries)
+ *   GX_COLL_REDUCE_SCATTERV host_buf[offsets[rank]..offsets[rank+1]) <- the
+ *                           reduction over ranks of that slice (only this
+ *                           slice is read back)
+ * dtype: GX_DT_U32 / GX_DT_F32 / GX_DT_F64; op: GX_OP_SUM / GX_OP_MIN.
+ * Errors: GX_E_INVALID (fn NULL, rank outside [0, world)), GX_E_CUDA. */
+#define GX_COLL_ALLREDUCE 0
+#define GX_COLL_ALLGATHERV 1
+#define GX_COLL_REDUCE_SCATTERV 2
+#define GX_DT_U32 0
+#define GX_DT_F32 1
+#define GX_DT_F64 2
+#define GX_OP_SUM 0
+#define GX_OP_MIN 1
+typedef int (*gx_coll_fn)(int32_t kind, void* host_buf, int64_t count, int32_t dtype, int32_t op,
+                          const int64_t* offsets, int32_t world, void* user);
+gx_status gx_ctx_create_hosted(gx_ctx** out, int device, void* cuda_stream, int rank, int world,
+                               gx_coll_fn fn, void* user);
+
 /* Device allocator hook (e.g. torch's caching allocator).  alloc returns a
  * device pointer or NULL; release frees it.  Must be set before uploads. */
 typedef void* (*gx_alloc_fn)(size_t bytes, void* stream, void* user);

@@ -17,7 +17,8 @@ from dataclasses import dataclass, fields
 
 import numpy as np
 
-from ._binding import (ALGOS, ALLOC_FN, GX_ASYNC_UPLOAD, GX_CANONICAL, GX_DL_ASYNC, GX_MAP_AUTO, GX_MAP_LB, GX_MAP_PB, GX_MAP_TPV, GX_MAP_VNS, GX_OUT_BC_F64,
+from ._binding import (ALGOS, ALLOC_FN, COLL_FN, GX_COLL_ALLGATHERV, GX_COLL_ALLREDUCE, GX_COLL_REDUCE_SCATTERV,
+                       GX_DT_F32, GX_DT_F64, GX_DT_U32, GX_OP_MIN, GX_ASYNC_UPLOAD, GX_CANONICAL, GX_DL_ASYNC, GX_MAP_AUTO, GX_MAP_LB, GX_MAP_PB, GX_MAP_TPV, GX_MAP_VNS, GX_OUT_BC_F64,
                        GX_OUT_DIST_U32, GX_OUT_LABEL_I32, GX_OUT_MST_WEIGHT_U64, GX_OUT_RANK_F64,
                        GX_PTRS_DEVICE, GX_PTRS_HOST, GX_VALIDATE, RELEASE_FN, GraffixError, GxExport,
                        GxExportSizes, GxKnobs, GxRunInfo, GxRunOpts, GxTransformInfo, _check, _ptr, lib)
@@ -73,7 +74,9 @@ class Context:
 
     @classmethod
     def distributed(cls, device: int, rank: int, world: int, group=None, stream=None):
-        """One context per rank; the NCCL id is broadcast with torch.distributed."""
+        """One context per rank with an NCCL communicator; the NCCL unique id is
+        broadcast with torch.distributed (any backend: the id travels as a Python
+        object, so an NCCL-only process group works -- ADVICE r1)."""
         import glob
         import os
 
@@ -85,16 +88,62 @@ class Context:
                                            "libnccl.so.2"))
             if cands:
                 os.environ["GX_NCCL_LIB"] = os.path.realpath(cands[0])
-        uid = torch.zeros(128, dtype=torch.uint8)
+        obj = [None]
         if rank == 0:
             buf = (C.c_uint8 * 128)()
             _check(lib().gx_get_nccl_unique_id(buf))
-            uid = torch.tensor(list(bytes(buf)), dtype=torch.uint8)
-        dist.broadcast(uid, src=0, group=group)
+            obj = [bytes(buf)]
+        if dist.get_backend(group) == "nccl":
+            torch.cuda.set_device(device)   # broadcast_object_list stages through the current device
+        dist.broadcast_object_list(obj, src=0, group=group)
         h = C.c_void_p()
-        ub = (C.c_uint8 * 128)(*uid.tolist())
+        ub = (C.c_uint8 * 128)(*obj[0])
         _check(lib().gx_ctx_create_dist(C.byref(h), device, C.c_void_p(stream) if stream else None, rank, world, ub))
         return cls(device, _handle=h)
+
+    @classmethod
+    def hosted(cls, device: int, rank: int, world: int, group=None, stream=None):
+        """One context per rank whose partitioned-path collectives go through
+        torch.distributed on HOST buffers (gx_ctx_create_hosted), e.g. a gloo
+        group -- so several processes may share one GPU and still run the
+        library's real 1-D partitioned code (staging and transport only; every
+        sweep, layout and reduction decision stays in libgraffix).  The
+        allgather-v and reduce-scatter-v are carried as an allreduce: sum over
+        a buffer holding only this rank's slice, min over the whole buffer."""
+        import torch
+        import torch.distributed as dist
+        np_dt = {GX_DT_U32: np.uint32, GX_DT_F32: np.float32, GX_DT_F64: np.float64}
+        th_dt = {GX_DT_U32: torch.int64, GX_DT_F32: torch.float32, GX_DT_F64: torch.float64}
+
+        def _coll(kind, buf, count, dtype, op, offsets, nw, user):
+            try:
+                if count == 0:
+                    return 0
+                a = np.ctypeslib.as_array((C.c_char * (count * np.dtype(np_dt[dtype]).itemsize)).from_address(buf))
+                a = a.view(np_dt[dtype])
+                # gloo has no uint32 reductions: carry u32 as int64 (exact)
+                t = torch.from_numpy(a.astype(np.int64) if dtype == GX_DT_U32 else a.copy())
+                rop = dist.ReduceOp.MIN if op == GX_OP_MIN else dist.ReduceOp.SUM
+                if kind == GX_COLL_ALLGATHERV:
+                    lo, hi = offsets[rank], offsets[rank + 1]
+                    t[:lo] = 0
+                    t[hi:] = 0
+                    rop = dist.ReduceOp.SUM          # exact: every slot has one non-zero term
+                dist.all_reduce(t, op=rop, group=group)
+                a[:] = t.numpy().astype(np_dt[dtype])
+                return 0
+            except Exception as e:   # reported as GX_E_NCCL by the library
+                import sys
+                print(f"graffix hosted exchange failed: {e!r}", file=sys.stderr)
+                return 1
+
+        cb = COLL_FN(_coll)
+        h = C.c_void_p()
+        _check(lib().gx_ctx_create_hosted(C.byref(h), device, C.c_void_p(stream) if stream else None, rank, world,
+                                          cb, None))
+        ctx = cls(device, _handle=h)
+        ctx._coll_cb = cb                    # keep the trampoline alive with the context
+        return ctx
 
     def _hook_torch(self):
         try:

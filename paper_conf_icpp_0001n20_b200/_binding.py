@@ -32,7 +32,7 @@ EXPORTED = [
     "gx_set_allocator", "gx_ctx_destroy", "gx_ctx_stream", "gx_graph_upload_csr", "gx_graph_destroy",
     "gx_graph_info", "gx_knobs_default", "gx_transform", "gx_export_sizes", "gx_export_transformed",
     "gx_run", "gx_run_ex", "gx_run_opts_default", "gx_download", "gx_sync", "gx_graph_create_host",
-    "gx_partition_rows",
+    "gx_partition_rows", "gx_ctx_create_hosted",
 ]
 
 
@@ -77,6 +77,12 @@ class GxExport(C.Structure):
 
 ALLOC_FN = C.CFUNCTYPE(C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
 RELEASE_FN = C.CFUNCTYPE(None, C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
+# gx_coll_fn (include/graffix.h, hosted exchange)
+COLL_FN = C.CFUNCTYPE(C.c_int, C.c_int32, C.c_void_p, C.c_int64, C.c_int32, C.c_int32, C.POINTER(C.c_int64),
+                      C.c_int32, C.c_void_p)
+GX_COLL_ALLREDUCE, GX_COLL_ALLGATHERV, GX_COLL_REDUCE_SCATTERV = 0, 1, 2
+GX_DT_U32, GX_DT_F32, GX_DT_F64 = 0, 1, 2
+GX_OP_SUM, GX_OP_MIN = 0, 1
 
 
 class GraffixError(RuntimeError):
@@ -121,6 +127,7 @@ def lib():
         "gx_sync": ([P], C.c_int),
         "gx_graph_create_host": ([C.POINTER(P), i64, i64, P, P, P, u32], C.c_int),
         "gx_partition_rows": ([i64, P, i32, i64, P], C.c_int),
+        "gx_ctx_create_hosted": ([C.POINTER(P), C.c_int, P, C.c_int, C.c_int, COLL_FN, P], C.c_int),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)

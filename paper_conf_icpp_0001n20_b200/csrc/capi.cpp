@@ -154,6 +154,7 @@ void gx_ctx_destroy(gx_ctx* ctx) {
   cudaSetDevice(ctx->device);
   if (ctx->stream) cudaStreamSynchronize(ctx->stream);
   if (ctx->nccl) gx_comm_destroy(ctx->nccl);
+  if (ctx->hstage) cudaFreeHost(ctx->hstage);
   if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
   if (ctx->copy_stream) {
     cudaStreamSynchronize(ctx->copy_stream);

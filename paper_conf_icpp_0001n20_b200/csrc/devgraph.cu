@@ -17,6 +17,7 @@
 #include "gx_internal.h"
 #include "kernels_common.cuh"
 #include "sell.cuh"
+#include "dist.h"
 
 namespace gx {
 
@@ -401,6 +402,7 @@ void build_device_slots(gx_graph* g) {
     gptr.push_back((int32_t)gslots.size());
   }
   d.n_groups = (int64_t)gown.size();
+  d.n_gslots = (int64_t)gslots.size();
   // in-edges of each group's owner slot: (src slot, w)
   std::vector<int32_t> gin_ptr(d.n_groups + 1, 0);
   std::vector<uint2> gin;
@@ -475,6 +477,123 @@ void build_device_slots(gx_graph* g) {
   }
   if (!sg.sched.empty()) up(d.sched, sg.sched.data(), sizeof(int32_t) * sg.sched.size());
   CUDA_OK(cudaStreamSynchronize(s));  // host vectors go out of scope
+}
+
+}  // namespace gx
+
+// ---- rank-local PageRank layout of the partitioned path (dist.h) ----
+namespace gx {
+
+__global__ void k_indeg(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj, int64_t n,
+                        uint32_t* __restrict__ cnt) {
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t u = warp; u < n; u += nw)
+    for (uint32_t e = rp[u] + lane_id(); e < rp[u + 1]; e += 32) atomicAdd(&cnt[adj[e].x], 1u);
+}
+// (dst << 32 | src) per out-edge, in source order
+__global__ void k_pairs_u64(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj, int64_t n,
+                            unsigned long long* __restrict__ out) {
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t u = warp; u < n; u += nw)
+    for (uint32_t e = rp[u] + lane_id(); e < rp[u + 1]; e += 32)
+      out[e] = ((unsigned long long)adj[e].x << 32) | (unsigned long long)u;
+}
+__global__ void k_rebase_u32(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, int64_t n1) {
+  const uint32_t b = in[0];
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n1; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = in[i] - b;
+}
+__global__ void k_lo32(const unsigned long long* __restrict__ in, uint32_t* __restrict__ out, int64_t m) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = (uint32_t)in[i];
+}
+struct DstInRange {
+  unsigned long long lo, hi;
+  __host__ __device__ bool operator()(const unsigned long long& p) const {
+    const unsigned long long d = p >> 32;
+    return d >= lo && d < hi;
+  }
+};
+
+// In-CSC of rows [lo, hi) for each rank (all P when `all`, else this rank),
+// balanced by in-edges: the (dst, src) pairs with dst in the range are
+// selected in source order and stably sorted by dst, so each local row lists
+// its sources ascending (the same order as the full CSC); the windowed SELL-32
+// is built over the local rows.  Only the slices stay resident.
+RankLayouts& ensure_pr_ranks(gx_graph* g, int P, bool all) {
+  DevGraph& d = g->dg;
+  RankLayouts& L = d.rk_pr;
+  Ctx* c = g->ctx;
+  const int want_rank = all ? -1 : c->rank;
+  if (L.P == P && L.rank == want_rank) return L;
+  L = RankLayouts();
+  cudaStream_t s = c->stream;
+  const int64_t n = d.n_slots, m = d.m_slots;
+  DBuf cnt, crp;
+  cnt.alloc(c, sizeof(uint32_t) * (n + 1));
+  crp.alloc(c, sizeof(uint32_t) * (n + 1));
+  CUDA_OK(cudaMemsetAsync(cnt.p, 0, sizeof(uint32_t) * (n + 1), s));
+  if (m) k_indeg<<<grid_for(c, n * 32), 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), n, cnt.as<uint32_t>());
+  {
+    size_t tb = 0;
+    CUDA_OK(cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt.as<uint32_t>(), crp.as<uint32_t>(), n + 1, s));
+    DBuf t;
+    t.alloc(c, tb);
+    CUDA_OK(cub::DeviceScan::ExclusiveSum(t.p, tb, cnt.as<uint32_t>(), crp.as<uint32_t>(), n + 1, s));
+  }
+  cnt.reset();
+  std::vector<uint32_t> hcrp(n + 1);
+  CUDA_OK(cudaMemcpyAsync(hcrp.data(), crp.p, sizeof(uint32_t) * (n + 1), cudaMemcpyDeviceToHost, s));
+  CUDA_OK(cudaStreamSynchronize(s));
+  L.bounds = partition_rows(std::vector<int64_t>(hcrp.begin(), hcrp.end()), n, P, PRW_ALIGN);
+  L.P = P;
+  L.rank = want_rank;
+  DBuf pairs;
+  pairs.alloc(c, sizeof(unsigned long long) * std::max<int64_t>(m, 1));
+  if (m) k_pairs_u64<<<grid_for(c, n * 32), 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), n,
+                                                         pairs.as<unsigned long long>());
+  int bits = 1;
+  while ((int64_t(1) << bits) < n) bits++;
+  for (int p = 0; p < P; p++) {
+    if (!all && p != c->rank) continue;
+    RankSlice sl;
+    sl.lo = L.bounds[p];
+    sl.hi = L.bounds[p + 1];
+    const int64_t nl = sl.hi - sl.lo;
+    sl.m = (int64_t)hcrp[sl.hi] - (int64_t)hcrp[sl.lo];
+    sl.crp.alloc(c, sizeof(uint32_t) * (nl + 1));
+    k_rebase_u32<<<grid_for(c, nl + 1), 256, 0, s>>>(crp.as<uint32_t>() + sl.lo, sl.crp.as<uint32_t>(), nl + 1);
+    sl.csrc.alloc(c, sizeof(int32_t) * std::max<int64_t>(sl.m, 1));
+    if (sl.m) {
+      DBuf sel, sel2, nsel, tmp;
+      sel.alloc(c, sizeof(unsigned long long) * sl.m);
+      sel2.alloc(c, sizeof(unsigned long long) * sl.m);
+      nsel.alloc(c, 8);
+      size_t tb = 0;
+      DstInRange pred{(unsigned long long)sl.lo, (unsigned long long)sl.hi};
+      CUDA_OK(cub::DeviceSelect::If(nullptr, tb, pairs.as<unsigned long long>(), sel.as<unsigned long long>(),
+                                    nsel.as<int64_t>(), m, pred, s));
+      tmp.alloc(c, tb);
+      CUDA_OK(cub::DeviceSelect::If(tmp.p, tb, pairs.as<unsigned long long>(), sel.as<unsigned long long>(),
+                                    nsel.as<int64_t>(), m, pred, s));
+      cub::DoubleBuffer<unsigned long long> kb(sel.as<unsigned long long>(), sel2.as<unsigned long long>());
+      size_t sb = 0;
+      CUDA_OK(cub::DeviceRadixSort::SortKeys(nullptr, sb, kb, sl.m, 32, 32 + bits, s));
+      DBuf t2;
+      t2.alloc(c, sb);
+      CUDA_OK(cub::DeviceRadixSort::SortKeys(t2.p, sb, kb, sl.m, 32, 32 + bits, s));
+      k_lo32<<<grid_for(c, sl.m), 256, 0, s>>>(kb.Current(), reinterpret_cast<uint32_t*>(sl.csrc.p), sl.m);
+      CUDA_OK(cudaGetLastError());
+      CUDA_OK(cudaStreamSynchronize(s));   // the scratch buffers go out of scope
+    }
+    build_window_sell<uint32_t>(c, sl.crp.as<uint32_t>(), reinterpret_cast<const uint32_t*>(sl.csrc.p), nl, PR_SENT,
+                                sl.sell);
+    L.r.push_back(std::move(sl));
+  }
+  CUDA_OK(cudaStreamSynchronize(s));
+  return L;
 }
 
 }  // namespace gx

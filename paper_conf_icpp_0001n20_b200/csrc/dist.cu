@@ -6,7 +6,10 @@
 
 namespace gx {
 
-void comm_allreduce(Ctx* c, const void* in, void* out, size_t count, int dtype, int op);  // comm.cpp
+void comm_allreduce(Ctx* c, const void* in, void* out, size_t count, int dtype, int op);             // comm.cpp
+void comm_allgatherv(Ctx* c, void* buf, const std::vector<int64_t>& off, int dtype, size_t esize);   // comm.cpp
+void comm_reduce_scatterv(Ctx* c, void* buf, const std::vector<int64_t>& off, int dtype, int op, size_t esize);
+// ncclDataType / ncclRedOp values (nccl.h)
 enum { NCCL_UINT32 = 3, NCCL_FLOAT32 = 7, NCCL_FLOAT64 = 8 };
 enum { NCCL_SUM = 0, NCCL_MIN = 3 };
 
@@ -38,6 +41,11 @@ std::vector<int64_t> partition_rows_dev(Ctx* c, const uint32_t* rp_dev, int64_t 
   return partition_rows(rp, n, P, align);
 }
 
+static size_t esize(Dt dt) { return dt == Dt::F64 ? 8 : 4; }
+static int nccl_dt(Dt dt) { return dt == Dt::U32 ? NCCL_UINT32 : dt == Dt::F32 ? NCCL_FLOAT32 : NCCL_FLOAT64; }
+static int nccl_op(Op op) { return op == Op::MIN ? NCCL_MIN : NCCL_SUM; }
+
+// ---- simulated ranks: P copies on one device
 struct PtrArr {
   void* p[8];
 };
@@ -55,7 +63,7 @@ __global__ void k_reduce_copies(PtrArr a, int P, int64_t n) {
 }
 
 template <class T, bool MIN>
-static void sim_reduce(Ctx* c, const std::vector<T*>& bufs, int64_t n) {
+static void sim_reduce(Ctx* c, const std::vector<void*>& bufs, int64_t n) {
   if ((int)bufs.size() > 8) GX_THROW(GX_E_UNSUPPORTED, "at most 8 simulated ranks");
   PtrArr a;
   for (size_t q = 0; q < bufs.size(); q++) a.p[q] = bufs[q];
@@ -63,21 +71,74 @@ static void sim_reduce(Ctx* c, const std::vector<T*>& bufs, int64_t n) {
   CUDA_OK(cudaGetLastError());
 }
 
-void Exch::min_u32(const std::vector<uint32_t*>& bufs, int64_t n) {
-  if (sim) sim_reduce<uint32_t, true>(c, bufs, n);
-  else if (P > 1) comm_allreduce(c, bufs[0], bufs[0], (size_t)n, NCCL_UINT32, NCCL_MIN);
+static void sim_allreduce(Ctx* c, const std::vector<void*>& bufs, int64_t n, Dt dt, Op op) {
+  const bool mn = op == Op::MIN;
+  if (dt == Dt::U32) mn ? sim_reduce<uint32_t, true>(c, bufs, n) : sim_reduce<uint32_t, false>(c, bufs, n);
+  else if (dt == Dt::F32) mn ? sim_reduce<float, true>(c, bufs, n) : sim_reduce<float, false>(c, bufs, n);
+  else mn ? sim_reduce<double, true>(c, bufs, n) : sim_reduce<double, false>(c, bufs, n);
 }
-void Exch::sum_f32(const std::vector<float*>& bufs, int64_t n) {
-  if (sim) sim_reduce<float, false>(c, bufs, n);
-  else if (P > 1) comm_allreduce(c, bufs[0], bufs[0], (size_t)n, NCCL_FLOAT32, NCCL_SUM);
+
+// ---- hosted exchange: stage through the context's pinned host buffer
+static void* host_stage(Ctx* c, size_t bytes) {
+  if (c->hstage_bytes < bytes) {
+    if (c->hstage) CUDA_OK(cudaFreeHost(c->hstage));
+    c->hstage = nullptr;
+    c->hstage_bytes = 0;
+    CUDA_OK(cudaMallocHost(&c->hstage, std::max<size_t>(bytes, 4096)));
+    c->hstage_bytes = std::max<size_t>(bytes, 4096);
+  }
+  return c->hstage;
 }
-void Exch::sum_f64(const std::vector<double*>& bufs, int64_t n) {
-  if (sim) sim_reduce<double, false>(c, bufs, n);
-  else if (P > 1) comm_allreduce(c, bufs[0], bufs[0], (size_t)n, NCCL_FLOAT64, NCCL_SUM);
+
+static void hosted(Ctx* c, int kind, void* dbuf, int64_t n, Dt dt, Op op, const std::vector<int64_t>* off) {
+  const size_t es = esize(dt);
+  void* h = host_stage(c, (size_t)n * es);
+  if (n) CUDA_OK(cudaMemcpyAsync(h, dbuf, (size_t)n * es, cudaMemcpyDeviceToHost, c->stream));
+  CUDA_OK(cudaStreamSynchronize(c->stream));
+  const int r = c->coll(kind, h, n, (int32_t)dt, (int32_t)op, off ? off->data() : nullptr, c->world, c->coll_user);
+  if (r != 0) GX_THROW(GX_E_NCCL, "hosted exchange callback failed");
+  if (kind == GX_COLL_REDUCE_SCATTERV) {   // only this rank's slice is defined
+    const int64_t a = (*off)[c->rank], b = (*off)[c->rank + 1];
+    if (b > a)
+      CUDA_OK(cudaMemcpyAsync(static_cast<char*>(dbuf) + a * es, static_cast<char*>(h) + a * es, (size_t)(b - a) * es,
+                              cudaMemcpyHostToDevice, c->stream));
+  } else if (n) {
+    CUDA_OK(cudaMemcpyAsync(dbuf, h, (size_t)n * es, cudaMemcpyHostToDevice, c->stream));
+  }
+  CUDA_OK(cudaStreamSynchronize(c->stream));   // the staging buffer is reused by the next collective
 }
-void Exch::sum_u32(const std::vector<uint32_t*>& bufs, int64_t n) {
-  if (sim) sim_reduce<uint32_t, false>(c, bufs, n);
-  else if (P > 1) comm_allreduce(c, bufs[0], bufs[0], (size_t)n, NCCL_UINT32, NCCL_SUM);
+
+void Exch::allreduce(const std::vector<void*>& bufs, int64_t n, Dt dt, Op op) {
+  if (P <= 1 || n <= 0) return;
+  if (sim) sim_allreduce(c, bufs, n, dt, op);
+  else if (c->coll) hosted(c, GX_COLL_ALLREDUCE, bufs[0], n, dt, op, nullptr);
+  else comm_allreduce(c, bufs[0], bufs[0], (size_t)n, nccl_dt(dt), nccl_op(op));
+}
+
+void Exch::allgatherv(const std::vector<void*>& bufs, const std::vector<int64_t>& off, Dt dt) {
+  if (P <= 1) return;
+  const size_t es = esize(dt);
+  if (sim) {
+    for (int p = 0; p < P; p++) {
+      const int64_t a = off[p], b = off[p + 1];
+      if (b <= a) continue;
+      for (int q = 0; q < P; q++)
+        if (q != p)
+          CUDA_OK(cudaMemcpyAsync(static_cast<char*>(bufs[q]) + a * es, static_cast<char*>(bufs[p]) + a * es,
+                                  (size_t)(b - a) * es, cudaMemcpyDeviceToDevice, c->stream));
+    }
+  } else if (c->coll) {
+    hosted(c, GX_COLL_ALLGATHERV, bufs[0], off[P], dt, Op::SUM, &off);
+  } else {
+    comm_allgatherv(c, bufs[0], off, nccl_dt(dt), es);
+  }
+}
+
+void Exch::reduce_scatterv(const std::vector<void*>& bufs, const std::vector<int64_t>& off, Dt dt, Op op) {
+  if (P <= 1) return;
+  if (sim) sim_allreduce(c, bufs, off[P], dt, op);   // a superset: every slice reduced in every copy
+  else if (c->coll) hosted(c, GX_COLL_REDUCE_SCATTERV, bufs[0], off[P], dt, op, &off);
+  else comm_reduce_scatterv(c, bufs[0], off, nccl_dt(dt), nccl_op(op), esize(dt));
 }
 
 }  // namespace gx

@@ -62,6 +62,10 @@ struct Ctx {
   void* user = nullptr;
   int rank = 0, world = 1;
   void* nccl = nullptr;  // ncclComm_t
+  gx_coll_fn coll = nullptr;   // hosted exchange (gx_ctx_create_hosted): caller's transport
+  void* coll_user = nullptr;
+  void* hstage = nullptr;      // pinned staging buffer of the hosted exchange
+  size_t hstage_bytes = 0;
   int num_sms = 148;
   size_t smem_optin = 0;
   void* dmalloc(size_t b);
@@ -123,6 +127,29 @@ struct PbLayout {
   bool built() const { return q.p != nullptr; }
 };
 
+// Rank-local sweep layouts of the 1-D partitioned path (dist.h): one rank's
+// rows [lo, hi) only.  SSSP: the out-CSR slice (rp rebased to 0, edges
+// packed {dst << wbits | w} when they fit 32 bits, else {dst, w}), its static
+// heavy-chunk list (hc_row = GLOBAL row, hc_start = local edge index) and
+// heavy-row bitmap.  PageRank: the in-CSC slice (crp rebased, csrc = GLOBAL
+// source slots, each row sorted by source) and its windowed SELL-32 (rows
+// local).  Built once per (kind, P) from the slot graph and cached.
+struct RankSlice {
+  int64_t lo = 0, hi = 0, m = 0;
+  DBuf rp, adj, adjp;          // SSSP
+  uint32_t wbits = 0;
+  DBuf hc_row, hc_start, heavy;
+  int64_t nhc = 0;
+  DBuf crp, csrc;              // PageRank
+  SellLayout sell;
+};
+struct RankLayouts {
+  int P = 0;                      // 0: not built
+  int rank = -1;                  // -1: all P slices (simulated ranks)
+  std::vector<int64_t> bounds;    // [P + 1]
+  std::vector<RankSlice> r;       // P slices (simulated) or this rank's slice
+};
+
 // Device layouts of the current slot graph.
 struct DevGraph {
   int64_t n = 0, n_slots = 0, m_slots = 0;
@@ -140,12 +167,13 @@ struct DevGraph {
   DBuf kind;                   // u8 [n_slots] (null in exact mode)
   DBuf gid;                    // i32 [n_slots]: group id or -1 (null if no groups)
   DBuf gptr, gslots;           // groups: ptr [ng+1], slots (owner first)
-  int64_t n_groups = 0;
+  int64_t n_groups = 0, n_gslots = 0;   // groups, and their slots (owners + replicas)
   DBuf g_in_ptr, g_in;         // per-group owner in-edges (src slot, w) for SSSP pull
   // windowed SELL-32 layouts (sell.cu): PR pull over in-edges, SSSP dense
   // push over out-edges
   SellLayout pr_sell, sssp_sell;
   PbLayout pr_pb;              // propagation-blocked PR (built on first use)
+  RankLayouts rk_sssp, rk_pr;  // partitioned path (dist.h): this rank's rows only
   // LB SSSP: static chunk list of rows with out-degree > HEAVY_DEG, heavy bitmap
   int64_t nhc = 0;
   // SSSP block-local mode (sssp.cu): block size the locality was measured for,

@@ -57,8 +57,9 @@ struct PrArgs {
   const uint32_t* crp;
   const int32_t* csrc;
   int64_t nwin;
-  int64_t win_lo, win_hi;  // this rank's windows (dist.h); [0, nwin) on one rank
-  int64_t n_slots;
+  int64_t win_lo, win_hi;  // windows to sweep: [0, nwin)
+  int64_t n_slots;         // rows of the layout (a rank's row count in the partitioned path)
+  int64_t row0;            // global slot of layout row 0 (the rank's first row; 0 on one GPU)
   double* x;
   float* contrib[2];
   const uint32_t* D;
@@ -269,8 +270,8 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell2(PrArgs a) {
     if (bulk && threadIdx.x == 0) {
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       mbar_expect_tx(&bar, PRW * 12);
-      tma_load_1d(s_x, a.x + base, PRW * 8, &bar, pf);
-      tma_load_1d(s_D, a.D + base, PRW * 4, &bar, pf);
+      tma_load_1d(s_x, a.x + a.row0 + base, PRW * 8, &bar, pf);
+      tma_load_1d(s_D, a.D + a.row0 + base, PRW * 4, &bar, pf);
     }
     const int64_t s0 = a.win_slice[w], h0 = a.win_heavy[w];
     const int nh = (int)(a.win_heavy[w + 1] - h0), nit = nh + (int)(a.win_slice[w + 1] - s0);
@@ -324,9 +325,9 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell2(PrArgs a) {
     __syncthreads();
     if (threadIdx.x == 0) s_next = 0;    // published by the barrier below
     for (int i = threadIdx.x; i < nrows; i += PR_CTA) {
-      const double xo = bulk ? s_x[i] : __ldcs(a.x + base + i);
-      const uint32_t Dv = bulk ? s_D[i] : __ldcs(a.D + base + i);
-      pr_finalize<SLOTS>(a, base + i, s_y[i], xo, Dv, addc, cout, my_delta, my_dang, merge_now, sc,
+      const double xo = bulk ? s_x[i] : __ldcs(a.x + a.row0 + base + i);
+      const uint32_t Dv = bulk ? s_D[i] : __ldcs(a.D + a.row0 + base + i);
+      pr_finalize<SLOTS>(a, a.row0 + base + i, s_y[i], xo, Dv, addc, cout, my_delta, my_dang, merge_now, sc,
                                               my_mass);
     }
     __syncthreads();
@@ -1124,58 +1125,88 @@ void ensure_csc(gx_graph* g);  // devgraph.cu
 void ensure_pb(gx_graph* g);   // devgraph.cu
 void ensure_tpv(gx_graph* g);  // tpv.cu
 
-__global__ void k_mask_outside(double* __restrict__ x, int64_t n, int64_t lo, int64_t hi) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-    if (i < lo || i >= hi) x[i] = 0.0;
+RankLayouts& ensure_pr_ranks(gx_graph* g, int P, bool all);   // devgraph.cu
+
+// the three scalars of iteration t (slot (t+1)%3: L1 delta, dangling mass,
+// total mass) to / from the exchange buffer; a stopped loop leaves both alone
+__global__ void k_pr_xch(PrState* st, double* xch, int unpack) {
+  if (st->stop) return;
+  const unsigned k = (st->iter + 1) % 3;
+  if (!unpack) {
+    xch[0] = st->delta[k];
+    xch[1] = st->dang[k];
+    xch[2] = st->mass[k];
+  } else {
+    st->delta[k] = xch[0];
+    st->dang[k] = xch[1];
+    st->mass[k] = xch[2];
+  }
 }
 
-// 1-D partitioned PageRank (dist.h): each rank pulls the windows of its own
-// row range and writes x / next contrib for those rows only; the exchange sums
-// the owned contrib slices (zero elsewhere, so the sum is exact), the L1 delta
-// and the dangling mass, and the owners' new values of replicated vertices;
-// the §2.4 merge then runs identically on every rank.
+// 1-D partitioned PageRank (dist.h): rank p owns slot rows
+// [lo_p, hi_p) (edge-balanced over in-edges) and stores only their in-CSC and
+// windowed SELL (ensure_pr_ranks).  Per iteration:
+//   sweep   k_pr_sell2 over the rank's windows, asynchronous in place inside
+//           the rank (its own contrib slice is updated as it goes; the other
+//           slices hold the previous exchange's values -- a chaotic
+//           relaxation step, Theorem E3 keeps the fixed point)
+//   reduce  ONE allreduce(sum) of [L1 delta, dangling, mass, group values]
+//   gather  allgather(v) of the owned contrib slices (north_star: "allgathers
+//           the rank vector for PageRank")
+//   merge   §2.4 confluence, identical on every rank; advance (stop flag)
+// No host synchronisation inside a batch of check_every iterations: every
+// rank takes the same stop decision from the same reduced scalars, and the
+// host reads the flag once per batch.
 static void run_pagerank_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, const PrArgs& a0, int P,
                               bool sim) {
   Ctx* c = g->ctx;
   cudaStream_t s = c->stream;
   DevGraph& d = g->dg;
   RunState& r = g->rs;
-  const int64_t ns = d.n_slots, ng = std::max<int64_t>(d.n_groups, 1);
-  const std::vector<int64_t> bounds = partition_rows_dev(c, d.crp.as<uint32_t>(), ns, P, PRW_ALIGN);
+  const int64_t ns = d.n_slots, ng = d.n_groups;
+  RankLayouts& RL = ensure_pr_ranks(g, P, sim);
+  const std::vector<int64_t>& bounds = RL.bounds;
   const int nloc = sim ? P : 1;
   struct Rank {
-    DBuf x, c0, c1, gnew, st;
+    DBuf x, cb, xch, st;
     PrArgs a;
-    int64_t lo, hi;
   };
   std::vector<Rank> R(nloc);
   cudaEvent_t e0, e1;
   CUDA_OK(cudaEventCreate(&e0));
   CUDA_OK(cudaEventCreate(&e1));
   CUDA_OK(cudaEventRecord(e0, s));
+  int64_t m_local = 0;
   for (int p = 0; p < nloc; p++) {
     Rank& K = R[p];
+    const RankSlice& sl = RL.r[p];
     DBuf& x = p == 0 ? r.x : K.x;
-    DBuf& c0 = p == 0 ? r.contrib[0] : K.c0;
-    DBuf& c1 = p == 0 ? r.contrib[1] : K.c1;
-    DBuf& gn = p == 0 ? r.gnew : K.gnew;
+    DBuf& cb = p == 0 ? r.contrib[0] : K.cb;
     DBuf& st = p == 0 ? r.pst : K.st;
     x.alloc(c, sizeof(double) * ns);
-    c0.alloc(c, sizeof(float) * ns);
-    c1.alloc(c, sizeof(float) * ns);
-    gn.alloc(c, sizeof(double) * ng);
+    cb.alloc(c, sizeof(float) * ns);
     st.alloc(c, sizeof(PrState));
+    K.xch.alloc(c, sizeof(double) * (3 + ng));
     K.a = a0;
     K.a.x = x.as<double>();
-    K.a.contrib[0] = c0.as<float>();
-    K.a.contrib[1] = c1.as<float>();
-    K.a.gnew = gn.as<double>();
+    K.a.contrib[0] = K.a.contrib[1] = cb.as<float>();   // one buffer: in place inside the rank
+    K.a.gnew = K.xch.as<double>() + 3;                  // group values ride in the fused allreduce
     K.a.st = st.as<PrState>();
-    const int rank = sim ? p : c->rank;
-    K.lo = bounds[rank];
-    K.hi = bounds[rank + 1];
-    K.a.win_lo = K.lo / PRW;
-    K.a.win_hi = (K.hi + PRW - 1) / PRW;
+    K.a.slab = sl.sell.slab.as<uint32_t>();
+    K.a.slice_len = sl.sell.slice_len.as<uint32_t>();
+    K.a.slice_off = sl.sell.slice_off.as<uint64_t>();
+    K.a.lane_row = sl.sell.lane_row.as<int32_t>();
+    K.a.heavy_row = sl.sell.heavy_row.as<int32_t>();
+    K.a.win_slice = sl.sell.win_slice.as<int64_t>();
+    K.a.win_heavy = sl.sell.win_heavy.as<int64_t>();
+    K.a.crp = sl.crp.as<uint32_t>();
+    K.a.csrc = sl.csrc.as<int32_t>();
+    K.a.nwin = sl.sell.nwin;
+    K.a.win_lo = 0;
+    K.a.win_hi = sl.sell.nwin;
+    K.a.n_slots = sl.hi - sl.lo;
+    K.a.row0 = sl.lo;
+    m_local += sl.m;
     pr_state_init(st.as<PrState>(), 1, s);
     if (d.identity) k_pr_init<false><<<grid_for(c, ns), 256, 0, s>>>(K.a, ns, 1.0 / (double)g->n);
     else k_pr_init<true><<<grid_for(c, ns), 256, 0, s>>>(K.a, ns, 1.0 / (double)g->n);
@@ -1185,52 +1216,49 @@ static void run_pagerank_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& in
   X.P = P;
   X.sim = sim;
   int occ = 0;
-  CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell<true, false>, PR_CTA, 0));
-  const int grid = (int)std::max<int64_t>(1, (int64_t)std::max(1, occ) * c->num_sms);
-  const int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 255) / 256, c->num_sms * 4));
-  int launches = nloc, t = 0;
+  CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pr_sell2<true, true>, PR_CTA, 0));
+  const int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((ng + 255) / 256, c->num_sms * 4));
+  std::vector<void*> cbs, xs, xchs;
+  for (int p = 0; p < nloc; p++) {
+    cbs.push_back(R[p].a.contrib[0]);
+    xs.push_back(R[p].a.x);
+    xchs.push_back(R[p].xch.p);
+  }
+  const int batch = std::max(1, o.check_every);
+  int launches = nloc, iters_enq = 0;
   PrState h;
-  for (;; t++) {
-    std::vector<float*> cn;
-    std::vector<double*> dl, dg, gl, ml;
-    for (int p = 0; p < nloc; p++) {
-      PrArgs& A = R[p].a;
-      float* cnext = A.contrib[(t + 1) & 1];
-      CUDA_OK(cudaMemsetAsync(cnext, 0, sizeof(float) * ns, s));
-      if (d.n_groups) CUDA_OK(cudaMemsetAsync(A.gnew, 0, sizeof(double) * ng, s));
-      if (d.identity) k_pr_sell<false, false><<<grid, PR_CTA, 0, s>>>(A);
-      else k_pr_sell<true, false><<<grid, PR_CTA, 0, s>>>(A);
-      launches++;
-      cn.push_back(cnext);
-      dl.push_back(&A.st->delta[0]);
-      dg.push_back(&A.st->dang[0]);
-      ml.push_back(&A.st->mass[0]);
-      gl.push_back(A.gnew);
-    }
-    X.sum_f32(cn, ns);                                  // the exchange
-    X.sum_f64(dl, 3);
-    X.sum_f64(dg, 3);
-    X.sum_f64(ml, 3);
-    if (d.n_groups) X.sum_f64(gl, d.n_groups);
-    for (int p = 0; p < nloc; p++) {
-      if (d.n_groups) {
-        k_pr_merge<<<grid_merge, 256, 0, s>>>(R[p].a, d.gptr.as<int32_t>(), d.gslots.as<int32_t>(), d.n_groups);
+  for (;;) {
+    for (int it = 0; it < batch; it++, iters_enq++) {
+      for (int p = 0; p < nloc; p++) {
+        const PrArgs& A = R[p].a;
+        if (ng) CUDA_OK(cudaMemsetAsync(A.gnew, 0, sizeof(double) * ng, s));
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(A.nwin, (int64_t)std::max(1, occ) * c->num_sms));
+        if (d.identity) k_pr_sell2<false, true><<<grid, PR_CTA, 0, s>>>(A);
+        else k_pr_sell2<true, true><<<grid, PR_CTA, 0, s>>>(A);
+        k_pr_xch<<<1, 1, 0, s>>>(A.st, R[p].xch.as<double>(), 0);
+        launches += 2;
+      }
+      X.allreduce(xchs, 3 + ng, Dt::F64, Op::SUM);   // delta, dangling, mass (+ group values): one collective
+      for (int p = 0; p < nloc; p++) {
+        k_pr_xch<<<1, 1, 0, s>>>(R[p].a.st, R[p].xch.as<double>(), 1);
         launches++;
       }
-      k_pr_advance<<<1, 1, 0, s>>>(R[p].a.st, o.tol, o.max_iters);
-      launches++;
+      X.allgatherv(cbs, bounds, Dt::F32);             // the owned contrib slices -> every rank
+      for (int p = 0; p < nloc; p++) {
+        if (ng) {
+          k_pr_merge<<<grid_merge, 256, 0, s>>>(R[p].a, d.gptr.as<int32_t>(), d.gslots.as<int32_t>(), ng);
+          launches++;
+        }
+        k_pr_advance<<<1, 1, 0, s>>>(R[p].a.st, o.tol, o.max_iters);
+        launches++;
+      }
     }
+    CUDA_OK(cudaGetLastError());
     CUDA_OK(cudaMemcpyAsync(&h, R[0].a.st, sizeof(PrState), cudaMemcpyDeviceToHost, s));
     CUDA_OK(cudaStreamSynchronize(s));
     if (h.stop) break;
   }
-  // assemble x: each slot from the rank that owns it
-  std::vector<double*> xl;
-  for (int p = 0; p < nloc; p++) {
-    k_mask_outside<<<grid_for(c, ns), 256, 0, s>>>(R[p].a.x, ns, R[p].lo, R[p].hi);
-    xl.push_back(R[p].a.x);
-  }
-  X.sum_f64(xl, ns);
+  X.allgatherv(xs, bounds, Dt::F64);   // x: each slot from the rank that owns it
   CUDA_OK(cudaEventRecord(e1, s));
   CUDA_OK(cudaEventSynchronize(e1));
   float ms = 0;
@@ -1241,9 +1269,10 @@ static void run_pagerank_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& in
   info.converged = h.stop == 1 ? 1 : (h.stop == 3 ? 2 : 0);   // 2 = fp32 noise floor (R55)
   info.loop_ms = ms;
   info.last_delta = h.last_delta;
-  info.edges_scanned = (int64_t)h.iter * d.m_slots;
-  info.vertices_active = (int64_t)h.iter * ns;
-  info.bytes_model = (int64_t)h.iter * (8 * d.m_slots + 24 * ns);
+  // this rank's share of the work (the bench sums over ranks)
+  info.edges_scanned = (int64_t)h.iter * (sim ? d.m_slots : m_local);
+  info.vertices_active = (int64_t)h.iter * (sim ? ns : (RL.r[0].hi - RL.r[0].lo));
+  info.bytes_model = 8 * info.edges_scanned + 32 * info.vertices_active;   // SURVEY §8(d) pull model
   info.kernel_launches = launches;
   info.mapping_used = GX_MAP_LB;
   r.have[GX_PAGERANK] = true;
@@ -1272,19 +1301,19 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
                     : (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
   }
   if (mapping == GX_MAP_VNS) mapping = GX_MAP_TPV;   // a pull row is not split (graffix.h)
-  if (P_ranks > 1 || mapping != GX_MAP_PB || tiles) {
-    resolve_pending(g);   // GX_ASYNC_UPLOAD: these layouts read the {col, w} pairs
-    ensure_csc(g);
-  }
-  r.x.alloc(c, sizeof(double) * ns);
-  r.contrib[0].alloc(c, sizeof(float) * ns);
+  if (P_ranks > 1 || mapping != GX_MAP_PB || tiles) resolve_pending(g);   // GX_ASYNC_UPLOAD: these layouts read {col, w}
+  if (P_ranks == 1 && (mapping != GX_MAP_PB || tiles)) ensure_csc(g);   // partitioned: rank-local CSC only
   const bool sim_ = c->world == 1 && o.sim_ranks > 1;
   // the asynchronous schedule keeps ONE contrib buffer (read and written in
   // place by the sweep); Jacobi and the partitioned path need two
   const bool async = o.pr_schedule == GX_PR_ASYNC && c->world == 1 && !sim_;
-  if (!async) r.contrib[1].alloc(c, sizeof(float) * ns);
-  r.gnew.alloc(c, sizeof(double) * std::max<int64_t>(d.n_groups, 1));
-  r.pst.alloc(c, sizeof(PrState));
+  if (P_ranks == 1) {
+    r.x.alloc(c, sizeof(double) * ns);
+    r.contrib[0].alloc(c, sizeof(float) * ns);
+    if (!async) r.contrib[1].alloc(c, sizeof(float) * ns);
+    r.gnew.alloc(c, sizeof(double) * std::max<int64_t>(d.n_groups, 1));
+    r.pst.alloc(c, sizeof(PrState));
+  }
   PrArgs a;
   const SellLayout& PL = d.pr_sell;
   a.slab = PL.slab.as<uint32_t>();
@@ -1300,9 +1329,10 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   a.win_lo = 0;
   a.win_hi = PL.nwin;
   a.n_slots = ns;
+  a.row0 = 0;
   a.x = r.x.as<double>();
   a.contrib[0] = r.contrib[0].as<float>();
-  a.contrib[1] = async ? a.contrib[0] : r.contrib[1].as<float>();
+  a.contrib[1] = async ? a.contrib[0] : r.contrib[1].as<float>();   // (the partitioned path sets its own)
   a.D = d.D.as<uint32_t>();
   a.kind = d.identity ? nullptr : d.kind.as<uint8_t>();
   a.gid = d.n_groups ? d.gid.as<int32_t>() : nullptr;
@@ -1464,9 +1494,10 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   info.last_delta = h.last_delta;
   info.edges_scanned = (int64_t)h.iter * d.m_slots;
   info.vertices_active = (int64_t)h.iter * ns;
-  // bytes model: 8 B per in-edge (source id 4 + contrib gather 4) and
-  // 24 B per slot (x read 8 + x write 8 + contrib write 4 + D 4)
-  info.bytes_model = (int64_t)h.iter * (8 * d.m_slots + 24 * ns);
+  // bytes model (SURVEY.md §8(d) pull model): 8 B per in-edge (source id 4 +
+  // contrib gather 4) and 32 B per slot (row_ptr 8 + x read 8 + x write 8 +
+  // contrib write 4 + D 4)
+  info.bytes_model = (int64_t)h.iter * (8 * d.m_slots + 32 * ns);
   info.kernel_launches = launches;
   info.sweep_launches = kt.launches();
   info.sweep_ms = kt.total_ms();

@@ -125,6 +125,9 @@ __device__ __forceinline__ void clear_bitmap(uint32_t* bm, int64_t nwords) {
 #define GX_SSSP_SU 3
 #endif
 constexpr int SU = GX_SSSP_SU;   // edges in flight per lane per round
+#ifndef GX_SSSP_PIPE
+#define GX_SSSP_PIPE 1
+#endif
 #ifndef GX_SSSP_TPB
 #define GX_SSSP_TPB 256
 #endif
@@ -178,14 +181,23 @@ __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, con
         else a = max(a, le);
         if (a >= b) continue;
       }
+      uint2 ed[SU];
+      bool ok[SU];
+#pragma unroll
+      for (int q = 0; q < SU; q++) {
+        const uint32_t e = a + q * 32 + lane;
+        ok[q] = e < b;
+        ed[q] = ok[q] ? ld_edge(adj, ax, e, pf) : make_uint2(0, 0);
+      }
       for (uint32_t e0 = a; e0 < b; e0 += 32 * SU) {
-        uint2 ed[SU];
-        bool ok[SU];
+        // the next round's edges are loaded before this round's gathers
+        uint2 en[SU];
+        bool kn[SU];
 #pragma unroll
         for (int q = 0; q < SU; q++) {
-          uint32_t e = e0 + q * 32 + lane;
-          ok[q] = e < b;
-          ed[q] = ok[q] ? ld_edge(adj, ax, e, pf) : make_uint2(0, 0);
+          const uint32_t e = e0 + 32 * SU + q * 32 + lane;
+          kn[q] = e < b;
+          en[q] = kn[q] ? ld_edge(adj, ax, e, pf) : make_uint2(0, 0);
         }
         uint32_t cv[SU];
 #pragma unroll
@@ -193,6 +205,11 @@ __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, con
 #pragma unroll
         for (int q = 0; q < SU; q++)
           if (ok[q]) relax_nf(ed[q], du, cv[q], dist, bm_next, ax.far, tau, my_min, my_push, pl);
+#pragma unroll
+        for (int q = 0; q < SU; q++) {
+          ed[q] = en[q];
+          ok[q] = kn[q];
+        }
       }
       if (lane == 0) my_edges += b - a;
     }
@@ -265,10 +282,9 @@ __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, con
       const uint32_t dincl = warp_incl_scan_u32(deg);
       const uint32_t dexcl = dincl - deg;
       const uint32_t dtot = __shfl_sync(FULL, dincl, 31);
-      for (uint32_t k0 = 0; k0 < dtot; k0 += 32 * SU) {
-        uint2 ed[SU];
-        uint32_t od[SU];
-        bool ok[SU];
+      // round k0: the SU edges k0 + q*32 + lane of the batch's concatenated rows
+      // (binary search of the owning row over the warp's exclusive scan)
+      auto fetch = [&](uint32_t k0, uint2 (&ed)[SU], uint32_t (&od)[SU], bool (&ok)[SU]) {
 #pragma unroll
         for (int q = 0; q < SU; q++) {
           const uint32_t kk = k0 + q * 32 + lane;
@@ -284,6 +300,42 @@ __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, con
           ok[q] = kk < dtot;
           ed[q] = ok[q] ? ld_edge(adj, ax, os + (kk - oe), pf) : make_uint2(0, 0);
         }
+      };
+#if GX_SSSP_PIPE
+      // software pipeline: round k0 + 32*SU's edge loads are issued before
+      // round k0's dist gathers, so each lane keeps 2*SU loads in flight and
+      // the edge-stream latency hides behind the gathers'
+      uint2 ed[SU];
+      uint32_t od[SU];
+      bool ok[SU];
+      if (dtot) fetch(0, ed, od, ok);
+      for (uint32_t k0 = 0; k0 < dtot; k0 += 32 * SU) {
+        const bool more = k0 + 32 * SU < dtot;   // warp-uniform
+        uint2 en[SU];
+        uint32_t on[SU];
+        bool kn[SU];
+        if (more) fetch(k0 + 32 * SU, en, on, kn);
+        uint32_t cv[SU];
+#pragma unroll
+        for (int q = 0; q < SU; q++) cv[q] = ok[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
+#pragma unroll
+        for (int q = 0; q < SU; q++)
+          if (ok[q]) relax_nf(ed[q], od[q], cv[q], dist, bm_next, ax.far, tau, my_min, my_push, pl);
+        if (more) {
+#pragma unroll
+          for (int q = 0; q < SU; q++) {
+            ed[q] = en[q];
+            od[q] = on[q];
+            ok[q] = kn[q];
+          }
+        }
+      }
+#else
+      for (uint32_t k0 = 0; k0 < dtot; k0 += 32 * SU) {
+        uint2 ed[SU];
+        uint32_t od[SU];
+        bool ok[SU];
+        fetch(k0, ed, od, ok);
         uint32_t cv[SU];
 #pragma unroll
         for (int q = 0; q < SU; q++) cv[q] = ok[q] ? ld_l2_u32(dist + ed[q].x, pl) : 0u;
@@ -291,6 +343,7 @@ __device__ __forceinline__ void sssp_lb_dev(const uint32_t* __restrict__ rp, con
         for (int q = 0; q < SU; q++)
           if (ok[q]) relax_nf(ed[q], od[q], cv[q], dist, bm_next, ax.far, tau, my_min, my_push, pl);
       }
+#endif
       if (lane == 0) my_edges += dtot;
     }
     __syncwarp();
@@ -893,13 +946,13 @@ __global__ void k_heavy_chunks_count(const uint32_t* __restrict__ rp, int64_t n,
   }
 }
 __global__ void k_heavy_chunks_fill(const uint32_t* __restrict__ rp, int64_t n, const uint32_t* __restrict__ off,
-                                    int32_t* __restrict__ hrow, uint32_t* __restrict__ hstart) {
+                                    int32_t* __restrict__ hrow, uint32_t* __restrict__ hstart, int64_t row_base = 0) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
     const uint32_t d = rp[v + 1] - rp[v];
     if (d <= HEAVY_DEG) continue;
     const uint32_t k = (d + HCHUNK - 1) / HCHUNK, o = off[v];
     for (uint32_t i = 0; i < k; i++) {
-      hrow[o + i] = (int32_t)v;
+      hrow[o + i] = (int32_t)(row_base + v);
       hstart[o + i] = rp[v] + i * HCHUNK;
     }
   }
@@ -1082,23 +1135,116 @@ static void ensure_heavy_chunks(gx_graph* g) {
   CUDA_OK(cudaStreamSynchronize(s));
 }
 
-// owned slots whose distance dropped in this iteration (any rank's relaxation,
-// visible after the allreduce) join this rank's next frontier, or its far
-// pile when the new distance is at or above the near-far threshold
-__global__ void k_frontier_diff(const uint32_t* __restrict__ dist, const uint32_t* __restrict__ dold, SsspAux ax,
-                                SsspState* __restrict__ st, int64_t lo, int64_t hi) {
+// ---------------------------------------------------------------- partitioned path (dist.h)
+// pointer to element -base of a (device) array, so that a rank-local array of
+// rows [lo, hi) is indexed with global row ids u in [lo, hi)
+template <class T>
+static T* shifted(T* p, int64_t base) {
+  return reinterpret_cast<T*>(reinterpret_cast<uintptr_t>(p) - (uintptr_t)(base * (int64_t)sizeof(T)));
+}
+
+__global__ void k_rebase_rows(const uint32_t* __restrict__ rp, int64_t lo, int64_t n1, uint32_t* __restrict__ out) {
+  const uint32_t b = rp[lo];
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n1; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = rp[lo + i] - b;
+}
+
+// Rank-local out-CSR of rows [lo, hi) per rank (all P when `all`, else this
+// rank), balanced by out-edges: rebased row offsets, the edge slice packed to
+// 4 bytes when ids and weights fit, the heavy-chunk list and heavy bitmap.
+static RankLayouts& ensure_sssp_ranks(gx_graph* g, int P, bool all) {
+  DevGraph& d = g->dg;
+  RankLayouts& L = d.rk_sssp;
+  Ctx* c = g->ctx;
+  const int want_rank = all ? -1 : c->rank;
+  if (L.P == P && L.rank == want_rank) return L;
+  L = RankLayouts();
+  cudaStream_t s = c->stream;
+  const int64_t n = d.n_slots;
+  std::vector<uint32_t> hrp(n + 1);
+  CUDA_OK(cudaMemcpyAsync(hrp.data(), d.rp.p, sizeof(uint32_t) * (n + 1), cudaMemcpyDeviceToHost, s));
+  CUDA_OK(cudaStreamSynchronize(s));
+  L.bounds = partition_rows(std::vector<int64_t>(hrp.begin(), hrp.end()), n, P, PRW_ALIGN);
+  L.P = P;
+  L.rank = want_rank;
+  // packing width: the slot graph's largest weight
+  unsigned int wmax = d.max_w;
+  if (!d.identity) {
+    DBuf mx;
+    mx.alloc(c, 4);
+    CUDA_OK(cudaMemsetAsync(mx.p, 0, 4, s));
+    if (d.m_slots) k_adj_wmax<<<grid_for(c, d.m_slots), 256, 0, s>>>(d.adj.as<uint2>(), d.m_slots, mx.as<unsigned int>());
+    CUDA_OK(cudaMemcpyAsync(&wmax, mx.p, 4, cudaMemcpyDeviceToHost, s));
+    CUDA_OK(cudaStreamSynchronize(s));
+  }
+  uint32_t wb = 1;
+  while (wb < 32 && (wmax >> wb)) wb++;
+  const bool pack = !getenv("GX_SSSP_NO_PACK") && wb < 16 && n <= (int64_t(1) << (32 - wb));
+  for (int p = 0; p < P; p++) {
+    if (!all && p != c->rank) continue;
+    RankSlice sl;
+    sl.lo = L.bounds[p];
+    sl.hi = L.bounds[p + 1];
+    const int64_t nl = sl.hi - sl.lo;
+    const int64_t e0 = hrp[sl.lo];
+    sl.m = (int64_t)hrp[sl.hi] - e0;
+    sl.rp.alloc(c, sizeof(uint32_t) * (nl + 1));
+    k_rebase_rows<<<grid_for(c, nl + 1), 256, 0, s>>>(d.rp.as<uint32_t>(), sl.lo, nl + 1, sl.rp.as<uint32_t>());
+    if (pack) {
+      sl.adjp.alloc(c, sizeof(uint32_t) * std::max<int64_t>(sl.m, 1));
+      if (sl.m) k_adj_pack<<<grid_for(c, sl.m), 256, 0, s>>>(d.adj.as<uint2>() + e0, sl.m, wb, sl.adjp.as<uint32_t>());
+      sl.wbits = wb;
+    } else {
+      sl.adj.alloc(c, sizeof(uint2) * std::max<int64_t>(sl.m, 1));
+      if (sl.m)
+        CUDA_OK(cudaMemcpyAsync(sl.adj.p, d.adj.as<uint2>() + e0, sizeof(uint2) * sl.m, cudaMemcpyDeviceToDevice, s));
+    }
+    // heavy chunks of the local rows (hc_row global, hc_start local edge index)
+    DBuf cnt, off, tmp;
+    cnt.alloc(c, sizeof(uint32_t) * (nl + 1));
+    off.alloc(c, sizeof(uint32_t) * (nl + 1));
+    CUDA_OK(cudaMemsetAsync(cnt.p, 0, sizeof(uint32_t) * (nl + 1), s));
+    if (nl) k_heavy_chunks_count<<<grid_for(c, nl), 256, 0, s>>>(sl.rp.as<uint32_t>(), nl, cnt.as<uint32_t>());
+    size_t tb = 0;
+    CUDA_OK(cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt.as<uint32_t>(), off.as<uint32_t>(), nl + 1, s));
+    tmp.alloc(c, tb);
+    CUDA_OK(cub::DeviceScan::ExclusiveSum(tmp.p, tb, cnt.as<uint32_t>(), off.as<uint32_t>(), nl + 1, s));
+    uint32_t nhc = 0;
+    CUDA_OK(cudaMemcpyAsync(&nhc, off.as<uint32_t>() + nl, 4, cudaMemcpyDeviceToHost, s));
+    CUDA_OK(cudaStreamSynchronize(s));
+    sl.nhc = nhc;
+    sl.hc_row.alloc(c, sizeof(int32_t) * std::max<uint32_t>(nhc, 1));
+    sl.hc_start.alloc(c, sizeof(uint32_t) * std::max<uint32_t>(nhc, 1));
+    if (nl)
+      k_heavy_chunks_fill<<<grid_for(c, nl), 256, 0, s>>>(sl.rp.as<uint32_t>(), nl, off.as<uint32_t>(),
+                                                         sl.hc_row.as<int32_t>(), sl.hc_start.as<uint32_t>(), sl.lo);
+    sl.heavy.alloc(c, sizeof(uint32_t) * std::max<int64_t>((nl + 31) / 32, 1));
+    if (nl) k_heavy_bitmap<<<grid_for(c, nl), 256, 0, s>>>(sl.rp.as<uint32_t>(), nl, sl.heavy.as<uint32_t>());
+    CUDA_OK(cudaGetLastError());
+    CUDA_OK(cudaStreamSynchronize(s));
+    L.r.push_back(std::move(sl));
+  }
+  return L;
+}
+
+// after the exchange the owner holds the reduced distances of its rows; a
+// row below its last authoritative value joins the next frontier (or the far
+// pile when at or above tau) and becomes the new authoritative value
+__global__ void k_frontier_apply(const uint32_t* __restrict__ dist, uint32_t* __restrict__ dauth, SsspAux ax,
+                                 SsspState* __restrict__ st, int64_t lo, int64_t hi) {
   if (st->stop) return;
   uint32_t* bm_next = ax.bm[(st->iter + 1) % 3];
   const uint32_t tau = st->tau;
   uint32_t my_min = INF, my_push = 0;
-  const int64_t w_lo = lo >> 5, w_hi = min((hi + 31) >> 5, ax.nwords);
+  const int64_t w_lo = lo >> 5, w_hi = (hi + 31) >> 5;   // lo is 32-aligned
   for (int64_t w = w_lo + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < w_hi; w += (int64_t)gridDim.x * blockDim.x) {
     uint32_t near = 0, far = 0;
     for (int b = 0; b < 32; b++) {
       const int64_t v = w * 32 + b;
-      if (v < lo || v >= hi) continue;
+      if (v >= hi) break;
       const uint32_t nd = dist[v];
-      if (nd >= dold[v]) continue;
+      if (nd >= dauth[v - lo]) continue;
+      dauth[v - lo] = nd;
       if (nd < tau) {
         near |= 1u << b;
       } else {
@@ -1113,16 +1259,63 @@ __global__ void k_frontier_diff(const uint32_t* __restrict__ dist, const uint32_
   flush_counters(st, st->iter, 0, 0, my_push, my_min);
 }
 
+// the merge changed group slots on every rank identically: their new values
+// become the owners' authoritative values
+__global__ void k_auth_groups(const uint32_t* __restrict__ dist, uint32_t* __restrict__ dauth,
+                              const int32_t* __restrict__ gslots, int64_t nslots, int64_t lo, int64_t hi,
+                              const SsspState* __restrict__ st) {
+  if (st->stop) return;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nslots; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t v = gslots[i];
+    if (v >= lo && v < hi) dauth[v - lo] = dist[v];
+  }
+}
+
+__global__ void k_init_auth(const uint32_t* __restrict__ dist, uint32_t* __restrict__ dauth, int64_t lo, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    dauth[i] = dist[lo + i];
+}
+
+// the frontier counters of iteration t (active, pushed) and the far-pile
+// minimum to / from the exchange buffers; a stopped loop leaves both alone
+__global__ void k_sssp_xch(SsspState* st, uint32_t* xs, int unpack) {
+  if (st->stop) return;
+  const unsigned k = st->iter % 3;
+  if (!unpack) {
+    xs[0] = st->active[k];
+    xs[1] = st->pushed[k];
+    xs[2] = st->far_min;
+  } else {
+    st->active[k] = xs[0];
+    st->pushed[k] = xs[1];
+    st->far_min = xs[2];
+  }
+}
+
 struct SsspRank {
-  DBuf dist, mark, st, dold;
+  DBuf dist, mark, st, dauth, xs;
   SsspAux ax{};
+  const uint32_t* rp = nullptr;   // rank-local row offsets, indexed by global row
+  const uint2* adj = nullptr;
   int64_t lo = 0, hi = 0;
 };
 
-// 1-D partitioned SSSP (dist.h): each rank relaxes the frontier slots of its
-// own range; after every sweep dist is allreduced with min, the owners rebuild
-// their next frontier from the distances that dropped, and the frontier
-// counters are allreduced so every rank takes the same near-far decision.
+// 1-D partitioned SSSP (dist.h): rank p owns slot rows
+// [lo_p, hi_p) (edge-balanced over out-edges) and stores only their out-CSR
+// (ensure_sssp_ranks).  Per iteration:
+//   sweep   k_sssp_lb over the rank's frontier rows, relaxing into its
+//           full-length copy of dist (fire-and-forget red.min)
+//   reduce  reduce-scatter(min) of dist onto the owners' ranges -- a rank only
+//           ever reads authoritative values of its own rows (the heads of the
+//           edges it relaxes); stale copies of other rows are upper bounds,
+//           so they can only cost extra pushes.  With replica groups the
+//           reduction is an allreduce(min): the §2.4 merge needs every copy
+//   apply   the owners turn rows that dropped below their last authoritative
+//           value into the next frontier / far pile (no full-vector copy:
+//           the authoritative values are rank-local, n/P)
+//   counters one sum of (active, pushed) and one min of the far minimum, so
+//           every rank takes the same near-far decision; advance / refill
+// No host synchronisation inside a batch of check_every iterations.
 static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, int P, bool sim, int64_t src,
                           unsigned delta) {
   Ctx* c = g->ctx;
@@ -1130,7 +1323,8 @@ static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, 
   DevGraph& d = g->dg;
   RunState& r = g->rs;
   const int64_t ns = d.n_slots, nwords = (ns + 31) / 32;
-  const std::vector<int64_t> bounds = partition_rows_dev(c, d.rp.as<uint32_t>(), ns, P, PRW_ALIGN);
+  RankLayouts& RL = ensure_sssp_ranks(g, P, sim);
+  const std::vector<int64_t>& bounds = RL.bounds;
   const int nloc = sim ? P : 1;
   std::vector<SsspRank> R(nloc);
   std::vector<int32_t> srcs{d.identity ? (int32_t)src : g->sg.owner_slot[src]};
@@ -1154,27 +1348,33 @@ static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, 
   CUDA_OK(cudaEventRecord(e0, s));
   for (int p = 0; p < nloc; p++) {
     SsspRank& K = R[p];
+    const RankSlice& sl = RL.r[p];
     DBuf& dist = p == 0 ? r.dist : K.dist;
     DBuf& mark = p == 0 ? r.mark : K.mark;
     DBuf& st = p == 0 ? r.st : K.st;
     dist.alloc(c, sizeof(uint32_t) * ns);
     mark.alloc(c, sizeof(uint32_t) * 4 * nwords);
     st.alloc(c, sizeof(SsspState));
-    K.dold.alloc(c, sizeof(uint32_t) * ns);
+    K.lo = sl.lo;
+    K.hi = sl.hi;
+    K.dauth.alloc(c, sizeof(uint32_t) * std::max<int64_t>(K.hi - K.lo, 1));
+    K.xs.alloc(c, sizeof(uint32_t) * 4);
     for (int i = 0; i < 3; i++) K.ax.bm[i] = mark.as<uint32_t>() + i * nwords;
     K.ax.far = mark.as<uint32_t>() + 3 * nwords;
-    K.ax.heavy = d.heavy_bm.as<uint32_t>();
+    K.ax.heavy = shifted(sl.heavy.as<uint32_t>(), K.lo >> 5);
     K.ax.nwords = nwords;
-    K.ax.hc_row = d.hc_row.as<int32_t>();
-    K.ax.hc_start = d.hc_start.as<uint32_t>();
-    K.ax.nhc = d.nhc;
-    const int rank = sim ? p : c->rank;
-    K.lo = bounds[rank];
-    K.hi = bounds[rank + 1];
+    K.ax.hc_row = sl.hc_row.as<int32_t>();
+    K.ax.hc_start = sl.hc_start.as<uint32_t>();
+    K.ax.nhc = sl.nhc;
+    K.ax.adjp = sl.adjp.p ? sl.adjp.as<uint32_t>() : nullptr;
+    K.ax.wbits = sl.wbits;
+    K.rp = shifted(sl.rp.as<uint32_t>(), K.lo);
+    K.adj = sl.adj.p ? sl.adj.as<uint2>() : nullptr;
     CUDA_OK(cudaMemsetAsync(dist.p, 0xFF, sizeof(uint32_t) * ns, s));
     CUDA_OK(cudaMemsetAsync(mark.p, 0, sizeof(uint32_t) * 4 * nwords, s));
     CUDA_OK(cudaMemcpyAsync(st.p, &init, sizeof(SsspState), cudaMemcpyHostToDevice, s));
     k_sssp_init<<<1, 32, 0, s>>>(dist.as<uint32_t>(), dsrc.as<int32_t>(), (int)srcs.size(), K.ax.bm[0]);
+    if (K.hi > K.lo) k_init_auth<<<grid_for(c, K.hi - K.lo), 256, 0, s>>>(dist.as<uint32_t>(), K.dauth.as<uint32_t>(), K.lo, K.hi - K.lo);
   }
   auto D = [&](int p) { return (p == 0 ? r.dist : R[p].dist).as<uint32_t>(); };
   auto S = [&](int p) { return (p == 0 ? r.st : R[p].st).as<SsspState>(); };
@@ -1188,48 +1388,63 @@ static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, 
   const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 8));
   const int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 7) / 8, (int64_t)c->num_sms * 8));
   const bool merge_min = g->knobs.merge_op == GX_MERGE_MIN;
-  int launches = 0;
-  SsspState hst;
-  std::vector<uint32_t*> dl, al, fl;
+  std::vector<void*> dl, xsl, xml;
   for (int p = 0; p < nloc; p++) {
     dl.push_back(D(p));
-    al.push_back(&S(p)->active[0]);
-    fl.push_back(&S(p)->far_min);
+    xsl.push_back(R[p].xs.p);
+    xml.push_back(R[p].xs.as<uint32_t>() + 2);
   }
+  const int batch = std::max(1, o.check_every);
+  int launches = 0;
+  SsspState hst;
   for (;;) {
-    for (int p = 0; p < nloc; p++) {
-      CUDA_OK(cudaMemcpyAsync(R[p].dold.p, D(p), sizeof(uint32_t) * ns, cudaMemcpyDeviceToDevice, s));
-      k_sssp_lb<<<grid_lb, 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), D(p), R[p].ax, S(p), R[p].lo, R[p].hi);
-      launches++;
-      if (d.n_tiles && g->knobs.smem) {
-        k_sssp_local<<<grid_local, 256, 0, s>>>(d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(), d.t_eptr.as<int32_t>(),
-                                                d.t_edges.as<uint2>(), d.t_iters.as<int32_t>(), d.n_tiles, D(p), R[p].ax,
-                                                S(p), nullptr, nullptr);
+    for (int it = 0; it < batch; it++) {
+      for (int p = 0; p < nloc; p++) {
+        k_sssp_lb<<<grid_lb, 256, 0, s>>>(R[p].rp, R[p].adj, D(p), R[p].ax, S(p), R[p].lo, R[p].hi);
+        launches++;
+        if (d.n_tiles && g->knobs.smem) {
+          k_sssp_local<<<grid_local, 256, 0, s>>>(d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(), d.t_eptr.as<int32_t>(),
+                                                  d.t_edges.as<uint2>(), d.t_iters.as<int32_t>(), d.n_tiles, D(p), R[p].ax,
+                                                  S(p), nullptr, nullptr);
+          launches++;
+        }
+      }
+      if (d.n_groups) X.allreduce(dl, ns, Dt::U32, Op::MIN);     // the merge reads every copy
+      else X.reduce_scatterv(dl, bounds, Dt::U32, Op::MIN);      // owners' ranges only
+      for (int p = 0; p < nloc; p++) {
+        k_frontier_apply<<<grid_for(c, (R[p].hi - R[p].lo + 31) / 32 + 1), 256, 0, s>>>(D(p), R[p].dauth.as<uint32_t>(),
+                                                                                         R[p].ax, S(p), R[p].lo, R[p].hi);
+        launches++;
+        if (d.n_groups) {
+          k_sssp_merge<<<grid_merge, 256, 0, s>>>(d.gptr.as<int32_t>(), d.gslots.as<int32_t>(), d.g_in_ptr.as<int32_t>(),
+                                                  d.g_in.as<uint2>(), d.n_groups, merge_min ? 1 : 0, D(p), R[p].ax, S(p));
+          k_auth_groups<<<grid_for(c, d.n_gslots), 256, 0, s>>>(D(p), R[p].dauth.as<uint32_t>(), d.gslots.as<int32_t>(),
+                                                                d.n_gslots, R[p].lo, R[p].hi, S(p));
+          launches += 2;
+        }
+        k_sssp_xch<<<1, 1, 0, s>>>(S(p), R[p].xs.as<uint32_t>(), 0);
         launches++;
       }
-    }
-    X.min_u32(dl, ns);                                  // the exchange
-    for (int p = 0; p < nloc; p++) {
-      if (d.n_groups) {
-        k_sssp_merge<<<grid_merge, 256, 0, s>>>(d.gptr.as<int32_t>(), d.gslots.as<int32_t>(), d.g_in_ptr.as<int32_t>(),
-                                                d.g_in.as<uint2>(), d.n_groups, merge_min ? 1 : 0, D(p), R[p].ax, S(p));
-        launches++;
+      X.allreduce(xsl, 2, Dt::U32, Op::SUM);   // active, pushed of iteration t
+      X.allreduce(xml, 1, Dt::U32, Op::MIN);   // far-pile minimum: the same bucket decision everywhere
+      for (int p = 0; p < nloc; p++) {
+        k_sssp_xch<<<1, 1, 0, s>>>(S(p), R[p].xs.as<uint32_t>(), 1);
+        k_sssp_advance<<<1, 1, 0, s>>>(S(p), o.max_iters);
+        k_sssp_split<<<grid_for(c, nwords), 256, 0, s>>>(D(p), R[p].ax, S(p), R[p].lo, R[p].hi);
+        launches += 3;
       }
-      k_frontier_diff<<<grid_for(c, nwords), 256, 0, s>>>(D(p), R[p].dold.as<uint32_t>(), R[p].ax, S(p), R[p].lo,
-                                                           R[p].hi);
-      launches++;
     }
-    X.sum_u32(al, 6);                                   // active[3] + pushed[3]
-    X.min_u32(fl, 1);                                   // every rank takes the same bucket decision
-    for (int p = 0; p < nloc; p++) {
-      k_sssp_advance<<<1, 1, 0, s>>>(S(p), o.max_iters);
-      k_sssp_split<<<grid_for(c, nwords), 256, 0, s>>>(D(p), R[p].ax, S(p), R[p].lo, R[p].hi);
-      launches += 2;
-    }
+    CUDA_OK(cudaGetLastError());
     CUDA_OK(cudaMemcpyAsync(&hst, S(0), sizeof(SsspState), cudaMemcpyDeviceToHost, s));
     CUDA_OK(cudaStreamSynchronize(s));
     if (hst.stop) break;
   }
+  // result: each rank's authoritative rows -> every rank
+  for (int p = 0; p < nloc; p++)
+    if (R[p].hi > R[p].lo)
+      CUDA_OK(cudaMemcpyAsync(D(p) + R[p].lo, R[p].dauth.p, sizeof(uint32_t) * (R[p].hi - R[p].lo),
+                              cudaMemcpyDeviceToDevice, s));
+  X.allgatherv(dl, bounds, Dt::U32);
   unsigned long long edges = 0;
   for (int p = 0; p < nloc; p++) {
     SsspState h;
@@ -1246,10 +1461,11 @@ static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, 
   info.iterations = (int32_t)hst.iter;
   info.converged = hst.stop == 1;
   info.loop_ms = ms;
-  info.edges_scanned = (int64_t)edges;
-  info.vertices_active = (int64_t)hst.act_total;
-  info.bytes_model = 12 * (int64_t)edges + 12 * (int64_t)hst.act_total;
+  info.edges_scanned = (int64_t)edges;                 // this rank's relaxations (all simulated ranks when sim)
+  info.vertices_active = (int64_t)hst.act_total;       // global (the counters are reduced)
+  info.bytes_model = 12 * (int64_t)edges + 14 * (int64_t)hst.act_total / (sim ? 1 : P);
   info.kernel_launches = launches;
+  info.mapping_used = GX_MAP_LB;
   r.have[GX_SSSP] = true;
 }
 
@@ -1274,7 +1490,6 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
     GX_CHECK_ARG(P <= 8, "at most 8 ranks");
     GX_CHECK_ARG(o.mapping != GX_MAP_TPV && o.mapping != GX_MAP_VNS, "the partitioned path uses the LB mapping");
     GX_CHECK_ARG(o.merge_every == 1 || !d.n_groups, "the partitioned path merges after every iteration");
-    ensure_heavy_chunks(g);
     unsigned delta = sssp_delta(g);
     if (const char* e = getenv("GX_SSSP_DELTA")) delta = (unsigned)std::max(0, atoi(e));
     run_sssp_dist(g, o, info, P, sim, src, delta);

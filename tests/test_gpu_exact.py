@@ -30,7 +30,13 @@ GRAPHS = {
 
 @pytest.mark.parametrize("name", list(GRAPHS))
 @pytest.mark.parametrize("mode", ["graphs", "eager1"])
-def test_sssp_exact_bit_exact(name, mode):
+@pytest.mark.parametrize("pack", ["packed", "unpacked"])
+def test_sssp_exact_bit_exact(name, mode, pack, monkeypatch):
+    """pack=unpacked (GX_SSSP_NO_PACK=1) forces the {dst, w} 8-byte edge stream
+    that every graph whose slot ids and weights need more than 32 bits takes
+    (C5: RMAT-26, 26 + 7 bits), heavy chunks included (star_hub)."""
+    if pack == "unpacked":
+        monkeypatch.setenv("GX_SSSP_NO_PACK", "1")
     raw = GRAPHS[name]()
     g = from_raw(raw)
     s = sssp_source(g)
@@ -206,6 +212,9 @@ FULL = {   # BASELINE.json's configurations at their full sizes
     "C3_road4900": (lambda: graphgen.road(4900), None),
     "C4_uniform16M_256M": (lambda: graphgen.uniform(1 << 24, 1 << 28), None),
     "C2_rmat22_coalesce": (lambda: graphgen.rmat(22), dict(coalesce=True, chunk_k=16, replicate_threshold=0.6)),
+    # the paper's rmat26 (P@35940): 2^26 slots x 7 weight bits do not pack into
+    # 32 bits, so SSSP streams the unpacked {dst, w} edges (the C5 path)
+    "C5_rmat26": (lambda: graphgen.rmat(26), None),
 }
 
 
@@ -230,6 +239,8 @@ def test_full_size_certificates(cfg):
     s = sssp_source(g)
     r = G.run("sssp", source=-1, mapping="lb")
     assert r["converged"] == 1
+    if cfg == "C5_rmat26":
+        assert r["sweep_bytes"] == 12 * r["edges_scanned"] + 12 * r["vertices_active"], "expected the unpacked stream"
     dist = G.download("dist")
     cert = sssp_certificate(g, s, dist)
     assert cert["ok"], cert
@@ -252,13 +263,16 @@ def test_full_size_certificates(cfg):
 
 @pytest.mark.parametrize("name", ["rmat12", "uniform", "road64", "star_hub", "dups_loops", "isolated"])
 @pytest.mark.parametrize("persist,block", [("0", None), ("1", "0"), ("1", "1")])
-def test_sssp_loop_modes_bit_exact(name, persist, block, monkeypatch):
+@pytest.mark.parametrize("pack", ["packed", "unpacked"])
+def test_sssp_loop_modes_bit_exact(name, persist, block, pack, monkeypatch):
     """Every LB loop variant reaches Dijkstra exactly: per-kernel launches
     (GX_SSSP_PERSIST=0), the cooperative persistent loop, and its block-local
     mode (shared-memory queues over contiguous id blocks) forced on any graph."""
     monkeypatch.setenv("GX_SSSP_PERSIST", persist)
     if block is not None:
         monkeypatch.setenv("GX_SSSP_BLOCK", block)
+    if pack == "unpacked":
+        monkeypatch.setenv("GX_SSSP_NO_PACK", "1")
     raw = GRAPHS[name]()
     g = from_raw(raw)
     want = A.sssp_dijkstra(graph_to_edgelist(g), sssp_source(g))
