@@ -813,6 +813,8 @@ struct SsspLoop {
   const int32_t* slot_tile;
   uint32_t* tmark;
   int32_t* tlist;
+  unsigned long long* trace;   // GX_SSSP_PTRACE: per iteration {globaltimer ns, edges so far, active, tau}
+  int trace_cap;
 };
 
 constexpr int PERSIST_POOL = SB_WARPS * 1024 * 4;   // 32 KB at 256 threads: LB compaction buffer / block-mode queues
@@ -907,6 +909,14 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
       rf = fm;
     }
     if (!stop && (int)(t + 1) >= a.max_iters) stop = 2;
+    if (lead && a.trace && (int)t < a.trace_cap) {
+      unsigned long long ns;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(ns));
+      a.trace[4 * t] = ns;
+      a.trace[4 * t + 1] = *(volatile unsigned long long*)&st->edges;
+      a.trace[4 * t + 2] = *(volatile unsigned*)&st->active[t % 3];
+      a.trace[4 * t + 3] = tau;
+    }
     if (lead) {
       st->act_total += st->active[t % 3];
       st->active[(t + 2) % 3] = 0;
@@ -925,6 +935,12 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
       grid.sync();
     }
   }
+}
+
+__global__ void k_stamp(unsigned long long* p) {
+  unsigned long long ns;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(ns));
+  *p = ns;
 }
 
 __global__ void k_sssp_init(uint32_t* __restrict__ dist, const int32_t* __restrict__ slots, int nslots,
@@ -1716,14 +1732,39 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
       L.ax.pend[0] = r.mark.as<uint32_t>() + 4 * nwords;
       L.ax.pend[1] = r.mark.as<uint32_t>() + 5 * nwords;
     }
+    // GX_SSSP_PTRACE=1: per-iteration timestamps of the persistent loop (stderr)
+    DBuf trace_buf;
+    L.trace = nullptr;
+    L.trace_cap = 0;
+    if (getenv("GX_SSSP_PTRACE")) {
+      L.trace_cap = 1 << 16;
+      trace_buf.alloc(c, sizeof(unsigned long long) * 4 * (L.trace_cap + 1));
+      L.trace = trace_buf.as<unsigned long long>() + 4;
+      unsigned long long t0 = 0;
+      CUDA_OK(cudaMemsetAsync(trace_buf.p, 0, 32, s));
+      (void)t0;
+    }
     void* args[] = {&L};
     kt.begin();
+    if (L.trace) k_stamp<<<1, 1, 0, s>>>(trace_buf.as<unsigned long long>());
     CUDA_OK(cudaLaunchCooperativeKernel((void*)k_sssp_persist, dim3((unsigned)(occp * c->num_sms)), dim3(PERSIST_TPB), args,
                                         0, s));
     kt.end();
     launches += 1;
     CUDA_OK(cudaMemcpyAsync(&hst, st, sizeof(SsspState), cudaMemcpyDeviceToHost, s));
     CUDA_OK(cudaStreamSynchronize(s));
+    if (L.trace) {
+      const int nt = std::min<int>((int)hst.iter, L.trace_cap);
+      std::vector<unsigned long long> h(4 * (nt + 1));
+      CUDA_OK(cudaMemcpy(h.data(), trace_buf.p, sizeof(unsigned long long) * h.size(), cudaMemcpyDeviceToHost));
+      unsigned long long prev_e = 0;
+      for (int t = 0; t < nt; t++) {
+        const unsigned long long* r = &h[4 * (t + 1)];
+        fprintf(stderr, "sssp-ptrace t=%d us=%.2f act=%llu edges=%llu tau=%llu\n", t, (r[0] - h[4 * t]) * 1e-3, r[2],
+                r[1] - prev_e, r[3]);
+        prev_e = r[1];
+      }
+    }
   }
   while (!persist) {
     if (gexec) {

@@ -4,7 +4,7 @@
 TAG=${1:-r1}
 python -m paper_conf_icpp_0001n20_b200.build > /dev/null
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_bench_$TAG.csv \
-    python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/bench_under_ncu_$TAG.log 2>&1
+    python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-e2e --no-knobs > gpurun_out/bench_under_ncu_$TAG.log 2>&1
 ncu --set full --clock-control none --import-source on -k regex:"k_pr_pb" -s 5 -c 1 -o gpurun_out/prof_prpb_$TAG \
     python tools/prof_run.py --scale 24 --algos pagerank --mapping pb > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:"k_sssp_persist" -s 1 -c 1 -o gpurun_out/prof_ssspLB_$TAG \
