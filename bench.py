@@ -313,7 +313,10 @@ def main():
     for name, idx in ((sssp_kernel, 0), (pr_kernel, 1)):
         if world == 1:
             ms = sum(r[idx]["sweep_ms"] for r in runs)
-            nl = sum(r[idx]["sweep_launches"] for r in runs)
+            # SSSP: the one cooperative launch per run; PR: the sweeps that did work
+            # (a CUDA-graph batch may end with launches that return at once after
+            # convergence; their ~3 us stay in ms, so this slightly under-claims)
+            nl = sum(r[idx]["sweep_launches"] if idx == 0 else r[idx]["iterations"] for r in runs)
         else:
             ms = sum(r[idx]["loop_ms"] for r in runs)
             nl = len(runs)
