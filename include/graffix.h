@@ -84,6 +84,10 @@ typedef enum { GX_MAP_AUTO = 0, GX_MAP_LB = 1, GX_MAP_TPV = 2, GX_MAP_PB = 3, GX
 #define GX_VALIDATE 2u        /* check monotone row_ptr, col range, weights >= 1 */
 #define GX_CANONICAL 4u       /* caller asserts: no self-loops, no duplicates    */
 #define GX_DL_ASYNC 16u       /* gx_download: see there                          */
+#define GX_W_U8 32u           /* gx_graph_upload_csr: w points to uint8_t weights
+                                 (1..255), widened to 32 bits on the device: a
+                                 quarter of the weights' PCIe bytes; device
+                                 pointers need GX_CANONICAL                      */
 #define GX_ASYNC_UPLOAD 8u    /* with GX_CANONICAL and host pointers, no GX_VALIDATE:
                                  the weights are copied on a second stream; see below */
 
@@ -282,6 +286,7 @@ gx_status gx_ctx_stream(gx_ctx* ctx, void** stream_out);
  * joins the copy: gx_run of any other algorithm or mapping, gx_transform,
  * gx_export_*, gx_sync or gx_graph_destroy.  Pinned host memory is needed for
  * the copies to overlap anything.
+ * GX_W_U8: w is read as m uint8_t values (the paper-style weights 1..100 fit).
  * Errors: GX_E_INVALID (n < 0, m < 0, with GX_VALIDATE: non-monotone row_ptr,
  * col out of [0,n), w = 0), GX_E_UNSUPPORTED (m >= 2^32 or n >= 2^31). */
 gx_status gx_graph_upload_csr(gx_ctx* ctx, gx_graph** out, int64_t n, int64_t m,

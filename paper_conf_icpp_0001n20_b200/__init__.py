@@ -19,7 +19,7 @@ import numpy as np
 
 from ._binding import (ALGOS, ALLOC_FN, COLL_FN, GX_COLL_ALLGATHERV, GX_COLL_ALLREDUCE, GX_COLL_REDUCE_SCATTERV,
                        GX_DT_F32, GX_DT_F64, GX_DT_U32, GX_OP_MIN, GX_ASYNC_UPLOAD, GX_CANONICAL, GX_DL_ASYNC, GX_MAP_AUTO, GX_MAP_LB, GX_MAP_PB, GX_MAP_TPV, GX_MAP_VNS, GX_OUT_BC_F64,
-                       GX_OUT_DIST_U32, GX_OUT_LABEL_I32, GX_OUT_MST_WEIGHT_U64, GX_OUT_RANK_F64,
+                       GX_OUT_DIST_U32, GX_OUT_LABEL_I32, GX_OUT_MST_WEIGHT_U64, GX_OUT_RANK_F64, GX_W_U8,
                        GX_PTRS_DEVICE, GX_PTRS_HOST, GX_VALIDATE, RELEASE_FN, GraffixError, GxExport,
                        GxExportSizes, GxKnobs, GxRunInfo, GxRunOpts, GxTransformInfo, _check, _ptr, lib)
 
@@ -208,16 +208,19 @@ class Graph:
                async_upload: bool = False):
         """Upload a CSR graph.  numpy arrays => host pointers; torch CUDA tensors => device.
         async_upload (GX_ASYNC_UPLOAD, with canonical host arrays): the weights are copied on a
-        second stream; the arrays are kept referenced by the Graph until it is closed."""
+        second stream; the arrays are kept referenced by the Graph until it is closed.
+        uint8 weights (numpy uint8 / torch uint8) are uploaded as bytes (GX_W_U8) and widened
+        on the device."""
         dev = hasattr(row_ptr, "is_cuda") and row_ptr.is_cuda
+        w8 = w is not None and str(getattr(w, "dtype", "")) in ("uint8", "torch.uint8")
         if not dev:
             row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
             col = np.ascontiguousarray(col, dtype=np.int32)
-            w = None if w is None else np.ascontiguousarray(w, dtype=np.uint32)
+            w = None if w is None else np.ascontiguousarray(w, dtype=np.uint8 if w8 else np.uint32)
         n = int(row_ptr.shape[0]) - 1
         m = int(col.shape[0])
         flags = (GX_PTRS_DEVICE if dev else GX_PTRS_HOST) | (GX_VALIDATE if validate else 0) | \
-            (GX_CANONICAL if canonical else 0) | (GX_ASYNC_UPLOAD if async_upload else 0)
+            (GX_CANONICAL if canonical else 0) | (GX_ASYNC_UPLOAD if async_upload else 0) | (GX_W_U8 if w8 else 0)
         h = C.c_void_p()
         _check(lib().gx_graph_upload_csr(ctx._h, C.byref(h), n, m, _ptr(row_ptr), _ptr(col), _ptr(w), flags))
         G = cls(ctx, h)

@@ -23,7 +23,7 @@ ALGOS = {"sssp": GX_SSSP, "pagerank": GX_PAGERANK, "pr": GX_PAGERANK, "scc": GX_
          "bc": GX_BC}
 GX_MERGE_MEAN, GX_MERGE_MIN = 0, 1
 GX_MAP_AUTO, GX_MAP_LB, GX_MAP_TPV, GX_MAP_PB, GX_MAP_VNS = 0, 1, 2, 3, 4
-GX_PTRS_HOST, GX_PTRS_DEVICE, GX_VALIDATE, GX_CANONICAL, GX_ASYNC_UPLOAD, GX_DL_ASYNC = 0, 1, 2, 4, 8, 16
+GX_PTRS_HOST, GX_PTRS_DEVICE, GX_VALIDATE, GX_CANONICAL, GX_ASYNC_UPLOAD, GX_DL_ASYNC, GX_W_U8 = 0, 1, 2, 4, 8, 16, 32
 GX_OUT_DIST_U32, GX_OUT_RANK_F64, GX_OUT_LABEL_I32, GX_OUT_BC_F64, GX_OUT_MST_WEIGHT_U64 = 1, 2, 3, 4, 5
 
 # every symbol include/graffix.h declares (checked by tests/test_capi_symbols.py)

@@ -60,7 +60,7 @@ void DBuf::alloc(Ctx* c, size_t b) {
 
 // upload helpers implemented in devgraph.cu
 void device_upload_input(gx_graph* g, const int64_t* rp, const int32_t* col, const uint32_t* w,
-                         bool device_ptrs, bool validate, bool async = false);
+                         bool device_ptrs, bool validate, bool async = false, bool w8 = false);
 
 }  // namespace gx
 
@@ -189,10 +189,21 @@ gx_status gx_graph_upload_csr(gx_ctx* ctx, gx_graph** out, int64_t n, int64_t m,
   g->ctx = ctx;
   gx_knobs_default(&g->knobs);
   try {
+    std::vector<uint32_t> w_wide;   // GX_W_U8 on the canonicalising path: widened on the host
+    if ((flags & GX_W_U8) && w && !(flags & GX_CANONICAL)) {
+      std::vector<uint8_t> w_b(m);
+      if (m) CUDA_OK(cudaMemcpy(w_b.data(), w, m, dev ? cudaMemcpyDeviceToHost : cudaMemcpyHostToHost));
+      w_wide.assign(w_b.begin(), w_b.end());
+      if (dev) {   // the canonicalising path reads every array back from the device anyway
+        GX_THROW(GX_E_INVALID, "GX_W_U8 with device pointers needs GX_CANONICAL");
+      }
+      w = w_wide.data();
+    }
     if (flags & GX_CANONICAL) {
       g->n = n;
       g->m = m;
-      device_upload_input(g, row_ptr, col, w, dev, validate, (flags & GX_ASYNC_UPLOAD) != 0);
+      device_upload_input(g, row_ptr, col, w, dev, validate, (flags & GX_ASYNC_UPLOAD) != 0,
+                          (flags & GX_W_U8) != 0 && w);
     } else {
       // canonicalise on the host (reading R2); device inputs come back first
       std::vector<int64_t> hrp;

@@ -79,8 +79,28 @@ __global__ void k_csc_pairs(const uint32_t* __restrict__ rp, const uint2* __rest
 
 // ------------------------------------------------------------------ host side
 
+// GX_W_U8: 8-bit weights (a quarter of the PCIe bytes) widened on the device
+__global__ void k_widen_u8(const uint8_t* __restrict__ in, uint32_t* __restrict__ out, int64_t m) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = in[i];
+}
+
+// the weights into g->in_w on stream st: a u32 copy, or (w8) a byte copy + widening
+static void upload_weights(gx_graph* g, const uint32_t* w, bool w8, cudaMemcpyKind kind, cudaStream_t st) {
+  Ctx* c = g->ctx;
+  const int64_t m = g->m;
+  if (!w8) {
+    CUDA_OK(cudaMemcpyAsync(g->in_w.p, w, sizeof(uint32_t) * m, kind, st));
+    return;
+  }
+  g->in_w8.alloc(c, (size_t)m);
+  CUDA_OK(cudaMemcpyAsync(g->in_w8.p, w, (size_t)m, kind, st));
+  k_widen_u8<<<grid_for(c, m), 256, 0, st>>>(g->in_w8.as<uint8_t>(), g->in_w.as<uint32_t>(), m);
+  CUDA_OK(cudaGetLastError());
+}
+
 void device_upload_input(gx_graph* g, const int64_t* rp, const int32_t* col, const uint32_t* w,
-                         bool device_ptrs, bool validate, bool async) {
+                         bool device_ptrs, bool validate, bool async, bool w8) {
   Ctx* c = g->ctx;
   cudaStream_t s = c->stream;
   int64_t n = g->n, m = g->m;
@@ -102,7 +122,7 @@ void device_upload_input(gx_graph* g, const int64_t* rp, const int32_t* col, con
     CUDA_OK(cudaEventRecord(ev, s));
     CUDA_OK(cudaStreamWaitEvent(c->copy_stream, ev, 0));
     CUDA_OK(cudaEventDestroy(ev));
-    CUDA_OK(cudaMemcpyAsync(g->in_w.p, w, sizeof(uint32_t) * m, kind, c->copy_stream));
+    upload_weights(g, w, w8, kind, c->copy_stream);
     k_max_u32<<<grid_for(c, m), 256, 0, c->copy_stream>>>(g->in_w.as<uint32_t>(), m, g->maxw_buf.as<unsigned int>());
     CUDA_OK(cudaGetLastError());
     g->maxw_pending = true;
@@ -113,7 +133,7 @@ void device_upload_input(gx_graph* g, const int64_t* rp, const int32_t* col, con
   if (m) {
     CUDA_OK(cudaMemcpyAsync(g->in_col.p, col, sizeof(int32_t) * m, kind, s));
     if (w) {
-      CUDA_OK(cudaMemcpyAsync(g->in_w.p, w, sizeof(uint32_t) * m, kind, s));
+      upload_weights(g, w, w8, kind, s);
     } else {
       launch_fill_u32(c, g->in_w.as<uint32_t>(), 1u, m);  // all-ones weights
     }

@@ -343,7 +343,7 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell2(PrArgs a) {
 // One CTA per SM claims sink bins in ascending order and, for bin b:
 //   (1) streams the bin's contiguous range of val + 16-bit sink index with
 //       16-byte loads and adds each term into a shared-memory accumulator of
-//       its sink row (unsigned 64-bit fixed point, 2^-56 units, kept as two
+//       its sink row (unsigned 64-bit fixed point, 2^-52 units, kept as two
 //       32-bit words: exact, so the sum does not depend on the order); meanwhile the bin's
 //       x / D rows and block b's scatter segments are bulk-prefetched into L2;
 //   (2) runs the PR update of the bin's rows (x, delta, dangling and total
@@ -417,22 +417,30 @@ __device__ __forceinline__ void l2_prefetch_bulk(const void* p, uint32_t bytes) 
 }
 // fixed-point accumulation with the one native shared-memory atomic (32-bit
 // ATOMS.ADD; 64-bit and float adds compile to CAS loops): a term t >= 0 is
-// v = rn(t * 2^56) (quantum 1.4e-17, at most ~7e-18 per edge), split into
-// 32-bit halves; the low half is added with a returning atomic and a carry
-// out of it (rare: the low word holds up to 6e-8 of rank) goes to the high word.
-// rn(t * 2^56) for a term 0 <= t <= 1 with integer instructions: the same
-// value as __float2ull_rn(t * 0x1p56f) (the scaling is exact in f32, a
-// subnormal t rounds to 0 either way) without the 64-bit F2I, which issues to
-// the same MIO queue as the shared-memory atomics it feeds
+// v = rn(t * 2^F) (F = GX_PB_FIXBITS), kept as two 32-bit halves; the low half
+// is added with a returning atomic and the high half (the term's own high bits
+// plus the carry out of the low word) only when non-zero.  Exact and order
+// independent.  F = 52 (quantum 2.2e-16, at most 1.1e-16 per edge, so the
+// rounding of a whole sweep is below m * 2^-53 = 3e-8 in L1 at RMAT-24, well
+// inside the 1e-6 tolerance) makes every term below 2^-20 -- all but a handful
+// of RMAT terms x/D ~ 1e-8..1e-7 -- a single 32-bit value: measured, F = 56
+// needed the second (high-word) atomic on 61 % of the terms (ncu source page,
+// profiles/r2/pb_phase_split.txt).  The 64-bit accumulator holds sums up to
+// 2^(64-F) = 4096 >= 1.
+#ifndef GX_PB_FIXBITS
+#define GX_PB_FIXBITS 52
+#endif
 #ifndef GX_PB_IFIX
 #define GX_PB_IFIX 0    // measured slower: 713.5 (F2I.U64) vs 758 us per sweep (profiles/r1f/ifix_variants.txt)
 #endif
-__device__ __forceinline__ unsigned long long pb_fix56(float t) {
-  if (!GX_PB_IFIX) return __float2ull_rn(t * 0x1p56f);
+constexpr float PB_FIX_SCALE = (float)(1ull << GX_PB_FIXBITS);
+__device__ __forceinline__ unsigned long long pb_fix(float t) {
+  // rn(t * 2^F) for a term 0 <= t <= 1 (the scaling is exact in f32, a subnormal t rounds to 0)
+  if (!GX_PB_IFIX) return __float2ull_rn(t * PB_FIX_SCALE);
   const uint32_t b = __float_as_uint(t);
   const int e = (int)(b >> 23);   // biased exponent (t >= 0)
   const uint32_t m = (b & 0x7fffffu) | 0x800000u;
-  const int sh = e - 94;          // t * 2^56 = m * 2^(e - 127 - 23 + 56)
+  const int sh = e - (150 - GX_PB_FIXBITS);   // t * 2^F = m * 2^(e - 127 - 23 + F)
   if (sh >= 0) return (unsigned long long)m << sh;
   const int r = -sh;
   if (e == 0 || r > 25) return 0ull;
@@ -445,7 +453,7 @@ __device__ __forceinline__ void pb_add4(uint32_t* lo, uint32_t* hi, uint2 r, flo
   unsigned long long v[4];
   uint32_t old[4];
 #pragma unroll
-  for (int i = 0; i < 4; i++) v[i] = pb_fix56(tt[i]);
+  for (int i = 0; i < 4; i++) v[i] = pb_fix(tt[i]);
   // the returning atomics are independent: issue them back to back
 #pragma unroll
   for (int i = 0; i < 4; i++) old[i] = atomicAdd(&lo[rr[i]], (uint32_t)v[i]);
@@ -644,7 +652,7 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
   constexpr unsigned NW = PB_THREADS / 32;
   const int64_t nb = p.nb;
   const uint32_t* qend = p.q + nb * nb;
-  const double inv_fix = 1.0 / 72057594037927936.0;   // 2^-56
+  const double inv_fix = 1.0 / (double)(1ull << GX_PB_FIXBITS);   // 2^-F
   if (threadIdx.x < 8) acc_lo[PB_R + threadIdx.x] = 0u;  // s_c[R..R+7] = 0.0f
   if (threadIdx.x == 0) {
     for (int i = 0; i < PB_NST; i++) {
