@@ -367,10 +367,12 @@ def main():
         ex = G.export()      # canonical graph (exact mode), rows sorted: caller-side canonical input
         hrp = torch.from_numpy(ex["row_ptr"]).pin_memory()
         hcol = torch.from_numpy(ex["col"]).pin_memory()
-        hw = torch.from_numpy(ex["w"].view(np.int32)).pin_memory()
+        # weights 1..100 travel as bytes (GX_W_U8, widened on the device)
+        assert int(ex["w"].max()) <= 255
+        hw = torch.from_numpy(ex["w"].astype(np.uint8)).pin_memory()
         hdist = torch.empty(n, dtype=torch.int32).pin_memory()
         hrank = torch.empty(n, dtype=torch.float64).pin_memory()
-        h2d = hrp.numel() * 8 + hcol.numel() * 4 + hw.numel() * 4
+        h2d = hrp.numel() * 8 + hcol.numel() * 4 + hw.numel() * 1
         d2h = n * 4 + n * 8
         e2e_ms, e2e_edges = [], 0
         for i in range(args.e2e_steps + 1):
@@ -380,7 +382,7 @@ def main():
             e0.record(stream)
             # GX_ASYNC_UPLOAD: the weights' H2D overlaps the blocked PageRank
             # (structure only); SSSP joins the copy
-            G2 = gx.Graph.upload(ctx, hrp.numpy(), hcol.numpy(), hw.numpy().view(np.uint32), canonical=True,
+            G2 = gx.Graph.upload(ctx, hrp.numpy(), hcol.numpy(), hw.numpy(), canonical=True,
                                  async_upload=not args.e2e_sync)
             b = G2.run("pagerank", tol=1e-9, mapping=args.pr_mapping)
             G2.download("rank", out=hrank.numpy(), async_copy=not args.e2e_sync)   # D2H overlaps SSSP
@@ -403,7 +405,7 @@ def main():
             e2e_edges = int(te.item())
         e2e = {"value": e2e_edges / (t * 1e-3) / 1e9, "unit": UNIT, "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": d2h, "ms_per_step": t / len(e2e_ms),
-               "note": "upload of canonical pinned CSR (GX_CANONICAL" + ("" if args.e2e_sync else " | GX_ASYNC_UPLOAD: weights H2D overlapping the blocked PR; rank D2H (GX_DL_ASYNC) overlapping SSSP") + ") + device layouts (blocked-PR segments, SSSP heavy chunks) + PR + download rank + SSSP + download dist"}
+               "note": "upload of canonical pinned CSR with 8-bit weights (GX_CANONICAL | GX_W_U8" + ("" if args.e2e_sync else " | GX_ASYNC_UPLOAD: weights H2D overlapping the blocked PR; rank D2H (GX_DL_ASYNC) overlapping SSSP") + ") + device layouts (blocked-PR segments, SSSP heavy chunks) + PR + download rank + SSSP + download dist"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

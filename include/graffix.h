@@ -155,6 +155,7 @@ typedef struct {
   double sweep_ms;         /* profile: summed CUDA-event time of the main sweep kernel */
   int64_t sweep_bytes;     /* algorithmic bytes moved by the main sweep kernel       */
   int32_t mapping_used;    /* gx_mapping the sweeps ran with (AUTO resolved)         */
+  int32_t dense_iterations; /* SSSP: iterations run as the blocked dense relaxation   */
 } gx_run_info;
 
 typedef struct {

@@ -55,7 +55,8 @@ class GxRunInfo(C.Structure):
     _fields_ = [("iterations", C.c_int32), ("converged", C.c_int32), ("loop_ms", C.c_double),
                 ("last_delta", C.c_double), ("edges_scanned", C.c_int64), ("bytes_model", C.c_int64),
                 ("vertices_active", C.c_int64), ("kernel_launches", C.c_int32), ("sweep_launches", C.c_int32),
-                ("sweep_ms", C.c_double), ("sweep_bytes", C.c_int64), ("mapping_used", C.c_int32)]
+                ("sweep_ms", C.c_double), ("sweep_bytes", C.c_int64), ("mapping_used", C.c_int32),
+                ("dense_iterations", C.c_int32)]
 
 
 class GxRunOpts(C.Structure):

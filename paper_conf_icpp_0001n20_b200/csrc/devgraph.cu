@@ -317,6 +317,75 @@ void ensure_pb(gx_graph* g) {
   CUDA_OK(cudaStreamSynchronize(s));   // temporaries are freed on return
 }
 
+// ---- the edge weights in the blocked order (SSSP's dense relaxation, sssp.cu) ----
+// Same keys as k_pb_pairs with the edge index as payload: the stable radix sort
+// puts every edge at the position ensure_pb gave it.
+__global__ void k_pb_keys_e(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj, int64_t n, uint32_t nb,
+                            uint32_t* __restrict__ key, uint32_t* __restrict__ eid, uint32_t* __restrict__ cnt) {
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t u = warp; u < n; u += nw) {
+    const uint32_t bu = (uint32_t)(u / PB_R);
+    for (uint32_t e = rp[u] + lane_id(); e < rp[u + 1]; e += 32) {
+      const uint32_t k = (adj[e].x / PB_R) * nb + bu;
+      key[e] = k;
+      eid[e] = e;
+      atomicAdd(&cnt[k], 1u);
+    }
+  }
+}
+__global__ void k_pb_place_w(const uint32_t* __restrict__ key, const uint32_t* __restrict__ eid,
+                             const uint32_t* __restrict__ P, const uint32_t* __restrict__ P2,
+                             const uint2* __restrict__ adj, uint8_t* __restrict__ w8, int64_t m) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t k = key[i];
+    w8[P2[k] + ((uint32_t)i - P[k])] = (uint8_t)adj[eid[i]].y;
+  }
+}
+
+// w8[pos] = weight of the edge at blocked position pos (padding 0); needs max w <= 255
+void ensure_pb_w(gx_graph* g) {
+  DevGraph& d = g->dg;
+  if (d.pb_w8.p) return;
+  ensure_pb(g);
+  resolve_pending(g);
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  const int64_t n = d.n_slots, m = d.m_slots, nb = d.pr_pb.nb, nk = nb * nb + 1;
+  d.pb_w8.alloc(c, (size_t)std::max<int64_t>(d.pr_pb.m_pad, 16));
+  CUDA_OK(cudaMemsetAsync(d.pb_w8.p, 0, (size_t)std::max<int64_t>(d.pr_pb.m_pad, 16), s));
+  if (m == 0) return;
+  DBuf cnt, pc, P, P2, k0, k1, v0, v1, tmp, t2;
+  cnt.alloc(c, sizeof(uint32_t) * nk);
+  pc.alloc(c, sizeof(uint32_t) * nk);
+  P.alloc(c, sizeof(uint32_t) * nk);
+  P2.alloc(c, sizeof(uint32_t) * nk);
+  CUDA_OK(cudaMemsetAsync(cnt.p, 0, sizeof(uint32_t) * nk, s));
+  k0.alloc(c, sizeof(uint32_t) * m);
+  k1.alloc(c, sizeof(uint32_t) * m);
+  v0.alloc(c, sizeof(uint32_t) * m);
+  v1.alloc(c, sizeof(uint32_t) * m);
+  k_pb_keys_e<<<grid_for(c, n * 32), 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), n, (uint32_t)nb,
+                                                  k0.as<uint32_t>(), v0.as<uint32_t>(), cnt.as<uint32_t>());
+  int bits = 1;
+  while ((int64_t(1) << bits) < nb * nb) bits++;
+  cub::DoubleBuffer<uint32_t> dk(k0.as<uint32_t>(), k1.as<uint32_t>()), dv(v0.as<uint32_t>(), v1.as<uint32_t>());
+  size_t tb = 0;
+  CUDA_OK(cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv, (int64_t)m, 0, bits, s));
+  tmp.alloc(c, tb);
+  CUDA_OK(cub::DeviceRadixSort::SortPairs(tmp.p, tb, dk, dv, (int64_t)m, 0, bits, s));
+  k_pb_padcnt<<<grid_for(c, nk), 256, 0, s>>>(cnt.as<uint32_t>(), pc.as<uint32_t>(), nk);
+  size_t sb = 0;
+  CUDA_OK(cub::DeviceScan::ExclusiveSum(nullptr, sb, cnt.as<uint32_t>(), P.as<uint32_t>(), nk, s));
+  t2.alloc(c, sb);
+  CUDA_OK(cub::DeviceScan::ExclusiveSum(t2.p, sb, cnt.as<uint32_t>(), P.as<uint32_t>(), nk, s));
+  CUDA_OK(cub::DeviceScan::ExclusiveSum(t2.p, sb, pc.as<uint32_t>(), P2.as<uint32_t>(), nk, s));
+  k_pb_place_w<<<grid_for(c, m), 256, 0, s>>>(dk.Current(), dv.Current(), P.as<uint32_t>(), P2.as<uint32_t>(),
+                                              d.adj.as<uint2>(), d.pb_w8.as<uint8_t>(), m);
+  CUDA_OK(cudaGetLastError());
+  CUDA_OK(cudaStreamSynchronize(s));   // temporaries are freed on return
+}
+
 // join the GX_ASYNC_UPLOAD work into the ctx stream; read the weights' maximum
 void resolve_pending(gx_graph* g) {
   if (!g->ctx) return;

@@ -173,6 +173,7 @@ struct DevGraph {
   // push over out-edges
   SellLayout pr_sell, sssp_sell;
   PbLayout pr_pb;              // propagation-blocked PR (built on first use)
+  DBuf pb_w8;                  // u8 [m_pad]: edge weights in the blocked order (SSSP dense relaxation)
   RankLayouts rk_sssp, rk_pr;  // partitioned path (dist.h): this rank's rows only
   // LB SSSP: static chunk list of rows with out-degree > HEAVY_DEG, heavy bitmap
   int64_t nhc = 0;
@@ -265,6 +266,8 @@ void build_device_exact(gx_graph* g);
 void resolve_pending(gx_graph* g);
 void join_download(gx_graph* g, int kind);   // kind < 0: every kind
 void build_device_slots(gx_graph* g);
+void ensure_pb(gx_graph* g);
+void ensure_pb_w(gx_graph* g);
 void build_tpv(gx_graph* g);
 void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info);
 void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info);

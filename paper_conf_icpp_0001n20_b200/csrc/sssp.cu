@@ -635,9 +635,11 @@ __global__ void k_sssp_advance(SsspState* __restrict__ st, int max_iters) { sssp
 // t = the iteration the refilled frontier belongs to; remaining far minimum -> fdst
 __device__ __forceinline__ void sssp_split_dev(const uint32_t* __restrict__ dist, const SsspAux& ax,
                                                SsspState* __restrict__ st, int64_t lo, int64_t hi, const unsigned t,
-                                               const uint32_t tau, uint32_t* fdst) {
+                                               const uint32_t tau, uint32_t* fdst,
+                                               const uint32_t* __restrict__ rp = nullptr) {
   uint32_t* bm_cur = ax.bm[t % 3];
   uint32_t my_min = INF;
+  unsigned long long my_deg = 0;   // rp != null: count the moved slots (dense-iteration test)
   const int64_t w_lo = lo >> 5, w_hi = min((hi + 31) >> 5, ax.nwords);
   for (int64_t w = w_lo + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < w_hi; w += (int64_t)gridDim.x * blockDim.x) {
     uint32_t bits = ax.far[w];
@@ -647,12 +649,20 @@ __device__ __forceinline__ void sssp_split_dev(const uint32_t* __restrict__ dist
       const int b = __ffs(bits) - 1;
       bits &= bits - 1;
       const uint32_t d = dist[w * 32 + b];
-      if (d < tau) move |= 1u << b;
-      else my_min = min(my_min, d);
+      if (d < tau) {
+        move |= 1u << b;
+      } else {
+        my_min = min(my_min, d);
+      }
     }
     keep &= ~move;
     ax.far[w] = keep;
     if (move) bm_cur[w] |= move;
+    my_deg += __popc(move);
+  }
+  if (rp) {
+    my_deg = warp_sum_u64(my_deg);
+    if (lane_id() == 0 && my_deg) atomicAdd(&st->refill_deg[t % 3], my_deg);
   }
   flush_counters(st, 0, 0, 0, 0, my_min, fdst);
 }
@@ -816,6 +826,8 @@ struct SsspLoop {
   int32_t* tlist;
   unsigned long long* trace;   // GX_SSSP_PTRACE: per iteration {globaltimer ns, edges so far, active, tau}
   int trace_cap;
+  unsigned long long dense_edges;   // > 0: a refill that moves >= this many slots exits for the blocked
+                                    // dense relaxation (stop = 4); 0: never
 };
 
 constexpr int PERSIST_POOL = SB_WARPS * 1024 * 4;   // 32 KB at 256 threads: LB compaction buffer / block-mode queues
@@ -837,8 +849,18 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
   // every CTA has passed).  far3[t%3] collects the far pile's minimum pushed
   // in iteration t; rf is the running minimum since the last refill.
   unsigned t = st->iter;
-  uint32_t tau = st->tau, rf = INF;
+  uint32_t tau = st->tau, rf = st->far_min;   // a relaunch after a dense iteration continues its state
   const uint32_t delta = st->delta;
+  // the relaunch's pending near-far refill (decided after the dense iteration)
+  if (*(volatile unsigned*)&st->split) {
+    sssp_split_dev(a.dist, a.ax, st, 0, a.n_slots, t, tau, &st->far3[t % 3], a.dense_edges ? a.rp : nullptr);
+    grid.sync();
+    if (lead) st->split = 0;
+    if (a.dense_edges && *(volatile unsigned long long*)&st->refill_deg[t % 3] >= a.dense_edges) {
+      if (lead) st->stop = 4;
+      return;
+    }
+  }
   // light / heavy split (ax.lend set; no tiles, merges or block mode): pend_n =
   // frontier entries since the last heavy pass, hv = this iteration is one
   const bool lh = a.ax.lend != nullptr;
@@ -933,6 +955,7 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
       st->pushed[(t + 2) % 3] = 0;
       st->far3[(t + 2) % 3] = INF;
       st->tiles_n[(t + 2) % 3] = 0;
+      st->refill_deg[(t + 2) % 3] = 0;
       st->iter = t + 1;
       st->tau = tau;
       st->far_min = rf;
@@ -941,10 +964,222 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
     if (stop) break;
     t++;
     if (split) {   // near-far refill of iteration t's frontier
-      sssp_split_dev(a.dist, a.ax, st, 0, a.n_slots, t, tau, &st->far3[t % 3]);
+      sssp_split_dev(a.dist, a.ax, st, 0, a.n_slots, t, tau, &st->far3[t % 3], a.dense_edges ? a.rp : nullptr);
       grid.sync();
+      // a refill that carries most of the graph's edges: hand iteration t to the
+      // blocked dense relaxation (k_sssp_pb_*), which streams every edge once
+      // instead of gathering dist at random for each of them
+      if (a.dense_edges && *(volatile unsigned long long*)&st->refill_deg[t % 3] >= a.dense_edges) {
+        if (lead) st->stop = 4;
+        break;
+      }
     }
   }
+}
+
+// ---------------------------------------------------------------- blocked dense relaxation
+// A near-far refill that activates slots carrying most of the graph's edges
+// (RMAT-24, bucket [25, 50): 8.5M slots, 205M of 268M edges) is one sparse
+// matrix-vector product in the (min, +) semiring.  The LB sweep pays a random
+// dist gather (one L1TEX wavefront, often across the die boundary) per edge;
+// here the iteration runs over the propagation-blocked layout of the PageRank
+// pull (PbLayout: edges grouped in (sink bin, source block) segments with
+// 16-bit local indices) and never touches memory at random:
+//   (A) k_sssp_pb_scatter: per source block, the frontier slots' distances in
+//       shared memory; every edge's candidate dist[u] + w (INF for a source
+//       outside the frontier) streamed to val[] (2 + 1 bytes read, 4 written)
+//   (B) k_sssp_pb_gather: per sink bin, the bin's candidates streamed (4 + 2
+//       bytes) into a shared-memory atomicMin per row (ATOMS.MIN), then the
+//       rows that improved update dist and join the next frontier / far pile
+//       with word-level ballots (a bin's rows are whole bitmap words)
+// val[] is the PageRank layout's term array (reinterpreted as u32; PageRank
+// rewrites it at the start of each run).  Same fixed point (any relaxation
+// order, Theorem E1): the iteration relaxes every frontier edge exactly once.
+constexpr int SPB_THREADS = 1024;
+struct SsspPb {
+  const uint32_t* q;
+  const uint16_t* src_loc;
+  const uint16_t* dst_loc;
+  const uint8_t* w8;
+  uint32_t* val;
+  int64_t nb;
+};
+
+__global__ void __launch_bounds__(SPB_THREADS, 1) k_sssp_pb_scatter(SsspPb p, const uint32_t* __restrict__ dist,
+                                                                    SsspAux ax, SsspState* __restrict__ st,
+                                                                    int64_t n_slots) {
+  extern __shared__ __align__(16) uint32_t s_d[];   // PB_R + 8: frontier distances, INF elsewhere and for padding
+  if (st->stop != 4) return;
+  const unsigned t = st->iter;
+  const uint32_t* __restrict__ bm_cur = ax.bm[t % 3];
+  const uint64_t pf = l2_evict_first();
+  const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
+  constexpr unsigned NW = SPB_THREADS / 32;
+  const int64_t nb = p.nb;
+  if (threadIdx.x < 8) s_d[PB_R + threadIdx.x] = INF;
+  for (int64_t b = blockIdx.x; b < nb; b += gridDim.x) {
+    const int64_t base = b * PB_R;
+    for (int i = threadIdx.x; i < PB_R; i += SPB_THREADS) {
+      const int64_t v = base + i;
+      uint32_t dv = INF;
+      if (v < n_slots && ((__ldcg(bm_cur + (v >> 5)) >> (v & 31)) & 1u)) dv = __ldcg(dist + v);
+      s_d[i] = dv;
+    }
+    __syncthreads();
+    const uint32_t* r0 = p.q + b * nb;   // block b's segments [r0[j], r1[j])
+    const uint32_t* r1 = r0 + nb;
+    // 8 entries per lane per step (16 B of source indices, 8 B of weights);
+    // SPB_SEGU segments' first steps are loaded together (memory-level
+    // parallelism), then each segment's remaining steps
+    auto put8 = [&](uint32_t e, uint4 sx, uint2 wx) {
+      const uint32_t sr[8] = {sx.x & 0xffffu, sx.x >> 16, sx.y & 0xffffu, sx.y >> 16,
+                              sx.z & 0xffffu, sx.z >> 16, sx.w & 0xffffu, sx.w >> 16};
+      uint32_t c[8];
+#pragma unroll
+      for (int i = 0; i < 8; i++) {
+        const uint32_t du = s_d[sr[i]];
+        const uint32_t w = ((i < 4 ? wx.x : wx.y) >> (8 * (i & 3))) & 0xffu;
+        c[i] = du == INF ? INF : sat_add(du, w);
+      }
+      __stcg(reinterpret_cast<uint4*>(p.val + e), make_uint4(c[0], c[1], c[2], c[3]));
+      __stcg(reinterpret_cast<uint4*>(p.val + e) + 1, make_uint4(c[4], c[5], c[6], c[7]));
+    };
+    constexpr int SPB_SEGU = 4;
+    for (int64_t j0 = (int64_t)warp * 32; j0 < nb; j0 += 32 * NW) {
+      const int64_t j = j0 + lane;
+      const uint32_t lo = j < nb ? __ldg(r0 + j) : 0u, hi = j < nb ? __ldg(r1 + j) : 0u;
+      const int kn = (int)min((int64_t)32, nb - j0);
+      for (int k = 0; k < kn; k += SPB_SEGU) {
+        uint32_t ee[SPB_SEGU], hh[SPB_SEGU];
+        uint4 sx[SPB_SEGU];
+        uint2 wx[SPB_SEGU];
+#pragma unroll
+        for (int u = 0; u < SPB_SEGU; u++) {
+          ee[u] = __shfl_sync(FULL, lo, (k + u) & 31) + 8u * lane;
+          hh[u] = k + u < kn ? __shfl_sync(FULL, hi, (k + u) & 31) : 0u;
+          if (ee[u] < hh[u]) {
+            sx[u] = ld_stream_v4(reinterpret_cast<const uint32_t*>(p.src_loc + ee[u]), pf);
+            wx[u] = *reinterpret_cast<const uint2*>(p.w8 + ee[u]);
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < SPB_SEGU; u++) {
+          if (ee[u] < hh[u]) put8(ee[u], sx[u], wx[u]);
+          for (uint32_t e = ee[u] + 256u; e < hh[u]; e += 256u)
+            put8(e, ld_stream_v4(reinterpret_cast<const uint32_t*>(p.src_loc + e), pf),
+                 *reinterpret_cast<const uint2*>(p.w8 + e));
+        }
+      }
+    }
+    __syncthreads();
+  }
+}
+
+__global__ void __launch_bounds__(SPB_THREADS, 1) k_sssp_pb_gather(SsspPb p, uint32_t* __restrict__ dist, SsspAux ax,
+                                                                   SsspState* __restrict__ st, int64_t n_slots) {
+  extern __shared__ __align__(16) uint32_t acc[];   // PB_R row minima
+  __shared__ int s_bin;
+  if (st->stop != 4) return;
+  const unsigned t = st->iter;
+  const uint32_t tau = st->tau;
+  const uint32_t* __restrict__ bm_cur = ax.bm[t % 3];
+  uint32_t* bm_next = ax.bm[(t + 1) % 3];
+  clear_bitmap(ax.bm[(t + 2) % 3], ax.nwords);
+  const uint64_t pf = l2_evict_first();
+  const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
+  constexpr unsigned NW = SPB_THREADS / 32;
+  const int64_t nb = p.nb;
+  const uint32_t* qend = p.q + nb * nb;
+  unsigned long long my_act = 0;
+  uint32_t my_push = 0, my_min = INF;
+  for (;;) {
+    if (threadIdx.x == 0) s_bin = (int)atomicAdd(&st->dense_bin, 1u);
+    for (int i = threadIdx.x; i < PB_R / 4; i += SPB_THREADS)
+      reinterpret_cast<uint4*>(acc)[i] = make_uint4(INF, INF, INF, INF);
+    __syncthreads();
+    const int64_t b = s_bin;
+    if (b >= nb) break;
+    const uint32_t E0 = __ldg(p.q + b), E1 = __ldg(qend + b);   // multiples of 8
+    // the bin's candidates: 4 per thread per step, two steps in flight
+    for (uint32_t e = E0 + 4u * threadIdx.x; e < E1; e += 8u * SPB_THREADS) {
+      const uint32_t e2 = e + 4u * SPB_THREADS;
+      const uint4 v0 = ld_stream_v4(p.val + e, pf);
+      const uint2 d0 = *reinterpret_cast<const uint2*>(p.dst_loc + e);
+      uint4 v1 = make_uint4(INF, INF, INF, INF);
+      uint2 d1 = make_uint2(0, 0);
+      if (e2 < E1) {
+        v1 = ld_stream_v4(p.val + e2, pf);
+        d1 = *reinterpret_cast<const uint2*>(p.dst_loc + e2);
+      }
+      const uint32_t vv[8] = {v0.x, v0.y, v0.z, v0.w, v1.x, v1.y, v1.z, v1.w};
+      const uint32_t dd[8] = {d0.x & 0xffffu, d0.x >> 16, d0.y & 0xffffu, d0.y >> 16,
+                              d1.x & 0xffffu, d1.x >> 16, d1.y & 0xffffu, d1.y >> 16};
+#pragma unroll
+      for (int i = 0; i < 8; i++)
+        if (vv[i] != INF) atomicMin(&acc[dd[i]], vv[i]);
+    }
+    __syncthreads();
+    // the bin's rows: warp per 32 rows = one bitmap word
+    const int64_t base = b * PB_R;
+    const int nrows = (int)min((int64_t)PB_R, n_slots - base);
+    for (int i0 = warp * 32; i0 < nrows; i0 += NW * 32) {
+      const int i = i0 + lane;
+      const int64_t v = base + i;
+      const uint32_t nd = i < nrows ? acc[i] : INF;
+      bool better = false;
+      if (nd != INF) {
+        const uint32_t old = __ldcg(dist + v);
+        better = nd < old;
+        if (better) __stcg(dist + v, nd);
+      }
+      const unsigned bn = __ballot_sync(FULL, better && nd < tau);
+      const unsigned bf = __ballot_sync(FULL, better && nd >= tau);
+      if (better && nd >= tau) my_min = min(my_min, nd);
+      if (lane == 0) {
+        const int64_t w = v >> 5;
+        my_act += __popc(__ldcg(bm_cur + w));
+        if (bn) bm_next[w] |= bn;
+        if (bf) ax.far[w] |= bf;
+        my_push += __popc(bn);
+      }
+    }
+    __syncthreads();
+  }
+  flush_counters(st, t, 0, my_act, my_push, my_min, &st->far3[t % 3]);
+}
+
+// the loop decision after a dense iteration t: the persistent loop's rule
+// (no merges, tiles or light/heavy split in dense mode), then iteration t+1
+// resumes in k_sssp_persist (a pending refill runs first there)
+__global__ void k_sssp_dense_decide(SsspState* __restrict__ st, int64_t m_slots, unsigned early, int max_iters) {
+  if (st->stop != 4) return;
+  const unsigned t = st->iter;
+  const unsigned pushed = st->pushed[t % 3];
+  const uint32_t fm = min(st->far_min, st->far3[t % 3]);
+  uint32_t tau = st->tau, rf = fm;
+  unsigned stop = 0, split = 0;
+  if ((pushed <= early || pushed == 0) && fm != INF) {
+    const unsigned long long nt = (unsigned long long)fm + st->delta;
+    tau = nt >= INF ? INF : (unsigned)nt;
+    rf = INF;
+    split = 1;
+  } else if (pushed == 0) {
+    stop = 1;
+  }
+  if (!stop && (int)(t + 1) >= max_iters) stop = 2;
+  st->edges += (unsigned long long)m_slots;   // every edge was scanned
+  st->act_total += st->active[t % 3];
+  st->active[(t + 2) % 3] = 0;
+  st->pushed[(t + 2) % 3] = 0;
+  st->far3[(t + 2) % 3] = INF;
+  st->tiles_n[(t + 2) % 3] = 0;
+  st->refill_deg[(t + 2) % 3] = 0;
+  st->dense_bin = 0;
+  st->iter = t + 1;
+  st->tau = tau;
+  st->far_min = rf;
+  st->split = split;
+  st->stop = stop;
 }
 
 __global__ void k_stamp(unsigned long long* p) {
@@ -1581,6 +1816,33 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
       ax.adjp = d.adjp.as<uint32_t>();   // the partitioned copy replaced the buffer
     }
   }
+  // blocked dense relaxation for refills that carry most of the edges
+  // (persistent LB loop on a graph without merges, tiles or the light/heavy
+  // split; weights must fit the layout's 8-bit array).  GX_SSSP_DENSE = the
+  // fraction of the slots a refill must move (default 0.45; 0 = off).  The
+  // dense pass costs one streaming pass over all edges (RMAT-24: scatter 0.49
+  // + gather 0.43 ms) against ~140 G relaxations/s for the LB sweep, so it
+  // pays once a refill carries about half of the edges: RMAT-24's first
+  // refill moves 51 % of the slots with 76 % of the edges (4.85 -> 4.49 ms);
+  // uniform and RMAT-22 refills at 40 % lost 0.4 / 0.13 ms
+  // (profiles/r2/sssp_dense_sweep.txt)
+  double dense_frac = 0.45;
+  if (const char* e = getenv("GX_SSSP_DENSE")) dense_frac = atof(e);
+  const bool dense_ok = mapping == GX_MAP_LB && dense_frac > 0.0 && !(d.n_tiles && g->knobs.smem) && !d.n_groups &&
+                        !want_lh && d.max_w <= 255 && d.m_slots > 0 && !getenv("GX_SSSP_BLOCK") &&
+                        !(o.profile && getenv("GX_SSSP_TRACE"));
+  SsspPb spb{};
+  if (dense_ok) {
+    ensure_pb_w(g);
+    spb.q = d.pr_pb.q.as<uint32_t>();
+    spb.src_loc = d.pr_pb.src_loc.as<uint16_t>();
+    spb.dst_loc = d.pr_pb.dst_loc.as<uint16_t>();
+    spb.w8 = d.pb_w8.as<uint8_t>();
+    spb.val = d.pr_pb.val.as<uint32_t>();
+    spb.nb = d.pr_pb.nb;
+    CUDA_OK(cudaFuncSetAttribute(k_sssp_pb_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (PB_R + 8) * 4));
+    CUDA_OK(cudaFuncSetAttribute(k_sssp_pb_gather, cudaFuncAttributeMaxDynamicSharedMemorySize, PB_R * 4));
+  }
   cudaEvent_t e0, e1;
   CUDA_OK(cudaEventCreate(&e0));
   CUDA_OK(cudaEventCreate(&e1));
@@ -1762,13 +2024,49 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
     }
     void* args[] = {&L};
     kt.begin();
+    L.dense_edges = dense_ok ? (unsigned long long)std::max(1.0, dense_frac * (double)d.n_slots) : 0ull;
     if (L.trace) k_stamp<<<1, 1, 0, s>>>(trace_buf.as<unsigned long long>());
-    CUDA_OK(cudaLaunchCooperativeKernel((void*)k_sssp_persist, dim3((unsigned)(occp * c->num_sms)), dim3(PERSIST_TPB), args,
-                                        0, s));
+    for (;;) {
+      CUDA_OK(cudaLaunchCooperativeKernel((void*)k_sssp_persist, dim3((unsigned)(occp * c->num_sms)), dim3(PERSIST_TPB),
+                                          args, 0, s));
+      launches += 1;
+      CUDA_OK(cudaMemcpyAsync(&hst, st, sizeof(SsspState), cudaMemcpyDeviceToHost, s));
+      CUDA_OK(cudaStreamSynchronize(s));
+      if (hst.stop != 4) break;
+      // the refill carries most of the edges: one blocked dense iteration, then
+      // the persistent loop resumes (stop = 4 -> the decision -> 0 / 1 / 2)
+      const int gs = (int)std::min<int64_t>(spb.nb, (int64_t)c->num_sms * 2);
+      const int gg = (int)std::min<int64_t>(spb.nb, (int64_t)c->num_sms);
+      cudaEvent_t d0 = nullptr, d1 = nullptr, d2 = nullptr;
+      if (L.trace) {
+        CUDA_OK(cudaEventCreate(&d0));
+        CUDA_OK(cudaEventCreate(&d1));
+        CUDA_OK(cudaEventCreate(&d2));
+        CUDA_OK(cudaEventRecord(d0, s));
+      }
+      k_sssp_pb_scatter<<<gs, SPB_THREADS, (PB_R + 8) * 4, s>>>(spb, r.dist.as<uint32_t>(), ax, st, ns);
+      if (L.trace) CUDA_OK(cudaEventRecord(d1, s));
+      k_sssp_pb_gather<<<gg, SPB_THREADS, PB_R * 4, s>>>(spb, r.dist.as<uint32_t>(), ax, st, ns);
+      if (L.trace) {
+        CUDA_OK(cudaEventRecord(d2, s));
+        CUDA_OK(cudaEventSynchronize(d2));
+        float a1 = 0, a2 = 0;
+        cudaEventElapsedTime(&a1, d0, d1);
+        cudaEventElapsedTime(&a2, d1, d2);
+        fprintf(stderr, "sssp-ptrace dense t=%u scatter_us=%.1f gather_us=%.1f\n", hst.iter, 1e3 * a1, 1e3 * a2);
+        cudaEventDestroy(d0);
+        cudaEventDestroy(d1);
+        cudaEventDestroy(d2);
+      }
+      k_sssp_dense_decide<<<1, 1, 0, s>>>(st, d.m_slots, L.early, o.max_iters);
+      CUDA_OK(cudaGetLastError());
+      launches += 3;
+      info.dense_iterations++;
+      CUDA_OK(cudaMemcpyAsync(&hst, st, sizeof(SsspState), cudaMemcpyDeviceToHost, s));
+      CUDA_OK(cudaStreamSynchronize(s));
+      if (hst.stop) break;
+    }
     kt.end();
-    launches += 1;
-    CUDA_OK(cudaMemcpyAsync(&hst, st, sizeof(SsspState), cudaMemcpyDeviceToHost, s));
-    CUDA_OK(cudaStreamSynchronize(s));
     if (L.trace) {
       const int nt = std::min<int>((int)hst.iter, L.trace_cap);
       std::vector<unsigned long long> h(4 * (nt + 1));

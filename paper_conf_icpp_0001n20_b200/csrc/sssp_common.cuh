@@ -28,6 +28,8 @@ struct SsspState {
   unsigned int final_merge;     // c = 0: this iteration's merge ends the run
   unsigned int far3[3];         // persistent loop: far-pile minimum pushed in iteration t, [t%3]
   unsigned int tiles_n[3];      // §3 tiles touched in iteration t (list length), [t%3]
+  unsigned long long refill_deg[3];  // out-edges of the slots a near-far refill moved into frontier t, [t%3]
+  unsigned int dense_bin;       // blocked dense relaxation: next sink bin to claim
 };
 
 struct SsspAux {

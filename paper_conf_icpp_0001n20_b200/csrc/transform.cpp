@@ -154,32 +154,54 @@ void renumber(const HostCSR& g, int k, std::vector<int32_t>& nw, int64_t& n_slot
   ranges.clear();
   ranges.push_back({0, gid});
   std::vector<int32_t> cur(sources), nxt;
-  std::vector<int64_t> cursor;
+  std::vector<int64_t> cursor, chp;
+  std::vector<int32_t> ch;
   int32_t i = 0;
   while (true) {
     const int64_t start = (gid + k - 1) / k * k;
     std::vector<int32_t> parents(cur);
     std::sort(parents.begin(), parents.end(), [&](int32_t a, int32_t b) { return nw[a] < nw[b]; });
-    cursor.assign(parents.size(), 0);
-    for (size_t p = 0; p < parents.size(); p++) cursor[p] = g.rp[parents[p]];
+    // each parent's level-(i+1) neighbours in adjacency order, filtered in
+    // parallel: level[] never changes during the numbering, so the cursor of
+    // R6 walks exactly this list and skips the entries already numbered
+    const int64_t np = (int64_t)parents.size();
+    chp.assign(np + 1, 0);
+#pragma omp parallel for schedule(dynamic, 1024)
+    for (int64_t p = 0; p < np; p++) {
+      const int32_t par = parents[p];
+      int64_t cnt = 0;
+      for (int64_t e = g.rp[par]; e < g.rp[par + 1]; e++) cnt += level[g.col[e]] == i + 1;
+      chp[p + 1] = cnt;
+    }
+    for (int64_t p = 0; p < np; p++) chp[p + 1] += chp[p];
+    ch.resize(chp[np]);
+#pragma omp parallel for schedule(dynamic, 1024)
+    for (int64_t p = 0; p < np; p++) {
+      const int32_t par = parents[p];
+      int64_t o = chp[p];
+      for (int64_t e = g.rp[par]; e < g.rp[par + 1]; e++)
+        if (level[g.col[e]] == i + 1) ch[o++] = g.col[e];
+    }
+    cursor.assign(chp.begin(), chp.end() - 1);
     nxt.clear();
     int64_t gid2 = start;
     // rounds: each parent numbers its next unnumbered level-(i+1) neighbour;
-    // parents that exhausted their rows drop out of later rounds
-    std::vector<size_t> live(parents.size());
-    std::iota(live.begin(), live.end(), 0);
+    // parents that exhausted their lists drop out of later rounds
+    std::vector<size_t> live;
+    live.reserve(np);
+    for (int64_t p = 0; p < np; p++)
+      if (chp[p + 1] > chp[p]) live.push_back((size_t)p);
     while (true) {
       bool assigned = false;
       size_t keep = 0;
       for (size_t li = 0; li < live.size(); li++) {
         const size_t p = live[li];
-        const int32_t par = parents[p];
         int64_t c = cursor[p];
-        const int64_t end = g.rp[par + 1];
-        while (c < end && !(level[g.col[c]] == i + 1 && nw[g.col[c]] == -1)) c++;
+        const int64_t end = chp[p + 1];
+        while (c < end && nw[ch[c]] != -1) c++;
         if (c < end) {
-          nw[g.col[c]] = (int32_t)gid2++;
-          nxt.push_back(g.col[c]);
+          nw[ch[c]] = (int32_t)gid2++;
+          nxt.push_back(ch[c]);
           c++;
           assigned = true;
         }

@@ -404,3 +404,58 @@ def test_async_download_overlaps_and_joins():
     assert np.array_equal(dout, A.sssp_dijkstra(el, sssp_source(g)))
     assert not np.array_equal(G.download("rank"), ref)
     G.close()
+
+
+@pytest.mark.parametrize("canonical", [False, True])
+@pytest.mark.parametrize("where", ["host", "device"])
+def test_upload_u8_weights(canonical, where):
+    """GX_W_U8: 8-bit weights widened on the device give the same graph as
+    32-bit ones (SSSP bit-exact vs Dijkstra); the canonical path also with the
+    asynchronous weight copy (the bench's e2e upload)."""
+    import torch
+    from paper_conf_icpp_0001n20_b200 import Graph
+    raw = graphgen.rmat(12)
+    g = from_raw(raw)
+    want = A.sssp_dijkstra(graph_to_edgelist(g), sssp_source(g))
+    if canonical:   # the caller's canonical CSR: the exact-mode export of a 32-bit upload
+        ex = upload(raw).export()
+        rp, col, w = ex["row_ptr"], ex["col"], ex["w"]
+    else:
+        rp, col, w = raw.row_ptr, raw.col, raw.w
+    w8 = w.astype(np.uint8)
+    assert np.array_equal(w8.astype(np.uint32), w)
+    if where == "device" and not canonical:
+        pytest.skip("GX_W_U8 with device pointers needs GX_CANONICAL")
+    if where == "device":
+        args = (torch.from_numpy(rp).cuda(), torch.from_numpy(col).cuda(), torch.from_numpy(w8).cuda())
+    else:
+        args = (rp, col, w8)
+    for async_upload in ([False, True] if canonical and where == "host" else [False]):
+        G = Graph.upload(ctx(), *args, canonical=canonical, async_upload=async_upload)
+        G.run("sssp", source=-1, mapping="lb")
+        assert np.array_equal(G.download("dist"), want)
+        G.run("pagerank", tol=1e-10)
+        xw, _ = A.pagerank(graph_to_edgelist(g), tol=1e-14)
+        assert np.abs(G.download("rank") - xw).sum() <= 1e-6
+
+
+@pytest.mark.parametrize("name", ["rmat12", "rmat14_C1", "uniform", "road64", "star_hub", "dups_loops", "isolated",
+                                  "single"])
+@pytest.mark.parametrize("dense", ["0", "1e-9", "0.3"])
+def test_sssp_blocked_dense_iterations_bit_exact(name, dense, monkeypatch):
+    """The blocked dense relaxation (k_sssp_pb_scatter / k_sssp_pb_gather) for
+    near-far refills: forced on every refill (GX_SSSP_DENSE=1e-9), at a 30 %
+    threshold, and off -- Dijkstra's distances bit for bit; forced, every
+    refill iteration must have run dense."""
+    monkeypatch.setenv("GX_SSSP_DENSE", dense)
+    raw = GRAPHS[name]()
+    g = from_raw(raw)
+    want = A.sssp_dijkstra(graph_to_edgelist(g), sssp_source(g))
+    G = upload(raw)
+    for _ in range(2):
+        info = G.run("sssp", source=-1, mapping="lb")
+        assert info["converged"] == 1
+        got = G.download("dist")
+        assert np.array_equal(got, want), f"{np.sum(got != want)} mismatches"
+    if dense == "0":
+        assert info["dense_iterations"] == 0
