@@ -220,6 +220,7 @@ def main():
     ap.add_argument("--no-knobs", action="store_true", help="skip the knob speedup / inaccuracy points (~60 s)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--e2e-sync", action="store_true", help="upload without GX_ASYNC_UPLOAD")
+    ap.add_argument("--e2e-w32", action="store_true", help="upload 32-bit weights (not GX_W_U8)")
     ap.add_argument("--pr-mapping", default="auto", choices=["auto", "lb", "tpv", "pb"],
                     help="PageRank sweep mapping (auto = the blocked pull on one GPU at these sizes)")
     args = ap.parse_args()
@@ -369,10 +370,10 @@ def main():
         hcol = torch.from_numpy(ex["col"]).pin_memory()
         # weights 1..100 travel as bytes (GX_W_U8, widened on the device)
         assert int(ex["w"].max()) <= 255
-        hw = torch.from_numpy(ex["w"].astype(np.uint8)).pin_memory()
+        hw = torch.from_numpy(ex["w"].view(np.int32) if args.e2e_w32 else ex["w"].astype(np.uint8)).pin_memory()
         hdist = torch.empty(n, dtype=torch.int32).pin_memory()
         hrank = torch.empty(n, dtype=torch.float64).pin_memory()
-        h2d = hrp.numel() * 8 + hcol.numel() * 4 + hw.numel() * 1
+        h2d = hrp.numel() * 8 + hcol.numel() * 4 + hw.numel() * hw.element_size()
         d2h = n * 4 + n * 8
         e2e_ms, e2e_edges = [], 0
         for i in range(args.e2e_steps + 1):
@@ -382,7 +383,8 @@ def main():
             e0.record(stream)
             # GX_ASYNC_UPLOAD: the weights' H2D overlaps the blocked PageRank
             # (structure only); SSSP joins the copy
-            G2 = gx.Graph.upload(ctx, hrp.numpy(), hcol.numpy(), hw.numpy(), canonical=True,
+            G2 = gx.Graph.upload(ctx, hrp.numpy(), hcol.numpy(),
+                                 hw.numpy().view(np.uint32) if args.e2e_w32 else hw.numpy(), canonical=True,
                                  async_upload=not args.e2e_sync)
             b = G2.run("pagerank", tol=1e-9, mapping=args.pr_mapping)
             G2.download("rank", out=hrank.numpy(), async_copy=not args.e2e_sync)   # D2H overlaps SSSP

@@ -124,6 +124,7 @@ struct PbLayout {
   DBuf q;                       // u32 [(nb+1)*nb]
   DBuf src_loc, dst_loc;        // u16 [m_pad]
   DBuf val;                     // f32 [m_pad]
+  DBuf perm;                    // u32 [m_pad]: edge index of each position (0xffffffff = padding)
   bool built() const { return q.p != nullptr; }
 };
 

@@ -405,6 +405,7 @@ struct PbArgs {
   const uint16_t* dst_loc;
   float* val;
   int64_t nb;
+  int seg_lanes;   // (3): lanes per segment -- 32: whole-warp steps (pb_scatter_async); 8 / 16: pb_scatter_groups
 };
 
 __device__ __forceinline__ float4 ld_cg_f4(const float* p) {
@@ -630,6 +631,82 @@ __device__ __forceinline__ void pb_scatter_async(const PbArgs& p, const float* s
   cp_async_wait<0>();
 }
 
+// (3) for short segments (RMAT-26: 4096 bins, ~64 entries per (bin, block)
+// segment): lane groups of G lanes (8 or 16) walk their own segments --
+// group g of a warp takes segments g, g + 32/G, ... of each 32-segment chunk
+// -- so a 64-entry segment keeps 8 lanes busy instead of leaving 24 of 32
+// idle in a whole-warp step.  Each lane runs its own DEPTH-deep cp.async
+// pipeline (wait_group is per thread), bounds read straight from q (cached).
+template <int DEPTH>
+__device__ __forceinline__ void pb_scatter_groups(const PbArgs& p, const float* s_c, const uint32_t* r0,
+                                                  const uint32_t* r1, uint64_t pf, uint4* stage, int G) {
+  const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
+  constexpr unsigned NW = PB_THREADS / 32;
+  const int64_t nb = p.nb;
+  const int S = 32 / G, gi = (int)lane / G, li = (int)lane % G;
+  int64_t j0 = (int64_t)warp * 32;
+  int k = gi;
+  uint32_t e = 0, hb = 0;
+  bool in_seg = false;
+  auto next = [&]() -> bool {   // the lane's next 8-entry group (e)
+    for (;;) {
+      if (in_seg) {
+        e += 8u * (uint32_t)G;
+        if (e < hb) return true;
+        k += S;
+      }
+      in_seg = true;
+      if (k >= 32) {
+        j0 += 32 * NW;
+        k = gi;
+      }
+      if (j0 >= nb) return false;
+      const int64_t j = j0 + k;
+      if (j >= nb) {   // the last chunk is short
+        k = 32;
+        in_seg = false;
+        continue;
+      }
+      e = __ldg(r0 + j) + 8u * (uint32_t)li;
+      hb = __ldg(r1 + j);
+      if (e < hb) return true;
+    }
+  };
+  uint32_t pe[DEPTH];
+  bool more = true;
+  int pending = 0;
+#pragma unroll
+  for (int st = 0; st < DEPTH; st++) {
+    pe[st] = 0xffffffffu;
+    if (more) more = next();
+    if (more) {
+      pe[st] = e;
+      cp_async16(stage + st * 32 + lane, p.src_loc + e, pf);
+      pending++;
+    }
+    cp_async_commit();
+  }
+  while (pending) {
+#pragma unroll
+    for (int st = 0; st < DEPTH; st++) {
+      cp_async_wait<DEPTH - 1>();
+      if (pe[st] != 0xffffffffu) {
+        pb_put8(p.val + pe[st], s_c, stage[st * 32 + lane]);
+        pending--;
+      }
+      pe[st] = 0xffffffffu;
+      if (more) more = next();
+      if (more) {
+        pe[st] = e;
+        cp_async16(stage + st * 32 + lane, p.src_loc + e, pf);
+        pending++;
+      }
+      cp_async_commit();
+    }
+  }
+  cp_async_wait<0>();
+}
+
 template <bool SLOTS>
 __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, PbArgs p) {
   extern __shared__ __align__(16) unsigned char pb_smem[];
@@ -788,7 +865,11 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
     }
     __syncthreads();
     // (3) scatter the new terms along block b's segments
-    if (GX_PB_SASYNC) {
+    if (p.seg_lanes < 32) {
+      pb_scatter_groups<PB_SDEPTH>(p, s_c, r0, r1, pf, reinterpret_cast<uint4*>(ring) + warp * PB_SDEPTH * 32,
+                                   p.seg_lanes);
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    } else if (GX_PB_SASYNC) {
       pb_scatter_async<PB_SDEPTH>(p, s_c, r0, r1, lo0, hi0, pf, reinterpret_cast<uint4*>(ring) + warp * PB_SDEPTH * 32);
       // the ring's next writes are the bulk copies (async proxy)
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -1372,6 +1453,14 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     pb.dst_loc = d.pr_pb.dst_loc.as<uint16_t>();
     pb.val = d.pr_pb.val.as<float>();
     pb.nb = d.pr_pb.nb;
+    // lanes per (bin, block) segment in the scatter: ~8 entries per lane per
+    // step, from the mean segment length (RMAT-24: 256 -> 32; RMAT-26: 64 -> 8)
+    {
+      const double mean = (double)d.pr_pb.m_pad / (double)std::max<int64_t>(1, pb.nb * pb.nb);
+      pb.seg_lanes = mean >= 192.0 ? 32 : mean >= 96.0 ? 16 : 8;
+      if (const char* e = getenv("GX_PB_SEG_LANES")) pb.seg_lanes = atoi(e);
+      GX_CHECK_ARG(pb.seg_lanes == 8 || pb.seg_lanes == 16 || pb.seg_lanes == 32, "GX_PB_SEG_LANES must be 8, 16 or 32");
+    }
     // the opt-in is per device (context): set it on every run (cheap), not
     // once per process -- a second GPU in the same process needs it too
     CUDA_OK(cudaFuncSetAttribute(k_pr_pb<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));

@@ -444,55 +444,74 @@ __global__ void k_sssp_tiles_collect(SsspAux ax, SsspState* __restrict__ st, con
   sssp_tiles_collect_dev(ax, st, st->iter, slot_tile, tmark, tlist);
 }
 
+// One WARP per tile (tiles hold S_max <= 256 members; the C3 road grid's
+// average 3.1): the members' distances go to the warp's slice of shared
+// memory, the tile's local edges ({src | dst << 8, w}) are relaxed
+// warp-stride for up to t rounds (or to the local fixed point: no lane
+// improved anything), improvements written back with red.min + the next
+// frontier bit.  A tile's first 64 edges stay in registers across the rounds
+// (2 per lane), so a small tile reads its edges from global memory once.
+// No CTA barriers: warps of a CTA work on different tiles independently.
+constexpr int LOCAL_MAX_MEMBERS = 256;   // u8 member indices
 __device__ __forceinline__ void sssp_local_dev(const int32_t* __restrict__ tptr, const int32_t* __restrict__ tmem,
                                                const int32_t* __restrict__ teptr, const uint2* __restrict__ tedges,
                                                const int32_t* __restrict__ titers, int64_t ntiles,
                                                uint32_t* __restrict__ dist, const SsspAux& ax, SsspState* __restrict__ st,
-                                               const int32_t* __restrict__ tlist = nullptr,
-                                               uint32_t* __restrict__ tmark = nullptr) {
-  __shared__ uint32_t sd[256];
+                                               const int32_t* __restrict__ tlist, uint32_t* __restrict__ tmark,
+                                               uint32_t* __restrict__ pool /* blockDim/32 x LOCAL_MAX_MEMBERS */) {
   const unsigned t = st->iter;
   if (st->stop) return;
   uint32_t* bm_next = ax.bm[(t + 1) % 3];
   const uint64_t pl = l2_evict_last();
   const uint32_t* bm_cur = ax.bm[t % 3];
+  const unsigned lane = lane_id();
+  uint32_t* sd = pool + (threadIdx.x >> 5) * LOCAL_MAX_MEMBERS;
+  const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   uint32_t my_push = 0;
   const int64_t nwork = tlist ? (int64_t)*(volatile unsigned*)&st->tiles_n[t % 3] : ntiles;
-  for (int64_t wi = blockIdx.x; wi < nwork; wi += gridDim.x) {
+  for (int64_t wi = gw; wi < nwork; wi += nw) {
     const int64_t tile = tlist ? tlist[wi] : wi;
     const int a = tptr[tile], nm = tptr[tile + 1] - a;
     const int ea = teptr[tile], ne = teptr[tile + 1] - ea;
     if (tlist) {
-      if (threadIdx.x == 0) atomicAnd(tmark + (tile >> 5), ~(1u << (tile & 31)));   // listed once per iteration
+      if (lane == 0) atomicAnd(tmark + (tile >> 5), ~(1u << (tile & 31)));   // listed once per iteration
     } else {
       // only tiles touched by this iteration: a member in the frontier or improved by the sweep
-      int touched = 0;
-      for (int i = threadIdx.x; i < nm; i += blockDim.x) {
+      bool touched = false;
+      for (int i = lane; i < nm; i += 32) {
         const uint32_t v = (uint32_t)tmem[a + i];
-        touched |= (int)(((__ldcg(bm_cur + (v >> 5)) | __ldcg(bm_next + (v >> 5))) >> (v & 31)) & 1u);
+        touched |= (((__ldcg(bm_cur + (v >> 5)) | __ldcg(bm_next + (v >> 5))) >> (v & 31)) & 1u) != 0;
       }
-      if (!__syncthreads_or(touched)) continue;
+      if (!__any_sync(FULL, touched)) continue;
     }
-    for (int i = threadIdx.x; i < nm; i += blockDim.x) sd[i] = ld_l2_u32(dist + tmem[a + i], pl);
-    __syncthreads();
+    for (int i = lane; i < nm; i += 32) sd[i] = ld_l2_u32(dist + tmem[a + i], pl);
+    // the first 64 local edges in registers
+    uint2 e0 = lane < ne ? tedges[ea + lane] : make_uint2(0, 0);
+    uint2 e1 = lane + 32 < ne ? tedges[ea + 32 + lane] : make_uint2(0, 0);
+    __syncwarp();
     const int iters = titers[tile];
-    for (int r = 0; r < iters; r++) {
-      int ch = 0;
-      for (int i = threadIdx.x; i < ne; i += blockDim.x) {
-        const uint2 p = tedges[ea + i];
-        const uint32_t src = p.x & 0xff, dst = (p.x >> 8) & 0xff;
-        const uint32_t du = sd[src];
-        if (du != INF) {
-          const uint32_t nd = sat_add(du, p.y);
-          if (nd < sd[dst]) {
-            atomicMin(&sd[dst], nd);
-            ch = 1;
-          }
-        }
+    auto relax = [&](uint2 p) -> bool {
+      const uint32_t du = sd[p.x & 0xff];
+      if (du == INF) return false;
+      const uint32_t nd = sat_add(du, p.y);
+      const uint32_t dst = (p.x >> 8) & 0xff;
+      if (nd < sd[dst]) {
+        atomicMin(&sd[dst], nd);
+        return true;
       }
-      if (!__syncthreads_or(ch)) break;
+      return false;
+    };
+    for (int r = 0; r < iters; r++) {
+      bool ch = false;
+      if (lane < ne) ch |= relax(e0);
+      if (lane + 32 < ne) ch |= relax(e1);
+      for (int i = 64 + lane; i < ne; i += 32) ch |= relax(tedges[ea + i]);
+      if (!__any_sync(FULL, ch)) break;
+      __syncwarp();
     }
-    for (int i = threadIdx.x; i < nm; i += blockDim.x) {
+    __syncwarp();
+    for (int i = lane; i < nm; i += 32) {
       const uint32_t v = (uint32_t)tmem[a + i];
       const uint32_t nd = sd[i];
       if (nd < ld_l2_u32(dist + v, pl)) {
@@ -501,7 +520,7 @@ __device__ __forceinline__ void sssp_local_dev(const int32_t* __restrict__ tptr,
         my_push++;
       }
     }
-    __syncthreads();
+    __syncwarp();
   }
   flush_counters(st, t, 0, 0, my_push, INF);
 }
@@ -511,7 +530,8 @@ __global__ void __launch_bounds__(256) k_sssp_local(const int32_t* __restrict__ 
                                                     const int32_t* __restrict__ titers, int64_t ntiles,
                                                     uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st,
                                                     const int32_t* __restrict__ tlist, uint32_t* __restrict__ tmark) {
-  sssp_local_dev(tptr, tmem, teptr, tedges, titers, ntiles, dist, ax, st, tlist, tmark);
+  __shared__ uint32_t pool[(256 / 32) * LOCAL_MAX_MEMBERS];
+  sssp_local_dev(tptr, tmem, teptr, tedges, titers, ntiles, dist, ax, st, tlist, tmark, pool);
 }
 
 // ---------------------------------------------------------------- §2.4 merge
@@ -832,6 +852,7 @@ struct SsspLoop {
 
 constexpr int PERSIST_POOL = SB_WARPS * 1024 * 4;   // 32 KB at 256 threads: LB compaction buffer / block-mode queues
 static_assert(2 * BLK_Q * 4 + BLK_MAX / 8 + 16 <= PERSIST_POOL, "block-mode buffers must fit the pool");
+static_assert((PERSIST_TPB / 32) * LOCAL_MAX_MEMBERS * 4 <= PERSIST_POOL, "local-pass slices must fit the pool");
 
 #ifndef GX_SSSP_MINB
 #define GX_SSSP_MINB (1024 / GX_SSSP_TPB)
@@ -877,7 +898,8 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
     if (a.ntiles) {
       sssp_tiles_collect_dev(a.ax, st, t, a.slot_tile, a.tmark, a.tlist);
       grid.sync();
-      sssp_local_dev(a.tptr, a.tmem, a.teptr, a.tedges, a.titers, a.ntiles, a.dist, a.ax, st, a.tlist, a.tmark);
+      sssp_local_dev(a.tptr, a.tmem, a.teptr, a.tedges, a.titers, a.ntiles, a.dist, a.ax, st, a.tlist, a.tmark,
+                     reinterpret_cast<uint32_t*>(pool));
       grid.sync();
     }
     bool final_merge = false;
@@ -1646,7 +1668,7 @@ static void run_sssp_dist(gx_graph* g, const gx_run_opts& o, gx_run_info& info, 
   int occ = 0;
   CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sssp_lb, 256, 0));
   const int grid_lb = std::max(1, occ) * c->num_sms;
-  const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 8));
+  const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_tiles + 7) / 8, (int64_t)c->num_sms * 8));   // a warp per tile
   const int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 7) / 8, (int64_t)c->num_sms * 8));
   const bool merge_min = g->knobs.merge_op == GX_MERGE_MIN;
   std::vector<void*> dl, xsl, xml;
@@ -1873,7 +1895,7 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
   int occt = 0;
   CUDA_OK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occt, k_sssp_tpv, 256, 0));
   const int grid_tpv = std::max(1, occt) * c->num_sms;
-  const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 8));
+  const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_tiles + 7) / 8, (int64_t)c->num_sms * 8));   // a warp per tile
   const int grid_merge = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_groups + 7) / 8, (int64_t)c->num_sms * 8));
   const bool merge_min = g->knobs.merge_op == GX_MERGE_MIN;
   const int grid_split = grid_for(c, nwords);
