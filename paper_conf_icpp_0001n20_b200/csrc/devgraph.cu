@@ -203,8 +203,7 @@ static void build_csc_and_tiles(gx_graph* g) {
 // two local indices; histogram of keys for the segment offsets
 __global__ void k_pb_pairs(const uint32_t* __restrict__ rp, const uint32_t* __restrict__ colp, uint32_t cstride,
                            int64_t n, uint32_t nb,
-                           uint32_t* __restrict__ key, uint32_t* __restrict__ val, uint32_t* __restrict__ cnt,
-                           uint32_t* __restrict__ eid) {
+                           uint32_t* __restrict__ key, uint32_t* __restrict__ val, uint32_t* __restrict__ cnt) {
   int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   int lane = threadIdx.x & 31;
   int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -216,7 +215,26 @@ __global__ void k_pb_pairs(const uint32_t* __restrict__ rp, const uint32_t* __re
       const uint32_t k = (v / PB_R) * nb + bu;
       key[e] = k;
       val[e] = lu | ((v % PB_R) << 16);
-      eid[e] = e;
+      atomicAdd(&cnt[k], 1u);
+    }
+  }
+}
+// the same with the edge's 8-bit weight in the payload's high word (weights
+// resident and <= 255): the sort then also yields the weights in blocked order
+__global__ void k_pb_pairs_w(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj, int64_t n, uint32_t nb,
+                             uint32_t* __restrict__ key, unsigned long long* __restrict__ val,
+                             uint32_t* __restrict__ cnt) {
+  int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  int lane = threadIdx.x & 31;
+  int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t u = warp; u < n; u += nw) {
+    const uint32_t a = rp[u], b = rp[u + 1];
+    const uint32_t bu = (uint32_t)(u / PB_R), lu = (uint32_t)(u % PB_R);
+    for (uint32_t e = a + lane; e < b; e += 32) {
+      const uint2 vw = adj[e];
+      const uint32_t k = (vw.x / PB_R) * nb + bu;
+      key[e] = k;
+      val[e] = ((unsigned long long)vw.y << 32) | (lu | ((vw.x % PB_R) << 16));
       atomicAdd(&cnt[k], 1u);
     }
   }
@@ -228,19 +246,20 @@ __global__ void k_pb_padcnt(const uint32_t* __restrict__ cnt, uint32_t* __restri
     pc[i] = i + 1 < nk ? (cnt[i] + PB_PAD - 1) / PB_PAD * PB_PAD : 0u;
 }
 
-// element i of the sorted order (key k, edge e) -> padded position
-// pos = P2[k] + (i - P[k]): its local indices, and perm[pos] = e (the
-// weights in blocked order are one gather through perm, ensure_pb_w)
-__global__ void k_pb_place(const uint32_t* __restrict__ key, const uint32_t* __restrict__ eid,
-                           const uint32_t* __restrict__ loc, const uint32_t* __restrict__ P,
-                           const uint32_t* __restrict__ P2, uint16_t* __restrict__ sl, uint16_t* __restrict__ dl,
-                           uint32_t* __restrict__ perm, int64_t m) {
+// element i of the sorted order (key k) -> padded position P2[k] + (i - P[k])
+template <class V>
+__global__ void k_pb_place(const uint32_t* __restrict__ key, const V* __restrict__ pay,
+                           const uint32_t* __restrict__ P, const uint32_t* __restrict__ P2, uint16_t* __restrict__ sl,
+                           uint16_t* __restrict__ dl, uint8_t* __restrict__ w8, int64_t m) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
-    const uint32_t k = key[i], e = eid[i], p = loc[e];
+    const uint32_t k = key[i];
+    const V p = pay[i];
     const uint32_t pos = P2[k] + ((uint32_t)i - P[k]);
     sl[pos] = (uint16_t)(p & 0xffffu);
-    dl[pos] = (uint16_t)(p >> 16);
-    perm[pos] = e;
+    dl[pos] = (uint16_t)((p >> 16) & 0xffffu);
+    if constexpr (sizeof(V) == 8) {
+      if (w8) w8[pos] = (uint8_t)(p >> 32);
+    }
   }
 }
 
@@ -270,31 +289,46 @@ void ensure_pb(gx_graph* g) {
   P.alloc(c, sizeof(uint32_t) * nk);
   P2.alloc(c, sizeof(uint32_t) * nk);
   CUDA_OK(cudaMemsetAsync(cnt.p, 0, sizeof(uint32_t) * nk, s));
-  DBuf k0, k1, v0, v1, loc, tmp;
+  // with resident 8-bit weights the sort carries them too (SSSP's dense
+  // relaxation reads them in blocked order); an asynchronous upload's
+  // blocked PageRank builds from col alone, and SSSP then runs without the
+  // dense pass on this graph (it never gathers the weights at random)
+  const bool with_w = d.max_w <= 255 && !g->maxw_pending && m > 0;
+  DBuf k0, k1, v0, v1, tmp;
   cub::DoubleBuffer<uint32_t> dk, dv;
+  cub::DoubleBuffer<unsigned long long> dv64;
   if (m > 0) {
     k0.alloc(c, sizeof(uint32_t) * m);
     k1.alloc(c, sizeof(uint32_t) * m);
-    v0.alloc(c, sizeof(uint32_t) * m);
-    v1.alloc(c, sizeof(uint32_t) * m);
-    loc.alloc(c, sizeof(uint32_t) * m);
-    // exact mode reads the uploaded col (not the {col, w} pairs, which an
-    // asynchronous upload may still be producing)
-    const bool ident = d.identity && g->in_col.p;
-    k_pb_pairs<<<grid_for(c, n * 32), 256, 0, s>>>(d.rp.as<uint32_t>(),
-                                                   ident ? g->in_col.as<uint32_t>() : d.adj.as<uint32_t>(),
-                                                   ident ? 1u : 2u, n, (uint32_t)nb,
-                                                   k0.as<uint32_t>(), loc.as<uint32_t>(), cnt.as<uint32_t>(),
-                                                   v0.as<uint32_t>());
-    CUDA_OK(cudaGetLastError());
+    v0.alloc(c, (with_w ? 8 : 4) * m);
+    v1.alloc(c, (with_w ? 8 : 4) * m);
     int bits = 1;
     while ((int64_t(1) << bits) < nb * nb) bits++;
     size_t tb = 0;
     dk = cub::DoubleBuffer<uint32_t>(k0.as<uint32_t>(), k1.as<uint32_t>());
-    dv = cub::DoubleBuffer<uint32_t>(v0.as<uint32_t>(), v1.as<uint32_t>());
-    CUDA_OK(cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv, (int64_t)m, 0, bits, s));
-    tmp.alloc(c, tb);
-    CUDA_OK(cub::DeviceRadixSort::SortPairs(tmp.p, tb, dk, dv, (int64_t)m, 0, bits, s));
+    if (with_w) {
+      k_pb_pairs_w<<<grid_for(c, n * 32), 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), n, (uint32_t)nb,
+                                                       k0.as<uint32_t>(), v0.as<unsigned long long>(),
+                                                       cnt.as<uint32_t>());
+      CUDA_OK(cudaGetLastError());
+      dv64 = cub::DoubleBuffer<unsigned long long>(v0.as<unsigned long long>(), v1.as<unsigned long long>());
+      CUDA_OK(cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv64, (int64_t)m, 0, bits, s));
+      tmp.alloc(c, tb);
+      CUDA_OK(cub::DeviceRadixSort::SortPairs(tmp.p, tb, dk, dv64, (int64_t)m, 0, bits, s));
+    } else {
+      // exact mode reads the uploaded col (not the {col, w} pairs, which an
+      // asynchronous upload may still be producing)
+      const bool ident = d.identity && g->in_col.p;
+      k_pb_pairs<<<grid_for(c, n * 32), 256, 0, s>>>(d.rp.as<uint32_t>(),
+                                                     ident ? g->in_col.as<uint32_t>() : d.adj.as<uint32_t>(),
+                                                     ident ? 1u : 2u, n, (uint32_t)nb,
+                                                     k0.as<uint32_t>(), v0.as<uint32_t>(), cnt.as<uint32_t>());
+      CUDA_OK(cudaGetLastError());
+      dv = cub::DoubleBuffer<uint32_t>(v0.as<uint32_t>(), v1.as<uint32_t>());
+      CUDA_OK(cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv, (int64_t)m, 0, bits, s));
+      tmp.alloc(c, tb);
+      CUDA_OK(cub::DeviceRadixSort::SortPairs(tmp.p, tb, dk, dv, (int64_t)m, 0, bits, s));
+    }
   }
   k_pb_padcnt<<<grid_for(c, nk), 256, 0, s>>>(cnt.as<uint32_t>(), pc.as<uint32_t>(), nk);
   size_t sb = 0;
@@ -312,16 +346,25 @@ void ensure_pb(gx_graph* g) {
   L.src_loc.alloc(c, sizeof(uint16_t) * mm);
   L.dst_loc.alloc(c, sizeof(uint16_t) * mm);
   L.val.alloc(c, sizeof(float) * mm);
-  L.perm.alloc(c, sizeof(uint32_t) * mm);
-  launch_fill_u32(c, L.perm.as<uint32_t>(), 0xffffffffu, mm);   // padding: no edge
+  if (with_w) {
+    d.pb_w8.alloc(c, (size_t)mm);
+    CUDA_OK(cudaMemsetAsync(d.pb_w8.p, 0, (size_t)mm, s));
+  }
   // padding entries: source index PB_R (a zero term in shared memory), sink 0
   launch_fill_u32(c, L.src_loc.as<uint32_t>(), (uint32_t)PB_R * 0x10001u, mm / 2);   // mm is a multiple of 8
   CUDA_OK(cudaMemsetAsync(L.dst_loc.p, 0, sizeof(uint16_t) * mm, s));
   CUDA_OK(cudaMemsetAsync(L.val.p, 0, sizeof(float) * mm, s));
   if (m > 0)
-    k_pb_place<<<grid_for(c, m), 256, 0, s>>>(dk.Current(), dv.Current(), loc.as<uint32_t>(), P.as<uint32_t>(),
-                                              P2.as<uint32_t>(), L.src_loc.as<uint16_t>(), L.dst_loc.as<uint16_t>(),
-                                              L.perm.as<uint32_t>(), m);
+  {
+    if (with_w)
+      k_pb_place<unsigned long long><<<grid_for(c, m), 256, 0, s>>>(dk.Current(), dv64.Current(), P.as<uint32_t>(),
+                                                                    P2.as<uint32_t>(), L.src_loc.as<uint16_t>(),
+                                                                    L.dst_loc.as<uint16_t>(), d.pb_w8.as<uint8_t>(), m);
+    else
+      k_pb_place<uint32_t><<<grid_for(c, m), 256, 0, s>>>(dk.Current(), dv.Current(), P.as<uint32_t>(),
+                                                          P2.as<uint32_t>(), L.src_loc.as<uint16_t>(),
+                                                          L.dst_loc.as<uint16_t>(), nullptr, m);
+  }
   L.q.alloc(c, sizeof(uint32_t) * (nb + 1) * nb);
   k_pb_transpose<<<grid_for(c, (nb + 1) * nb), 256, 0, s>>>(P2.as<uint32_t>(), L.q.as<uint32_t>(), nb);
   CUDA_OK(cudaGetLastError());
@@ -329,28 +372,10 @@ void ensure_pb(gx_graph* g) {
 }
 
 // ---- the edge weights in the blocked order (SSSP's dense relaxation, sssp.cu) ----
-__global__ void k_pb_gather_w8(const uint32_t* __restrict__ perm, const uint2* __restrict__ adj,
-                               uint8_t* __restrict__ w8, int64_t mm) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < mm; i += (int64_t)gridDim.x * blockDim.x) {
-    const uint32_t e = perm[i];
-    w8[i] = e == 0xffffffffu ? (uint8_t)0 : (uint8_t)adj[e].y;
-  }
-}
-
-// w8[pos] = weight of the edge at blocked position pos (padding 0): one gather
-// through the layout's permutation; needs max w <= 255
-void ensure_pb_w(gx_graph* g) {
-  DevGraph& d = g->dg;
-  if (d.pb_w8.p) return;
+// true when the blocked layout carries them (built with resident weights <= 255)
+bool ensure_pb_w(gx_graph* g) {
   ensure_pb(g);
-  resolve_pending(g);
-  Ctx* c = g->ctx;
-  cudaStream_t s = c->stream;
-  const int64_t mm = std::max<int64_t>(d.pr_pb.m_pad, 8);
-  d.pb_w8.alloc(c, (size_t)std::max<int64_t>(mm, 16));
-  k_pb_gather_w8<<<grid_for(c, mm), 256, 0, s>>>(d.pr_pb.perm.as<uint32_t>(), d.adj.as<uint2>(), d.pb_w8.as<uint8_t>(),
-                                                 mm);
-  CUDA_OK(cudaGetLastError());
+  return g->dg.pb_w8.p != nullptr;
 }
 
 // join the GX_ASYNC_UPLOAD work into the ctx stream; read the weights' maximum

@@ -405,7 +405,6 @@ struct PbArgs {
   const uint16_t* dst_loc;
   float* val;
   int64_t nb;
-  int seg_lanes;   // (3): lanes per segment -- 32: whole-warp steps (pb_scatter_async); 8 / 16: pb_scatter_groups
 };
 
 __device__ __forceinline__ float4 ld_cg_f4(const float* p) {
@@ -631,82 +630,6 @@ __device__ __forceinline__ void pb_scatter_async(const PbArgs& p, const float* s
   cp_async_wait<0>();
 }
 
-// (3) for short segments (RMAT-26: 4096 bins, ~64 entries per (bin, block)
-// segment): lane groups of G lanes (8 or 16) walk their own segments --
-// group g of a warp takes segments g, g + 32/G, ... of each 32-segment chunk
-// -- so a 64-entry segment keeps 8 lanes busy instead of leaving 24 of 32
-// idle in a whole-warp step.  Each lane runs its own DEPTH-deep cp.async
-// pipeline (wait_group is per thread), bounds read straight from q (cached).
-template <int DEPTH>
-__device__ __forceinline__ void pb_scatter_groups(const PbArgs& p, const float* s_c, const uint32_t* r0,
-                                                  const uint32_t* r1, uint64_t pf, uint4* stage, int G) {
-  const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
-  constexpr unsigned NW = PB_THREADS / 32;
-  const int64_t nb = p.nb;
-  const int S = 32 / G, gi = (int)lane / G, li = (int)lane % G;
-  int64_t j0 = (int64_t)warp * 32;
-  int k = gi;
-  uint32_t e = 0, hb = 0;
-  bool in_seg = false;
-  auto next = [&]() -> bool {   // the lane's next 8-entry group (e)
-    for (;;) {
-      if (in_seg) {
-        e += 8u * (uint32_t)G;
-        if (e < hb) return true;
-        k += S;
-      }
-      in_seg = true;
-      if (k >= 32) {
-        j0 += 32 * NW;
-        k = gi;
-      }
-      if (j0 >= nb) return false;
-      const int64_t j = j0 + k;
-      if (j >= nb) {   // the last chunk is short
-        k = 32;
-        in_seg = false;
-        continue;
-      }
-      e = __ldg(r0 + j) + 8u * (uint32_t)li;
-      hb = __ldg(r1 + j);
-      if (e < hb) return true;
-    }
-  };
-  uint32_t pe[DEPTH];
-  bool more = true;
-  int pending = 0;
-#pragma unroll
-  for (int st = 0; st < DEPTH; st++) {
-    pe[st] = 0xffffffffu;
-    if (more) more = next();
-    if (more) {
-      pe[st] = e;
-      cp_async16(stage + st * 32 + lane, p.src_loc + e, pf);
-      pending++;
-    }
-    cp_async_commit();
-  }
-  while (pending) {
-#pragma unroll
-    for (int st = 0; st < DEPTH; st++) {
-      cp_async_wait<DEPTH - 1>();
-      if (pe[st] != 0xffffffffu) {
-        pb_put8(p.val + pe[st], s_c, stage[st * 32 + lane]);
-        pending--;
-      }
-      pe[st] = 0xffffffffu;
-      if (more) more = next();
-      if (more) {
-        pe[st] = e;
-        cp_async16(stage + st * 32 + lane, p.src_loc + e, pf);
-        pending++;
-      }
-      cp_async_commit();
-    }
-  }
-  cp_async_wait<0>();
-}
-
 template <bool SLOTS>
 __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, PbArgs p) {
   extern __shared__ __align__(16) unsigned char pb_smem[];
@@ -865,11 +788,7 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
     }
     __syncthreads();
     // (3) scatter the new terms along block b's segments
-    if (p.seg_lanes < 32) {
-      pb_scatter_groups<PB_SDEPTH>(p, s_c, r0, r1, pf, reinterpret_cast<uint4*>(ring) + warp * PB_SDEPTH * 32,
-                                   p.seg_lanes);
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-    } else if (GX_PB_SASYNC) {
+    if (GX_PB_SASYNC) {
       pb_scatter_async<PB_SDEPTH>(p, s_c, r0, r1, lo0, hi0, pf, reinterpret_cast<uint4*>(ring) + warp * PB_SDEPTH * 32);
       // the ring's next writes are the bulk copies (async proxy)
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -1088,6 +1007,142 @@ __global__ void __launch_bounds__(PRL_THREADS) k_pr_local(PrArgs a, const int32_
       if (!Ds[i]) my_dang += xs[i] - old;
     }
     __syncthreads();
+  }
+  pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
+}
+
+// Warp-per-tile version of k_pr_local (the default): each warp owns one tile
+// at a time in its slice of dynamic shared memory (members, their values,
+// sink-sorted local in-edges), so a 3-member tile costs a few warp
+// instructions and no CTA barrier; the steps and the arithmetic are those of
+// k_pr_local above.  Slice layout for TM members (multiple of 32) and TE
+// local edges: double xs, xn, ext, cs [TM] | u32 Ds [TM] | i32 id [TM] |
+// i32 in_ptr [TM + 1], cur [TM] | u8 fixed [TM] | u8 in_src [TE].
+constexpr int PRLW_THREADS = 256;
+__host__ __device__ inline size_t prlw_slice_bytes(int TM, int TE) {
+  return (((size_t)TM * (4 * 8 + 4 + 4 + 4 + 4 + 1) + 4 + (size_t)TE) + 15) / 16 * 16;
+}
+template <bool SLOTS>
+__global__ void __launch_bounds__(PRLW_THREADS) k_pr_local_warp(PrArgs a, const int32_t* __restrict__ tptr,
+                                                              const int32_t* __restrict__ tmem,
+                                                              const int32_t* __restrict__ teptr,
+                                                              const uint2* __restrict__ tedges,
+                                                              const int32_t* __restrict__ titers, int64_t ntiles,
+                                                              int TM, int TE) {
+  extern __shared__ __align__(16) unsigned char prlw_smem[];
+  __shared__ double s_red[32];
+  PrState* st = a.st;
+  if (st->stop) return;
+  const unsigned t = st->iter;
+  const float* cin = a.contrib[t & 1];
+  float* cout = a.contrib[(t + 1) & 1];
+  const double sc = st->scale;
+  const double addc = a.base + a.damp * sc * st->dang[t % 3] * a.invN;
+  double my_delta = 0, my_dang = 0, my_mass = 0;
+  const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
+  unsigned char* sl = prlw_smem + warp * prlw_slice_bytes(TM, TE);
+  double* xs = reinterpret_cast<double*>(sl);
+  double* xn = xs + TM;
+  double* ext = xn + TM;
+  double* cs = ext + TM;
+  uint32_t* Ds = reinterpret_cast<uint32_t*>(cs + TM);
+  int32_t* id = reinterpret_cast<int32_t*>(Ds + TM);
+  int* in_ptr = id + TM;
+  int* cur = in_ptr + TM + 1;
+  uint8_t* fixed = reinterpret_cast<uint8_t*>(cur + TM);
+  uint8_t* in_src = fixed + TM;
+  const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t tile = gw; tile < ntiles; tile += nw) {
+    const int b0 = tptr[tile], nm = tptr[tile + 1] - b0;
+    const int e0 = teptr[tile], ne = teptr[tile + 1] - e0;
+    for (int i = lane; i < nm; i += 32) {
+      const int32_t v = tmem[b0 + i];
+      fixed[i] = SLOTS && (a.kind[v] != OWNER || (a.gid && a.gid[v] >= 0));
+      xs[i] = a.x[v];
+      Ds[i] = a.D[v];
+      id[i] = v;
+      cur[i] = 0;
+    }
+    __syncwarp();
+    for (int e = lane; e < ne; e += 32) atomicAdd(&cur[(tedges[e0 + e].x >> 8) & 0xff], 1);
+    __syncwarp();
+    // exclusive scan of the in-degrees (nm <= 255: 8 steps of the warp scan)
+    int carry = 0;
+    for (int i0 = 0; i0 < nm; i0 += 32) {
+      const int i = i0 + lane;
+      const int c = i < nm ? cur[i] : 0;
+      const int inc = (int)warp_incl_scan_u32((uint32_t)c);
+      if (i < nm) {
+        in_ptr[i] = carry + inc - c;
+        cur[i] = carry + inc - c;
+      }
+      carry += __shfl_sync(FULL, inc, 31);
+    }
+    if (lane == 0) in_ptr[nm] = carry;
+    __syncwarp();
+    // edges regrouped by sink member, tile-edge order within a sink (match_any ranks)
+    for (int c0 = 0; c0 < ne; c0 += 32) {
+      const int e = c0 + (int)lane;
+      const bool ok = e < ne;
+      const uint32_t px = ok ? tedges[e0 + e].x : 0u;
+      const int dd = ok ? (int)((px >> 8) & 0xff) : 256 + (int)lane;
+      const unsigned same = __match_any_sync(FULL, dd);
+      const int rank = __popc(same & lanemask_lt());
+      if (ok) in_src[cur[dd] + rank] = (uint8_t)(px & 0xff);
+      __syncwarp();
+      if (ok && rank == 0) cur[dd] += __popc(same);
+      __syncwarp();
+    }
+    // external inflow per member: the warp walks the member's CSC in-edges
+    for (int i = 0; i < nm; i++) {
+      double in = 0.0;
+      if (!fixed[i]) {
+        const int32_t v = id[i];
+        for (uint32_t e = a.crp[v] + lane; e < a.crp[v + 1]; e += 32) {
+          const int32_t u = a.csrc[e];
+          int lo = 0, hi = nm;   // members are sorted slot ids
+          while (lo < hi) {
+            const int mid = (lo + hi) >> 1;
+            if (id[mid] < u) lo = mid + 1;
+            else hi = mid;
+          }
+          const bool inside = lo < nm && id[lo] == u && !fixed[lo];
+          if (!inside) in += (double)cin[u];
+        }
+      }
+      in = warp_sum_f64(in);
+      if (lane == 0) ext[i] = sc * in;
+    }
+    __syncwarp();
+    const int iters = titers[tile];
+    for (int r = 0; r < iters; r++) {
+      for (int i = lane; i < nm; i += 32) cs[i] = (!fixed[i] && Ds[i]) ? xs[i] / (double)Ds[i] : 0.0;
+      __syncwarp();
+      for (int i = lane; i < nm; i += 32) {
+        if (fixed[i]) {
+          xn[i] = xs[i];
+          continue;
+        }
+        double in = ext[i];
+        for (int k = in_ptr[i]; k < in_ptr[i + 1]; k++) in += cs[in_src[k]];
+        xn[i] = addc + a.damp * in;
+      }
+      __syncwarp();
+      for (int i = lane; i < nm; i += 32) xs[i] = xn[i];
+      __syncwarp();
+    }
+    for (int i = lane; i < nm; i += 32) {
+      if (fixed[i]) continue;
+      const int32_t v = id[i];
+      const double old = a.x[v];
+      a.x[v] = xs[i];
+      cout[v] = Ds[i] ? (float)(xs[i] / (double)Ds[i]) : 0.0f;
+      my_delta += fabs(xs[i] - old);
+      my_mass += xs[i] - old;
+      if (!Ds[i]) my_dang += xs[i] - old;
+    }
+    __syncwarp();
   }
   pr_flush(st, t, my_delta, my_dang, my_mass, s_red);
 }
@@ -1453,14 +1508,6 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     pb.dst_loc = d.pr_pb.dst_loc.as<uint16_t>();
     pb.val = d.pr_pb.val.as<float>();
     pb.nb = d.pr_pb.nb;
-    // lanes per (bin, block) segment in the scatter: ~8 entries per lane per
-    // step, from the mean segment length (RMAT-24: 256 -> 32; RMAT-26: 64 -> 8)
-    {
-      const double mean = (double)d.pr_pb.m_pad / (double)std::max<int64_t>(1, pb.nb * pb.nb);
-      pb.seg_lanes = mean >= 192.0 ? 32 : mean >= 96.0 ? 16 : 8;
-      if (const char* e = getenv("GX_PB_SEG_LANES")) pb.seg_lanes = atoi(e);
-      GX_CHECK_ARG(pb.seg_lanes == 8 || pb.seg_lanes == 16 || pb.seg_lanes == 32, "GX_PB_SEG_LANES must be 8, 16 or 32");
-    }
     // the opt-in is per device (context): set it on every run (cheap), not
     // once per process -- a second GPU in the same process needs it too
     CUDA_OK(cudaFuncSetAttribute(k_pr_pb<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
@@ -1476,6 +1523,10 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     a.tpv_nslices = d.tpv_nslices;
   }
 
+  if (tiles) {   // the warp-per-tile local pass may need more than 48 KB of dynamic shared memory
+    CUDA_OK(cudaFuncSetAttribute(k_pr_local_warp<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+    CUDA_OK(cudaFuncSetAttribute(k_pr_local_warp<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+  }
   cudaEvent_t e0, e1;
   CUDA_OK(cudaEventCreate(&e0));
   CUDA_OK(cudaEventCreate(&e1));
@@ -1535,6 +1586,22 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     kt.end();
     nl++;
     if (tiles) {
+      // a warp per tile (k_pr_local_warp); GX_PR_LOCAL_CTA=1: the CTA-per-tile k_pr_local
+      const int TM = (int)((std::max<int64_t>(d.t_max_members, 1) + 31) / 32 * 32);
+      const int TE = (int)std::max<int64_t>(d.t_max_edges, 16);
+      const size_t wsm = prlw_slice_bytes(TM, TE) * (PRLW_THREADS / 32);
+      if (!getenv("GX_PR_LOCAL_CTA") && wsm <= 200 * 1024) {
+        const int grid_lw = (int)std::max<int64_t>(1, std::min<int64_t>((d.n_tiles + 7) / 8, (int64_t)c->num_sms * 8));
+        if (slots)
+          k_pr_local_warp<true><<<grid_lw, PRLW_THREADS, wsm, s>>>(a, d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(),
+                                                                  d.t_eptr.as<int32_t>(), d.t_edges.as<uint2>(),
+                                                                  d.t_iters.as<int32_t>(), d.n_tiles, TM, TE);
+        else
+          k_pr_local_warp<false><<<grid_lw, PRLW_THREADS, wsm, s>>>(a, d.t_ptr.as<int32_t>(), d.t_members.as<int32_t>(),
+                                                                   d.t_eptr.as<int32_t>(), d.t_edges.as<uint2>(),
+                                                                   d.t_iters.as<int32_t>(), d.n_tiles, TM, TE);
+        nl++;
+      } else {
       const int grid_local = (int)std::max<int64_t>(1, std::min<int64_t>(d.n_tiles, (int64_t)c->num_sms * 16));
       const size_t prl_smem = (size_t)std::max<int64_t>(d.t_max_edges, 16);
       if (slots)
@@ -1546,6 +1613,7 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
                                                      d.t_eptr.as<int32_t>(), d.t_edges.as<uint2>(),
                                                      d.t_iters.as<int32_t>(), d.n_tiles);
       nl++;
+      }
     }
     if (d.n_groups) {
       k_pr_merge<<<grid_merge, 256, 0, s>>>(a, d.gptr.as<int32_t>(), d.gslots.as<int32_t>(), d.n_groups);

@@ -1854,8 +1854,9 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
                         !want_lh && d.max_w <= 255 && d.m_slots > 0 && !getenv("GX_SSSP_BLOCK") &&
                         !(o.profile && getenv("GX_SSSP_TRACE"));
   SsspPb spb{};
-  if (dense_ok) {
-    ensure_pb_w(g);
+  bool dense_on = dense_ok;
+  if (dense_on) dense_on = ensure_pb_w(g);   // false after an asynchronous upload's structure-only layout
+  if (dense_on) {
     spb.q = d.pr_pb.q.as<uint32_t>();
     spb.src_loc = d.pr_pb.src_loc.as<uint16_t>();
     spb.dst_loc = d.pr_pb.dst_loc.as<uint16_t>();
@@ -2046,7 +2047,7 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
     }
     void* args[] = {&L};
     kt.begin();
-    L.dense_edges = dense_ok ? (unsigned long long)std::max(1.0, dense_frac * (double)d.n_slots) : 0ull;
+    L.dense_edges = dense_on ? (unsigned long long)std::max(1.0, dense_frac * (double)d.n_slots) : 0ull;
     if (L.trace) k_stamp<<<1, 1, 0, s>>>(trace_buf.as<unsigned long long>());
     for (;;) {
       CUDA_OK(cudaLaunchCooperativeKernel((void*)k_sssp_persist, dim3((unsigned)(occp * c->num_sms)), dim3(PERSIST_TPB),

@@ -459,18 +459,3 @@ def test_sssp_blocked_dense_iterations_bit_exact(name, dense, monkeypatch):
         assert np.array_equal(got, want), f"{np.sum(got != want)} mismatches"
     if dense == "0":
         assert info["dense_iterations"] == 0
-
-
-@pytest.mark.parametrize("name", ["rmat14_C1", "uniform", "road64", "star_hub", "dups_loops"])
-@pytest.mark.parametrize("lanes", ["8", "16", "32"])
-def test_pagerank_blocked_scatter_lane_groups(name, lanes, monkeypatch):
-    """The blocked pull's scatter with 8 / 16 lanes per (bin, block) segment
-    (pb_scatter_groups, chosen for short segments such as RMAT-26's) and the
-    whole-warp scatter reach the oracle's PageRank within L1 1e-6."""
-    monkeypatch.setenv("GX_PB_SEG_LANES", lanes)
-    raw = GRAPHS[name]()
-    g = from_raw(raw)
-    want, _ = A.pagerank(graph_to_edgelist(g), tol=1e-14)
-    G = upload(raw)
-    G.run("pagerank", tol=1e-11, max_iters=5000, mapping="pb")
-    assert np.abs(G.download("rank") - want).sum() <= 1e-6

@@ -221,3 +221,22 @@ def test_n3_sssp_pagerank_on_GL(gname, kname, mapping):
     xw, _ = A.pagerank(L, tol=1e-14)
     G.run("pagerank", tol=1e-11, max_iters=5000, mapping=mapping)
     assert np.abs(G.download("rank") - xw).sum() <= 1e-6
+
+
+@pytest.mark.parametrize("gname", list(GRAPHS))
+@pytest.mark.parametrize("variant", ["warp", "cta"])
+@pytest.mark.parametrize("mapping", ["lb", "pb"])
+def test_pagerank_local_pass_variants(gname, variant, mapping, monkeypatch):
+    """The §3 PageRank local pass, one warp per tile (default, k_pr_local_warp)
+    and one CTA per tile (GX_PR_LOCAL_CTA=1, k_pr_local): same fixed point
+    (Theorem E3), within L1 1e-6 of the oracle's PageRank of G_L."""
+    if variant == "cta":
+        monkeypatch.setenv("GX_PR_LOCAL_CTA", "1")
+    raw = GRAPHS[gname]()
+    g = from_raw(raw)
+    kn = T.Knobs(smem=True, cc_threshold=0.3, added_edge_budget=-1)
+    want, _ = A.pagerank(T.transform(g, kn).logical(), tol=1e-14)
+    G = upload(raw)
+    G.transform(knobs_c(kn))
+    G.run("pagerank", mapping=mapping, tol=1e-11, max_iters=5000)
+    assert np.abs(G.download("rank") - want).sum() <= 1e-6
