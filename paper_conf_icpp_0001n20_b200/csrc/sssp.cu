@@ -545,7 +545,7 @@ __device__ __forceinline__ void sssp_merge_dev(const int32_t* __restrict__ gptr,
                                                int64_t ngroups, int merge_min, uint32_t* __restrict__ dist,
                                                const SsspAux& ax, SsspState* __restrict__ st) {
   const unsigned t = st->iter;
-  if (st->stop || !st->do_merge) return;
+  if ((st->stop && st->stop != 4) || !st->do_merge) return;   // 4: a blocked dense iteration in progress
   uint32_t* bm_next = ax.bm[(t + 1) % 3];
   const unsigned lane = lane_id();
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -1850,7 +1850,9 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
   // (profiles/r2/sssp_dense_sweep.txt)
   double dense_frac = 0.45;
   if (const char* e = getenv("GX_SSSP_DENSE")) dense_frac = atof(e);
-  const bool dense_ok = mapping == GX_MAP_LB && dense_frac > 0.0 && !(d.n_tiles && g->knobs.smem) && !d.n_groups &&
+  // (with §3 tiles the dense iteration skips the local pass, schedule-only by
+  // E1; with replica groups it merges after the gather, every iteration only)
+  const bool dense_ok = mapping == GX_MAP_LB && dense_frac > 0.0 && (!d.n_groups || o.merge_every == 1) &&
                         !want_lh && d.max_w <= 255 && d.m_slots > 0 && !getenv("GX_SSSP_BLOCK") &&
                         !(o.profile && getenv("GX_SSSP_TRACE"));
   SsspPb spb{};
@@ -2081,6 +2083,10 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
         cudaEventDestroy(d1);
         cudaEventDestroy(d2);
       }
+      if (d.n_groups)   // §2.4 confluence of the dense iteration (stop == 4 is still running)
+        k_sssp_merge<<<grid_merge, 256, 0, s>>>(d.gptr.as<int32_t>(), d.gslots.as<int32_t>(), d.g_in_ptr.as<int32_t>(),
+                                                d.g_in.as<uint2>(), d.n_groups, merge_min ? 1 : 0,
+                                                r.dist.as<uint32_t>(), ax, st);
       k_sssp_dense_decide<<<1, 1, 0, s>>>(st, d.m_slots, L.early, o.max_iters);
       CUDA_OK(cudaGetLastError());
       launches += 3;

@@ -43,10 +43,13 @@ def knobs_c(kn, merge_op=0):
 
 @pytest.mark.parametrize("gname", list(GRAPHS))
 @pytest.mark.parametrize("kname", list(KNOBS))
-@pytest.mark.parametrize("mapping", ["auto", "lb", "tpv", "vns", "lb_unpacked"])
+@pytest.mark.parametrize("mapping", ["auto", "lb", "tpv", "vns", "lb_unpacked", "lb_dense"])
 def test_sssp_transformed_bit_exact(gname, kname, mapping, monkeypatch):
     if mapping == "lb_unpacked":   # the {dst, w} stream C5 takes (26 id + 7 weight bits > 32)
         monkeypatch.setenv("GX_SSSP_NO_PACK", "1")
+        mapping = "lb"
+    if mapping == "lb_dense":      # every refill as the blocked dense relaxation (+ merge, no local pass)
+        monkeypatch.setenv("GX_SSSP_DENSE", "1e-9")
         mapping = "lb"
     raw = GRAPHS[gname]()
     g = from_raw(raw)
