@@ -220,7 +220,7 @@ __global__ void k_pb_pairs(const uint32_t* __restrict__ rp, const uint32_t* __re
   }
 }
 // the same with the edge's 8-bit weight in the payload's high word (weights
-// resident and <= 255): the sort then also yields the weights in blocked order
+// resident and < 2^16): the sort then also yields the weights in blocked order
 __global__ void k_pb_pairs_w(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj, int64_t n, uint32_t nb,
                              uint32_t* __restrict__ key, unsigned long long* __restrict__ val,
                              uint32_t* __restrict__ cnt) {
@@ -250,7 +250,7 @@ __global__ void k_pb_padcnt(const uint32_t* __restrict__ cnt, uint32_t* __restri
 template <class V>
 __global__ void k_pb_place(const uint32_t* __restrict__ key, const V* __restrict__ pay,
                            const uint32_t* __restrict__ P, const uint32_t* __restrict__ P2, uint16_t* __restrict__ sl,
-                           uint16_t* __restrict__ dl, uint8_t* __restrict__ w8, int64_t m) {
+                           uint16_t* __restrict__ dl, uint16_t* __restrict__ w16, int64_t m) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
     const uint32_t k = key[i];
     const V p = pay[i];
@@ -258,7 +258,7 @@ __global__ void k_pb_place(const uint32_t* __restrict__ key, const V* __restrict
     sl[pos] = (uint16_t)(p & 0xffffu);
     dl[pos] = (uint16_t)((p >> 16) & 0xffffu);
     if constexpr (sizeof(V) == 8) {
-      if (w8) w8[pos] = (uint8_t)(p >> 32);
+      if (w16) w16[pos] = (uint16_t)(p >> 32);
     }
   }
 }
@@ -293,7 +293,7 @@ void ensure_pb(gx_graph* g) {
   // relaxation reads them in blocked order); an asynchronous upload's
   // blocked PageRank builds from col alone, and SSSP then runs without the
   // dense pass on this graph (it never gathers the weights at random)
-  const bool with_w = d.max_w <= 255 && !g->maxw_pending && m > 0;
+  const bool with_w = d.max_w <= 0xffffu && !g->maxw_pending && m > 0;
   DBuf k0, k1, v0, v1, tmp;
   cub::DoubleBuffer<uint32_t> dk, dv;
   cub::DoubleBuffer<unsigned long long> dv64;
@@ -347,8 +347,8 @@ void ensure_pb(gx_graph* g) {
   L.dst_loc.alloc(c, sizeof(uint16_t) * mm);
   L.val.alloc(c, sizeof(float) * mm);
   if (with_w) {
-    d.pb_w8.alloc(c, (size_t)mm);
-    CUDA_OK(cudaMemsetAsync(d.pb_w8.p, 0, (size_t)mm, s));
+    d.pb_w16.alloc(c, sizeof(uint16_t) * mm);
+    CUDA_OK(cudaMemsetAsync(d.pb_w16.p, 0, sizeof(uint16_t) * mm, s));
   }
   // padding entries: source index PB_R (a zero term in shared memory), sink 0
   launch_fill_u32(c, L.src_loc.as<uint32_t>(), (uint32_t)PB_R * 0x10001u, mm / 2);   // mm is a multiple of 8
@@ -359,7 +359,7 @@ void ensure_pb(gx_graph* g) {
     if (with_w)
       k_pb_place<unsigned long long><<<grid_for(c, m), 256, 0, s>>>(dk.Current(), dv64.Current(), P.as<uint32_t>(),
                                                                     P2.as<uint32_t>(), L.src_loc.as<uint16_t>(),
-                                                                    L.dst_loc.as<uint16_t>(), d.pb_w8.as<uint8_t>(), m);
+                                                                    L.dst_loc.as<uint16_t>(), d.pb_w16.as<uint16_t>(), m);
     else
       k_pb_place<uint32_t><<<grid_for(c, m), 256, 0, s>>>(dk.Current(), dv.Current(), P.as<uint32_t>(),
                                                           P2.as<uint32_t>(), L.src_loc.as<uint16_t>(),
@@ -372,10 +372,10 @@ void ensure_pb(gx_graph* g) {
 }
 
 // ---- the edge weights in the blocked order (SSSP's dense relaxation, sssp.cu) ----
-// true when the blocked layout carries them (built with resident weights <= 255)
+// true when the blocked layout carries them (built with resident weights < 2^16)
 bool ensure_pb_w(gx_graph* g) {
   ensure_pb(g);
-  return g->dg.pb_w8.p != nullptr;
+  return g->dg.pb_w16.p != nullptr;
 }
 
 // join the GX_ASYNC_UPLOAD work into the ctx stream; read the weights' maximum

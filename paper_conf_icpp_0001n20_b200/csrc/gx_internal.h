@@ -173,8 +173,8 @@ struct DevGraph {
   // push over out-edges
   SellLayout pr_sell, sssp_sell;
   PbLayout pr_pb;              // propagation-blocked PR (built on first use)
-  DBuf pb_w8;                  // u8 [m_pad]: edge weights in the blocked order (SSSP dense relaxation), built
-                               // with the layout when the weights are resident and <= 255
+  DBuf pb_w16;                 // u16 [m_pad]: edge weights in the blocked order (SSSP dense relaxation), built
+                               // with the layout when the weights are resident and < 2^16
   RankLayouts rk_sssp, rk_pr;  // partitioned path (dist.h): this rank's rows only
   // LB SSSP: static chunk list of rows with out-degree > HEAVY_DEG, heavy bitmap
   int64_t nhc = 0;
@@ -268,7 +268,7 @@ void resolve_pending(gx_graph* g);
 void join_download(gx_graph* g, int kind);   // kind < 0: every kind
 void build_device_slots(gx_graph* g);
 void ensure_pb(gx_graph* g);
-bool ensure_pb_w(gx_graph* g);   // the blocked layout + its 8-bit weights (false: built without them)
+bool ensure_pb_w(gx_graph* g);   // the blocked layout + its 16-bit weights (false: built without them)
 void build_tpv(gx_graph* g);
 void run_sssp(gx_graph* g, const gx_run_opts& o, gx_run_info& info);
 void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info);

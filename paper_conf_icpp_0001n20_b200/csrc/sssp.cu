@@ -1022,7 +1022,7 @@ struct SsspPb {
   const uint32_t* q;
   const uint16_t* src_loc;
   const uint16_t* dst_loc;
-  const uint8_t* w8;
+  const uint16_t* w16;
   uint32_t* val;
   int64_t nb;
 };
@@ -1053,14 +1053,15 @@ __global__ void __launch_bounds__(SPB_THREADS, 1) k_sssp_pb_scatter(SsspPb p, co
     // 8 entries per lane per step (16 B of source indices, 8 B of weights);
     // SPB_SEGU segments' first steps are loaded together (memory-level
     // parallelism), then each segment's remaining steps
-    auto put8 = [&](uint32_t e, uint4 sx, uint2 wx) {
+    auto put8 = [&](uint32_t e, uint4 sx, uint4 wx) {
       const uint32_t sr[8] = {sx.x & 0xffffu, sx.x >> 16, sx.y & 0xffffu, sx.y >> 16,
                               sx.z & 0xffffu, sx.z >> 16, sx.w & 0xffffu, sx.w >> 16};
       uint32_t c[8];
 #pragma unroll
       for (int i = 0; i < 8; i++) {
         const uint32_t du = s_d[sr[i]];
-        const uint32_t w = ((i < 4 ? wx.x : wx.y) >> (8 * (i & 3))) & 0xffu;
+        const uint32_t ww = i < 2 ? wx.x : i < 4 ? wx.y : i < 6 ? wx.z : wx.w;
+        const uint32_t w = (ww >> (16 * (i & 1))) & 0xffffu;
         c[i] = du == INF ? INF : sat_add(du, w);
       }
       __stcg(reinterpret_cast<uint4*>(p.val + e), make_uint4(c[0], c[1], c[2], c[3]));
@@ -1074,14 +1075,14 @@ __global__ void __launch_bounds__(SPB_THREADS, 1) k_sssp_pb_scatter(SsspPb p, co
       for (int k = 0; k < kn; k += SPB_SEGU) {
         uint32_t ee[SPB_SEGU], hh[SPB_SEGU];
         uint4 sx[SPB_SEGU];
-        uint2 wx[SPB_SEGU];
+        uint4 wx[SPB_SEGU];
 #pragma unroll
         for (int u = 0; u < SPB_SEGU; u++) {
           ee[u] = __shfl_sync(FULL, lo, (k + u) & 31) + 8u * lane;
           hh[u] = k + u < kn ? __shfl_sync(FULL, hi, (k + u) & 31) : 0u;
           if (ee[u] < hh[u]) {
             sx[u] = ld_stream_v4(reinterpret_cast<const uint32_t*>(p.src_loc + ee[u]), pf);
-            wx[u] = *reinterpret_cast<const uint2*>(p.w8 + ee[u]);
+            wx[u] = ld_stream_v4(reinterpret_cast<const uint32_t*>(p.w16 + ee[u]), pf);
           }
         }
 #pragma unroll
@@ -1089,7 +1090,7 @@ __global__ void __launch_bounds__(SPB_THREADS, 1) k_sssp_pb_scatter(SsspPb p, co
           if (ee[u] < hh[u]) put8(ee[u], sx[u], wx[u]);
           for (uint32_t e = ee[u] + 256u; e < hh[u]; e += 256u)
             put8(e, ld_stream_v4(reinterpret_cast<const uint32_t*>(p.src_loc + e), pf),
-                 *reinterpret_cast<const uint2*>(p.w8 + e));
+                 ld_stream_v4(reinterpret_cast<const uint32_t*>(p.w16 + e), pf));
         }
       }
     }
@@ -1853,7 +1854,7 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
   // (with §3 tiles the dense iteration skips the local pass, schedule-only by
   // E1; with replica groups it merges after the gather, every iteration only)
   const bool dense_ok = mapping == GX_MAP_LB && dense_frac > 0.0 && (!d.n_groups || o.merge_every == 1) &&
-                        !want_lh && d.max_w <= 255 && d.m_slots > 0 && !getenv("GX_SSSP_BLOCK") &&
+                        !want_lh && d.max_w <= 0xffffu && d.m_slots > 0 && !getenv("GX_SSSP_BLOCK") &&
                         !(o.profile && getenv("GX_SSSP_TRACE"));
   SsspPb spb{};
   bool dense_on = dense_ok;
@@ -1862,7 +1863,7 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
     spb.q = d.pr_pb.q.as<uint32_t>();
     spb.src_loc = d.pr_pb.src_loc.as<uint16_t>();
     spb.dst_loc = d.pr_pb.dst_loc.as<uint16_t>();
-    spb.w8 = d.pb_w8.as<uint8_t>();
+    spb.w16 = d.pb_w16.as<uint16_t>();
     spb.val = d.pr_pb.val.as<uint32_t>();
     spb.nb = d.pr_pb.nb;
     CUDA_OK(cudaFuncSetAttribute(k_sssp_pb_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (PB_R + 8) * 4));
