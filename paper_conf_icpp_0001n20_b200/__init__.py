@@ -58,6 +58,42 @@ class Knobs:
         return k
 
 
+def hosted_collective(rank: int, group=None):
+    """The gx_coll_fn of a hosted context (include/graffix.h): a Python callable
+    (kind, host_ptr, count, dtype, op, offsets, world, user) -> 0 / 1 that runs
+    the collective with torch.distributed on the host buffer, in place.  The
+    allgather-v and reduce-scatter-v travel as an allreduce: sum over a buffer
+    holding only this rank's slice (exact: one non-zero term per element), min
+    over the whole buffer (a superset of the reduce-scatter).  u32 travels as
+    int64 (gloo has no unsigned reductions).  Needs no GPU (the library stages
+    device data through pinned host memory before calling it)."""
+    import torch
+    import torch.distributed as dist
+    np_dt = {GX_DT_U32: np.uint32, GX_DT_F32: np.float32, GX_DT_F64: np.float64}
+
+    def _coll(kind, buf, count, dtype, op, offsets, nw, user):
+        try:
+            if count == 0:
+                return 0
+            a = np.ctypeslib.as_array((C.c_char * (count * np.dtype(np_dt[dtype]).itemsize)).from_address(buf))
+            a = a.view(np_dt[dtype])
+            t = torch.from_numpy(a.astype(np.int64) if dtype == GX_DT_U32 else a.copy())
+            rop = dist.ReduceOp.MIN if op == GX_OP_MIN else dist.ReduceOp.SUM
+            if kind == GX_COLL_ALLGATHERV:
+                lo, hi = offsets[rank], offsets[rank + 1]
+                t[:lo] = 0
+                t[hi:] = 0
+                rop = dist.ReduceOp.SUM
+            dist.all_reduce(t, op=rop, group=group)
+            a[:] = t.numpy().astype(np_dt[dtype])
+            return 0
+        except Exception as e:   # reported as GX_E_NCCL by the library
+            import sys
+            print(f"graffix hosted exchange failed: {e!r}", file=sys.stderr)
+            return 1
+    return _coll
+
+
 class Context:
     """A CUDA device + stream (+ optional NCCL communicator)."""
 
@@ -110,33 +146,7 @@ class Context:
         sweep, layout and reduction decision stays in libgraffix).  The
         allgather-v and reduce-scatter-v are carried as an allreduce: sum over
         a buffer holding only this rank's slice, min over the whole buffer."""
-        import torch
-        import torch.distributed as dist
-        np_dt = {GX_DT_U32: np.uint32, GX_DT_F32: np.float32, GX_DT_F64: np.float64}
-        th_dt = {GX_DT_U32: torch.int64, GX_DT_F32: torch.float32, GX_DT_F64: torch.float64}
-
-        def _coll(kind, buf, count, dtype, op, offsets, nw, user):
-            try:
-                if count == 0:
-                    return 0
-                a = np.ctypeslib.as_array((C.c_char * (count * np.dtype(np_dt[dtype]).itemsize)).from_address(buf))
-                a = a.view(np_dt[dtype])
-                # gloo has no uint32 reductions: carry u32 as int64 (exact)
-                t = torch.from_numpy(a.astype(np.int64) if dtype == GX_DT_U32 else a.copy())
-                rop = dist.ReduceOp.MIN if op == GX_OP_MIN else dist.ReduceOp.SUM
-                if kind == GX_COLL_ALLGATHERV:
-                    lo, hi = offsets[rank], offsets[rank + 1]
-                    t[:lo] = 0
-                    t[hi:] = 0
-                    rop = dist.ReduceOp.SUM          # exact: every slot has one non-zero term
-                dist.all_reduce(t, op=rop, group=group)
-                a[:] = t.numpy().astype(np_dt[dtype])
-                return 0
-            except Exception as e:   # reported as GX_E_NCCL by the library
-                import sys
-                print(f"graffix hosted exchange failed: {e!r}", file=sys.stderr)
-                return 1
-
+        _coll = hosted_collective(rank, group)
         cb = COLL_FN(_coll)
         h = C.c_void_p()
         _check(lib().gx_ctx_create_hosted(C.byref(h), device, C.c_void_p(stream) if stream else None, rank, world,

@@ -12,6 +12,7 @@
 namespace gx {
 
 static thread_local std::string g_last_error;
+void set_last_error(const std::string& m) { g_last_error = m; }   // for entry points outside this file (comm.cpp)
 
 void* Ctx::dmalloc(size_t b) {
   if (b == 0) b = 16;

@@ -10,6 +10,7 @@
 #include "gx_internal.h"
 
 namespace gx {
+void set_last_error(const std::string& m);   // capi.cpp
 namespace nccl {
 typedef struct { char internal[128]; } UniqueId;
 typedef void* Comm;
@@ -133,6 +134,7 @@ gx_status gx_get_nccl_unique_id(uint8_t out[128]) {
     std::memcpy(out, id.internal, 128);
     return GX_OK;
   } catch (const gx::Error& e) {
+    gx::set_last_error(e.what());
     return e.st;
   }
 }
@@ -166,6 +168,7 @@ gx_status gx_ctx_create_dist(gx_ctx** out, int device, void* cuda_stream, int ra
     (*out)->world = world;
     return GX_OK;
   } catch (const gx::Error& e) {
+    gx::set_last_error(e.what());
     gx_ctx_destroy(*out);
     *out = nullptr;
     return e.st;

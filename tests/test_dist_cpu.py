@@ -147,3 +147,57 @@ def test_gloo_world2_exchange_protocol(gx, worker):
         assert out[0] and out[1]
     else:
         assert out[0] < 1e-9 and out[1] < 1e-9
+
+
+def _coll_worker(rank, world, port, out):
+    """One rank driving the hosted-exchange transport (the library's gx_coll_fn
+    implementation in the binding) on host buffers, as libgraffix calls it."""
+    import ctypes as C
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_icpp_0001n20_b200 import hosted_collective
+    from paper_conf_icpp_0001n20_b200._binding import (GX_COLL_ALLGATHERV, GX_COLL_ALLREDUCE, GX_COLL_REDUCE_SCATTERV,
+                                                       GX_DT_F32, GX_DT_F64, GX_DT_U32, GX_OP_MIN, GX_OP_SUM)
+    f = hosted_collective(rank)
+    offs = np.array([0, 5, 11], dtype=np.int64)             # unequal slices, as edge-balanced bounds are
+    offp = offs.ctypes.data_as(C.POINTER(C.c_int64))
+    res = {}
+    # allreduce(min) of u32 distances, INF included
+    d = np.array([7, 0xFFFFFFFF, 3 + rank, 0xFFFFFFFE, 9 * rank, 1, 2, 3, 4, 5, 6], dtype=np.uint32)
+    assert f(GX_COLL_ALLREDUCE, d.ctypes.data, d.size, GX_DT_U32, GX_OP_MIN, None, world, None) == 0
+    res["min_u32"] = d.copy()
+    # fused scalar allreduce(sum) of f64
+    x = np.array([0.25 * (rank + 1), 1e-17, -3.0], dtype=np.float64)
+    assert f(GX_COLL_ALLREDUCE, x.ctypes.data, x.size, GX_DT_F64, GX_OP_SUM, None, world, None) == 0
+    res["sum_f64"] = x.copy()
+    # allgather-v of f32 slices: rank r owns [offs[r], offs[r+1]); other slices hold stale values
+    c = np.full(11, 99.0, dtype=np.float32)
+    c[offs[rank]:offs[rank + 1]] = np.arange(offs[rank], offs[rank + 1], dtype=np.float32) + 0.5
+    assert f(GX_COLL_ALLGATHERV, c.ctypes.data, c.size, GX_DT_F32, GX_OP_SUM, offp, world, None) == 0
+    res["gather_f32"] = c.copy()
+    # reduce-scatter-v(min) of u32: this rank's slice must hold the min over ranks
+    r = np.arange(11, dtype=np.uint32) * (rank + 1) + (10 if rank == 0 else 0)
+    assert f(GX_COLL_REDUCE_SCATTERV, r.ctypes.data, r.size, GX_DT_U32, GX_OP_MIN, offp, world, None) == 0
+    res["rs_u32"] = r.copy()
+    np.savez(os.path.join(out, f"coll{rank}.npz"), **res)
+    dist.destroy_process_group()
+
+
+def test_hosted_exchange_transport_world2(tmp_path):
+    """The hosted exchange's transport (include/graffix.h gx_coll_fn, binding
+    `hosted_collective`) between two gloo processes on CPU: allreduce min/sum,
+    allgather-v with unequal slices, reduce-scatter-v -- the collectives the
+    partitioned path issues; the GPU side is tested with two
+    processes on one B200 (tests/test_gpu_dist_procs.py)."""
+    world = 2
+    mp.start_processes(_coll_worker, args=(world, _free_port(), str(tmp_path)), nprocs=world, join=True,
+                       start_method="spawn")
+    offs = [0, 5, 11]
+    for rank in range(world):
+        z = np.load(tmp_path / f"coll{rank}.npz")
+        assert list(z["min_u32"]) == [7, 0xFFFFFFFF, 3, 0xFFFFFFFE, 0, 1, 2, 3, 4, 5, 6]
+        assert np.array_equal(z["sum_f64"], np.array([0.75, 2e-17, -6.0]))
+        assert np.array_equal(z["gather_f32"], np.arange(11, dtype=np.float32) + 0.5)
+        want = np.minimum(np.arange(11) * 1 + 10, np.arange(11) * 2)
+        lo, hi = offs[rank], offs[rank + 1]
+        assert np.array_equal(z["rs_u32"][lo:hi], want[lo:hi].astype(np.uint32))
