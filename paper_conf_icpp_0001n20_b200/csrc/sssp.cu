@@ -659,7 +659,7 @@ __device__ __forceinline__ void sssp_split_dev(const uint32_t* __restrict__ dist
                                                const uint32_t* __restrict__ rp = nullptr) {
   uint32_t* bm_cur = ax.bm[t % 3];
   uint32_t my_min = INF;
-  unsigned long long my_deg = 0;   // rp != null: count the moved slots (dense-iteration test)
+  unsigned long long my_deg = 0;   // the moved slots (dense-iteration test, adaptive window)
   const int64_t w_lo = lo >> 5, w_hi = min((hi + 31) >> 5, ax.nwords);
   for (int64_t w = w_lo + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < w_hi; w += (int64_t)gridDim.x * blockDim.x) {
     uint32_t bits = ax.far[w];
@@ -680,10 +680,9 @@ __device__ __forceinline__ void sssp_split_dev(const uint32_t* __restrict__ dist
     if (move) bm_cur[w] |= move;
     my_deg += __popc(move);
   }
-  if (rp) {
-    my_deg = warp_sum_u64(my_deg);
-    if (lane_id() == 0 && my_deg) atomicAdd(&st->refill_deg[t % 3], my_deg);
-  }
+  (void)rp;
+  my_deg = warp_sum_u64(my_deg);
+  if (lane_id() == 0 && my_deg) atomicAdd(&st->refill_deg[t % 3], my_deg);
   flush_counters(st, 0, 0, 0, 0, my_min, fdst);
 }
 __global__ void k_sssp_split(const uint32_t* __restrict__ dist, SsspAux ax, SsspState* __restrict__ st, int64_t lo,
@@ -840,6 +839,8 @@ struct SsspLoop {
   int64_t ngroups;
   int merge_min, cadence, max_iters;
   unsigned early;       // refill the next bucket once the near frontier's pushes are <= early (0: only when empty)
+  unsigned long long small_refill;   // a refill moving fewer slots doubles the next window (up to wmul_cap)
+  unsigned wmul_cap;
   int64_t block_rows;   // > 0: block-local mode with this many rows per CTA
   const int32_t* slot_tile;
   uint32_t* tmark;
@@ -872,11 +873,21 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
   unsigned t = st->iter;
   uint32_t tau = st->tau, rf = st->far_min;   // a relaunch after a dense iteration continues its state
   const uint32_t delta = st->delta;
+  // adaptive window: the tail buckets of a power-law graph hold few slots but
+  // each refill scans the whole far pile (~1M slots on RMAT-24) -- a refill
+  // that moves fewer than small_refill slots doubles the next window
+  uint32_t wmul = st->wmul ? st->wmul : 1u;
+  auto adapt = [&](unsigned tt) {
+    const unsigned long long moved = *(volatile unsigned long long*)&st->refill_deg[tt % 3];
+    wmul = moved < a.small_refill ? min(wmul * 2u, a.wmul_cap) : 1u;
+    if (lead) st->wmul = wmul;
+  };
   // the relaunch's pending near-far refill (decided after the dense iteration)
   if (*(volatile unsigned*)&st->split) {
     sssp_split_dev(a.dist, a.ax, st, 0, a.n_slots, t, tau, &st->far3[t % 3], a.dense_edges ? a.rp : nullptr);
     grid.sync();
     if (lead) st->split = 0;
+    adapt(t);
     if (a.dense_edges && *(volatile unsigned long long*)&st->refill_deg[t % 3] >= a.dense_edges) {
       if (lead) st->stop = 4;
       return;
@@ -946,7 +957,7 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
       // early): raise tau past the nearest far slot; the refill joins the tail
       // in the next frontier (any relaxation order reaches the same fixed
       // point, Theorem E1), instead of one ~10 us iteration per tail hop
-      const unsigned long long nt = (unsigned long long)fm + delta;
+      const unsigned long long nt = (unsigned long long)fm + (unsigned long long)delta * wmul;
       tau = nt >= INF ? INF : (unsigned)nt;
       rf = INF;
       split = true;
@@ -954,7 +965,7 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
       if (fm == INF) {
         stop = 1;
       } else {   // the bucket drained: raise tau past the nearest far slot
-        const unsigned long long nt = (unsigned long long)fm + delta;
+        const unsigned long long nt = (unsigned long long)fm + (unsigned long long)delta * wmul;
         tau = nt >= INF ? INF : (unsigned)nt;
         rf = INF;
         split = true;
@@ -988,6 +999,7 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
     if (split) {   // near-far refill of iteration t's frontier
       sssp_split_dev(a.dist, a.ax, st, 0, a.n_slots, t, tau, &st->far3[t % 3], a.dense_edges ? a.rp : nullptr);
       grid.sync();
+      adapt(t);
       // a refill that carries most of the graph's edges: hand iteration t to the
       // blocked dense relaxation (k_sssp_pb_*), which streams every edge once
       // instead of gathering dist at random for each of them
@@ -1182,7 +1194,7 @@ __global__ void k_sssp_dense_decide(SsspState* __restrict__ st, int64_t m_slots,
   uint32_t tau = st->tau, rf = fm;
   unsigned stop = 0, split = 0;
   if ((pushed <= early || pushed == 0) && fm != INF) {
-    const unsigned long long nt = (unsigned long long)fm + st->delta;
+    const unsigned long long nt = (unsigned long long)fm + (unsigned long long)st->delta * (st->wmul ? st->wmul : 1u);
     tau = nt >= INF ? INF : (unsigned)nt;
     rf = INF;
     split = 1;
@@ -2004,6 +2016,10 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
     // bucket before it settles (451M -> 841M relaxations)
     L.early = 256;
     if (const char* e = getenv("GX_SSSP_EARLY")) L.early = (unsigned)std::max(0, atoi(e));
+    // adaptive window (GX_SSSP_WMUL_CAP = 1 turns it off)
+    L.small_refill = (unsigned long long)std::max<int64_t>(1, ns / 256);
+    L.wmul_cap = 64;
+    if (const char* e = getenv("GX_SSSP_WMUL_CAP")) L.wmul_cap = (unsigned)std::max(1, atoi(e));
     // block-local mode when most edges stay inside the CTA id blocks and rows
     // are short (thread-per-slot relaxation); GX_SSSP_BLOCK=0/1 overrides
     const int64_t gridp = (int64_t)occp * c->num_sms;

@@ -30,6 +30,7 @@ struct SsspState {
   unsigned int tiles_n[3];      // §3 tiles touched in iteration t (list length), [t%3]
   unsigned long long refill_deg[3];  // out-edges of the slots a near-far refill moved into frontier t, [t%3]
   unsigned int dense_bin;       // blocked dense relaxation: next sink bin to claim
+  unsigned int wmul;            // near-far window = delta * wmul (doubles after small refills; 0 reads as 1)
 };
 
 struct SsspAux {

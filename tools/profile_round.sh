@@ -9,7 +9,9 @@ ncu --set full --clock-control none --import-source on -k regex:"k_pr_pb" -s 5 -
     python tools/prof_run.py --scale 24 --algos pagerank --mapping pb > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:"k_sssp_persist" -s 1 -c 1 -o gpurun_out/prof_ssspLB_$TAG \
     python tools/prof_run.py --scale 24 --algos sssp --reps 2 > /dev/null 2>&1
-for f in gpurun_out/prof_prpb_$TAG gpurun_out/prof_ssspLB_$TAG; do
+ncu --set full --clock-control none --import-source on -k regex:"k_sssp_pb_" -s 2 -c 2 -o gpurun_out/prof_ssspPB_$TAG \
+    python tools/prof_run.py --scale 24 --algos sssp --reps 2 > /dev/null 2>&1
+for f in gpurun_out/prof_prpb_$TAG gpurun_out/prof_ssspLB_$TAG gpurun_out/prof_ssspPB_$TAG; do
   ncu -i $f.ncu-rep --page details --csv > $f.details.csv 2>/dev/null
   ncu -i $f.ncu-rep --page raw --csv > $f.raw.csv 2>/dev/null
 done
