@@ -2016,9 +2016,14 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
     // bucket before it settles (451M -> 841M relaxations)
     L.early = 256;
     if (const char* e = getenv("GX_SSSP_EARLY")) L.early = (unsigned)std::max(0, atoi(e));
-    // adaptive window (GX_SSSP_WMUL_CAP = 1 turns it off)
+    // adaptive window (GX_SSSP_WMUL_CAP = 1 turns it off).  Measured
+    // (profiles/r2/sssp_wmul_sweep.txt): RMAT-24 4.66 -> 4.55 ms, uniform
+    // 16M/256M 4.69 -> 4.07 ms (cap 8 = cap 64); off for sparse high-diameter
+    // graphs (the avg-degree < 4 rule of sssp_delta), whose buckets are always
+    // small wavefronts: road 4900^2 151 -> 175-187 ms with it
     L.small_refill = (unsigned long long)std::max<int64_t>(1, ns / 256);
-    L.wmul_cap = 64;
+    const double avg_deg = (double)g->m / (double)std::max<int64_t>(1, g->n);
+    L.wmul_cap = avg_deg < 4.0 ? 1u : 8u;
     if (const char* e = getenv("GX_SSSP_WMUL_CAP")) L.wmul_cap = (unsigned)std::max(1, atoi(e));
     // block-local mode when most edges stay inside the CTA id blocks and rows
     // are short (thread-per-slot relaxation); GX_SSSP_BLOCK=0/1 overrides
