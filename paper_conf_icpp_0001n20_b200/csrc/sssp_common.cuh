@@ -60,16 +60,31 @@ __device__ __forceinline__ uint32_t sat_add(uint32_t du, uint32_t w) {
   return (nd < du || nd == 0xFFFFFFFFu) ? 0xFFFFFFFEu : nd;
 }
 
-// the out-edge e as {dst, w}
+// the out-edge e as {dst, w}.  volatile: the LB sweep issues the next round's
+// edge loads before this round's dist gathers (software pipeline); without it
+// the compiler sinks these loads to their use and every round waits twice
+// (ncu source page, profiles/r2: the gather address waited on the edge load)
+#ifndef GX_SSSP_EDGE_VOLATILE
+#define GX_SSSP_EDGE_VOLATILE 1
+#endif
+#if GX_SSSP_EDGE_VOLATILE
+#define GX_EDGE_ASM asm volatile
+#else
+#define GX_EDGE_ASM asm
+#endif
+__device__ __forceinline__ uint32_t ld_edge_raw(const uint32_t* p, uint64_t pol) {
+  uint32_t v;
+  GX_EDGE_ASM("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+  return v;
+}
 __device__ __forceinline__ uint2 ld_edge(const uint2* __restrict__ adj, const SsspAux& ax, uint32_t e, uint64_t pol) {
   if (ax.adjp) {
-    uint32_t v;
-    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(ax.adjp + e), "l"(pol));
+    const uint32_t v = ld_edge_raw(ax.adjp + e, pol);
     return make_uint2(v >> ax.wbits, v & ((1u << ax.wbits) - 1u));
   }
   uint2 v;
-  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0, %1}, [%2], %3;" : "=r"(v.x), "=r"(v.y) : "l"(adj + e),
-      "l"(pol));
+  GX_EDGE_ASM("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0, %1}, [%2], %3;" : "=r"(v.x), "=r"(v.y)
+              : "l"(adj + e), "l"(pol));
   return v;
 }
 
