@@ -1022,14 +1022,25 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
 //   (A) k_sssp_pb_scatter: per source block, the frontier slots' distances in
 //       shared memory; every edge's candidate dist[u] + w (INF for a source
 //       outside the frontier) streamed to val[] (2 + 1 bytes read, 4 written)
-//   (B) k_sssp_pb_gather: per sink bin, the bin's candidates streamed (4 + 2
-//       bytes) into a shared-memory atomicMin per row (ATOMS.MIN), then the
-//       rows that improved update dist and join the next frontier / far pile
-//       with word-level ballots (a bin's rows are whole bitmap words)
+//   (B) k_sssp_pb_gather: per sink bin, the rows' distances in shared memory,
+//       the bin's candidates streamed (4 + 2 bytes) and tested against them;
+//       an improving one issues a shared atomicMin (ATOMS.MIN); then the rows
+//       that improved update dist and join the next frontier / far pile with
+//       word-level ballots (a bin's rows are whole bitmap words)
 // val[] is the PageRank layout's term array (reinterpreted as u32; PageRank
 // rewrites it at the start of each run).  Same fixed point (any relaxation
 // order, Theorem E1): the iteration relaxes every frontier edge exactly once.
 constexpr int SPB_THREADS = 1024;
+#ifndef GX_SPB_GDEPTH
+#define GX_SPB_GDEPTH 4
+#endif
+#ifndef GX_SPB_SEGU
+#define GX_SPB_SEGU 4
+#endif
+#ifndef GX_SPB_TEST
+#define GX_SPB_TEST 1   // gather: test a candidate against the row before the atomic
+#endif
+constexpr int SPB_GDEPTH = GX_SPB_GDEPTH;   // gather: steps of 4 candidates per thread in flight
 struct SsspPb {
   const uint32_t* q;
   const uint16_t* src_loc;
@@ -1079,7 +1090,7 @@ __global__ void __launch_bounds__(SPB_THREADS, 1) k_sssp_pb_scatter(SsspPb p, co
       __stcg(reinterpret_cast<uint4*>(p.val + e), make_uint4(c[0], c[1], c[2], c[3]));
       __stcg(reinterpret_cast<uint4*>(p.val + e) + 1, make_uint4(c[4], c[5], c[6], c[7]));
     };
-    constexpr int SPB_SEGU = 4;
+    constexpr int SPB_SEGU = GX_SPB_SEGU;   // scatter: segments' first steps in flight per warp
     for (int64_t j0 = (int64_t)warp * 32; j0 < nb; j0 += 32 * NW) {
       const int64_t j = j0 + lane;
       const uint32_t lo = j < nb ? __ldg(r0 + j) : 0u, hi = j < nb ? __ldg(r1 + j) : 0u;
@@ -1129,29 +1140,42 @@ __global__ void __launch_bounds__(SPB_THREADS, 1) k_sssp_pb_gather(SsspPb p, uin
   uint32_t my_push = 0, my_min = INF;
   for (;;) {
     if (threadIdx.x == 0) s_bin = (int)atomicAdd(&st->dense_bin, 1u);
-    for (int i = threadIdx.x; i < PB_R / 4; i += SPB_THREADS)
-      reinterpret_cast<uint4*>(acc)[i] = make_uint4(INF, INF, INF, INF);
     __syncthreads();
     const int64_t b = s_bin;
     if (b >= nb) break;
+    // the accumulator starts at the rows' current distances: a candidate is
+    // tested against it first and only an improvement issues the atomic (most
+    // candidates of a refill land on rows already closer, RMAT's hubs above all)
+    {
+      const int64_t base0 = b * PB_R;
+      for (int i = threadIdx.x; i < PB_R; i += SPB_THREADS)
+        acc[i] = base0 + i < n_slots ? __ldcg(dist + base0 + i) : INF;
+    }
+    __syncthreads();
     const uint32_t E0 = __ldg(p.q + b), E1 = __ldg(qend + b);   // multiples of 8
-    // the bin's candidates: 4 per thread per step, two steps in flight
-    for (uint32_t e = E0 + 4u * threadIdx.x; e < E1; e += 8u * SPB_THREADS) {
-      const uint32_t e2 = e + 4u * SPB_THREADS;
-      const uint4 v0 = ld_stream_v4(p.val + e, pf);
-      const uint2 d0 = *reinterpret_cast<const uint2*>(p.dst_loc + e);
-      uint4 v1 = make_uint4(INF, INF, INF, INF);
-      uint2 d1 = make_uint2(0, 0);
-      if (e2 < E1) {
-        v1 = ld_stream_v4(p.val + e2, pf);
-        d1 = *reinterpret_cast<const uint2*>(p.dst_loc + e2);
-      }
-      const uint32_t vv[8] = {v0.x, v0.y, v0.z, v0.w, v1.x, v1.y, v1.z, v1.w};
-      const uint32_t dd[8] = {d0.x & 0xffffu, d0.x >> 16, d0.y & 0xffffu, d0.y >> 16,
-                              d1.x & 0xffffu, d1.x >> 16, d1.y & 0xffffu, d1.y >> 16};
+    // the bin's candidates: 4 per thread per step, SPB_GDEPTH steps in flight;
+    // a candidate is tested against the row's current value first
+    for (uint32_t e = E0 + 4u * threadIdx.x; e < E1; e += (uint32_t)SPB_GDEPTH * 4u * SPB_THREADS) {
+      uint4 v[SPB_GDEPTH];
+      uint2 dd[SPB_GDEPTH];
 #pragma unroll
-      for (int i = 0; i < 8; i++)
-        if (vv[i] != INF) atomicMin(&acc[dd[i]], vv[i]);
+      for (int q = 0; q < SPB_GDEPTH; q++) {
+        const uint32_t eq = e + (uint32_t)q * 4u * SPB_THREADS;
+        v[q] = make_uint4(INF, INF, INF, INF);
+        dd[q] = make_uint2(0, 0);
+        if (eq < E1) {
+          v[q] = ld_stream_v4(p.val + eq, pf);
+          dd[q] = *reinterpret_cast<const uint2*>(p.dst_loc + eq);
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < SPB_GDEPTH; q++) {
+        const uint32_t vv[4] = {v[q].x, v[q].y, v[q].z, v[q].w};
+        const uint32_t di[4] = {dd[q].x & 0xffffu, dd[q].x >> 16, dd[q].y & 0xffffu, dd[q].y >> 16};
+#pragma unroll
+        for (int i = 0; i < 4; i++)
+          if (GX_SPB_TEST ? vv[i] < acc[di[i]] : vv[i] != INF) atomicMin(&acc[di[i]], vv[i]);
+      }
     }
     __syncthreads();
     // the bin's rows: warp per 32 rows = one bitmap word

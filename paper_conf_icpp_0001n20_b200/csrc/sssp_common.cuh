@@ -60,12 +60,13 @@ __device__ __forceinline__ uint32_t sat_add(uint32_t du, uint32_t w) {
   return (nd < du || nd == 0xFFFFFFFFu) ? 0xFFFFFFFEu : nd;
 }
 
-// the out-edge e as {dst, w}.  volatile: the LB sweep issues the next round's
-// edge loads before this round's dist gathers (software pipeline); without it
-// the compiler sinks these loads to their use and every round waits twice
-// (ncu source page, profiles/r2: the gather address waited on the edge load)
+// the out-edge e as {dst, w}.  GX_SSSP_EDGE_VOLATILE=1 pins the program order
+// (the LB sweep's next-round edge loads before this round's dist gathers); the
+// compiler otherwise sinks them to their use (ncu source page, profiles/r2),
+// but pinned they measured slower: RMAT-24 4.60 (free) vs 4.94-5.02 ms
+// (SU 2-4, profiles/r2/sssp_edge_volatile_variants.txt)
 #ifndef GX_SSSP_EDGE_VOLATILE
-#define GX_SSSP_EDGE_VOLATILE 1
+#define GX_SSSP_EDGE_VOLATILE 0
 #endif
 #if GX_SSSP_EDGE_VOLATILE
 #define GX_EDGE_ASM asm volatile

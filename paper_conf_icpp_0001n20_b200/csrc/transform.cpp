@@ -39,6 +39,16 @@ struct PhaseTimer {
   }
 };
 
+// Release a vector of per-vertex vectors in parallel: the transforms build
+// ~10^8 small rows at RMAT-26, whose serial destruction took seconds per
+// structure (profiles/r2/c5_full_all3_transform_trace.txt)
+template <class T>
+void par_free(std::vector<std::vector<T>>& v) {
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int64_t i = 0; i < (int64_t)v.size(); i++) std::vector<T>().swap(v[i]);
+  std::vector<std::vector<T>>().swap(v);
+}
+
 // Weight of an added edge standing for the 2-hop path with hop weights w1, w2
 // (gx_knobs.added_weight_rule): the sum (P@34493, R17) or one of
 // the "alternative" rules P@34692 allows.
@@ -234,7 +244,6 @@ void coalesce(const HostCSR& g, int k, int64_t theta_ppm, int wrule, Work& W, Ct
   W.slot_to_orig.assign(n_slots, -1);
   W.kind.assign(n_slots, HOLE);
   W.owner = nw;
-  W.rows.assign(n_slots, {});
   for (int64_t u = 0; u < n; u++) {
     W.slot_to_orig[nw[u]] = (int32_t)u;
     W.kind[nw[u]] = OWNER;
@@ -320,20 +329,22 @@ void coalesce(const HostCSR& g, int k, int64_t theta_ppm, int wrule, Work& W, Ct
       asg.push_back({std::get<1>(c), std::get<2>(c), h++});
     }
   }
-  // owner rows start as the renumbered rows
-  for (int64_t s = 0; s < n_slots; s++) W.rows[s] = radj[s];
+  // replica rows from the pre-move rows (R16: 2-hop paths use n's pre-move
+  // edges), then the owner rows take the renumbered rows by move -- no copy of
+  // the whole adjacency -- and lose the moved edges
   int64_t added = 0;
-  for (const Asg& a : asg) {
+  std::vector<std::vector<Edge>> rep_rows(asg.size());
+#pragma omp parallel for schedule(dynamic, 1) reduction(+ : added)
+  for (size_t ai = 0; ai < asg.size(); ai++) {
+    const Asg& a = asg[ai];
     const auto& orow = radj[a.s];
     std::vector<int32_t> nplus;
     nplus.reserve(orow.size());
     for (const Edge& e : orow) nplus.push_back(e.dst);
     std::sort(nplus.begin(), nplus.end());
-    std::vector<Edge> moved;
+    std::vector<Edge> row;
     for (const Edge& e : orow)
-      if (e.dst / k == a.C) moved.push_back(e);
-    auto& own = W.rows[a.s];
-    own.erase(std::remove_if(own.begin(), own.end(), [&](const Edge& e) { return e.dst / k == a.C; }), own.end());
+      if (e.dst / k == a.C) row.push_back(e);   // moved
     // 2-hop edges into chunk C with the minimum path weight (R16, R17)
     std::unordered_map<int32_t, uint32_t> best;
     for (const Edge& ev : orow)
@@ -345,13 +356,20 @@ void coalesce(const HostCSR& g, int k, int64_t theta_ppm, int wrule, Work& W, Ct
         auto it = best.find(q);
         if (it == best.end() || w < it->second) best[q] = w;
       }
-    std::vector<Edge> row = moved;
     for (auto& kv : best) row.push_back({kv.first, kv.second, ADD_COALESCE});
-    W.rows[a.hole] = std::move(row);
+    added += (int64_t)best.size();
+    rep_rows[ai] = std::move(row);
+  }
+  W.rows = std::move(radj);
+  for (size_t ai = 0; ai < asg.size(); ai++) {
+    const Asg& a = asg[ai];
+    auto& own = W.rows[a.s];
+    own.erase(std::remove_if(own.begin(), own.end(), [&](const Edge& e) { return e.dst / k == a.C; }), own.end());
+    W.rows[a.hole] = std::move(rep_rows[ai]);
     W.kind[a.hole] = REPLICA;
     W.slot_to_orig[a.hole] = W.slot_to_orig[a.s];
-    added += (int64_t)best.size();
   }
+  pt("replica rows");
   int64_t holes_left = 0;
   for (int64_t s = 0; s < n_slots; s++) holes_left += W.kind[s] == HOLE;
   W.n_repl = (int64_t)asg.size();
@@ -767,11 +785,15 @@ void degnorm(Work& W, int64_t th, int64_t f, bool combined, int wrule, std::vect
   pt("padding candidates");
   }
   added = 0;
+#pragma omp parallel for schedule(dynamic, 4096) reduction(+ : added)
   for (int64_t s = 0; s < ns; s++) {
     added += (int64_t)adds[s].size();
     for (auto& e : adds[s]) W.rows[s].push_back(e);
   }
+  par_free(adds);
+  par_free(lout);
   sched = order;
+  pt("padding applied + freed");
 }
 
 }  // namespace
@@ -804,6 +826,9 @@ void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out, Ctx* de
     phase("subgraphs");
     for (auto& e : sm.added)
       W.rows[W.owner[std::get<0>(e)]].push_back({W.owner[std::get<1>(e)], std::get<2>(e), ADD_SMEM});
+    par_free(L.out);
+    par_free(L.N);
+    phase("smem free");
   }
   std::vector<int32_t> sched;
   int64_t added_dn = 0;

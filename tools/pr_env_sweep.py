@@ -1,8 +1,9 @@
-"""PageRank over-relaxation experiment (GX_PR_OMEGA): sweeps to tol and the
-fixed-point residual ||x - F(x)||_1 of each result (bound r / (1 - d) on the
-distance to the PageRank vector; F = the PR map of PAPER.md P@36969, R35).
+"""PageRank for each value of one environment knob (GX_PB_SYM, ...): sweeps to
+tol, time, and the fixed-point residual ||x - F(x)||_1 of each result (bound
+r / (1 - d) on the distance to the PageRank vector; F = the PR map of
+PAPER.md P@36969, R35).  (Round 2 used it as pr_omega.py for GX_PR_OMEGA.)
 
-    python tools/pr_omega.py --scale 24 --omegas 1.0,1.1,1.2,1.3
+    python tools/pr_env_sweep.py --scale 24 --env GX_PB_SYM --values 0,1
 """
 import argparse
 import os
@@ -27,7 +28,8 @@ def residual(rp, col, x, d=0.85):
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--scale", type=int, default=24)
-ap.add_argument("--omegas", default="1.0,1.1,1.2,1.3,1.4")
+ap.add_argument("--env", default="GX_PB_SYM")
+ap.add_argument("--values", default="0,1")
 ap.add_argument("--mapping", default="pb")
 a = ap.parse_args()
 raw = graphgen.rmat(a.scale)
@@ -35,11 +37,11 @@ ctx = gx.Context(0)
 G = gx.Graph.upload(ctx, raw.row_ptr, raw.col, raw.w)
 ex = G.export()
 rp, col = ex["row_ptr"], ex["col"]
-for om in [float(v) for v in a.omegas.split(",")]:
-    os.environ["GX_PR_OMEGA"] = str(om)
+for om in a.values.split(","):
+    os.environ[a.env] = om
     runs = [G.run("pagerank", tol=1e-9, mapping=a.mapping) for _ in range(3)]
     r = min(runs, key=lambda q: q["loop_ms"])
     x = G.download("rank")
     res = residual(rp, col, x)
-    print(f"omega={om} sweeps={r['iterations']} loop_ms={r['loop_ms']:.2f} last_delta={r['last_delta']:.3e} "
+    print(f"{a.env}={om} sweeps={r['iterations']} loop_ms={r['loop_ms']:.2f} last_delta={r['last_delta']:.3e} "
           f"converged={r['converged']} residual={res:.3e} bound={res / 0.15:.3e} mass={x.sum():.12f}", flush=True)
