@@ -405,7 +405,6 @@ struct PbArgs {
   const uint16_t* dst_loc;
   float* val;
   int64_t nb;
-  int sym;        // odd sweeps walk the bins in descending order (GX_PB_SYM=1)
 };
 
 __device__ __forceinline__ float4 ld_cg_f4(const float* p) {
@@ -680,10 +679,8 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
       reinterpret_cast<uint4*>(acc_hi)[i] = make_uint4(0, 0, 0, 0);
     }
     __syncthreads();
-    if (s_bin >= nb) break;
-    // bin order: ascending, or (p.sym) descending on odd sweeps -- a symmetric
-    // Gauss-Seidel ordering of the asynchronous schedule (same fixed point, E3)
-    const int64_t b = (p.sym && (t & 1)) ? nb - 1 - s_bin : s_bin;
+    const int64_t b = s_bin;
+    if (b >= nb) break;
     const int64_t base = b * PB_R;
     const int nrows = (int)min((int64_t)PB_R, a.n_slots - base);
     const uint32_t* r0 = p.q + b * nb;   // block b's scatter segments: [r0[j], r1[j])
@@ -1511,7 +1508,6 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     pb.dst_loc = d.pr_pb.dst_loc.as<uint16_t>();
     pb.val = d.pr_pb.val.as<float>();
     pb.nb = d.pr_pb.nb;
-    pb.sym = getenv("GX_PB_SYM") ? atoi(getenv("GX_PB_SYM")) : 0;
     // the opt-in is per device (context): set it on every run (cheap), not
     // once per process -- a second GPU in the same process needs it too
     CUDA_OK(cudaFuncSetAttribute(k_pr_pb<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
