@@ -185,12 +185,60 @@ def cpu_cores_used() -> int:
     return 1   # the oracle is single-threaded Python/numpy (numpy bincount is serial)
 
 
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+class pinned_core:
+    """Run the oracle on one host core (os.sched_setaffinity, the taskset of
+    SURVEY §8(d)); the previous affinity is restored afterwards."""
+    def __enter__(self):
+        self.old = os.sched_getaffinity(0)
+        self.core = min(self.old)
+        os.sched_setaffinity(0, {self.core})
+        return self
+
+    def __exit__(self, *exc):
+        os.sched_setaffinity(0, self.old)
+
+
+def oracle_knob_points():
+    """The oracle on C1 (RMAT-14) per knob setting (the oracle per
+    (graph, knob) point in the same job): transform, Dijkstra and fp64 PageRank
+    on the transformed graph's G_L, seconds each (bounded: a few seconds)."""
+    import graphgen
+    from oracle import algos as A
+    from oracle import transform as T
+    from oracle.graph import from_raw, graph_to_edgelist, sssp_source
+    g = from_raw(graphgen.rmat(14))
+    pts = []
+    for name, kn in (("exact", None), ("coalesce k16 theta0.6", T.Knobs(coalesce=True)),
+                     ("degnorm theta0.3", T.Knobs(degree_norm=True, degsim_threshold=0.3))):
+        t0 = time.perf_counter()
+        el = T.transform(g, kn).logical() if kn else graph_to_edgelist(g)
+        t1 = time.perf_counter()
+        A.sssp_dijkstra(el, sssp_source(g))
+        t2 = time.perf_counter()
+        _, it = A.pagerank(el, tol=1e-9)
+        t3 = time.perf_counter()
+        pts.append({"config": f"C1 rmat14 {name}", "transform_s": t1 - t0, "sssp_s": t2 - t1, "pagerank_s": t3 - t2,
+                    "pagerank_iterations": it})
+    return pts
+
+
 def run_reference(args, rank, world):
     if rank != 0:
         return 0
-    for _ in range(args.warmup):
-        oracle_sample()
-    res = [oracle_sample() for _ in range(args.steps)]
+    with pinned_core() as pc:
+        for _ in range(args.warmup):
+            oracle_sample()
+        res = [oracle_sample() for _ in range(args.steps)]
     edges = sum(r["edges"] for r in res)
     sec = sum(r["sec"] for r in res)
     v = edges / sec / 1e9
@@ -202,7 +250,8 @@ def run_reference(args, rank, world):
             "data": "synthetic", "config": {"workload": WORKLOADS[args.workload]["desc"], "graph": f"rmat{WORKLOADS[args.workload]['scale']}",
                                             "sample": f"rmat{CPU_SAMPLE_SCALE}"},
             "cpu_baseline": {"value": v, "unit": UNIT, "cores": cpu_cores_used(), "kind": "oracle",
-                             "sample": sample},
+                             "sample": sample, "cpu_model": cpu_model(),
+                             "pinned": f"host core {pc.core} (os.sched_setaffinity)"},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line))
     return 0
@@ -411,11 +460,14 @@ def main():
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        r = oracle_sample()
+        with pinned_core() as pc:
+            r = oracle_sample()
+            knob_pts = oracle_knob_points()
         cpu = {"value": r["edges"] / r["sec"] / 1e9, "unit": UNIT, "cores": cpu_cores_used(), "kind": "oracle",
                "sample": f"oracle Dijkstra + fp64 PR (tol 1e-9, {r['pr_iters']} iters) on RMAT-{CPU_SAMPLE_SCALE} "
                          f"(n={r['n']}, m={r['m']}; same generator, 1/{1 << (24 - CPU_SAMPLE_SCALE)} of T24), "
-                         f"{r['sec']:.1f} s", "host_cores": os.cpu_count()}
+                         f"{r['sec']:.1f} s", "host_cores": os.cpu_count(), "cpu_model": cpu_model(),
+               "pinned": f"host core {pc.core} (os.sched_setaffinity)", "knob_points": knob_pts}
 
     knobs = None
     if rank == 0 and world == 1 and not args.no_knobs:
