@@ -45,7 +45,7 @@ def graph_for(cfg, small):
     if cfg == "c2":
         s = 20 if small else 22
         return graphgen.rmat(s), f"rmat{s}"
-    if cfg == "c3":
+    if cfg in ("c3", "c3cc", "c3conn"):
         side = 1024 if small else 4900
         return graphgen.road(side), f"road{side}"
     if cfg == "c4":
@@ -70,6 +70,11 @@ def points(cfg):
     if cfg == "c3":
         return [(f"smem t0.5 budget {b}%", K(smem=True, cc_threshold=0.5, added_edge_budget=-2 if b < 0 else 0))
                 for b in (0,)] + [(f"coalesce road t{t}", K(coalesce=True, replicate_threshold=t)) for t in (0.4, 0.6)]
+    if cfg == "c3cc":   # Fig 8 (P@52695-53380): the CC threshold at a 1% budget
+        return [(f"smem tcc{t} budget 1%", K(smem=True, cc_threshold=t)) for t in (0.3, 0.4, 0.5, 0.6, 0.7, 0.8, 0.9)]
+    if cfg == "c3conn":   # Fig 7's connectedness sweep on the road grid (replication only bites here)
+        return [(f"coalesce road t{t}", K(coalesce=True, replicate_threshold=t)) for t in (2.0, 0.9, 0.6, 0.4, 0.2)] + \
+               [(f"coalesce road t{t} aware-merge", K(coalesce=True, replicate_threshold=t, merge_op=1)) for t in (0.4,)]
     if cfg == "c4":
         return [(f"degnorm t{t}", K(degree_norm=True, degsim_threshold=t)) for t in (0.0, 0.1, 0.2, 0.3, 0.4, 0.5)]
     if cfg == "c5":
@@ -94,7 +99,8 @@ def c5_partitioned(G, tag, base):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--config", default="c1", choices=["c1", "c2", "c3", "c4", "c5"])
+    ap.add_argument("--config", default="c1", choices=["c1", "c2", "c3", "c3cc", "c3conn", "c4", "c5"])
+    ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--scale-down", action="store_true")
     ap.add_argument("--budgets", default="0,0.1,0.5,1,2,5")
     a = ap.parse_args()
@@ -135,7 +141,7 @@ def main():
                    subgraphs=info["n_subgraphs"])
         for algo in ("sssp", "pagerank"):
             for mp in (("tpv", "lb", "pb") if algo == "pagerank" else ("tpv", "lb")):
-                r = timed(G, algo, mp, **({"tol": 1e-9} if algo == "pagerank" else {}))
+                r = timed(G, algo, mp, reps=a.reps, **({"tol": 1e-9} if algo == "pagerank" else {}))
                 row[f"{algo}_{mp}_ms"] = r["loop_ms"]
                 row[f"{algo}_{mp}_speedup_same_mapping"] = ex[(algo, mp)]["loop_ms"] / r["loop_ms"]
                 row[f"{algo}_{mp}_speedup_vs_best_exact"] = best[algo] / r["loop_ms"]
