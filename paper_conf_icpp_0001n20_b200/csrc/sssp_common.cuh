@@ -28,9 +28,20 @@ struct SsspState {
   unsigned int final_merge;     // c = 0: this iteration's merge ends the run
   unsigned int far3[3];         // persistent loop: far-pile minimum pushed in iteration t, [t%3]
   unsigned int tiles_n[3];      // §3 tiles touched in iteration t (list length), [t%3]
-  unsigned long long refill_deg[3];  // out-edges of the slots a near-far refill moved into frontier t, [t%3]
+  unsigned long long refill_deg[3];  // slots a near-far refill moved into frontier t, [t%3]
   unsigned int dense_bin;       // blocked dense relaxation: next sink bin to claim
   unsigned int wmul;            // near-far window = delta * wmul (doubles after small refills; 0 reads as 1)
+  // frontier windows (persistent LB loop, win_on): the bits of frontier k
+  // (bm[k%3]) lie only in words [wlo[k%6], whi[k%6]] (wlo > whi: empty), the
+  // far pile's bits in [flo[e&1], fhi[e&1]] for refill epoch e; the scan, the
+  // clear of the recycled bitmap and the refill touch only those words.  Six
+  // slots, not three: the lead empties frontier k's slot in the decision of
+  // iteration k+1 (no barrier follows it), and that slot's next pushes come
+  // three grid barriers later (frontier k+6), never racing the reset
+  unsigned int win_on;
+  unsigned int wlo[6], whi[6];
+  unsigned int flo[2], fhi[2];
+  unsigned int epoch;
 };
 
 struct SsspAux {

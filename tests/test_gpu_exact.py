@@ -464,3 +464,39 @@ def test_sssp_blocked_dense_iterations_bit_exact(name, dense, monkeypatch):
         assert np.array_equal(got, want), f"{np.sum(got != want)} mismatches"
     if dense == "0":
         assert info["dense_iterations"] == 0
+
+
+@pytest.mark.parametrize("name", ["rmat12", "uniform", "road64", "star_hub", "dups_loops", "isolated", "single"])
+@pytest.mark.parametrize("window", ["0", "1"])
+@pytest.mark.parametrize("dense", ["0", "1e-9"])
+def test_sssp_frontier_windows_bit_exact(name, window, dense, monkeypatch):
+    """The persistent loop's frontier windows (scan / clear / refill only the
+    bitmap words that can hold bits) on and off, with and without blocked
+    dense iterations (which reset the windows to the full range): Dijkstra's
+    distances bit for bit, twice on the same graph."""
+    monkeypatch.setenv("GX_SSSP_WINDOW", window)
+    monkeypatch.setenv("GX_SSSP_DENSE", dense)
+    raw = GRAPHS[name]()
+    g = from_raw(raw)
+    want = A.sssp_dijkstra(graph_to_edgelist(g), sssp_source(g))
+    G = upload(raw)
+    for _ in range(2):
+        info = G.run("sssp", source=-1, mapping="lb")
+        assert info["converged"] == 1
+        assert np.array_equal(G.download("dist"), want)
+
+
+def test_sssp_windows_road_renumbered_bit_exact(monkeypatch):
+    """Frontier windows on the §2-renumbered road grid (renumber only,
+    theta > 1: the BFS-level ids keep a wavefront in a narrow word band);
+    forced on (the default turns them on from 4M slots)."""
+    import paper_conf_icpp_0001n20_b200 as gx
+    monkeypatch.setenv("GX_SSSP_WINDOW", "1")
+    raw = graphgen.road(96)
+    g = from_raw(raw)
+    want = A.sssp_dijkstra(graph_to_edgelist(g), sssp_source(g))
+    G = upload(raw)
+    G.transform(gx.Knobs(coalesce=True, replicate_threshold=2.0))
+    for mp in ("lb", "tpv"):
+        assert G.run("sssp", source=-1, mapping=mp)["converged"] == 1
+        assert np.array_equal(G.download("dist"), want)

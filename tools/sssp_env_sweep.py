@@ -14,7 +14,7 @@ import graphgen  # noqa: E402
 import paper_conf_icpp_0001n20_b200 as gx  # noqa: E402
 
 MAKE = {"rmat24": lambda: graphgen.rmat(24), "rmat22": lambda: graphgen.rmat(22), "rmat26": lambda: graphgen.rmat(26),
-        "uniform24": lambda: graphgen.uniform(1 << 24, 1 << 28), "road4900": lambda: graphgen.road(4900)}
+        "uniform24": lambda: graphgen.uniform(1 << 24, 1 << 28), "road4900": lambda: graphgen.road(4900), "road1024": lambda: graphgen.road(1024)}
 ap = argparse.ArgumentParser()
 ap.add_argument("--env", required=True)
 ap.add_argument("--values", required=True)
