@@ -73,7 +73,7 @@ __device__ __forceinline__ void relax_nf(uint2 ed, uint32_t du, uint32_t cur, ui
       wn.nlo = min(wn.nlo, w);
       wn.nhi = max(wn.nhi, w);
     } else {
-      red_or_l2(far + w, 1u << (ed.x & 31), pl);
+      if (far) red_or_l2(far + w, 1u << (ed.x & 31), pl);   // null: far pile by scan (sssp_split_dev)
       far_min = min(far_min, nd);
       wn.flo = min(wn.flo, w);
       wn.fhi = max(wn.fhi, w);
@@ -722,7 +722,7 @@ __device__ __forceinline__ void sssp_split_dev(const uint32_t* __restrict__ dist
                                                SsspState* __restrict__ st, int64_t lo, int64_t hi, const unsigned t,
                                                const uint32_t tau, uint32_t* fdst,
                                                const uint32_t* __restrict__ rp = nullptr, const bool win = false,
-                                               const unsigned fslot = 0) {
+                                               const unsigned fslot = 0, const uint32_t tau_prev = 0) {
   // win: the far pile's bits lie in words [flo[fslot], fhi[fslot]]; the moved
   // bits' words widen bm[t%3]'s window, the kept bits' words form the far
   // window of the next epoch (slot fslot ^ 1, empty before)
@@ -730,7 +730,60 @@ __device__ __forceinline__ void sssp_split_dev(const uint32_t* __restrict__ dist
   uint32_t my_min = INF;
   unsigned long long my_deg = 0;   // the moved slots (dense-iteration test, adaptive window)
   Win wn;
-  int64_t w_lo = lo >> 5, w_hi = min((hi + 31) >> 5, ax.nwords);
+  if (!ax.far) {
+    // far pile by scan (ax.far null: no far bitmap, the persistent loop on
+    // graphs without merges / tiles / windows): the far pile is exactly the
+    // rows with tau_prev <= dist < INF.  A row is only ever processed in a
+    // near frontier at a value below that frontier's tau <= tau_prev, and dist
+    // only decreases, so a row at >= tau_prev was never processed at its value;
+    // a row below tau_prev was processed at its value or still waits in the
+    // near frontier (early refill).  One coalesced read of dist per refill
+    // instead of a red.or per far push (and no stale far bits re-activated)
+    const int64_t gwp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwp = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    // 128 slots (4 bitmap words) per warp load: lane l holds slots 4l..4l+3
+    // (one uint4), its 4-bit move mask is OR-reduced over the 8 lanes of a
+    // word; FS_U chunks per warp loaded together.  lo == 0 (persistent loop).
+    const unsigned lane = lane_id();
+    const int64_t c_end = (hi + 127) >> 7;
+    constexpr int FS_U = 4;
+    for (int64_t cb = gwp; cb < c_end; cb += nwp * FS_U) {
+      uint4 q[FS_U];
+#pragma unroll
+      for (int k = 0; k < FS_U; k++) {
+        const int64_t ch = cb + k * nwp;
+        const int64_t v = ch * 128 + 4 * lane;
+        if (ch < c_end && v + 3 < hi) {
+          q[k] = __ldcg(reinterpret_cast<const uint4*>(dist + v));
+        } else {
+          const bool in = ch < c_end;
+          q[k].x = in && v < hi ? __ldcg(dist + v) : INF;
+          q[k].y = in && v + 1 < hi ? __ldcg(dist + v + 1) : INF;
+          q[k].z = in && v + 2 < hi ? __ldcg(dist + v + 2) : INF;
+          q[k].w = INF;
+        }
+      }
+#pragma unroll
+      for (int k = 0; k < FS_U; k++) {
+        const uint32_t dd[4] = {q[k].x, q[k].y, q[k].z, q[k].w};
+        unsigned nib = 0;
+#pragma unroll
+        for (int c = 0; c < 4; c++) {
+          if (dd[c] >= tau_prev && dd[c] < tau) nib |= 1u << c;
+          if (dd[c] >= tau && dd[c] != INF) my_min = min(my_min, dd[c]);
+        }
+        unsigned x = nib << (4 * (lane & 7));
+        x |= __shfl_xor_sync(FULL, x, 1);
+        x |= __shfl_xor_sync(FULL, x, 2);
+        x |= __shfl_xor_sync(FULL, x, 4);
+        if ((lane & 7) == 0 && x) {
+          atomicOr(bm_cur + (cb + k * nwp) * 4 + (lane >> 3), x);   // RED: the word may hold near pushes
+          my_deg += __popc(x);
+        }
+      }
+    }
+  }
+  int64_t w_lo = lo >> 5, w_hi = ax.far ? min((hi + 31) >> 5, ax.nwords) : w_lo;
   if (win) {
     w_lo = max(w_lo, (int64_t)st->flo[fslot]);
     w_hi = min(w_hi, (int64_t)st->fhi[fslot] + 1);
@@ -971,9 +1024,9 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
   // after the previous refill (replicated like tau)
   const bool win = st->win_on != 0;
   unsigned epoch = st->epoch;
-  auto refill = [&](unsigned tt) {
+  auto refill = [&](unsigned tt, uint32_t tau_prev) {
     sssp_split_dev(a.dist, a.ax, st, 0, a.n_slots, tt, tau, &st->far3[tt % 3], a.dense_edges ? a.rp : nullptr, win,
-                   epoch & 1u);
+                   epoch & 1u, tau_prev);
     grid.sync();
     if (lead) {
       st->flo[epoch & 1u] = 0xFFFFFFFFu;   // read by this refill only; the next refill builds it
@@ -984,7 +1037,7 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
   };
   // the relaunch's pending near-far refill (decided after the dense iteration)
   if (*(volatile unsigned*)&st->split) {
-    refill(t);
+    refill(t, st->tau_prev);
     if (lead) st->split = 0;
     adapt(t);
     if (a.dense_edges && *(volatile unsigned long long*)&st->refill_deg[t % 3] >= a.dense_edges) {
@@ -1033,6 +1086,7 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
       }
     }
     // ---- decision (every thread, identical inputs)
+    const uint32_t tau_b = tau;   // the bucket bound the refill's far-by-scan starts from
     const unsigned pushed = *(volatile unsigned*)&st->pushed[t % 3];
     const uint32_t fm = min(rf, *(volatile unsigned*)&st->far3[t % 3]);
     unsigned stop = 0;
@@ -1098,7 +1152,7 @@ __global__ void __launch_bounds__(PERSIST_TPB, GX_SSSP_MINB) k_sssp_persist(Sssp
     if (stop) break;
     t++;
     if (split) {   // near-far refill of iteration t's frontier
-      refill(t);
+      refill(t, tau_b);
       adapt(t);
       // a refill that carries most of the graph's edges: hand iteration t to the
       // blocked dense relaxation (k_sssp_pb_*), which streams every edge once
@@ -1298,7 +1352,7 @@ __global__ void __launch_bounds__(SPB_THREADS, 1) k_sssp_pb_gather(SsspPb p, uin
         const int64_t w = v >> 5;
         my_act += __popc(__ldcg(bm_cur + w));
         if (bn) bm_next[w] |= bn;
-        if (bf) ax.far[w] |= bf;
+        if (bf && ax.far) ax.far[w] |= bf;
         my_push += __popc(bn);
       }
     }
@@ -1317,6 +1371,7 @@ __global__ void k_sssp_dense_decide(SsspState* __restrict__ st, int64_t m_slots,
   const unsigned pushed = st->pushed[t % 3];
   const uint32_t fm = min(st->far_min, st->far3[t % 3]);
   uint32_t tau = st->tau, rf = fm;
+  st->tau_prev = tau;
   unsigned stop = 0, split = 0;
   if ((pushed <= early || pushed == 0) && fm != INF) {
     const unsigned long long nt = (unsigned long long)fm + (unsigned long long)st->delta * (st->wmul ? st->wmul : 1u);
@@ -2031,6 +2086,7 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
   CUDA_OK(cudaEventRecord(e0, s));
   CUDA_OK(cudaMemsetAsync(r.dist.p, 0xFF, sizeof(uint32_t) * ns, s));
   CUDA_OK(cudaMemsetAsync(r.mark.p, 0, sizeof(uint32_t) * 6 * nwords, s));
+  bool win_h = false;
   {
     // near-far bucket width (LB mapping only; 0 = plain frontier Bellman-Ford)
     static SsspState init;
@@ -2055,6 +2111,7 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
                         !getenv("GX_SSSP_BLOCK");
     const bool win_auto = (double)g->m < 4.0 * (double)std::max<int64_t>(1, g->n) && d.n_slots >= (int64_t(1) << 22);
     init.win_on = win_ok && (we ? atoi(we) != 0 : win_auto) ? 1u : 0u;
+    win_h = init.win_on != 0;
     init.wlo[0] = 0xFFFFFFFFu;
     for (int32_t sv : srcs) {
       init.wlo[0] = std::min(init.wlo[0], (unsigned)(sv >> 5));
@@ -2214,6 +2271,18 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
       // each local round still pays an L2 round trip per hop)
       const bool want = be ? atoi(be) != 0 && d.blk_maxdeg <= 64 : false;
       if (want) L.block_rows = B;
+    }
+    // far pile by scan (sssp_split_dev): no far bitmap, so a relaxation that
+    // lands beyond tau issues one reduction (dist) instead of two; the refill
+    // reads dist once, coalesced.  Not with windows (a scan of all of dist per
+    // refill, ~10^3 refills on a road grid), merges, §3 tiles, the
+    // light/heavy split or the block mode (they push far bits of their own).
+    // GX_SSSP_FARSCAN=0 keeps the bitmap
+    const char* fse = getenv("GX_SSSP_FARSCAN");
+    const bool far_scan = !win_h && !d.n_groups && !tiles && !want_lh && L.block_rows == 0 && !(fse && atoi(fse) == 0);
+    if (far_scan) {
+      L.ax.far = nullptr;
+      ax.far = nullptr;   // the dense iteration's gather too
     }
     if (want_lh && L.block_rows == 0) {
       L.ax.lend = d.lh_lend.as<uint32_t>();

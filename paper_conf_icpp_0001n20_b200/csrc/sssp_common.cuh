@@ -42,6 +42,7 @@ struct SsspState {
   unsigned int wlo[6], whi[6];
   unsigned int flo[2], fhi[2];
   unsigned int epoch;
+  unsigned int tau_prev;        // far-by-scan refills: the bucket bound before the last raise of tau
 };
 
 struct SsspAux {
