@@ -167,16 +167,20 @@ __device__ __forceinline__ void clear_bitmap(uint32_t* bm, int64_t nwords) {
 // measured (RMAT-24 exact, persistent loop, profiles/r1e/sssp_hint_variants.txt):
 // row_ptr loads with L2 evict_first (the gathered dist keeps the L2) and 3
 // edges in flight per lane: 5.04 -> 4.78 ms; SU 8: 5.8 ms; 5-6 CTAs/SM
-// (__launch_bounds__ min blocks, spills): 5.9-9.8 ms
+// (__launch_bounds__ min blocks, spills): 5.9-9.8 ms.  Round 2, after the far
+// pile by scan (profiles/r2/sssp_su_pipe_variants.txt): the software pipeline
+// off and 5 edges in flight per lane: RMAT-24 4.06 -> 3.67 ms, uniform
+// 16M/256M 4.05 -> 3.83, RMAT-22 1.93 -> 1.70 (SU 3 / 4 / 6 and the pipeline
+// on are slower; 3 CTAs per SM 4.39)
 #ifndef GX_SSSP_RP_EF
 #define GX_SSSP_RP_EF 1
 #endif
 #ifndef GX_SSSP_SU
-#define GX_SSSP_SU 3
+#define GX_SSSP_SU 5
 #endif
 constexpr int SU = GX_SSSP_SU;   // edges in flight per lane per round
 #ifndef GX_SSSP_PIPE
-#define GX_SSSP_PIPE 1
+#define GX_SSSP_PIPE 0
 #endif
 #ifndef GX_SSSP_TPB
 #define GX_SSSP_TPB 256
