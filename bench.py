@@ -129,8 +129,10 @@ def inaccuracy_pct(approx, exact, inf=None):
 
 def knob_points(ctx, reps=2):
     """BASELINE metric's "speedup vs exact at inaccuracy%" (Tables 6 and 8,
-    P@42046-42906, P@43835-44682) at two paper-style settings: C2 (RMAT-22) §2
-    coalescing k=16, theta_conn=0.6 with the algorithm-aware merge; C4 (uniform
+    P@42046-42906, P@43835-44682) at three paper-style settings: C2 (RMAT-22) §2
+    coalescing k=16, theta_conn=0.6 with the algorithm-aware merge; C3 (road
+    grid 4900^2) §2 renumbering alone (theta_conn=2.0: no vertex can reach it, so
+    no replicas -- the BFS-level isomorph of Alg 2 l.10-20 only); C4 (uniform
     16M/256M) §4 degree normalisation theta_d=0.3, f=0.85.  Per algorithm: the
     knob's best mapping vs the best exact mapping, and per mapping vs the same
     mapping exact; inaccuracy (R40) of the knob run vs the exact run; transform
@@ -141,6 +143,8 @@ def knob_points(ctx, reps=2):
     cases = [
         ("C2 rmat22 coalesce k16 theta0.6 aware-merge", lambda: graphgen.rmat(22),
          gx.Knobs(coalesce=True, chunk_k=16, replicate_threshold=0.6, merge_op=1)),
+        ("C3 road4900 coalesce k16 renumber-only (theta_conn 2.0)", lambda: graphgen.road(4900),
+         gx.Knobs(coalesce=True, chunk_k=16, replicate_threshold=2.0)),
         ("C4 uniform16M/256M degnorm theta0.3 f0.85", lambda: graphgen.uniform(1 << 24, 1 << 28),
          gx.Knobs(degree_norm=True, degsim_threshold=0.3, degree_target=0.85)),
     ]
@@ -266,7 +270,7 @@ def main():
     ap.add_argument("--workload", default="t24", choices=list(WORKLOADS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--no-knobs", action="store_true", help="skip the knob speedup / inaccuracy points (~60 s)")
+    ap.add_argument("--no-knobs", action="store_true", help="skip the knob speedup / inaccuracy points (~90 s)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--e2e-sync", action="store_true", help="upload without GX_ASYNC_UPLOAD")
     ap.add_argument("--e2e-w32", action="store_true", help="upload 32-bit weights (not GX_W_U8)")

@@ -111,15 +111,27 @@ __global__ void k_tri(const uint64_t* __restrict__ fp, const int32_t* __restrict
 void gpu_triangles(Ctx* c, int64_t n, const int64_t* np, const int32_t* nc, int64_t* T) {
   cudaStream_t s = c->stream;
   const int64_t mm = np[n];
-  DBuf dnp, dnc, fc, fp, fw, dT, tmp;
+  DBuf dnp, dnc, dT;
   dnp.alloc(c, sizeof(int64_t) * (n + 1));
   dnc.alloc(c, sizeof(int32_t) * std::max<int64_t>(mm, 1));
   CUDA_OK(cudaMemcpyAsync(dnp.p, np, sizeof(int64_t) * (n + 1), cudaMemcpyHostToDevice, s));
   if (mm) CUDA_OK(cudaMemcpyAsync(dnc.p, nc, sizeof(int32_t) * mm, cudaMemcpyHostToDevice, s));
+  dT.alloc(c, sizeof(unsigned long long) * std::max<int64_t>(n, 1));
+  gpu_triangles_dev(c, n, dnp.as<int64_t>(), dnc.as<int32_t>(), mm, dT.as<unsigned long long>());
+  if (n) CUDA_OK(cudaMemcpyAsync(T, dT.p, sizeof(int64_t) * n, cudaMemcpyDeviceToHost, s));
+  CUDA_OK(cudaStreamSynchronize(s));
+}
+
+// device-resident form: U as device CSR (dnp [n+1], dnc [mm]); dT [n] out
+void gpu_triangles_dev(Ctx* c, int64_t n, const int64_t* dnp, const int32_t* dnc, int64_t mm,
+                       unsigned long long* dT) {
+  cudaStream_t s = c->stream;
+  (void)mm;
+  DBuf fc, fp, fw, tmp;
   fc.alloc(c, sizeof(uint64_t) * (n + 1));
   CUDA_OK(cudaMemsetAsync(fc.p, 0, sizeof(uint64_t) * (n + 1), s));
   const int grid = c->num_sms * 16;
-  k_fwd_count<<<grid, 256, 0, s>>>(dnp.as<int64_t>(), dnc.as<int32_t>(), n, fc.as<uint32_t>());
+  k_fwd_count<<<grid, 256, 0, s>>>(dnp, dnc, n, fc.as<uint32_t>());
   CUDA_OK(cudaGetLastError());
   // u64 offsets of the forward lists (their total can exceed 2^32)
   fp.alloc(c, sizeof(uint64_t) * (n + 1));
@@ -135,14 +147,11 @@ void gpu_triangles(Ctx* c, int64_t n, const int64_t* np, const int32_t* nc, int6
   CUDA_OK(cudaMemcpyAsync(&nf, fp.as<uint64_t>() + n, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
   CUDA_OK(cudaStreamSynchronize(s));
   fw.alloc(c, sizeof(int32_t) * std::max<uint64_t>(nf, 1));
-  k_fwd_fill<<<grid, 256, 0, s>>>(dnp.as<int64_t>(), dnc.as<int32_t>(), n, fp.as<uint64_t>(), fw.as<int32_t>());
+  k_fwd_fill<<<grid, 256, 0, s>>>(dnp, dnc, n, fp.as<uint64_t>(), fw.as<int32_t>());
   CUDA_OK(cudaGetLastError());
-  dnc.reset();
-  dT.alloc(c, sizeof(unsigned long long) * std::max<int64_t>(n, 1));
-  CUDA_OK(cudaMemsetAsync(dT.p, 0, sizeof(unsigned long long) * std::max<int64_t>(n, 1), s));
-  k_tri<<<grid, 256, 0, s>>>(fp.as<uint64_t>(), fw.as<int32_t>(), n, dT.as<unsigned long long>());
+  CUDA_OK(cudaMemsetAsync(dT, 0, sizeof(unsigned long long) * std::max<int64_t>(n, 1), s));
+  k_tri<<<grid, 256, 0, s>>>(fp.as<uint64_t>(), fw.as<int32_t>(), n, dT);
   CUDA_OK(cudaGetLastError());
-  if (n) CUDA_OK(cudaMemcpyAsync(T, dT.p, sizeof(int64_t) * n, cudaMemcpyDeviceToHost, s));
   CUDA_OK(cudaStreamSynchronize(s));
 }
 
@@ -406,7 +415,7 @@ void gpu_pad_candidates(Ctx* c, int64_t n, const int64_t* lp, const int32_t* ld,
   rkeys.clear();
   if (nq == 0) return;
   const int64_t m = lp[n];
-  DBuf dlp, dld, dlw, dqu, cnt, off, tmp, k0, k1, sb, kout;
+  DBuf dlp, dld, dlw, dqu;
   dlp.alloc(c, sizeof(int64_t) * (n + 1));
   dld.alloc(c, sizeof(int32_t) * std::max<int64_t>(m, 1));
   dlw.alloc(c, sizeof(uint32_t) * std::max<int64_t>(m, 1));
@@ -417,11 +426,26 @@ void gpu_pad_candidates(Ctx* c, int64_t n, const int64_t* lp, const int32_t* ld,
     CUDA_OK(cudaMemcpyAsync(dlw.p, lw, sizeof(uint32_t) * m, cudaMemcpyHostToDevice, s));
   }
   CUDA_OK(cudaMemcpyAsync(dqu.p, qu, sizeof(int32_t) * nq, cudaMemcpyHostToDevice, s));
+  gpu_pad_candidates_dev(c, n, dlp.as<int64_t>(), dld.as<int32_t>(), dlw.as<uint32_t>(), nq, dqu.as<int32_t>(), qtake,
+                         rule, rptr, rkeys);
+}
+
+// device-resident form: G_L as device CSR (dlp, dld, dlw), queries dqu on the
+// device, their budgets qtake on the host
+void gpu_pad_candidates_dev(Ctx* c, int64_t n, const int64_t* dlp_, const int32_t* dld_, const uint32_t* dlw_,
+                            int64_t nq, const int32_t* dqu_, const int32_t* qtake, int rule,
+                            std::vector<int64_t>& rptr, std::vector<uint64_t>& rkeys) {
+  cudaStream_t s = c->stream;
+  rptr.assign(nq + 1, 0);
+  rkeys.clear();
+  if (nq == 0) return;
+  (void)n;
+  DBuf cnt, off, tmp, k0, k1, sb, kout;
   cnt.alloc(c, sizeof(uint64_t) * (nq + 1));
   off.alloc(c, sizeof(uint64_t) * (nq + 1));
   CUDA_OK(cudaMemsetAsync(cnt.p, 0, sizeof(uint64_t) * (nq + 1), s));
   const int grid = c->num_sms * 16;
-  k_pad_count<<<grid, 256, 0, s>>>(dlp.as<int64_t>(), dld.as<int32_t>(), dqu.as<int32_t>(), nq, cnt.as<uint64_t>());
+  k_pad_count<<<grid, 256, 0, s>>>(dlp_, dld_, dqu_, nq, cnt.as<uint64_t>());
   CUDA_OK(cudaGetLastError());
   size_t tb = 0;
   CUDA_OK(cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt.as<uint64_t>(), off.as<uint64_t>(), nq + 1, s));
@@ -452,7 +476,7 @@ void gpu_pad_candidates(Ctx* c, int64_t n, const int64_t* lp, const int32_t* ld,
     for (int64_t i = 0; i <= bq; i++) seg[i] = (int64_t)(hoff[i0 + i] - base);
     CUDA_OK(cudaMemcpyAsync(sb.p, seg.data(), sizeof(int64_t) * (bq + 1), cudaMemcpyHostToDevice, s));
     if (tot) {
-      k_pad_fill<<<grid, 256, 0, s>>>(dlp.as<int64_t>(), dld.as<int32_t>(), dlw.as<uint32_t>(), dqu.as<int32_t>() + i0,
+      k_pad_fill<<<grid, 256, 0, s>>>(dlp_, dld_, dlw_, dqu_ + i0,
                                       bq, off.as<uint64_t>() + i0, base, rule, k0.as<unsigned long long>());
       CUDA_OK(cudaGetLastError());
       size_t t1 = 0;

@@ -263,6 +263,40 @@ void gpu_bfs_forest(Ctx* c, int64_t n, const int64_t* rp, const int32_t* col, st
 void gpu_pad_candidates(Ctx* c, int64_t n, const int64_t* lp, const int32_t* ld, const uint32_t* lw, int64_t nq,
                         const int32_t* qu, const int32_t* qtake, int rule, std::vector<int64_t>& rptr,
                         std::vector<uint64_t>& rkeys);
+// device pipeline of the transforms (dtransform.cu, driven by transform.cpp's
+// transform_device): the slot graph as one edge list in HBM,
+// key = src slot << 32 | dst slot, val = weight | AddKind << 32
+struct DEdges {
+  DBuf key, val;
+  int64_t m = 0;
+};
+struct DtCand { int32_t lv, cnt, s, C; };   // a (slot, chunk) replica candidate of level lv
+struct DtAsg { int32_t s, C; int64_t hole; };
+// din: the canonical graph resident on the device ({row_ptr i64, col i32, w u32}
+// = gx_graph in_rp/in_col/in_w, identical to g), or all null (uploaded from g)
+struct DevCSR { const int64_t* rp = nullptr; const int32_t* col = nullptr; const uint32_t* w = nullptr; };
+void transform_device(const HostCSR& g, const gx_knobs& k, SlotGraph& out, Ctx* dev, DevCSR din = {});
+void dt_from_csr(Ctx* c, const HostCSR& g, const int32_t* nw, DEdges& E, const int64_t* drp = nullptr,
+                 const int32_t* dcol = nullptr, const uint32_t* dw = nullptr);
+void dt_sort(Ctx* c, DEdges& E, int64_t ns);
+void dt_row_ptr(Ctx* c, const DEdges& E, int64_t ns, DBuf& rp);
+void dt_replica_candidates(Ctx* c, const DEdges& E, int k, const std::vector<int32_t>& chunk_lv,
+                           const std::vector<int32_t>& nonhole, int64_t theta_ppm, std::vector<DtCand>& out);
+int64_t dt_replicate(Ctx* c, DEdges& E, int64_t ns, int k, const std::vector<DtAsg>& asg,
+                     const std::vector<uint8_t>& kind, int rule);
+void dt_append_dev(Ctx* c, DEdges& E, const DBuf& key, const DBuf& val, int64_t na);
+void dt_append(Ctx* c, DEdges& E, const std::vector<uint64_t>& key, const std::vector<uint64_t>& val);
+void dt_logical(Ctx* c, const DEdges& E, const DBuf& s2o, int64_t n, DBuf& lp, DBuf& ld, DBuf& lw, DBuf* keys);
+int64_t dt_undirected(Ctx* c, int64_t n, const DBuf& lkey, int64_t ml, DBuf& np, DBuf& nc);
+void dt_degnorm(Ctx* c, DEdges& E, int64_t ns, int64_t n, const std::vector<uint8_t>& kind, const DBuf& s2o,
+                const std::vector<int32_t>& owner, int64_t th, int64_t f, bool combined, int rule,
+                std::vector<int32_t>& sched, int64_t& added);
+void dt_export(Ctx* c, DEdges& E, int64_t ns, SlotGraph& out);
+void gpu_triangles_dev(Ctx* c, int64_t n, const int64_t* dnp, const int32_t* dnc, int64_t mm,
+                       unsigned long long* dT);
+void gpu_pad_candidates_dev(Ctx* c, int64_t n, const int64_t* dlp, const int32_t* dld, const uint32_t* dlw, int64_t nq,
+                            const int32_t* dqu, const int32_t* qtake, int rule, std::vector<int64_t>& rptr,
+                            std::vector<uint64_t>& rkeys);
 void build_device_exact(gx_graph* g);
 void resolve_pending(gx_graph* g);
 void join_download(gx_graph* g, int kind);   // kind < 0: every kind

@@ -899,3 +899,196 @@ void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out, Ctx* de
 }
 
 }  // namespace gx
+
+namespace gx {
+
+// The same three transforms with the slot graph resident in HBM (SURVEY.md
+// §8(f) N1, dtransform.cu): relabel, replica candidates and rows, G_L and its
+// undirected view, triangles, degree buckets, the warp schedule, padding and
+// the final CSR rebuild run on the device; the host keeps the sequential
+// decisions -- the cursor numbering (Alg 2 l.10-20), the choice of each
+// level's h best replica candidates (Alg 2 l.24-27, R13/R14), the §3
+// budgeted insertion and subgraph packing -- and the per-slot metadata
+// (slot -> vertex, slot kind, vertex -> owner slot).  Output equals
+// transform_host's bit for bit.
+void transform_device(const HostCSR& g, const gx_knobs& k, SlotGraph& out, Ctx* dev, DevCSR din) {
+  auto t0 = std::chrono::steady_clock::now();
+  const bool trace = getenv("GX_TRANSFORM_TRACE") != nullptr;
+  auto tp = t0;
+  auto phase = [&](const char* name) {
+    if (!trace) return;
+    auto now = std::chrono::steady_clock::now();
+    fprintf(stderr, "transform %-18s %8.1f ms\n", name, std::chrono::duration<double, std::milli>(now - tp).count());
+    tp = now;
+  };
+  const int64_t n = g.n;
+  int64_t ns = n, n_holes = 0, n_repl = 0, added_coal = 0;
+  std::vector<int32_t> s2o, owner;
+  std::vector<uint8_t> kind;
+  DEdges E;
+  if (k.coalesce) {
+    const int kk = k.chunk_k;
+    std::vector<std::pair<int64_t, int64_t>> ranges;
+    renumber(g, kk, owner, ns, ranges, dev);
+    s2o.assign(ns, -1);
+    kind.assign(ns, HOLE);
+    for (int64_t u = 0; u < n; u++) {
+      s2o[owner[u]] = (int32_t)u;
+      kind[owner[u]] = OWNER;
+    }
+    phase("slot maps");
+    dt_from_csr(dev, g, owner.data(), E, din.rp, din.col, din.w);
+    phase("relabel (GPU)");
+    dt_sort(dev, E, ns);
+    phase("sort (GPU)");
+    // chunks of levels >= 1 whose previous level has holes (Alg 2 l.21-23)
+    const int64_t nchunks = (ns + kk - 1) / kk;
+    std::vector<int32_t> nonhole(std::max<int64_t>(nchunks, 1), 0), chunk_lv(std::max<int64_t>(nchunks, 1), -1);
+    for (int64_t s = 0; s < ns; s++)
+      if (kind[s] != HOLE) nonhole[s / kk]++;
+    const size_t nlv = ranges.size();
+    std::vector<int64_t> lv_holes(nlv, 0);
+    for (size_t li = 1; li < nlv; li++) {
+      lv_holes[li] = std::max<int64_t>(0, ranges[li].first - ranges[li - 1].second);
+      if (lv_holes[li] <= 0) continue;
+      for (int64_t C = ranges[li].first / kk; C <= (ranges[li].second - 1) / kk; C++) chunk_lv[C] = (int32_t)li;
+    }
+    std::vector<DtCand> cands;
+    dt_replica_candidates(dev, E, kk, chunk_lv, nonhole, ppm(k.replicate_threshold), cands);
+    // per level, the h holes go to the candidates in (count desc, slot, chunk) order
+    std::vector<std::vector<std::tuple<int64_t, int32_t, int64_t>>> per(nlv);
+    for (const DtCand& c : cands) per[c.lv].push_back({-(int64_t)c.cnt, c.s, (int64_t)c.C});
+    std::vector<DtAsg> asg;
+    for (size_t li = 1; li < nlv; li++) {
+      const int64_t h0 = ranges[li - 1].second, h1 = ranges[li].first;
+      if (h1 <= h0 || per[li].empty()) continue;
+      auto& cl = per[li];
+      const size_t h = (size_t)(h1 - h0);
+      if (cl.size() > h) {
+        std::nth_element(cl.begin(), cl.begin() + h, cl.end());
+        cl.resize(h);
+      }
+      std::sort(cl.begin(), cl.end());
+      int64_t hole = h0;
+      for (auto& c : cl) asg.push_back({std::get<1>(c), (int32_t)std::get<2>(c), hole++});
+    }
+    phase("replica candidates (GPU)");
+    added_coal = dt_replicate(dev, E, ns, kk, asg, kind, k.added_weight_rule);
+    for (const DtAsg& a : asg) {
+      kind[a.hole] = REPLICA;
+      s2o[a.hole] = s2o[a.s];
+    }
+    int64_t holes_left = 0;
+    for (int64_t s = 0; s < ns; s++) holes_left += kind[s] == HOLE;
+    n_repl = (int64_t)asg.size();
+    n_holes = holes_left + n_repl;
+    phase("replica rows (GPU)");
+  } else {
+    s2o.resize(n);
+    owner.resize(n);
+    std::iota(s2o.begin(), s2o.end(), 0);
+    std::iota(owner.begin(), owner.end(), 0);
+    kind.assign(n, OWNER);
+    dt_from_csr(dev, g, nullptr, E, din.rp, din.col, din.w);
+    phase("edges (GPU)");
+  }
+  DBuf ds2o;
+  ds2o.alloc(dev, sizeof(int32_t) * std::max<int64_t>(ns, 1));
+  if (ns) CUDA_OK(cudaMemcpyAsync(ds2o.p, s2o.data(), sizeof(int32_t) * ns, cudaMemcpyHostToDevice, dev->stream));
+  SmemOut sm;
+  if (k.smem) {
+    // G_L, U and the triangle counts on the device; the greedy insertion
+    // (P@31015-31268, R22-R26) and the packing (R27, R28) on the host
+    Logical L;
+    L.n = n;
+    DBuf lp, ld, lw, lkey, np, nc, dT;
+    dt_logical(dev, E, ds2o, n, lp, ld, lw, &lkey);
+    const int64_t ml = E.m;
+    const int64_t mu = dt_undirected(dev, n, lkey, ml, np, nc);
+    lkey.reset();
+    dT.alloc(dev, sizeof(int64_t) * std::max<int64_t>(n, 1));
+    gpu_triangles_dev(dev, n, np.as<int64_t>(), nc.as<int32_t>(), mu, dT.as<unsigned long long>());
+    phase("logical+U+tri (GPU)");
+    std::vector<int64_t> hlp(n + 1), hnp(n + 1);
+    std::vector<int32_t> hld(std::max<int64_t>(ml, 1)), hnc(std::max<int64_t>(mu, 1));
+    std::vector<uint32_t> hlw(std::max<int64_t>(ml, 1));
+    L.T.assign(n, 0);
+    cudaStream_t st = dev->stream;
+    CUDA_OK(cudaMemcpyAsync(hlp.data(), lp.p, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost, st));
+    CUDA_OK(cudaMemcpyAsync(hnp.data(), np.p, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost, st));
+    if (ml) {
+      CUDA_OK(cudaMemcpyAsync(hld.data(), ld.p, sizeof(int32_t) * ml, cudaMemcpyDeviceToHost, st));
+      CUDA_OK(cudaMemcpyAsync(hlw.data(), lw.p, sizeof(uint32_t) * ml, cudaMemcpyDeviceToHost, st));
+    }
+    if (mu) CUDA_OK(cudaMemcpyAsync(hnc.data(), nc.p, sizeof(int32_t) * mu, cudaMemcpyDeviceToHost, st));
+    if (n) CUDA_OK(cudaMemcpyAsync(L.T.data(), dT.p, sizeof(int64_t) * n, cudaMemcpyDeviceToHost, st));
+    CUDA_OK(cudaStreamSynchronize(st));
+    lp.reset(); ld.reset(); lw.reset(); np.reset(); nc.reset(); dT.reset();
+    L.out.assign(n, {});
+    L.N.assign(n, {});
+#pragma omp parallel for schedule(dynamic, 4096)
+    for (int64_t u = 0; u < n; u++) {
+      auto& r = L.out[u];
+      r.reserve(hlp[u + 1] - hlp[u]);
+      for (int64_t e = hlp[u]; e < hlp[u + 1]; e++) r.push_back({hld[e], hlw[e]});
+      L.N[u].assign(hnc.begin() + hnp[u], hnc.begin() + hnp[u + 1]);
+    }
+    phase("logical to host");
+    const int64_t th = ppm(k.cc_threshold);
+    const int64_t budget = k.added_edge_budget >= 0 ? k.added_edge_budget : g.m / 100;
+    cc_edges(L, th, budget, k.added_weight_rule, k.sibling_undirected != 0, sm);
+    phase("cc_edges");
+    subgraphs(L, th, k.smem_max_nodes, k.smem_iters, sm);
+    phase("subgraphs");
+    std::vector<uint64_t> ak, av;
+    ak.reserve(sm.added.size());
+    av.reserve(sm.added.size());
+    for (auto& e : sm.added) {
+      ak.push_back(((uint64_t)(uint32_t)owner[std::get<0>(e)] << 32) | (uint32_t)owner[std::get<1>(e)]);
+      av.push_back((uint64_t)std::get<2>(e) | ((uint64_t)ADD_SMEM << 32));
+    }
+    dt_append(dev, E, ak, av);
+    par_free(L.out);
+    par_free(L.N);
+    phase("smem append+free");
+  }
+  std::vector<int32_t> sched;
+  int64_t added_dn = 0;
+  if (k.degree_norm) {
+    dt_degnorm(dev, E, ns, n, kind, ds2o, owner, ppm(k.degsim_threshold), ppm(k.degree_target), k.coalesce != 0,
+               k.added_weight_rule, sched, added_dn);
+    phase("degnorm (GPU)");
+  }
+  out = SlotGraph();
+  out.n = n;
+  out.n_slots = ns;
+  dt_export(dev, E, ns, out);
+  out.slot_to_orig = std::move(s2o);
+  out.kind = std::move(kind);
+  out.owner_slot = std::move(owner);
+  out.sched = std::move(sched);
+  out.tile_ptr.assign(1, 0);
+  for (auto& t : sm.tiles) {
+    out.tile_centre.push_back(std::get<0>(t));
+    for (int32_t v : std::get<1>(t)) out.tile_members.push_back(v);
+    out.tile_ptr.push_back((int64_t)out.tile_members.size());
+    out.tile_iters.push_back(std::get<2>(t));
+  }
+  phase("assemble (GPU)");
+  gx_transform_info& I = out.info;
+  std::memset(&I, 0, sizeof(I));
+  I.n_slots = ns;
+  I.m_slots = out.m_slots;
+  I.n_holes = n_holes;
+  I.n_replicas = n_repl;
+  I.holes_filled = n_repl;
+  I.edges_added_coalesce = added_coal;
+  I.edges_added_smem = (int64_t)sm.added.size();
+  I.edges_added_degnorm = added_dn;
+  I.n_subgraphs = (int64_t)sm.tiles.size();
+  I.subgraph_vertices = (int64_t)out.tile_members.size();
+  I.extra_space_pct = 100.0 * (double)((ns - n) + (out.m_slots - g.m)) / (double)std::max<int64_t>(1, g.n + g.m);
+  I.transform_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+}
+
+}  // namespace gx

@@ -3,9 +3,13 @@
 edge insertion and the subgraph selection) and the §2 source order,
 reachability forest and multi-source BFS levels (Alg 2 l.2-6) and the §4
 padding candidates (2-hop out-neighbours ranked by (weight, id), P@33654) are
-computed on the GPU (gtransform.cu).  The exported transformed graph must be bit-identical to
-the oracle's and to the host-only library path (no device), element by
-element -- the triangle counts feed integer decisions only."""
+computed on the GPU (gtransform.cu), and with a device context the whole slot
+graph is built in HBM (dtransform.cu: relabel, replica candidates and rows,
+G_L / U, degree buckets and warp schedule, padding, the CSR rebuild); the host
+keeps the cursor numbering and the greedy decisions.  The exported transformed
+graph must be bit-identical to the oracle's and to the host-only library path
+(no device), element by element -- the triangle counts feed integer decisions
+only."""
 import numpy as np
 import pytest
 
@@ -92,3 +96,67 @@ def test_device_levels_road_grid():
     a, b = G.export(), H.export()
     for k in ("row_ptr", "col", "slot_to_orig", "slot_kind"):
         assert np.array_equal(np.asarray(a[k]), np.asarray(b[k])), k
+
+
+EXPORT_KEYS = ("row_ptr", "col", "w", "edge_added", "slot_to_orig", "slot_kind", "sched", "tile_ptr",
+               "tile_members", "tile_centre", "tile_iters")
+INFO_KEYS = ("n_slots", "m_slots", "n_replicas", "n_holes", "edges_added_coalesce", "edges_added_smem",
+             "edges_added_degnorm", "n_subgraphs", "subgraph_vertices")
+
+PIPE_GRAPHS = {
+    "rmat14": lambda: graphgen.rmat(14),
+    "road120": lambda: graphgen.road(120),
+    "uniform": lambda: graphgen.uniform(5000, 60000),
+    "star_hub": lambda: graphgen.from_edge_list(
+        2000, [(0, v, 1 + v % 7) for v in range(1, 2000)] + [(v, (v * 7 + 3) % 2000, 1 + v % 5) for v in range(1, 2000)]
+        + [(v, (v + 1) % 2000, 2) for v in range(1, 2000)]),
+    "empty_rows": lambda: graphgen.from_edge_list(64, [(1, 2, 3), (2, 5, 1), (5, 1, 4), (9, 2, 2), (40, 41, 9)]),
+}
+PIPE_KNOBS = {
+    # chunk_k = 32: the replica kernel's lane masks use every bit
+    "coal_k32": T.Knobs(coalesce=True, chunk_k=32, replicate_threshold=0.1),
+    "coal_k4_max": T.Knobs(coalesce=True, chunk_k=4, replicate_threshold=0.2, added_weight="max"),
+    "coal_k8_mean": T.Knobs(coalesce=True, chunk_k=8, replicate_threshold=0.25, added_weight="mean"),
+    "coal_degnorm": T.Knobs(coalesce=True, chunk_k=16, replicate_threshold=0.3, degree_norm=True,
+                            degsim_threshold=0.5),
+    "smem_degnorm": T.Knobs(smem=True, cc_threshold=0.3, degree_norm=True, degsim_threshold=0.6),
+    "degnorm_f": T.Knobs(degree_norm=True, degsim_threshold=0.7, degree_target=0.6),
+    "all_mean": T.Knobs(coalesce=True, chunk_k=8, replicate_threshold=0.2, smem=True, cc_threshold=0.4,
+                        degree_norm=True, degsim_threshold=0.5, added_weight="mean"),
+}
+
+
+@pytest.mark.parametrize("gname", list(PIPE_GRAPHS))
+@pytest.mark.parametrize("kname", list(PIPE_KNOBS))
+@pytest.mark.parametrize("mode", ["device", "mixed"])
+def test_transform_pipelines_agree(gname, kname, mode, monkeypatch):
+    """N1: the device-resident pipeline (default with a context) and the round-1
+    host pipeline with device helpers (GX_TRANSFORM=mixed) export exactly the
+    host-only library's slot graph, which the CPU suite pins to the oracle."""
+    import paper_conf_icpp_0001n20_b200 as gx
+    ctx()
+    if mode == "mixed":
+        monkeypatch.setenv("GX_TRANSFORM", "mixed")
+    raw = PIPE_GRAPHS[gname]()
+    kn = PIPE_KNOBS[kname]
+    G = upload(raw)
+    info = G.transform(_knobs(gx, kn))
+    H = gx.Graph.host_only(raw.row_ptr, raw.col, raw.w)
+    hinfo = H.transform(_knobs(gx, kn))
+    a, b = G.export(), H.export()
+    for k in EXPORT_KEYS:
+        assert np.array_equal(np.asarray(a[k]), np.asarray(b[k])), k
+    for k in INFO_KEYS:
+        assert info[k] == hinfo[k], k
+
+
+def test_device_pipeline_oracle_replicas():
+    """A graph where §2 places many replicas (low theta_conn, k = 4): the device
+    pipeline's export equals the oracle's element by element."""
+    import paper_conf_icpp_0001n20_b200 as gx
+    raw = graphgen.rmat(11)
+    kn = T.Knobs(coalesce=True, chunk_k=4, replicate_threshold=0.1)
+    G = upload(raw)
+    info = G.transform(_knobs(gx, kn))
+    assert info["n_replicas"] > 0
+    assert_same(G.export(), oracle_export(raw, kn), info)
