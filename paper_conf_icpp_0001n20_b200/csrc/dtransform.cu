@@ -205,6 +205,12 @@ __global__ void k_dt_split(const unsigned long long* __restrict__ key, const uns
   }
 }
 
+__global__ void k_dt_pairs(const int32_t* __restrict__ d, const uint32_t* __restrict__ w, int64_t m,
+                           unsigned long long* __restrict__ out) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x)
+    out[e] = ((unsigned long long)w[e] << 32) | (uint32_t)d[e];
+}
+
 // U: both directions of every G_L edge (sorted + deduplicated by the caller)
 __global__ void k_dt_sym(const unsigned long long* __restrict__ lkey, int64_t m, unsigned long long* __restrict__ ukey) {
   for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x) {
@@ -435,6 +441,14 @@ void dt_logical(Ctx* c, const DEdges& E, const DBuf& s2o, int64_t n, DBuf& lp, D
   CUDA_OK(cudaGetLastError());
   CUDA_OK(cudaStreamSynchronize(s));
   if (keys) std::swap(*keys, L.key);
+}
+
+void dt_pairs(Ctx* c, const DBuf& ld, const DBuf& lw, int64_t m, DBuf& out) {
+  out.alloc(c, sizeof(uint64_t) * std::max<int64_t>(m, 1));
+  if (m)
+    k_dt_pairs<<<grid_for(c, m), 256, 0, c->stream>>>(ld.as<int32_t>(), lw.as<uint32_t>(), m,
+                                                       out.as<unsigned long long>());
+  CUDA_OK(cudaGetLastError());
 }
 
 int64_t dt_undirected(Ctx* c, int64_t n, const DBuf& lkey, int64_t ml, DBuf& np, DBuf& nc) {

@@ -287,6 +287,8 @@ int64_t dt_replicate(Ctx* c, DEdges& E, int64_t ns, int k, const std::vector<DtA
 void dt_append_dev(Ctx* c, DEdges& E, const DBuf& key, const DBuf& val, int64_t na);
 void dt_append(Ctx* c, DEdges& E, const std::vector<uint64_t>& key, const std::vector<uint64_t>& val);
 void dt_logical(Ctx* c, const DEdges& E, const DBuf& s2o, int64_t n, DBuf& lp, DBuf& ld, DBuf& lw, DBuf* keys);
+// (dst, w) pairs of a device CSR as u64 = w << 32 | dst (host layout of std::pair<int32_t, uint32_t>)
+void dt_pairs(Ctx* c, const DBuf& ld, const DBuf& lw, int64_t m, DBuf& out);
 int64_t dt_undirected(Ctx* c, int64_t n, const DBuf& lkey, int64_t ml, DBuf& np, DBuf& nc);
 void dt_degnorm(Ctx* c, DEdges& E, int64_t ns, int64_t n, const std::vector<uint8_t>& kind, const DBuf& s2o,
                 const std::vector<int32_t>& owner, int64_t th, int64_t f, bool combined, int rule,

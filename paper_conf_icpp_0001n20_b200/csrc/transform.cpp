@@ -388,23 +388,70 @@ void coalesce(const HostCSR& g, int k, int64_t theta_ppm, int wrule, Work& W, Ct
 }
 
 // ---------------------------------------------------------------- §3
-// Mutable logical graph (original ids) with its undirected view U.
+// Mutable logical graph (original ids) with its undirected view U: flat CSR
+// bases (built in one pass, or copied from the device) plus an overlay row per
+// vertex the §3 insertion changed (<= 2 * budget of them), so no per-vertex
+// containers are built or freed for the whole graph.
+template <class T>
+struct Span {
+  const T* p = nullptr;
+  size_t k = 0;
+  Span() = default;
+  Span(const T* p_, size_t k_) : p(p_), k(k_) {}
+  Span(const std::vector<T>& v) : p(v.data()), k(v.size()) {}
+  const T* begin() const { return p; }
+  const T* end() const { return p + k; }
+  size_t size() const { return k; }
+  const T& operator[](size_t i) const { return p[i]; }
+};
+using OutE = std::pair<int32_t, uint32_t>;
 struct Logical {
-  int64_t n;
-  std::vector<std::vector<std::pair<int32_t, uint32_t>>> out;  // sorted by dst
-  std::vector<std::vector<int32_t>> N;                         // sorted neighbours in U
-  std::vector<int64_t> T;                                      // triangles at each vertex
+  int64_t n = 0;
+  std::vector<int64_t> op, np;   // row offsets of the bases [n + 1]
+  std::vector<OutE> oe;          // G_L out-edges (dst, w), rows sorted by dst
+  std::vector<int32_t> ne;       // U neighbours, rows sorted ascending
+  std::vector<int32_t> ovo, ovn; // vertex -> overlay row, or -1 (the base row)
+  std::vector<std::vector<OutE>> xo;
+  std::vector<std::vector<int32_t>> xn;
+  std::vector<int64_t> T;        // triangles at each vertex
 
-  int64_t d(int32_t c) const { return (int64_t)N[c].size(); }
+  void init_overlays() {
+    ovo.assign(n, -1);
+    ovn.assign(n, -1);
+  }
+  Span<OutE> out(int32_t a) const {
+    const int32_t i = ovo[a];
+    return i < 0 ? Span<OutE>(oe.data() + op[a], (size_t)(op[a + 1] - op[a])) : Span<OutE>(xo[i]);
+  }
+  Span<int32_t> N(int32_t c) const {
+    const int32_t i = ovn[c];
+    return i < 0 ? Span<int32_t>(ne.data() + np[c], (size_t)(np[c + 1] - np[c])) : Span<int32_t>(xn[i]);
+  }
+  std::vector<OutE>& out_mut(int32_t a) {
+    if (ovo[a] < 0) {
+      const Span<OutE> b = out(a);
+      ovo[a] = (int32_t)xo.size();
+      xo.emplace_back(b.begin(), b.end());
+    }
+    return xo[ovo[a]];
+  }
+  std::vector<int32_t>& N_mut(int32_t c) {
+    if (ovn[c] < 0) {
+      const Span<int32_t> b = N(c);
+      ovn[c] = (int32_t)xn.size();
+      xn.emplace_back(b.begin(), b.end());
+    }
+    return xn[ovn[c]];
+  }
+
+  int64_t d(int32_t c) const { return (int64_t)N(c).size(); }
   int64_t P(int32_t c) const { int64_t x = d(c); return x * (x - 1) / 2; }
   bool high(int32_t c, int64_t th) const { return (__int128)T[c] * 1000000 > (__int128)th * P(c); }
-  bool adj(int32_t a, int32_t b) const { return std::binary_search(N[a].begin(), N[a].end(), b); }
+  bool adj(int32_t a, int32_t b) const { const auto r = N(a); return std::binary_search(r.begin(), r.end(), b); }
   const uint32_t* outw(int32_t a, int32_t b) const {
-    auto& r = out[a];
+    const auto r = out(a);
     auto it = std::lower_bound(r.begin(), r.end(), std::make_pair(b, 0u),
-                               [](const std::pair<int32_t, uint32_t>& x, const std::pair<int32_t, uint32_t>& y) {
-                                 return x.first < y.first;
-                               });
+                               [](const OutE& x, const OutE& y) { return x.first < y.first; });
     return (it != r.end() && it->first == b) ? &it->second : nullptr;
   }
   // sibling edge a->b for centre c: along a directed 2-path (R23), or any two
@@ -418,7 +465,7 @@ struct Logical {
     const uint32_t* y = outw(b, a);
     return x && y ? std::min(*x, *y) : (x ? *x : *y);
   }
-  static int64_t inter(const std::vector<int32_t>& x, const std::vector<int32_t>& y) {
+  static int64_t inter(Span<int32_t> x, Span<int32_t> y) {
     int64_t r = 0;
     size_t i = 0, j = 0;
     while (i < x.size() && j < y.size()) {
@@ -430,17 +477,15 @@ struct Logical {
   }
   void link(int32_t a, int32_t b, uint32_t w) {
     const bool fresh = !adj(a, b);
-    auto& r = out[a];
+    auto& r = out_mut(a);
     auto it = std::lower_bound(r.begin(), r.end(), std::make_pair(b, 0u),
-                               [](const std::pair<int32_t, uint32_t>& x, const std::pair<int32_t, uint32_t>& y) {
-                                 return x.first < y.first;
-                               });
+                               [](const OutE& x, const OutE& y) { return x.first < y.first; });
     r.insert(it, {b, w});
     if (fresh) {
       // common neighbours gain a triangle; a and b gain |common| each
       int64_t cnt = 0;
       size_t i = 0, j = 0;
-      const auto &x = N[a], &y = N[b];
+      const auto x = N(a), y = N(b);
       while (i < x.size() && j < y.size()) {
         if (x[i] < y[j]) i++;
         else if (x[i] > y[j]) j++;
@@ -448,8 +493,10 @@ struct Logical {
       }
       T[a] += cnt;
       T[b] += cnt;
-      N[a].insert(std::lower_bound(N[a].begin(), N[a].end(), b), b);
-      N[b].insert(std::lower_bound(N[b].begin(), N[b].end(), a), a);
+      auto& na = N_mut(a);
+      na.insert(std::lower_bound(na.begin(), na.end(), b), b);
+      auto& nb = N_mut(b);
+      nb.insert(std::lower_bound(nb.begin(), nb.end(), a), a);
     }
   }
 };
@@ -479,40 +526,61 @@ void build_logical(const Work& W, Logical& L, Ctx* dev) {
   PhaseTimer pt;
   const int64_t n = W.n;
   L.n = n;
-  logical_out(W, L.out);
+  {
+    std::vector<std::vector<OutE>> out;
+    logical_out(W, out);
+    L.op.assign(n + 1, 0);
+    for (int64_t u = 0; u < n; u++) L.op[u + 1] = L.op[u] + (int64_t)out[u].size();
+    L.oe.resize(L.op[n]);
+#pragma omp parallel for schedule(dynamic, 4096)
+    for (int64_t u = 0; u < n; u++) std::copy(out[u].begin(), out[u].end(), L.oe.begin() + L.op[u]);
+    par_free(out);
+  }
   // in-adjacency by counting (CSC of G_L)
   std::vector<int64_t> ip(n + 1, 0);
 #pragma omp parallel for schedule(dynamic, 4096)
-  for (int64_t u = 0; u < n; u++)
-    for (auto& e : L.out[u]) __atomic_fetch_add(&ip[e.first + 1], 1, __ATOMIC_RELAXED);
+  for (int64_t e = 0; e < L.op[n]; e++) __atomic_fetch_add(&ip[L.oe[e].first + 1], 1, __ATOMIC_RELAXED);
   for (int64_t v = 0; v < n; v++) ip[v + 1] += ip[v];
   std::vector<int32_t> isrc(ip[n]);
   std::vector<int64_t> cur(ip.begin(), ip.end() - 1);
 #pragma omp parallel for schedule(dynamic, 4096)
   for (int64_t u = 0; u < n; u++)
-    for (auto& e : L.out[u]) isrc[__atomic_fetch_add(&cur[e.first], 1, __ATOMIC_RELAXED)] = (int32_t)u;
+    for (int64_t e = L.op[u]; e < L.op[u + 1]; e++)
+      isrc[__atomic_fetch_add(&cur[L.oe[e].first], 1, __ATOMIC_RELAXED)] = (int32_t)u;
   pt("logical out+in");
-  L.N.assign(n, {});
+  // U: sorted union of out- and in-neighbours, counted then filled
+  std::vector<int64_t> cnt(n + 1, 0);
+  std::vector<std::vector<int32_t>> tmp(omp_get_max_threads());
 #pragma omp parallel for schedule(dynamic, 4096)
   for (int64_t u = 0; u < n; u++) {
-    auto& v = L.N[u];
-    v.reserve(L.out[u].size() + (ip[u + 1] - ip[u]));
-    for (auto& e : L.out[u]) v.push_back(e.first);
+    auto& v = tmp[omp_get_thread_num()];
+    v.clear();
+    for (int64_t e = L.op[u]; e < L.op[u + 1]; e++) v.push_back(L.oe[e].first);
+    for (int64_t i = ip[u]; i < ip[u + 1]; i++) v.push_back(isrc[i]);
+    std::sort(v.begin(), v.end());
+    cnt[u + 1] = (int64_t)(std::unique(v.begin(), v.end()) - v.begin());
+  }
+  L.np.assign(n + 1, 0);
+  for (int64_t u = 0; u < n; u++) L.np[u + 1] = L.np[u] + cnt[u + 1];
+  L.ne.resize(L.np[n]);
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int64_t u = 0; u < n; u++) {
+    auto& v = tmp[omp_get_thread_num()];
+    v.clear();
+    for (int64_t e = L.op[u]; e < L.op[u + 1]; e++) v.push_back(L.oe[e].first);
     for (int64_t i = ip[u]; i < ip[u + 1]; i++) v.push_back(isrc[i]);
     std::sort(v.begin(), v.end());
     v.erase(std::unique(v.begin(), v.end()), v.end());
+    std::copy(v.begin(), v.end(), L.ne.begin() + L.np[u]);
   }
+  L.init_overlays();
   pt("undirected N");
   if (dev) {
     // N1: the forward-algorithm triangle count on the graph's device
-    std::vector<int64_t> np(n + 1, 0);
-    for (int64_t u = 0; u < n; u++) np[u + 1] = np[u] + (int64_t)L.N[u].size();
-    std::vector<int32_t> nc(std::max<int64_t>(np[n], 1));
-#pragma omp parallel for schedule(dynamic, 4096)
-    for (int64_t u = 0; u < n; u++) std::copy(L.N[u].begin(), L.N[u].end(), nc.begin() + np[u]);
-    pt("flatten U");
     L.T.assign(n, 0);
-    gpu_triangles(dev, n, np.data(), nc.data(), L.T.data());
+    std::vector<int32_t> nc(L.ne);
+    if (nc.empty()) nc.push_back(0);
+    gpu_triangles(dev, n, L.np.data(), nc.data(), L.T.data());
     pt("triangles (GPU)");
     return;
   }
@@ -520,11 +588,11 @@ void build_logical(const Work& W, Logical& L, Ctx* dev) {
   L.T.assign(n, 0);
   std::vector<std::vector<int32_t>> fwd(n);
   auto rank_less = [&](int32_t a, int32_t b) {
-    return L.N[a].size() < L.N[b].size() || (L.N[a].size() == L.N[b].size() && a < b);
+    return L.d(a) < L.d(b) || (L.d(a) == L.d(b) && a < b);
   };
 #pragma omp parallel for schedule(dynamic, 4096)
   for (int64_t u = 0; u < n; u++) {
-    for (int32_t v : L.N[u])
+    for (int32_t v : L.N((int32_t)u))
       if (rank_less((int32_t)u, v)) fwd[u].push_back(v);
     std::sort(fwd[u].begin(), fwd[u].end());
   }
@@ -532,7 +600,6 @@ void build_logical(const Work& W, Logical& L, Ctx* dev) {
   std::vector<int64_t> tl(n, 0);
 #pragma omp parallel
   {
-    std::vector<int64_t> loc;  // per-thread counts for vertices touched
 #pragma omp for schedule(dynamic, 1024)
     for (int64_t u = 0; u < n; u++) {
       for (int32_t v : fwd[u]) {
@@ -601,12 +668,13 @@ void cc_edges(Logical& L, int64_t th, int64_t budget, int wrule, bool und, SmemO
     const int64_t need = (int64_t)(((__int128)th * P) / 1000000) + 1 - L.T[c];
     if (need <= 0) continue;
     if (P - L.T[c] < need) continue;
-    const std::vector<int32_t> Nc = L.N[c];
+    const Span<int32_t> nsp = L.N(c);
+    const std::vector<int32_t> Nc(nsp.begin(), nsp.end());
     std::vector<std::tuple<int64_t, int32_t, int32_t>> pairs;
     for (size_t i = 0; i < Nc.size(); i++)
       for (size_t j = i + 1; j < Nc.size(); j++) {
         const int32_t a = Nc[i], b = Nc[j];
-        if (linkable(c, a, b)) pairs.push_back({-Logical::inter(L.N[a], L.N[b]), a, b});
+        if (linkable(c, a, b)) pairs.push_back({-Logical::inter(L.N(a), L.N(b)), a, b});
       }
     if ((int64_t)pairs.size() < need) continue;
     std::sort(pairs.begin(), pairs.end());
@@ -630,9 +698,10 @@ void cc_edges(Logical& L, int64_t th, int64_t budget, int wrule, bool und, SmemO
       bool any = false;
       for (int32_t c : highs) {
         if (rem <= 0) break;
-        const std::vector<int32_t> Nc = L.N[c];
+        const Span<int32_t> nsp = L.N(c);
+        const std::vector<int32_t> Nc(nsp.begin(), nsp.end());
         std::unordered_map<int32_t, int64_t> intdeg;
-        for (int32_t a : Nc) intdeg[a] = Logical::inter(L.N[a], Nc);
+        for (int32_t a : Nc) intdeg[a] = Logical::inter(L.N(a), Nc);
         std::vector<int32_t> sib(Nc);
         std::sort(sib.begin(), sib.end(), [&](int32_t x, int32_t y) {
           return intdeg[x] != intdeg[y] ? intdeg[x] < intdeg[y] : x < y;
@@ -672,9 +741,10 @@ void subgraphs(const Logical& L, int64_t th, int smax, int smem_iters, SmemOut& 
   std::vector<uint8_t> used(n, 0);
   for (int32_t c : cs) {
     bool free = !used[c];
-    for (int32_t v : L.N[c]) free = free && !used[v];
+    const Span<int32_t> nsp = L.N(c);
+    for (int32_t v : nsp) free = free && !used[v];
     if (!free) continue;
-    std::vector<int32_t> S(L.N[c]);
+    std::vector<int32_t> S(nsp.begin(), nsp.end());
     S.push_back(c);
     std::sort(S.begin(), S.end());
     for (int32_t v : S) used[v] = 1;
@@ -836,8 +906,6 @@ void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out, Ctx* de
     phase("subgraphs");
     for (auto& e : sm.added)
       W.rows[W.owner[std::get<0>(e)]].push_back({W.owner[std::get<1>(e)], std::get<2>(e), ADD_SMEM});
-    par_free(L.out);
-    par_free(L.N);
     phase("smem free");
   }
   std::vector<int32_t> sched;
@@ -1009,30 +1077,26 @@ void transform_device(const HostCSR& g, const gx_knobs& k, SlotGraph& out, Ctx* 
     dT.alloc(dev, sizeof(int64_t) * std::max<int64_t>(n, 1));
     gpu_triangles_dev(dev, n, np.as<int64_t>(), nc.as<int32_t>(), mu, dT.as<unsigned long long>());
     phase("logical+U+tri (GPU)");
-    std::vector<int64_t> hlp(n + 1), hnp(n + 1);
-    std::vector<int32_t> hld(std::max<int64_t>(ml, 1)), hnc(std::max<int64_t>(mu, 1));
-    std::vector<uint32_t> hlw(std::max<int64_t>(ml, 1));
-    L.T.assign(n, 0);
+    // the flat bases straight into the Logical (no per-vertex containers)
+    DBuf pairs;
+    dt_pairs(dev, ld, lw, ml, pairs);
+    ld.reset();
+    lw.reset();
     cudaStream_t st = dev->stream;
-    CUDA_OK(cudaMemcpyAsync(hlp.data(), lp.p, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost, st));
-    CUDA_OK(cudaMemcpyAsync(hnp.data(), np.p, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost, st));
-    if (ml) {
-      CUDA_OK(cudaMemcpyAsync(hld.data(), ld.p, sizeof(int32_t) * ml, cudaMemcpyDeviceToHost, st));
-      CUDA_OK(cudaMemcpyAsync(hlw.data(), lw.p, sizeof(uint32_t) * ml, cudaMemcpyDeviceToHost, st));
-    }
-    if (mu) CUDA_OK(cudaMemcpyAsync(hnc.data(), nc.p, sizeof(int32_t) * mu, cudaMemcpyDeviceToHost, st));
+    L.op.resize(n + 1);
+    L.np.resize(n + 1);
+    L.oe.resize(ml);
+    L.ne.resize(mu);
+    L.T.assign(n, 0);
+    static_assert(sizeof(OutE) == 8, "OutE is {int32 dst, uint32 w}");
+    CUDA_OK(cudaMemcpyAsync(L.op.data(), lp.p, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost, st));
+    CUDA_OK(cudaMemcpyAsync(L.np.data(), np.p, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost, st));
+    if (ml) CUDA_OK(cudaMemcpyAsync(L.oe.data(), pairs.p, sizeof(OutE) * ml, cudaMemcpyDeviceToHost, st));
+    if (mu) CUDA_OK(cudaMemcpyAsync(L.ne.data(), nc.p, sizeof(int32_t) * mu, cudaMemcpyDeviceToHost, st));
     if (n) CUDA_OK(cudaMemcpyAsync(L.T.data(), dT.p, sizeof(int64_t) * n, cudaMemcpyDeviceToHost, st));
     CUDA_OK(cudaStreamSynchronize(st));
-    lp.reset(); ld.reset(); lw.reset(); np.reset(); nc.reset(); dT.reset();
-    L.out.assign(n, {});
-    L.N.assign(n, {});
-#pragma omp parallel for schedule(dynamic, 4096)
-    for (int64_t u = 0; u < n; u++) {
-      auto& r = L.out[u];
-      r.reserve(hlp[u + 1] - hlp[u]);
-      for (int64_t e = hlp[u]; e < hlp[u + 1]; e++) r.push_back({hld[e], hlw[e]});
-      L.N[u].assign(hnc.begin() + hnp[u], hnc.begin() + hnp[u + 1]);
-    }
+    lp.reset(); pairs.reset(); np.reset(); nc.reset(); dT.reset();
+    L.init_overlays();
     phase("logical to host");
     const int64_t th = ppm(k.cc_threshold);
     const int64_t budget = k.added_edge_budget >= 0 ? k.added_edge_budget : g.m / 100;
@@ -1048,9 +1112,7 @@ void transform_device(const HostCSR& g, const gx_knobs& k, SlotGraph& out, Ctx* 
       av.push_back((uint64_t)std::get<2>(e) | ((uint64_t)ADD_SMEM << 32));
     }
     dt_append(dev, E, ak, av);
-    par_free(L.out);
-    par_free(L.N);
-    phase("smem append+free");
+    phase("smem append");
   }
   std::vector<int32_t> sched;
   int64_t added_dn = 0;
