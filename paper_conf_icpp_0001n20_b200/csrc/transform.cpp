@@ -465,16 +465,31 @@ struct Logical {
     const uint32_t* y = outw(b, a);
     return x && y ? std::min(*x, *y) : (x ? *x : *y);
   }
-  static int64_t inter(Span<int32_t> x, Span<int32_t> y) {
+  // |x ∩ y| of two sorted lists; f(v) for every common v.  A hub's list is
+  // 10^5 long on RMAT, so a short list is searched into a long one
+  // (O(|x| log |y|)) instead of merged (O(|x| + |y|)): the same set
+  template <class F>
+  static int64_t common(Span<int32_t> x, Span<int32_t> y, F&& f) {
+    if (x.size() > y.size()) std::swap(x, y);
     int64_t r = 0;
+    if (x.size() * 16 < y.size()) {
+      const int32_t* lo = y.begin();
+      for (int32_t v : x) {
+        lo = std::lower_bound(lo, y.end(), v);
+        if (lo == y.end()) break;
+        if (*lo == v) { f(v); r++; }
+      }
+      return r;
+    }
     size_t i = 0, j = 0;
     while (i < x.size() && j < y.size()) {
       if (x[i] < y[j]) i++;
       else if (x[i] > y[j]) j++;
-      else { r++; i++; j++; }
+      else { f(x[i]); r++; i++; j++; }
     }
     return r;
   }
+  static int64_t inter(Span<int32_t> x, Span<int32_t> y) { return common(x, y, [](int32_t) {}); }
   void link(int32_t a, int32_t b, uint32_t w) {
     const bool fresh = !adj(a, b);
     auto& r = out_mut(a);
@@ -483,14 +498,7 @@ struct Logical {
     r.insert(it, {b, w});
     if (fresh) {
       // common neighbours gain a triangle; a and b gain |common| each
-      int64_t cnt = 0;
-      size_t i = 0, j = 0;
-      const auto x = N(a), y = N(b);
-      while (i < x.size() && j < y.size()) {
-        if (x[i] < y[j]) i++;
-        else if (x[i] > y[j]) j++;
-        else { T[x[i]]++; cnt++; i++; j++; }
-      }
+      const int64_t cnt = common(N(a), N(b), [&](int32_t v) { T[v]++; });
       T[a] += cnt;
       T[b] += cnt;
       auto& na = N_mut(a);
@@ -634,6 +642,7 @@ struct SmemOut {
 
 // CC edge insertion: case 1 (R22) then case 2 (R24, R25); budget in directed edges (R26)
 void cc_edges(Logical& L, int64_t th, int64_t budget, int wrule, bool und, SmemOut& out) {
+  PhaseTimer pt;
   const int64_t n = L.n;
   int64_t rem = budget;
   auto linkable = [&](int32_t c, int32_t a, int32_t b) {
@@ -661,6 +670,7 @@ void cc_edges(Logical& L, int64_t th, int64_t budget, int wrule, bool und, SmemO
     }
   }
   std::sort(cands.begin(), cands.end());
+  pt("case-1 centres");
   for (auto& cn : cands) {
     if (rem <= 0) break;
     const int32_t c = cn.second;
@@ -684,6 +694,7 @@ void cc_edges(Logical& L, int64_t th, int64_t budget, int wrule, bool und, SmemO
       if (linkable(c, a, b)) do_link(c, a, b);
     }
   }
+  pt("case 1");
   // case 2
   if (rem > 0) {
     std::vector<int32_t> highs;
