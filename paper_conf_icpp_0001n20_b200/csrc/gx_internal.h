@@ -117,7 +117,10 @@ struct SellLayout {
 // [q[b], q[nb*nb + b]); segment (s, b) = [q[s*nb + b], q[(s+1)*nb + b]).
 // val f32[m_pad] carries x_u/D_u along every edge (written by the source
 // block's scatter, read by the sink bin).
-constexpr int PB_R = 16384;
+#ifndef GX_PB_R
+#define GX_PB_R 16384
+#endif
+constexpr int PB_R = GX_PB_R;
 constexpr int PB_PAD = 8;
 struct PbLayout {
   int64_t nb = 0, m_pad = 0;

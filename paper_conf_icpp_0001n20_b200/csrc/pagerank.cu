@@ -363,8 +363,14 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell2(PrArgs a) {
 // running one bin's (1) beside the previous bin's (3) on separate warps was
 // 5 % slower per sweep and needed 17 sweeps instead of 15, the scatter lagging
 // one bin behind -- profiles/README.md "third session")
-constexpr int PB_THREADS = 1024;
-constexpr int PB_CTAS_PER_SM = 1;
+#ifndef GX_PB_THREADS
+#define GX_PB_THREADS 1024
+#endif
+#ifndef GX_PB_CPS
+#define GX_PB_CPS 1
+#endif
+constexpr int PB_THREADS = GX_PB_THREADS;
+constexpr int PB_CTAS_PER_SM = GX_PB_CPS;
 #ifndef GX_PB_PRODUCER
 #define GX_PB_PRODUCER 1    // measured: 774 vs 813 us per sweep (RMAT-24)
 #endif
