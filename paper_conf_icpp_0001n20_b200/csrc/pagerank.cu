@@ -411,6 +411,7 @@ struct PbArgs {
   const uint16_t* dst_loc;
   float* val;
   int64_t nb;
+  int pack;   // (3) in packed steps (pb_scatter_packed): segments average fewer than PB_PACK_BELOW entries
 };
 
 __device__ __forceinline__ float4 ld_cg_f4(const float* p) {
@@ -636,7 +637,121 @@ __device__ __forceinline__ void pb_scatter_async(const PbArgs& p, const float* s
   cp_async_wait<0>();
 }
 
-template <bool SLOTS>
+// (3) with packed steps: a warp's 32 segments are treated as one run of
+// 8-entry groups (a warp-wide inclusive scan of their group counts), and each
+// step hands the next 32 groups to the 32 lanes whatever segment they fall in
+// (a 5-round shuffle search of the scan), so short segments no longer leave
+// most lanes of a step idle.  RMAT-24 averages 256 entries per segment, RMAT-26
+// 64 (16.8M segments): one step per segment used 25 % of the lanes there.
+// Loads asynchronous as in pb_scatter_async (cp.async into the warp's slice).
+// Measured (profiles/r2/pb_pack_variants.txt, PageRank to 1e-9, per sweep):
+// RMAT-26 (64 entries per segment) 3.72 -> 3.52 ms, RMAT-24 (256) 788 -> 783 us,
+// RMAT-22 (1024) 214 -> 218 us: packed below 512 entries per segment
+#ifndef GX_PB_PACK
+#define GX_PB_PACK 1
+#endif
+#ifndef GX_PB_PACK_BELOW
+#define GX_PB_PACK_BELOW 512
+#endif
+template <int DEPTH>
+__device__ __forceinline__ void pb_scatter_packed(const PbArgs& p, const float* s_c, const uint32_t* r0,
+                                                  const uint32_t* r1, uint32_t lo0, uint32_t hi0, uint64_t pf,
+                                                  uint4* stage /* this warp's DEPTH x 32 uint4 */) {
+  const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
+  constexpr unsigned NW = PB_THREADS / 32;
+  const int64_t nb = p.nb;
+  int64_t j0 = (int64_t)warp * 32;
+  uint32_t lo = 0, incl = 0, G = 0, s0 = 0;
+  // the segment holding group s0 (warp-uniform): its start, first group and end
+  uint32_t ck = 0, clo = 0, cex = 0, cend = 0;
+  auto locate = [&]() {
+    ck = __ffs(__ballot_sync(FULL, incl > s0)) - 1;
+    clo = __shfl_sync(FULL, lo, ck);
+    cend = __shfl_sync(FULL, incl, ck);
+    cex = __shfl_sync(FULL, incl, ck > 0 ? ck - 1 : 0);
+    if (ck == 0) cex = 0u;
+  };
+  // the next 32-segment group holding any entry: lo = this lane's segment
+  // start, incl = inclusive scan of the group counts, G = their total
+  auto load_group = [&]() -> bool {
+    while (j0 < nb) {
+      const int64_t j = j0 + lane;
+      uint32_t l = 0, h = 0;
+      if (j < nb) {
+        if (j0 < 32 * (int64_t)NW) {   // segment j = threadIdx.x: the caller's registers
+          l = lo0;
+          h = hi0;
+        } else {
+          l = __ldg(r0 + j);
+          h = __ldg(r1 + j);
+        }
+      }
+      lo = l;
+      incl = warp_incl_scan_u32((h - l) >> 3);
+      G = __shfl_sync(FULL, incl, 31);
+      s0 = 0;
+      if (G) {
+        locate();
+        return true;
+      }
+      j0 += 32 * NW;
+    }
+    return false;
+  };
+  bool more = load_group();
+  uint32_t pe[DEPTH];
+  int pending = 0;
+  auto refill = [&](int s) {
+    pe[s] = 0xffffffffu;
+    if (more) {
+      const uint32_t g = s0 + lane;
+      uint32_t e;
+      if (s0 + 32 <= cend) {   // the whole step inside one segment (long segments)
+        e = clo + 8u * (g - cex);
+      } else {                 // several segments: the segment of each lane's group by a shuffle search
+        const uint32_t gq = min(g, G - 1u);
+        int k = 0;
+#pragma unroll
+        for (int sft = 16; sft; sft >>= 1) {
+          const uint32_t v = __shfl_sync(FULL, incl, k + sft - 1);
+          if (v <= gq) k += sft;
+        }
+        uint32_t ex = __shfl_sync(FULL, incl, k > 0 ? k - 1 : 0);
+        if (k == 0) ex = 0u;
+        e = __shfl_sync(FULL, lo, k) + 8u * (gq - ex);
+      }
+      if (g < G) {
+        pe[s] = e;
+        cp_async16(stage + s * 32 + lane, p.src_loc + e, pf);
+      }
+      pending++;
+      s0 += 32;
+      if (s0 >= G) {
+        j0 += 32 * NW;
+        more = load_group();
+      } else if (s0 >= cend) {
+        locate();
+      }
+    }
+    cp_async_commit();
+  };
+#pragma unroll
+  for (int s = 0; s < DEPTH; s++) refill(s);
+  while (pending) {
+#pragma unroll
+    for (int s = 0; s < DEPTH; s++) {
+      cp_async_wait<DEPTH - 1>();
+      if (pe[s] != 0xffffffffu) pb_put8(p.val + pe[s], s_c, stage[s * 32 + lane]);
+      if (pending) pending--;   // stage s's step (issued in order) is consumed
+      refill(s);
+    }
+  }
+  cp_async_wait<0>();
+}
+
+// PACK: (3) in packed steps (one kernel per scatter: a run-time choice between
+// the two inside one kernel measured an illegal-instruction fault on B200)
+template <bool SLOTS, bool PACK>
 __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, PbArgs p) {
   extern __shared__ __align__(16) unsigned char pb_smem[];
   uint32_t* acc_lo = reinterpret_cast<uint32_t*>(pb_smem);
@@ -795,7 +910,10 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
     __syncthreads();
     // (3) scatter the new terms along block b's segments
     if (GX_PB_SASYNC) {
-      pb_scatter_async<PB_SDEPTH>(p, s_c, r0, r1, lo0, hi0, pf, reinterpret_cast<uint4*>(ring) + warp * PB_SDEPTH * 32);
+      if (PACK)
+        pb_scatter_packed<PB_SDEPTH>(p, s_c, r0, r1, lo0, hi0, pf, reinterpret_cast<uint4*>(ring) + warp * PB_SDEPTH * 32);
+      else
+        pb_scatter_async<PB_SDEPTH>(p, s_c, r0, r1, lo0, hi0, pf, reinterpret_cast<uint4*>(ring) + warp * PB_SDEPTH * 32);
       // the ring's next writes are the bulk copies (async proxy)
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     } else
@@ -813,6 +931,7 @@ constexpr size_t PB_INIT_SMEM = (size_t)(PB_R + 8) * 4 + (GX_PB_SASYNC ? (size_t
 #ifndef GX_PB_INIT_MINB
 #define GX_PB_INIT_MINB 1    // measured: 1 and 2 (32 registers, spill) tie (profiles/r1f/init_variants.txt)
 #endif
+template <bool PACK>
 __global__ void __launch_bounds__(PB_THREADS, GX_PB_INIT_MINB) k_pb_init_val(PbArgs p, const float* __restrict__ contrib,
                                                                int64_t n_slots) {
   extern __shared__ __align__(16) float pb_init_s[];
@@ -826,10 +945,14 @@ __global__ void __launch_bounds__(PB_THREADS, GX_PB_INIT_MINB) k_pb_init_val(PbA
     const uint32_t* r1 = r0 + p.nb;
     const uint32_t lo0 = threadIdx.x < p.nb ? r0[threadIdx.x] : 0u, hi0 = threadIdx.x < p.nb ? r1[threadIdx.x] : 0u;
     __syncthreads();
-    if (GX_PB_SASYNC)
-      pb_scatter_async<PB_INIT_SDEPTH>(p, s_c, r0, r1, lo0, hi0, pf,
-                                       reinterpret_cast<uint4*>(s_c + PB_R + 8) + (threadIdx.x >> 5) * PB_INIT_SDEPTH * 32);
-    else
+    if (GX_PB_SASYNC) {
+      if (PACK)
+        pb_scatter_packed<PB_INIT_SDEPTH>(p, s_c, r0, r1, lo0, hi0, pf,
+                                          reinterpret_cast<uint4*>(s_c + PB_R + 8) + (threadIdx.x >> 5) * PB_INIT_SDEPTH * 32);
+      else
+        pb_scatter_async<PB_INIT_SDEPTH>(p, s_c, r0, r1, lo0, hi0, pf,
+                                         reinterpret_cast<uint4*>(s_c + PB_R + 8) + (threadIdx.x >> 5) * PB_INIT_SDEPTH * 32);
+    } else
       pb_scatter(p, s_c, r0, r1, lo0, hi0, pf);
     __syncthreads();
   }
@@ -1514,11 +1637,16 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
     pb.dst_loc = d.pr_pb.dst_loc.as<uint16_t>();
     pb.val = d.pr_pb.val.as<float>();
     pb.nb = d.pr_pb.nb;
+    pb.pack = (double)d.pr_pb.m_pad < (double)GX_PB_PACK_BELOW * (double)pb.nb * (double)pb.nb ? 1 : 0;
+    if (const char* e = getenv("GX_PB_PACK_FORCE")) pb.pack = atoi(e) != 0;   // tests: either path on any graph
     // the opt-in is per device (context): set it on every run (cheap), not
     // once per process -- a second GPU in the same process needs it too
-    CUDA_OK(cudaFuncSetAttribute(k_pr_pb<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
-    CUDA_OK(cudaFuncSetAttribute(k_pr_pb<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
-    CUDA_OK(cudaFuncSetAttribute(k_pb_init_val, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_INIT_SMEM));
+    CUDA_OK(cudaFuncSetAttribute(k_pr_pb<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
+    CUDA_OK(cudaFuncSetAttribute(k_pr_pb<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
+    CUDA_OK(cudaFuncSetAttribute(k_pr_pb<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
+    CUDA_OK(cudaFuncSetAttribute(k_pr_pb<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_SMEM));
+    CUDA_OK(cudaFuncSetAttribute(k_pb_init_val<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_INIT_SMEM));
+    CUDA_OK(cudaFuncSetAttribute(k_pb_init_val<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PB_INIT_SMEM));
   }
   if (mapping == GX_MAP_TPV) {
     ensure_tpv(g);
@@ -1541,7 +1669,12 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   int gi = grid_for(c, ns);
   if (slots) k_pr_init<true><<<gi, 256, 0, s>>>(a, ns, 1.0 / (double)g->n);
   else k_pr_init<false><<<gi, 256, 0, s>>>(a, ns, 1.0 / (double)g->n);
-  if (mapping == GX_MAP_PB) k_pb_init_val<<<(int)std::min<int64_t>(pb.nb, c->num_sms * 2), PB_THREADS, PB_INIT_SMEM, s>>>(pb, a.contrib[0], ns);
+  const bool pack = GX_PB_PACK && pb.pack;
+  if (mapping == GX_MAP_PB) {
+    const int gi_pb = (int)std::min<int64_t>(pb.nb, c->num_sms * 2);
+    if (pack) k_pb_init_val<true><<<gi_pb, PB_THREADS, PB_INIT_SMEM, s>>>(pb, a.contrib[0], ns);
+    else k_pb_init_val<false><<<gi_pb, PB_THREADS, PB_INIT_SMEM, s>>>(pb, a.contrib[0], ns);
+  }
   CUDA_OK(cudaGetLastError());
   int launches = mapping == GX_MAP_PB ? 2 : 1;
   const int grid_pb = (int)std::max<int64_t>(1, std::min<int64_t>(pb.nb, (int64_t)c->num_sms * PB_CTAS_PER_SM));
@@ -1562,8 +1695,13 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   auto one_iter = [&](int& nl) {
     kt.begin();
     if (mapping == GX_MAP_PB) {
-      if (slots) k_pr_pb<true><<<grid_pb, PB_THREADS, PB_SMEM, s>>>(a, pb);
-      else k_pr_pb<false><<<grid_pb, PB_THREADS, PB_SMEM, s>>>(a, pb);
+      if (pack) {
+        if (slots) k_pr_pb<true, true><<<grid_pb, PB_THREADS, PB_SMEM, s>>>(a, pb);
+        else k_pr_pb<false, true><<<grid_pb, PB_THREADS, PB_SMEM, s>>>(a, pb);
+      } else {
+        if (slots) k_pr_pb<true, false><<<grid_pb, PB_THREADS, PB_SMEM, s>>>(a, pb);
+        else k_pr_pb<false, false><<<grid_pb, PB_THREADS, PB_SMEM, s>>>(a, pb);
+      }
     } else if (mapping == GX_MAP_TPV) {
       if (async) {
         if (slots) k_pr_tpv<true, true><<<grid_tpv, 256, 0, s>>>(a);

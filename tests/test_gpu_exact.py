@@ -81,10 +81,14 @@ PB_GRAPHS = {   # several 16384-slot blocks each, ragged last block
 
 
 @pytest.mark.parametrize("name", list(PB_GRAPHS))
-def test_pagerank_blocked_multiblock(name):
+@pytest.mark.parametrize("pack", ["0", "1"])
+def test_pagerank_blocked_multiblock(name, pack, monkeypatch):
     """The propagation-blocked pull (GX_MAP_PB) across several source blocks /
     sink bins, incl. a ragged last block, in-hub and out-hub rows, dangling
-    vertices: L1 <= 1e-6 against the oracle; the LB kernel agrees too."""
+    vertices: L1 <= 1e-6 against the oracle; the LB kernel agrees too.  Both
+    scatters: one step per segment, and packed steps that span segments
+    (pb_scatter_packed, forced with GX_PB_PACK_FORCE)."""
+    monkeypatch.setenv("GX_PB_PACK_FORCE", pack)
     raw = PB_GRAPHS[name]()
     g = from_raw(raw)
     want, _ = A.pagerank(graph_to_edgelist(g), tol=1e-14)
