@@ -65,9 +65,11 @@ typedef enum { GX_MERGE_MEAN = 0, GX_MERGE_MIN = 1 } gx_merge;
  * propagation-blocked pull -- the x_u/D_u terms of the sum in P@36969 are
  * streamed along the edges in (source block, sink block) segments and summed
  * in shared memory, so no random global gathers remain; single GPU,
- * asynchronous schedule.  AUTO = PB for PageRank on one GPU when the graph
- * spans at least GX_PB_MIN_BINS_PER_SM blocks of 16384 slots per SM and no §3
- * tiles are present, else LB in exact mode and TPV when §2 or §4 is on. */
+ * asynchronous schedule.  AUTO = the mapping measured fastest on B200 for
+ * every configuration (exact and every knob): PB for PageRank
+ * on one GPU when the graph spans at least GX_PB_MIN_BINS_PER_SM blocks of
+ * 16384 slots per SM (with or without §3 tiles), else LB; LB for every other
+ * algorithm.  TPV stays available as the paper's own mapping. */
 /* VNS (the paper's second workload P@11477-11746: Graffix
  * layouts under another engine's mapping): Tigr-style virtual node splitting
  * on our own kernels -- every slot's out-row is cut into virtual nodes of at
@@ -76,7 +78,7 @@ typedef enum { GX_MERGE_MEAN = 0, GX_MERGE_MIN = 1 } gx_merge;
  * bounded by K.  SSSP; PageRank runs TPV under it (a pull row cannot be split
  * without a combine step). */
 typedef enum { GX_MAP_AUTO = 0, GX_MAP_LB = 1, GX_MAP_TPV = 2, GX_MAP_PB = 3, GX_MAP_VNS = 4 } gx_mapping;
-#define GX_PB_MIN_BINS_PER_SM 3
+#define GX_PB_MIN_BINS_PER_SM 1
 
 /* upload / download flags */
 #define GX_PTRS_HOST 0u       /* pointers are host memory (pageable or pinned)   */

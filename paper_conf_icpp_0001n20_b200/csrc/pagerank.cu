@@ -1565,13 +1565,13 @@ void run_pagerank(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   const bool tiles = d.n_tiles && g->knobs.smem;
   int mapping = o.mapping;
   if (mapping == GX_MAP_AUTO) {
-    // one CTA per SM claims sink bins: with fewer than ~3 bins per SM the last
-    // wave leaves most SMs idle (RMAT-22, 256 bins: 5.5 ms vs LB 4.5 ms;
-    // RMAT-24, 1024 bins: 12.2 vs 16.1 ms)
-    const bool pb_ok = async_ && !tiles && (ns + PB_R - 1) / PB_R >= (int64_t)GX_PB_MIN_BINS_PER_SM * c->num_sms &&
+    // one CTA per SM claims sink bins: with fewer bins than SMs the last wave
+    // leaves SMs idle.  Measured (profiles/r2): RMAT-22 (256 bins) PB 3.83 vs
+    // LB 4.50 ms, RMAT-24 11.7 vs 17.2; with §3 tiles (C3 road) PB 176-395 vs
+    // LB 380-895 and TPV 285-474 ms; §2 / §4 graphs PB best too (knobs tables)
+    const bool pb_ok = async_ && (ns + PB_R - 1) / PB_R >= (int64_t)GX_PB_MIN_BINS_PER_SM * c->num_sms &&
                        !getenv("GX_NO_PB");
-    mapping = pb_ok ? GX_MAP_PB
-                    : (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
+    mapping = pb_ok ? GX_MAP_PB : GX_MAP_LB;
   }
   if (mapping == GX_MAP_VNS) mapping = GX_MAP_TPV;   // a pull row is not split (graffix.h)
   if (P_ranks > 1 || mapping != GX_MAP_PB || tiles) resolve_pending(g);   // GX_ASYNC_UPLOAD: these layouts read {col, w}

@@ -1995,8 +1995,10 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
     return;
   }
   int mapping = o.mapping == GX_MAP_PB ? GX_MAP_LB : o.mapping;   // PB is a PageRank mapping
-  if (mapping == GX_MAP_AUTO)
-    mapping = (g->transformed && (g->knobs.coalesce || g->knobs.degree_norm)) ? GX_MAP_TPV : GX_MAP_LB;
+  // AUTO = LB, measured fastest on every configuration incl. the §2 / §4
+  // graphs (RMAT-22 §2: LB 2.8 vs TPV 8.9 ms; road §2: 116 vs 1246; uniform
+  // §4: 4.2 vs 14.4; profiles/r2/knobs); TPV = the paper's mapping, on request
+  if (mapping == GX_MAP_AUTO) mapping = GX_MAP_LB;
   if (mapping == GX_MAP_TPV) ensure_tpv(g);
   if (mapping == GX_MAP_VNS) ensure_vns(g);
   ensure_heavy_chunks(g);
