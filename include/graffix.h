@@ -307,8 +307,9 @@ gx_status gx_graph_info(gx_graph* g, int64_t* n, int64_t* m);
 /* Paper defaults, all techniques OFF (= exact mode). */
 gx_status gx_knobs_default(gx_knobs* k);
 
-/* Host-side transforms §2 -> §3 -> §4 (composition reading R34) and the
- * device layouts they need.  NULL knobs => exact mode (identity).
+/* The transforms §2 -> §3 -> §4 (composition reading R34) and the device
+ * layouts they need; with a device context the slot graph is built in HBM
+ * (SURVEY §8(f) N1), only the sequential steps run on the host.  NULL knobs => exact mode (identity).
  * Errors: GX_E_INVALID (k not in 1..32, thresholds not in [0,1] except
  * replicate_threshold >= 0, degree_target not in (0,1], smem_max_nodes not
  * in 2..255). */
@@ -318,7 +319,11 @@ gx_status gx_export_sizes(gx_graph* g, gx_export_sizes_t* sizes);
 gx_status gx_export_transformed(gx_graph* g, gx_export_t* out);
 
 /* Run one algorithm to its fixed point on the transformed graph.  Not
- * converging within max_iters is not an error (converged = 0).
+ * converging within max_iters is not an error (converged = 0).  On a
+ * partitioned context (world > 1): SSSP and PageRank sweep the
+ * rank's rows and exchange after every sweep; BC is source-parallel (rank p
+ * takes sources p, p+P, ..., then one allreduce(sum) of bc); SCC and MST run
+ * on every rank's full graph copy.  Every rank returns the whole result.
  * Errors: GX_E_STATE (no graph), GX_E_INVALID (source out of range),
  * GX_E_UNSUPPORTED (SSSP: a shortest-path length reached 2^32-2, the saturation
  * value of the uint32 distances, reading R51; the result is then not valid). */

@@ -16,6 +16,7 @@
 #include <chrono>
 #include <cub/cub.cuh>
 
+#include "dist.h"
 #include "gx_internal.h"
 #include "kernels_common.cuh"
 
@@ -661,6 +662,32 @@ void run_bc(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   GX_CHECK_ARG(o.bc_sources != nullptr && o.n_bc_sources > 0, "BC needs bc_sources (reading R37)");
   for (int64_t i = 0; i < o.n_bc_sources; i++)
     GX_CHECK_ARG(o.bc_sources[i] >= 0 && o.bc_sources[i] < n, "BC source out of range");
+  if (c->world > 1) {
+    // partitioned context (SURVEY §8(e) "BC: source-parallel"): rank p takes the
+    // sources p, p + P, p + 2P, ... on its full graph copy, then ONE
+    // allreduce(sum) of the bc vector; every rank ends with the whole result
+    std::vector<int64_t> mine;
+    for (int64_t i = c->rank; i < o.n_bc_sources; i += c->world) mine.push_back(o.bc_sources[i]);
+    gx_run_opts ol = o;
+    ol.bc_sources = mine.data();
+    ol.n_bc_sources = (int64_t)mine.size();
+    r.bc.alloc(c, sizeof(double) * n);
+    if (mine.empty()) {
+      CUDA_OK(cudaMemsetAsync(r.bc.p, 0, sizeof(double) * n, s));
+      info = gx_run_info{};
+      info.converged = 1;
+    } else {
+      run_bc_batched(g, ol, info, L);
+    }
+    Exch X;
+    X.c = c;
+    X.P = c->world;
+    X.sim = false;
+    X.allreduce({r.bc.p}, n, Dt::F64, Op::SUM);
+    CUDA_OK(cudaStreamSynchronize(s));
+    r.have[GX_BC] = true;
+    return;
+  }
   if (!getenv("GX_BC_SINGLE")) {   // batched sources (default); GX_BC_SINGLE=1: one source at a time
     run_bc_batched(g, o, info, L);
     return;

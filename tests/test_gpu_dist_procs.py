@@ -27,6 +27,7 @@ KNOBS = {
                    degree_norm=True, degsim_threshold=0.5),
 }
 GRAPHS = {"rmat13": lambda: graphgen.rmat(13), "road48": lambda: graphgen.road(48)}
+BC_SOURCES = [0, 7, 100, 1000, 2047]
 
 
 def _free_port():
@@ -55,10 +56,13 @@ def _worker(rank, world, port, gname, kname, out_dir):
     dist_ = G.download("dist")
     b = G.run("pagerank", mapping="lb", tol=1e-11, max_iters=5000, check_every=4)
     rank_ = G.download("rank")
+    # BC source-parallel: 5 sources split 3 / 2 over the ranks, one allreduce(sum)
+    c = G.run("bc", bc_sources=BC_SOURCES)
+    np.save(os.path.join(out_dir, f"bc{rank}.npy"), G.download("bc"))
     np.save(os.path.join(out_dir, f"dist{rank}.npy"), dist_)
     np.save(os.path.join(out_dir, f"rank{rank}.npy"), rank_)
     with open(os.path.join(out_dir, f"info{rank}.json"), "w") as f:
-        json.dump({"sssp": a, "pr": b}, f)
+        json.dump({"sssp": a, "pr": b, "bc": c}, f)
     G.close()
     ctx.close()
     dist.destroy_process_group()
@@ -81,10 +85,13 @@ def test_two_process_partitioned_run(tmp_path, gname, kname):
     want_d = A.sssp_dijkstra(el, sssp_source(g))
     want_x, _ = A.pagerank(el, tol=1e-14)
     infos = [json.load(open(tmp_path / f"info{r}.json")) for r in range(world)]
+    want_bc = A.bc_brandes(el, BC_SOURCES)
     for r in range(world):
         assert np.array_equal(np.load(tmp_path / f"dist{r}.npy"), want_d), r
         assert np.abs(np.load(tmp_path / f"rank{r}.npy") - want_x).sum() <= 1e-6, r
         assert infos[r]["sssp"]["converged"] == 1 and infos[r]["pr"]["converged"] >= 1
+        got_bc = np.load(tmp_path / f"bc{r}.npy")
+        assert np.allclose(got_bc, want_bc, rtol=1e-9, atol=1e-9 * max(1.0, float(np.abs(want_bc).max()))), r
     # the two ranks took the same decisions (same iteration counts) and split the relaxations
     assert infos[0]["sssp"]["iterations"] == infos[1]["sssp"]["iterations"]
     assert infos[0]["pr"]["iterations"] == infos[1]["pr"]["iterations"]
