@@ -322,8 +322,10 @@ gx_status gx_export_transformed(gx_graph* g, gx_export_t* out);
  * converging within max_iters is not an error (converged = 0).  On a
  * partitioned context (world > 1): SSSP and PageRank sweep the
  * rank's rows and exchange after every sweep; BC is source-parallel (rank p
- * takes sources p, p+P, ..., then one allreduce(sum) of bc); SCC and MST run
- * on every rank's full graph copy.  Every rank returns the whole result.
+ * takes sources p, p+P, ..., then one allreduce(sum) of bc); SCC and MST sweep
+ * the rank's share of the logical edges and reduce the per-vertex colours /
+ * per-component proposals over the ranks every round.  Every rank returns the
+ * whole result.
  * Errors: GX_E_STATE (no graph), GX_E_INVALID (source out of range),
  * GX_E_UNSUPPORTED (SSSP: a shortest-path length reached 2^32-2, the saturation
  * value of the uint32 distances, reading R51; the result is then not valid). */

@@ -147,6 +147,142 @@ __global__ void k_scc_final(const int32_t* __restrict__ label, const int32_t* __
   GRID_STRIDE(v, n) out[v] = smin[label[v]];
 }
 
+// ---- partitioned contexts: every rank sweeps its share of the
+// logical edges (a contiguous range of the edge list), the per-vertex state is
+// reduced across ranks after every sweep and the rest runs identically on
+// every rank's full copy.  The transports reduce u32 with MIN / SUM (dist.h),
+// so a max is a min of complements and a u64 min two u32 mins (high word,
+// then the low word among the copies holding the minimum high word).
+__global__ void k_not_u32(uint32_t* __restrict__ a, int64_t n) { GRID_STRIDE(i, n) a[i] = ~a[i]; }
+__global__ void k_u8_to_u32(const uint8_t* __restrict__ a, uint32_t* __restrict__ b, int64_t n) {
+  GRID_STRIDE(i, n) b[i] = a[i];
+}
+__global__ void k_u32_to_u8(const uint32_t* __restrict__ b, uint8_t* __restrict__ a, int64_t n) {
+  GRID_STRIDE(i, n) a[i] = b[i] ? 1 : 0;
+}
+__global__ void k_u64_hi(const unsigned long long* __restrict__ k, uint32_t* __restrict__ hi, int64_t n) {
+  GRID_STRIDE(i, n) hi[i] = (uint32_t)(k[i] >> 32);
+}
+__global__ void k_u64_lo(const unsigned long long* __restrict__ k, const uint32_t* __restrict__ hi,
+                         uint32_t* __restrict__ lo, int64_t n) {
+  GRID_STRIDE(i, n) lo[i] = (uint32_t)(k[i] >> 32) == hi[i] ? (uint32_t)k[i] : 0xFFFFFFFFu;
+}
+__global__ void k_u64_join(unsigned long long* __restrict__ k, const uint32_t* __restrict__ hi,
+                           const uint32_t* __restrict__ lo, int64_t n) {
+  GRID_STRIDE(i, n) k[i] = ((unsigned long long)hi[i] << 32) | lo[i];
+}
+__global__ void k_iota_from(uint32_t* __restrict__ a, int64_t n, uint32_t base) {
+  GRID_STRIDE(i, n) a[i] = base + (uint32_t)i;
+}
+
+static Exch rank_exch(Ctx* c) {
+  Exch X;
+  X.c = c;
+  X.P = c->world;
+  X.sim = false;
+  return X;
+}
+// this rank's share [lo, hi) of the logical edges
+static void rank_edges(Ctx* c, int64_t m, int64_t& lo, int64_t& hi) {
+  lo = m * c->rank / c->world;
+  hi = m * (c->rank + 1) / c->world;
+}
+// a u32 flag summed over the ranks
+static int sum_flag(Exch& X, int* flag, cudaStream_t s) {
+  X.allreduce({flag}, 1, Dt::U32, Op::SUM);
+  int h = 0;
+  CUDA_OK(cudaMemcpyAsync(&h, flag, 4, cudaMemcpyDeviceToHost, s));
+  CUDA_OK(cudaStreamSynchronize(s));
+  return h;
+}
+
+static void run_scc_dist(gx_graph* g, gx_run_info& info, LG L) {
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  RunState& r = g->rs;
+  const int64_t n = L.n;
+  Exch X = rank_exch(c);
+  int64_t e0_, e1_;
+  rank_edges(c, L.m, e0_, e1_);
+  LG Lr = L;   // this rank's edges
+  Lr.adj = L.adj + e0_;
+  Lr.esrc = L.esrc + e0_;
+  Lr.m = e1_ - e0_;
+  r.label.alloc(c, sizeof(int32_t) * n);
+  r.label2.alloc(c, sizeof(int32_t) * n);
+  r.comp.alloc(c, sizeof(uint32_t) * n);
+  r.changed.alloc(c, 64);
+  DBuf vis, vis32;
+  vis.alloc(c, n);
+  vis32.alloc(c, sizeof(uint32_t) * n);
+  int32_t* label = r.label.as<int32_t>();
+  uint32_t* color = r.comp.as<uint32_t>();
+  int* changed = r.changed.as<int>();
+  unsigned long long* left = reinterpret_cast<unsigned long long*>(r.changed.as<char>() + 8);
+  const int gn = grid_for(c, n), ge = grid_for(c, std::max<int64_t>(Lr.m, 1));
+  cudaEvent_t ev0, ev1;
+  CUDA_OK(cudaEventCreate(&ev0));
+  CUDA_OK(cudaEventCreate(&ev1));
+  CUDA_OK(cudaEventRecord(ev0, s));
+  CUDA_OK(cudaMemsetAsync(label, 0xFF, sizeof(int32_t) * n, s));
+  int launches = 0, rounds = 0;
+  int64_t edges = 0;
+  while (true) {
+    k_scc_color_init<<<gn, 256, 0, s>>>(label, color, vis.as<uint8_t>(), n);
+    launches++;
+    for (;;) {   // forward max-colour rounds: this rank's edges, then the max over the ranks
+      CUDA_OK(cudaMemsetAsync(changed, 0, 4, s));
+      if (Lr.m) k_scc_fw<<<ge, 256, 0, s>>>(Lr, label, color, changed);
+      k_not_u32<<<gn, 256, 0, s>>>(color, n);
+      X.allreduce({color}, n, Dt::U32, Op::MIN);
+      k_not_u32<<<gn, 256, 0, s>>>(color, n);
+      launches += 3;
+      rounds++;
+      edges += Lr.m;
+      if (!sum_flag(X, changed, s)) break;
+    }
+    k_scc_roots<<<gn, 256, 0, s>>>(label, color, vis.as<uint8_t>(), n);
+    launches++;
+    for (;;) {   // backward closure rounds: this rank's edges, then the OR over the ranks
+      CUDA_OK(cudaMemsetAsync(changed, 0, 4, s));
+      if (Lr.m) k_scc_bw<<<ge, 256, 0, s>>>(Lr, label, color, vis.as<uint8_t>(), changed);
+      k_u8_to_u32<<<gn, 256, 0, s>>>(vis.as<uint8_t>(), vis32.as<uint32_t>(), n);
+      X.allreduce({vis32.p}, n, Dt::U32, Op::SUM);
+      k_u32_to_u8<<<gn, 256, 0, s>>>(vis32.as<uint32_t>(), vis.as<uint8_t>(), n);
+      launches += 3;
+      rounds++;
+      edges += Lr.m;
+      if (!sum_flag(X, changed, s)) break;
+    }
+    unsigned long long hl = 0;   // labels and vis agree on every rank: so does the count
+    CUDA_OK(cudaMemsetAsync(left, 0, 8, s));
+    k_scc_assign<<<gn, 256, 0, s>>>(label, color, vis.as<uint8_t>(), n, left);
+    launches++;
+    CUDA_OK(cudaMemcpyAsync(&hl, left, 8, cudaMemcpyDeviceToHost, s));
+    CUDA_OK(cudaStreamSynchronize(s));
+    if (hl == 0) break;
+  }
+  DBuf smin;
+  smin.alloc(c, sizeof(int32_t) * n);
+  CUDA_OK(cudaMemsetAsync(smin.p, 0x7F, sizeof(int32_t) * n, s));
+  k_scc_min<<<gn, 256, 0, s>>>(label, smin.as<int32_t>(), n);
+  k_scc_final<<<gn, 256, 0, s>>>(label, smin.as<int32_t>(), r.label2.as<int32_t>(), n);
+  launches += 2;
+  CUDA_OK(cudaEventRecord(ev1, s));
+  CUDA_OK(cudaEventSynchronize(ev1));
+  float ms = 0;
+  CUDA_OK(cudaEventElapsedTime(&ms, ev0, ev1));
+  cudaEventDestroy(ev0);
+  cudaEventDestroy(ev1);
+  info.iterations = rounds;
+  info.converged = 1;
+  info.loop_ms = ms;
+  info.edges_scanned = edges;
+  info.bytes_model = edges * 16;
+  info.kernel_launches = launches;
+  r.have[GX_SCC] = true;
+}
+
 void run_scc(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   Ctx* c = g->ctx;
   cudaStream_t s = c->stream;
@@ -154,6 +290,10 @@ void run_scc(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   RunState& r = g->rs;
   const int64_t n = L.n;
   GX_CHECK_ARG(n > 0, "empty graph");
+  if (c->world > 1) {
+    run_scc_dist(g, info, L);
+    return;
+  }
   r.label.alloc(c, sizeof(int32_t) * n);
   r.label2.alloc(c, sizeof(int32_t) * n);
   r.comp.alloc(c, sizeof(uint32_t) * n);
@@ -306,6 +446,108 @@ __global__ void k_mst_relabel(uint32_t* __restrict__ comp, const uint32_t* __res
 }
 __global__ void k_iota_u32(uint32_t* __restrict__ a, int64_t n) { GRID_STRIDE(i, n) a[i] = (uint32_t)i; }
 
+// Borůvka on a partitioned context: each rank proposes the lightest edge of
+// every component over ITS active edges, the proposals are min-reduced over the
+// ranks (two u32 mins: weight word, then the edge id among the copies holding
+// the minimum weight), and hooking / pointer jumping / relabelling run
+// identically on every rank's full copy; each rank compacts its own edges
+static void run_mst_dist(gx_graph* g, gx_run_info& info, LG L) {
+  Ctx* c = g->ctx;
+  cudaStream_t s = c->stream;
+  RunState& r = g->rs;
+  const int64_t n = L.n;
+  Exch X = rank_exch(c);
+  int64_t e0_, e1_;
+  rank_edges(c, L.m, e0_, e1_);
+  r.comp.alloc(c, sizeof(uint32_t) * n);
+  r.mst_best.alloc(c, sizeof(unsigned long long) * n);
+  r.changed.alloc(c, 64);
+  DBuf parent, hi, lo;
+  parent.alloc(c, sizeof(uint32_t) * n);
+  hi.alloc(c, sizeof(uint32_t) * n);
+  lo.alloc(c, sizeof(uint32_t) * n);
+  uint32_t* comp = r.comp.as<uint32_t>();
+  unsigned long long* best = r.mst_best.as<unsigned long long>();
+  int* flag = r.changed.as<int>();
+  unsigned long long* wsum = reinterpret_cast<unsigned long long*>(r.changed.as<char>() + 8);
+  const int gn = grid_for(c, n);
+  cudaEvent_t ev0, ev1;
+  CUDA_OK(cudaEventCreate(&ev0));
+  CUDA_OK(cudaEventCreate(&ev1));
+  CUDA_OK(cudaEventRecord(ev0, s));
+  k_iota_u32<<<gn, 256, 0, s>>>(comp, n);
+  CUDA_OK(cudaMemsetAsync(wsum, 0, 8, s));
+  int launches = 1, rounds = 0;
+  int64_t edges = 0;
+  DBuf act[2], nsel, stmp;
+  int64_t na = e1_ - e0_;
+  act[0].alloc(c, sizeof(uint32_t) * std::max<int64_t>(na, 1));
+  act[1].alloc(c, sizeof(uint32_t) * std::max<int64_t>(na, 1));
+  nsel.alloc(c, 8);
+  if (na) k_iota_from<<<grid_for(c, na), 256, 0, s>>>(act[0].as<uint32_t>(), na, (uint32_t)e0_);
+  int cur = 0;
+  while (true) {
+    CUDA_OK(cudaMemsetAsync(best, 0xFF, sizeof(unsigned long long) * n, s));
+    CUDA_OK(cudaMemsetAsync(flag, 0, 4, s));
+    if (na)
+      k_mst_best<<<grid_for(c, na), 256, 0, s>>>(L, act[cur].as<uint32_t>(), na, comp, best, flag);
+    k_u64_hi<<<gn, 256, 0, s>>>(best, hi.as<uint32_t>(), n);
+    X.allreduce({hi.p}, n, Dt::U32, Op::MIN);
+    k_u64_lo<<<gn, 256, 0, s>>>(best, hi.as<uint32_t>(), lo.as<uint32_t>(), n);
+    X.allreduce({lo.p}, n, Dt::U32, Op::MIN);
+    k_u64_join<<<gn, 256, 0, s>>>(best, hi.as<uint32_t>(), lo.as<uint32_t>(), n);
+    edges += na;
+    rounds++;
+    launches += 4;
+    if (!sum_flag(X, flag, s)) break;
+    k_mst_hook<<<gn, 256, 0, s>>>(L, comp, best, parent.as<uint32_t>(), n);
+    k_mst_resolve<<<gn, 256, 0, s>>>(comp, best, parent.as<uint32_t>(), n, wsum);
+    k_mst_root<<<gn, 256, 0, s>>>(comp, best, parent.as<uint32_t>(), n);
+    launches += 3;
+    for (;;) {
+      int ch = 0;
+      CUDA_OK(cudaMemsetAsync(flag, 0, 4, s));
+      k_mst_jump<<<gn, 256, 0, s>>>(parent.as<uint32_t>(), n, flag);
+      launches++;
+      CUDA_OK(cudaMemcpyAsync(&ch, flag, 4, cudaMemcpyDeviceToHost, s));
+      CUDA_OK(cudaStreamSynchronize(s));
+      if (!ch) break;
+    }
+    k_mst_relabel<<<gn, 256, 0, s>>>(comp, parent.as<uint32_t>(), n);
+    launches++;
+    MstCross pred{L.esrc, L.adj, comp};
+    size_t tb = 0;
+    const uint32_t* al = act[cur].as<uint32_t>();
+    CUDA_OK(cub::DeviceSelect::If(nullptr, tb, al, act[cur ^ 1].as<uint32_t>(), nsel.as<int64_t>(), std::max<int64_t>(na, 1), pred, s));
+    stmp.alloc(c, tb);
+    int64_t hn = 0;
+    if (na) {
+      CUDA_OK(cub::DeviceSelect::If(stmp.p, tb, al, act[cur ^ 1].as<uint32_t>(), nsel.as<int64_t>(), na, pred, s));
+      launches++;
+      CUDA_OK(cudaMemcpyAsync(&hn, nsel.p, 8, cudaMemcpyDeviceToHost, s));
+    }
+    CUDA_OK(cudaStreamSynchronize(s));
+    cur ^= 1;
+    na = hn;
+  }
+  unsigned long long W = 0;   // the chosen edges agree on every rank: so does the weight
+  CUDA_OK(cudaMemcpyAsync(&W, wsum, 8, cudaMemcpyDeviceToHost, s));
+  CUDA_OK(cudaEventRecord(ev1, s));
+  CUDA_OK(cudaEventSynchronize(ev1));
+  float ms = 0;
+  CUDA_OK(cudaEventElapsedTime(&ms, ev0, ev1));
+  cudaEventDestroy(ev0);
+  cudaEventDestroy(ev1);
+  r.mst_weight = W;
+  info.iterations = rounds;
+  info.converged = 1;
+  info.loop_ms = ms;
+  info.edges_scanned = edges;
+  info.bytes_model = edges * 20;
+  info.kernel_launches = launches;
+  r.have[GX_MST] = true;
+}
+
 void run_mst(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   Ctx* c = g->ctx;
   cudaStream_t s = c->stream;
@@ -314,6 +556,10 @@ void run_mst(gx_graph* g, const gx_run_opts& o, gx_run_info& info) {
   const int64_t n = L.n;
   GX_CHECK_ARG(n > 0, "empty graph");
   GX_CHECK_ARG(L.m < (int64_t(1) << 32), "too many edges for 32-bit edge keys");
+  if (c->world > 1) {
+    run_mst_dist(g, info, L);
+    return;
+  }
   r.comp.alloc(c, sizeof(uint32_t) * n);
   r.mst_best.alloc(c, sizeof(unsigned long long) * n);
   r.changed.alloc(c, 64);

@@ -4,7 +4,9 @@ whose collectives go through torch.distributed over gloo.  Everything but the
 transport is the library's partitioned code: rank-local layouts (rows [lo,hi)
 only), the sweeps, the reduce-scatter / allgather / fused scalar exchanges
 and the device-side stop decisions.  SSSP must equal the oracle's Dijkstra
-bit for bit, PageRank be within L1 1e-6 of the oracle -- for exact mode and a
+bit for bit, PageRank be within L1 1e-6 of the oracle, BC (source-parallel)
+within rel 1e-9 of Brandes, SCC labels equal Tarjan's and the MST weight
+Kruskal's (each rank sweeping its share of the edges) -- for exact mode and a
 transformed graph with replica groups, §3 tiles and §4 padding (the
 allreduce + merge branch)."""
 import json
@@ -59,10 +61,15 @@ def _worker(rank, world, port, gname, kname, out_dir):
     # BC source-parallel: 5 sources split 3 / 2 over the ranks, one allreduce(sum)
     c = G.run("bc", bc_sources=BC_SOURCES)
     np.save(os.path.join(out_dir, f"bc{rank}.npy"), G.download("bc"))
+    # SCC (colour rounds, max over the ranks) and MST (Borůvka, min proposals over the ranks)
+    d = G.run("scc")
+    np.save(os.path.join(out_dir, f"scc{rank}.npy"), G.download("label"))
+    e = G.run("mst")
+    mst_w = int(G.download("mst_weight"))
     np.save(os.path.join(out_dir, f"dist{rank}.npy"), dist_)
     np.save(os.path.join(out_dir, f"rank{rank}.npy"), rank_)
     with open(os.path.join(out_dir, f"info{rank}.json"), "w") as f:
-        json.dump({"sssp": a, "pr": b, "bc": c}, f)
+        json.dump({"sssp": a, "pr": b, "bc": c, "scc": d, "mst": e, "mst_w": mst_w}, f)
     G.close()
     ctx.close()
     dist.destroy_process_group()
@@ -86,12 +93,19 @@ def test_two_process_partitioned_run(tmp_path, gname, kname):
     want_x, _ = A.pagerank(el, tol=1e-14)
     infos = [json.load(open(tmp_path / f"info{r}.json")) for r in range(world)]
     want_bc = A.bc_brandes(el, BC_SOURCES)
+    want_scc = A.scc_tarjan(el)
+    want_mst = A.mst_kruskal(el)
     for r in range(world):
         assert np.array_equal(np.load(tmp_path / f"dist{r}.npy"), want_d), r
         assert np.abs(np.load(tmp_path / f"rank{r}.npy") - want_x).sum() <= 1e-6, r
         assert infos[r]["sssp"]["converged"] == 1 and infos[r]["pr"]["converged"] >= 1
         got_bc = np.load(tmp_path / f"bc{r}.npy")
         assert np.allclose(got_bc, want_bc, rtol=1e-9, atol=1e-9 * max(1.0, float(np.abs(want_bc).max()))), r
+        assert np.array_equal(np.load(tmp_path / f"scc{r}.npy").astype(np.int64), want_scc), r
+        assert infos[r]["mst_w"] == want_mst, r
+    # each rank swept its share of the logical edges
+    assert infos[0]["scc"]["iterations"] == infos[1]["scc"]["iterations"]
+    assert infos[0]["mst"]["iterations"] == infos[1]["mst"]["iterations"]
     # the two ranks took the same decisions (same iteration counts) and split the relaxations
     assert infos[0]["sssp"]["iterations"] == infos[1]["sssp"]["iterations"]
     assert infos[0]["pr"]["iterations"] == infos[1]["pr"]["iterations"]
