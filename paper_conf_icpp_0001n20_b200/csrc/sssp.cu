@@ -2281,11 +2281,14 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
     // far pile by scan (sssp_split_dev): no far bitmap, so a relaxation that
     // lands beyond tau issues one reduction (dist) instead of two; the refill
     // reads dist once, coalesced.  Not with windows (a scan of all of dist per
-    // refill, ~10^3 refills on a road grid), merges, §3 tiles, the
-    // light/heavy split or the block mode (they push far bits of their own).
-    // GX_SSSP_FARSCAN=0 keeps the bitmap
+    // refill, ~10^3 refills on a road grid), the light/heavy split or the
+    // block mode (they push far bits of their own).  Merges and §3 local passes
+    // keep it: every value they lower is pushed into the next near frontier
+    // (processed there, at any value), and a value a mean merge raises is at
+    // worst processed once more by a later scan -- any relaxation order
+    // reaches the same fixed point (E1).  GX_SSSP_FARSCAN=0 keeps the bitmap
     const char* fse = getenv("GX_SSSP_FARSCAN");
-    const bool far_scan = !win_h && !d.n_groups && !tiles && !want_lh && L.block_rows == 0 && !(fse && atoi(fse) == 0);
+    const bool far_scan = !win_h && !want_lh && L.block_rows == 0 && !(fse && atoi(fse) == 0);
     if (far_scan) {
       L.ax.far = nullptr;
       ax.far = nullptr;   // the dense iteration's gather too
