@@ -2066,7 +2066,10 @@ static void run_sssp_impl(gx_graph* g, const gx_run_opts& o, gx_run_info& info) 
   // refill moves 51 % of the slots with 76 % of the edges (4.85 -> 4.49 ms);
   // uniform and RMAT-22 refills at 40 % lost 0.4 / 0.13 ms
   // (profiles/r2/sssp_dense_sweep.txt)
-  double dense_frac = 0.45;
+  // When dist no longer fits the L2 (RMAT-26: 256 MB), the LB sweep's gathers
+  // go to DRAM and the streamed pass pays from smaller refills: RMAT-26 at
+  // 0.25-0.3: 30.1 -> 26.3 ms (profiles/r2/sssp_dense_rmat26_farscan.txt)
+  double dense_frac = (double)d.n_slots * 4.0 > 96.0 * (1 << 20) ? 0.25 : 0.45;
   if (const char* e = getenv("GX_SSSP_DENSE")) dense_frac = atof(e);
   // (with §3 tiles the dense iteration skips the local pass, schedule-only by
   // E1; with replica groups it merges after the gather, every iteration only)
