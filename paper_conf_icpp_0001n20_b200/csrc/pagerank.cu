@@ -650,6 +650,9 @@ __device__ __forceinline__ void pb_scatter_async(const PbArgs& p, const float* s
 #ifndef GX_PB_PACK
 #define GX_PB_PACK 1
 #endif
+#ifndef GX_PB_XPF
+#define GX_PB_XPF 1   // (2)'s x / D rows prefetched into L2 at bin start
+#endif
 #ifndef GX_PB_PACK_BELOW
 #define GX_PB_PACK_BELOW 512
 #endif
@@ -816,19 +819,20 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
     if (threadIdx.x == 0) {
       if (!PB_PRODUCER)
         for (uint32_t c = 0; c < nch && c < PB_NST; c++) issue(g + c, E0, E1, c);
-      // L2 prefetch for (2) and (3)
-      l2_prefetch_bulk(a.x + base, (uint32_t)nrows * 8u);
-      l2_prefetch_bulk(a.D + base, (uint32_t)nrows * 4u);
-    }
-    // (3)'s first PB_THREADS segment bounds stay in registers
-    uint32_t lo0 = 0, hi0 = 0;
-    for (int64_t j = threadIdx.x; j < nb; j += PB_THREADS) {
-      const uint32_t lo = __ldg(r0 + j), hi = __ldg(r1 + j);
-      if (j == threadIdx.x) {
-        lo0 = lo;
-        hi0 = hi;
+      // L2 prefetch for (2)
+      if (GX_PB_XPF) {
+        l2_prefetch_bulk(a.x + base, (uint32_t)nrows * 8u);
+        l2_prefetch_bulk(a.D + base, (uint32_t)nrows * 4u);
       }
-      if (hi > lo) l2_prefetch_bulk(p.src_loc + lo, (hi - lo) * 2u);
+    }
+    // (3)'s first PB_THREADS segment bounds stay in registers.  (An L2 prefetch
+    // of every segment's source-index run here cost 6 % at RMAT-24 and 12 % at
+    // RMAT-26 -- one bulk prefetch per segment, 16.8M per sweep there:
+    // profiles/r2/pb_srcpf_variants.txt)
+    uint32_t lo0 = 0, hi0 = 0;
+    if (threadIdx.x < nb) {
+      lo0 = __ldg(r0 + threadIdx.x);
+      hi0 = __ldg(r1 + threadIdx.x);
     }
     if (PB_PRODUCER && threadIdx.x >= PB_CONSUMERS) {
       if (threadIdx.x == PB_CONSUMERS)
