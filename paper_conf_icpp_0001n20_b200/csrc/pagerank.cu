@@ -930,7 +930,10 @@ __global__ void __launch_bounds__(PB_THREADS, PB_CTAS_PER_SM) k_pr_pb(PrArgs a, 
 // val[] <- the initial terms contrib_0[u] along every edge: (3) for every
 // source block with s_c = contrib_0 of the block, each warp with a
 // 2-deep cp.async staging slice after s_c
-constexpr int PB_INIT_SDEPTH = 2;
+#ifndef GX_PB_INIT_SDEPTH
+#define GX_PB_INIT_SDEPTH 2
+#endif
+constexpr int PB_INIT_SDEPTH = GX_PB_INIT_SDEPTH;
 constexpr size_t PB_INIT_SMEM = (size_t)(PB_R + 8) * 4 + (GX_PB_SASYNC ? (size_t)(PB_THREADS / 32) * PB_INIT_SDEPTH * 512 : 0);
 #ifndef GX_PB_INIT_MINB
 #define GX_PB_INIT_MINB 1    // measured: 1 and 2 (32 registers, spill) tie (profiles/r1f/init_variants.txt)
