@@ -345,7 +345,7 @@ __global__ void __launch_bounds__(PR_CTA, GX_PR_MINB) k_pr_sell2(PrArgs a) {
 //       16-byte loads and adds each term into a shared-memory accumulator of
 //       its sink row (unsigned 64-bit fixed point, 2^-52 units, kept as two
 //       32-bit words: exact, so the sum does not depend on the order); meanwhile the bin's
-//       x / D rows and block b's scatter segments are bulk-prefetched into L2;
+//       x / D rows are bulk-prefetched into L2;
 //   (2) runs the PR update of the bin's rows (x, delta, dangling and total
 //       mass as in pr_finalize) and keeps the new x/D of every row in shared
 //       memory;
