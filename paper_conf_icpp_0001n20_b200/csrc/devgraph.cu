@@ -202,7 +202,7 @@ static void build_csc_and_tiles(gx_graph* g) {
 // key = bin(v) * nb + block(u) per out-edge (sink-bin major), payload = the
 // two local indices; histogram of keys for the segment offsets
 __global__ void k_pb_pairs(const uint32_t* __restrict__ rp, const uint32_t* __restrict__ colp, uint32_t cstride,
-                           int64_t n, uint32_t nb,
+                           int64_t n, uint32_t nb, uint32_t bblk,
                            uint32_t* __restrict__ key, uint32_t* __restrict__ val, uint32_t* __restrict__ cnt) {
   int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   int lane = threadIdx.x & 31;
@@ -212,17 +212,16 @@ __global__ void k_pb_pairs(const uint32_t* __restrict__ rp, const uint32_t* __re
     const uint32_t bu = (uint32_t)(u / PB_R), lu = (uint32_t)(u % PB_R);
     for (uint32_t e = a + lane; e < b; e += 32) {
       const uint32_t v = colp[(size_t)e * cstride];
-      const uint32_t k = (v / PB_R) * nb + bu;
-      key[e] = k;
+      key[e] = ((v / PB_R) << bblk) | bu;
       val[e] = lu | ((v % PB_R) << 16);
-      atomicAdd(&cnt[k], 1u);
+      atomicAdd(&cnt[(v / PB_R) * nb + bu], 1u);
     }
   }
 }
 // the same with the edge's 8-bit weight in the payload's high word (weights
 // resident and < 2^16): the sort then also yields the weights in blocked order
 __global__ void k_pb_pairs_w(const uint32_t* __restrict__ rp, const uint2* __restrict__ adj, int64_t n, uint32_t nb,
-                             uint32_t* __restrict__ key, unsigned long long* __restrict__ val,
+                             uint32_t bblk, uint32_t* __restrict__ key, unsigned long long* __restrict__ val,
                              uint32_t* __restrict__ cnt) {
   int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   int lane = threadIdx.x & 31;
@@ -232,10 +231,9 @@ __global__ void k_pb_pairs_w(const uint32_t* __restrict__ rp, const uint2* __res
     const uint32_t bu = (uint32_t)(u / PB_R), lu = (uint32_t)(u % PB_R);
     for (uint32_t e = a + lane; e < b; e += 32) {
       const uint2 vw = adj[e];
-      const uint32_t k = (vw.x / PB_R) * nb + bu;
-      key[e] = k;
+      key[e] = ((vw.x / PB_R) << bblk) | bu;
       val[e] = ((unsigned long long)vw.y << 32) | (lu | ((vw.x % PB_R) << 16));
-      atomicAdd(&cnt[k], 1u);
+      atomicAdd(&cnt[(vw.x / PB_R) * nb + bu], 1u);
     }
   }
 }
@@ -246,13 +244,16 @@ __global__ void k_pb_padcnt(const uint32_t* __restrict__ cnt, uint32_t* __restri
     pc[i] = i + 1 < nk ? (cnt[i] + PB_PAD - 1) / PB_PAD * PB_PAD : 0u;
 }
 
-// element i of the sorted order (key k) -> padded position P2[k] + (i - P[k])
+// element i of the sorted order (segment k = bin * nb + block) -> padded
+// position P2[k] + (i - P[k])
 template <class V>
 __global__ void k_pb_place(const uint32_t* __restrict__ key, const V* __restrict__ pay,
                            const uint32_t* __restrict__ P, const uint32_t* __restrict__ P2, uint16_t* __restrict__ sl,
-                           uint16_t* __restrict__ dl, uint16_t* __restrict__ w16, int64_t m) {
+                           uint16_t* __restrict__ dl, uint16_t* __restrict__ w16, int64_t m, uint32_t nb,
+                           uint32_t bblk) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
-    const uint32_t k = key[i];
+    const uint32_t kk = key[i];
+    const uint32_t k = (kk >> bblk) * nb + (kk & ((1u << bblk) - 1u));
     const V p = pay[i];
     const uint32_t pos = P2[k] + ((uint32_t)i - P[k]);
     sl[pos] = (uint16_t)(p & 0xffffu);
@@ -294,6 +295,12 @@ void ensure_pb(gx_graph* g) {
   // blocked PageRank builds from col alone, and SSSP then runs without the
   // dense pass on this graph (it never gathers the weights at random)
   const bool with_w = d.max_w <= 0xffffu && !g->maxw_pending && m > 0;
+  // key = bin << bblk | block; the edges arrive in CSR (= source block) order
+  // and the radix sort is stable, so sorting the bin bits alone yields the
+  // (bin, block) segment order: ceil(log2 nb) bits, 2 passes at RMAT-24/26
+  // instead of 3 over the whole (bin, block) key
+  int bits = 1;
+  while ((int64_t(1) << bits) < nb) bits++;
   DBuf k0, k1, v0, v1, tmp;
   cub::DoubleBuffer<uint32_t> dk, dv;
   cub::DoubleBuffer<unsigned long long> dv64;
@@ -302,32 +309,31 @@ void ensure_pb(gx_graph* g) {
     k1.alloc(c, sizeof(uint32_t) * m);
     v0.alloc(c, (with_w ? 8 : 4) * m);
     v1.alloc(c, (with_w ? 8 : 4) * m);
-    int bits = 1;
-    while ((int64_t(1) << bits) < nb * nb) bits++;
+
     size_t tb = 0;
     dk = cub::DoubleBuffer<uint32_t>(k0.as<uint32_t>(), k1.as<uint32_t>());
     if (with_w) {
       k_pb_pairs_w<<<grid_for(c, n * 32), 256, 0, s>>>(d.rp.as<uint32_t>(), d.adj.as<uint2>(), n, (uint32_t)nb,
-                                                       k0.as<uint32_t>(), v0.as<unsigned long long>(),
+                                                       (uint32_t)bits, k0.as<uint32_t>(), v0.as<unsigned long long>(),
                                                        cnt.as<uint32_t>());
       CUDA_OK(cudaGetLastError());
       dv64 = cub::DoubleBuffer<unsigned long long>(v0.as<unsigned long long>(), v1.as<unsigned long long>());
-      CUDA_OK(cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv64, (int64_t)m, 0, bits, s));
+      CUDA_OK(cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv64, (int64_t)m, bits, 2 * bits, s));
       tmp.alloc(c, tb);
-      CUDA_OK(cub::DeviceRadixSort::SortPairs(tmp.p, tb, dk, dv64, (int64_t)m, 0, bits, s));
+      CUDA_OK(cub::DeviceRadixSort::SortPairs(tmp.p, tb, dk, dv64, (int64_t)m, bits, 2 * bits, s));
     } else {
       // exact mode reads the uploaded col (not the {col, w} pairs, which an
       // asynchronous upload may still be producing)
       const bool ident = d.identity && g->in_col.p;
       k_pb_pairs<<<grid_for(c, n * 32), 256, 0, s>>>(d.rp.as<uint32_t>(),
                                                      ident ? g->in_col.as<uint32_t>() : d.adj.as<uint32_t>(),
-                                                     ident ? 1u : 2u, n, (uint32_t)nb,
+                                                     ident ? 1u : 2u, n, (uint32_t)nb, (uint32_t)bits,
                                                      k0.as<uint32_t>(), v0.as<uint32_t>(), cnt.as<uint32_t>());
       CUDA_OK(cudaGetLastError());
       dv = cub::DoubleBuffer<uint32_t>(v0.as<uint32_t>(), v1.as<uint32_t>());
-      CUDA_OK(cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv, (int64_t)m, 0, bits, s));
+      CUDA_OK(cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv, (int64_t)m, bits, 2 * bits, s));
       tmp.alloc(c, tb);
-      CUDA_OK(cub::DeviceRadixSort::SortPairs(tmp.p, tb, dk, dv, (int64_t)m, 0, bits, s));
+      CUDA_OK(cub::DeviceRadixSort::SortPairs(tmp.p, tb, dk, dv, (int64_t)m, bits, 2 * bits, s));
     }
   }
   k_pb_padcnt<<<grid_for(c, nk), 256, 0, s>>>(cnt.as<uint32_t>(), pc.as<uint32_t>(), nk);
@@ -359,11 +365,13 @@ void ensure_pb(gx_graph* g) {
     if (with_w)
       k_pb_place<unsigned long long><<<grid_for(c, m), 256, 0, s>>>(dk.Current(), dv64.Current(), P.as<uint32_t>(),
                                                                     P2.as<uint32_t>(), L.src_loc.as<uint16_t>(),
-                                                                    L.dst_loc.as<uint16_t>(), d.pb_w16.as<uint16_t>(), m);
+                                                                    L.dst_loc.as<uint16_t>(), d.pb_w16.as<uint16_t>(), m,
+                                                                    (uint32_t)nb, (uint32_t)bits);
     else
       k_pb_place<uint32_t><<<grid_for(c, m), 256, 0, s>>>(dk.Current(), dv.Current(), P.as<uint32_t>(),
                                                           P2.as<uint32_t>(), L.src_loc.as<uint16_t>(),
-                                                          L.dst_loc.as<uint16_t>(), nullptr, m);
+                                                          L.dst_loc.as<uint16_t>(), nullptr, m, (uint32_t)nb,
+                                                          (uint32_t)bits);
   }
   L.q.alloc(c, sizeof(uint32_t) * (nb + 1) * nb);
   k_pb_transpose<<<grid_for(c, (nb + 1) * nb), 256, 0, s>>>(P2.as<uint32_t>(), L.q.as<uint32_t>(), nb);
