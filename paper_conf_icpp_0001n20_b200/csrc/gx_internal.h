@@ -235,6 +235,7 @@ struct gx_graph {
   gx::HostCSR host;            // canonical input (host copy, lazily filled)
   bool host_valid = false;
   gx::DBuf in_rp, in_col, in_w;   // canonical input on device (original ids)
+  int64_t default_src = -1;       // R36 source (max out-degree of the canonical input), cached
   gx::DBuf in_w8;                 // GX_W_U8: the 8-bit weights as copied (widened into in_w)
   int64_t n = 0, m = 0;
   uint32_t max_w = 1;

@@ -1473,6 +1473,7 @@ __global__ void k_argmax_deg(const int64_t* __restrict__ rp, int64_t n, unsigned
 }
 
 int64_t default_source(gx_graph* g) {
+  if (g->default_src >= 0) return g->default_src;   // the canonical input never changes
   Ctx* c = g->ctx;
   DBuf b;
   b.alloc(c, 8);
@@ -1482,7 +1483,8 @@ int64_t default_source(gx_graph* g) {
   unsigned long long h = 0;
   CUDA_OK(cudaMemcpyAsync(&h, b.p, 8, cudaMemcpyDeviceToHost, c->stream));
   CUDA_OK(cudaStreamSynchronize(c->stream));
-  return (int64_t)(0xffffffffull - (h & 0xffffffffull));
+  g->default_src = (int64_t)(0xffffffffull - (h & 0xffffffffull));
+  return g->default_src;
 }
 
 // ---------------------------------------------------------------- driver
