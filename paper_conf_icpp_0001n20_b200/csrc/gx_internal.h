@@ -258,7 +258,7 @@ namespace gx {
 void canonicalize_host(int64_t n, const int64_t* rp, const int32_t* col, const uint32_t* w,
                        HostCSR& out);
 void ensure_host(gx_graph* g);
-// dev: the graph's device context, or null (host-only graph / GX_TRANSFORM_HOST=1):
+// dev: the graph's device context (GX_TRANSFORM=mixed), or null (host-only graph, GX_TRANSFORM=host):
 // with a device the bulk-parallel steps run there (gtransform.cu, N1)
 void transform_host(const HostCSR& g, const gx_knobs& k, SlotGraph& out, Ctx* dev = nullptr);
 void gpu_triangles(Ctx* c, int64_t n, const int64_t* np, const int32_t* nc, int64_t* T);
