@@ -13,6 +13,7 @@
 // thresholds are compared in integer ppm.  The oracle (oracle/transform.py)
 // implements the same readings independently; tests compare the exports.
 #include <omp.h>
+#include <parallel/algorithm>
 
 #include <algorithm>
 #include <chrono>
@@ -640,6 +641,27 @@ struct SmemOut {
   std::vector<std::tuple<int32_t, std::vector<int32_t>, int32_t>> tiles;
 };
 
+// The ids c in [0, n) with pred(c), ascending, collected in parallel (each
+// thread a contiguous static range; the ranges are concatenated in order)
+template <class T, class Pred, class Make>
+std::vector<T> par_filter(int64_t n, Pred pred, Make make) {
+  const int nt = omp_get_max_threads();
+  std::vector<std::vector<T>> loc(nt);
+#pragma omp parallel num_threads(nt)
+  {
+    const int t = omp_get_thread_num();
+    const int64_t a = n * t / nt, b = n * (t + 1) / nt;
+    for (int64_t c = a; c < b; c++)
+      if (pred((int32_t)c)) loc[t].push_back(make((int32_t)c));
+  }
+  size_t tot = 0;
+  for (auto& v : loc) tot += v.size();
+  std::vector<T> out;
+  out.reserve(tot);
+  for (auto& v : loc) out.insert(out.end(), v.begin(), v.end());
+  return out;
+}
+
 // CC edge insertion: case 1 (R22) then case 2 (R24, R25); budget in directed edges (R26)
 void cc_edges(Logical& L, int64_t th, int64_t budget, int wrule, bool und, SmemOut& out) {
   PhaseTimer pt;
@@ -662,14 +684,13 @@ void cc_edges(Logical& L, int64_t th, int64_t budget, int wrule, bool und, SmemO
     }
   };
   // case 1
-  std::vector<std::pair<int64_t, int32_t>> cands;
-  for (int64_t c = 0; c < n; c++) {
-    if (L.d((int32_t)c) >= 2 && !L.high((int32_t)c, th)) {
-      const int64_t need = (int64_t)(((__int128)th * L.P((int32_t)c)) / 1000000) + 1 - L.T[c];
-      cands.push_back({need, (int32_t)c});
-    }
-  }
-  std::sort(cands.begin(), cands.end());
+  // (keys are unique: the parallel sort gives the sequential order)
+  std::vector<std::pair<int64_t, int32_t>> cands = par_filter<std::pair<int64_t, int32_t>>(
+      n, [&](int32_t c) { return L.d(c) >= 2 && !L.high(c, th); },
+      [&](int32_t c) {
+        return std::make_pair((int64_t)(((__int128)th * L.P(c)) / 1000000) + 1 - L.T[c], c);
+      });
+  __gnu_parallel::sort(cands.begin(), cands.end());
   pt("case-1 centres");
   for (auto& cn : cands) {
     if (rem <= 0) break;
@@ -697,10 +718,9 @@ void cc_edges(Logical& L, int64_t th, int64_t budget, int wrule, bool und, SmemO
   pt("case 1");
   // case 2
   if (rem > 0) {
-    std::vector<int32_t> highs;
-    for (int64_t c = 0; c < n; c++)
-      if (L.high((int32_t)c, th)) highs.push_back((int32_t)c);
-    std::sort(highs.begin(), highs.end(), [&](int32_t x, int32_t y) {
+    std::vector<int32_t> highs =
+        par_filter<int32_t>(n, [&](int32_t c) { return L.high(c, th); }, [](int32_t c) { return c; });
+    __gnu_parallel::sort(highs.begin(), highs.end(), [&](int32_t x, int32_t y) {
       const __int128 lhs = (__int128)L.T[x] * L.P(y), rhs = (__int128)L.T[y] * L.P(x);
       if (lhs != rhs) return lhs > rhs;
       return x < y;
@@ -740,10 +760,9 @@ void cc_edges(Logical& L, int64_t th, int64_t budget, int wrule, bool und, SmemO
 // disjoint shared-memory subgraphs (R27, R28)
 void subgraphs(const Logical& L, int64_t th, int smax, int smem_iters, SmemOut& out) {
   const int64_t n = L.n;
-  std::vector<int32_t> cs;
-  for (int64_t c = 0; c < n; c++)
-    if (L.high((int32_t)c, th) && 1 + L.d((int32_t)c) <= smax) cs.push_back((int32_t)c);
-  std::sort(cs.begin(), cs.end(), [&](int32_t x, int32_t y) {
+  std::vector<int32_t> cs = par_filter<int32_t>(
+      n, [&](int32_t c) { return L.high(c, th) && 1 + L.d(c) <= smax; }, [](int32_t c) { return c; });
+  __gnu_parallel::sort(cs.begin(), cs.end(), [&](int32_t x, int32_t y) {
     const __int128 lhs = (__int128)L.T[x] * L.P(y), rhs = (__int128)L.T[y] * L.P(x);
     if (lhs != rhs) return lhs > rhs;
     if (L.d(x) != L.d(y)) return L.d(x) > L.d(y);
