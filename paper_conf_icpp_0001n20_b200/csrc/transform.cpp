@@ -180,7 +180,8 @@ void renumber(const HostCSR& g, int k, std::vector<int32_t>& nw, int64_t& n_slot
   while (true) {
     const int64_t start = (gid + k - 1) / k * k;
     std::vector<int32_t> parents(cur);
-    std::sort(parents.begin(), parents.end(), [&](int32_t a, int32_t b) { return nw[a] < nw[b]; });
+    // (nw values are unique: the parallel sort gives the sequential order)
+    __gnu_parallel::sort(parents.begin(), parents.end(), [&](int32_t a, int32_t b) { return nw[a] < nw[b]; });
     // each parent's level-(i+1) neighbours in adjacency order, filtered in
     // parallel: level[] never changes during the numbering, so the cursor of
     // R6 walks exactly this list and skips the entries already numbered
@@ -219,8 +220,8 @@ void renumber(const HostCSR& g, int k, std::vector<int32_t>& nw, int64_t& n_slot
         int64_t c = cursor[p];
         const int64_t end = chp[p + 1];
         while (c < end && is_num(ch[c])) c++;
-        if (c < end) {
-          nw[ch[c]] = (int32_t)gid2++;
+        if (c < end) {   // nxt[j] gets id start + j (written after the rounds, in parallel)
+          gid2++;
           set_num(ch[c]);
           nxt.push_back(ch[c]);
           c++;
@@ -232,6 +233,11 @@ void renumber(const HostCSR& g, int k, std::vector<int32_t>& nw, int64_t& n_slot
       live.resize(keep);
       if (!assigned) break;
     }
+    // the level's ids: nw is not read inside the rounds (the numbered bits are),
+    // so its random writes leave the sequential loop
+    const int64_t nn = (int64_t)nxt.size();
+#pragma omp parallel for schedule(static)
+    for (int64_t j = 0; j < nn; j++) nw[nxt[j]] = (int32_t)(start + j);
     if (nxt.empty()) break;
     ranges.push_back({start, gid2});
     gid = gid2;
