@@ -442,7 +442,11 @@ def main():
         h2d = hrp.numel() * 8 + hcol.numel() * 4 + hw.numel() * hw.element_size()
         d2h = n * 4 + n * 8
         e2e_ms, e2e_edges = [], 0
-        for i in range(args.e2e_steps + 1):
+        # two untimed passes: the torch caching allocator (hooked into the library) takes
+        # two passes to hold every block size the upload and the layout builds ask for
+        # (profiles/r2/e2e_variance.txt: 125-142 ms PageRank calls in passes 0-1, 18.7 ms after)
+        E2E_WARM = 2
+        for i in range(args.e2e_steps + E2E_WARM):
             torch.cuda.synchronize()
             e0 = torch.cuda.Event(enable_timing=True)
             e1 = torch.cuda.Event(enable_timing=True)
@@ -460,7 +464,7 @@ def main():
             e1.record(stream)
             torch.cuda.synchronize()
             G2.close()
-            if i > 0:                           # first pass warms the allocator
+            if i >= E2E_WARM:
                 e2e_ms.append(e0.elapsed_time(e1))
                 e2e_edges += a["edges_scanned"] + b["edges_scanned"]
         t = sum(e2e_ms)
