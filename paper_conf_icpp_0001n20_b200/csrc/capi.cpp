@@ -377,22 +377,40 @@ gx_status gx_transform(gx_graph* g, const gx_knobs* knobs, gx_transform_info* in
     g->sg.info.m_slots = g->m;
   } else {
     ensure_host(g);
+    // the current layouts and results are rebuilt after the transform: free them
+    // first (the device pipeline needs several edge-list copies in HBM; RMAT-26
+    // with every exact-mode layout resident ran out of memory)
+    if (g->ctx) {
+      g->dg = DevGraph();
+      g->rs = RunState();
+      g->transformed = false;
+    }
     SlotGraph sg;
     // with a device: the device-resident pipeline (N1, dtransform.cu);
     // GX_TRANSFORM=mixed: the host pipeline with its device helpers (round 1);
     // GX_TRANSFORM=host (or GX_TRANSFORM_HOST=1, or no device): host only
     const char* tm = getenv("GX_TRANSFORM");
     const bool host_only = !g->ctx || getenv("GX_TRANSFORM_HOST") || (tm && !strcmp(tm, "host"));
-    if (host_only) transform_host(g->host, k, sg, nullptr);
-    else if (tm && !strcmp(tm, "mixed")) transform_host(g->host, k, sg, g->ctx);
-    else {
-      DevCSR din;   // the canonical input stays resident on the device: no upload
-      if (g->in_rp.p && g->in_col.p && g->in_w.p && g->host.m == g->m) {
-        din.rp = g->in_rp.as<int64_t>();
-        din.col = g->in_col.as<int32_t>();
-        din.w = g->in_w.as<uint32_t>();
+    try {
+      if (host_only) transform_host(g->host, k, sg, nullptr);
+      else if (tm && !strcmp(tm, "mixed")) transform_host(g->host, k, sg, g->ctx);
+      else {
+        DevCSR din;   // the canonical input stays resident on the device: no upload
+        if (g->in_rp.p && g->in_col.p && g->in_w.p && g->host.m == g->m) {
+          din.rp = g->in_rp.as<int64_t>();
+          din.col = g->in_col.as<int32_t>();
+          din.w = g->in_w.as<uint32_t>();
+        }
+        transform_device(g->host, k, sg, g->ctx, din);
       }
-      transform_device(g->host, k, sg, g->ctx, din);
+    } catch (...) {
+      // a failed transform leaves the graph in exact mode (its layouts rebuilt)
+      if (g->ctx) {
+        g->sg = SlotGraph();
+        gx_knobs_default(&g->knobs);
+        build_device_exact(g);
+      }
+      throw;
     }
     g->sg = std::move(sg);
     g->transformed = true;
