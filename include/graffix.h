@@ -310,8 +310,9 @@ gx_status gx_knobs_default(gx_knobs* k);
 /* The transforms §2 -> §3 -> §4 (composition reading R34) and the device
  * layouts they need; with a device context the slot graph is built in HBM
  * (SURVEY §8(f) N1), only the sequential steps run on the host.  NULL knobs => exact mode (identity).
- * The graph's previous device layouts and results are released before the
- * transform runs (their memory is needed for the edge lists).
+ * With env GX_TRANSFORM_FREE_LAYOUTS=1 the graph's previous device layouts
+ * and results are released before the transform runs (their memory is needed
+ * for the edge lists at RMAT-26 scale).
  * Errors: GX_E_INVALID (k not in 1..32, thresholds not in [0,1] except
  * replicate_threshold >= 0, degree_target not in (0,1], smem_max_nodes not
  * in 2..255); GX_E_OOM / GX_E_CUDA from the device pipeline, after which the

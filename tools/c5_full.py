@@ -11,6 +11,10 @@ knob run (R40, P@40990).  One JSON line.
 import argparse
 import json
 import os
+
+# the exact-mode layouts of every mapping are resident when the transform runs:
+# release them first (the device pipeline needs the memory, include/graffix.h)
+os.environ.setdefault("GX_TRANSFORM_FREE_LAYOUTS", "1")
 import resource
 import sys
 import time
